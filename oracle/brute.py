@@ -1,0 +1,53 @@
+"""Brute-force enumeration of embeddings -- TEST INFRASTRUCTURE ONLY (pin P4).
+
+Enumerates every injective tuple (f(0), ..., f(n_q-1)) of data nodes and keeps
+those satisfying Def. 2.1 conditions (1) and (2) with bond labels
+compared on every query edge (R1-R3).  Exponential; use
+only for n_g <= 8, n_q <= 5.
+"""
+from __future__ import annotations
+
+import itertools
+
+
+def brute_embeddings(qgraph, dgraph):
+    """Yield every embedding f (tuple, f[i] = data node of query node i)."""
+    qlab, qedges = qgraph
+    dlab, dedges = dgraph
+    nq, nd = len(qlab), len(dlab)
+    bond = {}
+    for (u, v, b) in dedges:
+        bond[(u, v)] = b
+        bond[(v, u)] = b
+    for f in itertools.permutations(range(nd), nq):
+        if any(qlab[i] != dlab[f[i]] for i in range(nq)):           # condition (1)
+            continue
+        if any(bond.get((f[u], f[v])) != b for (u, v, b) in qedges):  # condition (2) + bond labels
+            continue
+        yield f
+
+
+def brute_count(qgraph, dgraph) -> int:
+    """qgraph/dgraph: (labels, [(u, v, bond), ...]) with local ids."""
+    qlab, qedges = qgraph
+    dlab, dedges = dgraph
+    nq, nd = len(qlab), len(dlab)
+    bond = {}
+    for (u, v, b) in dedges:
+        bond[(u, v)] = b
+        bond[(v, u)] = b
+    total = 0
+    for f in itertools.permutations(range(nd), nq):
+        if any(qlab[i] != dlab[f[i]] for i in range(nq)):           # condition (1)
+            continue
+        if any(bond.get((f[u], f[v])) != b for (u, v, b) in qedges):  # condition (2) + bond labels
+            continue
+        total += 1
+    return total
+
+
+def brute_dense(qgraphs, dgraphs, find_first: bool = False):
+    out = [[brute_count(q, d) for d in dgraphs] for q in qgraphs]
+    if find_first:
+        out = [[1 if c else 0 for c in row] for row in out]
+    return out
