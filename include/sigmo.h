@@ -1,0 +1,200 @@
+/*
+ * sigmo.h -- C ABI of the B200-native SIGMo hot path (libsigmo.so).
+ *
+ * SIGMo: batched molecular subgraph isomorphism (De Caro et al., SC '25;
+ * /root/reference/PAPER.md, cited as P:<line>).  The library computes, for
+ * every (query graph q, data graph g) pair of a batch, the number of
+ * label- and bond-preserving injective maps V_q -> V_g (Find All) or whether
+ * one exists (Find First):
+ *   problem  : Def. 2.1, NLSM, bond labels checked
+ *              (P:724-726); non-induced reading R1, mappings counted R2;
+ *   modes    : Find All / Find First;
+ *   pipeline : CSR-GO load (section 4.1) -> multi-level signature
+ *              filter (Alg. 1; section 4.2-4.4) ->
+ *              GMCR mapping (section 4.5) -> DFS join
+ *              (section 4.6).
+ * Readings of the paper (R1-R20) are listed in DESIGN.md.
+ *
+ * Conventions (all calls):
+ *   * Every call returns sigmo_status; 0 = SIGMO_OK.  On error the context
+ *     keeps a message readable with sigmo_last_error(ctx).  No C++ exception
+ *     crosses the ABI; bad input never aborts.
+ *   * Host pointers passed in are read during the call only, never retained.
+ *     Output buffers are caller-allocated; sizes are obtained first.
+ *   * All device work is enqueued on the context's CUDA stream.  Getters that
+ *     return host data synchronize that stream before returning.
+ *   * State machine: load_batch -> filter -> join -> get_*.  Out-of-order
+ *     calls return SIGMO_ERR_STATE.  A new load_batch invalidates results;
+ *     filter may be re-run with other levels/flags, join with other modes.
+ *   * A context is bound to one device and one stream; it is not thread-safe.
+ */
+#ifndef SIGMO_H_
+#define SIGMO_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define SIGMO_API __attribute__((visibility("default")))
+#else
+#define SIGMO_API
+#endif
+
+typedef enum {
+  SIGMO_OK = 0,
+  SIGMO_ERR_INVALID_ARG = -1,   /* NULL pointer, bad enum, levels out of range, buffer too small */
+  SIGMO_ERR_INVALID_GRAPH = -2, /* malformed CSR-GO (see sigmo_load_batch) */
+  SIGMO_ERR_LIMIT = -3,         /* a documented size limit is exceeded */
+  SIGMO_ERR_STATE = -4,         /* call out of order (e.g. join before filter) */
+  SIGMO_ERR_OOM = -5,           /* device allocation failed */
+  SIGMO_ERR_CUDA = -6           /* CUDA runtime error (message has the CUDA text) */
+} sigmo_status;
+
+/* Join modes. */
+typedef enum { SIGMO_FIND_ALL = 0, SIGMO_FIND_FIRST = 1 } sigmo_mode;
+
+/* sigmo_filter flags.  NEIGHBOR_SUPPORT: after the signature levels, remove
+ * v_d from C(v_q) while some query edge (v_q,u_q,b) has no data edge
+ * (v_d,u_d,b) with u_d in C(u_q); iterate to the unique greatest fixed point
+ * (BASELINE.json north_star; not in the paper -- DESIGN.md R9). */
+enum { SIGMO_FILTER_NEIGHBOR_SUPPORT = 1u << 0 };
+
+/* Limits (SIGMO_ERR_LIMIT). */
+enum {
+  SIGMO_MAX_QUERY_NODES = 32,  /* paper: queries <= 30 nodes */
+  SIGMO_MAX_DATA_NODES = 256,  /* per data graph; fast path <= 64 */
+  SIGMO_MAX_LEVELS = 16,
+  SIGMO_MAX_BOND_CLASSES = 8   /* distinct bond labels among query edges */
+};
+
+typedef struct sigmo_ctx sigmo_ctx; /* opaque */
+
+/* A CSR-GO batch (section 4.1; Fig. 3): all graphs of
+ * the batch form one disconnected graph.  Host pointers.
+ *   graph_offsets[num_graphs+1] : node id of each graph's first node,
+ *                                 graph_offsets[0]=0, non-decreasing,
+ *                                 graph_offsets[num_graphs]=num_nodes
+ *   row_offsets[num_nodes+1]    : CSR row offsets, row_offsets[0]=0
+ *   col_indices[row_offsets[num_nodes]] : GLOBAL node ids, both directions
+ *                                 of every undirected edge
+ *   node_labels[num_nodes]      : atom label (atomic number by convention)
+ *   edge_labels[row_offsets[num_nodes]] : bond label per adjacency entry
+ *                                 (1 single, 2 double, 3 triple, 4 aromatic
+ *                                 by convention; any u8 allowed, equality only) */
+typedef struct {
+  int64_t num_graphs, num_nodes;
+  const int64_t *graph_offsets;
+  const int64_t *row_offsets;
+  const int32_t *col_indices;
+  const uint8_t *node_labels;
+  const uint8_t *edge_labels;
+} sigmo_graph_batch;
+
+/* Optional device allocator (e.g. the PyTorch caching allocator).  alloc must
+ * return device memory usable on `stream`, or NULL on failure. */
+typedef struct {
+  void *(*alloc)(size_t bytes, void *stream, void *user);
+  void (*free)(void *ptr, void *stream, void *user);
+  void *user;
+} sigmo_allocator;
+
+/* Per-stage device times of the last filter/join (CUDA events on the ctx
+ * stream; only filled when timing is enabled). Milliseconds. */
+typedef struct {
+  float query_prep_ms;  /* query signatures + plane/row programs (cached per levels) */
+  float filter_ms;      /* fused signature + dominance + bitmap + GMCR test kernel */
+  float support_ms;     /* neighbour-support fixed point (0 if flag off) */
+  float mapping_ms;     /* GMCR scan + chunking */
+  float join_ms;        /* DFS join + per-query totals */
+  int64_t filter_launches, join_launches;  /* kernels launched by the last filter / join */
+} sigmo_timings;
+
+/* Create a context on `device` (CUDA ordinal) enqueuing on `cuda_stream`
+ * (a cudaStream_t; NULL = the legacy default stream).  alloc NULL ->
+ * cudaMallocAsync/cudaFreeAsync on the stream.  *out receives the context. */
+SIGMO_API sigmo_status sigmo_create(int device, void *cuda_stream, const sigmo_allocator *alloc, sigmo_ctx **out);
+
+/* Validate, pack and upload one query batch and one data batch (step S1).
+ * Rejected with SIGMO_ERR_INVALID_GRAPH: offsets not starting at 0 or
+ * decreasing, num_nodes inconsistent, a column outside the owning graph,
+ * self-loops, duplicate edges, asymmetric adjacency, an edge label that
+ * differs between (u,v) and (v,u), an empty (0-node) query graph.
+ * SIGMO_ERR_LIMIT: a query graph > 32 nodes, a data graph > 256 nodes,
+ * > 2^31-1 nodes or adjacency entries, > 8 distinct query bond labels.
+ * Disconnected graphs and single-node queries are accepted; an empty data
+ * batch is accepted (all results empty).  Blocks until the inputs are
+ * packed into pinned staging memory; the upload is asynchronous. */
+SIGMO_API sigmo_status sigmo_load_batch(sigmo_ctx *ctx, const sigmo_graph_batch *queries, const sigmo_graph_batch *data);
+
+/* Build the candidate bitmap C_L (Alg. 1) and the GMCR.
+ * levels L in 1..16 (reading R6): L=1 -> labels only (InitializeCandidates,
+ * Alg.1 l.29-37); L>=2 also applies signature dominance at radii 1..L-1
+ * (GenerateSignatures l.11-18 cumulative per R4, RefineCandidates l.19-28 on
+ * every field per R5, saturating fields per R7/R8).  flags: 0 or
+ * SIGMO_FILTER_NEIGHBOR_SUPPORT.  Asynchronous, except that the first call
+ * for a given `levels` after load_batch synchronizes once to size the
+ * query-side plane program. */
+SIGMO_API sigmo_status sigmo_filter(sigmo_ctx *ctx, int levels, uint32_t flags);
+
+/* Stack-based DFS join over the GMCR pairs (section 4.6).
+ * FIND_ALL: per-pair u64 embedding counts; FIND_FIRST: per-pair 0/1.
+ * Also accumulates per-query totals (sum over data graphs).  If
+ * total_matches_out (host) is non-NULL, it receives the sum over all pairs
+ * (synchronizes); otherwise the call is asynchronous. */
+SIGMO_API sigmo_status sigmo_join(sigmo_ctx *ctx, sigmo_mode mode, uint64_t *total_matches_out);
+
+/* Number of (query, data graph) pairs that survived the GMCR rule (after filter). */
+SIGMO_API sigmo_status sigmo_num_pairs(sigmo_ctx *ctx, int64_t *n_pairs);
+
+/* Sparse per-pair results after join, grouped by data graph ascending, then
+ * query ascending.  cap = capacity of the three host arrays; *n receives the
+ * number of pairs (SIGMO_ERR_INVALID_ARG if cap < n; n is still set).
+ * result: count (FIND_ALL) or 0/1 (FIND_FIRST).  Any array may be NULL. */
+SIGMO_API sigmo_status sigmo_get_pair_results(sigmo_ctx *ctx, int64_t cap, int64_t *n, int64_t *data_idx,
+                                    int32_t *query_idx, uint64_t *result);
+
+/* Dense results out[q*num_data_graphs + g] (host, NQ*ND u64); pairs pruned by
+ * the GMCR are 0.  Intended for small batches and tests. */
+SIGMO_API sigmo_status sigmo_get_dense_results(sigmo_ctx *ctx, uint64_t *out);
+
+/* Per-query totals (sum over data graphs of the join results), NQ u64.
+ * device_ptr = 0: `out` is host memory (synchronizes); 1: `out` is device
+ * memory on this ctx's device (asynchronous copy on the ctx stream). */
+SIGMO_API sigmo_status sigmo_get_query_totals(sigmo_ctx *ctx, uint64_t *out, int device_ptr);
+
+/* Candidate bitmap view (reading R10): host out[VQ*ceil(VD/32)] u32,
+ * row = global query node, bit j of word w = data node 32w+j (LSB-first). */
+SIGMO_API sigmo_status sigmo_get_candidates(sigmo_ctx *ctx, uint32_t *out);
+
+/* Packed masked-bitset signatures (section 4.2; field table R7,
+ * saturation R8) at `radius` in 1..255 of every node: which = 0 queries, 1 data.
+ * Host out[V] u64.  Requires load_batch only. */
+SIGMO_API sigmo_status sigmo_get_signatures(sigmo_ctx *ctx, int which, int radius, uint64_t *out);
+
+/* Enable/disable per-stage CUDA-event timing (default off) and read it. */
+SIGMO_API sigmo_status sigmo_set_timing(sigmo_ctx *ctx, int enable);
+SIGMO_API sigmo_status sigmo_get_timings(sigmo_ctx *ctx, sigmo_timings *out);
+
+/* Host-only structural validation of one batch (no device needed): the
+ * checks of sigmo_load_batch for a query (is_query=1) or data batch.
+ * msg (nullable) receives a NUL-terminated reason. */
+SIGMO_API sigmo_status sigmo_validate_batch(const sigmo_graph_batch *batch, int is_query, char *msg, size_t msg_len);
+
+/* Message of the last error on this context ("" if none).  Valid until the
+ * next call on the context. */
+SIGMO_API const char *sigmo_last_error(const sigmo_ctx *ctx);
+
+/* Library version string, e.g. "sigmo-b200 0.1". */
+SIGMO_API const char *sigmo_version(void);
+
+/* Release all device and host resources of the context (synchronizes). */
+SIGMO_API sigmo_status sigmo_destroy(sigmo_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SIGMO_H_ */

@@ -1,0 +1,203 @@
+"""B200-native SIGMo hot path: thin Python binding over libsigmo.so.
+
+The binding only marshals arguments; every step of the path (signatures,
+filter, GMCR, join, reductions) runs in the CUDA kernels of ``csrc/``.
+PyTorch is used for streams and the process group only.  See
+``include/sigmo.h`` for the contract of each call and DESIGN.md for the
+design.
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Optional
+
+import numpy as np
+
+from . import _native
+from ._native import (SIGMO_FILTER_NEIGHBOR_SUPPORT, SIGMO_FIND_ALL, SIGMO_FIND_FIRST, STATUS_NAMES,
+                      load_library)
+
+__all__ = ["Context", "SigmoError", "validate_batch", "load_library", "SIGMO_FIND_ALL", "SIGMO_FIND_FIRST",
+           "SIGMO_FILTER_NEIGHBOR_SUPPORT", "as_c_batch"]
+
+
+class SigmoError(RuntimeError):
+    def __init__(self, status: int, message: str):
+        super().__init__(f"{STATUS_NAMES.get(status, status)}: {message}")
+        self.status = status
+        self.message = message
+
+
+def _arr(a, dt):
+    return np.ascontiguousarray(a, dtype=dt)
+
+
+class _CBatch:
+    """Keeps the numpy arrays alive while the C struct points at them."""
+
+    def __init__(self, b):
+        self.goff = _arr(b.graph_offsets, np.int64)
+        self.roff = _arr(b.row_offsets, np.int64)
+        self.col = _arr(b.col_indices, np.int32)
+        self.nlab = _arr(b.node_labels, np.uint8)
+        self.elab = _arr(b.edge_labels, np.uint8)
+        s = _native.sigmo_graph_batch()
+        s.num_graphs = int(self.goff.shape[0] - 1)
+        s.num_nodes = int(self.nlab.shape[0])
+        s.graph_offsets = self.goff.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+        s.row_offsets = self.roff.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+        s.col_indices = self.col.ctypes.data_as(ctypes.POINTER(ctypes.c_int32))
+        s.node_labels = self.nlab.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8))
+        s.edge_labels = self.elab.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8))
+        self.struct = s
+        self.num_graphs = s.num_graphs
+        self.num_nodes = s.num_nodes
+
+
+def as_c_batch(b) -> _CBatch:
+    return b if isinstance(b, _CBatch) else _CBatch(b)
+
+
+def validate_batch(batch, is_query: bool):
+    """sigmo_validate_batch: host-only structural validation -> (status, message)."""
+    lib = load_library()
+    cb = as_c_batch(batch)
+    buf = ctypes.create_string_buffer(512)
+    st = lib.sigmo_validate_batch(ctypes.byref(cb.struct), 1 if is_query else 0, buf, 512)
+    return st, buf.value.decode()
+
+
+def _stream_handle(stream) -> int:
+    if stream is None:
+        import torch
+        return int(torch.cuda.current_stream().cuda_stream)
+    if isinstance(stream, int):
+        return stream
+    return int(stream.cuda_stream)
+
+
+class Context:
+    """One sigmo_ctx: a device, a stream and the device state of one batch."""
+
+    def __init__(self, device: int = 0, stream=None):
+        self._lib = load_library()
+        self.device = device
+        self._handle = ctypes.c_void_p()
+        self._stream = _stream_handle(stream)
+        st = self._lib.sigmo_create(device, ctypes.c_void_p(self._stream), None, ctypes.byref(self._handle))
+        if st != 0:
+            raise SigmoError(st, f"sigmo_create(device={device}) failed")
+        self.nq = self.nd = self.vq = self.vd = 0
+
+    # -- helpers --
+    def _check(self, st: int, what: str):
+        if st != 0:
+            msg = self._lib.sigmo_last_error(self._handle)
+            raise SigmoError(st, f"{what}: {msg.decode() if msg else ''}")
+
+    def close(self):
+        if self._handle:
+            self._lib.sigmo_destroy(self._handle)
+            self._handle = ctypes.c_void_p()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # -- ABI calls --
+    def load_batch(self, queries, data):
+        cq, cd = as_c_batch(queries), as_c_batch(data)
+        self._check(self._lib.sigmo_load_batch(self._handle, ctypes.byref(cq.struct), ctypes.byref(cd.struct)),
+                    "sigmo_load_batch")
+        self.nq, self.nd, self.vq, self.vd = cq.num_graphs, cd.num_graphs, cq.num_nodes, cd.num_nodes
+        return self
+
+    def filter(self, levels: int = 4, neighbor_support: bool = False, flags: Optional[int] = None):
+        f = flags if flags is not None else (SIGMO_FILTER_NEIGHBOR_SUPPORT if neighbor_support else 0)
+        self._check(self._lib.sigmo_filter(self._handle, int(levels), int(f)), "sigmo_filter")
+        return self
+
+    def join(self, mode=SIGMO_FIND_ALL, total: bool = True):
+        if isinstance(mode, str):
+            mode = {"all": SIGMO_FIND_ALL, "first": SIGMO_FIND_FIRST}[mode]
+        if total:
+            t = ctypes.c_uint64(0)
+            self._check(self._lib.sigmo_join(self._handle, int(mode), ctypes.byref(t)), "sigmo_join")
+            return int(t.value)
+        self._check(self._lib.sigmo_join(self._handle, int(mode), None), "sigmo_join")
+        return None
+
+    def num_pairs(self) -> int:
+        n = ctypes.c_int64(0)
+        self._check(self._lib.sigmo_num_pairs(self._handle, ctypes.byref(n)), "sigmo_num_pairs")
+        return int(n.value)
+
+    def pair_results(self):
+        P = self.num_pairs()
+        di = np.zeros(P, np.int64)
+        qi = np.zeros(P, np.int32)
+        r = np.zeros(P, np.uint64)
+        n = ctypes.c_int64(0)
+        self._check(self._lib.sigmo_get_pair_results(self._handle, P, ctypes.byref(n),
+                                                     di.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                                     qi.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)),
+                                                     r.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))),
+                    "sigmo_get_pair_results")
+        return di, qi, r
+
+    def dense_results(self) -> np.ndarray:
+        out = np.zeros((self.nq, self.nd), np.uint64)
+        self._check(self._lib.sigmo_get_dense_results(self._handle,
+                                                      out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))),
+                    "sigmo_get_dense_results")
+        return out
+
+    def query_totals(self, device_tensor=None):
+        """Host numpy uint64 [NQ], or copy into a device tensor (torch int64/uint64, NQ)."""
+        if device_tensor is not None:
+            self._check(self._lib.sigmo_get_query_totals(self._handle, ctypes.c_void_p(device_tensor.data_ptr()), 1),
+                        "sigmo_get_query_totals")
+            return device_tensor
+        out = np.zeros(self.nq, np.uint64)
+        self._check(self._lib.sigmo_get_query_totals(self._handle, ctypes.c_void_p(out.ctypes.data), 0),
+                    "sigmo_get_query_totals")
+        return out
+
+    def candidates(self) -> np.ndarray:
+        W = (self.vd + 31) // 32
+        out = np.zeros((self.vq, W), np.uint32)
+        self._check(self._lib.sigmo_get_candidates(self._handle, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32))),
+                    "sigmo_get_candidates")
+        return out
+
+    def signatures(self, which: int, radius: int) -> np.ndarray:
+        n = self.vq if which == 0 else self.vd
+        out = np.zeros(n, np.uint64)
+        self._check(self._lib.sigmo_get_signatures(self._handle, int(which), int(radius),
+                                                   out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))),
+                    "sigmo_get_signatures")
+        return out
+
+    def set_timing(self, enable: bool = True):
+        self._check(self._lib.sigmo_set_timing(self._handle, 1 if enable else 0), "sigmo_set_timing")
+
+    def timings(self) -> dict:
+        t = _native.sigmo_timings()
+        self._check(self._lib.sigmo_get_timings(self._handle, ctypes.byref(t)), "sigmo_get_timings")
+        return {k: getattr(t, k) for k, _ in t._fields_}
+
+    @property
+    def stream(self) -> int:
+        return self._stream
+
+
+def version() -> str:
+    return load_library().sigmo_version().decode()

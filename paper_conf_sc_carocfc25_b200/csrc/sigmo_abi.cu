@@ -1,0 +1,989 @@
+// sigmo_abi.cu -- host side of libsigmo.so: the C ABI of include/sigmo.h,
+// batch validation, CSR-GO packing (section 4.1), the query DFS
+// planner, device buffer management and the launch sequence of the hot path.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/sigmo.h"
+#include "sigmo_internal.h"
+
+using namespace sigmo;
+
+namespace {
+
+// ---------------------------------------------------------------------------
+// device buffers
+// ---------------------------------------------------------------------------
+struct DBuf {
+  void *p = nullptr;
+  size_t cap = 0;
+};
+
+struct Pinned {
+  void *p = nullptr;
+  size_t cap = 0;
+};
+
+struct Timing {
+  bool enabled = false;
+  cudaEvent_t ev[8] = {};
+  int n = 0;
+};
+
+struct ProgCache {
+  QueryProg prog;
+  DBuf buf;
+  bool valid = false;
+};
+
+struct HostGraphs {  // validated input view (int64 offsets as given)
+  int64_t G = 0, V = 0, E = 0;
+  const int64_t *goff = nullptr, *roff = nullptr;
+  const int32_t *col = nullptr;
+  const uint8_t *nlab = nullptr, *elab = nullptr;
+};
+
+int num_host_threads(int64_t work) {
+  unsigned hc = std::thread::hardware_concurrency();
+  int t = (int)std::min<unsigned>(hc ? hc : 1, 32);
+  int64_t by_work = work / 20000 + 1;
+  return (int)std::max<int64_t>(1, std::min<int64_t>(t, by_work));
+}
+
+template <typename F>
+void parallel_for_graphs(int64_t G, int64_t work, F &&fn) {
+  const int T = num_host_threads(work);
+  if (T <= 1 || G < 2) {
+    fn(0, 0, G);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (int t = 0; t < T; t++) {
+    int64_t a = G * t / T, b = G * (t + 1) / T;
+    th.emplace_back([&fn, t, a, b] { fn(t, a, b); });
+  }
+  for (auto &x : th) x.join();
+}
+
+}  // namespace
+
+struct sigmo_ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  sigmo_allocator alloc{};
+  bool has_alloc = false;
+  std::string err;
+  int state = 0;  // 0 empty, 1 loaded, 2 filtered, 3 joined
+  int sm_count = 148;
+  size_t max_smem = 227 * 1024;
+
+  // ---- load ----
+  Pinned staging;
+  cudaEvent_t h2d_done = nullptr;
+  DBuf arena;
+  DevGraphs dq, dd;
+  int NQ = 0, VQ = 0, EQ = 0, NQW = 0, maxq = 0, NB = 0;
+  int ND = 0, VD = 0, ED = 0, maxn = 0, NW = 1;
+  bool has_empty_graph = false;
+  int W = 0, Wpad = 0;
+  int32_t *qp_row = nullptr, *qp_beoff = nullptr;
+  uint16_t *qp_be = nullptr;
+  uint8_t *bclass = nullptr;
+  // filter tile geometry per TW (32,16,8,4,2,1)
+  int tile_extn[6] = {}, tile_extw[6] = {}, tile_molcap[6] = {};
+
+  // ---- filter ----
+  std::map<int, ProgCache> progs;  // keyed by R = levels-1
+  DBuf qcounts;
+  DBuf bitmap, gm, mol_cnt, off, scan_tmp, chunk_start, nchunks;
+  size_t scan_tmp_bytes = 0;
+  int levels = 0;
+  uint32_t flags = 0;
+  int PC = 512, AC = 512, CMC = 2048, MC = 128;
+
+  // ---- join ----
+  DBuf pair_query, pair_result, jcnt;  // jcnt = [counter (8 B) | totals NQ u64]
+  int last_mode = 0;
+  DBuf sig_tmp;
+
+  Timing timing;
+  sigmo_timings last{};
+};
+
+namespace {
+
+sigmo_status set_err(sigmo_ctx *c, sigmo_status s, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  if (c) c->err = buf;
+  return s;
+}
+
+#define CUDA_TRY(ctx, call)                                                                          \
+  do {                                                                                               \
+    cudaError_t e_ = (call);                                                                         \
+    if (e_ != cudaSuccess) {                                                                         \
+      return set_err(ctx, e_ == cudaErrorMemoryAllocation ? SIGMO_ERR_OOM : SIGMO_ERR_CUDA,          \
+                     "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__);           \
+    }                                                                                                \
+  } while (0)
+
+void dfree(sigmo_ctx *c, DBuf &b) {
+  if (!b.p) return;
+  if (c->has_alloc) c->alloc.free(b.p, (void *)c->stream, c->alloc.user);
+  else cudaFreeAsync(b.p, c->stream);
+  b.p = nullptr;
+  b.cap = 0;
+}
+
+sigmo_status dreserve(sigmo_ctx *c, DBuf &b, size_t bytes, const char *what) {
+  if (bytes == 0) bytes = 16;
+  if (b.cap >= bytes) return SIGMO_OK;
+  dfree(c, b);
+  void *p = nullptr;
+  if (c->has_alloc) {
+    p = c->alloc.alloc(bytes, (void *)c->stream, c->alloc.user);
+    if (!p) return set_err(c, SIGMO_ERR_OOM, "allocator returned NULL for %s (%zu bytes)", what, bytes);
+  } else {
+    cudaError_t e = cudaMallocAsync(&p, bytes, c->stream);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return set_err(c, SIGMO_ERR_OOM, "cudaMallocAsync %s (%zu bytes): %s", what, bytes, cudaGetErrorString(e));
+    }
+  }
+  b.p = p;
+  b.cap = bytes;
+  return SIGMO_OK;
+}
+
+#define SIGMO_TRY(x)                  \
+  do {                                \
+    sigmo_status s_ = (x);            \
+    if (s_ != SIGMO_OK) return s_;    \
+  } while (0)
+
+// ---------------------------------------------------------------------------
+// validation (sigmo_load_batch contract)
+// ---------------------------------------------------------------------------
+sigmo_status validate(const sigmo_graph_batch *b, int is_query, std::string &msg, HostGraphs &out) {
+  auto fail = [&](sigmo_status s, const char *fmt, long long x, long long y) {
+    char buf[256];
+    snprintf(buf, sizeof(buf), fmt, x, y);
+    msg = buf;
+    return s;
+  };
+  if (!b) return fail(SIGMO_ERR_INVALID_ARG, "batch pointer is NULL", 0, 0) ;
+  if (b->num_graphs < 0 || b->num_nodes < 0) return fail(SIGMO_ERR_INVALID_ARG, "negative num_graphs %lld / num_nodes %lld", b->num_graphs, b->num_nodes);
+  if (!b->graph_offsets || !b->row_offsets) return fail(SIGMO_ERR_INVALID_ARG, "graph_offsets/row_offsets NULL", 0, 0);
+  if (b->num_nodes >= (1ll << 31) - 1) return fail(SIGMO_ERR_LIMIT, "num_nodes %lld >= 2^31-1", b->num_nodes, 0);
+  if (b->num_graphs >= (1ll << 31) - 1) return fail(SIGMO_ERR_LIMIT, "num_graphs %lld >= 2^31-1", b->num_graphs, 0);
+  const int64_t G = b->num_graphs, V = b->num_nodes;
+  const int64_t *go = b->graph_offsets, *ro = b->row_offsets;
+  if (go[0] != 0) return fail(SIGMO_ERR_INVALID_GRAPH, "graph_offsets[0] = %lld, expected 0", go[0], 0);
+  for (int64_t g = 0; g < G; g++) {
+    if (go[g + 1] < go[g]) return fail(SIGMO_ERR_INVALID_GRAPH, "graph_offsets decreasing at graph %lld (%lld)", g, go[g + 1]);
+    const int64_t n = go[g + 1] - go[g];
+    if (is_query && n == 0) return fail(SIGMO_ERR_INVALID_GRAPH, "query graph %lld is empty", g, 0);
+    if (is_query && n > SIGMO_MAX_QUERY_NODES) return fail(SIGMO_ERR_LIMIT, "query graph %lld has %lld nodes > 32", g, n);
+    if (!is_query && n > SIGMO_MAX_DATA_NODES) return fail(SIGMO_ERR_LIMIT, "data graph %lld has %lld nodes > 256", g, n);
+  }
+  if (go[G] != V) return fail(SIGMO_ERR_INVALID_GRAPH, "graph_offsets[num_graphs] = %lld != num_nodes %lld", go[G], V);
+  if (ro[0] != 0) return fail(SIGMO_ERR_INVALID_GRAPH, "row_offsets[0] = %lld, expected 0", ro[0], 0);
+  for (int64_t v = 0; v < V; v++)
+    if (ro[v + 1] < ro[v]) return fail(SIGMO_ERR_INVALID_GRAPH, "row_offsets decreasing at node %lld (%lld)", v, ro[v + 1]);
+  const int64_t E = ro[V];
+  if (E >= (1ll << 31) - 1) return fail(SIGMO_ERR_LIMIT, "adjacency entries %lld >= 2^31-1", E, 0);
+  if (V > 0 && !b->node_labels) return fail(SIGMO_ERR_INVALID_ARG, "node_labels NULL", 0, 0);
+  if (E > 0 && (!b->col_indices || !b->edge_labels)) return fail(SIGMO_ERR_INVALID_ARG, "col_indices/edge_labels NULL", 0, 0);
+  const int32_t *col = b->col_indices;
+  const uint8_t *el = b->edge_labels;
+  // per-graph structural checks, parallel over graphs; first error by graph index
+  std::vector<int64_t> bad_graph(64, -1);
+  std::vector<std::string> bad_msg(64);
+  std::vector<sigmo_status> bad_st(64, SIGMO_OK);
+  parallel_for_graphs(G, E + V, [&](int t, int64_t ga, int64_t gb) {
+    char buf[256];
+    for (int64_t g = ga; g < gb; g++) {
+      const int64_t lo = go[g], hi = go[g + 1];
+      for (int64_t u = lo; u < hi; u++) {
+        for (int64_t e = ro[u]; e < ro[u + 1]; e++) {
+          const int64_t v = col[e];
+          const char *why = nullptr;
+          long long a1 = 0, a2 = 0;
+          if (v < lo || v >= hi) {
+            why = "column %lld of node %lld outside its graph";
+            a1 = v; a2 = u;
+          } else if (v == u) {
+            why = "self-loop at node %lld";
+            a1 = u;
+          } else {
+            int dup = 0;
+            for (int64_t f = ro[u]; f < ro[u + 1]; f++) dup += (col[f] == v);
+            if (dup > 1) {
+              why = "duplicate edge %lld -> %lld";
+              a1 = u; a2 = v;
+            } else {
+              bool sym = false;
+              for (int64_t f = ro[v]; f < ro[v + 1] && !sym; f++)
+                if (col[f] == u && el[f] == el[e]) sym = true;
+              if (!sym) {
+                why = "asymmetric edge or edge label %lld -> %lld";
+                a1 = u; a2 = v;
+              }
+            }
+          }
+          if (why) {
+            snprintf(buf, sizeof(buf), why, a1, a2);
+            bad_graph[t] = g;
+            bad_msg[t] = buf;
+            bad_st[t] = SIGMO_ERR_INVALID_GRAPH;
+            return;
+          }
+        }
+      }
+    }
+  });
+  int64_t first = -1;
+  int ft = -1;
+  for (int t = 0; t < 64; t++)
+    if (bad_graph[t] >= 0 && (first < 0 || bad_graph[t] < first)) {
+      first = bad_graph[t];
+      ft = t;
+    }
+  if (ft >= 0) {
+    msg = std::string(is_query ? "query" : "data") + " graph " + std::to_string(first) + ": " + bad_msg[ft];
+    return bad_st[ft];
+  }
+  out.G = G;
+  out.V = V;
+  out.E = E;
+  out.goff = go;
+  out.roff = ro;
+  out.col = col;
+  out.nlab = b->node_labels;
+  out.elab = el;
+  return SIGMO_OK;
+}
+
+// ---------------------------------------------------------------------------
+// packing into pinned staging
+// ---------------------------------------------------------------------------
+struct Layout {
+  size_t off = 0;
+  size_t take(size_t bytes) {
+    size_t o = off;
+    off = (off + bytes + 255) & ~(size_t)255;
+    return o;
+  }
+};
+
+struct PackedOffsets {
+  size_t goff, label, local, roff, nbr;
+};
+
+PackedOffsets plan_graphs(Layout &L, const HostGraphs &h) {
+  PackedOffsets p;
+  p.goff = L.take(4 * (size_t)(h.G + 1));
+  p.label = L.take((size_t)h.V);
+  p.local = L.take((size_t)h.V);
+  p.roff = L.take(4 * (size_t)(h.V + 1));
+  p.nbr = L.take(2 * (size_t)h.E);
+  return p;
+}
+
+void pack_graphs(unsigned char *base, const PackedOffsets &p, const HostGraphs &h) {
+  int32_t *goff = (int32_t *)(base + p.goff);
+  uint8_t *label = base + p.label;
+  uint8_t *local = base + p.local;
+  int32_t *roff = (int32_t *)(base + p.roff);
+  uint16_t *nbr = (uint16_t *)(base + p.nbr);
+  goff[h.G] = (int32_t)h.V;
+  roff[h.V] = (int32_t)h.E;
+  parallel_for_graphs(h.G, h.E + h.V, [&](int, int64_t ga, int64_t gb) {
+    for (int64_t g = ga; g < gb; g++) {
+      const int64_t lo = h.goff[g], hi = h.goff[g + 1];
+      goff[g] = (int32_t)lo;
+      for (int64_t u = lo; u < hi; u++) {
+        label[u] = h.nlab[u];
+        local[u] = (uint8_t)(u - lo);
+        roff[u] = (int32_t)h.roff[u];
+        for (int64_t e = h.roff[u]; e < h.roff[u + 1]; e++)
+          nbr[e] = (uint16_t)(((h.col[e] - lo) << 8) | h.elab[e]);
+      }
+    }
+  });
+}
+
+DevGraphs dev_view(unsigned char *dbase, const PackedOffsets &p, const HostGraphs &h) {
+  DevGraphs d;
+  d.num_graphs = (int)h.G;
+  d.num_nodes = (int)h.V;
+  d.num_adj = (int)h.E;
+  d.max_nodes = 0;
+  for (int64_t g = 0; g < h.G; g++) d.max_nodes = std::max<int>(d.max_nodes, (int)(h.goff[g + 1] - h.goff[g]));
+  d.goff = (const int32_t *)(dbase + p.goff);
+  d.label = dbase + p.label;
+  d.local = dbase + p.local;
+  d.roff = (const int32_t *)(dbase + p.roff);
+  d.nbr = (const uint16_t *)(dbase + p.nbr);
+  return d;
+}
+
+// ---------------------------------------------------------------------------
+// query DFS planner (host, step S1).  Static matching order per query:
+// root = rarest label in the data batch (ties: higher degree, lower id); then
+// repeatedly the unordered node with most edges into the ordered set (ties:
+// rarer label, higher degree, lower id).  Any order yields the same counts
+// (reading R12); this one prunes early.
+// ---------------------------------------------------------------------------
+struct QPlan {
+  std::vector<int32_t> row;     // [VQ] global query node of depth e
+  std::vector<int32_t> beoff;   // [VQ+1]
+  std::vector<uint16_t> be;     // (j << 8) | class
+};
+
+void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const uint8_t *bclass, QPlan &out) {
+  out.row.assign((size_t)q.V, 0);
+  out.beoff.assign((size_t)q.V + 1, 0);
+  out.be.clear();
+  for (int64_t g = 0; g < q.G; g++) {
+    const int64_t lo = q.goff[g];
+    const int n = (int)(q.goff[g + 1] - lo);
+    std::vector<int> pos(n, -1), order;
+    auto deg = [&](int u) { return (int)(q.roff[lo + u + 1] - q.roff[lo + u]); };
+    auto fr = [&](int u) { return freq[q.nlab[lo + u]]; };
+    for (int i = 0; i < n; i++) {
+      int best = -1, bc = -1;
+      for (int u = 0; u < n; u++) {
+        if (pos[u] >= 0) continue;
+        int conn = 0;
+        for (int64_t e = q.roff[lo + u]; e < q.roff[lo + u + 1]; e++)
+          if (pos[q.col[e] - lo] >= 0) conn++;
+        bool better = false;
+        if (best < 0) better = true;
+        else if (conn != bc) better = conn > bc;
+        else if (fr(u) != fr(best)) better = fr(u) < fr(best);
+        else if (deg(u) != deg(best)) better = deg(u) > deg(best);
+        if (better) {
+          best = u;
+          bc = conn;
+        }
+      }
+      pos[best] = i;
+      order.push_back(best);
+    }
+    for (int e = 0; e < n; e++) {
+      const int u = order[e];
+      out.row[lo + e] = (int32_t)(lo + u);
+      out.beoff[lo + e] = (int32_t)out.be.size();
+      for (int64_t k = q.roff[lo + u]; k < q.roff[lo + u + 1]; k++) {
+        const int w = (int)(q.col[k] - lo);
+        if (pos[w] < e) out.be.push_back((uint16_t)((pos[w] << 8) | bclass[q.elab[k]]));
+      }
+    }
+  }
+  out.beoff[q.V] = (int32_t)out.be.size();
+}
+
+int graph_of_host(const int64_t *goff, int64_t G, int64_t n) {
+  int64_t lo = 0, hi = G;
+  while (lo < hi) {
+    int64_t mid = (lo + hi + 1) >> 1;
+    if (goff[mid] <= n) lo = mid;
+    else hi = mid - 1;
+  }
+  return (int)lo;
+}
+
+void timing_mark(sigmo_ctx *c) {
+  if (c->timing.enabled && c->timing.n < 8) cudaEventRecord(c->timing.ev[c->timing.n++], c->stream);
+}
+
+float timing_ms(sigmo_ctx *c, int a, int b) {
+  float ms = 0.f;
+  if (a < c->timing.n && b < c->timing.n) cudaEventElapsedTime(&ms, c->timing.ev[a], c->timing.ev[b]);
+  return ms;
+}
+
+
+// ---------------------------------------------------------------------------
+// query plane program (cached per R = levels - 1)
+// ---------------------------------------------------------------------------
+constexpr int kMaxPlanes = kMaxRadius * kNumFields * 256;  // 49920 keys
+
+sigmo_status ensure_prog(sigmo_ctx *c, int R, QueryProg *&out) {
+  auto it = c->progs.find(R);
+  if (it != c->progs.end() && it->second.valid) {
+    out = &it->second.prog;
+    return SIGMO_OK;
+  }
+  ProgCache &pc = c->progs[R];
+  const int VQ = c->VQ;
+  const size_t rowcap = (size_t)VQ * (R > 0 ? R : 1) * kNumFields + 1;
+  Layout L;
+  const size_t o_pt = L.take(kMaxPlanes);
+  const size_t o_gp = L.take(2 * 256);
+  const size_t o_gf = L.take(256);
+  const size_t o_rg = L.take(2 * 32);
+  const size_t o_fs = L.take(16);
+  const size_t o_lv = L.take(256);
+  const size_t o_rl = L.take((size_t)VQ + 1);
+  const size_t o_ro = L.take(4 * ((size_t)VQ + 1));
+  const size_t o_ri = L.take(2 * rowcap);
+  const size_t o_me = L.take(sizeof(QueryProgMeta));
+  SIGMO_TRY(dreserve(c, pc.buf, L.off, "query program"));
+  unsigned char *b = (unsigned char *)pc.buf.p;
+  QueryProg &P = pc.prog;
+  P.R = R;
+  P.p_t = b + o_pt;
+  P.grp_poff = (int16_t *)(b + o_gp);
+  P.grp_f = b + o_gf;
+  P.rg_off = (int16_t *)(b + o_rg);
+  P.fslot = (int8_t *)(b + o_fs);
+  P.lab_val = b + o_lv;
+  P.row_lab = b + o_rl;
+  P.row_off = (int32_t *)(b + o_ro);
+  P.row_ids = (uint16_t *)(b + o_ri);
+  P.d_meta = (QueryProgMeta *)(b + o_me);
+  timing_mark(c);
+  if (R > 0) {
+    SIGMO_TRY(dreserve(c, c->qcounts, (size_t)VQ * R * kNumFields, "query counts"));
+    CUDA_TRY(c, launch_sig_counts(c->dq, R, (uint8_t *)c->qcounts.p, c->stream));
+  }
+  CUDA_TRY(c, launch_query_prep(c->dq, R, (const uint8_t *)c->qcounts.p, P, c->stream));
+  CUDA_TRY(c, cudaMemcpyAsync(&P.meta, P.d_meta, sizeof(QueryProgMeta), cudaMemcpyDeviceToHost, c->stream));
+  timing_mark(c);
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  if (P.meta.err) return set_err(c, SIGMO_ERR_LIMIT, "query program error %d", P.meta.err);
+  pc.valid = true;
+  out = &P;
+  return SIGMO_OK;
+}
+
+// per-TW tile geometry (EXTN, EXTW, MOLCAP) of the data batch
+void tile_geometry(sigmo_ctx *c, const HostGraphs &d) {
+  const int tws[6] = {32, 16, 8, 4, 2, 1};
+  for (int k = 0; k < 6; k++) {
+    const int TW = tws[k];
+    int extn = 1, extw = 1, molcap = 1;
+    const int64_t W = c->W;
+    for (int64_t w0 = 0; w0 < W; w0 += TW) {
+      const int64_t n0 = w0 * 32, n1 = std::min<int64_t>(n0 + 32ll * TW, d.V);
+      const int g0 = graph_of_host(d.goff, d.G, n0);
+      const int g1 = graph_of_host(d.goff, d.G, n1 - 1) + 1;
+      const int64_t gs = d.goff[g0], ge = d.goff[g1];
+      extn = std::max<int>(extn, (int)(ge - gs));
+      extw = std::max<int>(extw, (int)(((ge - 1) >> 5) - (gs >> 5) + 1));
+      molcap = std::max<int>(molcap, g1 - g0);
+    }
+    c->tile_extn[k] = extn;
+    c->tile_extw[k] = extw;
+    c->tile_molcap[k] = molcap;
+  }
+}
+
+void free_all(sigmo_ctx *c) {
+  for (auto &kv : c->progs) dfree(c, kv.second.buf);
+  c->progs.clear();
+  DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
+                  &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_result, &c->jcnt, &c->sig_tmp};
+  for (DBuf *b : bufs) dfree(c, *b);
+}
+
+}  // namespace
+
+// ===========================================================================
+// C ABI
+// ===========================================================================
+extern "C" {
+
+const char *sigmo_version(void) { return "sigmo-b200 0.1 (sm_100a)"; }
+
+const char *sigmo_last_error(const sigmo_ctx *ctx) { return ctx ? ctx->err.c_str() : "NULL context"; }
+
+sigmo_status sigmo_validate_batch(const sigmo_graph_batch *batch, int is_query, char *msg, size_t msg_len) {
+  std::string m;
+  HostGraphs h;
+  sigmo_status s;
+  try {
+    s = validate(batch, is_query, m, h);
+  } catch (...) {
+    s = SIGMO_ERR_INVALID_ARG;
+    m = "exception during validation";
+  }
+  if (msg && msg_len) {
+    snprintf(msg, msg_len, "%s", m.c_str());
+  }
+  return s;
+}
+
+sigmo_status sigmo_create(int device, void *cuda_stream, const sigmo_allocator *alloc, sigmo_ctx **out) {
+  if (!out) return SIGMO_ERR_INVALID_ARG;
+  *out = nullptr;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    cudaGetLastError();
+    return SIGMO_ERR_CUDA;
+  }
+  if (alloc && (!alloc->alloc || !alloc->free)) return SIGMO_ERR_INVALID_ARG;
+  sigmo_ctx *c = new (std::nothrow) sigmo_ctx();
+  if (!c) return SIGMO_ERR_OOM;
+  c->device = device;
+  c->stream = (cudaStream_t)cuda_stream;
+  if (alloc) {
+    c->alloc = *alloc;
+    c->has_alloc = true;
+  }
+  if (cudaSetDevice(device) != cudaSuccess) {
+    delete c;
+    return SIGMO_ERR_CUDA;
+  }
+  cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, device);
+  int smem = 0;
+  cudaDeviceGetAttribute(&smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+  if (smem > 0) c->max_smem = (size_t)smem;
+  if (cudaEventCreateWithFlags(&c->h2d_done, cudaEventDisableTiming) != cudaSuccess) {
+    delete c;
+    return SIGMO_ERR_CUDA;
+  }
+  for (int i = 0; i < 8; i++) cudaEventCreate(&c->timing.ev[i]);
+  *out = c;
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_destroy(sigmo_ctx *c) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  cudaSetDevice(c->device);
+  cudaStreamSynchronize(c->stream);
+  free_all(c);
+  cudaStreamSynchronize(c->stream);
+  if (c->staging.p) cudaFreeHost(c->staging.p);
+  if (c->h2d_done) cudaEventDestroy(c->h2d_done);
+  for (int i = 0; i < 8; i++)
+    if (c->timing.ev[i]) cudaEventDestroy(c->timing.ev[i]);
+  delete c;
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_set_timing(sigmo_ctx *c, int enable) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  c->timing.enabled = enable != 0;
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_get_timings(sigmo_ctx *c, sigmo_timings *out) {
+  if (!c || !out) return SIGMO_ERR_INVALID_ARG;
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  *out = c->last;
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, const sigmo_graph_batch *data) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  if (!queries || !data) return set_err(c, SIGMO_ERR_INVALID_ARG, "queries/data batch is NULL");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  HostGraphs hq, hd;
+  std::string msg;
+  sigmo_status s = validate(queries, 1, msg, hq);
+  if (s != SIGMO_OK) return set_err(c, s, "query batch: %s", msg.c_str());
+  s = validate(data, 0, msg, hd);
+  if (s != SIGMO_OK) return set_err(c, s, "data batch: %s", msg.c_str());
+  // bond classes = distinct query bond labels
+  uint8_t bclass[256];
+  memset(bclass, 255, sizeof(bclass));
+  {
+    bool seen[256] = {};
+    for (int64_t e = 0; e < hq.E; e++) seen[hq.elab[e]] = true;
+    int nb = 0;
+    for (int l = 0; l < 256; l++)
+      if (seen[l]) {
+        if (nb >= SIGMO_MAX_BOND_CLASSES)
+          return set_err(c, SIGMO_ERR_LIMIT, "more than %d distinct query bond labels", SIGMO_MAX_BOND_CLASSES);
+        bclass[l] = (uint8_t)nb++;
+      }
+    c->NB = nb;
+  }
+  c->state = 0;
+  // label frequencies of the data batch (planner heuristic)
+  std::vector<int64_t> freq(256, 0);
+  for (int64_t v = 0; v < hd.V; v++) freq[hd.nlab[v]]++;
+  QPlan plan;
+  plan_queries(hq, freq, bclass, plan);
+
+  // ---- staging layout ----
+  Layout L;
+  const PackedOffsets pq = plan_graphs(L, hq);
+  const size_t o_row = L.take(4 * (size_t)hq.V);
+  const size_t o_beoff = L.take(4 * ((size_t)hq.V + 1));
+  const size_t o_be = L.take(2 * plan.be.size() + 2);
+  const size_t o_bc = L.take(256);
+  const PackedOffsets pd = plan_graphs(L, hd);
+  const size_t total = L.off;
+  // wait until the previous upload no longer reads the staging buffer
+  CUDA_TRY(c, cudaEventSynchronize(c->h2d_done));
+  if (c->staging.cap < total) {
+    if (c->staging.p) cudaFreeHost(c->staging.p);
+    c->staging.p = nullptr;
+    c->staging.cap = 0;
+    size_t cap = std::max<size_t>(total, c->staging.cap * 3 / 2);
+    CUDA_TRY(c, cudaHostAlloc(&c->staging.p, cap, cudaHostAllocDefault));
+    c->staging.cap = cap;
+  }
+  unsigned char *hb = (unsigned char *)c->staging.p;
+  pack_graphs(hb, pq, hq);
+  memcpy(hb + o_row, plan.row.data(), 4 * plan.row.size());
+  memcpy(hb + o_beoff, plan.beoff.data(), 4 * plan.beoff.size());
+  if (!plan.be.empty()) memcpy(hb + o_be, plan.be.data(), 2 * plan.be.size());
+  memcpy(hb + o_bc, bclass, 256);
+  pack_graphs(hb, pd, hd);
+
+  // ---- device arena + one H2D copy ----
+  SIGMO_TRY(dreserve(c, c->arena, total, "input arena"));
+  unsigned char *db = (unsigned char *)c->arena.p;
+  CUDA_TRY(c, cudaMemcpyAsync(db, hb, total, cudaMemcpyHostToDevice, c->stream));
+  CUDA_TRY(c, cudaEventRecord(c->h2d_done, c->stream));
+  c->dq = dev_view(db, pq, hq);
+  c->dd = dev_view(db, pd, hd);
+  c->qp_row = (int32_t *)(db + o_row);
+  c->qp_beoff = (int32_t *)(db + o_beoff);
+  c->qp_be = (uint16_t *)(db + o_be);
+  c->bclass = db + o_bc;
+  c->NQ = (int)hq.G;
+  c->VQ = (int)hq.V;
+  c->EQ = (int)hq.E;
+  c->NQW = (c->NQ + 31) / 32;
+  c->maxq = c->dq.max_nodes;
+  c->ND = (int)hd.G;
+  c->VD = (int)hd.V;
+  c->ED = (int)hd.E;
+  c->maxn = c->dd.max_nodes;
+  c->NW = c->maxn <= 64 ? 1 : (c->maxn <= 128 ? 2 : 4);
+  c->has_empty_graph = false;
+  for (int64_t g = 0; g < hd.G && !c->has_empty_graph; g++) c->has_empty_graph = hd.goff[g + 1] == hd.goff[g];
+  c->W = (c->VD + 31) / 32;
+  c->Wpad = ((c->W + 31) / 32) * 32;
+  if (c->Wpad == 0) c->Wpad = 32;
+  tile_geometry(c, hd);
+  // join chunk capacities (pairs, atoms, candidate masks, graphs per chunk):
+  // shrink until the join's shared memory fits one SM
+  {
+    c->PC = 512;
+    c->AC = 512;
+    c->CMC = 2048;
+    c->MC = 128;
+    for (int tries = 0; tries < 12; tries++) {
+      JoinParams jp{};
+      jp.NQ = c->NQ;
+      jp.NB = c->NB;
+      jp.maxq = std::max(c->maxq, 2);
+      jp.PCAP = c->PC + c->NQ;
+      jp.ACAP = c->AC + c->maxn;
+      jp.CMCAP = c->CMC + c->VQ;
+      jp.MCAP = c->MC;
+      if (join_smem_bytes(c->NW, jp) <= c->max_smem) break;
+      c->PC = std::max(c->PC / 2, 1);
+      c->AC = std::max(c->AC / 2, 1);
+      c->CMC = std::max(c->CMC / 2, 1);
+      c->MC = std::max(c->MC / 2, 1);
+    }
+  }
+  // query programs depend on the query batch only, but the batch changed
+  for (auto &kv : c->progs) kv.second.valid = false;
+
+  // ---- per-batch device buffers ----
+  const size_t bm_bytes = 4 * (size_t)std::max(c->VQ, 1) * c->Wpad;
+  const bool bm_grow = c->bitmap.cap < bm_bytes;
+  SIGMO_TRY(dreserve(c, c->bitmap, bm_bytes, "candidate bitmap"));
+  // padding words (>= W) are never written by the filter: zero once
+  if (bm_grow || true) CUDA_TRY(c, cudaMemsetAsync(c->bitmap.p, 0, bm_bytes, c->stream));
+  SIGMO_TRY(dreserve(c, c->gm, 4 * (size_t)std::max(c->ND, 1) * std::max(c->NQW, 1), "gmcr bits"));
+  SIGMO_TRY(dreserve(c, c->mol_cnt, sizeof(I64x2) * ((size_t)c->ND + 1), "gmcr counts"));
+  CUDA_TRY(c, cudaMemsetAsync(c->mol_cnt.p, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
+  SIGMO_TRY(dreserve(c, c->off, sizeof(I64x2) * ((size_t)c->ND + 1), "gmcr offsets"));
+  size_t tb = 0;
+  CUDA_TRY(c, launch_scan(nullptr, nullptr, c->ND + 1, nullptr, &tb, c->stream));
+  SIGMO_TRY(dreserve(c, c->scan_tmp, tb, "scan temp"));
+  c->scan_tmp_bytes = std::max(tb, (size_t)16);
+  const long long pair_cap = (long long)c->NQ * c->ND;
+  const long long max_chunks = pair_cap / c->PC + (long long)c->VD / c->AC + (long long)c->VQ * c->ND / c->CMC +
+                               (long long)c->ND / c->MC + 4;
+  SIGMO_TRY(dreserve(c, c->chunk_start, 4 * (size_t)max_chunks, "chunk starts"));
+  SIGMO_TRY(dreserve(c, c->nchunks, 16, "chunk count"));
+  SIGMO_TRY(dreserve(c, c->pair_query, 4 * (size_t)std::max(pair_cap, 1ll), "pair queries"));
+  SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
+  SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 2), "join counters"));
+  c->state = 1;
+  c->err.clear();
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 1) return set_err(c, SIGMO_ERR_STATE, "sigmo_filter before sigmo_load_batch");
+  if (levels < 1 || levels > SIGMO_MAX_LEVELS) return set_err(c, SIGMO_ERR_INVALID_ARG, "levels %d not in 1..16", levels);
+  if (flags & ~(uint32_t)SIGMO_FILTER_NEIGHBOR_SUPPORT) return set_err(c, SIGMO_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
+  if (flags & SIGMO_FILTER_NEIGHBOR_SUPPORT)
+    return set_err(c, SIGMO_ERR_INVALID_ARG, "SIGMO_FILTER_NEIGHBOR_SUPPORT not available in this build");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  const int R = levels - 1;
+  c->timing.n = 0;
+  QueryProg *prog = nullptr;
+  SIGMO_TRY(ensure_prog(c, R, prog));
+  const bool prog_timed = c->timing.n == 2;
+  if (c->timing.enabled && !prog_timed) c->timing.n = 0;
+  const int t0 = c->timing.n;
+  timing_mark(c);
+  int launches = 0;
+  if (c->ND > 0 && c->VD > 0) {
+    const QueryProgMeta &m = prog->meta;
+    // tile width: largest TW whose shared memory fits
+    const int tws[6] = {32, 16, 8, 4, 2, 1};
+    int k = 0;
+    size_t smem = 0;
+    for (k = 0; k < 6; k++) {
+      smem = filter_smem_bytes(c->NW, c->tile_extn[k], c->tile_extw[k], c->tile_molcap[k], m.NFU, m.NLAB, m.P);
+      if (smem <= c->max_smem) break;
+    }
+    if (k == 6) return set_err(c, SIGMO_ERR_LIMIT, "filter shared memory %zu exceeds %zu (P=%d)", smem, c->max_smem, m.P);
+    FilterParams fp{};
+    fp.D = c->dd;
+    fp.TW = tws[k];
+    fp.W = c->W;
+    fp.Wpad = c->Wpad;
+    fp.VQ = c->VQ;
+    fp.NQ = c->NQ;
+    fp.NQW = c->NQW;
+    fp.R = R;
+    fp.P = m.P;
+    fp.G = m.G;
+    fp.NFU = m.NFU;
+    fp.NLAB = m.NLAB;
+    fp.p_t = prog->p_t;
+    fp.grp_poff = prog->grp_poff;
+    fp.grp_f = prog->grp_f;
+    fp.rg_off = prog->rg_off;
+    fp.fslot = prog->fslot;
+    fp.lab_val = prog->lab_val;
+    fp.row_lab = prog->row_lab;
+    fp.row_off = prog->row_off;
+    fp.row_ids = prog->row_ids;
+    fp.qgoff = c->dq.goff;
+    fp.bitmap = (uint32_t *)c->bitmap.p;
+    fp.gm = (uint32_t *)c->gm.p;
+    fp.mol_cnt = (I64x2 *)c->mol_cnt.p;
+    fp.EXTN = c->tile_extn[k];
+    fp.EXTW = c->tile_extw[k];
+    fp.MOLCAP = c->tile_molcap[k];
+    fp.smem_bytes = smem;
+    if (c->has_empty_graph) {
+      CUDA_TRY(c, cudaMemsetAsync(c->gm.p, 0, 4 * (size_t)c->ND * c->NQW, c->stream));
+      CUDA_TRY(c, cudaMemsetAsync(c->mol_cnt.p, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
+    }
+    const int tiles = (c->W + fp.TW - 1) / fp.TW;
+    CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));
+    launches++;
+    timing_mark(c);
+    size_t tb = c->scan_tmp_bytes;
+    CUDA_TRY(c, launch_scan((const I64x2 *)c->mol_cnt.p, (I64x2 *)c->off.p, c->ND + 1, c->scan_tmp.p, &tb, c->stream));
+    launches += 2;
+    ChunkParams cp;
+    cp.ND = c->ND;
+    cp.goff = c->dd.goff;
+    cp.off = (const I64x2 *)c->off.p;
+    cp.PC = c->PC;
+    cp.AC = c->AC;
+    cp.CMC = c->CMC;
+    cp.MC = c->MC;
+    cp.chunk_start = (int32_t *)c->chunk_start.p;
+    cp.nchunks = (int32_t *)c->nchunks.p;
+    CUDA_TRY(c, launch_chunks(cp, c->stream));
+    launches++;
+    timing_mark(c);
+  }
+  if (c->timing.enabled) {
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    c->last.query_prep_ms = prog_timed ? timing_ms(c, 0, 1) : 0.f;
+    c->last.filter_ms = timing_ms(c, t0, t0 + 1);
+    c->last.support_ms = 0.f;
+    c->last.mapping_ms = timing_ms(c, t0 + 1, t0 + 2);
+  }
+  c->last.filter_launches = launches;
+  c->levels = levels;
+  c->flags = flags;
+  c->state = 2;
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_out) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_join before sigmo_filter");
+  if (mode != SIGMO_FIND_ALL && mode != SIGMO_FIND_FIRST) return set_err(c, SIGMO_ERR_INVALID_ARG, "bad mode %d", (int)mode);
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  c->timing.n = 0;
+  timing_mark(c);
+  CUDA_TRY(c, cudaMemsetAsync(c->jcnt.p, 0, 8 * ((size_t)c->NQ + 2), c->stream));
+  int launches = 0;
+  if (c->ND > 0 && c->VD > 0 && c->NQ > 0) {
+    JoinParams jp{};
+    jp.ND = c->ND;
+    jp.NQ = c->NQ;
+    jp.NQW = c->NQW;
+    jp.VQ = c->VQ;
+    jp.Wpad = c->Wpad;
+    jp.NB = c->NB;
+    jp.goff = c->dd.goff;
+    jp.roff = c->dd.roff;
+    jp.nbr = c->dd.nbr;
+    jp.bclass = c->bclass;
+    jp.bitmap = (const uint32_t *)c->bitmap.p;
+    jp.gm = (const uint32_t *)c->gm.p;
+    jp.off = (const I64x2 *)c->off.p;
+    jp.chunk_start = (const int32_t *)c->chunk_start.p;
+    jp.nchunks = (const int32_t *)c->nchunks.p;
+    jp.chunk_counter = (int *)c->jcnt.p;
+    jp.qgoff = c->dq.goff;
+    jp.qp_row = c->qp_row;
+    jp.qp_beoff = c->qp_beoff;
+    jp.qp_be = c->qp_be;
+    jp.pair_query = (int32_t *)c->pair_query.p;
+    jp.pair_result = (unsigned long long *)c->pair_result.p;
+    jp.totals = (unsigned long long *)c->jcnt.p + 2;
+    jp.maxq = std::max(c->maxq, 2);
+    jp.PCAP = c->PC + c->NQ;
+    jp.ACAP = c->AC + c->maxn;
+    jp.CMCAP = c->CMC + c->VQ;
+    jp.MCAP = c->MC;
+    const size_t smem = join_smem_bytes(c->NW, jp);
+    if (smem > c->max_smem) return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
+    jp.smem_bytes = smem;
+    const int bps = join_blocks_per_sm(c->NW, (int)mode, smem);
+    const int grid = bps * c->sm_count;
+    CUDA_TRY(c, launch_join(c->NW, (int)mode, jp, grid, c->stream));
+    launches++;
+  }
+  timing_mark(c);
+  if (c->timing.enabled) {
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    c->last.join_ms = timing_ms(c, 0, 1);
+  }
+  c->last.join_launches = launches;
+  c->last_mode = (int)mode;
+  c->state = 3;
+  if (total_matches_out) {
+    std::vector<uint64_t> t((size_t)c->NQ + 1);
+    if (c->NQ > 0)
+      CUDA_TRY(c, cudaMemcpyAsync(t.data(), (uint64_t *)c->jcnt.p + 2, 8 * (size_t)c->NQ, cudaMemcpyDeviceToHost,
+                                  c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    uint64_t s = 0;
+    for (int q = 0; q < c->NQ; q++) s += t[q];
+    *total_matches_out = s;
+  }
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_num_pairs(sigmo_ctx *c, int64_t *n) {
+  if (!c || !n) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_num_pairs before sigmo_filter");
+  if (c->ND == 0 || c->VD == 0) {
+    *n = 0;
+    return SIGMO_OK;
+  }
+  I64x2 t;
+  CUDA_TRY(c, cudaMemcpyAsync(&t, (I64x2 *)c->off.p + c->ND, sizeof(I64x2), cudaMemcpyDeviceToHost, c->stream));
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  *n = t.a;
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_get_pair_results(sigmo_ctx *c, int64_t cap, int64_t *n, int64_t *data_idx, int32_t *query_idx,
+                                    uint64_t *result) {
+  if (!c || !n) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 3) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_pair_results before sigmo_join");
+  int64_t P = 0;
+  SIGMO_TRY(sigmo_num_pairs(c, &P));
+  *n = P;
+  if (cap < P) return set_err(c, SIGMO_ERR_INVALID_ARG, "capacity %lld < %lld pairs", (long long)cap, (long long)P);
+  if (P == 0) return SIGMO_OK;
+  if (query_idx)
+    CUDA_TRY(c, cudaMemcpyAsync(query_idx, c->pair_query.p, 4 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
+  if (result)
+    CUDA_TRY(c, cudaMemcpyAsync(result, c->pair_result.p, 8 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
+  std::vector<I64x2> off;
+  if (data_idx) {
+    off.resize((size_t)c->ND + 1);
+    CUDA_TRY(c, cudaMemcpyAsync(off.data(), c->off.p, sizeof(I64x2) * off.size(), cudaMemcpyDeviceToHost, c->stream));
+  }
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  if (data_idx)
+    for (int g = 0; g < c->ND; g++)
+      for (long long p = off[g].a; p < off[g + 1].a; p++) data_idx[p] = g;
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_get_dense_results(sigmo_ctx *c, uint64_t *out) {
+  if (!c || !out) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 3) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_dense_results before sigmo_join");
+  int64_t P = 0;
+  SIGMO_TRY(sigmo_num_pairs(c, &P));
+  std::vector<int64_t> di((size_t)P);
+  std::vector<int32_t> qi((size_t)P);
+  std::vector<uint64_t> r((size_t)P);
+  int64_t n = 0;
+  SIGMO_TRY(sigmo_get_pair_results(c, P, &n, di.data(), qi.data(), r.data()));
+  memset(out, 0, 8 * (size_t)c->NQ * c->ND);
+  for (int64_t p = 0; p < n; p++) out[(size_t)qi[p] * c->ND + di[p]] = r[p];
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_get_query_totals(sigmo_ctx *c, uint64_t *out, int device_ptr) {
+  if (!c || !out) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 3) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_query_totals before sigmo_join");
+  if (c->NQ == 0) return SIGMO_OK;
+  if (device_ptr) {
+    CUDA_TRY(c, cudaMemcpyAsync(out, (uint64_t *)c->jcnt.p + 2, 8 * (size_t)c->NQ, cudaMemcpyDeviceToDevice, c->stream));
+  } else {
+    CUDA_TRY(c, cudaMemcpyAsync(out, (uint64_t *)c->jcnt.p + 2, 8 * (size_t)c->NQ, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  }
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_get_candidates(sigmo_ctx *c, uint32_t *out) {
+  if (!c || !out) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_candidates before sigmo_filter");
+  if (c->VQ == 0 || c->W == 0) return SIGMO_OK;
+  CUDA_TRY(c, cudaMemcpy2DAsync(out, 4 * (size_t)c->W, c->bitmap.p, 4 * (size_t)c->Wpad, 4 * (size_t)c->W,
+                                (size_t)c->VQ, cudaMemcpyDeviceToHost, c->stream));
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_get_signatures(sigmo_ctx *c, int which, int radius, uint64_t *out) {
+  if (!c || !out || (which != 0 && which != 1)) return SIGMO_ERR_INVALID_ARG;
+  if (radius < 1 || radius > 255) return set_err(c, SIGMO_ERR_INVALID_ARG, "radius %d not in 1..255", radius);
+  if (c->state < 1) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_signatures before sigmo_load_batch");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  const DevGraphs &g = which == 0 ? c->dq : c->dd;
+  if (g.num_nodes == 0) return SIGMO_OK;
+  SIGMO_TRY(dreserve(c, c->sig_tmp, 8 * (size_t)g.num_nodes, "signature export"));
+  CUDA_TRY(c, launch_sig_pack(g, radius, (unsigned long long *)c->sig_tmp.p, c->stream));
+  CUDA_TRY(c, cudaMemcpyAsync(out, c->sig_tmp.p, 8 * (size_t)g.num_nodes, cudaMemcpyDeviceToHost, c->stream));
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  return SIGMO_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,126 @@
+// sigmo_internal.h -- internal (non-ABI) structures shared by the host side
+// (sigmo_abi.cu) and the device side (sigmo_kernels.cu) of libsigmo.so.
+// Nothing here is visible to the oracle (oracle/ shares no code with this).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace sigmo {
+
+constexpr int kNumFields = 13;   // R7 field table (see sigmo_kernels.cu kFieldWidth)
+constexpr int kMaxRadius = 15;   // levels <= 16
+constexpr int kFilterThreads = 256;
+constexpr int kJoinThreads = 256;
+constexpr int kQueryPrepThreads = 1024;
+
+struct I64x2 {
+  long long a, b;
+};
+
+// Packed CSR-GO batch on the device (produced by sigmo_load_batch).
+//   nbr[e] = (molecule-local index of the neighbour << 8) | bond label
+struct DevGraphs {
+  int num_graphs = 0, num_nodes = 0, num_adj = 0, max_nodes = 0;
+  const int32_t *goff = nullptr;   // [G+1]
+  const uint8_t *label = nullptr;  // [V]
+  const uint8_t *local = nullptr;  // [V] index of the node inside its graph
+  const int32_t *roff = nullptr;   // [V+1]
+  const uint16_t *nbr = nullptr;   // [E2]
+};
+
+// Query-side plane program, built on the device by k_query_prep from the
+// query signatures (one per `levels`); see DESIGN.md "Filter".
+struct QueryProgMeta {
+  int P;       // distinct (radius, field, threshold) planes
+  int G;       // distinct (radius, field) count groups
+  int NFU;     // fields used by any plane
+  int NLAB;    // distinct query labels (label planes)
+  int row_entries;
+  int err;
+};
+
+struct QueryProg {
+  QueryProgMeta meta{};
+  int R = 0;                   // levels - 1
+  // device arrays
+  uint8_t *p_t = nullptr;      // [P]   threshold t of plane p
+  int16_t *grp_poff = nullptr; // [G+1] plane range of group
+  uint8_t *grp_f = nullptr;    // [G]   field of group
+  int16_t *rg_off = nullptr;   // [R+1] group range per radius
+  int8_t *fslot = nullptr;     // [13]  used-field slot or -1
+  uint8_t *lab_val = nullptr;  // [NLAB]
+  uint8_t *row_lab = nullptr;  // [VQ]  label-plane index of query node
+  int32_t *row_off = nullptr;  // [VQ+1]
+  uint16_t *row_ids = nullptr; // plane ids per query node
+  QueryProgMeta *d_meta = nullptr;
+};
+
+struct FilterParams {
+  DevGraphs D;
+  int TW, W, Wpad;
+  int VQ, NQ, NQW;
+  int R;
+  int P, G, NFU, NLAB;
+  const uint8_t *p_t;
+  const int16_t *grp_poff;
+  const uint8_t *grp_f;
+  const int16_t *rg_off;
+  const int8_t *fslot;
+  const uint8_t *lab_val;
+  const uint8_t *row_lab;
+  const int32_t *row_off;
+  const uint16_t *row_ids;
+  const int32_t *qgoff;        // [NQ+1] query node offsets (rows)
+  uint32_t *bitmap;            // [VQ][Wpad]
+  uint32_t *gm;                // [ND][NQW] surviving-query bits per data graph
+  I64x2 *mol_cnt;              // [ND+1] (surviving pairs, candidate-mask entries)
+  int EXTN, EXTW, MOLCAP;
+  size_t smem_bytes;
+};
+
+struct JoinParams {
+  int ND, NQ, NQW, VQ, Wpad, NB;
+  const int32_t *goff;
+  const int32_t *roff;
+  const uint16_t *nbr;
+  const uint8_t *bclass;       // [256] bond label -> class (255 = not in any query)
+  const uint32_t *bitmap;
+  const uint32_t *gm;
+  const I64x2 *off;            // [ND+1] exclusive scan of mol_cnt
+  const int32_t *chunk_start;  // [nchunks+1]
+  const int32_t *nchunks;      // device scalar
+  int *chunk_counter;          // device scalar (zeroed before launch)
+  const int32_t *qgoff;        // [NQ+1]
+  const int32_t *qp_row;       // [VQ] plan order: global query node of depth e
+  const int32_t *qp_beoff;     // [VQ+1] back-edge list per (query, depth)
+  const uint16_t *qp_be;       // (depth j << 8) | bond class
+  int32_t *pair_query;
+  unsigned long long *pair_result;
+  unsigned long long *totals;  // [NQ]
+  int PCAP, ACAP, CMCAP, MCAP, maxq;
+  size_t smem_bytes;
+};
+
+struct ChunkParams {
+  int ND;
+  const int32_t *goff;
+  const I64x2 *off;
+  long long PC, AC, CMC, MC;
+  int32_t *chunk_start;
+  int32_t *nchunks;
+};
+
+// ---- launchers (sigmo_kernels.cu); all enqueue on `st` ----
+cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, cudaStream_t st);
+cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *out, cudaStream_t st);
+cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts, QueryProg &prog,
+                              cudaStream_t st);
+cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
+size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P);
+cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);
+cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
+cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);
+size_t join_smem_bytes(int NW, const JoinParams &p);
+int join_blocks_per_sm(int NW, int mode, size_t smem);
+
+}  // namespace sigmo

@@ -1,0 +1,214 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle (bit-exact).
+
+Every count and flag is an exact integer: bitmaps,
+signatures, GMCR pairs, Find All counts and Find First flags must be equal
+element by element.  Sizes span many filter tiles (1024 data nodes each),
+many join chunks and ragged tails."""
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from oracle import filter_ref as fr
+from synth import GraphBatch
+
+pytestmark = pytest.mark.gpu
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+@pytest.fixture(scope="module")
+def sigmo():
+    import torch
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_sc_carocfc25_b200 as s
+    torch.cuda.set_device(0)
+    return s
+
+
+@pytest.fixture()
+def ctx(sigmo):
+    c = sigmo.Context(0)
+    yield c
+    c.close()
+
+
+def run(ctx, Q, D, levels, mode):
+    ctx.load_batch(Q, D)
+    ctx.filter(levels)
+    total = ctx.join(mode)
+    return total, ctx.dense_results()
+
+
+def ring(n, lab=6, bond=1):
+    return [lab] * n, [(i, (i + 1) % n, bond) for i in range(n)]
+
+
+def path(n, lab=6, bond=1):
+    return [lab] * n, [(i, i + 1, bond) for i in range(n - 1)]
+
+
+def star(d, lab=6, bond=1):
+    return [lab] * (d + 1), [(0, i, bond) for i in range(1, d + 1)]
+
+
+def test_fig3_closed_forms(ctx, sigmo):
+    D = synth.fig3_batch()
+    Q = GraphBatch.from_graphs([path(2), path(3), ring(5), star(3)])
+    expect = np.array([[10, 6], [10, 6], [10, 0], [0, 6]], np.uint64)
+    for L in (1, 2, 3, 4, 7):
+        tot, dense = run(ctx, Q, D, L, sigmo.SIGMO_FIND_ALL)
+        assert np.array_equal(dense, expect), L
+        assert tot == int(expect.sum())
+        ctx.join(sigmo.SIGMO_FIND_FIRST)
+        assert np.array_equal(ctx.dense_results(), (expect > 0).astype(np.uint64))
+
+
+def test_signatures_match_reference(ctx):
+    Q = synth.config_queries(4)  # includes 20-30-atom ring systems
+    D = synth.config_data(1)
+    ctx.load_batch(Q, D)
+    for r in (1, 2, 3, 5):
+        assert np.array_equal(ctx.signatures(0, r), fr.signatures(Q, r)), ("query", r)
+        assert np.array_equal(ctx.signatures(1, r), fr.signatures(D, r)), ("data", r)
+
+
+def test_signature_saturation(ctx):
+    # a 100-atom N chain: the 6-bit N field saturates at 63 (R8)
+    D = GraphBatch.from_graphs([path(100, 7), ring(6, 6, 4)])
+    Q = GraphBatch.from_graphs([path(3, 7)])
+    ctx.load_batch(Q, D)
+    for r in (1, 10, 40, 70):
+        assert np.array_equal(ctx.signatures(1, r), fr.signatures(D, r)), r
+
+
+@pytest.mark.parametrize("levels", [1, 2, 3, 4, 5])
+def test_c1_bitmap_and_counts(ctx, sigmo, levels):
+    Q, D = synth.config_queries(1), synth.config_data(1)
+    ctx.load_batch(Q, D)
+    ctx.filter(levels)
+    assert np.array_equal(ctx.candidates(), fr.candidates(Q, D, levels))
+    Cb = fr.candidates_bool(Q, D, levels)
+    G = fr.gmcr(Q, D, Cb)
+    assert ctx.num_pairs() == int(G.sum())
+    tot = ctx.join(sigmo.SIGMO_FIND_ALL)
+    ref = oracle.count_dense(Q, D)
+    assert np.array_equal(ctx.dense_results(), ref)
+    assert tot == int(ref.sum())
+    di, qi, r = ctx.pair_results()
+    assert np.array_equal(G[qi, di], np.ones(len(di), bool))  # exactly the GMCR pairs
+    assert np.all(np.diff(di) >= 0)
+    assert np.array_equal(ctx.query_totals(), ref.sum(axis=1).astype(np.uint64))
+    ctx.join(sigmo.SIGMO_FIND_FIRST)
+    assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D, oracle.FIND_FIRST))
+
+
+def test_levels_monotone_and_sound(ctx):
+    Q, D = synth.config_queries(2), synth.config_data(2, count=300)
+    ctx.load_batch(Q, D)
+    prev = None
+    for L in range(1, 8):
+        ctx.filter(L)
+        bm = ctx.candidates()
+        if prev is not None:
+            assert not np.any(bm & ~prev)
+        prev = bm
+    ctx.filter(6)
+    assert np.array_equal(ctx.candidates(), fr.candidates(Q, D, 6))
+
+
+def test_edge_cases_batch(ctx, sigmo):
+    """empty data graphs, single-atom graphs, disconnected graphs, single-node
+    and disconnected queries, graphs > 64 atoms (multi-word masks)."""
+    rng = np.random.default_rng(11)
+    mols = synth.molecules(synth.DATA_SEED_BASE + 77, 0, 120, mode=2)
+    graphs = mols.graphs()
+    graphs.insert(0, ([], []))
+    graphs.insert(5, ([6], []))
+    graphs.insert(9, ([], []))
+    graphs.append(([6, 6, 8, 6], [(0, 1, 1), (2, 3, 1)]))
+    graphs.append(([], []))
+    big = ([6] * 100, [(i, i + 1, 1) for i in range(99)] + [(0, 99, 1)])
+    graphs.insert(50, big)
+    D = GraphBatch.from_graphs(graphs)
+    assert D.sizes().max() > 64
+    qs = synth.library(synth.C1_NAMES) + [([6], []), ([8], []), ([6, 8], []), ([6, 6, 6], [(0, 1, 1)]),
+                                          path(7), ring(6, 6, 4)]
+    Q = GraphBatch.from_graphs(qs)
+    for L in (1, 3, 5):
+        tot, dense = run(ctx, Q, D, L, sigmo.SIGMO_FIND_ALL)
+        ref = oracle.count_dense(Q, D)
+        assert np.array_equal(dense, ref), L
+        assert np.array_equal(ctx.candidates(), fr.candidates(Q, D, L))
+        ctx.join(sigmo.SIGMO_FIND_FIRST)
+        assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D, oracle.FIND_FIRST))
+
+
+def test_large_ring_system_queries(ctx, sigmo):
+    Q = synth.config_queries(4)
+    D = synth.config_data(4, count=400)
+    ctx.load_batch(Q, D)
+    ctx.filter(4)
+    ctx.join(sigmo.SIGMO_FIND_ALL)
+    assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D))
+    ctx.join(sigmo.SIGMO_FIND_FIRST)
+    assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D, oracle.FIND_FIRST))
+
+
+def test_random_tiny_graphs_vs_oracle(ctx, sigmo):
+    rng = np.random.default_rng(2024)
+    ds = [synth.random_labelled_graph(rng, int(rng.integers(0, 12)), float(rng.uniform(0.1, 0.7)),
+                                      labels=(6, 7), bonds=(1, 2)) for _ in range(400)]
+    qs = [synth.random_labelled_graph(rng, int(rng.integers(1, 6)), float(rng.uniform(0.3, 1.0)),
+                                      labels=(6, 7), bonds=(1, 2)) for _ in range(40)]
+    Q, D = GraphBatch.from_graphs(qs), GraphBatch.from_graphs(ds)
+    for L in (1, 2, 4):
+        _, dense = run(ctx, Q, D, L, sigmo.SIGMO_FIND_ALL)
+        assert np.array_equal(dense, oracle.count_dense(Q, D)), L
+
+
+def test_empty_data_batch_and_state_errors(ctx, sigmo):
+    Q = synth.config_queries(1)
+    with pytest.raises(sigmo.SigmoError) as e:
+        ctx.filter(2)
+    assert e.value.status == -4
+    ctx.load_batch(Q, GraphBatch.empty())
+    with pytest.raises(sigmo.SigmoError) as e:
+        ctx.join(sigmo.SIGMO_FIND_ALL)
+    assert e.value.status == -4
+    ctx.filter(3)
+    assert ctx.num_pairs() == 0
+    assert ctx.join(sigmo.SIGMO_FIND_ALL) == 0
+    assert ctx.query_totals().sum() == 0
+    with pytest.raises(sigmo.SigmoError) as e:
+        ctx.filter(17)
+    assert e.value.status == -1
+
+
+def test_c2_full_size_parity(ctx, sigmo):
+    """configs[1] at full size in the bench's launch configuration: every one
+    of the 5M pairs bit-exact against the oracle (Find All and Find First)."""
+    Q, D = synth.config_queries(2), synth.config_data(2)
+    ctx.load_batch(Q, D)
+    ctx.filter(4)
+    tot = ctx.join(sigmo.SIGMO_FIND_ALL)
+    got = ctx.dense_results()
+    ref = oracle.count_dense(Q, D)
+    assert tot == int(ref.sum())
+    assert np.array_equal(got, ref)
+    ctx.join(sigmo.SIGMO_FIND_FIRST)
+    assert np.array_equal(ctx.dense_results(), (ref > 0).astype(np.uint64))
+    # bitmap on sampled molecules vs the filter reference
+    rng = np.random.default_rng(5)
+    gs = sorted(int(g) for g in rng.choice(D.num_graphs, 60, replace=False))
+    bm = ctx.candidates()
+    Cb = fr.candidates_bool(Q, D, 4, data_graphs=gs)
+    ref_bits = fr.to_bitmap(Cb)
+    for g in gs:
+        lo, hi = int(D.graph_offsets[g]), int(D.graph_offsets[g + 1])
+        for v in range(lo, hi):
+            w, b = v >> 5, v & 31
+            assert np.array_equal((bm[:, w] >> b) & 1, (ref_bits[:, w] >> b) & 1), (g, v)
