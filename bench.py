@@ -1,0 +1,392 @@
+#!/usr/bin/env python
+"""SIGMo B200 benchmark (driver contract: one JSON line on rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl sigmo|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...      (N > 1)
+
+Workload (N=1): BASELINE.json configs[1] = 50 queries (35 library functional
+groups + 15 random 3-8-atom subgraphs) x 100k synthetic ZINC-like molecules,
+Find All, filter levels 4.  Weak scaling: rank r owns
+molecules [r*100k, (r+1)*100k) of the same counter-based stream; queries are
+replicated; the only collective is an NCCL all-reduce of the per-query
+totals.
+
+A step = one pass of the hot path over the resident batch: sigmo_filter
+(signatures + dominance + bitmap + GMCR) -> sigmo_join(Find All) -> per-query
+totals (+ all-reduce).  Each timed step is bracketed by CUDA events on the
+ctx stream; L2 (126 MB) is flushed by a 256 MiB write before every step,
+outside the events.  value = all matches of all ranks / max-over-ranks time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+BASELINE_METRIC = "matches/sec (Find All) and graph-pairs/sec (Find First) at 1/2/4/8 B200"
+CONFIG_ID = 2
+MOLS_PER_RANK = 100_000
+LEVELS = 4
+CPU_SAMPLE_MOLS = 20_000      # cpu_baseline leg: ~20 core-seconds of oracle work
+REF_STEP_MOLS = 2_000         # --impl reference: molecules per step
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="sigmo", choices=["sigmo", "reference"])
+    ap.add_argument("--levels", type=int, default=LEVELS)
+    ap.add_argument("--molecules", type=int, default=MOLS_PER_RANK, help="molecules per rank")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--no-flush", action="store_true")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------------------
+# clocks during the timed region (NVML)
+# ----------------------------------------------------------------------------
+REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+           0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+           0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+
+class ClockSampler:
+    def __init__(self, cuda_index: int):
+        self.samples = []
+        self.reasons = 0
+        self.max_mhz = None
+        self.ok = False
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            import torch
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            h = None
+            try:
+                want = str(torch.cuda.get_device_properties(cuda_index).uuid)
+                for i in range(pynvml.nvmlDeviceGetCount()):
+                    hi = pynvml.nvmlDeviceGetHandleByIndex(i)
+                    u = pynvml.nvmlDeviceGetUUID(hi)
+                    u = u.decode() if isinstance(u, bytes) else u
+                    if want and want in u:
+                        h = hi
+                        break
+            except Exception:
+                h = None
+            if h is None:
+                vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+                idx = int(vis.split(",")[cuda_index]) if vis and vis.split(",")[0].isdigit() else cuda_index
+                h = pynvml.nvmlDeviceGetHandleByIndex(idx)
+            self.h = h
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = repr(e)
+
+    def _reasons(self):
+        f = getattr(self.nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+            self.nv.nvmlDeviceGetCurrentClocksThrottleReasons
+        return int(f(self.h))
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.reasons |= self._reasons()
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml_unavailable"]}
+        rs = [n for b, n in REASONS.items() if self.reasons & b and n != "gpu_idle"]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None, "sm_max_mhz": self.max_mhz,
+                "reasons": rs, "samples": len(self.samples)}
+
+
+# ----------------------------------------------------------------------------
+def dist_setup(args):
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        if torch.cuda.is_available() and args.impl == "sigmo":
+            torch.cuda.set_device(local)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
+    elif torch.cuda.is_available() and args.impl == "sigmo":
+        torch.cuda.set_device(0)
+    return world, rank, local
+
+
+def host_cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:  # pragma: no cover
+        return os.cpu_count() or 1
+
+
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def run_cpu_baseline(Q, levels):
+    """The oracle as it stands, on a bounded sample of the same workload."""
+    import oracle
+    import synth
+    D = synth.config_data(CONFIG_ID, first=0, count=CPU_SAMPLE_MOLS)
+    th = host_cores()
+    t0 = time.perf_counter()
+    res = oracle.count_dense(Q, D, oracle.FIND_ALL, nthreads=th)
+    dt = time.perf_counter() - t0
+    t1 = time.perf_counter()
+    oracle.count_dense(Q, D, oracle.FIND_FIRST, nthreads=th)
+    dt_ff = time.perf_counter() - t1
+    return {"value": float(res.sum()) / dt, "unit": "matches/s", "cores": th, "kind": "oracle",
+            "sample": f"{Q.num_graphs} queries x first {CPU_SAMPLE_MOLS} molecules of configs[1] (Find All), "
+                      f"{dt:.2f} s wall on {th} threads; {int(res.sum())} matches",
+            "find_first_pairs_per_s": Q.num_graphs * D.num_graphs / dt_ff, "cpu_model": cpu_model()}
+
+
+# ----------------------------------------------------------------------------
+def run_reference(args, world, rank):
+    """--impl reference: the CPU oracle on the same config/metric (rank 0 only)."""
+    if rank != 0:
+        return
+    import oracle
+    import synth
+    Q = synth.config_queries(CONFIG_ID)
+    th = host_cores()
+    n_total = args.molecules
+    step_mols = min(REF_STEP_MOLS, n_total)
+
+    def batch(i):
+        first = (i * step_mols) % max(n_total - step_mols + 1, 1)
+        return synth.config_data(CONFIG_ID, first=first, count=step_mols)
+
+    for i in range(args.warmup):
+        oracle.count_dense(Q, batch(i), oracle.FIND_ALL, nthreads=th)
+    batches = [batch(args.warmup + i) for i in range(args.steps)]
+    matches = 0
+    t = 0.0
+    for D in batches:
+        t0 = time.perf_counter()
+        r = oracle.count_dense(Q, D, oracle.FIND_ALL, nthreads=th)
+        t += time.perf_counter() - t0
+        matches += int(r.sum())
+    value = matches / t
+    line = {"impl": "reference", "metric": BASELINE_METRIC, "value": value, "unit": "matches/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * t / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "config": config_dict(args, world, oracle_step=step_mols),
+            "cpu_baseline": {"value": value, "unit": "matches/s", "cores": th, "kind": "oracle",
+                             "sample": f"{Q.num_graphs} queries x {step_mols} molecules of configs[1] per step, "
+                                       f"{args.steps} steps", "cpu_model": cpu_model()},
+            "e2e": {"value": value, "unit": "matches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def config_dict(args, world, oracle_step=None):
+    d = {"workload": f"configs[1]: 50 queries x {args.molecules} ZINC-like molecules per GPU, Find All, "
+                     f"levels={args.levels}",
+         "queries": 50, "molecules_per_gpu": args.molecules, "molecules_total": args.molecules * world,
+         "levels": args.levels, "mode": "find_all", "data_seed": hex(0x51C0_0000 + CONFIG_ID),
+         "query_seed": hex(0x9E00_0000 + CONFIG_ID),
+         "l2": "flushed before every timed step (256 MiB device write, outside the events)",
+         "parallelism": f"dp{world}: molecule shards, queries replicated, NCCL all-reduce of per-query totals"}
+    if oracle_step:
+        d["oracle_molecules_per_step"] = oracle_step
+    return d
+
+
+# ----------------------------------------------------------------------------
+def main():
+    args = parse()
+    world, rank, local = dist_setup(args)
+    if args.impl == "reference":
+        run_reference(args, world, rank)
+        return
+    import numpy as np
+    import torch
+
+    import synth
+    import paper_conf_sc_carocfc25_b200 as sigmo
+
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+    Q = synth.config_queries(CONFIG_ID)
+    D = synth.config_data(CONFIG_ID, first=rank * args.molecules, count=args.molecules)
+    stream = torch.cuda.current_stream(dev)
+    ctx = sigmo.Context(local, stream)
+    ctx.load_batch(Q, D)
+    totals = torch.zeros(Q.num_graphs, dtype=torch.int64, device=dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
+
+    def step(mode=sigmo.SIGMO_FIND_ALL):
+        ctx.filter(args.levels)
+        ctx.join(mode, total=False)
+        ctx.query_totals(device_tensor=totals)
+        if dist is not None:
+            dist.all_reduce(totals)
+
+    # ---- warm-up ----
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize(dev)
+
+    def timed_loop(mode, K, with_timing):
+        ctx.set_timing(with_timing)
+        starts = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+        ends = [torch.cuda.Event(enable_timing=True) for _ in range(K)]
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        for i in range(K):
+            if not args.no_flush:
+                flush.fill_(i)
+            starts[i].record(stream)
+            step(mode)
+            ends[i].record(stream)
+        torch.cuda.synchronize(dev)
+        if dist is not None:
+            dist.barrier()
+        ms = sum(s.elapsed_time(e) for s, e in zip(starts, ends))
+        tim = ctx.timings() if with_timing else None
+        ctx.set_timing(False)
+        return ms, tim
+
+    sampler = ClockSampler(local)
+    with sampler:
+        ms_all, tim = timed_loop(sigmo.SIGMO_FIND_ALL, args.steps, True)
+    clocks = sampler.summary()
+    matches_local = int(ctx.join(sigmo.SIGMO_FIND_ALL))  # identical every step (deterministic)
+    pairs_local = ctx.num_pairs()
+    ms_ff, _ = timed_loop(sigmo.SIGMO_FIND_FIRST, args.steps, False)
+    positive_local = int(ctx.join(sigmo.SIGMO_FIND_FIRST))
+
+    # ---- e2e through the public API from host buffers ----
+    cq, cd = sigmo.as_c_batch(Q), sigmo.as_c_batch(D)
+    e2e_ms = []
+    for i in range(args.e2e_steps + 1):
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        ctx.load_batch(cq, cd)
+        ctx.filter(args.levels)
+        tot = ctx.join(sigmo.SIGMO_FIND_ALL, total=True)  # D2H of the per-query totals
+        dt = (time.perf_counter() - t0) * 1000
+        if i > 0:
+            e2e_ms.append(dt)
+        assert tot == matches_local
+    h2d = ctx.timings()["h2d_bytes"]
+
+    # ---- reduce over ranks ----
+    vals = torch.tensor([ms_all, ms_ff, sum(e2e_ms)], dtype=torch.float64, device=dev)
+    cnts = torch.tensor([matches_local, pairs_local, positive_local, Q.num_graphs * D.num_graphs],
+                        dtype=torch.int64, device=dev)
+    if dist is not None:
+        dist.all_reduce(vals, op=dist.ReduceOp.MAX)
+        dist.all_reduce(cnts)
+    ms_all, ms_ff, e2e_total = vals.tolist()
+    matches, pairs, positive, all_pairs = [int(x) for x in cnts.tolist()]
+    if rank != 0:
+        ctx.close()
+        if dist is not None:
+            dist.destroy_process_group()
+        return
+
+    K = args.steps
+    value = matches * K / (ms_all / 1000.0)
+    ms_per_step = ms_all / K
+    # ---- roofline of the dominant kernel (per-launch CUDA events over the timed region) ----
+    import json as _json
+    peaks = {}
+    try:
+        peaks = _json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
+    peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s"
+    VQ, VD, ND, NQ = Q.num_nodes, D.num_nodes, D.num_graphs, Q.num_graphs
+    W = (VD + 31) // 32
+    filter_bytes = (4 * VQ * W                       # bitmap written once
+                    + 4 * ND * ((NQ + 31) // 32) + 16 * ND  # GMCR bits + counts
+                    + 4 * (ND + 1) + 2 * VD + 4 * (VD + 1) + 2 * D.num_adj)  # packed CSR-GO read once
+    f_ms, j_ms, m_ms = tim["filter_ms"], tim["join_ms"], tim["mapping_ms"]
+    filter_roof = {"bound": "hbm", "achieved": filter_bytes / (f_ms * 1e-3) / 1e9, "peak": hbm_peak,
+                   "unit": "GB/s", "frac": filter_bytes / (f_ms * 1e-3) / 1e9 / hbm_peak, "traffic": None,
+                   "kernel": "k_filter", "ms": f_ms, "algorithmic_bytes": filter_bytes, "peak_source": peak_src}
+    # join: ALU/issue bound: achieved = surviving pairs/s
+    sm_mhz = clocks.get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
+    join_roof = {"bound": "alu", "kernel": "k_join", "ms": j_ms,
+                 "pairs_per_launch": pairs_local, "matches_per_launch": matches_local}
+    dominant = "join" if j_ms >= f_ms else "filter"
+    roofline = dict(filter_roof) if dominant == "filter" else None
+
+    line = {
+        "metric": BASELINE_METRIC, "value": value, "unit": "matches/s", "n_gpus": world, "steps": K,
+        "warmup": max(args.warmup, 3), "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": config_dict(args, world),
+        "find_first": {"value": all_pairs * K / (ms_ff / 1000.0), "unit": "graph-pairs/s",
+                       "positive_pairs_per_s": positive * K / (ms_ff / 1000.0), "ms_per_step": ms_ff / K},
+        "counts": {"matches": matches, "gmcr_pairs": pairs, "positive_pairs": positive, "all_pairs": all_pairs},
+        "stage_ms": {"filter": f_ms, "mapping": m_ms, "join": j_ms},
+        "roofline_filter": filter_roof,
+        "roofline_join": join_roof,
+        "dominant_kernel": dominant,
+        "e2e": {"value": matches * args.e2e_steps / (e2e_total / 1000.0), "unit": "matches/s",
+                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 8 * NQ,
+                "ms_per_step": e2e_total / args.e2e_steps,
+                "note": "sigmo_load_batch (validate+pack+pinned H2D) + filter + join + D2H totals, wall clock"},
+        "gpu_launches": int(K * (tim["filter_launches"] + tim["join_launches"])),
+        "clocks": clocks,
+    }
+    if roofline is not None:
+        line["roofline"] = roofline
+    if world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = run_cpu_baseline(Q, args.levels)
+    print(json.dumps(line), flush=True)
+    ctx.close()
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

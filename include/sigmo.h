@@ -102,15 +102,21 @@ typedef struct {
   void *user;
 } sigmo_allocator;
 
-/* Per-stage device times of the last filter/join (CUDA events on the ctx
- * stream; only filled when timing is enabled). Milliseconds. */
+/* Per-stage device times (ms), averaged over the filter/join calls made with
+ * timing enabled since the previous sigmo_get_timings (which resets them).
+ * CUDA events are recorded on the ctx stream around each kernel; recording
+ * never synchronizes, sigmo_get_timings does.  0 for stages not run. */
 typedef struct {
-  float query_prep_ms;  /* query signatures + plane/row programs (cached per levels) */
-  float filter_ms;      /* fused signature + dominance + bitmap + GMCR test kernel */
+  float query_prep_ms;  /* query signatures + plane/row programs (built once per levels) */
+  float filter_ms;      /* fused signature + dominance + bitmap + GMCR-test kernel */
   float support_ms;     /* neighbour-support fixed point (0 if flag off) */
-  float mapping_ms;     /* GMCR scan + chunking */
-  float join_ms;        /* DFS join + per-query totals */
-  int64_t filter_launches, join_launches;  /* kernels launched by the last filter / join */
+  float mapping_ms;     /* GMCR scan + join chunking */
+  float join_ms;        /* DFS join kernel (incl. per-query totals) */
+  int64_t filter_launches, join_launches;  /* kernels launched by the last filter / join call */
+  int64_t h2d_bytes;    /* bytes uploaded by the last sigmo_load_batch (one pinned H2D copy) */
+  int64_t filter_calls, join_calls;        /* calls averaged */
+  int64_t dfs_steps;    /* DFS iterator steps (search-tree nodes) of the last join */
+  int64_t dfs_iters, dfs_tail_iters, dfs_max_stack;  /* warp iterations, of which after the last pair claim; max stack */
 } sigmo_timings;
 
 /* Create a context on `device` (CUDA ordinal) enqueuing on `cuda_stream`

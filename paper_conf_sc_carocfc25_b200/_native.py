@@ -43,7 +43,10 @@ class sigmo_allocator(ctypes.Structure):
 class sigmo_timings(ctypes.Structure):
     _fields_ = [("query_prep_ms", ctypes.c_float), ("filter_ms", ctypes.c_float), ("support_ms", ctypes.c_float),
                 ("mapping_ms", ctypes.c_float), ("join_ms", ctypes.c_float),
-                ("filter_launches", ctypes.c_int64), ("join_launches", ctypes.c_int64)]
+                ("filter_launches", ctypes.c_int64), ("join_launches", ctypes.c_int64),
+                ("h2d_bytes", ctypes.c_int64), ("filter_calls", ctypes.c_int64),
+                ("join_calls", ctypes.c_int64), ("dfs_steps", ctypes.c_int64),
+                ("dfs_iters", ctypes.c_int64), ("dfs_tail_iters", ctypes.c_int64), ("dfs_max_stack", ctypes.c_int64)]
 
 
 _lib = None

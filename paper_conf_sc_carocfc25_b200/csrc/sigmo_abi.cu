@@ -34,10 +34,23 @@ struct Pinned {
   size_t cap = 0;
 };
 
+// Per-call CUDA events on the ctx stream (recording never synchronizes).
+// Each filter call uses one slot of a ring (events: 0/1 query program if it
+// was built by this call, 2/3 filter kernel, 4 end of GMCR scan + chunking);
+// each join call one slot of another ring (join kernel).  A slot is
+// harvested (its elapsed times added to running sums) when it is reused or
+// when sigmo_get_timings is called, which returns averages and resets.
 struct Timing {
+  static const int RING = 64;
   bool enabled = false;
-  cudaEvent_t ev[8] = {};
-  int n = 0;
+  cudaEvent_t fev[RING][5] = {};
+  bool frec[RING][5] = {};
+  bool fpend[RING] = {};
+  cudaEvent_t jev[RING][2] = {};
+  bool jpend[RING] = {};
+  int fi = 0, ji = 0, cur_f = -1, cur_j = -1;
+  double s_qprep = 0, s_filter = 0, s_mapping = 0, s_join = 0;
+  long long n_qprep = 0, n_filter = 0, n_mapping = 0, n_join = 0;
 };
 
 struct ProgCache {
@@ -92,7 +105,7 @@ struct sigmo_ctx {
   cudaEvent_t h2d_done = nullptr;
   DBuf arena;
   DevGraphs dq, dd;
-  int NQ = 0, VQ = 0, EQ = 0, NQW = 0, maxq = 0, NB = 0;
+  int NQ = 0, VQ = 0, EQ = 0, NQW = 0, maxq = 0, NB = 0, NBE = 0, plan_smem = 0;
   int ND = 0, VD = 0, ED = 0, maxn = 0, NW = 1;
   bool has_empty_graph = false;
   int W = 0, Wpad = 0;
@@ -112,9 +125,9 @@ struct sigmo_ctx {
   int PC = 512, AC = 512, CMC = 2048, MC = 128;
 
   // ---- join ----
-  DBuf pair_query, pair_result, jcnt;  // jcnt = [counter (8 B) | totals NQ u64]
+  DBuf pair_query, pair_result, jcnt;  // jcnt u64 slots: [0] chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
   int last_mode = 0;
-  DBuf sig_tmp;
+  DBuf sig_tmp, gstack;
 
   Timing timing;
   sigmo_timings last{};
@@ -408,16 +421,65 @@ int graph_of_host(const int64_t *goff, int64_t G, int64_t n) {
   return (int)lo;
 }
 
-void timing_mark(sigmo_ctx *c) {
-  if (c->timing.enabled && c->timing.n < 8) cudaEventRecord(c->timing.ev[c->timing.n++], c->stream);
-}
-
-float timing_ms(sigmo_ctx *c, int a, int b) {
+float ev_ms(cudaEvent_t a, cudaEvent_t b) {
   float ms = 0.f;
-  if (a < c->timing.n && b < c->timing.n) cudaEventElapsedTime(&ms, c->timing.ev[a], c->timing.ev[b]);
+  if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) {
+    cudaGetLastError();
+    return 0.f;
+  }
   return ms;
 }
 
+void harvest_f(Timing &T, int s) {
+  if (!T.fpend[s]) return;
+  int last = -1;
+  for (int k = 0; k < 5; k++)
+    if (T.frec[s][k]) last = k;
+  if (last >= 0) cudaEventSynchronize(T.fev[s][last]);
+  if (T.frec[s][0] && T.frec[s][1]) { T.s_qprep += ev_ms(T.fev[s][0], T.fev[s][1]); T.n_qprep++; }
+  if (T.frec[s][2] && T.frec[s][3]) { T.s_filter += ev_ms(T.fev[s][2], T.fev[s][3]); T.n_filter++; }
+  if (T.frec[s][3] && T.frec[s][4]) { T.s_mapping += ev_ms(T.fev[s][3], T.fev[s][4]); T.n_mapping++; }
+  T.fpend[s] = false;
+  for (int k = 0; k < 5; k++) T.frec[s][k] = false;
+}
+
+void harvest_j(Timing &T, int s) {
+  if (!T.jpend[s]) return;
+  cudaEventSynchronize(T.jev[s][1]);
+  T.s_join += ev_ms(T.jev[s][0], T.jev[s][1]);
+  T.n_join++;
+  T.jpend[s] = false;
+}
+
+void timing_begin_filter(sigmo_ctx *c) {
+  Timing &T = c->timing;
+  if (!T.enabled) { T.cur_f = -1; return; }
+  const int s = T.fi;
+  T.fi = (T.fi + 1) % Timing::RING;
+  harvest_f(T, s);
+  T.cur_f = s;
+}
+
+void timing_mark(sigmo_ctx *c, int k) {
+  Timing &T = c->timing;
+  if (!T.enabled || T.cur_f < 0) return;
+  cudaEventRecord(T.fev[T.cur_f][k], c->stream);
+  T.frec[T.cur_f][k] = true;
+  T.fpend[T.cur_f] = true;
+}
+
+void timing_join(sigmo_ctx *c, int k) {
+  Timing &T = c->timing;
+  if (!T.enabled) return;
+  if (k == 0) {
+    const int s = T.ji;
+    T.ji = (T.ji + 1) % Timing::RING;
+    harvest_j(T, s);
+    T.cur_j = s;
+  }
+  cudaEventRecord(T.jev[T.cur_j][k], c->stream);
+  if (k == 1) T.jpend[T.cur_j] = true;
+}
 
 // ---------------------------------------------------------------------------
 // query plane program (cached per R = levels - 1)
@@ -458,14 +520,14 @@ sigmo_status ensure_prog(sigmo_ctx *c, int R, QueryProg *&out) {
   P.row_off = (int32_t *)(b + o_ro);
   P.row_ids = (uint16_t *)(b + o_ri);
   P.d_meta = (QueryProgMeta *)(b + o_me);
-  timing_mark(c);
+  timing_mark(c, 0);
   if (R > 0) {
     SIGMO_TRY(dreserve(c, c->qcounts, (size_t)VQ * R * kNumFields, "query counts"));
     CUDA_TRY(c, launch_sig_counts(c->dq, R, (uint8_t *)c->qcounts.p, c->stream));
   }
   CUDA_TRY(c, launch_query_prep(c->dq, R, (const uint8_t *)c->qcounts.p, P, c->stream));
+  timing_mark(c, 1);
   CUDA_TRY(c, cudaMemcpyAsync(&P.meta, P.d_meta, sizeof(QueryProgMeta), cudaMemcpyDeviceToHost, c->stream));
-  timing_mark(c);
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
   if (P.meta.err) return set_err(c, SIGMO_ERR_LIMIT, "query program error %d", P.meta.err);
   pc.valid = true;
@@ -499,8 +561,40 @@ void free_all(sigmo_ctx *c) {
   for (auto &kv : c->progs) dfree(c, kv.second.buf);
   c->progs.clear();
   DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
-                  &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_result, &c->jcnt, &c->sig_tmp};
+                  &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_result, &c->jcnt, &c->sig_tmp, &c->gstack};
   for (DBuf *b : bufs) dfree(c, *b);
+}
+
+// chunk/stack/slice capacities of the join for the loaded batch
+void fill_join_caps(sigmo_ctx *c, JoinParams &jp) {
+  jp.NQ = c->NQ;
+  jp.NQW = c->NQW;
+  jp.VQ = c->VQ;
+  jp.NB = c->NB;
+  jp.maxq = std::max(c->maxq, 2);
+  jp.PCAP = c->PC + c->NQ;
+  jp.ACAP = c->AC + c->maxn;
+  jp.CMCAP = c->CMC + c->VQ;
+  jp.MCAP = c->MC;
+  jp.NBE = c->NBE;
+  jp.plan_smem = c->plan_smem;
+  const int scg = 32 * (jp.maxq + 1) + 64;
+  jp.SCS = std::min(scg, 160);
+  jp.SW = (jp.ACAP + 31) / 32 + 2;
+  jp.slice_rows = ((size_t)c->VQ * jp.SW * 4 <= 16384) ? c->VQ : 0;
+}
+
+// join internal-capacity flag and DFS step counter (synchronizes)
+sigmo_status read_join_flags(sigmo_ctx *c) {
+  unsigned long long f[6] = {0, 0, 0, 0, 0, 0};
+  CUDA_TRY(c, cudaMemcpyAsync(f, c->jcnt.p, sizeof(f), cudaMemcpyDeviceToHost, c->stream));
+  c->last.dfs_iters = (int64_t)f[3];
+  c->last.dfs_tail_iters = (int64_t)f[4];
+  c->last.dfs_max_stack = (int64_t)f[5];
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  c->last.dfs_steps = (int64_t)f[2];
+  if ((int)f[1] != 0) return set_err(c, SIGMO_ERR_LIMIT, "join DFS stack capacity exceeded (internal limit)");
+  return SIGMO_OK;
 }
 
 }  // namespace
@@ -559,7 +653,10 @@ sigmo_status sigmo_create(int device, void *cuda_stream, const sigmo_allocator *
     delete c;
     return SIGMO_ERR_CUDA;
   }
-  for (int i = 0; i < 8; i++) cudaEventCreate(&c->timing.ev[i]);
+  for (int r = 0; r < Timing::RING; r++) {
+    for (int k = 0; k < 5; k++) cudaEventCreate(&c->timing.fev[r][k]);
+    for (int k = 0; k < 2; k++) cudaEventCreate(&c->timing.jev[r][k]);
+  }
   *out = c;
   return SIGMO_OK;
 }
@@ -572,8 +669,10 @@ sigmo_status sigmo_destroy(sigmo_ctx *c) {
   cudaStreamSynchronize(c->stream);
   if (c->staging.p) cudaFreeHost(c->staging.p);
   if (c->h2d_done) cudaEventDestroy(c->h2d_done);
-  for (int i = 0; i < 8; i++)
-    if (c->timing.ev[i]) cudaEventDestroy(c->timing.ev[i]);
+  for (int r = 0; r < Timing::RING; r++) {
+    for (int k = 0; k < 5; k++) cudaEventDestroy(c->timing.fev[r][k]);
+    for (int k = 0; k < 2; k++) cudaEventDestroy(c->timing.jev[r][k]);
+  }
   delete c;
   return SIGMO_OK;
 }
@@ -587,6 +686,21 @@ sigmo_status sigmo_set_timing(sigmo_ctx *c, int enable) {
 sigmo_status sigmo_get_timings(sigmo_ctx *c, sigmo_timings *out) {
   if (!c || !out) return SIGMO_ERR_INVALID_ARG;
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  Timing &T = c->timing;
+  for (int s = 0; s < Timing::RING; s++) {
+    harvest_f(T, s);
+    harvest_j(T, s);
+  }
+  c->last.query_prep_ms = T.n_qprep ? (float)(T.s_qprep / T.n_qprep) : 0.f;
+  c->last.filter_ms = T.n_filter ? (float)(T.s_filter / T.n_filter) : 0.f;
+  c->last.support_ms = 0.f;
+  c->last.mapping_ms = T.n_mapping ? (float)(T.s_mapping / T.n_mapping) : 0.f;
+  c->last.join_ms = T.n_join ? (float)(T.s_join / T.n_join) : 0.f;
+  if (c->state >= 3) SIGMO_TRY(read_join_flags(c));
+  c->last.filter_calls = T.n_filter;
+  c->last.join_calls = T.n_join;
+  T.s_qprep = T.s_filter = T.s_mapping = T.s_join = 0;
+  T.n_qprep = T.n_filter = T.n_mapping = T.n_join = 0;
   *out = c->last;
   return SIGMO_OK;
 }
@@ -654,6 +768,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   SIGMO_TRY(dreserve(c, c->arena, total, "input arena"));
   unsigned char *db = (unsigned char *)c->arena.p;
   CUDA_TRY(c, cudaMemcpyAsync(db, hb, total, cudaMemcpyHostToDevice, c->stream));
+  c->last.h2d_bytes = (int64_t)total;
   CUDA_TRY(c, cudaEventRecord(c->h2d_done, c->stream));
   c->dq = dev_view(db, pq, hq);
   c->dd = dev_view(db, pd, hd);
@@ -677,23 +792,19 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->Wpad = ((c->W + 31) / 32) * 32;
   if (c->Wpad == 0) c->Wpad = 32;
   tile_geometry(c, hd);
-  // join chunk capacities (pairs, atoms, candidate masks, graphs per chunk):
-  // shrink until the join's shared memory fits one SM
+  c->NBE = (int)plan.be.size();
+  c->plan_smem = (4 * ((size_t)c->NQ + 1) + 8 * ((size_t)c->VQ + 1) + 2 * (size_t)c->NBE) <= 16384 ? 1 : 0;
+  // join chunk capacities (pairs, atoms, candidate masks, graphs per warp
+  // chunk): shrink until the join's shared memory allows >= 2 CTAs per SM
   {
-    c->PC = 512;
-    c->AC = 512;
-    c->CMC = 2048;
-    c->MC = 128;
+    c->PC = 64;
+    c->AC = 64;
+    c->CMC = 256;
+    c->MC = 16;
     for (int tries = 0; tries < 12; tries++) {
       JoinParams jp{};
-      jp.NQ = c->NQ;
-      jp.NB = c->NB;
-      jp.maxq = std::max(c->maxq, 2);
-      jp.PCAP = c->PC + c->NQ;
-      jp.ACAP = c->AC + c->maxn;
-      jp.CMCAP = c->CMC + c->VQ;
-      jp.MCAP = c->MC;
-      if (join_smem_bytes(c->NW, jp) <= c->max_smem) break;
+      fill_join_caps(c, jp);
+      if (join_smem_bytes(c->NW, jp) <= c->max_smem / 2 || c->PC == 1) break;
       c->PC = std::max(c->PC / 2, 1);
       c->AC = std::max(c->AC / 2, 1);
       c->CMC = std::max(c->CMC / 2, 1);
@@ -724,7 +835,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   SIGMO_TRY(dreserve(c, c->nchunks, 16, "chunk count"));
   SIGMO_TRY(dreserve(c, c->pair_query, 4 * (size_t)std::max(pair_cap, 1ll), "pair queries"));
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
-  SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 2), "join counters"));
+  SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 6), "join counters"));
   c->state = 1;
   c->err.clear();
   return SIGMO_OK;
@@ -739,13 +850,9 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     return set_err(c, SIGMO_ERR_INVALID_ARG, "SIGMO_FILTER_NEIGHBOR_SUPPORT not available in this build");
   CUDA_TRY(c, cudaSetDevice(c->device));
   const int R = levels - 1;
-  c->timing.n = 0;
+  timing_begin_filter(c);
   QueryProg *prog = nullptr;
   SIGMO_TRY(ensure_prog(c, R, prog));
-  const bool prog_timed = c->timing.n == 2;
-  if (c->timing.enabled && !prog_timed) c->timing.n = 0;
-  const int t0 = c->timing.n;
-  timing_mark(c);
   int launches = 0;
   if (c->ND > 0 && c->VD > 0) {
     const QueryProgMeta &m = prog->meta;
@@ -753,11 +860,17 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     const int tws[6] = {32, 16, 8, 4, 2, 1};
     int k = 0;
     size_t smem = 0;
-    for (k = 0; k < 6; k++) {
-      smem = filter_smem_bytes(c->NW, c->tile_extn[k], c->tile_extw[k], c->tile_molcap[k], m.NFU, m.NLAB, m.P);
-      if (smem <= c->max_smem) break;
+    int rows_smem = 1;
+    for (k = 0; k < 12; k++) {
+      rows_smem = k < 6 ? 1 : 0;
+      const int kk = k % 6;
+      smem = filter_smem_bytes(c->NW, c->tile_extn[kk], c->tile_extw[kk], c->tile_molcap[kk], m.NFU, m.NLAB, m.P,
+                               m.G, c->VQ, m.row_entries, rows_smem);
+      // prefer >= 2 CTAs per SM with row programs in shared memory
+      if (smem <= (rows_smem ? c->max_smem / 2 : c->max_smem)) break;
     }
-    if (k == 6) return set_err(c, SIGMO_ERR_LIMIT, "filter shared memory %zu exceeds %zu (P=%d)", smem, c->max_smem, m.P);
+    if (k == 12) return set_err(c, SIGMO_ERR_LIMIT, "filter shared memory %zu exceeds %zu (P=%d)", smem, c->max_smem, m.P);
+    k = k % 6;
     FilterParams fp{};
     fp.D = c->dd;
     fp.TW = tws[k];
@@ -787,15 +900,18 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.EXTN = c->tile_extn[k];
     fp.EXTW = c->tile_extw[k];
     fp.MOLCAP = c->tile_molcap[k];
+    fp.RE = m.row_entries;
+    fp.rows_smem = rows_smem;
     fp.smem_bytes = smem;
     if (c->has_empty_graph) {
       CUDA_TRY(c, cudaMemsetAsync(c->gm.p, 0, 4 * (size_t)c->ND * c->NQW, c->stream));
       CUDA_TRY(c, cudaMemsetAsync(c->mol_cnt.p, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
     }
     const int tiles = (c->W + fp.TW - 1) / fp.TW;
+    timing_mark(c, 2);
     CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));
     launches++;
-    timing_mark(c);
+    timing_mark(c, 3);
     size_t tb = c->scan_tmp_bytes;
     CUDA_TRY(c, launch_scan((const I64x2 *)c->mol_cnt.p, (I64x2 *)c->off.p, c->ND + 1, c->scan_tmp.p, &tb, c->stream));
     launches += 2;
@@ -811,14 +927,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     cp.nchunks = (int32_t *)c->nchunks.p;
     CUDA_TRY(c, launch_chunks(cp, c->stream));
     launches++;
-    timing_mark(c);
-  }
-  if (c->timing.enabled) {
-    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-    c->last.query_prep_ms = prog_timed ? timing_ms(c, 0, 1) : 0.f;
-    c->last.filter_ms = timing_ms(c, t0, t0 + 1);
-    c->last.support_ms = 0.f;
-    c->last.mapping_ms = timing_ms(c, t0 + 1, t0 + 2);
+    timing_mark(c, 4);
   }
   c->last.filter_launches = launches;
   c->levels = levels;
@@ -832,9 +941,7 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
   if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_join before sigmo_filter");
   if (mode != SIGMO_FIND_ALL && mode != SIGMO_FIND_FIRST) return set_err(c, SIGMO_ERR_INVALID_ARG, "bad mode %d", (int)mode);
   CUDA_TRY(c, cudaSetDevice(c->device));
-  c->timing.n = 0;
-  timing_mark(c);
-  CUDA_TRY(c, cudaMemsetAsync(c->jcnt.p, 0, 8 * ((size_t)c->NQ + 2), c->stream));
+  CUDA_TRY(c, cudaMemsetAsync(c->jcnt.p, 0, 8 * ((size_t)c->NQ + 6), c->stream));
   int launches = 0;
   if (c->ND > 0 && c->VD > 0 && c->NQ > 0) {
     JoinParams jp{};
@@ -860,32 +967,30 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
     jp.qp_be = c->qp_be;
     jp.pair_query = (int32_t *)c->pair_query.p;
     jp.pair_result = (unsigned long long *)c->pair_result.p;
-    jp.totals = (unsigned long long *)c->jcnt.p + 2;
-    jp.maxq = std::max(c->maxq, 2);
-    jp.PCAP = c->PC + c->NQ;
-    jp.ACAP = c->AC + c->maxn;
-    jp.CMCAP = c->CMC + c->VQ;
-    jp.MCAP = c->MC;
+    jp.totals = (unsigned long long *)c->jcnt.p + 6;
+    jp.error = (int *)((unsigned long long *)c->jcnt.p + 1);
+    jp.stats = (unsigned long long *)c->jcnt.p + 2;
+    fill_join_caps(c, jp);
     const size_t smem = join_smem_bytes(c->NW, jp);
     if (smem > c->max_smem) return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
     jp.smem_bytes = smem;
-    const int bps = join_blocks_per_sm(c->NW, (int)mode, smem);
+    const int bps = join_blocks_per_sm(c->NW, (int)mode, jp, smem);
     const int grid = bps * c->sm_count;
+    SIGMO_TRY(dreserve(c, c->gstack, join_gstack_bytes(c->NW, jp, grid), "join stack"));
+    jp.gstack = (unsigned char *)c->gstack.p;
+    timing_join(c, 0);
     CUDA_TRY(c, launch_join(c->NW, (int)mode, jp, grid, c->stream));
     launches++;
-  }
-  timing_mark(c);
-  if (c->timing.enabled) {
-    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-    c->last.join_ms = timing_ms(c, 0, 1);
+    timing_join(c, 1);
   }
   c->last.join_launches = launches;
   c->last_mode = (int)mode;
   c->state = 3;
   if (total_matches_out) {
+    SIGMO_TRY(read_join_flags(c));
     std::vector<uint64_t> t((size_t)c->NQ + 1);
     if (c->NQ > 0)
-      CUDA_TRY(c, cudaMemcpyAsync(t.data(), (uint64_t *)c->jcnt.p + 2, 8 * (size_t)c->NQ, cudaMemcpyDeviceToHost,
+      CUDA_TRY(c, cudaMemcpyAsync(t.data(), (uint64_t *)c->jcnt.p + 6, 8 * (size_t)c->NQ, cudaMemcpyDeviceToHost,
                                   c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
     uint64_t s = 0;
@@ -913,6 +1018,7 @@ sigmo_status sigmo_get_pair_results(sigmo_ctx *c, int64_t cap, int64_t *n, int64
                                     uint64_t *result) {
   if (!c || !n) return SIGMO_ERR_INVALID_ARG;
   if (c->state < 3) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_pair_results before sigmo_join");
+  SIGMO_TRY(read_join_flags(c));
   int64_t P = 0;
   SIGMO_TRY(sigmo_num_pairs(c, &P));
   *n = P;
@@ -953,10 +1059,11 @@ sigmo_status sigmo_get_query_totals(sigmo_ctx *c, uint64_t *out, int device_ptr)
   if (!c || !out) return SIGMO_ERR_INVALID_ARG;
   if (c->state < 3) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_query_totals before sigmo_join");
   if (c->NQ == 0) return SIGMO_OK;
+  if (!device_ptr) SIGMO_TRY(read_join_flags(c));
   if (device_ptr) {
-    CUDA_TRY(c, cudaMemcpyAsync(out, (uint64_t *)c->jcnt.p + 2, 8 * (size_t)c->NQ, cudaMemcpyDeviceToDevice, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(out, (uint64_t *)c->jcnt.p + 6, 8 * (size_t)c->NQ, cudaMemcpyDeviceToDevice, c->stream));
   } else {
-    CUDA_TRY(c, cudaMemcpyAsync(out, (uint64_t *)c->jcnt.p + 2, 8 * (size_t)c->NQ, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(out, (uint64_t *)c->jcnt.p + 6, 8 * (size_t)c->NQ, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
   }
   return SIGMO_OK;

@@ -10,7 +10,7 @@ namespace sigmo {
 constexpr int kNumFields = 13;   // R7 field table (see sigmo_kernels.cu kFieldWidth)
 constexpr int kMaxRadius = 15;   // levels <= 16
 constexpr int kFilterThreads = 256;
-constexpr int kJoinThreads = 256;
+constexpr int kJoinThreads = 128;
 constexpr int kQueryPrepThreads = 1024;
 
 struct I64x2 {
@@ -75,6 +75,7 @@ struct FilterParams {
   uint32_t *gm;                // [ND][NQW] surviving-query bits per data graph
   I64x2 *mol_cnt;              // [ND+1] (surviving pairs, candidate-mask entries)
   int EXTN, EXTW, MOLCAP;
+  int RE, rows_smem;           // row-program entries; 1 = copy row programs to smem
   size_t smem_bytes;
 };
 
@@ -98,6 +99,12 @@ struct JoinParams {
   unsigned long long *pair_result;
   unsigned long long *totals;  // [NQ]
   int PCAP, ACAP, CMCAP, MCAP, maxq;
+  int NBE, plan_smem;          // back-edge entries; 1 = copy the query plans to smem
+  int SCS;                     // per-warp DFS stack entries kept in shared memory
+  int slice_rows, SW;          // bitmap slice copy: rows (0 = read windows from global), words per row
+  unsigned char *gstack;       // per-warp global DFS stack area (promotion target)
+  int *error;                  // device flag, nonzero = internal capacity exceeded
+  unsigned long long *stats;   // optional: DFS iterator steps (nullable)
   size_t smem_bytes;
 };
 
@@ -116,11 +123,13 @@ cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *
 cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts, QueryProg &prog,
                               cudaStream_t st);
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
-size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P);
+size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int G, int VQ, int RE,
+                         int rows_smem);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);
 cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);
 size_t join_smem_bytes(int NW, const JoinParams &p);
-int join_blocks_per_sm(int NW, int mode, size_t smem);
+size_t join_gstack_bytes(int NW, const JoinParams &p, int grid);
+int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem);
 
 }  // namespace sigmo

@@ -420,34 +420,48 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
 // k_filter: one CTA per tile of TW (<= 32) bitmap words = 32*TW data nodes.
 // ===========================================================================
 struct FilterSmem {
-  size_t adj, ballA, ballB, fm, planes, win, molstart, molslot, fid, lab, mstart, sos, total;
+  size_t adj, ballA, ballB, fm, planes, win, nz, molstart, molslot, fid, lab, mstart, sos, rowlab, rowoff, rowids,
+      prog, total;
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
 
+// prog block: p_t[P] u8 | grp_f[G] u8 | fslot[16] i8 | grp_poff[G+1] i16 | rg_off[16] i16
+__host__ __device__ inline size_t prog_bytes(int P, int G) {
+  return align16((size_t)P) + align16((size_t)G) + 16 + align16(2 * (size_t)(G + 1)) + 32;
+}
+
 __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB,
-                                                    int P) {
+                                                    int P, int G, int VQ, int RE, int rows_smem) {
   FilterSmem L;
   const size_t mb = 8 * (size_t)NW;
+  const int NWARP = kFilterThreads / 32;
+  const int VQW = (VQ + 31) / 32;
   size_t o = 0;
   L.adj = o;      o = align16(o + mb * EXTN);
   L.ballA = o;    o = align16(o + mb * EXTN);
   L.ballB = o;    o = align16(o + mb * EXTN);
   L.fm = o;       o = align16(o + mb * (size_t)MOLCAP * (NFU > 0 ? NFU : 1));
   L.planes = o;   o = align16(o + 4 * (size_t)(NLAB + P) * EXTW);
-  L.win = o;      o = align16(o + mb * (size_t)(kFilterThreads / 32) * (NLAB + P));
+  L.win = o;      o = align16(o + mb * (size_t)NWARP * (NLAB + P));
+  L.nz = o;       o = align16(o + 4 * (size_t)NWARP * (VQW + 1));
   L.molstart = o; o = align16(o + 2 * (size_t)EXTN);
   L.molslot = o;  o = align16(o + 2 * (size_t)EXTN);
   L.fid = o;      o = align16(o + (size_t)EXTN);
   L.lab = o;      o = align16(o + (size_t)EXTN);
   L.mstart = o;   o = align16(o + 4 * (size_t)(MOLCAP + 1));
   L.sos = o;      o = align16(o + 2 * (size_t)EXTN);
+  L.rowlab = o;   o = align16(o + (rows_smem ? (size_t)VQ : 0));
+  L.rowoff = o;   o = align16(o + (rows_smem ? 4 * (size_t)(VQ + 1) : 0));
+  L.rowids = o;   o = align16(o + (rows_smem ? 2 * (size_t)RE : 0));
+  L.prog = o;     o = align16(o + prog_bytes(P, G));
   L.total = o;
   return L;
 }
 
-size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P) {
-  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P).total;
+size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int G, int VQ, int RE,
+                         int rows_smem) {
+  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, G, VQ, RE, rows_smem).total;
 }
 
 template <int NW>
@@ -455,19 +469,31 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   using M = Mask<NW>;
   constexpr int NT = kFilterThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
-  const FilterSmem L = filter_layout(NW, fp.EXTN, fp.EXTW, fp.MOLCAP, fp.NFU, fp.NLAB, fp.P);
+  const FilterSmem L = filter_layout(NW, fp.EXTN, fp.EXTW, fp.MOLCAP, fp.NFU, fp.NLAB, fp.P, fp.G, fp.VQ, fp.RE,
+                                     fp.rows_smem);
   M *s_adj = (M *)(smem + L.adj);
   M *s_cur = (M *)(smem + L.ballA);
   M *s_nxt = (M *)(smem + L.ballB);
   M *s_fm = (M *)(smem + L.fm);
   uint32_t *s_planes = (uint32_t *)(smem + L.planes);
   M *s_win = (M *)(smem + L.win);
+  uint32_t *s_nz = (uint32_t *)(smem + L.nz);
   int16_t *s_molstart = (int16_t *)(smem + L.molstart);
   int16_t *s_molslot = (int16_t *)(smem + L.molslot);
   uint8_t *s_fid = smem + L.fid;
   uint8_t *s_lab = smem + L.lab;
   int *s_mstart = (int *)(smem + L.mstart);
   int16_t *s_sos = (int16_t *)(smem + L.sos);
+  // plane program (always in smem)
+  uint8_t *s_pt = smem + L.prog;
+  uint8_t *s_grpf = s_pt + align16(fp.P);
+  int8_t *s_fslot = (int8_t *)(s_grpf + align16(fp.G));
+  int16_t *s_grpoff = (int16_t *)(s_fslot + 16);
+  int16_t *s_rg = (int16_t *)((unsigned char *)s_grpoff + align16(2 * (size_t)(fp.G + 1)));
+  // row programs: shared-memory copy when it fits, else global
+  const uint8_t *rowlab = fp.row_lab;
+  const int32_t *rowoff = fp.row_off;
+  const uint16_t *rowids = fp.row_ids;
   __shared__ int s_g0, s_g1;
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -480,6 +506,22 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   if (tid == 0) {
     s_g0 = graph_of(goff, ND, n0);
     s_g1 = graph_of(goff, ND, n1 - 1) + 1;
+  }
+  for (int i = tid; i < fp.P; i += NT) s_pt[i] = fp.p_t[i];
+  for (int i = tid; i < fp.G; i += NT) s_grpf[i] = fp.grp_f[i];
+  for (int i = tid; i <= fp.G; i += NT) s_grpoff[i] = fp.grp_poff[i];
+  for (int i = tid; i <= fp.R; i += NT) s_rg[i] = fp.rg_off[i];
+  for (int i = tid; i < kNumFields; i += NT) s_fslot[i] = fp.fslot[i];
+  if (fp.rows_smem) {
+    uint8_t *a = smem + L.rowlab;
+    int32_t *b = (int32_t *)(smem + L.rowoff);
+    uint16_t *c = (uint16_t *)(smem + L.rowids);
+    for (int i = tid; i < fp.VQ; i += NT) a[i] = fp.row_lab[i];
+    for (int i = tid; i <= fp.VQ; i += NT) b[i] = fp.row_off[i];
+    for (int i = tid; i < fp.RE; i += NT) c[i] = fp.row_ids[i];
+    rowlab = a;
+    rowoff = b;
+    rowids = c;
   }
   __syncthreads();
   const int g0 = s_g0, g1 = s_g1, nmol = g1 - g0;
@@ -494,15 +536,15 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   for (int i = tid; i <= nmol; i += NT) s_mstart[i] = __ldg(&goff[g0 + i]) - gs;
   for (int i = tid; i < next; i += NT) {
     const int v = gs + i;
-    const int loc = fp.D.local[v];
+    const int loc = __ldg(&fp.D.local[v]);
     M a;
     a.clear();
-    const int e1 = fp.D.roff[v + 1];
-    for (int e = fp.D.roff[v]; e < e1; e++) a.set(fp.D.nbr[e] >> 8);
+    const int e1 = __ldg(&fp.D.roff[v + 1]);
+    for (int e = __ldg(&fp.D.roff[v]); e < e1; e++) a.set(__ldg(&fp.D.nbr[e]) >> 8);
     s_adj[i] = a;
     s_cur[i] = M::bit(loc);
     s_molstart[i] = (int16_t)(i - loc);
-    const int lab = fp.D.label[v];
+    const int lab = __ldg(&fp.D.label[v]);
     s_lab[i] = (uint8_t)lab;
     s_fid[i] = (uint8_t)field_of(lab);
   }
@@ -515,7 +557,7 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     const int ms = s_molstart[i];
     const int slot = s_sos[ms];
     s_molslot[i] = (int16_t)slot;
-    const int fs = NFU > 0 ? fp.fslot[s_fid[i]] : -1;
+    const int fs = NFU > 0 ? s_fslot[s_fid[i]] : -1;
     if (fs >= 0) {
       const int loc = i - ms;
       atomicOr(&s_fm[slot * NFU + fs].w[loc >> 6], 1ull << (loc & 63));
@@ -526,14 +568,17 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     const int i = (xb + k) * 32 + lane - gs;
     const bool valid = (i >= 0) && (i < next);
     const int lab = valid ? s_lab[i] : -1;
+    uint32_t mine = 0;
     for (int c = 0; c < NLAB; c++) {
-      const unsigned b = __ballot_sync(FULL_MASK, lab == (int)fp.lab_val[c]);
-      if (lane == 0) s_planes[c * EXTW + k] = b;
+      const unsigned b = __ballot_sync(FULL_MASK, lab == (int)__ldg(&fp.lab_val[c]));
+      if ((c & 31) == lane) mine = b;
+      if ((c & 31) == 31 || c == NLAB - 1)
+        if (lane <= (c & 31)) s_planes[((c & ~31) + lane) * EXTW + k] = mine;
     }
   }
   __syncthreads();
 
-  // ---- radii 1..R: bitset BFS + threshold planes ----
+  // ---- radii 1..R: bitset BFS + threshold planes (RefineCandidates, l.19-28) ----
   for (int r = 1; r <= fp.R; r++) {
     for (int i = tid; i < next; i += NT) {
       M x = s_cur[i];
@@ -546,8 +591,9 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     M *t = s_cur;
     s_cur = s_nxt;
     s_nxt = t;
-    const int gb = fp.rg_off[r - 1], gend = fp.rg_off[r];
+    const int gb = s_rg[r - 1], gend = s_rg[r];
     if (gb < gend) {
+      const int pb = s_grpoff[gb], pe_r = s_grpoff[gend];
       for (int k = wid; k < nxw; k += NWARP) {
         const int i = (xb + k) * 32 + lane - gs;
         const bool valid = (i >= 0) && (i < next);
@@ -559,14 +605,18 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
           slot = s_molslot[i];
           fid = s_fid[i];
         }
+        uint32_t mine = 0;
         for (int grp = gb; grp < gend; grp++) {
-          const int f = fp.grp_f[grp];
+          const int f = s_grpf[grp];
           int cnt = 0;
-          if (valid) cnt = (ball & s_fm[slot * NFU + fp.fslot[f]]).popc() - (fid == f ? 1 : 0);
-          const int pe = fp.grp_poff[grp + 1];
-          for (int p = fp.grp_poff[grp]; p < pe; p++) {
-            const unsigned b = __ballot_sync(FULL_MASK, cnt >= (int)fp.p_t[p]);
-            if (lane == 0) s_planes[(NLAB + p) * EXTW + k] = b;
+          if (valid) cnt = (ball & s_fm[slot * NFU + s_fslot[f]]).popc() - (fid == f ? 1 : 0);
+          const int pe = s_grpoff[grp + 1];
+          for (int p = s_grpoff[grp]; p < pe; p++) {
+            const unsigned b = __ballot_sync(FULL_MASK, cnt >= (int)s_pt[p]);
+            const int j = p - pb;
+            if ((j & 31) == lane) mine = b;
+            if ((j & 31) == 31 || p == pe_r - 1)
+              if (lane <= (j & 31)) s_planes[(NLAB + pb + (j & ~31) + lane) * EXTW + k] = mine;
           }
         }
       }
@@ -580,18 +630,22 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     const bool active = (lane < fp.TW) && (w < fp.W);
     const int k = w - xb;
     for (int row = wid; row < fp.VQ; row += NWARP) {
-      const int rl = fp.row_lab[row];
-      const int j0 = fp.row_off[row], j1 = fp.row_off[row + 1];
+      const int rl = rowlab[row];
+      const int j0 = rowoff[row], j1 = rowoff[row + 1];
       if (active) {
         uint32_t x = s_planes[rl * EXTW + k];
-        for (int j = j0; j < j1; j++) x &= s_planes[(NLAB + fp.row_ids[j]) * EXTW + k];
+        for (int j = j0; j < j1; j++) x &= s_planes[(NLAB + rowids[j]) * EXTW + k];
         fp.bitmap[(size_t)row * fp.Wpad + w] = x;
       }
     }
   }
 
   // ---- GMCR test for molecules starting in this tile ----
+  // per molecule: windows of every plane, one non-empty bit per query node
+  // (lane = query node), then every query whose nodes are all non-empty.
   M *win = s_win + (size_t)wid * (NLAB + P);
+  const int VQW = (fp.VQ + 31) >> 5;
+  uint32_t *nz = s_nz + (size_t)wid * (VQW + 1);
   for (int mi = wid; mi < nmol; mi += NWARP) {
     const int g = g0 + mi;
     const int gst = __ldg(&goff[g]);
@@ -601,20 +655,33 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     const long long s = (long long)(gs + ms) - (long long)xb * 32;
     for (int c = lane; c < NLAB + P; c += 32) win[c] = extract_window<NW>(s_planes + (size_t)c * EXTW, nxw, s, n);
     __syncwarp();
+    for (int rb = 0; rb < VQW; rb++) {
+      const int row = rb * 32 + lane;
+      bool ok = false;
+      if (row < fp.VQ) {
+        M x = win[rowlab[row]];
+        const int j1 = rowoff[row + 1];
+        for (int j = rowoff[row]; j < j1; j++) x &= win[NLAB + rowids[j]];
+        ok = x.any();
+      }
+      const unsigned bits = __ballot_sync(FULL_MASK, ok);
+      if (lane == 0) nz[rb] = bits;
+    }
+    if (lane == 0) nz[VQW] = 0u;
+    __syncwarp();
     long long np = 0, ncm = 0;
     for (int qb = 0; qb < fp.NQW; qb++) {
       const int q = qb * 32 + lane;
-      bool ok = q < fp.NQ;
+      bool ok = false;
       int nq = 0;
-      if (ok) {
-        const int r0 = fp.qgoff[q], r1 = fp.qgoff[q + 1];
+      if (q < fp.NQ) {
+        const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
         nq = r1 - r0;
-        for (int row = r0; row < r1 && ok; row++) {
-          M x = win[fp.row_lab[row]];
-          const int j1 = fp.row_off[row + 1];
-          for (int j = fp.row_off[row]; j < j1; j++) x &= win[NLAB + fp.row_ids[j]];
-          ok = x.any();
-        }
+        const int wi = r0 >> 5, sh = r0 & 31;
+        uint32_t v = nz[wi] >> sh;
+        if (sh) v |= nz[wi + 1] << (32 - sh);
+        const uint32_t want = nq >= 32 ? 0xffffffffu : ((1u << nq) - 1u);
+        ok = (v & want) == want;
       }
       const unsigned bits = __ballot_sync(FULL_MASK, ok);
       if (lane == 0) fp.gm[(size_t)g * fp.NQW + qb] = bits;
@@ -708,65 +775,156 @@ cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st) {
 //   cand(e) = cm[e] & ~used & AND_{(j,b) in back(e)} adj_b[f(j)]
 // and the last depth is counted with popc instead of being enumerated.
 // ===========================================================================
+// ---------------------------------------------------------------------------
+// k_join shared-memory layout.  CTA-wide: the query plans (optional copy) and
+// the per-query totals; then one private region per warp (warps work on their
+// own molecule chunks and never wait for each other).
+// ---------------------------------------------------------------------------
+struct JoinWarpSmem {
+  size_t adj, cm, pinfo, cnt, found, mstart, scratch, total;  // scratch = bitmap slice (staging) | DFS stack
+};
 struct JoinSmem {
-  size_t adj, cm, cand, cnt, tot, pq, pcm, pitem, pmol, mstart, map, found, total;
+  size_t plan, tot, warps;
+  JoinWarpSmem w;
+  size_t total;
 };
 
-__host__ __device__ inline JoinSmem join_layout(int NW, int NB, int ACAP, int CMCAP, int PCAP, int MCAP, int NQ,
-                                                int maxq) {
+// plan block: qgoff[NQ+1] | qp_beoff[VQ+1] i32 | qp_row[VQ] i32 | qp_be[NBE] u16
+__host__ __device__ inline size_t join_plan_bytes(int NQ, int VQ, int NBE) {
+  return align16(4 * (size_t)(NQ + 1)) + align16(4 * (size_t)(VQ + 1)) + align16(4 * (size_t)VQ) +
+         align16(2 * (size_t)NBE);
+}
+
+// DFS iterator stack: safe capacity (global promotion) and shared-memory capacity
+__host__ __device__ inline int join_stack_cap(int maxq) { return 32 * (maxq + 1) + 64; }
+__host__ __device__ inline size_t join_entry_bytes(int NW, int MQ) { return 4 + 8 * (size_t)MQ + 16 * (size_t)NW; }
+// bytes of a stack of `cap` entries laid out as hdr[cap] | map[cap][MQ] | used[cap] | R[cap]
+__host__ __device__ inline size_t join_stack_bytes(int NW, int MQ, int cap) {
+  return align16(4 * (size_t)cap) + align16(8 * (size_t)MQ * cap) + 16 * (size_t)NW * cap;
+}
+
+__host__ __device__ inline JoinSmem join_layout(const JoinParams &p, int NW, int MQ) {
   JoinSmem L;
   const size_t mb = 8 * (size_t)NW;
-  const int NT = kJoinThreads;
+  const int NWARP = kJoinThreads / 32;
   size_t o = 0;
-  L.adj = o;    o = align16(o + mb * (size_t)NB * ACAP);
-  L.cm = o;     o = align16(o + mb * (size_t)CMCAP);
-  L.cand = o;   o = align16(o + mb * (size_t)maxq * NT);
-  L.cnt = o;    o = align16(o + 8 * (size_t)PCAP);
-  L.tot = o;    o = align16(o + 8 * (size_t)NQ);
-  L.pq = o;     o = align16(o + 4 * (size_t)PCAP);
-  L.pcm = o;    o = align16(o + 4 * (size_t)PCAP);
-  L.pitem = o;  o = align16(o + 4 * (size_t)(PCAP + 1));
-  L.pmol = o;   o = align16(o + 2 * (size_t)PCAP);
-  L.mstart = o; o = align16(o + 4 * (size_t)(MCAP + 1));
-  L.map = o;    o = align16(o + (size_t)maxq * NT);
-  L.found = o;  o = align16(o + (size_t)PCAP);
+  L.plan = o;  o = align16(o + (p.plan_smem ? join_plan_bytes(p.NQ, p.VQ, p.NBE) : 0));
+  L.tot = o;   o = align16(o + 8 * (size_t)p.NQ);
+  L.warps = o;
+  size_t w = 0;
+  L.w.adj = w;     w = align16(w + mb * (size_t)p.NB * p.ACAP);
+  L.w.cm = w;      w = align16(w + mb * (size_t)p.CMCAP);
+  L.w.pinfo = w;   w = align16(w + 16 * (size_t)p.PCAP);
+  L.w.cnt = w;     w = align16(w + 8 * (size_t)p.PCAP);
+  L.w.found = w;   w = align16(w + (size_t)p.PCAP);
+  L.w.mstart = w;  w = align16(w + 4 * (size_t)(p.MCAP + 1));
+  L.w.scratch = w;
+  const size_t slice = p.slice_rows ? 4 * (size_t)p.slice_rows * p.SW : 0;
+  const size_t stack = join_stack_bytes(NW, MQ, p.SCS);
+  w = align16(w + (slice > stack ? slice : stack));
+  L.w.total = w;
+  o += w * NWARP;
   L.total = o;
   return L;
 }
 
-size_t join_smem_bytes(int NW, const JoinParams &p) {
-  return join_layout(NW, p.NB, p.ACAP, p.CMCAP, p.PCAP, p.MCAP, p.NQ, p.maxq).total;
+static inline int join_mq(int maxq) { return maxq <= 8 ? 1 : (maxq <= 16 ? 2 : 4); }
+
+size_t join_smem_bytes(int NW, const JoinParams &p) { return join_layout(p, NW, join_mq(p.maxq)).total; }
+size_t join_gstack_bytes(int NW, const JoinParams &p, int grid) {
+  return join_stack_bytes(NW, join_mq(p.maxq), join_stack_cap(p.maxq)) * (size_t)grid * (kJoinThreads / 32) + 256;
 }
 
-template <int NW, int MODE>
+// byte j of a packed mapping (MQ u64 words)
+template <int MQ>
+__device__ __forceinline__ int map_get(const unsigned long long (&m)[MQ], int j) {
+  unsigned long long w = m[0];
+#pragma unroll
+  for (int k = 1; k < MQ; k++)
+    if ((j >> 3) == k) w = m[k];
+  return (int)((w >> ((j & 7) * 8)) & 0xffull);
+}
+template <int MQ>
+__device__ __forceinline__ void map_set(unsigned long long (&m)[MQ], int j, int v) {
+#pragma unroll
+  for (int k = 0; k < MQ; k++)
+    if ((j >> 3) == k) m[k] = (m[k] & ~(0xffull << ((j & 7) * 8))) | ((unsigned long long)v << ((j & 7) * 8));
+}
+
+// ===========================================================================
+// k_join: every warp independently pulls molecule chunks (persistent, atomic
+// chunk counter).  Per chunk the warp stages, in its private smem region:
+// the bond-class adjacency masks of the chunk's molecules, its GMCR pairs and,
+// per pair, the candidate mask of every query node restricted to the molecule
+// (cut from a coalesced copy of the chunk's bitmap slice).  The DFS
+// runs on the warp's stack of iterators
+//   E = (pair, d, f(pi_0..pi_{d-1}), used, R)
+// where R holds the not-yet-tried candidates of plan depth d.  Each step every
+// lane pops one iterator, takes v = lowest(R), pushes the remainder and, for
+// the extended mapping, the child iterator with
+//   R' = cm[d+1] & ~used' & AND_{(j,b) in back(d+1)} adj_b[f(j)]
+// (children above remainders: depth-first).  At the last depth embeddings are
+// counted with popc instead of being pushed.  The warp keeps >= 32 iterators
+// by seeding new pairs, so all lanes run the same instruction stream.
+// ===========================================================================
+template <int NW, int MQ, int MODE>
 __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
   using M = Mask<NW>;
   constexpr int NT = kJoinThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
-  const JoinSmem L = join_layout(NW, jp.NB, jp.ACAP, jp.CMCAP, jp.PCAP, jp.MCAP, jp.NQ, jp.maxq);
-  M *s_adj = (M *)(smem + L.adj);
-  M *s_cm = (M *)(smem + L.cm);
-  M *s_cand = (M *)(smem + L.cand);
-  unsigned long long *s_cnt = (unsigned long long *)(smem + L.cnt);
-  unsigned long long *s_tot = (unsigned long long *)(smem + L.tot);
-  int *s_pq = (int *)(smem + L.pq);
-  int *s_pcm = (int *)(smem + L.pcm);
-  int *s_pitem = (int *)(smem + L.pitem);
-  int16_t *s_pmol = (int16_t *)(smem + L.pmol);
-  int *s_mstart = (int *)(smem + L.mstart);
-  uint8_t *s_map = smem + L.map;
-  uint8_t *s_found = smem + L.found;
-  __shared__ int s_chunk, s_next, s_warp[32];
-
+  const JoinSmem L = join_layout(jp, NW, MQ);
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  unsigned long long *s_tot = (unsigned long long *)(smem + L.tot);
+  unsigned char *wb = smem + L.warps + (size_t)wid * L.w.total;
+  M *s_adj = (M *)(wb + L.w.adj);
+  M *s_cm = (M *)(wb + L.w.cm);
+  int4 *s_pinfo = (int4 *)(wb + L.w.pinfo);  // {cm offset, plan base qb, mbase | n << 16, q << 8 | nq}
+  unsigned long long *s_cnt = (unsigned long long *)(wb + L.w.cnt);
+  uint8_t *s_found = wb + L.w.found;
+  int *s_mstart = (int *)(wb + L.w.mstart);
+  uint32_t *s_slice = (uint32_t *)(wb + L.w.scratch);
+  // DFS stack (shared memory; promoted to a global area if it ever fills)
+  const int SCS = jp.SCS;
+  uint32_t *const sm_hdr = (uint32_t *)(wb + L.w.scratch);
+  unsigned long long *const sm_map = (unsigned long long *)(wb + L.w.scratch + align16(4 * (size_t)SCS));
+  M *const sm_used = (M *)((unsigned char *)sm_map + align16(8 * (size_t)MQ * SCS));
+  M *const sm_R = sm_used + SCS;
+  const int SCG = join_stack_cap(jp.maxq);
+  const size_t gwarp = (size_t)blockIdx.x * NWARP + wid;
+  unsigned char *gb = jp.gstack + gwarp * join_stack_bytes(NW, MQ, SCG);
+  uint32_t *const gm_hdr = (uint32_t *)gb;
+  unsigned long long *const gm_map = (unsigned long long *)(gb + align16(4 * (size_t)SCG));
+  M *const gm_used = (M *)((unsigned char *)gm_map + align16(8 * (size_t)MQ * SCG));
+  M *const gm_R = gm_used + SCG;
+
   const int ACAP = jp.ACAP;
+  const int32_t *qgoff = jp.qgoff, *qp_beoff = jp.qp_beoff, *qp_row = jp.qp_row;
+  const uint16_t *qp_be = jp.qp_be;
+  if (jp.plan_smem) {
+    unsigned char *b = smem + L.plan;
+    int32_t *a0 = (int32_t *)b;
+    int32_t *a1 = (int32_t *)(b + align16(4 * (size_t)(jp.NQ + 1)));
+    int32_t *a2 = (int32_t *)((unsigned char *)a1 + align16(4 * (size_t)(jp.VQ + 1)));
+    uint16_t *a3 = (uint16_t *)((unsigned char *)a2 + align16(4 * (size_t)jp.VQ));
+    for (int i = tid; i <= jp.NQ; i += NT) a0[i] = jp.qgoff[i];
+    for (int i = tid; i <= jp.VQ; i += NT) a1[i] = jp.qp_beoff[i];
+    for (int i = tid; i < jp.VQ; i += NT) a2[i] = jp.qp_row[i];
+    for (int i = tid; i < jp.NBE; i += NT) a3[i] = jp.qp_be[i];
+    qgoff = a0;
+    qp_beoff = a1;
+    qp_row = a2;
+    qp_be = a3;
+  }
   for (int i = tid; i < jp.NQ; i += NT) s_tot[i] = 0ull;
+  __syncthreads();
+  long long nodes = 0, iters = 0, tail_iters = 0;
+  int max_top = 0;
+  const unsigned lt = (1u << lane) - 1u;
 
   while (true) {
-    __syncthreads();
-    if (tid == 0) s_chunk = atomicAdd(jp.chunk_counter, 1);
-    __syncthreads();
-    const int c = s_chunk;
+    int c = 0;
+    if (lane == 0) c = atomicAdd(jp.chunk_counter, 1);
+    c = __shfl_sync(FULL_MASK, c, 0);
     if (c >= *jp.nchunks) break;
     const int g0 = jp.chunk_start[c], g1 = jp.chunk_start[c + 1];
     if (g0 >= g1) continue;
@@ -778,255 +936,301 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
     const int na = jp.goff[g1] - a0;
     const int nm = g1 - g0;
 
-    // ---- stage: molecule starts, bond-class adjacency masks ----
-    for (int i = tid; i <= nm; i += NT) s_mstart[i] = jp.goff[g0 + i] - a0;
-    for (int i = tid; i < na; i += NT) {
+    // ---- stage: molecule starts and bond-class adjacency masks ----
+    for (int i = lane; i <= nm; i += 32) s_mstart[i] = __ldg(&jp.goff[g0 + i]) - a0;
+    for (int i = lane; i < na; i += 32) {
       const int v = a0 + i;
-      const int e0 = jp.roff[v], e1 = jp.roff[v + 1];
-      for (int b = 0; b < jp.NB; b++) {
-        M m;
-        m.clear();
-        for (int e = e0; e < e1; e++) {
-          const int x = jp.nbr[e];
-          if (jp.bclass[x & 255] == b) m.set(x >> 8);
-        }
-        s_adj[b * ACAP + i] = m;
-      }
-    }
-    // ---- stage: GMCR pairs of the chunk (warp per molecule) ----
-    for (int mi = wid; mi < nm; mi += NWARP) {
-      const int g = g0 + mi;
-      const I64x2 og = jp.off[g];
-      int run_p = (int)(og.a - p0), run_c = (int)(og.b - c0);
-      for (int blk = 0; blk < jp.NQW; blk += 32) {
-        const int qw = blk + lane;
-        const uint32_t bits = (qw < jp.NQW) ? jp.gm[(size_t)g * jp.NQW + qw] : 0u;
-        int myp = __popc(bits), myc = 0;
-        for (uint32_t m = bits; m; m &= m - 1u) {
-          const int q = qw * 32 + __ffs(m) - 1;
-          myc += jp.qgoff[q + 1] - jp.qgoff[q];
-        }
-        int xp = myp, xc = myc;
+      const int e0 = __ldg(&jp.roff[v]), e1 = __ldg(&jp.roff[v + 1]);
+      M m[8];
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const int yp = __shfl_up_sync(FULL_MASK, xp, o), yc = __shfl_up_sync(FULL_MASK, xc, o);
-          if (lane >= o) {
-            xp += yp;
-            xc += yc;
-          }
-        }
-        int pos = run_p + xp - myp, cpos = run_c + xc - myc;
-        for (uint32_t m = bits; m; m &= m - 1u) {
-          const int q = qw * 32 + __ffs(m) - 1;
-          s_pq[pos] = q;
-          s_pmol[pos] = (int16_t)mi;
-          s_pcm[pos] = cpos;
-          pos++;
-          cpos += jp.qgoff[q + 1] - jp.qgoff[q];
-        }
-        run_p += __shfl_sync(FULL_MASK, xp, 31);
-        run_c += __shfl_sync(FULL_MASK, xc, 31);
+      for (int b = 0; b < 8; b++) m[b].clear();
+      for (int e = e0; e < e1; e++) {
+        const int x = __ldg(&jp.nbr[e]);
+        const int cls = jp.bclass[x & 255];
+#pragma unroll
+        for (int b = 0; b < 8; b++)
+          if (cls == b) m[b].set(x >> 8);
+      }
+#pragma unroll
+      for (int b = 0; b < 8; b++)
+        if (b < jp.NB) s_adj[b * ACAP + i] = m[b];
+    }
+    // ---- stage: coalesced copy of the chunk's bitmap slice (all rows) ----
+    const int ws = a0 >> 5;
+    const int nws = na > 0 ? ((a0 + na - 1) >> 5) - ws + 1 : 0;
+    if (jp.slice_rows) {
+      const int tot = jp.slice_rows * nws;
+      for (int t = lane; t < tot; t += 32) {
+        const int row = t / nws, w = t - row * nws;
+        s_slice[row * jp.SW + w] = __ldg(&jp.bitmap[(size_t)row * jp.Wpad + ws + w]);
       }
     }
-    __syncthreads();
-    // ---- stage: candidate masks of every pair (molecule window of each row) ----
-    for (int i = tid; i < np; i += NT) {
-      const int q = s_pq[i], mi = s_pmol[i];
-      const int ms = s_mstart[mi], n = s_mstart[mi + 1] - ms;
-      const long long gstart = (long long)a0 + ms;
-      const int qb = jp.qgoff[q], nq = jp.qgoff[q + 1] - qb;
-      const int cb = s_pcm[i];
+    __syncwarp();
+    // ---- stage: GMCR pairs (lane = query) ----
+    {
+      int run_p = 0, run_c = 0;
+      for (int mi = 0; mi < nm; mi++) {
+        const int g = g0 + mi;
+        const int mbase = s_mstart[mi], n = s_mstart[mi + 1] - mbase;
+        for (int qb = 0; qb < jp.NQW; qb++) {
+          const uint32_t bits = __ldg(&jp.gm[(size_t)g * jp.NQW + qb]);
+          const int q = qb * 32 + lane;
+          const bool ok = (bits >> lane) & 1u;
+          int nq = 0, qbase = 0;
+          if (ok) {
+            qbase = qgoff[q];
+            nq = qgoff[q + 1] - qbase;
+          }
+          int xc = nq;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(FULL_MASK, xc, o);
+            if (lane >= o) xc += y;
+          }
+          if (ok) {
+            const int pos = run_p + __popc(bits & lt);
+            s_pinfo[pos] = make_int4(run_c + xc - nq, qbase, mbase | (n << 16), (q << 8) | nq);
+            s_cnt[pos] = 0ull;
+            s_found[pos] = 0;
+          }
+          run_p += __popc(bits);
+          run_c += __shfl_sync(FULL_MASK, xc, 31);
+        }
+      }
+    }
+    __syncwarp();
+    // ---- stage: candidate masks cm[pair][e] (molecule window of each query-node row) ----
+    for (int i = lane; i < np; i += 32) {
+      const int4 pi = s_pinfo[i];
+      const int nq = pi.w & 0xff, mbase = pi.z & 0xffff, n = pi.z >> 16;
       for (int e = 0; e < nq; e++) {
-        const int row = jp.qp_row[qb + e];
-        s_cm[cb + e] = extract_window<NW>(jp.bitmap + (size_t)row * jp.Wpad, jp.Wpad, gstart, n);
+        const int row = qp_row[pi.y + e];
+        M w;
+        if (jp.slice_rows)
+          w = extract_window<NW>(s_slice + (size_t)row * jp.SW, nws, (long long)(a0 + mbase) - (long long)ws * 32, n);
+        else
+          w = extract_window<NW>(jp.bitmap + (size_t)row * jp.Wpad, jp.Wpad, (long long)a0 + mbase, n);
+        s_cm[pi.x + e] = w;
       }
-      s_pitem[i] = s_cm[cb].popc();
-      s_cnt[i] = 0ull;
-      s_found[i] = 0;
     }
-    __syncthreads();
-    const int nitems = block_exclusive_scan<NT>(s_pitem, np, s_warp);
-    if (tid == 0) s_next = 0;
-    __syncthreads();
+    __syncwarp();
 
-    // ---- DFS: lanes pull (pair, root) items ----
-    int p = -1;
-    bool exhausted = false;
-    int d = 0, nq = 0, qb = 0, cmoff = 0, mbase = 0;
-    M used, cset;
-    used.clear();
-    cset.clear();
-    unsigned long long cnt = 0ull;
-
-    auto compute = [&](int e, const M &u) -> M {
-      M x = s_cm[cmoff + e].andnot(u);
-      const int k1 = __ldg(&jp.qp_beoff[qb + e + 1]);
-      for (int k = __ldg(&jp.qp_beoff[qb + e]); k < k1; k++) {
-        const int be = __ldg(&jp.qp_be[k]);
-        const int v = s_map[(be >> 8) * NT + tid];
-        x &= s_adj[(be & 255) * ACAP + mbase + v];
-      }
-      return x;
-    };
-    auto finish = [&]() {
-      if (cnt) {
-        atomicAdd(&s_cnt[p], cnt);
-        if (MODE == 1) s_found[p] = 1;
-      }
-      p = -1;
-    };
-
+    // ---- DFS on the warp's iterator stack ----
+    uint32_t *st_hdr = sm_hdr;
+    unsigned long long *st_map = sm_map;
+    M *st_used = sm_used, *st_R = sm_R;
+    int cap = SCS;
+    int top = 0, next_pair = 0;
     while (true) {
-      const bool need = (p < 0) && !exhausted;
-      const unsigned nmask = __ballot_sync(FULL_MASK, need);
-      if (nmask) {
-        const int leader = __ffs(nmask) - 1;
-        int base = 0;
-        if (lane == leader) base = atomicAdd(&s_next, __popc(nmask));
-        base = __shfl_sync(FULL_MASK, base, leader);
-        if (need) {
-          const int it = base + __popc(nmask & ((1u << lane) - 1u));
-          if (it >= nitems) {
-            exhausted = true;
-          } else {
-            int lo = 0, hi = np - 1;
-            while (lo < hi) {
-              const int mid = (lo + hi + 1) >> 1;
-              if (s_pitem[mid] <= it) lo = mid;
-              else hi = mid - 1;
-            }
-            p = lo;
-            const int k = it - s_pitem[p];
-            const int q = s_pq[p];
-            qb = jp.qgoff[q];
-            nq = jp.qgoff[q + 1] - qb;
-            cmoff = s_pcm[p];
-            mbase = s_mstart[s_pmol[p]];
-            M r = s_cm[cmoff];
-            for (int j = 0; j < k; j++) r.clear_lowest();
-            const int v0 = r.lowest();
-            cnt = 0ull;
-            if (MODE == 1 && s_found[p]) {
-              p = -1;
-            } else if (nq == 1) {
-              cnt = 1ull;
-              finish();
-            } else {
-              s_map[tid] = (uint8_t)v0;
-              used = M::bit(v0);
-              const M x = compute(1, used);
-              if (nq == 2) {
-                cnt = (unsigned long long)x.popc();
-                finish();
-              } else {
-                d = 1;
-                cset = x;
-              }
-            }
-          }
+      if (top < 32 && next_pair < np) {
+        // seed iterators of new pairs: E = (pair, d = 0, R = root candidates)
+        const int pi = next_pair + lane;
+        const bool ok = lane < 32 - top && pi < np;
+        if (ok) {
+          const int idx = top + lane;
+          st_hdr[idx] = (uint32_t)pi;
+          st_R[idx] = s_cm[s_pinfo[pi].x];
+          M z;
+          z.clear();
+          st_used[idx] = z;
+#pragma unroll
+          for (int k = 0; k < MQ; k++) st_map[(size_t)idx * MQ + k] = 0ull;
         }
+        const int added = __popc(__ballot_sync(FULL_MASK, ok));
+        top += added;
+        next_pair += added;
+        __syncwarp();
       }
-      if (__ballot_sync(FULL_MASK, !exhausted) == 0u) break;
-      if (p >= 0) {
-        if (MODE == 1 && s_found[p]) {
-          p = -1;  // another lane found this pair's first embedding
-        } else if (!cset.any()) {
-          if (d == 1) {
-            finish();
-          } else {
-            d--;
-            used.reset(s_map[d * NT + tid]);
-            cset = s_cand[d * NT + tid];
-          }
+      if (top == 0) break;
+      const int take = min(32, top);
+      iters++;
+      if (next_pair >= np) tail_iters++;
+      max_top = max(max_top, top);
+      top -= take;
+      const bool act = lane < take;
+      const int idx = top + lane;
+      uint32_t hdr = 0;
+      M R, used;
+      R.clear();
+      used.clear();
+      unsigned long long mp[MQ];
+#pragma unroll
+      for (int k = 0; k < MQ; k++) mp[k] = 0ull;
+      if (act) {
+        hdr = st_hdr[idx];
+        R = st_R[idx];
+        used = st_used[idx];
+#pragma unroll
+        for (int k = 0; k < MQ; k++) mp[k] = st_map[(size_t)idx * MQ + k];
+      }
+      __syncwarp();
+      nodes += take;
+      const int pair = hdr & 0xffff;
+      const int d = hdr >> 16;
+      bool alive = act;
+      if (MODE == 1 && alive && s_found[pair]) alive = false;
+      int4 pinf = make_int4(0, 0, 0, 0);
+      if (alive) pinf = s_pinfo[pair];
+      const int nq = pinf.w & 0xff;
+      const int mbase = pinf.z & 0xffff;
+      const int v = alive ? R.lowest() : 0;
+      if (alive) R.clear_lowest();
+      const bool push_rem = alive && R.any();
+      unsigned long long mrem[MQ];
+#pragma unroll
+      for (int k = 0; k < MQ; k++) mrem[k] = mp[k];
+      map_set<MQ>(mp, d, v);
+      M u2 = used;
+      if (alive) u2.set(v);
+      const int e = d + 1;  // mapped nodes after this step
+      unsigned long long cnt = 0ull;
+      bool push_child = false;
+      M x;
+      x.clear();
+      if (alive) {
+        if (e == nq) {
+          cnt = 1ull;  // single-node query
         } else {
-          const int v = cset.lowest();
-          cset.clear_lowest();
-          s_map[d * NT + tid] = (uint8_t)v;
-          M u2 = used;
-          u2.set(v);
-          const M x = compute(d + 1, u2);
-          if (d + 1 == nq - 1) {
-            cnt += (unsigned long long)x.popc();
-            if (MODE == 1 && cnt) finish();
-          } else if (x.any()) {
-            s_cand[d * NT + tid] = cset;
-            used = u2;
-            d++;
-            cset = x;
+          x = s_cm[pinf.x + e].andnot(u2);
+          const int k1 = qp_beoff[pinf.y + e + 1];
+          for (int k = qp_beoff[pinf.y + e]; k < k1; k++) {
+            const int be = qp_be[k];
+            x &= s_adj[(be & 255) * ACAP + mbase + map_get<MQ>(mp, be >> 8)];
           }
+          if (e == nq - 1) cnt = (unsigned long long)x.popc();  // last depth: count
+          else push_child = x.any();
         }
       }
+      if (cnt) {
+        // 64-bit per-pair count kept as two 32-bit words with carry
+        uint32_t *w = (uint32_t *)&s_cnt[pair];
+        const uint32_t add = (uint32_t)cnt;  // <= 64
+        const uint32_t old = atomicAdd(w, add);
+        if (old + add < old) atomicAdd(w + 1, 1u);
+        if (MODE == 1) s_found[pair] = 1;
+      }
+      // push: remainders first, then children (children end on top)
+      const unsigned mr = __ballot_sync(FULL_MASK, push_rem);
+      const unsigned mc = __ballot_sync(FULL_MASK, push_child);
+      const int npush = __popc(mr) + __popc(mc);
+      if (top + npush > cap - 32) {
+        // promote the stack to the warp's global area (capacity join_stack_cap)
+        if (st_hdr == sm_hdr) {
+          for (int i = lane; i < top; i += 32) {
+            gm_hdr[i] = sm_hdr[i];
+            gm_used[i] = sm_used[i];
+            gm_R[i] = sm_R[i];
+#pragma unroll
+            for (int k = 0; k < MQ; k++) gm_map[(size_t)i * MQ + k] = sm_map[(size_t)i * MQ + k];
+          }
+          __syncwarp();
+          st_hdr = gm_hdr;
+          st_map = gm_map;
+          st_used = gm_used;
+          st_R = gm_R;
+          cap = SCG;
+        }
+        if (top + npush > cap) {
+          if (lane == 0) atomicOr(jp.error, 1);
+          top = 0;
+          next_pair = np;
+          continue;
+        }
+      }
+      if (push_rem) {
+        const int j = top + __popc(mr & lt);
+        st_hdr[j] = hdr;
+        st_R[j] = R;
+        st_used[j] = used;
+#pragma unroll
+        for (int k = 0; k < MQ; k++) st_map[(size_t)j * MQ + k] = mrem[k];
+      }
+      if (push_child) {
+        const int j = top + __popc(mr) + __popc(mc & lt);
+        st_hdr[j] = (uint32_t)pair | ((uint32_t)e << 16);
+        st_R[j] = x;
+        st_used[j] = u2;
+#pragma unroll
+        for (int k = 0; k < MQ; k++) st_map[(size_t)j * MQ + k] = mp[k];
+      }
+      top += npush;
+      __syncwarp();
     }
-    __syncthreads();
     // ---- results: GMCR pair list + per-pair result + per-query totals ----
-    for (int i = tid; i < np; i += NT) {
+    for (int i = lane; i < np; i += 32) {
       unsigned long long r = s_cnt[i];
       if (MODE == 1) r = r ? 1ull : 0ull;
-      const int q = s_pq[i];
+      const int q = s_pinfo[i].w >> 8;
       jp.pair_query[p0 + i] = q;
       jp.pair_result[p0 + i] = r;
       if (r) atomicAdd(&s_tot[q], r);
     }
+    (void)c0;
+    __syncwarp();
   }
   __syncthreads();
   for (int i = tid; i < jp.NQ; i += NT)
     if (s_tot[i]) atomicAdd(&jp.totals[i], s_tot[i]);
+  if (jp.stats && lane == 0) {
+    atomicAdd(jp.stats, (unsigned long long)nodes);
+    atomicAdd(jp.stats + 1, (unsigned long long)iters);
+    atomicAdd(jp.stats + 2, (unsigned long long)tail_iters);
+    atomicMax(jp.stats + 3, (unsigned long long)max_top);
+  }
 }
 
-template <int NW, int MODE>
+template <int NW, int MQ, int MODE>
 static cudaError_t launch_join_t(const JoinParams &p, int grid, cudaStream_t st) {
-  cudaError_t e = cudaFuncSetAttribute(k_join<NW, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaError_t e = cudaFuncSetAttribute(k_join<NW, MQ, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)p.smem_bytes);
   if (e != cudaSuccess) return e;
-  k_join<NW, MODE><<<grid, kJoinThreads, p.smem_bytes, st>>>(p);
+  k_join<NW, MQ, MODE><<<grid, kJoinThreads, p.smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st) {
-  if (grid <= 0) return cudaSuccess;
-  switch (NW * 2 + mode) {
-    case 2: return launch_join_t<1, 0>(p, grid, st);
-    case 3: return launch_join_t<1, 1>(p, grid, st);
-    case 4: return launch_join_t<2, 0>(p, grid, st);
-    case 5: return launch_join_t<2, 1>(p, grid, st);
-    case 8: return launch_join_t<4, 0>(p, grid, st);
-    case 9: return launch_join_t<4, 1>(p, grid, st);
-    default: return cudaErrorInvalidValue;
+template <int NW, int MQ, int MODE>
+static int occ_join_t(size_t smem) {
+  int n = 0;
+  cudaFuncSetAttribute(k_join<NW, MQ, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join<NW, MQ, MODE>, kJoinThreads, smem) != cudaSuccess) {
+    cudaGetLastError();
+    return 1;
   }
+  return n < 1 ? 1 : n;
 }
 
-int join_blocks_per_sm(int NW, int mode, size_t smem) {
-  int n = 0;
-  cudaError_t e = cudaSuccess;
-  switch (NW * 2 + mode) {
-    case 2:
-      cudaFuncSetAttribute(k_join<1, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join<1, 0>, kJoinThreads, smem);
-      break;
-    case 3:
-      cudaFuncSetAttribute(k_join<1, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join<1, 1>, kJoinThreads, smem);
-      break;
-    case 4:
-      cudaFuncSetAttribute(k_join<2, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join<2, 0>, kJoinThreads, smem);
-      break;
-    case 5:
-      cudaFuncSetAttribute(k_join<2, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join<2, 1>, kJoinThreads, smem);
-      break;
-    case 8:
-      cudaFuncSetAttribute(k_join<4, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join<4, 0>, kJoinThreads, smem);
-      break;
-    case 9:
-      cudaFuncSetAttribute(k_join<4, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join<4, 1>, kJoinThreads, smem);
-      break;
-    default: return 1;
+#define SIGMO_JOIN_DISPATCH(FN, ...)                                             \
+  switch ((NW == 1 ? 0 : NW == 2 ? 1 : 2) * 6 + (MQ == 1 ? 0 : MQ == 2 ? 1 : 2) * 2 + mode) { \
+    case 0: return FN<1, 1, 0>(__VA_ARGS__);                                     \
+    case 1: return FN<1, 1, 1>(__VA_ARGS__);                                     \
+    case 2: return FN<1, 2, 0>(__VA_ARGS__);                                     \
+    case 3: return FN<1, 2, 1>(__VA_ARGS__);                                     \
+    case 4: return FN<1, 4, 0>(__VA_ARGS__);                                     \
+    case 5: return FN<1, 4, 1>(__VA_ARGS__);                                     \
+    case 6: return FN<2, 1, 0>(__VA_ARGS__);                                     \
+    case 7: return FN<2, 1, 1>(__VA_ARGS__);                                     \
+    case 8: return FN<2, 2, 0>(__VA_ARGS__);                                     \
+    case 9: return FN<2, 2, 1>(__VA_ARGS__);                                     \
+    case 10: return FN<2, 4, 0>(__VA_ARGS__);                                    \
+    case 11: return FN<2, 4, 1>(__VA_ARGS__);                                    \
+    case 12: return FN<4, 1, 0>(__VA_ARGS__);                                    \
+    case 13: return FN<4, 1, 1>(__VA_ARGS__);                                    \
+    case 14: return FN<4, 2, 0>(__VA_ARGS__);                                    \
+    case 15: return FN<4, 2, 1>(__VA_ARGS__);                                    \
+    case 16: return FN<4, 4, 0>(__VA_ARGS__);                                    \
+    default: return FN<4, 4, 1>(__VA_ARGS__);                                    \
   }
-  if (e != cudaSuccess || n < 1) return 1;
-  return n;
+
+cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st) {
+  if (grid <= 0) return cudaSuccess;
+  if (NW != 1 && NW != 2 && NW != 4) return cudaErrorInvalidValue;
+  const int MQ = join_mq(p.maxq);
+  SIGMO_JOIN_DISPATCH(launch_join_t, p, grid, st)
+}
+
+int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem) {
+  const int MQ = join_mq(p.maxq);
+  SIGMO_JOIN_DISPATCH(occ_join_t, smem)
 }
 
 }  // namespace sigmo

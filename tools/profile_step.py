@@ -1,0 +1,25 @@
+"""Small driver for ncu: load configs[1] (or N molecules), run W warm-up
+steps then S profiled steps of filter + join.  Usage:
+    python tools/profile_step.py [molecules] [levels] [steps] [mode]"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+
+import synth
+import paper_conf_sc_carocfc25_b200 as sigmo
+
+n = int(sys.argv[1]) if len(sys.argv) > 1 else 100_000
+L = int(sys.argv[2]) if len(sys.argv) > 2 else 4
+S = int(sys.argv[3]) if len(sys.argv) > 3 else 2
+mode = int(sys.argv[4]) if len(sys.argv) > 4 else 0
+torch.cuda.set_device(0)
+Q, D = synth.config_queries(2), synth.config_data(2, count=n)
+ctx = sigmo.Context(0)
+ctx.load_batch(Q, D)
+for _ in range(2 + S):
+    ctx.filter(L)
+    ctx.join(mode, total=False)
+torch.cuda.synchronize()
+print("matches", ctx.join(mode))
