@@ -7,6 +7,7 @@
 #include <atomic>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -111,6 +112,7 @@ struct sigmo_ctx {
   int W = 0, Wpad = 0;
   int32_t *qp_row = nullptr, *qp_beoff = nullptr;
   uint16_t *qp_be = nullptr;
+  uint32_t *qp_info = nullptr;
   uint8_t *bclass = nullptr;
   // filter tile geometry per TW (32,16,8,4,2,1)
   int tile_extn[6] = {}, tile_extw[6] = {}, tile_molcap[6] = {};
@@ -366,11 +368,13 @@ struct QPlan {
   std::vector<int32_t> row;     // [VQ] global query node of depth e
   std::vector<int32_t> beoff;   // [VQ+1]
   std::vector<uint16_t> be;     // (j << 8) | class
+  std::vector<uint32_t> info;   // [VQ] first back-edge j | class << 8 | (#back-edges - 1) << 16; j = 0xff: none
 };
 
 void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const uint8_t *bclass, QPlan &out) {
   out.row.assign((size_t)q.V, 0);
   out.beoff.assign((size_t)q.V + 1, 0);
+  out.info.assign((size_t)q.V, 0xffu);
   out.be.clear();
   for (int64_t g = 0; g < q.G; g++) {
     const int64_t lo = q.goff[g];
@@ -405,6 +409,11 @@ void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const u
       for (int64_t k = q.roff[lo + u]; k < q.roff[lo + u + 1]; k++) {
         const int w = (int)(q.col[k] - lo);
         if (pos[w] < e) out.be.push_back((uint16_t)((pos[w] << 8) | bclass[q.elab[k]]));
+      }
+      const int nbe = (int)out.be.size() - out.beoff[lo + e];
+      if (nbe > 0) {
+        const uint16_t f = out.be[out.beoff[lo + e]];
+        out.info[lo + e] = (uint32_t)(f >> 8) | ((uint32_t)(f & 0xff) << 8) | ((uint32_t)(nbe - 1) << 16);
       }
     }
   }
@@ -572,16 +581,17 @@ void fill_join_caps(sigmo_ctx *c, JoinParams &jp) {
   jp.VQ = c->VQ;
   jp.NB = c->NB;
   jp.maxq = std::max(c->maxq, 2);
-  jp.PCAP = c->PC + c->NQ;
+  jp.PCAP = c->PC;
   jp.ACAP = c->AC + c->maxn;
-  jp.CMCAP = c->CMC + c->VQ;
+  jp.CMCAP = std::max(c->CMC, jp.maxq);
   jp.MCAP = c->MC;
   jp.NBE = c->NBE;
   jp.plan_smem = c->plan_smem;
   const int scg = 32 * (jp.maxq + 1) + 64;
-  jp.SCS = std::min(scg, 160);
-  jp.SW = (jp.ACAP + 31) / 32 + 2;
-  jp.slice_rows = ((size_t)c->VQ * jp.SW * 4 <= 16384) ? c->VQ : 0;
+  jp.SCS = std::min(scg, 128);
+  if (const char *e = getenv("SIGMO_JOIN_SCS")) jp.SCS = std::max(128, atoi(e));  // test knob (spill path)
+  jp.SW = 0;
+  jp.slice_rows = 0;
 }
 
 // join internal-capacity flag and DFS step counter (synchronizes)
@@ -744,6 +754,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const size_t o_beoff = L.take(4 * ((size_t)hq.V + 1));
   const size_t o_be = L.take(2 * plan.be.size() + 2);
   const size_t o_bc = L.take(256);
+  const size_t o_info = L.take(4 * (size_t)hq.V + 4);
   const PackedOffsets pd = plan_graphs(L, hd);
   const size_t total = L.off;
   // wait until the previous upload no longer reads the staging buffer
@@ -762,6 +773,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   memcpy(hb + o_beoff, plan.beoff.data(), 4 * plan.beoff.size());
   if (!plan.be.empty()) memcpy(hb + o_be, plan.be.data(), 2 * plan.be.size());
   memcpy(hb + o_bc, bclass, 256);
+  if (!plan.info.empty()) memcpy(hb + o_info, plan.info.data(), 4 * plan.info.size());
   pack_graphs(hb, pd, hd);
 
   // ---- device arena + one H2D copy ----
@@ -776,6 +788,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->qp_beoff = (int32_t *)(db + o_beoff);
   c->qp_be = (uint16_t *)(db + o_be);
   c->bclass = db + o_bc;
+  c->qp_info = (uint32_t *)(db + o_info);
   c->NQ = (int)hq.G;
   c->VQ = (int)hq.V;
   c->EQ = (int)hq.E;
@@ -793,21 +806,21 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   if (c->Wpad == 0) c->Wpad = 32;
   tile_geometry(c, hd);
   c->NBE = (int)plan.be.size();
-  c->plan_smem = (4 * ((size_t)c->NQ + 1) + 8 * ((size_t)c->VQ + 1) + 2 * (size_t)c->NBE) <= 16384 ? 1 : 0;
+  c->plan_smem = 0;  // plans are read through the read-only cache
   // join chunk capacities (pairs, atoms, candidate masks, graphs per warp
   // chunk): shrink until the join's shared memory allows >= 2 CTAs per SM
   {
-    c->PC = 64;
-    c->AC = 64;
-    c->CMC = 256;
-    c->MC = 16;
+    c->PC = 80;
+    c->AC = 48;
+    c->CMC = 320;
+    c->MC = 8;
     for (int tries = 0; tries < 12; tries++) {
       JoinParams jp{};
       fill_join_caps(c, jp);
-      if (join_smem_bytes(c->NW, jp) <= c->max_smem / 2 || c->PC == 1) break;
-      c->PC = std::max(c->PC / 2, 1);
-      c->AC = std::max(c->AC / 2, 1);
-      c->CMC = std::max(c->CMC / 2, 1);
+      if (join_smem_bytes(c->NW, jp) <= c->max_smem / 2 || c->PC <= 8) break;
+      c->PC = std::max(c->PC / 2, 8);
+      c->AC = std::max(c->AC / 2, 8);
+      c->CMC = std::max(c->CMC / 2, 32);
       c->MC = std::max(c->MC / 2, 1);
     }
   }
@@ -829,8 +842,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   SIGMO_TRY(dreserve(c, c->scan_tmp, tb, "scan temp"));
   c->scan_tmp_bytes = std::max(tb, (size_t)16);
   const long long pair_cap = (long long)c->NQ * c->ND;
-  const long long max_chunks = pair_cap / c->PC + (long long)c->VD / c->AC + (long long)c->VQ * c->ND / c->CMC +
-                               (long long)c->ND / c->MC + 4;
+  const long long max_chunks = (long long)c->VD / c->AC + (long long)c->ND / c->MC + 4;
   SIGMO_TRY(dreserve(c, c->chunk_start, 4 * (size_t)max_chunks, "chunk starts"));
   SIGMO_TRY(dreserve(c, c->nchunks, 16, "chunk count"));
   SIGMO_TRY(dreserve(c, c->pair_query, 4 * (size_t)std::max(pair_cap, 1ll), "pair queries"));
@@ -965,6 +977,7 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
     jp.qp_row = c->qp_row;
     jp.qp_beoff = c->qp_beoff;
     jp.qp_be = c->qp_be;
+    jp.qp_info = c->qp_info;
     jp.pair_query = (int32_t *)c->pair_query.p;
     jp.pair_result = (unsigned long long *)c->pair_result.p;
     jp.totals = (unsigned long long *)c->jcnt.p + 6;

@@ -95,6 +95,7 @@ struct JoinParams {
   const int32_t *qp_row;       // [VQ] plan order: global query node of depth e
   const int32_t *qp_beoff;     // [VQ+1] back-edge list per (query, depth)
   const uint16_t *qp_be;       // (depth j << 8) | bond class
+  const uint32_t *qp_info;     // [VQ] first back-edge j | class << 8 | (#back-edges - 1) << 16 (j = 0xff: none)
   int32_t *pair_query;
   unsigned long long *pair_result;
   unsigned long long *totals;  // [NQ]

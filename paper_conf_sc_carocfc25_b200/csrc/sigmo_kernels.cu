@@ -749,7 +749,8 @@ __global__ void k_chunks(ChunkParams p) {
   const int g = blockIdx.x * blockDim.x + threadIdx.x;
   auto key = [&](int x) -> long long {
     const I64x2 o = p.off[x];
-    return o.a / p.PC + (long long)p.goff[x] / p.AC + o.b / p.CMC + (long long)x / p.MC;
+    (void)o;
+    return (long long)p.goff[x] / p.AC + (long long)x / p.MC;
   };
   if (g == 0) {
     p.chunk_start[0] = 0;
@@ -781,7 +782,7 @@ cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st) {
 // own molecule chunks and never wait for each other).
 // ---------------------------------------------------------------------------
 struct JoinWarpSmem {
-  size_t adj, cm, pinfo, cnt, found, mstart, scratch, total;  // scratch = bitmap slice (staging) | DFS stack
+  size_t adj, cm, cinfo, pinfo, cnt, found, mstart, scratch, total;  // scratch = bitmap slice (staging) | DFS stack
 };
 struct JoinSmem {
   size_t plan, tot, warps;
@@ -797,11 +798,17 @@ __host__ __device__ inline size_t join_plan_bytes(int NQ, int VQ, int NBE) {
 
 // DFS iterator stack: safe capacity (global promotion) and shared-memory capacity
 __host__ __device__ inline int join_stack_cap(int maxq) { return 32 * (maxq + 1) + 64; }
-__host__ __device__ inline size_t join_entry_bytes(int NW, int MQ) { return 4 + 8 * (size_t)MQ + 16 * (size_t)NW; }
-// bytes of a stack of `cap` entries laid out as hdr[cap] | map[cap][MQ] | used[cap] | R[cap]
-__host__ __device__ inline size_t join_stack_bytes(int NW, int MQ, int cap) {
-  return align16(4 * (size_t)cap) + align16(8 * (size_t)MQ * cap) + 16 * (size_t)NW * cap;
-}
+__host__ __device__ inline size_t join_entry_bytes(int NW, int MQ) { return align16(8 * (2 * (size_t)NW + MQ) + 4); }
+__host__ __device__ inline size_t join_stack_bytes(int NW, int MQ, int cap) { return join_entry_bytes(NW, MQ) * cap; }
+
+// one DFS iterator (array-of-structs, 16-byte aligned: vector loads/stores)
+template <int NW, int MQ>
+struct __align__(16) DfsEntry {
+  unsigned long long R[NW];     // candidates of depth d not yet tried
+  unsigned long long used[NW];  // data nodes of the partial mapping
+  unsigned long long map[MQ];   // f(pi_0..pi_{d-1}), one byte each
+  uint32_t hdr;                 // pair | d << 16
+};
 
 __host__ __device__ inline JoinSmem join_layout(const JoinParams &p, int NW, int MQ) {
   JoinSmem L;
@@ -814,14 +821,13 @@ __host__ __device__ inline JoinSmem join_layout(const JoinParams &p, int NW, int
   size_t w = 0;
   L.w.adj = w;     w = align16(w + mb * (size_t)p.NB * p.ACAP);
   L.w.cm = w;      w = align16(w + mb * (size_t)p.CMCAP);
+  L.w.cinfo = w;   w = align16(w + 4 * (size_t)p.CMCAP);
   L.w.pinfo = w;   w = align16(w + 16 * (size_t)p.PCAP);
   L.w.cnt = w;     w = align16(w + 8 * (size_t)p.PCAP);
   L.w.found = w;   w = align16(w + (size_t)p.PCAP);
   L.w.mstart = w;  w = align16(w + 4 * (size_t)(p.MCAP + 1));
   L.w.scratch = w;
-  const size_t slice = p.slice_rows ? 4 * (size_t)p.slice_rows * p.SW : 0;
-  const size_t stack = join_stack_bytes(NW, MQ, p.SCS);
-  w = align16(w + (slice > stack ? slice : stack));
+  w = align16(w + join_stack_bytes(NW, MQ, p.SCS));
   L.w.total = w;
   o += w * NWARP;
   L.total = o;
@@ -878,24 +884,18 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
   unsigned char *wb = smem + L.warps + (size_t)wid * L.w.total;
   M *s_adj = (M *)(wb + L.w.adj);
   M *s_cm = (M *)(wb + L.w.cm);
+  uint32_t *s_cinfo = (uint32_t *)(wb + L.w.cinfo);  // plan info of (pair, depth), parallel to s_cm
   int4 *s_pinfo = (int4 *)(wb + L.w.pinfo);  // {cm offset, plan base qb, mbase | n << 16, q << 8 | nq}
   unsigned long long *s_cnt = (unsigned long long *)(wb + L.w.cnt);
   uint8_t *s_found = wb + L.w.found;
   int *s_mstart = (int *)(wb + L.w.mstart);
-  uint32_t *s_slice = (uint32_t *)(wb + L.w.scratch);
   // DFS stack (shared memory; promoted to a global area if it ever fills)
+  using E = DfsEntry<NW, MQ>;
   const int SCS = jp.SCS;
-  uint32_t *const sm_hdr = (uint32_t *)(wb + L.w.scratch);
-  unsigned long long *const sm_map = (unsigned long long *)(wb + L.w.scratch + align16(4 * (size_t)SCS));
-  M *const sm_used = (M *)((unsigned char *)sm_map + align16(8 * (size_t)MQ * SCS));
-  M *const sm_R = sm_used + SCS;
+  E *const st = (E *)(wb + L.w.scratch);
   const int SCG = join_stack_cap(jp.maxq);
   const size_t gwarp = (size_t)blockIdx.x * NWARP + wid;
-  unsigned char *gb = jp.gstack + gwarp * join_stack_bytes(NW, MQ, SCG);
-  uint32_t *const gm_hdr = (uint32_t *)gb;
-  unsigned long long *const gm_map = (unsigned long long *)(gb + align16(4 * (size_t)SCG));
-  M *const gm_used = (M *)((unsigned char *)gm_map + align16(8 * (size_t)MQ * SCG));
-  M *const gm_R = gm_used + SCG;
+  E *const spill = (E *)(jp.gstack + gwarp * join_stack_bytes(NW, MQ, SCG));
 
   const int ACAP = jp.ACAP;
   const int32_t *qgoff = jp.qgoff, *qp_beoff = jp.qp_beoff, *qp_row = jp.qp_row;
@@ -917,8 +917,7 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
   }
   for (int i = tid; i < jp.NQ; i += NT) s_tot[i] = 0ull;
   __syncthreads();
-  long long nodes = 0, iters = 0, tail_iters = 0;
-  int max_top = 0;
+  long long nodes = 0, iters = 0;
   const unsigned lt = (1u << lane) - 1u;
 
   while (true) {
@@ -955,86 +954,108 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
       for (int b = 0; b < 8; b++)
         if (b < jp.NB) s_adj[b * ACAP + i] = m[b];
     }
-    // ---- stage: coalesced copy of the chunk's bitmap slice (all rows) ----
-    const int ws = a0 >> 5;
-    const int nws = na > 0 ? ((a0 + na - 1) >> 5) - ws + 1 : 0;
-    if (jp.slice_rows) {
-      const int tot = jp.slice_rows * nws;
-      for (int t = lane; t < tot; t += 32) {
-        const int row = t / nws, w = t - row * nws;
-        s_slice[row * jp.SW + w] = __ldg(&jp.bitmap[(size_t)row * jp.Wpad + ws + w]);
-      }
-    }
     __syncwarp();
-    // ---- stage: GMCR pairs (lane = query) ----
+    // The chunk's pairs are processed in passes that fit the warp's pair /
+    // candidate-mask capacity (PCAP, CMCAP >= the largest query); pairs are
+    // taken in GMCR order, so a pass is the contiguous range [done, done+pnp).
+    int done = 0, mi_start = 0;
+    while (done < np) {
+    // ---- stage: the pass's GMCR pairs (lane = query) ----
+    int pnp = 0;
     {
-      int run_p = 0, run_c = 0;
-      for (int mi = 0; mi < nm; mi++) {
+      int pos = 0, cpos = 0;
+      bool full = false;
+      for (int mi = mi_start; mi < nm && !full; mi++) {
         const int g = g0 + mi;
+        const int first = (int)(jp.off[g].a - p0);
+        if ((int)(jp.off[g + 1].a - p0) <= done) {
+          mi_start = mi + 1;
+          continue;
+        }
         const int mbase = s_mstart[mi], n = s_mstart[mi + 1] - mbase;
+        int gi = first;
         for (int qb = 0; qb < jp.NQW; qb++) {
           const uint32_t bits = __ldg(&jp.gm[(size_t)g * jp.NQW + qb]);
           const int q = qb * 32 + lane;
-          const bool ok = (bits >> lane) & 1u;
+          const bool take = ((bits >> lane) & 1u) && (gi + __popc(bits & lt) >= done);
           int nq = 0, qbase = 0;
-          if (ok) {
+          if (take) {
             qbase = qgoff[q];
             nq = qgoff[q + 1] - qbase;
           }
+          const unsigned tm = __ballot_sync(FULL_MASK, take);
           int xc = nq;
 #pragma unroll
           for (int o = 1; o < 32; o <<= 1) {
             const int y = __shfl_up_sync(FULL_MASK, xc, o);
             if (lane >= o) xc += y;
           }
-          if (ok) {
-            const int pos = run_p + __popc(bits & lt);
-            s_pinfo[pos] = make_int4(run_c + xc - nq, qbase, mbase | (n << 16), (q << 8) | nq);
-            s_cnt[pos] = 0ull;
-            s_found[pos] = 0;
+          const int tp = __popc(tm & lt);
+          const bool fits = take && (pos + tp < jp.PCAP) && (cpos + xc <= jp.CMCAP);
+          const unsigned fm = __ballot_sync(FULL_MASK, fits);
+          if (fits) {
+            s_pinfo[pos + tp] = make_int4(cpos + xc - nq, qbase, mbase | (n << 16), (q << 8) | nq);
+            s_cnt[pos + tp] = 0ull;
+            s_found[pos + tp] = 0;
           }
-          run_p += __popc(bits);
-          run_c += __shfl_sync(FULL_MASK, xc, 31);
+          pos += __popc(fm);
+          cpos += __shfl_sync(FULL_MASK, fits ? xc : 0, fm ? 31 - __clz(fm) : 0);
+          if (tm & ~fm) {
+            full = true;
+            break;
+          }
+          gi += __popc(bits);
         }
       }
+      pnp = pos;
     }
     __syncwarp();
     // ---- stage: candidate masks cm[pair][e] (molecule window of each query-node row) ----
-    for (int i = lane; i < np; i += 32) {
+    for (int i = lane; i < pnp; i += 32) {
       const int4 pi = s_pinfo[i];
       const int nq = pi.w & 0xff, mbase = pi.z & 0xffff, n = pi.z >> 16;
+#pragma unroll 2
       for (int e = 0; e < nq; e++) {
-        const int row = qp_row[pi.y + e];
-        M w;
-        if (jp.slice_rows)
-          w = extract_window<NW>(s_slice + (size_t)row * jp.SW, nws, (long long)(a0 + mbase) - (long long)ws * 32, n);
-        else
-          w = extract_window<NW>(jp.bitmap + (size_t)row * jp.Wpad, jp.Wpad, (long long)a0 + mbase, n);
-        s_cm[pi.x + e] = w;
+        const int row = __ldg(&qp_row[pi.y + e]);
+        s_cm[pi.x + e] = extract_window<NW>(jp.bitmap + (size_t)row * jp.Wpad, jp.Wpad, (long long)a0 + mbase, n);
+        s_cinfo[pi.x + e] = __ldg(&jp.qp_info[pi.y + e]);
       }
     }
     __syncwarp();
 
     // ---- DFS on the warp's iterator stack ----
-    uint32_t *st_hdr = sm_hdr;
-    unsigned long long *st_map = sm_map;
-    M *st_used = sm_used, *st_R = sm_R;
-    int cap = SCS;
-    int top = 0, next_pair = 0;
+    // hot part of the stack in shared memory (SCS entries); the oldest
+    // entries spill to the warp's global area when it fills (never on the
+    // common path) and come back when the shared part runs low.
+    int top = 0, nspill = 0, next_pair = 0;
     while (true) {
-      if (top < 32 && next_pair < np) {
+      if (top < 32 && nspill > 0) {
+        // restore: shift the shared entries up by r, bring back r spilled ones
+        const int r = min(nspill, SCS / 2);
+        E keep;
+        if (lane < top) keep = st[lane];
+        __syncwarp();
+        if (lane < top) st[r + lane] = keep;
+        for (int i = lane; i < r; i += 32) st[i] = spill[nspill - r + i];
+        nspill -= r;
+        top += r;
+        __syncwarp();
+      }
+      if (top < 32 && next_pair < pnp) {
         // seed iterators of new pairs: E = (pair, d = 0, R = root candidates)
         const int pi = next_pair + lane;
-        const bool ok = lane < 32 - top && pi < np;
+        const bool ok = lane < 32 - top && pi < pnp;
         if (ok) {
-          const int idx = top + lane;
-          st_hdr[idx] = (uint32_t)pi;
-          st_R[idx] = s_cm[s_pinfo[pi].x];
-          M z;
-          z.clear();
-          st_used[idx] = z;
+          E en;
 #pragma unroll
-          for (int k = 0; k < MQ; k++) st_map[(size_t)idx * MQ + k] = 0ull;
+          for (int k = 0; k < NW; k++) {
+            en.R[k] = s_cm[s_pinfo[pi].x].w[k];
+            en.used[k] = 0ull;
+          }
+#pragma unroll
+          for (int k = 0; k < MQ; k++) en.map[k] = 0ull;
+          en.hdr = (uint32_t)pi;
+          st[top + lane] = en;
         }
         const int added = __popc(__ballot_sync(FULL_MASK, ok));
         top += added;
@@ -1044,27 +1065,19 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
       if (top == 0) break;
       const int take = min(32, top);
       iters++;
-      if (next_pair >= np) tail_iters++;
-      max_top = max(max_top, top);
       top -= take;
       const bool act = lane < take;
-      const int idx = top + lane;
-      uint32_t hdr = 0;
-      M R, used;
-      R.clear();
-      used.clear();
-      unsigned long long mp[MQ];
-#pragma unroll
-      for (int k = 0; k < MQ; k++) mp[k] = 0ull;
-      if (act) {
-        hdr = st_hdr[idx];
-        R = st_R[idx];
-        used = st_used[idx];
-#pragma unroll
-        for (int k = 0; k < MQ; k++) mp[k] = st_map[(size_t)idx * MQ + k];
-      }
+      E en;
+      if (act) en = st[top + lane];
       __syncwarp();
       nodes += take;
+      M R, used;
+#pragma unroll
+      for (int k = 0; k < NW; k++) {
+        R.w[k] = act ? en.R[k] : 0ull;
+        used.w[k] = act ? en.used[k] : 0ull;
+      }
+      const uint32_t hdr = act ? en.hdr : 0u;
       const int pair = hdr & 0xffff;
       const int d = hdr >> 16;
       bool alive = act;
@@ -1076,9 +1089,11 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
       const int v = alive ? R.lowest() : 0;
       if (alive) R.clear_lowest();
       const bool push_rem = alive && R.any();
-      unsigned long long mrem[MQ];
 #pragma unroll
-      for (int k = 0; k < MQ; k++) mrem[k] = mp[k];
+      for (int k = 0; k < NW; k++) en.R[k] = R.w[k];  // remainder iterator (same depth, v removed)
+      unsigned long long mp[MQ];
+#pragma unroll
+      for (int k = 0; k < MQ; k++) mp[k] = en.map[k];
       map_set<MQ>(mp, d, v);
       M u2 = used;
       if (alive) u2.set(v);
@@ -1092,10 +1107,17 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
           cnt = 1ull;  // single-node query
         } else {
           x = s_cm[pinf.x + e].andnot(u2);
-          const int k1 = qp_beoff[pinf.y + e + 1];
-          for (int k = qp_beoff[pinf.y + e]; k < k1; k++) {
-            const int be = qp_be[k];
-            x &= s_adj[(be & 255) * ACAP + mbase + map_get<MQ>(mp, be >> 8)];
+          const uint32_t info = s_cinfo[pinf.x + e];
+          const int j0 = info & 0xff;
+          if (j0 != 0xff) x &= s_adj[((info >> 8) & 0xff) * ACAP + mbase + map_get<MQ>(mp, j0)];
+          const int ne = (info >> 16) & 0xff;
+          if (ne) {
+            const int k0 = __ldg(&jp.qp_beoff[pinf.y + e]) + 1;
+#pragma unroll 1
+            for (int k = 0; k < ne; k++) {
+              const int be = __ldg(&jp.qp_be[k0 + k]);
+              x &= s_adj[(be & 255) * ACAP + mbase + map_get<MQ>(mp, be >> 8)];
+            }
           }
           if (e == nq - 1) cnt = (unsigned long long)x.popc();  // last depth: count
           else push_child = x.any();
@@ -1112,61 +1134,60 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
       // push: remainders first, then children (children end on top)
       const unsigned mr = __ballot_sync(FULL_MASK, push_rem);
       const unsigned mc = __ballot_sync(FULL_MASK, push_child);
-      const int npush = __popc(mr) + __popc(mc);
-      if (top + npush > cap - 32) {
-        // promote the stack to the warp's global area (capacity join_stack_cap)
-        if (st_hdr == sm_hdr) {
-          for (int i = lane; i < top; i += 32) {
-            gm_hdr[i] = sm_hdr[i];
-            gm_used[i] = sm_used[i];
-            gm_R[i] = sm_R[i];
-#pragma unroll
-            for (int k = 0; k < MQ; k++) gm_map[(size_t)i * MQ + k] = sm_map[(size_t)i * MQ + k];
-          }
-          __syncwarp();
-          st_hdr = gm_hdr;
-          st_map = gm_map;
-          st_used = gm_used;
-          st_R = gm_R;
-          cap = SCG;
-        }
-        if (top + npush > cap) {
+      const int nr = __popc(mr);
+      const int npush = nr + __popc(mc);
+      if (top + npush > SCS) {
+        // spill the oldest m shared entries to global, shift the rest down
+        const int m = min(top, max(SCS / 2, top + npush - SCS));
+        if (nspill + m > SCG) {
           if (lane == 0) atomicOr(jp.error, 1);
           top = 0;
-          next_pair = np;
+          nspill = 0;
+          next_pair = pnp;
           continue;
         }
+        for (int i = lane; i < m; i += 32) spill[nspill + i] = st[i];
+        __syncwarp();
+        for (int base = m; base < top; base += 32) {
+          E t;
+          const int i = base + lane;
+          if (i < top) t = st[i];
+          __syncwarp();
+          if (i < top) st[i - m] = t;
+          __syncwarp();
+        }
+        nspill += m;
+        top -= m;
       }
-      if (push_rem) {
-        const int j = top + __popc(mr & lt);
-        st_hdr[j] = hdr;
-        st_R[j] = R;
-        st_used[j] = used;
-#pragma unroll
-        for (int k = 0; k < MQ; k++) st_map[(size_t)j * MQ + k] = mrem[k];
-      }
+      if (push_rem) st[top + __popc(mr & lt)] = en;
       if (push_child) {
-        const int j = top + __popc(mr) + __popc(mc & lt);
-        st_hdr[j] = (uint32_t)pair | ((uint32_t)e << 16);
-        st_R[j] = x;
-        st_used[j] = u2;
+        E ch;
 #pragma unroll
-        for (int k = 0; k < MQ; k++) st_map[(size_t)j * MQ + k] = mp[k];
+        for (int k = 0; k < NW; k++) {
+          ch.R[k] = x.w[k];
+          ch.used[k] = u2.w[k];
+        }
+#pragma unroll
+        for (int k = 0; k < MQ; k++) ch.map[k] = mp[k];
+        ch.hdr = (uint32_t)pair | ((uint32_t)e << 16);
+        st[top + nr + __popc(mc & lt)] = ch;
       }
       top += npush;
       __syncwarp();
     }
     // ---- results: GMCR pair list + per-pair result + per-query totals ----
-    for (int i = lane; i < np; i += 32) {
+    for (int i = lane; i < pnp; i += 32) {
       unsigned long long r = s_cnt[i];
       if (MODE == 1) r = r ? 1ull : 0ull;
       const int q = s_pinfo[i].w >> 8;
-      jp.pair_query[p0 + i] = q;
-      jp.pair_result[p0 + i] = r;
+      jp.pair_query[p0 + done + i] = q;
+      jp.pair_result[p0 + done + i] = r;
       if (r) atomicAdd(&s_tot[q], r);
     }
-    (void)c0;
+    done += pnp;
     __syncwarp();
+    }  // passes
+    (void)c0;
   }
   __syncthreads();
   for (int i = tid; i < jp.NQ; i += NT)
@@ -1174,8 +1195,6 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
   if (jp.stats && lane == 0) {
     atomicAdd(jp.stats, (unsigned long long)nodes);
     atomicAdd(jp.stats + 1, (unsigned long long)iters);
-    atomicAdd(jp.stats + 2, (unsigned long long)tail_iters);
-    atomicMax(jp.stats + 3, (unsigned long long)max_top);
   }
 }
 

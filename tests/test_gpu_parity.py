@@ -212,3 +212,19 @@ def test_c2_full_size_parity(ctx, sigmo):
         for v in range(lo, hi):
             w, b = v >> 5, v & 31
             assert np.array_equal((bm[:, w] >> b) & 1, (ref_bits[:, w] >> b) & 1), (g, v)
+
+
+def test_join_stack_spill_path(sigmo, monkeypatch):
+    """Force the smallest shared-memory DFS stack so that the global spill /
+    restore path runs (deep 20-30-atom ring-system queries), results unchanged."""
+    monkeypatch.setenv("SIGMO_JOIN_SCS", "128")
+    Q = synth.config_queries(4)
+    D = synth.config_data(4, count=150)
+    with sigmo.Context(0) as c:
+        c.load_batch(Q, D)
+        c.filter(2)
+        c.set_timing(True)
+        c.join(sigmo.SIGMO_FIND_ALL)
+        assert np.array_equal(c.dense_results(), oracle.count_dense(Q, D))
+        c.join(sigmo.SIGMO_FIND_FIRST)
+        assert np.array_equal(c.dense_results(), oracle.count_dense(Q, D, oracle.FIND_FIRST))
