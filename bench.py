@@ -34,7 +34,7 @@ BASELINE_METRIC = "matches/sec (Find All) and graph-pairs/sec (Find First) at 1/
 CONFIG_ID = 2
 MOLS_PER_RANK = 100_000
 LEVELS = 4
-CPU_SAMPLE_MOLS = 20_000      # cpu_baseline leg: ~20 core-seconds of oracle work
+CPU_SAMPLE_MOLS = 100_000     # cpu_baseline leg: all of configs[1] (~20 core-seconds of oracle work)
 REF_STEP_MOLS = 2_000         # --impl reference: molecules per step
 
 
@@ -257,12 +257,13 @@ def main():
     totals = torch.zeros(Q.num_graphs, dtype=torch.int64, device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
 
+    from paper_conf_sc_carocfc25_b200 import sharded
+
     def step(mode=sigmo.SIGMO_FIND_ALL):
         ctx.filter(args.levels)
         ctx.join(mode, total=False)
         ctx.query_totals(device_tensor=totals)
-        if dist is not None:
-            dist.all_reduce(totals)
+        sharded.allreduce_totals(totals)  # the only collective: NCCL sum of per-query totals
 
     # ---- warm-up ----
     for _ in range(max(args.warmup, 3)):
@@ -352,12 +353,24 @@ def main():
     filter_roof = {"bound": "hbm", "achieved": filter_bytes / (f_ms * 1e-3) / 1e9, "peak": hbm_peak,
                    "unit": "GB/s", "frac": filter_bytes / (f_ms * 1e-3) / 1e9 / hbm_peak, "traffic": None,
                    "kernel": "k_filter", "ms": f_ms, "algorithmic_bytes": filter_bytes, "peak_source": peak_src}
-    # join: ALU/issue bound: achieved = surviving pairs/s
-    sm_mhz = clocks.get("sm_mhz") or float(peaks.get("sm_max_mhz", 1965.0))
-    join_roof = {"bound": "alu", "kernel": "k_join", "ms": j_ms,
+    # join: ALU bound: algorithmic work = DFS iterator
+    # steps x 12 lane-ops; peak = 148 SMs x 128 lanes x SM clock
+    sm_mhz = float(clocks.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0))
+    traffic = {}
+    try:
+        traffic = _json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+    except Exception:
+        pass
+    steps = tim.get("dfs_steps", 0)
+    alu_peak = 148 * 128 * sm_mhz * 1e6 / 1e12
+    join_ach = 12.0 * steps / (j_ms * 1e-3) / 1e12 if j_ms > 0 else 0.0
+    join_roof = {"bound": "alu", "achieved": join_ach, "peak": alu_peak, "unit": "Tops/s", "frac": join_ach / alu_peak,
+                 "traffic": traffic.get("k_join"), "kernel": "k_join", "ms": j_ms, "dfs_steps_per_launch": steps,
+                 "ops_per_step": 12, "peak_source": f"148 SM x 128 int lanes x {sm_mhz:.0f} MHz (measured clock)",
                  "pairs_per_launch": pairs_local, "matches_per_launch": matches_local}
+    filter_roof["traffic"] = traffic.get("k_filter")
     dominant = "join" if j_ms >= f_ms else "filter"
-    roofline = dict(filter_roof) if dominant == "filter" else None
+    roofline = dict(join_roof) if dominant == "join" else dict(filter_roof)
 
     line = {
         "metric": BASELINE_METRIC, "value": value, "unit": "matches/s", "n_gpus": world, "steps": K,
@@ -377,9 +390,8 @@ def main():
                 "note": "sigmo_load_batch (validate+pack+pinned H2D) + filter + join + D2H totals, wall clock"},
         "gpu_launches": int(K * (tim["filter_launches"] + tim["join_launches"])),
         "clocks": clocks,
+        "roofline": roofline,
     }
-    if roofline is not None:
-        line["roofline"] = roofline
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = run_cpu_baseline(Q, args.levels)
     print(json.dumps(line), flush=True)

@@ -228,3 +228,24 @@ def test_join_stack_spill_path(sigmo, monkeypatch):
         assert np.array_equal(c.dense_results(), oracle.count_dense(Q, D))
         c.join(sigmo.SIGMO_FIND_FIRST)
         assert np.array_equal(c.dense_results(), oracle.count_dense(Q, D, oracle.FIND_FIRST))
+
+
+def test_shard_additivity_gpu(sigmo):
+    """Molecule shards (balanced by atoms) run one after another on the GPU:
+    per-query totals add up to the unsharded run and to the oracle (P6)."""
+    from paper_conf_sc_carocfc25_b200 import sharded
+    Q, D = synth.config_queries(2), synth.config_data(2, count=3000)
+    ref = oracle.count_dense(Q, D).sum(axis=1).astype(np.uint64)
+    with sigmo.Context(0) as c:
+        c.load_batch(Q, D)
+        c.filter(3)
+        c.join(sigmo.SIGMO_FIND_ALL)
+        assert np.array_equal(c.query_totals(), ref)
+        acc = np.zeros(Q.num_graphs, np.uint64)
+        for r in range(3):
+            g0, g1 = sharded.shard_range(D.graph_offsets, r, 3)
+            c.load_batch(Q, D.slice(g0, g1))
+            c.filter(3)
+            c.join(sigmo.SIGMO_FIND_ALL)
+            acc += c.query_totals()
+        assert np.array_equal(acc, ref)
