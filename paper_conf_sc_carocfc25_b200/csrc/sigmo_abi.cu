@@ -368,13 +368,13 @@ struct QPlan {
   std::vector<int32_t> row;     // [VQ] global query node of depth e
   std::vector<int32_t> beoff;   // [VQ+1]
   std::vector<uint16_t> be;     // (j << 8) | class
-  std::vector<uint32_t> info;   // [VQ] first back-edge j | class << 8 | (#back-edges - 1) << 16; j = 0xff: none
+  std::vector<uint32_t> info;   // [VQ] two back-edges inline + #extra + leaf-sum flag (see plan_queries)
 };
 
 void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const uint8_t *bclass, QPlan &out) {
   out.row.assign((size_t)q.V, 0);
   out.beoff.assign((size_t)q.V + 1, 0);
-  out.info.assign((size_t)q.V, 0xffu);
+  out.info.assign((size_t)q.V, 0x3fu | (0x3fu << 9));
   out.be.clear();
   for (int64_t g = 0; g < q.G; g++) {
     const int64_t lo = q.goff[g];
@@ -410,10 +410,25 @@ void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const u
         const int w = (int)(q.col[k] - lo);
         if (pos[w] < e) out.be.push_back((uint16_t)((pos[w] << 8) | bclass[q.elab[k]]));
       }
+      // info word: j0 (6 bits, 0x3f none) | b0 << 6 | j1 << 9 (0x3f none) | b1 << 15 |
+      // (#back-edges beyond two) << 18 | leaf-sum flag << 24
       const int nbe = (int)out.be.size() - out.beoff[lo + e];
+      uint32_t inf = 0x3fu | (0x3fu << 9);
       if (nbe > 0) {
         const uint16_t f = out.be[out.beoff[lo + e]];
-        out.info[lo + e] = (uint32_t)(f >> 8) | ((uint32_t)(f & 0xff) << 8) | ((uint32_t)(nbe - 1) << 16);
+        inf = (inf & ~0x1ffu) | (uint32_t)(f >> 8) | ((uint32_t)(f & 7) << 6);
+      }
+      if (nbe > 1) {
+        const uint16_t f = out.be[out.beoff[lo + e] + 1];
+        inf = (inf & ~(0x1ffu << 9)) | ((uint32_t)(f >> 8) << 9) | ((uint32_t)(f & 7) << 15);
+      }
+      if (nbe > 2) inf |= (uint32_t)(nbe - 2) << 18;
+      out.info[lo + e] = inf;
+      if (e == n - 1 && n >= 3) {
+        // bit 24: the last node has no back-edge to depth n-2 (leaf-sum closed form applies)
+        bool adj_prev = false;
+        for (int k = out.beoff[lo + e]; k < (int)out.be.size(); k++) adj_prev |= (out.be[k] >> 8) == n - 2;
+        if (!adj_prev) out.info[lo + e] |= 1u << 24;
       }
     }
   }
@@ -877,7 +892,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       rows_smem = k < 6 ? 1 : 0;
       const int kk = k % 6;
       smem = filter_smem_bytes(c->NW, c->tile_extn[kk], c->tile_extw[kk], c->tile_molcap[kk], m.NFU, m.NLAB, m.P,
-                               m.G, c->VQ, m.row_entries, rows_smem);
+                               m.G, c->VQ, m.row_entries, rows_smem, c->NQW);
       // prefer >= 2 CTAs per SM with row programs in shared memory
       if (smem <= (rows_smem ? c->max_smem / 2 : c->max_smem)) break;
     }

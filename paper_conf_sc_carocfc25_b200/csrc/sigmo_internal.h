@@ -125,7 +125,7 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
                               cudaStream_t st);
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int G, int VQ, int RE,
-                         int rows_smem);
+                         int rows_smem, int NQW);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);
 cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);

@@ -92,6 +92,12 @@ struct Mask {
     return c;
   }
   __device__ __forceinline__ int lowest() const {
+    if (NW == 1) {
+      // branch-free count of trailing zeros (w != 0 assumed by callers; 64 if 0 -> -1)
+      const unsigned long long x = w[0];
+      const int t = __popcll((x & (0ull - x)) - 1ull);
+      return x ? t : -1;
+    }
     int r = -1;
 #pragma unroll
     for (int k = NW - 1; k >= 0; k--)
@@ -420,19 +426,19 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
 // k_filter: one CTA per tile of TW (<= 32) bitmap words = 32*TW data nodes.
 // ===========================================================================
 struct FilterSmem {
-  size_t adj, ballA, ballB, fm, planes, win, nz, molstart, molslot, fid, lab, mstart, sos, rowlab, rowoff, rowids,
-      prog, total;
+  size_t adj, ballA, ballB, fm, planes, fplanes, win, nz, gmb, slotat, bnd, own, molstart, molslot, fid, lab, mstart,
+      sos, rowlab, rowoff, rowids, prog, total;
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
 
-// prog block: p_t[P] u8 | grp_f[G] u8 | fslot[16] i8 | grp_poff[G+1] i16 | rg_off[16] i16
+// prog block: p_t[P] u8 | p_grp[P] u8 | grp_f[G] u8 | fslot[16] i8 | grp_poff[G+1] i16 | rg_off[16] i16
 __host__ __device__ inline size_t prog_bytes(int P, int G) {
-  return align16((size_t)P) + align16((size_t)G) + 16 + align16(2 * (size_t)(G + 1)) + 32;
+  return 2 * align16((size_t)P) + align16((size_t)G) + 16 + align16(2 * (size_t)(G + 1)) + 32;
 }
 
 __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB,
-                                                    int P, int G, int VQ, int RE, int rows_smem) {
+                                                    int P, int G, int VQ, int RE, int rows_smem, int NQW) {
   FilterSmem L;
   const size_t mb = 8 * (size_t)NW;
   const int NWARP = kFilterThreads / 32;
@@ -443,8 +449,13 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   L.ballB = o;    o = align16(o + mb * EXTN);
   L.fm = o;       o = align16(o + mb * (size_t)MOLCAP * (NFU > 0 ? NFU : 1));
   L.planes = o;   o = align16(o + 4 * (size_t)(NLAB + P) * EXTW);
+  L.fplanes = o;  o = align16(o + 4 * (size_t)(NFU > 0 ? NFU : 1) * EXTW);
   L.win = o;      o = align16(o + mb * (size_t)NWARP * (NLAB + P));
   L.nz = o;       o = align16(o + 4 * (size_t)NWARP * (VQW + 1));
+  L.gmb = o;      o = align16(o + 4 * (size_t)MOLCAP * (NQW > 0 ? NQW : 1));
+  L.slotat = o;   o = align16(o + 2 * 32 * 32);
+  L.bnd = o;      o = align16(o + 4 * 32);
+  L.own = o;      o = align16(o + 4 * 32);
   L.molstart = o; o = align16(o + 2 * (size_t)EXTN);
   L.molslot = o;  o = align16(o + 2 * (size_t)EXTN);
   L.fid = o;      o = align16(o + (size_t)EXTN);
@@ -460,8 +471,8 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
 }
 
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int G, int VQ, int RE,
-                         int rows_smem) {
-  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, G, VQ, RE, rows_smem).total;
+                         int rows_smem, int NQW) {
+  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, G, VQ, RE, rows_smem, NQW).total;
 }
 
 template <int NW>
@@ -470,14 +481,19 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   constexpr int NT = kFilterThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
   const FilterSmem L = filter_layout(NW, fp.EXTN, fp.EXTW, fp.MOLCAP, fp.NFU, fp.NLAB, fp.P, fp.G, fp.VQ, fp.RE,
-                                     fp.rows_smem);
+                                     fp.rows_smem, fp.NQW);
   M *s_adj = (M *)(smem + L.adj);
   M *s_cur = (M *)(smem + L.ballA);
   M *s_nxt = (M *)(smem + L.ballB);
   M *s_fm = (M *)(smem + L.fm);
   uint32_t *s_planes = (uint32_t *)(smem + L.planes);
+  uint32_t *s_fplanes = (uint32_t *)(smem + L.fplanes);
   M *s_win = (M *)(smem + L.win);
   uint32_t *s_nz = (uint32_t *)(smem + L.nz);
+  uint32_t *s_gm = (uint32_t *)(smem + L.gmb);
+  int16_t *s_slotat = (int16_t *)(smem + L.slotat);
+  uint32_t *s_bnd = (uint32_t *)(smem + L.bnd);
+  uint32_t *s_own = (uint32_t *)(smem + L.own);
   int16_t *s_molstart = (int16_t *)(smem + L.molstart);
   int16_t *s_molslot = (int16_t *)(smem + L.molslot);
   uint8_t *s_fid = smem + L.fid;
@@ -486,7 +502,8 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   int16_t *s_sos = (int16_t *)(smem + L.sos);
   // plane program (always in smem)
   uint8_t *s_pt = smem + L.prog;
-  uint8_t *s_grpf = s_pt + align16(fp.P);
+  uint8_t *s_pgrp = s_pt + align16(fp.P);
+  uint8_t *s_grpf = s_pgrp + align16(fp.P);
   int8_t *s_fslot = (int8_t *)(s_grpf + align16(fp.G));
   int16_t *s_grpoff = (int16_t *)(s_fslot + 16);
   int16_t *s_rg = (int16_t *)((unsigned char *)s_grpoff + align16(2 * (size_t)(fp.G + 1)));
@@ -494,7 +511,7 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   const uint8_t *rowlab = fp.row_lab;
   const int32_t *rowoff = fp.row_off;
   const uint16_t *rowids = fp.row_ids;
-  __shared__ int s_g0, s_g1;
+  __shared__ int s_g0, s_g1, s_strad;
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int ND = fp.D.num_graphs, VD = fp.D.num_nodes;
@@ -506,9 +523,13 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   if (tid == 0) {
     s_g0 = graph_of(goff, ND, n0);
     s_g1 = graph_of(goff, ND, n1 - 1) + 1;
+    s_strad = -1;
   }
   for (int i = tid; i < fp.P; i += NT) s_pt[i] = fp.p_t[i];
-  for (int i = tid; i < fp.G; i += NT) s_grpf[i] = fp.grp_f[i];
+  for (int i = tid; i < fp.G; i += NT) {
+    s_grpf[i] = fp.grp_f[i];
+    for (int p = fp.grp_poff[i]; p < fp.grp_poff[i + 1]; p++) s_pgrp[p] = (uint8_t)i;
+  }
   for (int i = tid; i <= fp.G; i += NT) s_grpoff[i] = fp.grp_poff[i];
   for (int i = tid; i <= fp.R; i += NT) s_rg[i] = fp.rg_off[i];
   for (int i = tid; i < kNumFields; i += NT) s_fslot[i] = fp.fslot[i];
@@ -523,6 +544,10 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     rowoff = b;
     rowids = c;
   }
+  if (tid < 32) {
+    s_bnd[tid] = 0u;
+    s_own[tid] = 0u;
+  }
   __syncthreads();
   const int g0 = s_g0, g1 = s_g1, nmol = g1 - g0;
   const int gs = __ldg(&goff[g0]);
@@ -531,9 +556,28 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   const int xb = gs >> 5;                       // first ext word (global word index)
   const int nxw = ((ge - 1) >> 5) - xb + 1;     // ext words
   const int NLAB = fp.NLAB, P = fp.P, NFU = fp.NFU, EXTW = fp.EXTW;
+  const int tw_eff = min(fp.TW, fp.W - w0);     // words written by this tile
+  const int tbits = 32 * tw_eff;
 
   // ---- phase 1: nodes of all molecules overlapping the tile ----
-  for (int i = tid; i <= nmol; i += NT) s_mstart[i] = __ldg(&goff[g0 + i]) - gs;
+  for (int i = tid; i < nmol * fp.NQW; i += NT) s_gm[i] = 0u;
+  for (int i = tid; i <= nmol; i += NT) {
+    const int st = __ldg(&goff[g0 + i]) - gs;
+    s_mstart[i] = st;
+    if (i < nmol) {
+      const int n = __ldg(&goff[g0 + i + 1]) - gs - st;
+      const int tb = gs + st - n0;  // tile bit of the molecule start
+      if (n > 0 && tb >= 0 && tb < tbits) {
+        atomicOr(&s_bnd[tb >> 5], 1u << (tb & 31));
+        if (tb + n <= tbits && NW == 1) {
+          atomicOr(&s_own[tb >> 5], 1u << (tb & 31));
+          s_slotat[tb] = (int16_t)i;
+        } else {
+          s_strad = i;  // starts here, ends beyond the tile (or needs the multi-word path)
+        }
+      }
+    }
+  }
   for (int i = tid; i < next; i += NT) {
     const int v = gs + i;
     const int loc = __ldg(&fp.D.local[v]);
@@ -548,26 +592,15 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     s_lab[i] = (uint8_t)lab;
     s_fid[i] = (uint8_t)field_of(lab);
   }
-  for (int i = tid; i < nmol * NFU; i += NT) s_fm[i].clear();
   __syncthreads();
   for (int mi = tid; mi < nmol; mi += NT)
     if (s_mstart[mi] < s_mstart[mi + 1]) s_sos[s_mstart[mi]] = (int16_t)mi;
-  __syncthreads();
-  for (int i = tid; i < next; i += NT) {
-    const int ms = s_molstart[i];
-    const int slot = s_sos[ms];
-    s_molslot[i] = (int16_t)slot;
-    const int fs = NFU > 0 ? s_fslot[s_fid[i]] : -1;
-    if (fs >= 0) {
-      const int loc = i - ms;
-      atomicOr(&s_fm[slot * NFU + fs].w[loc >> 6], 1ull << (loc & 63));
-    }
-  }
-  // ---- label planes (InitializeCandidates, Alg.1 l.29-37) ----
+  // ---- label planes (InitializeCandidates, Alg.1 l.29-37) and field planes ----
   for (int k = wid; k < nxw; k += NWARP) {
     const int i = (xb + k) * 32 + lane - gs;
     const bool valid = (i >= 0) && (i < next);
     const int lab = valid ? s_lab[i] : -1;
+    const int fid = valid ? s_fid[i] : -1;
     uint32_t mine = 0;
     for (int c = 0; c < NLAB; c++) {
       const unsigned b = __ballot_sync(FULL_MASK, lab == (int)__ldg(&fp.lab_val[c]));
@@ -575,7 +608,21 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
       if ((c & 31) == 31 || c == NLAB - 1)
         if (lane <= (c & 31)) s_planes[((c & ~31) + lane) * EXTW + k] = mine;
     }
+    for (int f = 0; f < kNumFields; f++) {
+      const int fs = s_fslot[f];
+      if (fs < 0) continue;
+      const unsigned b = __ballot_sync(FULL_MASK, fid == f);
+      if (lane == 0) s_fplanes[fs * EXTW + k] = b;
+    }
   }
+  __syncthreads();
+  // per-molecule field masks = windows of the field planes
+  for (int t = tid; t < nmol * NFU; t += NT) {
+    const int mi = t / NFU, fs = t - mi * NFU;
+    const int ms = s_mstart[mi], n = s_mstart[mi + 1] - ms;
+    s_fm[t] = extract_window<NW>(s_fplanes + (size_t)fs * EXTW, nxw, (long long)(gs + ms) - (long long)xb * 32, n);
+  }
+  for (int i = tid; i < next; i += NT) s_molslot[i] = s_sos[s_molstart[i]];
   __syncthreads();
 
   // ---- radii 1..R: bitset BFS + threshold planes (RefineCandidates, l.19-28) ----
@@ -593,7 +640,7 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     s_nxt = t;
     const int gb = s_rg[r - 1], gend = s_rg[r];
     if (gb < gend) {
-      const int pb = s_grpoff[gb], pe_r = s_grpoff[gend];
+      const int pb = s_grpoff[gb], pe = s_grpoff[gend];
       for (int k = wid; k < nxw; k += NWARP) {
         const int i = (xb + k) * 32 + lane - gs;
         const bool valid = (i >= 0) && (i < next);
@@ -606,47 +653,84 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
           fid = s_fid[i];
         }
         uint32_t mine = 0;
-        for (int grp = gb; grp < gend; grp++) {
-          const int f = s_grpf[grp];
-          int cnt = 0;
-          if (valid) cnt = (ball & s_fm[slot * NFU + s_fslot[f]]).popc() - (fid == f ? 1 : 0);
-          const int pe = s_grpoff[grp + 1];
-          for (int p = s_grpoff[grp]; p < pe; p++) {
-            const unsigned b = __ballot_sync(FULL_MASK, cnt >= (int)s_pt[p]);
-            const int j = p - pb;
-            if ((j & 31) == lane) mine = b;
-            if ((j & 31) == 31 || p == pe_r - 1)
-              if (lane <= (j & 31)) s_planes[(NLAB + pb + (j & ~31) + lane) * EXTW + k] = mine;
+        int gprev = -1, cnt = 0;
+        for (int p = pb; p < pe; p++) {
+          const int g = s_pgrp[p];
+          if (g != gprev) {  // warp-uniform: planes are sorted by (r, f, t)
+            gprev = g;
+            const int f = s_grpf[g];
+            cnt = valid ? (ball & s_fm[slot * NFU + s_fslot[f]]).popc() - (fid == f ? 1 : 0) : 0;
           }
+          const unsigned b = __ballot_sync(FULL_MASK, cnt >= (int)s_pt[p]);
+          const int j = p - pb;
+          if ((j & 31) == lane) mine = b;
+          if ((j & 31) == 31 || p == pe - 1)
+            if (lane <= (j & 31)) s_planes[(NLAB + pb + (j & ~31) + lane) * EXTW + k] = mine;
         }
       }
     }
     __syncthreads();
   }
 
-  // ---- rows: C_L word = label plane AND its constraint planes; written once ----
+  // ---- rows (query-major): C_L word = label plane AND constraint planes,
+  // written once; GMCR of the molecules contained in the tile from the row
+  // words by a segmented OR ----
   {
     const int w = w0 + lane;
-    const bool active = (lane < fp.TW) && (w < fp.W);
+    const bool active = lane < tw_eff;
     const int k = w - xb;
-    for (int row = wid; row < fp.VQ; row += NWARP) {
-      const int rl = rowlab[row];
-      const int j0 = rowoff[row], j1 = rowoff[row + 1];
-      if (active) {
-        uint32_t x = s_planes[rl * EXTW + k];
-        for (int j = j0; j < j1; j++) x &= s_planes[(NLAB + rowids[j]) * EXTW + k];
-        fp.bitmap[(size_t)row * fp.Wpad + w] = x;
+    // per-lane segment data (NW == 1 path)
+    const uint32_t B = s_bnd[lane], OWN = s_own[lane];
+    const uint32_t Br = __brev(B), nBr = ~Br;
+    const uint32_t lowm = B ? ((B & (0u - B)) - 1u) : 0xffffffffu;  // bits below the first boundary
+    const uint32_t topb = B ? (0x80000000u >> __clz(B)) : 0u;          // highest boundary bit
+    const bool nob = (B == 0u);
+    const bool nob_next = __shfl_down_sync(FULL_MASK, nob, 1) && lane + 1 < tw_eff;
+    for (int q = wid; q < fp.NQ; q += NWARP) {
+      const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
+      uint32_t Aq = 0xffffffffu;
+      for (int row = r0; row < r1; row++) {
+        const int rl = rowlab[row];
+        const int j0 = rowoff[row], j1 = rowoff[row + 1];
+        uint32_t x = 0u;
+        if (active) {
+          x = s_planes[rl * EXTW + k];
+          for (int j = j0; j < j1; j++) x &= s_planes[(NLAB + rowids[j]) * EXTW + k];
+          fp.bitmap[(size_t)row * fp.Wpad + w] = x;
+        }
+        if (NW == 1) {
+          // any-bit per segment, reported at its boundary bit (bit-reversed add)
+          const uint32_t xr = __brev(x);
+          const uint32_t rr = (xr & nBr) + nBr;
+          uint32_t A = __brev((rr | xr) & Br);
+          // the top segment continues into the next word(s)
+          const bool loc = (x & lowm) != 0u;
+          const bool l1 = __shfl_down_sync(FULL_MASK, loc, 1) && lane + 1 < tw_eff;
+          const bool l2 = __shfl_down_sync(FULL_MASK, loc, 2) && lane + 2 < tw_eff;
+          if (l1 || (nob_next && l2)) A |= topb;
+          Aq &= A;
+        }
+      }
+      if (NW == 1) {
+        uint32_t bits = Aq & OWN;
+        while (bits) {
+          const int b = __ffs(bits) - 1;
+          bits &= bits - 1u;
+          const int mi = s_slotat[lane * 32 + b];
+          atomicOr(&s_gm[mi * fp.NQW + (q >> 5)], 1u << (q & 31));
+        }
       }
     }
   }
 
-  // ---- GMCR test for molecules starting in this tile ----
-  // per molecule: windows of every plane, one non-empty bit per query node
-  // (lane = query node), then every query whose nodes are all non-empty.
+  // ---- GMCR by plane windows: the molecule straddling the tile end (and,
+  // for multi-word masks, every molecule starting in the tile) ----
   M *win = s_win + (size_t)wid * (NLAB + P);
   const int VQW = (fp.VQ + 31) >> 5;
   uint32_t *nz = s_nz + (size_t)wid * (VQW + 1);
+  const int strad = s_strad;
   for (int mi = wid; mi < nmol; mi += NWARP) {
+    if (NW == 1 && mi != strad) continue;
     const int g = g0 + mi;
     const int gst = __ldg(&goff[g]);
     if (gst < n0) continue;  // owned by the previous tile
@@ -669,14 +753,12 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     }
     if (lane == 0) nz[VQW] = 0u;
     __syncwarp();
-    long long np = 0, ncm = 0;
     for (int qb = 0; qb < fp.NQW; qb++) {
       const int q = qb * 32 + lane;
       bool ok = false;
-      int nq = 0;
       if (q < fp.NQ) {
         const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
-        nq = r1 - r0;
+        const int nq = r1 - r0;
         const int wi = r0 >> 5, sh = r0 & 31;
         uint32_t v = nz[wi] >> sh;
         if (sh) v |= nz[wi + 1] << (32 - sh);
@@ -684,20 +766,25 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
         ok = (v & want) == want;
       }
       const unsigned bits = __ballot_sync(FULL_MASK, ok);
-      if (lane == 0) fp.gm[(size_t)g * fp.NQW + qb] = bits;
-      np += __popc(bits);
-      int c = ok ? nq : 0;
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(FULL_MASK, c, o);
-      ncm += c;
-    }
-    if (lane == 0) {
-      I64x2 v;
-      v.a = np;
-      v.b = ncm;
-      fp.mol_cnt[g] = v;
+      if (lane == 0) s_gm[mi * fp.NQW + qb] = bits;
     }
     __syncwarp();
+  }
+  __syncthreads();
+  // ---- write the GMCR bits and pair counts of the molecules starting here ----
+  for (int mi = tid; mi < nmol; mi += NT) {
+    const int g = g0 + mi;
+    if (__ldg(&goff[g]) < n0) continue;
+    long long np = 0;
+    for (int qb = 0; qb < fp.NQW; qb++) {
+      const uint32_t bits = s_gm[mi * fp.NQW + qb];
+      fp.gm[(size_t)g * fp.NQW + qb] = bits;
+      np += __popc(bits);
+    }
+    I64x2 v;
+    v.a = np;
+    v.b = 0;
+    fp.mol_cnt[g] = v;
   }
 }
 
@@ -917,7 +1004,7 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
   }
   for (int i = tid; i < jp.NQ; i += NT) s_tot[i] = 0ull;
   __syncthreads();
-  long long nodes = 0, iters = 0;
+  int nodes = 0, iters = 0;
   const unsigned lt = (1u << lane) - 1u;
 
   while (true) {
@@ -1082,53 +1169,78 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
       const int d = hdr >> 16;
       bool alive = act;
       if (MODE == 1 && alive && s_found[pair]) alive = false;
-      int4 pinf = make_int4(0, 0, 0, 0);
-      if (alive) pinf = s_pinfo[pair];
+      const int4 pinf = s_pinfo[pair];  // pair 0 is always staged; dead lanes are masked below
       const int nq = pinf.w & 0xff;
       const int mbase = pinf.z & 0xffff;
-      const int v = alive ? R.lowest() : 0;
-      if (alive) R.clear_lowest();
+      // one candidate v of depth d; the remainder keeps the others
+      const int v = R.lowest();
+      R.clear_lowest();
       const bool push_rem = alive && R.any();
 #pragma unroll
-      for (int k = 0; k < NW; k++) en.R[k] = R.w[k];  // remainder iterator (same depth, v removed)
+      for (int k = 0; k < NW; k++) en.R[k] = R.w[k];
       unsigned long long mp[MQ];
 #pragma unroll
       for (int k = 0; k < MQ; k++) mp[k] = en.map[k];
-      map_set<MQ>(mp, d, v);
+      map_set<MQ>(mp, d, v & 0xff);
       M u2 = used;
-      if (alive) u2.set(v);
-      const int e = d + 1;  // mapped nodes after this step
-      unsigned long long cnt = 0ull;
-      bool push_child = false;
-      M x;
-      x.clear();
-      if (alive) {
-        if (e == nq) {
-          cnt = 1ull;  // single-node query
-        } else {
-          x = s_cm[pinf.x + e].andnot(u2);
-          const uint32_t info = s_cinfo[pinf.x + e];
-          const int j0 = info & 0xff;
-          if (j0 != 0xff) x &= s_adj[((info >> 8) & 0xff) * ACAP + mbase + map_get<MQ>(mp, j0)];
-          const int ne = (info >> 16) & 0xff;
-          if (ne) {
-            const int k0 = __ldg(&jp.qp_beoff[pinf.y + e]) + 1;
+      u2.set(v & (64 * NW - 1));
+      const int e = d + 1;  // mapped nodes after this step (plan depth of the next node)
+      // candidates of depth e: cm & ~used & adj of its (<= 2 inline) back-edges
+      const int ec = min(e, nq - 1);
+      const uint32_t info = s_cinfo[pinf.x + ec];
+      M x = s_cm[pinf.x + ec].andnot(u2);
+      {
+        const int j0 = info & 0x3f, j1 = (info >> 9) & 0x3f;
+        const M a0 = s_adj[((info >> 6) & 7) * ACAP + mbase + map_get<MQ>(mp, j0 & 31)];
+        const M a1 = s_adj[((info >> 15) & 7) * ACAP + mbase + map_get<MQ>(mp, j1 & 31)];
+        if (j0 != 0x3f) x &= a0;
+        if (j1 != 0x3f) x &= a1;
+      }
+      const int nex = (info >> 18) & 0x3f;
+      if (nex) {  // > 2 back-edges at this depth (fused ring systems): rare
+        const int k0 = __ldg(&jp.qp_beoff[pinf.y + ec]) + 2;
 #pragma unroll 1
-            for (int k = 0; k < ne; k++) {
-              const int be = __ldg(&jp.qp_be[k0 + k]);
-              x &= s_adj[(be & 255) * ACAP + mbase + map_get<MQ>(mp, be >> 8)];
-            }
-          }
-          if (e == nq - 1) cnt = (unsigned long long)x.popc();  // last depth: count
-          else push_child = x.any();
+        for (int k = 0; k < nex; k++) {
+          const int be = __ldg(&jp.qp_be[k0 + k]);
+          x &= s_adj[(be & 255) * ACAP + mbase + map_get<MQ>(mp, be >> 8)];
         }
       }
+      // leaf sum (e == nq-2 and the last node is not adjacent to depth nq-2):
+      // X = candidates of the last depth given f(0..e-1) and v; then
+      // sum_{w in x} |X \ {w}| = |x||X| - |x & X|
+      const int lastd = max(nq - 1, 0);
+      const uint32_t li = s_cinfo[pinf.x + lastd];
+      const bool lsum = (e == nq - 2) && ((li >> 24) & 1u);
+      unsigned long long cnt = 0ull;
+      if (__any_sync(FULL_MASK, lsum && alive)) {
+        M X = s_cm[pinf.x + lastd].andnot(u2);
+        const int j0 = li & 0x3f, j1 = (li >> 9) & 0x3f;
+        const M a0 = s_adj[((li >> 6) & 7) * ACAP + mbase + map_get<MQ>(mp, j0 & 31)];
+        const M a1 = s_adj[((li >> 15) & 7) * ACAP + mbase + map_get<MQ>(mp, j1 & 31)];
+        if (j0 != 0x3f) X &= a0;
+        if (j1 != 0x3f) X &= a1;
+        const int lnex = (li >> 18) & 0x3f;
+        if (lsum && lnex) {
+          const int k0 = __ldg(&jp.qp_beoff[pinf.y + lastd]) + 2;
+#pragma unroll 1
+          for (int k = 0; k < lnex; k++) {
+            const int be = __ldg(&jp.qp_be[k0 + k]);
+            X &= s_adj[(be & 255) * ACAP + mbase + map_get<MQ>(mp, be >> 8)];
+          }
+        }
+        if (lsum) cnt = (unsigned long long)x.popc() * (unsigned long long)X.popc() - (unsigned long long)(x & X).popc();
+      }
+      if (e == nq - 1) cnt = (unsigned long long)x.popc();  // last depth: count
+      if (e == nq) cnt = 1ull;                                // single-node query
+      if (!alive) cnt = 0ull;
+      const bool push_child = alive && (e < nq - 1) && !lsum && x.any();
       if (cnt) {
         // 64-bit per-pair count kept as two 32-bit words with carry
         uint32_t *w = (uint32_t *)&s_cnt[pair];
-        const uint32_t add = (uint32_t)cnt;  // <= 64
+        const uint32_t add = (uint32_t)cnt;
         const uint32_t old = atomicAdd(w, add);
-        if (old + add < old) atomicAdd(w + 1, 1u);
+        const uint32_t hi = (uint32_t)(cnt >> 32) + ((old + add < old) ? 1u : 0u);
+        if (hi) atomicAdd(w + 1, hi);
         if (MODE == 1) s_found[pair] = 1;
       }
       // push: remainders first, then children (children end on top)
