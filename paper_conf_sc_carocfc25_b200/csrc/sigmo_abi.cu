@@ -113,6 +113,7 @@ struct sigmo_ctx {
   int32_t *qp_row = nullptr, *qp_beoff = nullptr;
   uint16_t *qp_be = nullptr;
   uint32_t *qp_info = nullptr;
+  int32_t *tile_g0 = nullptr, *tile_g1 = nullptr;
   uint8_t *bclass = nullptr;
   // filter tile geometry per TW (32,16,8,4,2,1)
   int tile_extn[6] = {}, tile_extw[6] = {}, tile_molcap[6] = {};
@@ -306,7 +307,8 @@ struct Layout {
 };
 
 struct PackedOffsets {
-  size_t goff, label, local, roff, nbr;
+  size_t goff, label, local, roff, nbr, adj64;
+  bool has_adj64;
 };
 
 PackedOffsets plan_graphs(Layout &L, const HostGraphs &h) {
@@ -316,6 +318,10 @@ PackedOffsets plan_graphs(Layout &L, const HostGraphs &h) {
   p.local = L.take((size_t)h.V);
   p.roff = L.take(4 * (size_t)(h.V + 1));
   p.nbr = L.take(2 * (size_t)h.E);
+  int64_t mx = 0;
+  for (int64_t g = 0; g < h.G; g++) mx = std::max<int64_t>(mx, h.goff[g + 1] - h.goff[g]);
+  p.has_adj64 = mx <= 64;
+  p.adj64 = p.has_adj64 ? L.take(8 * (size_t)h.V) : 0;
   return p;
 }
 
@@ -325,6 +331,7 @@ void pack_graphs(unsigned char *base, const PackedOffsets &p, const HostGraphs &
   uint8_t *local = base + p.local;
   int32_t *roff = (int32_t *)(base + p.roff);
   uint16_t *nbr = (uint16_t *)(base + p.nbr);
+  uint64_t *adj64 = p.has_adj64 ? (uint64_t *)(base + p.adj64) : nullptr;
   goff[h.G] = (int32_t)h.V;
   roff[h.V] = (int32_t)h.E;
   parallel_for_graphs(h.G, h.E + h.V, [&](int, int64_t ga, int64_t gb) {
@@ -335,8 +342,12 @@ void pack_graphs(unsigned char *base, const PackedOffsets &p, const HostGraphs &
         label[u] = h.nlab[u];
         local[u] = (uint8_t)(u - lo);
         roff[u] = (int32_t)h.roff[u];
-        for (int64_t e = h.roff[u]; e < h.roff[u + 1]; e++)
+        uint64_t m = 0;
+        for (int64_t e = h.roff[u]; e < h.roff[u + 1]; e++) {
           nbr[e] = (uint16_t)(((h.col[e] - lo) << 8) | h.elab[e]);
+          m |= 1ull << ((h.col[e] - lo) & 63);
+        }
+        if (adj64) adj64[u] = m;
       }
     }
   });
@@ -354,6 +365,7 @@ DevGraphs dev_view(unsigned char *dbase, const PackedOffsets &p, const HostGraph
   d.local = dbase + p.local;
   d.roff = (const int32_t *)(dbase + p.roff);
   d.nbr = (const uint16_t *)(dbase + p.nbr);
+  d.adj64 = p.has_adj64 ? (const unsigned long long *)(dbase + p.adj64) : nullptr;
   return d;
 }
 
@@ -762,6 +774,18 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   QPlan plan;
   plan_queries(hq, freq, bclass, plan);
 
+  // per-tile graph ranges of the filter for TW = 32 (1,024 nodes per tile)
+  std::vector<int32_t> tg0, tg1;
+  {
+    const int64_t W = (hd.V + 31) / 32, tiles = (W + 31) / 32;
+    tg0.resize((size_t)tiles + 1);
+    tg1.resize((size_t)tiles + 1);
+    for (int64_t t = 0; t < tiles; t++) {
+      const int64_t n0 = t * 1024, n1 = std::min<int64_t>(n0 + 1024, hd.V);
+      tg0[t] = graph_of_host(hd.goff, hd.G, n0);
+      tg1[t] = graph_of_host(hd.goff, hd.G, n1 - 1) + 1;
+    }
+  }
   // ---- staging layout ----
   Layout L;
   const PackedOffsets pq = plan_graphs(L, hq);
@@ -771,6 +795,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const size_t o_bc = L.take(256);
   const size_t o_info = L.take(4 * (size_t)hq.V + 4);
   const PackedOffsets pd = plan_graphs(L, hd);
+  const size_t o_tg0 = L.take(4 * tg0.size());
+  const size_t o_tg1 = L.take(4 * tg1.size());
   const size_t total = L.off;
   // wait until the previous upload no longer reads the staging buffer
   CUDA_TRY(c, cudaEventSynchronize(c->h2d_done));
@@ -790,6 +816,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   memcpy(hb + o_bc, bclass, 256);
   if (!plan.info.empty()) memcpy(hb + o_info, plan.info.data(), 4 * plan.info.size());
   pack_graphs(hb, pd, hd);
+  memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
+  memcpy(hb + o_tg1, tg1.data(), 4 * tg1.size());
 
   // ---- device arena + one H2D copy ----
   SIGMO_TRY(dreserve(c, c->arena, total, "input arena"));
@@ -803,6 +831,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->qp_beoff = (int32_t *)(db + o_beoff);
   c->qp_be = (uint16_t *)(db + o_be);
   c->bclass = db + o_bc;
+  c->tile_g0 = (int32_t *)(db + o_tg0);
+  c->tile_g1 = (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
   c->NQ = (int)hq.G;
   c->VQ = (int)hq.V;
@@ -873,8 +903,6 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
   if (c->state < 1) return set_err(c, SIGMO_ERR_STATE, "sigmo_filter before sigmo_load_batch");
   if (levels < 1 || levels > SIGMO_MAX_LEVELS) return set_err(c, SIGMO_ERR_INVALID_ARG, "levels %d not in 1..16", levels);
   if (flags & ~(uint32_t)SIGMO_FILTER_NEIGHBOR_SUPPORT) return set_err(c, SIGMO_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
-  if (flags & SIGMO_FILTER_NEIGHBOR_SUPPORT)
-    return set_err(c, SIGMO_ERR_INVALID_ARG, "SIGMO_FILTER_NEIGHBOR_SUPPORT not available in this build");
   CUDA_TRY(c, cudaSetDevice(c->device));
   const int R = levels - 1;
   timing_begin_filter(c);
@@ -928,6 +956,8 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.EXTW = c->tile_extw[k];
     fp.MOLCAP = c->tile_molcap[k];
     fp.RE = m.row_entries;
+    fp.tile_g0 = tws[k] == 32 ? c->tile_g0 : nullptr;
+    fp.tile_g1 = tws[k] == 32 ? c->tile_g1 : nullptr;
     fp.rows_smem = rows_smem;
     fp.smem_bytes = smem;
     if (c->has_empty_graph) {
@@ -938,6 +968,29 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     timing_mark(c, 2);
     CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));
     launches++;
+    if (flags & SIGMO_FILTER_NEIGHBOR_SUPPORT) {
+      SupportParams sp{};
+      sp.ND = c->ND;
+      sp.NQ = c->NQ;
+      sp.NQW = c->NQW;
+      sp.NB = c->NB;
+      sp.maxq = std::max(c->maxq, 1);
+      sp.Wpad = c->Wpad;
+      sp.goff = c->dd.goff;
+      sp.roff = c->dd.roff;
+      sp.nbr = c->dd.nbr;
+      sp.bclass = c->bclass;
+      sp.qgoff = c->dq.goff;
+      sp.qroff = c->dq.roff;
+      sp.qnbr = c->dq.nbr;
+      sp.bitmap = (uint32_t *)c->bitmap.p;
+      sp.gm = (uint32_t *)c->gm.p;
+      sp.mol_cnt = (I64x2 *)c->mol_cnt.p;
+      if (support_smem_bytes(c->NW, c->NB, sp.maxq, c->NQW) > c->max_smem)
+        return set_err(c, SIGMO_ERR_LIMIT, "neighbour-support shared memory exceeds the device limit");
+      CUDA_TRY(c, launch_support(c->NW, sp, c->stream));
+      launches++;
+    }
     timing_mark(c, 3);
     size_t tb = c->scan_tmp_bytes;
     CUDA_TRY(c, launch_scan((const I64x2 *)c->mol_cnt.p, (I64x2 *)c->off.p, c->ND + 1, c->scan_tmp.p, &tb, c->stream));

@@ -26,6 +26,7 @@ struct DevGraphs {
   const uint8_t *local = nullptr;  // [V] index of the node inside its graph
   const int32_t *roff = nullptr;   // [V+1]
   const uint16_t *nbr = nullptr;   // [E2]
+  const unsigned long long *adj64 = nullptr;  // [V] molecule-local adjacency mask (all graphs <= 64 nodes), else null
 };
 
 // Query-side plane program, built on the device by k_query_prep from the
@@ -76,6 +77,7 @@ struct FilterParams {
   I64x2 *mol_cnt;              // [ND+1] (surviving pairs, candidate-mask entries)
   int EXTN, EXTW, MOLCAP;
   int RE, rows_smem;           // row-program entries; 1 = copy row programs to smem
+  const int32_t *tile_g0, *tile_g1;  // per-tile graph range for TW = 32 (null: binary search)
   size_t smem_bytes;
 };
 
@@ -109,6 +111,18 @@ struct JoinParams {
   size_t smem_bytes;
 };
 
+struct SupportParams {
+  int ND, NQ, NQW, NB, maxq, Wpad;
+  const int32_t *goff, *roff;
+  const uint16_t *nbr;
+  const uint8_t *bclass;
+  const int32_t *qgoff, *qroff;  // query CSR (global query node ids; qnbr local index << 8 | bond)
+  const uint16_t *qnbr;
+  uint32_t *bitmap;
+  uint32_t *gm;
+  I64x2 *mol_cnt;
+};
+
 struct ChunkParams {
   int ND;
   const int32_t *goff;
@@ -126,6 +140,8 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int G, int VQ, int RE,
                          int rows_smem, int NQW);
+cudaError_t launch_support(int NW, const SupportParams &p, cudaStream_t st);
+size_t support_smem_bytes(int NW, int NB, int maxq, int NQW);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);
 cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);

@@ -476,7 +476,7 @@ size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NL
 }
 
 template <int NW>
-__global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
+__global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
   using M = Mask<NW>;
   constexpr int NT = kFilterThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
@@ -512,6 +512,7 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   const int32_t *rowoff = fp.row_off;
   const uint16_t *rowids = fp.row_ids;
   __shared__ int s_g0, s_g1, s_strad;
+  __shared__ uint8_t s_fused[kNumFields];
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int ND = fp.D.num_graphs, VD = fp.D.num_nodes;
@@ -521,8 +522,13 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   const int n1 = min(n0 + fp.TW * 32, VD);
   const int32_t *goff = fp.D.goff;
   if (tid == 0) {
-    s_g0 = graph_of(goff, ND, n0);
-    s_g1 = graph_of(goff, ND, n1 - 1) + 1;
+    if (fp.tile_g0) {
+      s_g0 = __ldg(&fp.tile_g0[blockIdx.x]);
+      s_g1 = __ldg(&fp.tile_g1[blockIdx.x]);
+    } else {
+      s_g0 = graph_of(goff, ND, n0);
+      s_g1 = graph_of(goff, ND, n1 - 1) + 1;
+    }
     s_strad = -1;
   }
   for (int i = tid; i < fp.P; i += NT) s_pt[i] = fp.p_t[i];
@@ -532,7 +538,10 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   }
   for (int i = tid; i <= fp.G; i += NT) s_grpoff[i] = fp.grp_poff[i];
   for (int i = tid; i <= fp.R; i += NT) s_rg[i] = fp.rg_off[i];
-  for (int i = tid; i < kNumFields; i += NT) s_fslot[i] = fp.fslot[i];
+  for (int i = tid; i < kNumFields; i += NT) {
+    s_fslot[i] = fp.fslot[i];
+    if (fp.fslot[i] >= 0) s_fused[fp.fslot[i]] = (uint8_t)i;
+  }
   if (fp.rows_smem) {
     uint8_t *a = smem + L.rowlab;
     int32_t *b = (int32_t *)(smem + L.rowoff);
@@ -583,8 +592,12 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     const int loc = __ldg(&fp.D.local[v]);
     M a;
     a.clear();
-    const int e1 = __ldg(&fp.D.roff[v + 1]);
-    for (int e = __ldg(&fp.D.roff[v]); e < e1; e++) a.set(__ldg(&fp.D.nbr[e]) >> 8);
+    if (NW == 1 && fp.D.adj64) {
+      a.w[0] = __ldg(&fp.D.adj64[v]);
+    } else {
+      const int e1 = __ldg(&fp.D.roff[v + 1]);
+      for (int e = __ldg(&fp.D.roff[v]); e < e1; e++) a.set(__ldg(&fp.D.nbr[e]) >> 8);
+    }
     s_adj[i] = a;
     s_cur[i] = M::bit(loc);
     s_molstart[i] = (int16_t)(i - loc);
@@ -608,10 +621,8 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
       if ((c & 31) == 31 || c == NLAB - 1)
         if (lane <= (c & 31)) s_planes[((c & ~31) + lane) * EXTW + k] = mine;
     }
-    for (int f = 0; f < kNumFields; f++) {
-      const int fs = s_fslot[f];
-      if (fs < 0) continue;
-      const unsigned b = __ballot_sync(FULL_MASK, fid == f);
+    for (int fs = 0; fs < NFU; fs++) {
+      const unsigned b = __ballot_sync(FULL_MASK, fid == (int)s_fused[fs]);
       if (lane == 0) s_fplanes[fs * EXTW + k] = b;
     }
   }
@@ -640,7 +651,7 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     s_nxt = t;
     const int gb = s_rg[r - 1], gend = s_rg[r];
     if (gb < gend) {
-      const int pb = s_grpoff[gb], pe = s_grpoff[gend];
+      const int pb = s_grpoff[gb];
       for (int k = wid; k < nxw; k += NWARP) {
         const int i = (xb + k) * 32 + lane - gs;
         const bool valid = (i >= 0) && (i < next);
@@ -652,20 +663,17 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
           slot = s_molslot[i];
           fid = s_fid[i];
         }
-        uint32_t mine = 0;
-        int gprev = -1, cnt = 0;
-        for (int p = pb; p < pe; p++) {
-          const int g = s_pgrp[p];
-          if (g != gprev) {  // warp-uniform: planes are sorted by (r, f, t)
-            gprev = g;
-            const int f = s_grpf[g];
-            cnt = valid ? (ball & s_fm[slot * NFU + s_fslot[f]]).popc() - (fid == f ? 1 : 0) : 0;
+        uint32_t *pl = s_planes + (size_t)(NLAB + pb) * EXTW + k;
+        for (int g = gb; g < gend; g++) {  // (r, f) groups; planes sorted by (r, f, t)
+          const int f = s_grpf[g];
+          const int cnt = valid ? (ball & s_fm[slot * NFU + s_fslot[f]]).popc() - (fid == f ? 1 : 0) : 0;
+          const int p1 = s_grpoff[g + 1];
+#pragma unroll 2
+          for (int p = s_grpoff[g]; p < p1; p++) {
+            const unsigned b = __ballot_sync(FULL_MASK, cnt >= (int)s_pt[p]);
+            if (lane == 0) *pl = b;
+            pl += EXTW;
           }
-          const unsigned b = __ballot_sync(FULL_MASK, cnt >= (int)s_pt[p]);
-          const int j = p - pb;
-          if ((j & 31) == lane) mine = b;
-          if ((j & 31) == 31 || p == pe - 1)
-            if (lane <= (j & 31)) s_planes[(NLAB + pb + (j & ~31) + lane) * EXTW + k] = mine;
         }
       }
     }
@@ -689,14 +697,16 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
     for (int q = wid; q < fp.NQ; q += NWARP) {
       const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
       uint32_t Aq = 0xffffffffu;
-      for (int row = r0; row < r1; row++) {
+      uint32_t *bp = fp.bitmap + (size_t)r0 * fp.Wpad + w;
+      const uint32_t *pk = s_planes + k;
+      for (int row = r0; row < r1; row++, bp += fp.Wpad) {
         const int rl = rowlab[row];
         const int j0 = rowoff[row], j1 = rowoff[row + 1];
         uint32_t x = 0u;
         if (active) {
-          x = s_planes[rl * EXTW + k];
-          for (int j = j0; j < j1; j++) x &= s_planes[(NLAB + rowids[j]) * EXTW + k];
-          fp.bitmap[(size_t)row * fp.Wpad + w] = x;
+          x = pk[rl * EXTW];
+          for (int j = j0; j < j1; j++) x &= pk[(NLAB + rowids[j]) * EXTW];
+          *bp = x;
         }
         if (NW == 1) {
           // any-bit per segment, reported at its boundary bit (bit-reversed add)
@@ -774,7 +784,7 @@ __global__ void __launch_bounds__(kFilterThreads) k_filter(FilterParams fp) {
   // ---- write the GMCR bits and pair counts of the molecules starting here ----
   for (int mi = tid; mi < nmol; mi += NT) {
     const int g = g0 + mi;
-    if (__ldg(&goff[g]) < n0) continue;
+    if (gs + s_mstart[mi] < n0) continue;
     long long np = 0;
     for (int qb = 0; qb < fp.NQW; qb++) {
       const uint32_t bits = s_gm[mi * fp.NQW + qb];
@@ -805,6 +815,177 @@ cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStre
   }
 #undef SIGMO_FILTER_CASE
   return cudaGetLastError();
+}
+
+// ===========================================================================
+// k_support: neighbour-support refinement to the greatest fixed point
+// (BASELINE.json north_star; R9).  For every (query q, molecule g)
+// the candidate masks cm[v_q] (molecule-local) are refined by
+//   cm[v_q] &= OR_{u in cm[u_q]} adj_b[u]   for every query edge (v_q,u_q,b)
+// (v has a b-neighbour in C(u_q)  <=>  v lies in the b-neighbourhood of some
+// u in C(u_q)) until nothing changes.  The fixed point is unique, so any
+// update order gives the same bitmap; cleared bits are removed from the global
+// bitmap with atomicAnd (molecule windows share words), and the GMCR bits /
+// pair counts of the molecule are recomputed.  One CTA per group of SUPPORT_MOLS
+// molecules; one thread per (molecule, query) pair at a time.
+// ===========================================================================
+template <int NW> struct SupportCfg {
+  static constexpr int kMols = 16 / NW;        // molecules per CTA
+  static constexpr int kThreads = 256 / NW;    // threads per CTA
+};
+
+template <int NW>
+__global__ void __launch_bounds__(SupportCfg<NW>::kThreads) k_support(SupportParams sp) {
+  using M = Mask<NW>;
+  constexpr int kSupportMols = SupportCfg<NW>::kMols, kSupportThreads = SupportCfg<NW>::kThreads;
+  extern __shared__ __align__(16) unsigned char smem[];
+  const int NB = sp.NB;
+  const int ACAP = kSupportMols * 64 * NW;
+  M *s_adj = (M *)smem;                                              // [NB][ACAP]
+  M *s_cm = s_adj + (size_t)NB * ACAP;                               // [threads][maxq]
+  uint32_t *s_gm = (uint32_t *)(s_cm + (size_t)kSupportThreads * sp.maxq);  // [mols][NQW]
+  __shared__ int s_mstart[kSupportMols + 1];
+  const int tid = threadIdx.x;
+  const int g0 = blockIdx.x * kSupportMols;
+  const int g1 = min(g0 + kSupportMols, sp.ND);
+  const int nm = g1 - g0;
+  if (nm <= 0) return;
+  const int a0 = sp.goff[g0];
+  const int na = sp.goff[g1] - a0;
+  for (int i = tid; i <= nm; i += kSupportThreads) s_mstart[i] = sp.goff[g0 + i] - a0;
+  for (int i = tid; i < nm * sp.NQW; i += kSupportThreads) s_gm[i] = 0u;
+  for (int i = tid; i < na; i += kSupportThreads) {
+    const int v = a0 + i;
+    const int e0 = __ldg(&sp.roff[v]), e1 = __ldg(&sp.roff[v + 1]);
+    M m[8];
+#pragma unroll
+    for (int b = 0; b < 8; b++) m[b].clear();
+    for (int e = e0; e < e1; e++) {
+      const int x = __ldg(&sp.nbr[e]);
+      const int cls = sp.bclass[x & 255];
+#pragma unroll
+      for (int b = 0; b < 8; b++)
+        if (cls == b) m[b].set(x >> 8);
+    }
+#pragma unroll
+    for (int b = 0; b < 8; b++)
+      if (b < NB) s_adj[b * ACAP + i] = m[b];
+  }
+  __syncthreads();
+  M *cm = s_cm + (size_t)tid * sp.maxq;
+  const long long npairs = (long long)nm * sp.NQ;
+  for (long long t = tid; t < npairs; t += kSupportThreads) {
+    const int mi = (int)(t / sp.NQ), q = (int)(t % sp.NQ);
+    const int ms = s_mstart[mi], n = s_mstart[mi + 1] - ms;
+    const int qb = __ldg(&sp.qgoff[q]), nq = __ldg(&sp.qgoff[q + 1]) - qb;
+    const long long gstart = (long long)a0 + ms;
+    bool all = n > 0;
+    for (int i = 0; i < nq; i++) {
+      cm[i] = extract_window<NW>(sp.bitmap + (size_t)(qb + i) * sp.Wpad, sp.Wpad, gstart, n);
+      all = all && cm[i].any();
+    }
+    // fixed point
+    bool changed = true;
+    bool any_change = false;
+    while (changed) {
+      changed = false;
+      for (int i = 0; i < nq; i++) {
+        M c = cm[i];
+        if (!c.any()) continue;
+        const int e1 = __ldg(&sp.qroff[qb + i + 1]);
+        for (int e = __ldg(&sp.qroff[qb + i]); e < e1; e++) {
+          const int x = __ldg(&sp.qnbr[e]);
+          const int j = x >> 8, b = sp.bclass[x & 255];
+          M supp;
+          supp.clear();
+          M u = cm[j];
+          while (u.any()) {
+            const int w = u.lowest();
+            u.clear_lowest();
+            supp |= s_adj[b * ACAP + ms + w];
+          }
+          c &= supp;
+        }
+        bool diff = false;
+#pragma unroll
+        for (int k = 0; k < NW; k++) diff |= c.w[k] != cm[i].w[k];
+        if (diff) {
+          cm[i] = c;
+          changed = true;
+          any_change = true;
+        }
+      }
+    }
+    if (any_change) {
+      all = n > 0;
+      for (int i = 0; i < nq; i++) {
+        all = all && cm[i].any();
+        // clear removed bits of this molecule window in the global bitmap
+        const M orig = extract_window<NW>(sp.bitmap + (size_t)(qb + i) * sp.Wpad, sp.Wpad, gstart, n);
+#pragma unroll
+        for (int k = 0; k < NW; k++) {
+          const unsigned long long rem = orig.w[k] & ~cm[i].w[k];
+          if (!rem) continue;
+          const long long bit = gstart + 64ll * k;
+          const long long wi = bit >> 5;
+          const int sh = (int)(bit & 31);
+          uint32_t *row = sp.bitmap + (size_t)(qb + i) * sp.Wpad;
+          const unsigned long long lo = rem << sh;
+          const uint32_t r0 = (uint32_t)lo, r1 = (uint32_t)(lo >> 32);
+          const uint32_t r2 = sh ? (uint32_t)(rem >> (64 - sh)) : 0u;
+          if (r0) atomicAnd(&row[wi], ~r0);
+          if (r1) atomicAnd(&row[wi + 1], ~r1);
+          if (r2) atomicAnd(&row[wi + 2], ~r2);
+        }
+      }
+    }
+    if (all) atomicOr(&s_gm[mi * sp.NQW + (q >> 5)], 1u << (q & 31));
+  }
+  __syncthreads();
+  for (int mi = tid; mi < nm; mi += kSupportThreads) {
+    long long np = 0;
+    for (int qb = 0; qb < sp.NQW; qb++) {
+      const uint32_t bits = s_gm[mi * sp.NQW + qb];
+      sp.gm[(size_t)(g0 + mi) * sp.NQW + qb] = bits;
+      np += __popc(bits);
+    }
+    I64x2 v;
+    v.a = np;
+    v.b = 0;
+    sp.mol_cnt[g0 + mi] = v;
+  }
+}
+
+template <int NW>
+static size_t support_smem_t(int NB, int maxq, int NQW) {
+  constexpr int mols = SupportCfg<NW>::kMols, thr = SupportCfg<NW>::kThreads;
+  return (size_t)8 * NW * ((size_t)NB * mols * 64 * NW + (size_t)thr * maxq) + 4 * (size_t)mols * NQW;
+}
+
+size_t support_smem_bytes(int NW, int NB, int maxq, int NQW) {
+  return NW == 1 ? support_smem_t<1>(NB, maxq, NQW) : NW == 2 ? support_smem_t<2>(NB, maxq, NQW)
+                                                              : support_smem_t<4>(NB, maxq, NQW);
+}
+
+template <int NW>
+static cudaError_t launch_support_t(const SupportParams &p, cudaStream_t st) {
+  constexpr int mols = SupportCfg<NW>::kMols, thr = SupportCfg<NW>::kThreads;
+  const int grid = (p.ND + mols - 1) / mols;
+  if (grid <= 0) return cudaSuccess;
+  const size_t smem = support_smem_t<NW>(p.NB, p.maxq, p.NQW);
+  cudaError_t e = cudaFuncSetAttribute(k_support<NW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  k_support<NW><<<grid, thr, smem, st>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_support(int NW, const SupportParams &p, cudaStream_t st) {
+  switch (NW) {
+    case 1: return launch_support_t<1>(p, st);
+    case 2: return launch_support_t<2>(p, st);
+    case 4: return launch_support_t<4>(p, st);
+    default: return cudaErrorInvalidValue;
+  }
 }
 
 // ===========================================================================

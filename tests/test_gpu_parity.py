@@ -249,3 +249,36 @@ def test_shard_additivity_gpu(sigmo):
             c.join(sigmo.SIGMO_FIND_ALL)
             acc += c.query_totals()
         assert np.array_equal(acc, ref)
+
+
+@pytest.mark.parametrize("levels", [1, 2, 4])
+def test_neighbour_support_bitmap_and_counts(ctx, sigmo, levels):
+    """SIGMO_FILTER_NEIGHBOR_SUPPORT: bitmap = the greatest fixed point of the
+    CPU reference, GMCR pairs = reference GMCR of that bitmap, counts unchanged."""
+    Q, D = synth.config_queries(1), synth.config_data(1)
+    ctx.load_batch(Q, D)
+    ctx.filter(levels, neighbor_support=True)
+    Cb = fr.neighbour_support(Q, D, fr.candidates_bool(Q, D, levels))
+    assert np.array_equal(ctx.candidates(), fr.to_bitmap(Cb))
+    assert ctx.num_pairs() == int(fr.gmcr(Q, D, Cb).sum())
+    ctx.join(sigmo.SIGMO_FIND_ALL)
+    assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D))
+    ctx.join(sigmo.SIGMO_FIND_FIRST)
+    assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D, oracle.FIND_FIRST))
+
+
+def test_neighbour_support_edge_cases(ctx, sigmo):
+    mols = synth.molecules(synth.DATA_SEED_BASE + 78, 0, 60, mode=2)
+    graphs = mols.graphs()
+    graphs.insert(3, ([], []))
+    graphs.insert(7, ([6], []))
+    graphs.append(([6] * 80, [(i, i + 1, 1) for i in range(79)]))
+    D = GraphBatch.from_graphs(graphs)
+    qs = synth.library(synth.C1_NAMES) + [([6], []), ([6, 8], []), path(5), ring(6, 6, 4)]
+    Q = GraphBatch.from_graphs(qs)
+    ctx.load_batch(Q, D)
+    ctx.filter(3, neighbor_support=True)
+    Cb = fr.neighbour_support(Q, D, fr.candidates_bool(Q, D, 3))
+    assert np.array_equal(ctx.candidates(), fr.to_bitmap(Cb))
+    ctx.join(sigmo.SIGMO_FIND_ALL)
+    assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D))
