@@ -56,7 +56,7 @@ struct Timing {
 
 struct ProgCache {
   QueryProg prog;
-  DBuf buf;
+  DBuf buf, pack;  // device program arrays; packed form for k_filter
   bool valid = false;
 };
 
@@ -307,8 +307,7 @@ struct Layout {
 };
 
 struct PackedOffsets {
-  size_t goff, label, local, roff, nbr, adj64;
-  bool has_adj64;
+  size_t goff, label, local, roff, nbr;
 };
 
 PackedOffsets plan_graphs(Layout &L, const HostGraphs &h) {
@@ -318,10 +317,6 @@ PackedOffsets plan_graphs(Layout &L, const HostGraphs &h) {
   p.local = L.take((size_t)h.V);
   p.roff = L.take(4 * (size_t)(h.V + 1));
   p.nbr = L.take(2 * (size_t)h.E);
-  int64_t mx = 0;
-  for (int64_t g = 0; g < h.G; g++) mx = std::max<int64_t>(mx, h.goff[g + 1] - h.goff[g]);
-  p.has_adj64 = mx <= 64;
-  p.adj64 = p.has_adj64 ? L.take(8 * (size_t)h.V) : 0;
   return p;
 }
 
@@ -331,7 +326,6 @@ void pack_graphs(unsigned char *base, const PackedOffsets &p, const HostGraphs &
   uint8_t *local = base + p.local;
   int32_t *roff = (int32_t *)(base + p.roff);
   uint16_t *nbr = (uint16_t *)(base + p.nbr);
-  uint64_t *adj64 = p.has_adj64 ? (uint64_t *)(base + p.adj64) : nullptr;
   goff[h.G] = (int32_t)h.V;
   roff[h.V] = (int32_t)h.E;
   parallel_for_graphs(h.G, h.E + h.V, [&](int, int64_t ga, int64_t gb) {
@@ -342,12 +336,7 @@ void pack_graphs(unsigned char *base, const PackedOffsets &p, const HostGraphs &
         label[u] = h.nlab[u];
         local[u] = (uint8_t)(u - lo);
         roff[u] = (int32_t)h.roff[u];
-        uint64_t m = 0;
-        for (int64_t e = h.roff[u]; e < h.roff[u + 1]; e++) {
-          nbr[e] = (uint16_t)(((h.col[e] - lo) << 8) | h.elab[e]);
-          m |= 1ull << ((h.col[e] - lo) & 63);
-        }
-        if (adj64) adj64[u] = m;
+        for (int64_t e = h.roff[u]; e < h.roff[u + 1]; e++) nbr[e] = (uint16_t)(((h.col[e] - lo) << 8) | h.elab[e]);
       }
     }
   });
@@ -365,7 +354,6 @@ DevGraphs dev_view(unsigned char *dbase, const PackedOffsets &p, const HostGraph
   d.local = dbase + p.local;
   d.roff = (const int32_t *)(dbase + p.roff);
   d.nbr = (const uint16_t *)(dbase + p.nbr);
-  d.adj64 = p.has_adj64 ? (const unsigned long long *)(dbase + p.adj64) : nullptr;
   return d;
 }
 
@@ -522,6 +510,122 @@ void timing_join(sigmo_ctx *c, int k) {
 // ---------------------------------------------------------------------------
 constexpr int kMaxPlanes = kMaxRadius * kNumFields * 256;  // 49920 keys
 
+// Host packing of the plane program for k_filter (see GroupRec): planes are
+// numbered p = 0..P-1 in (radius, field, threshold) order and grouped in
+// batches of 32; each (radius, field) group contributes one record per batch
+// it touches, whose table maps a count c to the bits of its planes with
+// t_p <= c.  Row programs list channel byte offsets, label channel first,
+// padded with the all-ones channel to whole 32-bit words.
+sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
+  QueryProg &P = pc.prog;
+  const QueryProgMeta &m = P.meta;
+  const int VQ = c->VQ, NP = m.P, G = m.G, NLAB = m.NLAB;
+  const int RE = m.row_entries;
+  std::vector<uint8_t> p_t((size_t)NP + 1), grp_f((size_t)G + 1), row_lab((size_t)VQ + 1);
+  std::vector<int16_t> grp_poff((size_t)G + 1), rg_off((size_t)R + 1);
+  std::vector<int8_t> fslot(kNumFields);
+  std::vector<int32_t> row_off((size_t)VQ + 1);
+  std::vector<uint16_t> row_ids((size_t)RE + 1);
+  cudaStream_t st = c->stream;
+  if (NP) CUDA_TRY(c, cudaMemcpyAsync(p_t.data(), P.p_t, NP, cudaMemcpyDeviceToHost, st));
+  if (G) CUDA_TRY(c, cudaMemcpyAsync(grp_f.data(), P.grp_f, G, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(c, cudaMemcpyAsync(grp_poff.data(), P.grp_poff, 2 * ((size_t)G + 1), cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(c, cudaMemcpyAsync(rg_off.data(), P.rg_off, 2 * ((size_t)R + 1), cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(c, cudaMemcpyAsync(fslot.data(), P.fslot, kNumFields, cudaMemcpyDeviceToHost, st));
+  if (VQ) CUDA_TRY(c, cudaMemcpyAsync(row_lab.data(), P.row_lab, VQ, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(c, cudaMemcpyAsync(row_off.data(), P.row_off, 4 * ((size_t)VQ + 1), cudaMemcpyDeviceToHost, st));
+  if (RE) CUDA_TRY(c, cudaMemcpyAsync(row_ids.data(), P.row_ids, 2 * (size_t)RE, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(c, cudaStreamSynchronize(st));
+  const int TS = c->NW == 1 ? 64 : 256;  // counts exclude the node: <= 63 in <= 64-node graphs
+  std::vector<GroupRec> rec;
+  std::vector<uint32_t> tab;
+  std::vector<int32_t> rrec((size_t)R + 1, 0), rcarry((size_t)R + 1, 0);
+  const int NBATCH = (NP + 31) / 32;
+  std::vector<int32_t> bdone((size_t)NBATCH + 1, 0);
+  for (int r0 = 0; r0 < R; r0++) {
+    rrec[r0] = (int)rec.size();
+    const int g0 = rg_off[r0], g1 = rg_off[r0 + 1];
+    if (g0 < g1) rcarry[r0] = (grp_poff[g0] % 32) != 0;
+    for (int g = g0; g < g1; g++) {
+      for (int p = grp_poff[g]; p < grp_poff[g + 1];) {
+        const int b = p / 32;
+        const int e = std::min<int>(grp_poff[g + 1], 32 * (b + 1));
+        GroupRec r{};
+        r.fslot = fslot[grp_f[g]];
+        r.toff = (int)tab.size();
+        r.batch = b;
+        rec.push_back(r);
+        for (int cc = 0; cc < TS; cc++) {
+          uint32_t bits = 0;
+          for (int q = p; q < e; q++)
+            if ((int)p_t[q] <= cc) bits |= 1u << (q % 32);
+          tab.push_back(bits);
+        }
+        for (int q = p; q < e; q++) bdone[q / 32] = r0;  // radius of the batch's last plane (planes ascend)
+        p = e;
+      }
+    }
+  }
+  rrec[R] = (int)rec.size();
+  // row programs: every row padded to RW words (the longest row) with
+  // all-ones channel pairs, so k_filter's row loop has a fixed trip count
+  std::vector<std::vector<int>> chans((size_t)VQ);
+  int RW = 1;
+  for (int v = 0; v < VQ; v++) {
+    std::vector<int> &ch = chans[v];
+    ch.push_back(row_lab[v]);
+    for (int j = row_off[v]; j < row_off[v + 1]; j++) ch.push_back(NLAB + 1 + row_ids[j]);
+    RW = std::max<int>(RW, (int)(ch.size() + 1) / 2);
+  }
+  if (4 * (NLAB + 1 + NP) > 0xffff) return set_err(c, SIGMO_ERR_LIMIT, "plane program too large (%d planes)", NP);
+  std::vector<int32_t> rowp_off((size_t)VQ + 1, 0);
+  std::vector<uint32_t> rowp((size_t)VQ * RW, (uint32_t)(4 * NLAB) | ((uint32_t)(4 * NLAB) << 16));
+  for (int v = 0; v < VQ; v++) {
+    rowp_off[v] = v * RW;
+    const std::vector<int> &ch = chans[v];
+    for (size_t j = 0; j < ch.size(); j += 2) {
+      const int hi = j + 1 < ch.size() ? ch[j + 1] : NLAB;
+      rowp[(size_t)v * RW + j / 2] = (uint32_t)(4 * ch[j]) | ((uint32_t)(4 * hi) << 16);
+    }
+  }
+  rowp_off[VQ] = VQ * RW;
+  // upload
+  Layout L;
+  const size_t o_rec = L.take(sizeof(GroupRec) * (rec.size() + 1));
+  const size_t o_tab = L.take(4 * (tab.size() + 4));
+  const size_t o_rr = L.take(4 * rrec.size());
+  const size_t o_rc = L.take(4 * rcarry.size());
+  const size_t o_bd = L.take(4 * bdone.size());
+  const size_t o_po = L.take(4 * rowp_off.size());
+  const size_t o_rp = L.take(4 * (rowp.size() + 1));
+  std::vector<unsigned char> hb(L.off, 0);
+  auto put = [&](size_t o, const void *src, size_t n) { if (n) memcpy(hb.data() + o, src, n); };
+  put(o_rec, rec.data(), sizeof(GroupRec) * rec.size());
+  put(o_tab, tab.data(), 4 * tab.size());
+  put(o_rr, rrec.data(), 4 * rrec.size());
+  put(o_rc, rcarry.data(), 4 * rcarry.size());
+  put(o_bd, bdone.data(), 4 * bdone.size());
+  put(o_po, rowp_off.data(), 4 * rowp_off.size());
+  put(o_rp, rowp.data(), 4 * rowp.size());
+  SIGMO_TRY(dreserve(c, pc.pack, L.off, "packed query program"));
+  unsigned char *db = (unsigned char *)pc.pack.p;
+  CUDA_TRY(c, cudaMemcpyAsync(db, hb.data(), L.off, cudaMemcpyHostToDevice, st));
+  CUDA_TRY(c, cudaStreamSynchronize(st));  // hb is pageable and goes out of scope
+  P.grec = (GroupRec *)(db + o_rec);
+  P.tab = (uint32_t *)(db + o_tab);
+  P.rrec_off = (int32_t *)(db + o_rr);
+  P.rcarry = (int32_t *)(db + o_rc);
+  P.bdone = (int32_t *)(db + o_bd);
+  P.rowp_off = (int32_t *)(db + o_po);
+  P.rowp = (uint32_t *)(db + o_rp);
+  P.meta.NREC = (int)rec.size();
+  P.meta.NRP = (int)rowp.size();
+  P.meta.RW = RW;
+  P.meta.NBATCH = NBATCH;
+  P.meta.TS = TS;
+  return SIGMO_OK;
+}
+
 sigmo_status ensure_prog(sigmo_ctx *c, int R, QueryProg *&out) {
   auto it = c->progs.find(R);
   if (it != c->progs.end() && it->second.valid) {
@@ -566,6 +670,7 @@ sigmo_status ensure_prog(sigmo_ctx *c, int R, QueryProg *&out) {
   CUDA_TRY(c, cudaMemcpyAsync(&P.meta, P.d_meta, sizeof(QueryProgMeta), cudaMemcpyDeviceToHost, c->stream));
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
   if (P.meta.err) return set_err(c, SIGMO_ERR_LIMIT, "query program error %d", P.meta.err);
+  SIGMO_TRY(pack_prog(c, R, pc));
   pc.valid = true;
   out = &P;
   return SIGMO_OK;
@@ -594,7 +699,10 @@ void tile_geometry(sigmo_ctx *c, const HostGraphs &d) {
 }
 
 void free_all(sigmo_ctx *c) {
-  for (auto &kv : c->progs) dfree(c, kv.second.buf);
+  for (auto &kv : c->progs) {
+    dfree(c, kv.second.buf);
+    dfree(c, kv.second.pack);
+  }
   c->progs.clear();
   DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
                   &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_result, &c->jcnt, &c->sig_tmp, &c->gstack};
@@ -920,7 +1028,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       rows_smem = k < 6 ? 1 : 0;
       const int kk = k % 6;
       smem = filter_smem_bytes(c->NW, c->tile_extn[kk], c->tile_extw[kk], c->tile_molcap[kk], m.NFU, m.NLAB, m.P,
-                               m.G, c->VQ, m.row_entries, rows_smem, c->NQW);
+                               m.NREC, c->VQ, m.NRP, rows_smem, c->NQW, m.TS);
       // prefer >= 2 CTAs per SM with row programs in shared memory
       if (smem <= (rows_smem ? c->max_smem / 2 : c->max_smem)) break;
     }
@@ -936,18 +1044,22 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.NQW = c->NQW;
     fp.R = R;
     fp.P = m.P;
-    fp.G = m.G;
     fp.NFU = m.NFU;
     fp.NLAB = m.NLAB;
-    fp.p_t = prog->p_t;
-    fp.grp_poff = prog->grp_poff;
-    fp.grp_f = prog->grp_f;
-    fp.rg_off = prog->rg_off;
+    fp.NREC = m.NREC;
+    fp.NRP = m.NRP;
+    fp.NBATCH = m.NBATCH;
+    fp.RW = m.RW;
+    fp.TS = m.TS;
+    fp.grec = prog->grec;
+    fp.rrec_off = prog->rrec_off;
+    fp.rcarry = prog->rcarry;
+    fp.bdone = prog->bdone;
+    fp.tab = prog->tab;
     fp.fslot = prog->fslot;
     fp.lab_val = prog->lab_val;
-    fp.row_lab = prog->row_lab;
-    fp.row_off = prog->row_off;
-    fp.row_ids = prog->row_ids;
+    fp.rowp_off = prog->rowp_off;
+    fp.rowp = prog->rowp;
     fp.qgoff = c->dq.goff;
     fp.bitmap = (uint32_t *)c->bitmap.p;
     fp.gm = (uint32_t *)c->gm.p;
@@ -955,7 +1067,6 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.EXTN = c->tile_extn[k];
     fp.EXTW = c->tile_extw[k];
     fp.MOLCAP = c->tile_molcap[k];
-    fp.RE = m.row_entries;
     fp.tile_g0 = tws[k] == 32 ? c->tile_g0 : nullptr;
     fp.tile_g1 = tws[k] == 32 ? c->tile_g1 : nullptr;
     fp.rows_smem = rows_smem;

@@ -5,6 +5,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <vector>
+
 namespace sigmo {
 
 constexpr int kNumFields = 13;   // R7 field table (see sigmo_kernels.cu kFieldWidth)
@@ -26,7 +28,6 @@ struct DevGraphs {
   const uint8_t *local = nullptr;  // [V] index of the node inside its graph
   const int32_t *roff = nullptr;   // [V+1]
   const uint16_t *nbr = nullptr;   // [E2]
-  const unsigned long long *adj64 = nullptr;  // [V] molecule-local adjacency mask (all graphs <= 64 nodes), else null
 };
 
 // Query-side plane program, built on the device by k_query_prep from the
@@ -38,6 +39,19 @@ struct QueryProgMeta {
   int NLAB;    // distinct query labels (label planes)
   int row_entries;
   int err;
+  int NREC;    // group records (one per group part per 32-plane batch)
+  int NRP;     // packed row-program words (two 16-bit channels each)
+  int NBATCH;  // 32-plane batches
+  int TS;      // threshold-table entries per record (64, or 256 for > 64-node graphs)
+  int RW;      // row-program words per query node (padded)
+};
+
+// One part of a (radius, field) count group inside one 32-plane batch of the
+// plane program, used by k_filter: with c = |ball_r(v) \ {v}| restricted to
+// field `fslot`, tab[toff + min(c, TS-1)] holds the bits (plane % 32) of the
+// batch's planes [c >= t] of this group (a thermometer code).
+struct __align__(16) GroupRec {
+  int fslot, toff, batch, pad;
 };
 
 struct QueryProg {
@@ -53,6 +67,15 @@ struct QueryProg {
   uint8_t *row_lab = nullptr;  // [VQ]  label-plane index of query node
   int32_t *row_off = nullptr;  // [VQ+1]
   uint16_t *row_ids = nullptr; // plane ids per query node
+  // packed form used by k_filter (built on the host from the arrays above).
+  // Channels: 0..NLAB-1 label planes, NLAB all ones, NLAB+1+p constraint plane p.
+  GroupRec *grec = nullptr;    // [NREC] sorted by (radius, batch)
+  int32_t *rrec_off = nullptr; // [R+1] record range per radius
+  int32_t *rcarry = nullptr;   // [R] 1 if the radius' first plane continues a batch of the previous radius
+  int32_t *bdone = nullptr;    // [NBATCH] radius index (r-1) of the batch's last plane
+  uint32_t *tab = nullptr;     // [NREC * TS] thermometer tables
+  int32_t *rowp_off = nullptr; // [VQ+1] row-program word range per query node
+  uint32_t *rowp = nullptr;    // [NRP] channel byte offsets (lo | hi << 16), label channel first
   QueryProgMeta *d_meta = nullptr;
 };
 
@@ -61,22 +84,22 @@ struct FilterParams {
   int TW, W, Wpad;
   int VQ, NQ, NQW;
   int R;
-  int P, G, NFU, NLAB;
-  const uint8_t *p_t;
-  const int16_t *grp_poff;
-  const uint8_t *grp_f;
-  const int16_t *rg_off;
+  int P, NFU, NLAB, NREC, NRP, NBATCH, TS, RW;
+  const GroupRec *grec;
+  const int32_t *rrec_off;
+  const int32_t *rcarry;
+  const int32_t *bdone;
+  const uint32_t *tab;
   const int8_t *fslot;
   const uint8_t *lab_val;
-  const uint8_t *row_lab;
-  const int32_t *row_off;
-  const uint16_t *row_ids;
+  const int32_t *rowp_off;
+  const uint32_t *rowp;
   const int32_t *qgoff;        // [NQ+1] query node offsets (rows)
   uint32_t *bitmap;            // [VQ][Wpad]
   uint32_t *gm;                // [ND][NQW] surviving-query bits per data graph
   I64x2 *mol_cnt;              // [ND+1] (surviving pairs, candidate-mask entries)
   int EXTN, EXTW, MOLCAP;
-  int RE, rows_smem;           // row-program entries; 1 = copy row programs to smem
+  int rows_smem;               // 1 = copy row programs to smem
   const int32_t *tile_g0, *tile_g1;  // per-tile graph range for TW = 32 (null: binary search)
   size_t smem_bytes;
 };
@@ -138,8 +161,8 @@ cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *
 cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts, QueryProg &prog,
                               cudaStream_t st);
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
-size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int G, int VQ, int RE,
-                         int rows_smem, int NQW);
+size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ,
+                         int NRP, int rows_smem, int NQW, int TS);
 cudaError_t launch_support(int NW, const SupportParams &p, cudaStream_t st);
 size_t support_smem_bytes(int NW, int NB, int maxq, int NQW);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);

@@ -22,6 +22,8 @@
 //                  per-CTA queue, per-query totals reduced in smem.
 #include <cub/cub.cuh>
 
+#include <type_traits>
+
 #include "sigmo_internal.h"
 
 namespace sigmo {
@@ -424,95 +426,138 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
 
 // ===========================================================================
 // k_filter: one CTA per tile of TW (<= 32) bitmap words = 32*TW data nodes.
+// Plane words are stored word-major (s_pl[k * PS + channel], PS odd), so the
+// rows phase (lane = word) reads them without bank conflicts and the plane
+// phase (warp = word) writes them with immediate offsets.
 // ===========================================================================
 struct FilterSmem {
-  size_t adj, ballA, ballB, fm, planes, fplanes, win, nz, gmb, slotat, bnd, own, molstart, molslot, fid, lab, mstart,
-      sos, rowlab, rowoff, rowids, prog, total;
+  size_t nb, ballA, ballB, fm, pl, fpl, memb, win, nz, gmb, slotat, endb, own, molstart, molslot, loc, fid, lab, mstart,
+      sos, grec, tab, bdone, rowpoff, rowp, total;
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
-
-// prog block: p_t[P] u8 | p_grp[P] u8 | grp_f[G] u8 | fslot[16] i8 | grp_poff[G+1] i16 | rg_off[16] i16
-__host__ __device__ inline size_t prog_bytes(int P, int G) {
-  return 2 * align16((size_t)P) + align16((size_t)G) + 16 + align16(2 * (size_t)(G + 1)) + 32;
-}
+__host__ __device__ inline int plane_stride(int NLAB, int P) { return (NLAB + 1 + P) | 1; }
 
 __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB,
-                                                    int P, int G, int VQ, int RE, int rows_smem, int NQW) {
+                                                    int P, int NREC, int VQ, int NRP, int rows_smem, int NQW,
+                                                    int TS) {
   FilterSmem L;
   const size_t mb = 8 * (size_t)NW;
   const int NWARP = kFilterThreads / 32;
   const int VQW = (VQ + 31) / 32;
+  const int NCH = NLAB + 1 + P;
   size_t o = 0;
-  L.adj = o;      o = align16(o + mb * EXTN);
+  L.nb = o;       o = align16(o + 4 * (size_t)EXTN);
   L.ballA = o;    o = align16(o + mb * EXTN);
-  L.ballB = o;    o = align16(o + mb * EXTN);
+  L.ballB = o;    o = align16(o + (NW == 1 ? 0 : mb * EXTN));  // NW == 1: in-place BFS via registers
   L.fm = o;       o = align16(o + mb * (size_t)MOLCAP * (NFU > 0 ? NFU : 1));
-  L.planes = o;   o = align16(o + 4 * (size_t)(NLAB + P) * EXTW);
-  L.fplanes = o;  o = align16(o + 4 * (size_t)(NFU > 0 ? NFU : 1) * EXTW);
-  L.win = o;      o = align16(o + mb * (size_t)NWARP * (NLAB + P));
+  L.pl = o;       o = align16(o + 4 * (size_t)plane_stride(NLAB, P) * EXTW);
+  L.fpl = o;      o = align16(o + 4 * (size_t)(NFU > 0 ? NFU : 1) * EXTW);
+  L.memb = o;     o = align16(o + 4 * 32 * (size_t)EXTW);
+  L.win = o;      o = align16(o + mb * (size_t)NWARP * NCH);
   L.nz = o;       o = align16(o + 4 * (size_t)NWARP * (VQW + 1));
   L.gmb = o;      o = align16(o + 4 * (size_t)MOLCAP * (NQW > 0 ? NQW : 1));
   L.slotat = o;   o = align16(o + 2 * 32 * 32);
-  L.bnd = o;      o = align16(o + 4 * 32);
+  L.endb = o;     o = align16(o + 4 * 32);
   L.own = o;      o = align16(o + 4 * 32);
   L.molstart = o; o = align16(o + 2 * (size_t)EXTN);
   L.molslot = o;  o = align16(o + 2 * (size_t)EXTN);
+  L.loc = o;      o = align16(o + (size_t)EXTN);
   L.fid = o;      o = align16(o + (size_t)EXTN);
   L.lab = o;      o = align16(o + (size_t)EXTN);
   L.mstart = o;   o = align16(o + 4 * (size_t)(MOLCAP + 1));
   L.sos = o;      o = align16(o + 2 * (size_t)EXTN);
-  L.rowlab = o;   o = align16(o + (rows_smem ? (size_t)VQ : 0));
-  L.rowoff = o;   o = align16(o + (rows_smem ? 4 * (size_t)(VQ + 1) : 0));
-  L.rowids = o;   o = align16(o + (rows_smem ? 2 * (size_t)RE : 0));
-  L.prog = o;     o = align16(o + prog_bytes(P, G));
+  L.grec = o;     o = align16(o + sizeof(GroupRec) * (size_t)(NREC > 0 ? NREC : 1));
+  L.tab = o;      o = align16(o + 4 * (size_t)TS * (NREC > 0 ? NREC : 1));
+  L.bdone = o;    o = align16(o + (size_t)(P / 32 + 1));
+  L.rowpoff = o;  o = align16(o + (rows_smem ? 4 * (size_t)(VQ + 1) : 0));
+  L.rowp = o;     o = align16(o + (rows_smem ? 4 * (size_t)NRP : 0));
   L.total = o;
   return L;
 }
 
-size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int G, int VQ, int RE,
-                         int rows_smem, int NQW) {
-  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, G, VQ, RE, rows_smem, NQW).total;
+size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ, int NRP,
+                         int rows_smem, int NQW, int TS) {
+  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, NREC, VQ, NRP, rows_smem, NQW, TS).total;
+}
+
+// 32x32 bit-matrix transpose across the warp: lane L holds row L (bit p =
+// element (L, p)); returns column `lane` (bit L = element (L, lane)).  Each of
+// the five stages exchanges bit j of the row index with bit j of the column
+// index.
+__device__ __forceinline__ uint32_t transpose32(uint32_t x, int lane) {
+#pragma unroll
+  for (int j = 16; j >= 1; j >>= 1) {
+    const uint32_t m = j == 16 ? 0x0000ffffu : j == 8 ? 0x00ff00ffu : j == 4 ? 0x0f0f0f0fu : j == 2 ? 0x33333333u
+                                                                                                     : 0x55555555u;
+    const uint32_t sw = ((x << j) & ~m) | ((x >> j) & m);
+    const uint32_t y = __shfl_xor_sync(FULL_MASK, sw, j);
+    const uint32_t K = (lane & j) ? ~m : m;
+    x = (x & K) | (y & ~K);
+  }
+  return x;
+}
+
+// extract_window over one channel of the word-major plane array
+template <int NW>
+__device__ __forceinline__ Mask<NW> extract_window_strided(const uint32_t *words, int stride, long long nw,
+                                                           long long s, int n) {
+  Mask<NW> m;
+#pragma unroll
+  for (int k = 0; k < NW; k++) {
+    long long b = s + 64ll * k;
+    long long wi = b >> 5;
+    int sh = (int)(b & 31);
+    unsigned long long w0 = (wi < nw) ? words[wi * stride] : 0u;
+    unsigned long long w1 = (wi + 1 < nw) ? words[(wi + 1) * stride] : 0u;
+    unsigned long long w2 = (wi + 2 < nw) ? words[(wi + 2) * stride] : 0u;
+    unsigned long long x = (w0 | (w1 << 32)) >> sh;
+    if (sh) x |= w2 << (64 - sh);
+    int rem = n - 64 * k;
+    if (rem <= 0) x = 0ull;
+    else if (rem < 64) x &= (1ull << rem) - 1ull;
+    m.w[k] = x;
+  }
+  return m;
 }
 
 template <int NW>
-__global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
+__global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_constant__ FilterParams fp) {
   using M = Mask<NW>;
   constexpr int NT = kFilterThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
-  const FilterSmem L = filter_layout(NW, fp.EXTN, fp.EXTW, fp.MOLCAP, fp.NFU, fp.NLAB, fp.P, fp.G, fp.VQ, fp.RE,
-                                     fp.rows_smem, fp.NQW);
-  M *s_adj = (M *)(smem + L.adj);
+  const FilterSmem L = filter_layout(NW, fp.EXTN, fp.EXTW, fp.MOLCAP, fp.NFU, fp.NLAB, fp.P, fp.NREC, fp.VQ, fp.NRP,
+                                     fp.rows_smem, fp.NQW, fp.TS);
+  uint32_t *s_nb = (uint32_t *)(smem + L.nb);
   M *s_cur = (M *)(smem + L.ballA);
   M *s_nxt = (M *)(smem + L.ballB);
   M *s_fm = (M *)(smem + L.fm);
-  uint32_t *s_planes = (uint32_t *)(smem + L.planes);
-  uint32_t *s_fplanes = (uint32_t *)(smem + L.fplanes);
+  uint32_t *s_pl = (uint32_t *)(smem + L.pl);
+  uint32_t *s_fpl = (uint32_t *)(smem + L.fpl);
+  uint32_t *s_memb = (uint32_t *)(smem + L.memb);
   M *s_win = (M *)(smem + L.win);
   uint32_t *s_nz = (uint32_t *)(smem + L.nz);
   uint32_t *s_gm = (uint32_t *)(smem + L.gmb);
   int16_t *s_slotat = (int16_t *)(smem + L.slotat);
-  uint32_t *s_bnd = (uint32_t *)(smem + L.bnd);
+  uint32_t *s_endb = (uint32_t *)(smem + L.endb);
   uint32_t *s_own = (uint32_t *)(smem + L.own);
   int16_t *s_molstart = (int16_t *)(smem + L.molstart);
   int16_t *s_molslot = (int16_t *)(smem + L.molslot);
+  uint8_t *s_loc = smem + L.loc;
   uint8_t *s_fid = smem + L.fid;
   uint8_t *s_lab = smem + L.lab;
   int *s_mstart = (int *)(smem + L.mstart);
   int16_t *s_sos = (int16_t *)(smem + L.sos);
-  // plane program (always in smem)
-  uint8_t *s_pt = smem + L.prog;
-  uint8_t *s_pgrp = s_pt + align16(fp.P);
-  uint8_t *s_grpf = s_pgrp + align16(fp.P);
-  int8_t *s_fslot = (int8_t *)(s_grpf + align16(fp.G));
-  int16_t *s_grpoff = (int16_t *)(s_fslot + 16);
-  int16_t *s_rg = (int16_t *)((unsigned char *)s_grpoff + align16(2 * (size_t)(fp.G + 1)));
-  // row programs: shared-memory copy when it fits, else global
-  const uint8_t *rowlab = fp.row_lab;
-  const int32_t *rowoff = fp.row_off;
-  const uint16_t *rowids = fp.row_ids;
+  GroupRec *s_grec = (GroupRec *)(smem + L.grec);
+  uint32_t *s_tab = (uint32_t *)(smem + L.tab);
+  uint8_t *s_bdone = smem + L.bdone;
   __shared__ int s_g0, s_g1, s_strad;
+  __shared__ int s_rrec[kMaxRadius + 1];
+  __shared__ int s_rcarry[kMaxRadius];
   __shared__ uint8_t s_fused[kNumFields];
+  __shared__ int8_t s_fslot[kNumFields];
+  __shared__ uint8_t s_labval[256];
+  __shared__ uint8_t s_labch[256];
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int ND = fp.D.num_graphs, VD = fp.D.num_nodes;
@@ -521,6 +566,8 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
   const int n0 = w0 * 32;
   const int n1 = min(n0 + fp.TW * 32, VD);
   const int32_t *goff = fp.D.goff;
+  const int NLAB = fp.NLAB, NFU = fp.NFU, EXTW = fp.EXTW;
+  const int PS = plane_stride(NLAB, fp.P);
   if (tid == 0) {
     if (fp.tile_g0) {
       s_g0 = __ldg(&fp.tile_g0[blockIdx.x]);
@@ -531,30 +578,31 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
     }
     s_strad = -1;
   }
-  for (int i = tid; i < fp.P; i += NT) s_pt[i] = fp.p_t[i];
-  for (int i = tid; i < fp.G; i += NT) {
-    s_grpf[i] = fp.grp_f[i];
-    for (int p = fp.grp_poff[i]; p < fp.grp_poff[i + 1]; p++) s_pgrp[p] = (uint8_t)i;
+  {
+    const int4 *src = (const int4 *)fp.grec;
+    int4 *dst = (int4 *)s_grec;
+    for (int i = tid; i < fp.NREC; i += NT) dst[i] = __ldg(&src[i]);
+    const uint4 *ts = (const uint4 *)fp.tab;
+    uint4 *td = (uint4 *)s_tab;
+    for (int i = tid; i < fp.NREC * fp.TS / 4; i += NT) td[i] = __ldg(&ts[i]);
   }
-  for (int i = tid; i <= fp.G; i += NT) s_grpoff[i] = fp.grp_poff[i];
-  for (int i = tid; i <= fp.R; i += NT) s_rg[i] = fp.rg_off[i];
+  for (int i = tid; i < fp.NBATCH; i += NT) s_bdone[i] = (uint8_t)fp.bdone[i];
+  for (int i = tid; i <= fp.R; i += NT) s_rrec[i] = fp.rrec_off[i];
+  for (int i = tid; i < fp.R; i += NT) s_rcarry[i] = fp.rcarry[i];
+  for (int i = tid; i < 256; i += NT) s_labch[i] = 0xff;
+  for (int i = tid; i < NLAB; i += NT) s_labval[i] = fp.lab_val[i];
   for (int i = tid; i < kNumFields; i += NT) {
     s_fslot[i] = fp.fslot[i];
     if (fp.fslot[i] >= 0) s_fused[fp.fslot[i]] = (uint8_t)i;
   }
   if (fp.rows_smem) {
-    uint8_t *a = smem + L.rowlab;
-    int32_t *b = (int32_t *)(smem + L.rowoff);
-    uint16_t *c = (uint16_t *)(smem + L.rowids);
-    for (int i = tid; i < fp.VQ; i += NT) a[i] = fp.row_lab[i];
-    for (int i = tid; i <= fp.VQ; i += NT) b[i] = fp.row_off[i];
-    for (int i = tid; i < fp.RE; i += NT) c[i] = fp.row_ids[i];
-    rowlab = a;
-    rowoff = b;
-    rowids = c;
+    int32_t *b = (int32_t *)(smem + L.rowpoff);
+    uint32_t *c = (uint32_t *)(smem + L.rowp);
+    for (int i = tid; i <= fp.VQ; i += NT) b[i] = fp.rowp_off[i];
+    for (int i = tid; i < fp.NRP; i += NT) c[i] = fp.rowp[i];
   }
   if (tid < 32) {
-    s_bnd[tid] = 0u;
+    s_endb[tid] = 0u;
     s_own[tid] = 0u;
   }
   __syncthreads();
@@ -564,25 +612,27 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
   const int next = ge - gs;
   const int xb = gs >> 5;                       // first ext word (global word index)
   const int nxw = ((ge - 1) >> 5) - xb + 1;     // ext words
-  const int NLAB = fp.NLAB, P = fp.P, NFU = fp.NFU, EXTW = fp.EXTW;
   const int tw_eff = min(fp.TW, fp.W - w0);     // words written by this tile
   const int tbits = 32 * tw_eff;
 
-  // ---- phase 1: nodes of all molecules overlapping the tile ----
+  // ---- phase 1: molecules and nodes overlapping the tile ----
   for (int i = tid; i < nmol * fp.NQW; i += NT) s_gm[i] = 0u;
   for (int i = tid; i <= nmol; i += NT) {
     const int st = __ldg(&goff[g0 + i]) - gs;
     s_mstart[i] = st;
     if (i < nmol) {
       const int n = __ldg(&goff[g0 + i + 1]) - gs - st;
-      const int tb = gs + st - n0;  // tile bit of the molecule start
-      if (n > 0 && tb >= 0 && tb < tbits) {
-        atomicOr(&s_bnd[tb >> 5], 1u << (tb & 31));
-        if (tb + n <= tbits && NW == 1) {
-          atomicOr(&s_own[tb >> 5], 1u << (tb & 31));
-          s_slotat[tb] = (int16_t)i;
-        } else {
-          s_strad = i;  // starts here, ends beyond the tile (or needs the multi-word path)
+      const int tb = gs + st - n0;  // tile bit of the molecule's first node
+      const int te = tb + n - 1;    // ... and of its last node
+      if (n > 0) {
+        if (te >= 0 && te < tbits) atomicOr(&s_endb[te >> 5], 1u << (te & 31));  // segment end
+        if (tb >= 0 && tb < tbits) {  // starts here: this tile owns its GMCR bits
+          if (te < tbits && NW == 1) {
+            atomicOr(&s_own[te >> 5], 1u << (te & 31));
+            s_slotat[te] = (int16_t)i;
+          } else {
+            s_strad = i;  // ends beyond the tile (or needs the multi-word path)
+          }
         }
       }
     }
@@ -590,40 +640,59 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
   for (int i = tid; i < next; i += NT) {
     const int v = gs + i;
     const int loc = __ldg(&fp.D.local[v]);
-    M a;
-    a.clear();
-    if (NW == 1 && fp.D.adj64) {
-      a.w[0] = __ldg(&fp.D.adj64[v]);
-    } else {
-      const int e1 = __ldg(&fp.D.roff[v + 1]);
-      for (int e = __ldg(&fp.D.roff[v]); e < e1; e++) a.set(__ldg(&fp.D.nbr[e]) >> 8);
-    }
-    s_adj[i] = a;
+    const int e0 = __ldg(&fp.D.roff[v]), e1 = __ldg(&fp.D.roff[v + 1]);
+    // up to 4 neighbours packed (unused slots = the node itself: OR-neutral)
+    uint32_t nb = (uint32_t)loc * 0x01010101u;
+    if (e1 - e0 <= 4)
+      for (int e = e0; e < e1; e++) {
+        const int sh = 8 * (e - e0);
+        nb = (nb & ~(0xffu << sh)) | ((uint32_t)(__ldg(&fp.D.nbr[e]) >> 8) << sh);
+      }
+    s_nb[i] = nb;
     s_cur[i] = M::bit(loc);
     s_molstart[i] = (int16_t)(i - loc);
+    s_loc[i] = (uint8_t)loc;
     const int lab = __ldg(&fp.D.label[v]);
     s_lab[i] = (uint8_t)lab;
-    s_fid[i] = (uint8_t)field_of(lab);
+    s_fid[i] = (uint8_t)(field_of(lab) | (e1 - e0 > 4 ? 0x80 : 0));
   }
   __syncthreads();
   for (int mi = tid; mi < nmol; mi += NT)
     if (s_mstart[mi] < s_mstart[mi + 1]) s_sos[s_mstart[mi]] = (int16_t)mi;
-  // ---- label planes (InitializeCandidates, Alg.1 l.29-37) and field planes ----
+  for (int c = tid; c < NLAB; c += NT) s_labch[s_labval[c]] = (uint8_t)c;
+  __syncthreads();
+  // ---- label planes (InitializeCandidates, Alg.1 l.29-37) and field planes:
+  // lane = node builds its one-hot membership word, a warp transpose turns
+  // it into plane words (lane = channel) ----
+  const bool onehot_fits = NLAB + 1 + NFU <= 32;
   for (int k = wid; k < nxw; k += NWARP) {
     const int i = (xb + k) * 32 + lane - gs;
     const bool valid = (i >= 0) && (i < next);
     const int lab = valid ? s_lab[i] : -1;
-    const int fid = valid ? s_fid[i] : -1;
-    uint32_t mine = 0;
-    for (int c = 0; c < NLAB; c++) {
-      const unsigned b = __ballot_sync(FULL_MASK, lab == (int)__ldg(&fp.lab_val[c]));
-      if ((c & 31) == lane) mine = b;
-      if ((c & 31) == 31 || c == NLAB - 1)
-        if (lane <= (c & 31)) s_planes[((c & ~31) + lane) * EXTW + k] = mine;
-    }
-    for (int fs = 0; fs < NFU; fs++) {
-      const unsigned b = __ballot_sync(FULL_MASK, fid == (int)s_fused[fs]);
-      if (lane == 0) s_fplanes[fs * EXTW + k] = b;
+    const int fid = valid ? (s_fid[i] & 0x7f) : -1;
+    uint32_t *plw = s_pl + (size_t)k * PS;
+    if (onehot_fits) {
+      uint32_t mb = 0u;
+      if (valid) {
+        const int lc = s_labch[lab];
+        const int fs = s_fslot[fid];
+        if (lc != 0xff) mb |= 1u << lc;
+        if (fs >= 0) mb |= 1u << (NLAB + 1 + fs);
+      }
+      const uint32_t T = transpose32(mb, lane);
+      if (lane < NLAB) plw[lane] = T;
+      else if (lane == NLAB) plw[NLAB] = 0xffffffffu;
+      else if (lane < NLAB + 1 + NFU) s_fpl[(lane - NLAB - 1) * EXTW + k] = T;
+    } else {
+      for (int c = 0; c < NLAB; c++) {
+        const unsigned b = __ballot_sync(FULL_MASK, lab == (int)s_labval[c]);
+        if (lane == 0) plw[c] = b;
+      }
+      if (lane == 0) plw[NLAB] = 0xffffffffu;
+      for (int fs = 0; fs < NFU; fs++) {
+        const unsigned b = __ballot_sync(FULL_MASK, fid == (int)s_fused[fs]);
+        if (lane == 0) s_fpl[fs * EXTW + k] = b;
+      }
     }
   }
   __syncthreads();
@@ -631,93 +700,139 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
   for (int t = tid; t < nmol * NFU; t += NT) {
     const int mi = t / NFU, fs = t - mi * NFU;
     const int ms = s_mstart[mi], n = s_mstart[mi + 1] - ms;
-    s_fm[t] = extract_window<NW>(s_fplanes + (size_t)fs * EXTW, nxw, (long long)(gs + ms) - (long long)xb * 32, n);
+    s_fm[t] = extract_window<NW>(s_fpl + (size_t)fs * EXTW, nxw, (long long)(gs + ms) - (long long)xb * 32, n);
   }
   for (int i = tid; i < next; i += NT) s_molslot[i] = s_sos[s_molstart[i]];
   __syncthreads();
 
   // ---- radii 1..R: bitset BFS + threshold planes (RefineCandidates, l.19-28) ----
+  auto bfs_node = [&](int i) -> M {  // ball_r(v) = ball_{r-1}(v) | OR_{u in N(v)} ball_{r-1}(u)
+    M x = s_cur[i];
+    const int ms = s_molstart[i];
+    if (!(s_fid[i] & 0x80)) {
+      const uint32_t nb = s_nb[i];
+      x |= s_cur[ms + (nb & 0xff)];
+      x |= s_cur[ms + ((nb >> 8) & 0xff)];
+      x |= s_cur[ms + ((nb >> 16) & 0xff)];
+      x |= s_cur[ms + (nb >> 24)];
+    } else {
+      const int v = gs + i;
+      const int e1 = __ldg(&fp.D.roff[v + 1]);
+      for (int e = __ldg(&fp.D.roff[v]); e < e1; e++) x |= s_cur[ms + (__ldg(&fp.D.nbr[e]) >> 8)];
+    }
+    return x;
+  };
   for (int r = 1; r <= fp.R; r++) {
-    for (int i = tid; i < next; i += NT) {
-      M x = s_cur[i];
-      M a = s_adj[i];
-      const int ms = s_molstart[i];
-      for (int u = a.lowest(); u >= 0; a.clear_lowest(), u = a.lowest()) x |= s_cur[ms + u];
-      s_nxt[i] = x;
+    if (NW == 1) {
+      // in place: all new balls are computed into registers before any is written
+      constexpr int kIt = (1024 + 2 * 63 + NT - 1) / NT;  // EXTN <= 32 * TW + 2 * 63 for <= 64-node graphs
+      M tmp[kIt];
+#pragma unroll
+      for (int it = 0; it < kIt; it++) {
+        const int i = tid + it * NT;
+        if (i < next) tmp[it] = bfs_node(i);
+      }
+      __syncthreads();
+#pragma unroll
+      for (int it = 0; it < kIt; it++) {
+        const int i = tid + it * NT;
+        if (i < next) s_cur[i] = tmp[it];
+      }
+    } else {
+      for (int i = tid; i < next; i += NT) s_nxt[i] = bfs_node(i);
+      __syncthreads();
+      M *t = s_cur;
+      s_cur = s_nxt;
+      s_nxt = t;
     }
     __syncthreads();
-    M *t = s_cur;
-    s_cur = s_nxt;
-    s_nxt = t;
-    const int gb = s_rg[r - 1], gend = s_rg[r];
-    if (gb < gend) {
-      const int pb = s_grpoff[gb];
+    const int r0 = r - 1;
+    const int rb = s_rrec[r0], re = s_rrec[r0 + 1];
+    if (rb < re) {
+      const int TSm = fp.TS - 1;
+      const bool carry = s_rcarry[r0] != 0;
       for (int k = wid; k < nxw; k += NWARP) {
         const int i = (xb + k) * 32 + lane - gs;
         const bool valid = (i >= 0) && (i < next);
         M ball;
         ball.clear();
-        int slot = 0, fid = -1;
+        const M *fmb = s_fm;
         if (valid) {
           ball = s_cur[i];
-          slot = s_molslot[i];
-          fid = s_fid[i];
+          ball.reset(s_loc[i]);  // the node itself is not counted (u != v)
+          fmb = s_fm + (size_t)s_molslot[i] * NFU;
         }
-        uint32_t *pl = s_planes + (size_t)(NLAB + pb) * EXTW + k;
-        for (int g = gb; g < gend; g++) {  // (r, f) groups; planes sorted by (r, f, t)
-          const int f = s_grpf[g];
-          const int cnt = valid ? (ball & s_fm[slot * NFU + s_fslot[f]]).popc() - (fid == f ? 1 : 0) : 0;
-          const int p1 = s_grpoff[g + 1];
-#pragma unroll 2
-          for (int p = s_grpoff[g]; p < p1; p++) {
-            const unsigned b = __ballot_sync(FULL_MASK, cnt >= (int)s_pt[p]);
-            if (lane == 0) *pl = b;
-            pl += EXTW;
+        uint32_t *plw = s_pl + (size_t)k * PS + NLAB + 1;
+        // membership word of the current 32-plane batch: bit (p % 32) = [count >= t_p]
+        uint32_t mb = carry ? s_memb[k * 32 + lane] : 0u;
+        int cur_b = s_grec[rb].batch;
+        for (int rec = rb; rec < re; rec++) {  // (r, f) group parts sorted by batch
+          const GroupRec g = s_grec[rec];
+          if (g.batch != cur_b) {
+            const uint32_t T = transpose32(mb, lane);
+            if (32 * cur_b + lane < fp.P) plw[32 * cur_b + lane] = T;
+            mb = 0u;
+            cur_b = g.batch;
           }
+          const int c = min((ball & fmb[g.fslot]).popc(), TSm);
+          mb |= s_tab[g.toff + c];
+        }
+        if (s_bdone[cur_b] == r0) {
+          const uint32_t T = transpose32(mb, lane);
+          if (32 * cur_b + lane < fp.P) plw[32 * cur_b + lane] = T;
+        } else {
+          s_memb[k * 32 + lane] = mb;  // the batch continues at the next radius
         }
       }
     }
     __syncthreads();
   }
 
-  // ---- rows (query-major): C_L word = label plane AND constraint planes,
-  // written once; GMCR of the molecules contained in the tile from the row
-  // words by a segmented OR ----
-  {
+  // ---- rows (query-major): C_L word = AND of the row's channels, written
+  // once; GMCR of the molecules contained in the tile from the row words:
+  // per-segment any by a carry chain (segments end at end bits E), the
+  // segment that continues from the previous word(s) by a ballot ----
+  // RWc: compile-time row width (0 = runtime fp.RW)
+  auto rows_phase = [&](auto RWc, const uint32_t *rowp) {
+    constexpr int RWk = decltype(RWc)::value;
+    const int RW = RWk ? RWk : fp.RW;
     const int w = w0 + lane;
     const bool active = lane < tw_eff;
-    const int k = w - xb;
-    // per-lane segment data (NW == 1 path)
-    const uint32_t B = s_bnd[lane], OWN = s_own[lane];
-    const uint32_t Br = __brev(B), nBr = ~Br;
-    const uint32_t lowm = B ? ((B & (0u - B)) - 1u) : 0xffffffffu;  // bits below the first boundary
-    const uint32_t topb = B ? (0x80000000u >> __clz(B)) : 0u;          // highest boundary bit
-    const bool nob = (B == 0u);
-    const bool nob_next = __shfl_down_sync(FULL_MASK, nob, 1) && lane + 1 < tw_eff;
+    const int k = active ? w - xb : 0;
+    const unsigned char *plk = (const unsigned char *)(s_pl + (size_t)k * PS);
+    const uint32_t E = s_endb[lane], OWN = s_own[lane];
+    const uint32_t m = ~E;
+    const uint32_t above = E ? ((0xffffffffu << (31 - __clz(E))) << 1) : 0xffffffffu;  // bits above the last end
+    const uint32_t firstE = E & (0u - E);
+    const uint32_t NoE = __ballot_sync(FULL_MASK, active && E == 0u);
+    const int lsh = lane > 0 ? lane - 1 : 31;  // lane 0: no continuation into word 0 is needed
+    const uint32_t firstE0 = lane > 0 ? firstE : 0u;
+    const size_t Wpad = fp.Wpad;
     for (int q = wid; q < fp.NQ; q += NWARP) {
       const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
       uint32_t Aq = 0xffffffffu;
-      uint32_t *bp = fp.bitmap + (size_t)r0 * fp.Wpad + w;
-      const uint32_t *pk = s_planes + k;
-      for (int row = r0; row < r1; row++, bp += fp.Wpad) {
-        const int rl = rowlab[row];
-        const int j0 = rowoff[row], j1 = rowoff[row + 1];
-        uint32_t x = 0u;
-        if (active) {
-          x = pk[rl * EXTW];
-          for (int j = j0; j < j1; j++) x &= pk[(NLAB + rowids[j]) * EXTW];
-          *bp = x;
+      uint32_t *bp = fp.bitmap + (size_t)r0 * Wpad + w;
+      const uint32_t *pr = rowp + (size_t)r0 * RW;
+      for (int row = r0; row < r1; row++, bp += Wpad, pr += RW) {
+        uint32_t x = 0xffffffffu;
+        if (RWk) {
+#pragma unroll
+          for (int j = 0; j < (RWk ? RWk : 1); j++) {
+            const uint32_t two = pr[j];
+            x &= *(const uint32_t *)(plk + (two & 0xffffu)) & *(const uint32_t *)(plk + (two >> 16));
+          }
+        } else {
+          for (int j = 0; j < RW; j++) {
+            const uint32_t two = pr[j];
+            x &= *(const uint32_t *)(plk + (two & 0xffffu)) & *(const uint32_t *)(plk + (two >> 16));
+          }
         }
+        if (active) *bp = x;
         if (NW == 1) {
-          // any-bit per segment, reported at its boundary bit (bit-reversed add)
-          const uint32_t xr = __brev(x);
-          const uint32_t rr = (xr & nBr) + nBr;
-          uint32_t A = __brev((rr | xr) & Br);
-          // the top segment continues into the next word(s)
-          const bool loc = (x & lowm) != 0u;
-          const bool l1 = __shfl_down_sync(FULL_MASK, loc, 1) && lane + 1 < tw_eff;
-          const bool l2 = __shfl_down_sync(FULL_MASK, loc, 2) && lane + 2 < tw_eff;
-          if (l1 || (nob_next && l2)) A |= topb;
+          uint32_t A = (((x & m) + m) | x) & E;
+          const uint32_t H = __ballot_sync(FULL_MASK, (x & above) != 0u);
+          const uint32_t G = H | ((H << 1) & NoE);
+          A |= ((G >> lsh) & 1u) ? firstE0 : 0u;
           Aq &= A;
         }
       }
@@ -731,14 +846,31 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
         }
       }
     }
+  };
+  {
+    const uint32_t *rp = fp.rows_smem ? (const uint32_t *)(smem + L.rowp) : fp.rowp;
+    if (fp.rows_smem) {
+      switch (fp.RW) {
+        case 1: rows_phase(std::integral_constant<int, 1>{}, (const uint32_t *)(smem + L.rowp)); break;
+        case 2: rows_phase(std::integral_constant<int, 2>{}, (const uint32_t *)(smem + L.rowp)); break;
+        case 3: rows_phase(std::integral_constant<int, 3>{}, (const uint32_t *)(smem + L.rowp)); break;
+        case 4: rows_phase(std::integral_constant<int, 4>{}, (const uint32_t *)(smem + L.rowp)); break;
+        default: rows_phase(std::integral_constant<int, 0>{}, (const uint32_t *)(smem + L.rowp)); break;
+      }
+    } else {
+      rows_phase(std::integral_constant<int, 0>{}, rp);
+    }
   }
 
   // ---- GMCR by plane windows: the molecule straddling the tile end (and,
   // for multi-word masks, every molecule starting in the tile) ----
-  M *win = s_win + (size_t)wid * (NLAB + P);
+  const int NCH = NLAB + 1 + fp.P;
+  M *win = s_win + (size_t)wid * NCH;
   const int VQW = (fp.VQ + 31) >> 5;
   uint32_t *nz = s_nz + (size_t)wid * (VQW + 1);
   const int strad = s_strad;
+  const int32_t *rowpoff = fp.rows_smem ? (const int32_t *)(smem + L.rowpoff) : fp.rowp_off;
+  const uint32_t *rowp = fp.rows_smem ? (const uint32_t *)(smem + L.rowp) : fp.rowp;
   for (int mi = wid; mi < nmol; mi += NWARP) {
     if (NW == 1 && mi != strad) continue;
     const int g = g0 + mi;
@@ -747,15 +879,19 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(FilterParams fp) {
     const int ms = s_mstart[mi];
     const int n = s_mstart[mi + 1] - ms;
     const long long s = (long long)(gs + ms) - (long long)xb * 32;
-    for (int c = lane; c < NLAB + P; c += 32) win[c] = extract_window<NW>(s_planes + (size_t)c * EXTW, nxw, s, n);
+    for (int c = lane; c < NCH; c += 32) win[c] = extract_window_strided<NW>(s_pl + c, PS, nxw, s, n);
     __syncwarp();
     for (int rb = 0; rb < VQW; rb++) {
       const int row = rb * 32 + lane;
       bool ok = false;
       if (row < fp.VQ) {
-        M x = win[rowlab[row]];
-        const int j1 = rowoff[row + 1];
-        for (int j = rowoff[row]; j < j1; j++) x &= win[NLAB + rowids[j]];
+        M x = win[NLAB];
+        const int j1 = rowpoff[row + 1];
+        for (int j = rowpoff[row]; j < j1; j++) {
+          const uint32_t two = rowp[j];
+          x &= win[(two & 0xffffu) >> 2];
+          x &= win[two >> 18];
+        }
         ok = x.any();
       }
       const unsigned bits = __ballot_sync(FULL_MASK, ok);
