@@ -113,6 +113,7 @@ struct sigmo_ctx {
   int32_t *qp_row = nullptr, *qp_beoff = nullptr;
   uint16_t *qp_be = nullptr;
   uint32_t *qp_info = nullptr;
+  const int4 *qp_ent = nullptr;
   int32_t *tile_g0 = nullptr, *tile_g1 = nullptr;
   uint8_t *bclass = nullptr;
   // filter tile geometry per TW (32,16,8,4,2,1)
@@ -128,7 +129,9 @@ struct sigmo_ctx {
   int PC = 512, AC = 512, CMC = 2048, MC = 128;
 
   // ---- join ----
-  DBuf pair_query, pair_result, jcnt;  // jcnt u64 slots: [0] chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
+  DBuf pair_query, pair_rec, pair_cm, pair_result, jcnt, adjb;
+  // jcnt u64 slots: [0] pair cursor / chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
+  bool lane_join = false;  // k_join_lane path (<= 64-node graphs, <= 16-node queries)
   int last_mode = 0;
   DBuf sig_tmp, gstack;
 
@@ -705,7 +708,8 @@ void free_all(sigmo_ctx *c) {
   }
   c->progs.clear();
   DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
-                  &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_result, &c->jcnt, &c->sig_tmp, &c->gstack};
+                  &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_rec, &c->pair_cm, &c->pair_result, &c->jcnt,
+                  &c->sig_tmp, &c->gstack, &c->adjb};
   for (DBuf *b : bufs) dfree(c, *b);
 }
 
@@ -902,6 +906,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const size_t o_be = L.take(2 * plan.be.size() + 2);
   const size_t o_bc = L.take(256);
   const size_t o_info = L.take(4 * (size_t)hq.V + 4);
+  const size_t o_ent = L.take(16 * (size_t)hq.V + 16);
   const PackedOffsets pd = plan_graphs(L, hd);
   const size_t o_tg0 = L.take(4 * tg0.size());
   const size_t o_tg1 = L.take(4 * tg1.size());
@@ -923,6 +928,23 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   if (!plan.be.empty()) memcpy(hb + o_be, plan.be.data(), 2 * plan.be.size());
   memcpy(hb + o_bc, bclass, 256);
   if (!plan.info.empty()) memcpy(hb + o_info, plan.info.data(), 4 * plan.info.size());
+  {
+    // per plan position: back-edge depths, bond-class offsets into adjb
+    // (class * VD) and the extra back-edge start, for k_join_lane
+    int4 *ent = (int4 *)(hb + o_ent);
+    const int64_t Wpad_ = std::max<int64_t>(((hd.V + 31) / 32 + 31) / 32 * 32, 32);
+    for (int64_t i = 0; i < hq.V; i++) {
+      const uint32_t inf = plan.info[i];
+      const int j0 = inf & 0x3f, j1 = (inf >> 9) & 0x3f;
+      int4 e4;
+      e4.x = (j0 == 0x3f ? 0xff : j0) | ((j1 == 0x3f ? 0xff : j1) << 8) | (int)(((inf >> 18) & 0x3f) << 16) |
+             (int)(((inf >> 24) & 1u) << 24);
+      e4.y = j0 == 0x3f ? 0 : (int)(((inf >> 6) & 7) * hd.V);
+      e4.z = j1 == 0x3f ? 0 : (int)(((inf >> 15) & 7) * hd.V);
+      e4.w = (int)((uint32_t)(plan.row[i] * Wpad_));  // first bitmap word of the row (unsigned)
+      ent[i] = e4;
+    }
+  }
   pack_graphs(hb, pd, hd);
   memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
   memcpy(hb + o_tg1, tg1.data(), 4 * tg1.size());
@@ -942,6 +964,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->tile_g0 = (int32_t *)(db + o_tg0);
   c->tile_g1 = (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
+  c->qp_ent = (const int4 *)(db + o_ent);
   c->NQ = (int)hq.G;
   c->VQ = (int)hq.V;
   c->EQ = (int)hq.E;
@@ -981,7 +1004,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   for (auto &kv : c->progs) kv.second.valid = false;
 
   // ---- per-batch device buffers ----
-  const size_t bm_bytes = 4 * (size_t)std::max(c->VQ, 1) * c->Wpad;
+  // (+64 B: the join reads up to two words past a molecule window)
+  const size_t bm_bytes = 4 * (size_t)std::max(c->VQ, 1) * c->Wpad + 64;
   const bool bm_grow = c->bitmap.cap < bm_bytes;
   SIGMO_TRY(dreserve(c, c->bitmap, bm_bytes, "candidate bitmap"));
   // padding words (>= W) are never written by the filter: zero once
@@ -999,6 +1023,22 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   SIGMO_TRY(dreserve(c, c->chunk_start, 4 * (size_t)max_chunks, "chunk starts"));
   SIGMO_TRY(dreserve(c, c->nchunks, 16, "chunk count"));
   SIGMO_TRY(dreserve(c, c->pair_query, 4 * (size_t)std::max(pair_cap, 1ll), "pair queries"));
+  // per-lane join: pair records, per-pair candidate masks, bond-class adjacency
+  {
+    const char *legacy = getenv("SIGMO_JOIN_LEGACY");
+    c->lane_join = c->NW == 1 && c->NB > 0 && c->maxq <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) &&
+                   (unsigned long long)pair_cap * (unsigned long long)std::max(c->maxq, 2) < (1ull << 32) &&
+                   (unsigned long long)c->NB * c->VD + 1 < (1ull << 31);
+  }
+  if (c->lane_join) {
+    const size_t mq = (size_t)std::max(c->maxq, 2);
+    SIGMO_TRY(dreserve(c, c->pair_rec, 16 * (size_t)std::max(pair_cap, 1ll), "pair records"));
+    SIGMO_TRY(dreserve(c, c->pair_cm, 8 * mq * (size_t)std::max(pair_cap, 1ll), "pair candidate masks"));
+    SIGMO_TRY(dreserve(c, c->adjb, 8 * ((size_t)c->NB * c->VD + 1), "bond-class adjacency"));
+    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, (unsigned long long *)c->adjb.p, c->stream));
+    // entry NB*VD = all ones: the target of absent back-edges
+    CUDA_TRY(c, cudaMemsetAsync((unsigned long long *)c->adjb.p + (size_t)c->NB * c->VD, 0xff, 8, c->stream));
+  }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
   SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 6), "join counters"));
   c->state = 1;
@@ -1118,6 +1158,27 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     cp.nchunks = (int32_t *)c->nchunks.p;
     CUDA_TRY(c, launch_chunks(cp, c->stream));
     launches++;
+    PairsParams pp{};
+    pp.ND = c->ND;
+    pp.NQ = c->NQ;
+    pp.NQW = c->NQW;
+    pp.MQ = std::max(c->maxq, 2);
+    pp.Wpad = c->Wpad;
+    pp.gm = (const uint32_t *)c->gm.p;
+    pp.off = (const I64x2 *)c->off.p;
+    pp.goff = c->dd.goff;
+    pp.qgoff = c->dq.goff;
+    pp.qp_row = c->qp_row;
+    pp.bitmap = (const uint32_t *)c->bitmap.p;
+    pp.pair_query = (int32_t *)c->pair_query.p;
+    pp.prec = c->lane_join ? (int4 *)c->pair_rec.p : nullptr;
+    pp.pcm = c->lane_join ? (unsigned long long *)c->pair_cm.p : nullptr;
+    CUDA_TRY(c, launch_pairs(pp, c->stream));
+    launches++;
+    if (c->lane_join) {
+      CUDA_TRY(c, launch_pair_masks(pp, c->sm_count * 8, c->stream));
+      launches++;
+    }
     timing_mark(c, 4);
   }
   c->last.filter_launches = launches;
@@ -1163,17 +1224,40 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
     jp.error = (int *)((unsigned long long *)c->jcnt.p + 1);
     jp.stats = (unsigned long long *)c->jcnt.p + 2;
     fill_join_caps(c, jp);
-    const size_t smem = join_smem_bytes(c->NW, jp);
-    if (smem > c->max_smem) return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
-    jp.smem_bytes = smem;
-    const int bps = join_blocks_per_sm(c->NW, (int)mode, jp, smem);
-    const int grid = bps * c->sm_count;
-    SIGMO_TRY(dreserve(c, c->gstack, join_gstack_bytes(c->NW, jp, grid), "join stack"));
-    jp.gstack = (unsigned char *)c->gstack.p;
-    timing_join(c, 0);
-    CUDA_TRY(c, launch_join(c->NW, (int)mode, jp, grid, c->stream));
-    launches++;
-    timing_join(c, 1);
+    if (c->lane_join) {
+      // one GMCR pair per lane (k_join_lane)
+      jp.maxq = std::max(c->maxq, 2);
+      jp.VD = c->VD;
+      jp.prec = (const int4 *)c->pair_rec.p;
+      jp.pcm = (const unsigned long long *)c->pair_cm.p;
+      jp.adjb = (const unsigned long long *)c->adjb.p;
+      jp.qp_ent = c->qp_ent;
+      jp.ones_idx = (unsigned)(c->NB * c->VD);
+      jp.batchK = 4;
+      if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
+      const size_t smem = join_lane_smem_bytes(jp);
+      if (smem > c->max_smem) return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
+      jp.smem_bytes = smem;
+      int bps = join_lane_blocks_per_sm((int)mode, jp, smem);
+      if (const char *e = getenv("SIGMO_JOIN_BPS")) bps = std::max(1, std::min(bps, atoi(e)));
+      const int grid = bps * c->sm_count;
+      timing_join(c, 0);
+      CUDA_TRY(c, launch_join_lane((int)mode, jp, grid, c->stream));
+      launches++;
+      timing_join(c, 1);
+    } else {
+      const size_t smem = join_smem_bytes(c->NW, jp);
+      if (smem > c->max_smem) return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
+      jp.smem_bytes = smem;
+      const int bps = join_blocks_per_sm(c->NW, (int)mode, jp, smem);
+      const int grid = bps * c->sm_count;
+      SIGMO_TRY(dreserve(c, c->gstack, join_gstack_bytes(c->NW, jp, grid), "join stack"));
+      jp.gstack = (unsigned char *)c->gstack.p;
+      timing_join(c, 0);
+      CUDA_TRY(c, launch_join(c->NW, (int)mode, jp, grid, c->stream));
+      launches++;
+      timing_join(c, 1);
+    }
   }
   c->last.join_launches = launches;
   c->last_mode = (int)mode;

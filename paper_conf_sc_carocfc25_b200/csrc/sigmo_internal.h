@@ -132,6 +132,26 @@ struct JoinParams {
   int *error;                  // device flag, nonzero = internal capacity exceeded
   unsigned long long *stats;   // optional: DFS iterator steps (nullable)
   size_t smem_bytes;
+  // per-lane DFS kernel (k_join_lane)
+  int VD;                      // data nodes
+  const int4 *prec;            // [P] pair records {graph start node, query, query node base, nq | graph size << 8}
+  const unsigned long long *pcm;   // [P * maxq] candidate masks of each pair in plan order
+  const unsigned long long *adjb;  // [NB][VD] bond-class adjacency masks (molecule-local bits) + all-ones entry
+  const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 8 | #extra << 16 | leaf-pair << 24, class0 * VD, class1 * VD, row * Wpad}
+  unsigned ones_idx;           // index of the all-ones entry of adjb (= NB * VD)
+  int batchK;                  // finish/assign pairs when >= batchK lanes are free
+};
+
+// k_pairs: GMCR pair list + per-pair candidate masks
+struct PairsParams {
+  int ND, NQ, NQW, MQ, Wpad;
+  const uint32_t *gm;
+  const I64x2 *off;
+  const int32_t *goff, *qgoff, *qp_row;
+  const uint32_t *bitmap;
+  int32_t *pair_query;
+  int4 *prec;                  // null: pair_query only
+  unsigned long long *pcm;
 };
 
 struct SupportParams {
@@ -168,6 +188,14 @@ size_t support_smem_bytes(int NW, int NB, int maxq, int NQW);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);
 cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);
+cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
+cudaError_t launch_pair_masks(const PairsParams &p, int grid, cudaStream_t st);
+cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsigned long long *adjb, cudaStream_t st);
+cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream_t st);
+size_t join_lane_smem_bytes(const JoinParams &p);
+int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem);
+constexpr int kJoinLaneThreads = 128;
+constexpr int kJoinLaneMaxQ = 16;  // k_join_lane handles queries <= 16 nodes in <= 64-node graphs
 size_t join_smem_bytes(int NW, const JoinParams &p);
 size_t join_gstack_bytes(int NW, const JoinParams &p, int grid);
 int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem);

@@ -1681,4 +1681,412 @@ int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem) {
   SIGMO_JOIN_DISPATCH(occ_join_t, smem)
 }
 
+// ===========================================================================
+// GMCR pair list (paper section 4.5, "mapping #2"): expand the
+// per-graph surviving-query bits into pair records at the scanned offsets,
+// with each pair's root candidates (the molecule window of the bitmap row of
+// its plan-depth-0 node).  One warp per data graph, lane = query of a
+// 32-query block.
+// ===========================================================================
+__global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
+  extern __shared__ int4 s_q[];  // per query: {first query node, nq, root row word offset, -}
+  for (int q = threadIdx.x; q < pp.NQ; q += blockDim.x) {
+    const int qs = __ldg(&pp.qgoff[q]);
+    s_q[q] = make_int4(qs, __ldg(&pp.qgoff[q + 1]) - qs, __ldg(&pp.qp_row[qs]) * pp.Wpad, 0);
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (g >= pp.ND) return;
+  const unsigned lt = (1u << lane) - 1u;
+  long long o = pp.off[g].a;
+  const int a = __ldg(&pp.goff[g]);
+  const int n = __ldg(&pp.goff[g + 1]) - a;
+  for (int qb = 0; qb < pp.NQW; qb++) {
+    const uint32_t bits = __ldg(&pp.gm[(size_t)g * pp.NQW + qb]);
+    if ((bits >> lane) & 1u) {
+      const int q = qb * 32 + lane;
+      const long long p = o + __popc(bits & lt);
+      const int4 qi = s_q[q];
+      pp.pair_query[p] = q;
+      if (pp.prec) {
+        pp.prec[p] = make_int4(a, q, qi.x, qi.y | (n << 8));
+        pp.pcm[p * pp.MQ] = extract_window<1>(pp.bitmap + (unsigned)qi.z, pp.Wpad, a, n).w[0];
+      }
+    }
+    o += __popc(bits);
+  }
+}
+
+// candidate masks of plan depths >= 1: pcm[p * MQ + e] = molecule window of
+// the bitmap row of the query node at depth e.  One thread per (pair, depth).
+__global__ void __launch_bounds__(256) k_pair_masks(PairsParams pp) {
+  const unsigned M1 = (unsigned)pp.MQ - 1u;
+  const long long P = pp.off[pp.ND].a;  // GMCR pairs (device value)
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  // (pair, depth) items; 32-bit division (P * M1 < 2^32 is a k_join_lane precondition)
+  const unsigned total = (unsigned)(P * M1);
+  for (unsigned t = blockIdx.x * blockDim.x + threadIdx.x; t < total; t += (unsigned)stride) {
+    const unsigned p = t / M1;
+    const int e = 1 + (int)(t - p * M1);
+    const int4 r = __ldg(&pp.prec[p]);
+    if (e >= (r.w & 0xff)) continue;
+    const int row = __ldg(&pp.qp_row[r.z + e]);
+    pp.pcm[(size_t)p * pp.MQ + e] = extract_window<1>(pp.bitmap + (size_t)row * pp.Wpad, pp.Wpad, r.x, r.w >> 8).w[0];
+  }
+}
+
+cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st) {
+  if (p.ND <= 0) return cudaSuccess;
+  const long long threads = 32ll * p.ND;
+  k_pairs<<<(unsigned)((threads + 255) / 256), 256, 16 * (size_t)(p.NQ > 0 ? p.NQ : 1), st>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pair_masks(const PairsParams &p, int grid, cudaStream_t st) {
+  if (p.MQ <= 1 || p.ND <= 0 || !p.prec) return cudaSuccess;
+  k_pair_masks<<<grid, 256, 0, st>>>(p);
+  return cudaGetLastError();
+}
+
+// ===========================================================================
+// Bond-class adjacency masks adjb[b][v] (molecule-local bits of the
+// neighbours of v joined by a bond of class b), for <= 64-node graphs.
+// ===========================================================================
+__global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, unsigned long long *adjb) {
+  const int v = blockIdx.x * blockDim.x + threadIdx.x;
+  if (v >= d.num_nodes) return;
+  unsigned long long m[8];
+#pragma unroll
+  for (int b = 0; b < 8; b++) m[b] = 0ull;
+  const int e1 = d.roff[v + 1];
+  for (int e = d.roff[v]; e < e1; e++) {
+    const int x = d.nbr[e];
+    const int cls = bclass[x & 255];
+#pragma unroll
+    for (int b = 0; b < 8; b++)
+      if (cls == b) m[b] |= 1ull << ((x >> 8) & 63);
+  }
+#pragma unroll
+  for (int b = 0; b < 8; b++)
+    if (b < NB) adjb[(size_t)b * d.num_nodes + v] = m[b];
+}
+
+cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsigned long long *adjb, cudaStream_t st) {
+  if (d.num_nodes <= 0 || NB <= 0) return cudaSuccess;
+  k_adjb<<<(d.num_nodes + 255) / 256, 256, 0, st>>>(d, bclass, NB, adjb);
+  return cudaGetLastError();
+}
+
+// ===========================================================================
+// k_join_lane: stack-based DFS (section 4.6) with ONE GMCR pair
+// per lane, for queries of <= 16 nodes in <= 64-node data graphs.
+//   * Each lane keeps its DFS stack in shared memory: per depth d the
+//     not-yet-tried candidates R_d and the used set U_d of f(pi_0..pi_{d-1});
+//     a bitmask `ne` of non-empty depths makes every step productive: a step
+//     pops the lowest candidate v of the deepest non-empty depth d
+//     (backtracking costs nothing) and builds the candidates of e = d+1:
+//       cm[e] & ~(U_d | {v}) & AND_{(j,b) in back(e)} adjb[b][f(j)]
+//     At the last depth they are counted with popc (Find All) or end the
+//     pair (Find First).
+//   * The candidate masks cm[e] of a pair were cut from the bitmap by
+//     k_pairs; a lane finishing its pair activates the next one it has
+//     prefetched, and lanes without a prefetched pair take new ones from a
+//     global cursor over the GMCR list (one atomic per warp).  Lanes of a
+//     warp thus run pairs of very different sizes without waiting for each
+//     other (the paper runs one work-item per query of a data graph and sits
+//     at ~48% occupancy, divergence-bound).
+// ===========================================================================
+__host__ __device__ inline size_t join_lane_warp_bytes(int MQ) {
+  const int SD = MQ - 1;
+  // DFS stack (R, U per depth), map bytes, pair queue (2 batches x 32 x {record, root mask})
+  return align16(16 * (size_t)SD * 32) + align16((size_t)MQ * 32) + 2 * 32 * (16 + 8);
+}
+__host__ __device__ inline size_t join_lane_smem(int NQ, int MQ) {
+  (void)NQ;
+  return join_lane_warp_bytes(MQ) * (kJoinLaneThreads / 32);
+}
+size_t join_lane_smem_bytes(const JoinParams &p) { return join_lane_smem(p.NQ, p.maxq); }
+
+__device__ __forceinline__ int ctz64(unsigned long long x) { return __ffsll((long long)x) - 1; }
+
+__device__ __forceinline__ void cp_async16(void *dst, const void *src) {
+  const unsigned s = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async8(void *dst, const void *src) {
+  const unsigned s = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+
+// n-th (0-based) set bit of m (m has > n set bits)
+__device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
+  for (int i = 0; i < n; i++) m &= m - 1u;
+  return __ffs(m) - 1;
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_constant__ JoinParams jp) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int MQ = jp.maxq, SD = MQ - 1;
+  // per-warp shared memory (byte offsets): DFS stack R[d], U[d] (column = lane,
+  // 256 B per depth), map bytes f(pi_d) (32 B per depth), pair queue
+  const unsigned wbase = (unsigned)(wid * join_lane_warp_bytes(MQ));
+  const unsigned oR = wbase;
+  const unsigned oU = wbase + (unsigned)SD * 256u;
+  const unsigned oM = wbase + (unsigned)align16(16 * (size_t)SD * 32);
+  const unsigned oQ = oM + (unsigned)align16((size_t)MQ * 32);
+#define SM64(off) (*(unsigned long long *)(smem + (off)))
+#define SM8(off) (*(uint8_t *)(smem + (off)))
+  int4 *q_rec = (int4 *)(smem + oQ);                                 // [2][32]
+  unsigned long long *q_R0 = (unsigned long long *)(smem + oQ + 1024);  // [2][32]
+  const unsigned myR = oR + 8u * lane, myU = oU + 8u * lane, myM = oM + lane;
+
+  const long long P = jp.off[jp.ND].a;
+  const unsigned lt = (1u << lane) - 1u;
+  unsigned long long *cursor = (unsigned long long *)jp.chunk_counter;
+  const unsigned long long *adjb = jp.adjb;
+  const unsigned long long *pcm = jp.pcm;
+  const int4 *qp_ent = jp.qp_ent;
+  const unsigned ones = jp.ones_idx;
+
+  // warp-uniform pair queue: two batches of up to 32 consecutive GMCR pairs
+  long long qbase0 = 0, qbase1 = 0;
+  int qcnt0 = 0, qcnt1 = 0;
+  auto fetch = [&](int s) {  // claim the next 32 pairs, copy their records asynchronously
+    long long base = 0;
+    if (lane == 0) base = (long long)atomicAdd(cursor, 32ull);
+    base = __shfl_sync(FULL_MASK, base, 0);
+    const int cntq = (int)max(0ll, min(32ll, P - base));
+    if (lane < cntq) {
+      cp_async16(&q_rec[s * 32 + lane], &jp.prec[base + lane]);
+      cp_async8(&q_R0[s * 32 + lane], &jp.pcm[(base + lane) * MQ]);
+    }
+    cp_async_commit();
+    if (s) {
+      qbase1 = base;
+      qcnt1 = cntq;
+    } else {
+      qbase0 = base;
+      qcnt0 = cntq;
+    }
+  };
+  fetch(0);
+  cp_async_wait_all();
+  __syncwarp();
+  fetch(1);
+  int cur = 0, head = 0;
+  bool drained = false;  // warp-uniform: no pairs left in the queue
+
+  // lane state: the current pair (or a part of a pair received from another lane)
+  bool act = false, shared = false;
+  long long cp = 0;
+  int cq = 0, cnq = 0, leafd = -1;
+  unsigned ca = 0, cqb = 0, cmo = 0;  // molecule start node, plan base, pcm offset of the pair
+  uint32_t ne = 0;
+  unsigned long long cnt = 0ull, steps = 0ull;
+
+  while (true) {
+    // ---- one DFS step: pop the lowest candidate v of the deepest non-empty
+    // depth d and build the candidates of depth e = d + 1.  A leaf-pair depth
+    // (the last node has no back-edge to it) is consumed whole instead:
+    // with Y = the last node's candidates, sum_{w in R} |Y \ {w}| = |R||Y| - |R & Y| ----
+    if (act && ne) {
+      const int d = 31 - __clz(ne);
+      const unsigned od = 256u * d;
+      const unsigned long long R = SM64(myR + od);
+      const unsigned long long U = SM64(myU + od);
+      const bool lp = d == leafd;
+      const unsigned lo = (unsigned)R, hi = (unsigned)(R >> 32);
+      const int v = lo ? __ffs(lo) - 1 : 31 + __ffs(hi);
+      const unsigned long long bit = 1ull << v;
+      const unsigned long long Rn = lp ? 0ull : R ^ bit;
+      SM64(myR + od) = Rn;
+      if (!Rn) ne ^= 1u << d;
+      SM8(myM + 32u * d) = (uint8_t)v;
+      const unsigned long long used = lp ? U : (U | bit);
+      const int e = lp ? cnq - 1 : d + 1;
+      // candidates of depth e: cm[e] & ~used & AND_{(j,b) in back(e)} adjb[b][f(j)]
+      const int4 en = __ldg(&qp_ent[cqb + e]);
+      const int j0 = en.x & 0xff, j1 = (en.x >> 8) & 0xff;
+      const int u0 = (j0 == d) ? v : (int)SM8(myM + 32u * (j0 & 31));
+      const int u1 = (j1 == d) ? v : (int)SM8(myM + 32u * (j1 & 31));
+      const unsigned i0 = j0 == 0xff ? ones : (unsigned)en.y + ca + (unsigned)u0;
+      const unsigned i1 = j1 == 0xff ? ones : (unsigned)en.z + ca + (unsigned)u1;
+      unsigned long long X = __ldg(&pcm[cmo + e]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
+      const int nex = (en.x >> 16) & 0xff;
+      if (nex) {  // > 2 back-edges at this depth (fused ring systems): rare
+        const int k0 = __ldg(&jp.qp_beoff[cqb + e]) + 2;
+        for (int k = 0; k < nex; k++) {
+          const int be = __ldg(&jp.qp_be[k0 + k]);
+          const int j = be >> 8;
+          const int u = (j == d) ? v : (int)SM8(myM + 32u * j);
+          X &= __ldg(&adjb[(unsigned)(be & 255) * (unsigned)jp.VD + ca + (unsigned)u]);
+        }
+      }
+      if (e == cnq - 1) {
+        const unsigned long long px = (unsigned long long)__popcll(X);
+        cnt += lp ? (unsigned long long)__popcll(R) * px - (unsigned long long)__popcll(R & X) : px;
+      } else if (X) {
+        SM64(myR + 256u * e) = X;
+        SM64(myU + 256u * e) = used;
+        ne |= 1u << e;
+      }
+      if (MODE == 1 && cnt) ne = 0u;  // Find First: the pair (part) is decided
+      steps++;
+    }
+    const bool done = act && ne == 0u;
+    const unsigned freem = __ballot_sync(FULL_MASK, !act || done);
+    if (__popc(freem) < (drained ? 1 : jp.batchK) && freem != FULL_MASK) continue;
+
+    // ---- finished pairs (parts): result, per-query total (fire-and-forget reductions) ----
+    if (done) {
+      if (MODE == 1) {
+        if (!shared) {
+          jp.pair_result[cp] = cnt ? 1ull : 0ull;
+          if (cnt) atomicAdd(&jp.totals[cq], 1ull);
+        } else if (cnt) {
+          if (atomicOr(&jp.pair_result[cp], 1ull) == 0ull) atomicAdd(&jp.totals[cq], 1ull);
+        }
+      } else {
+        if (!shared) jp.pair_result[cp] = cnt;
+        else if (cnt) atomicAdd(&jp.pair_result[cp], cnt);
+        if (cnt) atomicAdd(&jp.totals[cq], cnt);
+      }
+      act = false;
+      ne = 0u;
+    }
+    // ---- free lanes take the next pairs of the queue ----
+    unsigned idle = freem;
+    while (idle && !drained) {
+      if (head == (cur ? qcnt1 : qcnt0)) {
+        if ((cur ? qcnt0 : qcnt1) == 0) {
+          drained = true;
+          break;
+        }
+        cp_async_wait_all();
+        __syncwarp();
+        fetch(cur);  // refill the drained batch while the other one is consumed
+        cur ^= 1;
+        head = 0;
+      }
+      const int take = min(__popc(idle), (cur ? qcnt1 : qcnt0) - head);
+      const int rank = __popc(idle & lt);
+      if (!act && rank < take) {
+        const int ei = cur * 32 + head + rank;
+        const int4 r = q_rec[ei];
+        const unsigned long long R0 = q_R0[ei];
+        cp = (cur ? qbase1 : qbase0) + head + rank;
+        cq = r.y;
+        cnq = r.w & 0xff;
+        ca = (unsigned)r.x;
+        cqb = (unsigned)r.z;
+        cmo = (unsigned)(cp * MQ);
+        leafd = (cnq >= 3 && ((__ldg(&qp_ent[cqb + cnq - 1]).x >> 24) & 1)) ? cnq - 2 : -1;
+        act = true;
+        shared = false;
+        cnt = 0ull;
+        if (cnq == 1) {
+          cnt = (unsigned long long)__popcll(R0);
+          ne = 0u;
+        } else {
+          SM64(myR) = R0;
+          SM64(myU) = 0ull;
+          ne = R0 ? 1u : 0u;
+        }
+      }
+      head += take;
+      idle = __ballot_sync(FULL_MASK, !act);
+    }
+    // ---- tail: free lanes take the shallowest open depth of a busy lane ----
+    if (idle) {
+      const unsigned donors = __ballot_sync(FULL_MASK, act && (ne & (ne - 1u)) != 0u);
+      const int npair = min(__popc(idle), __popc(donors));
+      if (npair > 0) {
+        const bool recv = !act && __popc(idle & lt) < npair;
+        const bool give = act && ((donors >> lane) & 1u) && __popc(donors & lt) < npair;
+        const int src = recv ? nth_set_bit(donors, __popc(idle & lt)) : lane;
+        const int ds_own = __ffs(ne) - 1;  // shallowest non-empty depth
+        const int ds = __shfl_sync(FULL_MASK, ds_own, src);
+        const long long s_cp = __shfl_sync(FULL_MASK, cp, src);
+        const int s_cq = __shfl_sync(FULL_MASK, cq, src);
+        const int s_cnq = __shfl_sync(FULL_MASK, cnq, src);
+        const int s_leafd = __shfl_sync(FULL_MASK, leafd, src);
+        const unsigned s_ca = __shfl_sync(FULL_MASK, ca, src);
+        const unsigned s_cqb = __shfl_sync(FULL_MASK, cqb, src);
+        const unsigned s_cmo = __shfl_sync(FULL_MASK, cmo, src);
+        if (give && !shared) {
+          // the pair's result is accumulated from several lanes from now on
+          jp.pair_result[cp] = 0ull;
+          shared = true;
+        }
+        __syncwarp();
+        if (recv) {
+          const unsigned dR = oR + 8u * src, dU = oU + 8u * src, dM = oM + src;
+          SM64(myR + 256u * ds) = SM64(dR + 256u * ds);
+          SM64(myU + 256u * ds) = SM64(dU + 256u * ds);
+          for (int j = 0; j < ds; j++) SM8(myM + 32u * j) = SM8(dM + 32u * j);
+          cp = s_cp;
+          cq = s_cq;
+          cnq = s_cnq;
+          leafd = s_leafd;
+          ca = s_ca;
+          cqb = s_cqb;
+          cmo = s_cmo;
+          ne = 1u << ds;
+          cnt = 0ull;
+          act = true;
+          shared = true;
+        }
+        __syncwarp();
+        if (give) ne &= ~(1u << ds_own);
+      }
+    }
+    if (__ballot_sync(FULL_MASK, act) == 0u) break;
+  }
+#undef SM64
+#undef SM8
+  cp_async_wait_all();
+  if (jp.stats) {
+    unsigned long long s2 = steps;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s2 += __shfl_xor_sync(FULL_MASK, s2, o);
+    if (lane == 0) atomicAdd(jp.stats, s2);
+  }
+}
+
+template <int MODE>
+static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_t st) {
+  cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)p.smem_bytes);
+  if (e != cudaSuccess) return e;
+  k_join_lane<MODE><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream_t st) {
+  if (grid <= 0) return cudaSuccess;
+  return mode == 1 ? launch_join_lane_t<1>(p, grid, st) : launch_join_lane_t<0>(p, grid, st);
+}
+
+int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem) {
+  int n = 0;
+  cudaError_t e;
+  if (mode == 1) {
+    cudaFuncSetAttribute(k_join_lane<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<1>, kJoinLaneThreads, smem);
+  } else {
+    cudaFuncSetAttribute(k_join_lane<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<0>, kJoinLaneThreads, smem);
+  }
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return 1;
+  }
+  return n < 1 ? 1 : n;
+}
+
 }  // namespace sigmo
