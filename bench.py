@@ -4,12 +4,14 @@
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl sigmo|reference]
     torchrun --nproc-per-node N bench.py --gpus N ...      (N > 1)
 
-Workload (N=1): BASELINE.json configs[1] = 50 queries (35 library functional
-groups + 15 random 3-8-atom subgraphs) x 100k synthetic ZINC-like molecules,
-Find All, filter levels 4.  Weak scaling: rank r owns
-molecules [r*100k, (r+1)*100k) of the same counter-based stream; queries are
-replicated; the only collective is an NCCL all-reduce of the per-query
-totals.
+Workload (N=1): BASELINE.json configs[2] -- the configuration the metric is
+quoted on at 1/2/4/8 B200 -- = 100 queries (35 library functional groups +
+65 random 3-8-atom subgraphs) x 1M synthetic ZINC-like molecules per GPU,
+Find All, filter levels 4; `--config 1` selects configs[1]
+(50 queries x 100k molecules, the levels-sweep / Find First config).  Weak
+scaling: rank r owns molecules [r*M, (r+1)*M) of the same counter-based
+stream; queries are replicated; the only collective is an NCCL all-reduce of
+the per-query totals.
 
 A step = one pass of the hot path over the resident batch: sigmo_filter
 (signatures + dominance + bitmap + GMCR) -> sigmo_join(Find All) -> per-query
@@ -31,10 +33,10 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 BASELINE_METRIC = "matches/sec (Find All) and graph-pairs/sec (Find First) at 1/2/4/8 B200"
-CONFIG_ID = 2
-MOLS_PER_RANK = 100_000
+# BASELINE.json configs[i] -> synth config id i+1, molecules per rank
+CONFIGS = {1: (2, 100_000), 2: (3, 1_000_000)}
 LEVELS = 4
-CPU_SAMPLE_MOLS = 100_000     # cpu_baseline leg: all of configs[1] (~20 core-seconds of oracle work)
+CPU_SAMPLE_MOLS = 200_000     # cpu_baseline leg: oracle on the first 200k molecules (~100 core-seconds)
 REF_STEP_MOLS = 2_000         # --impl reference: molecules per step
 
 
@@ -45,11 +47,16 @@ def parse():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="sigmo", choices=["sigmo", "reference"])
     ap.add_argument("--levels", type=int, default=LEVELS)
-    ap.add_argument("--molecules", type=int, default=MOLS_PER_RANK, help="molecules per rank")
+    ap.add_argument("--config", type=int, default=2, choices=sorted(CONFIGS), help="BASELINE.json configs[i]")
+    ap.add_argument("--molecules", type=int, default=None, help="molecules per rank (default: the config's)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-flush", action="store_true")
-    return ap.parse_args()
+    a = ap.parse_args()
+    a.cid = CONFIGS[a.config][0]
+    if a.molecules is None:
+        a.molecules = CONFIGS[a.config][1]
+    return a
 
 
 # ----------------------------------------------------------------------------
@@ -163,11 +170,12 @@ def cpu_model() -> str:
     return "unknown"
 
 
-def run_cpu_baseline(Q, levels):
+def run_cpu_baseline(Q, args):
     """The oracle as it stands, on a bounded sample of the same workload."""
     import oracle
     import synth
-    D = synth.config_data(CONFIG_ID, first=0, count=CPU_SAMPLE_MOLS)
+    nmol = min(CPU_SAMPLE_MOLS, args.molecules)
+    D = synth.config_data(args.cid, first=0, count=nmol)
     th = host_cores()
     t0 = time.perf_counter()
     res = oracle.count_dense(Q, D, oracle.FIND_ALL, nthreads=th)
@@ -176,7 +184,7 @@ def run_cpu_baseline(Q, levels):
     oracle.count_dense(Q, D, oracle.FIND_FIRST, nthreads=th)
     dt_ff = time.perf_counter() - t1
     return {"value": float(res.sum()) / dt, "unit": "matches/s", "cores": th, "kind": "oracle",
-            "sample": f"{Q.num_graphs} queries x first {CPU_SAMPLE_MOLS} molecules of configs[1] (Find All), "
+            "sample": f"{Q.num_graphs} queries x first {nmol} molecules of configs[{args.config}] (Find All), "
                       f"{dt:.2f} s wall on {th} threads; {int(res.sum())} matches",
             "find_first_pairs_per_s": Q.num_graphs * D.num_graphs / dt_ff, "cpu_model": cpu_model()}
 
@@ -188,14 +196,14 @@ def run_reference(args, world, rank):
         return
     import oracle
     import synth
-    Q = synth.config_queries(CONFIG_ID)
+    Q = synth.config_queries(args.cid)
     th = host_cores()
     n_total = args.molecules
     step_mols = min(REF_STEP_MOLS, n_total)
 
     def batch(i):
         first = (i * step_mols) % max(n_total - step_mols + 1, 1)
-        return synth.config_data(CONFIG_ID, first=first, count=step_mols)
+        return synth.config_data(args.cid, first=first, count=step_mols)
 
     for i in range(args.warmup):
         oracle.count_dense(Q, batch(i), oracle.FIND_ALL, nthreads=th)
@@ -213,18 +221,19 @@ def run_reference(args, world, rank):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
             "config": config_dict(args, world, oracle_step=step_mols),
             "cpu_baseline": {"value": value, "unit": "matches/s", "cores": th, "kind": "oracle",
-                             "sample": f"{Q.num_graphs} queries x {step_mols} molecules of configs[1] per step, "
+                             "sample": f"{Q.num_graphs} queries x {step_mols} molecules of configs[{args.config}] per step, "
                                        f"{args.steps} steps", "cpu_model": cpu_model()},
             "e2e": {"value": value, "unit": "matches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 def config_dict(args, world, oracle_step=None):
-    d = {"workload": f"configs[1]: 50 queries x {args.molecules} ZINC-like molecules per GPU, Find All, "
-                     f"levels={args.levels}",
-         "queries": 50, "molecules_per_gpu": args.molecules, "molecules_total": args.molecules * world,
-         "levels": args.levels, "mode": "find_all", "data_seed": hex(0x51C0_0000 + CONFIG_ID),
-         "query_seed": hex(0x9E00_0000 + CONFIG_ID),
+    nq = {2: 50, 3: 100}[args.cid]
+    d = {"workload": f"configs[{args.config}]: {nq} queries x {args.molecules} ZINC-like molecules per GPU, "
+                     f"Find All, levels={args.levels}",
+         "queries": nq, "molecules_per_gpu": args.molecules, "molecules_total": args.molecules * world,
+         "levels": args.levels, "mode": "find_all", "data_seed": hex(0x51C0_0000 + args.cid),
+         "query_seed": hex(0x9E00_0000 + args.cid),
          "l2": "flushed before every timed step (256 MiB device write, outside the events)",
          "parallelism": f"dp{world}: molecule shards, queries replicated, NCCL all-reduce of per-query totals"}
     if oracle_step:
@@ -249,8 +258,8 @@ def main():
     dist = None
     if world > 1:
         import torch.distributed as dist
-    Q = synth.config_queries(CONFIG_ID)
-    D = synth.config_data(CONFIG_ID, first=rank * args.molecules, count=args.molecules)
+    Q = synth.config_queries(args.cid)
+    D = synth.config_data(args.cid, first=rank * args.molecules, count=args.molecules)
     stream = torch.cuda.current_stream(dev)
     ctx = sigmo.Context(local, stream)
     ctx.load_batch(Q, D)
@@ -393,7 +402,7 @@ def main():
         "roofline": roofline,
     }
     if world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = run_cpu_baseline(Q, args.levels)
+        line["cpu_baseline"] = run_cpu_baseline(Q, args)
     print(json.dumps(line), flush=True)
     ctx.close()
     if dist is not None:

@@ -131,7 +131,10 @@ struct sigmo_ctx {
   // ---- join ----
   DBuf pair_query, pair_rec, pair_cm, pair_result, jcnt, adjb;
   // jcnt u64 slots: [0] pair cursor / chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
-  bool lane_join = false;  // k_join_lane path (<= 64-node graphs, <= 16-node queries)
+  bool lane_join = false;  // per-lane join possible for this batch (<= 64-node graphs, <= 16-node queries)
+  bool mol_filter = false; // last sigmo_filter used molecule tiles (candidates in cmol layout)
+  int mol_extn = 0, mol_extw = 0;  // molecule-tile geometry (32 graphs per tile)
+  DBuf dense_tmp;          // dense view of cmol for sigmo_get_candidates
   int last_mode = 0;
   DBuf sig_tmp, gstack;
 
@@ -709,7 +712,7 @@ void free_all(sigmo_ctx *c) {
   c->progs.clear();
   DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
                   &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_rec, &c->pair_cm, &c->pair_result, &c->jcnt,
-                  &c->sig_tmp, &c->gstack, &c->adjb};
+                  &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp};
   for (DBuf *b : bufs) dfree(c, *b);
 }
 
@@ -898,6 +901,18 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       tg1[t] = graph_of_host(hd.goff, hd.G, n1 - 1) + 1;
     }
   }
+  // per-lane join + molecule-tile filter possible for this batch?
+  bool lane_ok = false;
+  {
+    int64_t maxn_h = 0, maxq_h = 0;
+    for (int64_t g = 0; g < hd.G; g++) maxn_h = std::max<int64_t>(maxn_h, hd.goff[g + 1] - hd.goff[g]);
+    for (int64_t g = 0; g < hq.G; g++) maxq_h = std::max<int64_t>(maxq_h, hq.goff[g + 1] - hq.goff[g]);
+    const char *legacy = getenv("SIGMO_JOIN_LEGACY");
+    lane_ok = maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) &&
+              (unsigned long long)std::max<int64_t>(hq.V, 1) * (unsigned long long)std::max<int64_t>(hd.G, 1) <
+                  (1ull << 32) &&
+              (unsigned long long)c->NB * hd.V + 1 < (1ull << 31);
+  }
   // ---- staging layout ----
   Layout L;
   const PackedOffsets pq = plan_graphs(L, hq);
@@ -932,7 +947,6 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     // per plan position: back-edge depths, bond-class offsets into adjb
     // (class * VD) and the extra back-edge start, for k_join_lane
     int4 *ent = (int4 *)(hb + o_ent);
-    const int64_t Wpad_ = std::max<int64_t>(((hd.V + 31) / 32 + 31) / 32 * 32, 32);
     for (int64_t i = 0; i < hq.V; i++) {
       const uint32_t inf = plan.info[i];
       const int j0 = inf & 0x3f, j1 = (inf >> 9) & 0x3f;
@@ -941,7 +955,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
              (int)(((inf >> 24) & 1u) << 24);
       e4.y = j0 == 0x3f ? 0 : (int)(((inf >> 6) & 7) * hd.V);
       e4.z = j1 == 0x3f ? 0 : (int)(((inf >> 15) & 7) * hd.V);
-      e4.w = (int)((uint32_t)(plan.row[i] * Wpad_));  // first bitmap word of the row (unsigned)
+      e4.w = plan.row[i];  // bitmap row (query node) of this plan position
       ent[i] = e4;
     }
   }
@@ -981,6 +995,13 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->Wpad = ((c->W + 31) / 32) * 32;
   if (c->Wpad == 0) c->Wpad = 32;
   tile_geometry(c, hd);
+  {
+    int extn = 1;
+    for (int64_t g0 = 0; g0 < hd.G; g0 += 32)
+      extn = std::max<int>(extn, (int)(hd.goff[std::min<int64_t>(g0 + 32, hd.G)] - hd.goff[g0]));
+    c->mol_extn = extn;
+    c->mol_extw = (extn + 31) / 32;
+  }
   c->NBE = (int)plan.be.size();
   c->plan_smem = 0;  // plans are read through the read-only cache
   // join chunk capacities (pairs, atoms, candidate masks, graphs per warp
@@ -1005,7 +1026,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
 
   // ---- per-batch device buffers ----
   // (+64 B: the join reads up to two words past a molecule window)
-  const size_t bm_bytes = 4 * (size_t)std::max(c->VQ, 1) * c->Wpad + 64;
+  size_t bm_bytes = 4 * (size_t)std::max(c->VQ, 1) * c->Wpad + 64;
+  if (lane_ok) bm_bytes = std::max(bm_bytes, 8 * (size_t)std::max(c->VQ, 1) * std::max(c->ND, 1));  // cmol layout
   const bool bm_grow = c->bitmap.cap < bm_bytes;
   SIGMO_TRY(dreserve(c, c->bitmap, bm_bytes, "candidate bitmap"));
   // padding words (>= W) are never written by the filter: zero once
@@ -1024,16 +1046,11 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   SIGMO_TRY(dreserve(c, c->nchunks, 16, "chunk count"));
   SIGMO_TRY(dreserve(c, c->pair_query, 4 * (size_t)std::max(pair_cap, 1ll), "pair queries"));
   // per-lane join: pair records, per-pair candidate masks, bond-class adjacency
-  {
-    const char *legacy = getenv("SIGMO_JOIN_LEGACY");
-    c->lane_join = c->NW == 1 && c->NB > 0 && c->maxq <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) &&
-                   (unsigned long long)pair_cap * (unsigned long long)std::max(c->maxq, 2) < (1ull << 32) &&
-                   (unsigned long long)c->NB * c->VD + 1 < (1ull << 31);
-  }
+  c->lane_join = lane_ok;
+  c->mol_filter = false;
   if (c->lane_join) {
-    const size_t mq = (size_t)std::max(c->maxq, 2);
     SIGMO_TRY(dreserve(c, c->pair_rec, 16 * (size_t)std::max(pair_cap, 1ll), "pair records"));
-    SIGMO_TRY(dreserve(c, c->pair_cm, 8 * mq * (size_t)std::max(pair_cap, 1ll), "pair candidate masks"));
+    SIGMO_TRY(dreserve(c, c->pair_cm, 8 * (size_t)std::max(pair_cap, 1ll), "pair root masks"));
     SIGMO_TRY(dreserve(c, c->adjb, 8 * ((size_t)c->NB * c->VD + 1), "bond-class adjacency"));
     CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, (unsigned long long *)c->adjb.p, c->stream));
     // entry NB*VD = all ones: the target of absent back-edges
@@ -1059,21 +1076,38 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
   int launches = 0;
   if (c->ND > 0 && c->VD > 0) {
     const QueryProgMeta &m = prog->meta;
+    // molecule tiles (cmol layout for the per-lane join) unless the
+    // neighbour-support pass (dense bitmap) is requested
+    bool mol = c->lane_join && !(flags & SIGMO_FILTER_NEIGHBOR_SUPPORT);
     // tile width: largest TW whose shared memory fits
     const int tws[6] = {32, 16, 8, 4, 2, 1};
     int k = 0;
     size_t smem = 0;
     int rows_smem = 1;
-    for (k = 0; k < 12; k++) {
-      rows_smem = k < 6 ? 1 : 0;
-      const int kk = k % 6;
-      smem = filter_smem_bytes(c->NW, c->tile_extn[kk], c->tile_extw[kk], c->tile_molcap[kk], m.NFU, m.NLAB, m.P,
-                               m.NREC, c->VQ, m.NRP, rows_smem, c->NQW, m.TS);
-      // prefer >= 2 CTAs per SM with row programs in shared memory
-      if (smem <= (rows_smem ? c->max_smem / 2 : c->max_smem)) break;
+    if (mol) {
+      rows_smem = 1;
+      smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NRP, 1, c->NQW,
+                               m.TS, 1);
+      if (smem > c->max_smem / 2) {
+        rows_smem = 0;
+        smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NRP, 0,
+                                 c->NQW, m.TS, 1);
+      }
+      if (smem > c->max_smem) mol = false;  // fall back to dense tiles
     }
-    if (k == 12) return set_err(c, SIGMO_ERR_LIMIT, "filter shared memory %zu exceeds %zu (P=%d)", smem, c->max_smem, m.P);
-    k = k % 6;
+    if (!mol) {
+      for (k = 0; k < 12; k++) {
+        rows_smem = k < 6 ? 1 : 0;
+        const int kk = k % 6;
+        smem = filter_smem_bytes(c->NW, c->tile_extn[kk], c->tile_extw[kk], c->tile_molcap[kk], m.NFU, m.NLAB, m.P,
+                                 m.NREC, c->VQ, m.NRP, rows_smem, c->NQW, m.TS, 0);
+        // prefer >= 2 CTAs per SM with row programs in shared memory
+        if (smem <= (rows_smem ? c->max_smem / 2 : c->max_smem)) break;
+      }
+      if (k == 12) return set_err(c, SIGMO_ERR_LIMIT, "filter shared memory %zu exceeds %zu (P=%d)", smem, c->max_smem, m.P);
+      k = k % 6;
+    }
+    c->mol_filter = mol;
     FilterParams fp{};
     fp.D = c->dd;
     fp.TW = tws[k];
@@ -1104,18 +1138,19 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.bitmap = (uint32_t *)c->bitmap.p;
     fp.gm = (uint32_t *)c->gm.p;
     fp.mol_cnt = (I64x2 *)c->mol_cnt.p;
-    fp.EXTN = c->tile_extn[k];
-    fp.EXTW = c->tile_extw[k];
-    fp.MOLCAP = c->tile_molcap[k];
-    fp.tile_g0 = tws[k] == 32 ? c->tile_g0 : nullptr;
-    fp.tile_g1 = tws[k] == 32 ? c->tile_g1 : nullptr;
+    fp.EXTN = mol ? c->mol_extn : c->tile_extn[k];
+    fp.EXTW = mol ? c->mol_extw : c->tile_extw[k];
+    fp.MOLCAP = mol ? 32 : c->tile_molcap[k];
+    fp.tile_g0 = (!mol && tws[k] == 32) ? c->tile_g0 : nullptr;
+    fp.tile_g1 = (!mol && tws[k] == 32) ? c->tile_g1 : nullptr;
+    fp.cmol = mol ? (unsigned long long *)c->bitmap.p : nullptr;
     fp.rows_smem = rows_smem;
     fp.smem_bytes = smem;
     if (c->has_empty_graph) {
       CUDA_TRY(c, cudaMemsetAsync(c->gm.p, 0, 4 * (size_t)c->ND * c->NQW, c->stream));
       CUDA_TRY(c, cudaMemsetAsync(c->mol_cnt.p, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
     }
-    const int tiles = (c->W + fp.TW - 1) / fp.TW;
+    const int tiles = mol ? (c->ND + 31) / 32 : (c->W + fp.TW - 1) / fp.TW;
     timing_mark(c, 2);
     CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));
     launches++;
@@ -1161,6 +1196,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     PairsParams pp{};
     pp.ND = c->ND;
     pp.NQ = c->NQ;
+    pp.VQ = c->VQ;
     pp.NQW = c->NQW;
     pp.MQ = std::max(c->maxq, 2);
     pp.Wpad = c->Wpad;
@@ -1171,14 +1207,11 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     pp.qp_row = c->qp_row;
     pp.bitmap = (const uint32_t *)c->bitmap.p;
     pp.pair_query = (int32_t *)c->pair_query.p;
-    pp.prec = c->lane_join ? (int4 *)c->pair_rec.p : nullptr;
-    pp.pcm = c->lane_join ? (unsigned long long *)c->pair_cm.p : nullptr;
+    pp.prec = mol ? (int4 *)c->pair_rec.p : nullptr;
+    pp.pcm = mol ? (unsigned long long *)c->pair_cm.p : nullptr;
+    pp.cmol = mol ? (const unsigned long long *)c->bitmap.p : nullptr;
     CUDA_TRY(c, launch_pairs(pp, c->stream));
     launches++;
-    if (c->lane_join) {
-      CUDA_TRY(c, launch_pair_masks(pp, c->sm_count * 8, c->stream));
-      launches++;
-    }
     timing_mark(c, 4);
   }
   c->last.filter_launches = launches;
@@ -1224,14 +1257,15 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
     jp.error = (int *)((unsigned long long *)c->jcnt.p + 1);
     jp.stats = (unsigned long long *)c->jcnt.p + 2;
     fill_join_caps(c, jp);
-    if (c->lane_join) {
-      // one GMCR pair per lane (k_join_lane)
+    if (c->mol_filter) {
+      // one GMCR pair per lane (k_join_lane) over the molecule-padded candidates
       jp.maxq = std::max(c->maxq, 2);
       jp.VD = c->VD;
       jp.prec = (const int4 *)c->pair_rec.p;
       jp.pcm = (const unsigned long long *)c->pair_cm.p;
       jp.adjb = (const unsigned long long *)c->adjb.p;
       jp.qp_ent = c->qp_ent;
+      jp.cmol = (const unsigned long long *)c->bitmap.p;
       jp.ones_idx = (unsigned)(c->NB * c->VD);
       jp.batchK = 4;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
@@ -1349,7 +1383,16 @@ sigmo_status sigmo_get_candidates(sigmo_ctx *c, uint32_t *out) {
   if (!c || !out) return SIGMO_ERR_INVALID_ARG;
   if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_candidates before sigmo_filter");
   if (c->VQ == 0 || c->W == 0) return SIGMO_OK;
-  CUDA_TRY(c, cudaMemcpy2DAsync(out, 4 * (size_t)c->W, c->bitmap.p, 4 * (size_t)c->Wpad, 4 * (size_t)c->W,
+  const void *src = c->bitmap.p;
+  if (c->mol_filter) {  // dense view of the molecule-padded layout
+    const size_t bytes = 4 * (size_t)c->VQ * c->Wpad;
+    SIGMO_TRY(dreserve(c, c->dense_tmp, bytes, "dense candidate view"));
+    CUDA_TRY(c, cudaMemsetAsync(c->dense_tmp.p, 0, bytes, c->stream));
+    CUDA_TRY(c, launch_unpad((const unsigned long long *)c->bitmap.p, c->dd.goff, c->ND, c->VQ, c->Wpad,
+                             (uint32_t *)c->dense_tmp.p, c->stream));
+    src = c->dense_tmp.p;
+  }
+  CUDA_TRY(c, cudaMemcpy2DAsync(out, 4 * (size_t)c->W, src, 4 * (size_t)c->Wpad, 4 * (size_t)c->W,
                                 (size_t)c->VQ, cudaMemcpyDeviceToHost, c->stream));
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
   return SIGMO_OK;

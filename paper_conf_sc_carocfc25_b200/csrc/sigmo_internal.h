@@ -95,7 +95,8 @@ struct FilterParams {
   const int32_t *rowp_off;
   const uint32_t *rowp;
   const int32_t *qgoff;        // [NQ+1] query node offsets (rows)
-  uint32_t *bitmap;            // [VQ][Wpad]
+  uint32_t *bitmap;            // [VQ][Wpad] (dense tiles)
+  unsigned long long *cmol;    // [ND][VQ] molecule-padded windows (molecule tiles), else null
   uint32_t *gm;                // [ND][NQW] surviving-query bits per data graph
   I64x2 *mol_cnt;              // [ND+1] (surviving pairs, candidate-mask entries)
   int EXTN, EXTW, MOLCAP;
@@ -134,24 +135,26 @@ struct JoinParams {
   size_t smem_bytes;
   // per-lane DFS kernel (k_join_lane)
   int VD;                      // data nodes
-  const int4 *prec;            // [P] pair records {graph start node, query, query node base, nq | graph size << 8}
-  const unsigned long long *pcm;   // [P * maxq] candidate masks of each pair in plan order
+  const int4 *prec;            // [P] pair records {graph start node, query, graph, nq | first query node << 8}
+  const unsigned long long *pcm;   // [P] root (plan depth 0) candidates of each pair
+  const unsigned long long *cmol;  // [ND][VQ] molecule-padded candidate windows (filter output)
   const unsigned long long *adjb;  // [NB][VD] bond-class adjacency masks (molecule-local bits) + all-ones entry
-  const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 8 | #extra << 16 | leaf-pair << 24, class0 * VD, class1 * VD, row * Wpad}
+  const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 8 | #extra << 16 | leaf-pair << 24, class0 * VD, class1 * VD, row}
   unsigned ones_idx;           // index of the all-ones entry of adjb (= NB * VD)
   int batchK;                  // finish/assign pairs when >= batchK lanes are free
 };
 
 // k_pairs: GMCR pair list + per-pair candidate masks
 struct PairsParams {
-  int ND, NQ, NQW, MQ, Wpad;
+  int ND, NQ, NQW, MQ, Wpad, VQ;
   const uint32_t *gm;
   const I64x2 *off;
   const int32_t *goff, *qgoff, *qp_row;
   const uint32_t *bitmap;
   int32_t *pair_query;
   int4 *prec;                  // null: pair_query only
-  unsigned long long *pcm;
+  unsigned long long *pcm;     // [P] root candidates
+  const unsigned long long *cmol;
 };
 
 struct SupportParams {
@@ -182,14 +185,15 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
                               cudaStream_t st);
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ,
-                         int NRP, int rows_smem, int NQW, int TS);
+                         int NRP, int rows_smem, int NQW, int TS, int mol);
 cudaError_t launch_support(int NW, const SupportParams &p, cudaStream_t st);
 size_t support_smem_bytes(int NW, int NB, int maxq, int NQW);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);
 cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
-cudaError_t launch_pair_masks(const PairsParams &p, int grid, cudaStream_t st);
+cudaError_t launch_unpad(const unsigned long long *cmol, const int32_t *goff, int ND, int VQ, int Wpad, uint32_t *dense,
+                         cudaStream_t st);
 cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsigned long long *adjb, cudaStream_t st);
 cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream_t st);
 size_t join_lane_smem_bytes(const JoinParams &p);

@@ -440,7 +440,7 @@ __host__ __device__ inline int plane_stride(int NLAB, int P) { return (NLAB + 1 
 
 __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB,
                                                     int P, int NREC, int VQ, int NRP, int rows_smem, int NQW,
-                                                    int TS) {
+                                                    int TS, int mol = 0) {
   FilterSmem L;
   const size_t mb = 8 * (size_t)NW;
   const int NWARP = kFilterThreads / 32;
@@ -454,7 +454,9 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   L.pl = o;       o = align16(o + 4 * (size_t)plane_stride(NLAB, P) * EXTW);
   L.fpl = o;      o = align16(o + 4 * (size_t)(NFU > 0 ? NFU : 1) * EXTW);
   L.memb = o;     o = align16(o + 4 * 32 * (size_t)EXTW);
-  L.win = o;      o = align16(o + mb * (size_t)NWARP * NCH);
+  // window path: per warp one molecule's channel windows; molecule tiles
+  // (mol): every channel window of the tile's 32 molecules, [channel][molecule]
+  L.win = o;      o = align16(o + mb * (size_t)(mol ? 32 : NWARP) * NCH);
   L.nz = o;       o = align16(o + 4 * (size_t)NWARP * (VQW + 1));
   L.gmb = o;      o = align16(o + 4 * (size_t)MOLCAP * (NQW > 0 ? NQW : 1));
   L.slotat = o;   o = align16(o + 2 * 32 * 32);
@@ -477,8 +479,8 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
 }
 
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ, int NRP,
-                         int rows_smem, int NQW, int TS) {
-  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, NREC, VQ, NRP, rows_smem, NQW, TS).total;
+                         int rows_smem, int NQW, int TS, int mol) {
+  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, NREC, VQ, NRP, rows_smem, NQW, TS, mol).total;
 }
 
 // 32x32 bit-matrix transpose across the warp: lane L holds row L (bit p =
@@ -521,13 +523,18 @@ __device__ __forceinline__ Mask<NW> extract_window_strided(const uint32_t *words
   return m;
 }
 
-template <int NW>
+// MOL: molecule tiles (32 consecutive data graphs per CTA, <= 64 nodes each)
+// writing the molecule-padded candidate layout cmol[g][row] (u64 window of
+// graph g in the row of query node `row`; a pair's rows are contiguous), used
+// by k_join_lane.  Otherwise
+// dense tiles of TW words writing the row-major bitmap.
+template <int NW, bool MOL>
 __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_constant__ FilterParams fp) {
   using M = Mask<NW>;
   constexpr int NT = kFilterThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
   const FilterSmem L = filter_layout(NW, fp.EXTN, fp.EXTW, fp.MOLCAP, fp.NFU, fp.NLAB, fp.P, fp.NREC, fp.VQ, fp.NRP,
-                                     fp.rows_smem, fp.NQW, fp.TS);
+                                     fp.rows_smem, fp.NQW, fp.TS, MOL ? 1 : 0);
   uint32_t *s_nb = (uint32_t *)(smem + L.nb);
   M *s_cur = (M *)(smem + L.ballA);
   M *s_nxt = (M *)(smem + L.ballB);
@@ -561,15 +568,18 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
 
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int ND = fp.D.num_graphs, VD = fp.D.num_nodes;
-  const int w0 = blockIdx.x * fp.TW;
-  if (w0 >= fp.W) return;
+  const int w0 = MOL ? 0 : blockIdx.x * fp.TW;
+  if (!MOL && w0 >= fp.W) return;
   const int n0 = w0 * 32;
-  const int n1 = min(n0 + fp.TW * 32, VD);
+  const int n1 = MOL ? 0 : min(n0 + fp.TW * 32, VD);
   const int32_t *goff = fp.D.goff;
   const int NLAB = fp.NLAB, NFU = fp.NFU, EXTW = fp.EXTW;
   const int PS = plane_stride(NLAB, fp.P);
   if (tid == 0) {
-    if (fp.tile_g0) {
+    if (MOL) {
+      s_g0 = blockIdx.x * 32;
+      s_g1 = min(s_g0 + 32, ND);
+    } else if (fp.tile_g0) {
       s_g0 = __ldg(&fp.tile_g0[blockIdx.x]);
       s_g1 = __ldg(&fp.tile_g1[blockIdx.x]);
     } else {
@@ -610,8 +620,11 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   const int gs = __ldg(&goff[g0]);
   const int ge = __ldg(&goff[g1]);
   const int next = ge - gs;
-  const int xb = gs >> 5;                       // first ext word (global word index)
-  const int nxw = ((ge - 1) >> 5) - xb + 1;     // ext words
+  // node i (relative to gs) sits at bit (xo - gs + i) of the ext words; dense
+  // tiles use the global 32-bit word grid, molecule tiles start at gs
+  const int xb = gs >> 5;                       // first ext word (global word index, dense)
+  const int xo = MOL ? gs : xb * 32;
+  const int nxw = MOL ? (next + 31) >> 5 : ((ge - 1) >> 5) - xb + 1;  // ext words
   const int tw_eff = min(fp.TW, fp.W - w0);     // words written by this tile
   const int tbits = 32 * tw_eff;
 
@@ -624,7 +637,7 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
       const int n = __ldg(&goff[g0 + i + 1]) - gs - st;
       const int tb = gs + st - n0;  // tile bit of the molecule's first node
       const int te = tb + n - 1;    // ... and of its last node
-      if (n > 0) {
+      if (n > 0 && !MOL) {
         if (te >= 0 && te < tbits) atomicOr(&s_endb[te >> 5], 1u << (te & 31));  // segment end
         if (tb >= 0 && tb < tbits) {  // starts here: this tile owns its GMCR bits
           if (te < tbits && NW == 1) {
@@ -666,7 +679,7 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   // it into plane words (lane = channel) ----
   const bool onehot_fits = NLAB + 1 + NFU <= 32;
   for (int k = wid; k < nxw; k += NWARP) {
-    const int i = (xb + k) * 32 + lane - gs;
+    const int i = xo + k * 32 + lane - gs;
     const bool valid = (i >= 0) && (i < next);
     const int lab = valid ? s_lab[i] : -1;
     const int fid = valid ? (s_fid[i] & 0x7f) : -1;
@@ -700,7 +713,7 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   for (int t = tid; t < nmol * NFU; t += NT) {
     const int mi = t / NFU, fs = t - mi * NFU;
     const int ms = s_mstart[mi], n = s_mstart[mi + 1] - ms;
-    s_fm[t] = extract_window<NW>(s_fpl + (size_t)fs * EXTW, nxw, (long long)(gs + ms) - (long long)xb * 32, n);
+    s_fm[t] = extract_window<NW>(s_fpl + (size_t)fs * EXTW, nxw, (long long)(gs + ms) - (long long)xo, n);
   }
   for (int i = tid; i < next; i += NT) s_molslot[i] = s_sos[s_molstart[i]];
   __syncthreads();
@@ -725,7 +738,8 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   for (int r = 1; r <= fp.R; r++) {
     if (NW == 1) {
       // in place: all new balls are computed into registers before any is written
-      constexpr int kIt = (1024 + 2 * 63 + NT - 1) / NT;  // EXTN <= 32 * TW + 2 * 63 for <= 64-node graphs
+      // EXTN <= 32 * TW + 2 * 63 (dense) or 32 * 64 (molecule tiles) for <= 64-node graphs
+      constexpr int kIt = MOL ? (2048 + NT - 1) / NT : (1024 + 2 * 63 + NT - 1) / NT;
       M tmp[kIt];
 #pragma unroll
       for (int it = 0; it < kIt; it++) {
@@ -752,7 +766,7 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
       const int TSm = fp.TS - 1;
       const bool carry = s_rcarry[r0] != 0;
       for (int k = wid; k < nxw; k += NWARP) {
-        const int i = (xb + k) * 32 + lane - gs;
+        const int i = xo + k * 32 + lane - gs;
         const bool valid = (i >= 0) && (i < next);
         M ball;
         ball.clear();
@@ -786,6 +800,45 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
       }
     }
     __syncthreads();
+  }
+
+  if (MOL) {
+    // ---- molecule tiles: channel windows of the 32 molecules, then rows with
+    // lane = molecule: the window of C_L = AND of the row's channel windows,
+    // written once to cmol[g][row]; GMCR: every row non-empty ----
+    const int NCHm = NLAB + 1 + fp.P;
+    M *win = s_win;  // [channel][32 molecules]
+    for (int t = tid; t < NCHm * 32; t += NT) {
+      const int c = t >> 5, mi = t & 31;
+      M w;
+      w.clear();
+      if (mi < nmol) {
+        const int ms = s_mstart[mi], n = s_mstart[mi + 1] - ms;
+        w = extract_window_strided<NW>(s_pl + c, PS, nxw, ms, n);
+      }
+      win[t] = w;
+    }
+    __syncthreads();
+    const int mi = lane;
+    const bool valid = mi < nmol;
+    const int RW = fp.RW;
+    const uint32_t *rowp = fp.rows_smem ? (const uint32_t *)(smem + L.rowp) : fp.rowp;
+    unsigned long long *cm = fp.cmol + (size_t)(g0 + mi) * fp.VQ;  // molecule-major: cmol[g][row]
+    for (int q = wid; q < fp.NQ; q += NWARP) {
+      const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
+      bool all = valid;
+      for (int row = r0; row < r1; row++) {
+        const uint32_t *pr = rowp + (size_t)row * RW;
+        unsigned long long x = ~0ull;
+        for (int j = 0; j < RW; j++) {
+          const uint32_t two = pr[j];
+          x &= win[((two & 0xffffu) >> 2) * 32 + mi].w[0] & win[(two >> 18) * 32 + mi].w[0];
+        }
+        if (valid) cm[row] = x;
+        all = all && x != 0ull;
+      }
+      if (all) atomicOr(&s_gm[mi * fp.NQW + (q >> 5)], 1u << (q & 31));
+    }
   }
 
   // ---- rows (query-major): C_L word = AND of the row's channels, written
@@ -847,7 +900,7 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
       }
     }
   };
-  {
+  if (!MOL) {
     const uint32_t *rp = fp.rows_smem ? (const uint32_t *)(smem + L.rowp) : fp.rowp;
     if (fp.rows_smem) {
       switch (fp.RW) {
@@ -871,14 +924,14 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   const int strad = s_strad;
   const int32_t *rowpoff = fp.rows_smem ? (const int32_t *)(smem + L.rowpoff) : fp.rowp_off;
   const uint32_t *rowp = fp.rows_smem ? (const uint32_t *)(smem + L.rowp) : fp.rowp;
-  for (int mi = wid; mi < nmol; mi += NWARP) {
+  for (int mi = wid; mi < nmol && !MOL; mi += NWARP) {
     if (NW == 1 && mi != strad) continue;
     const int g = g0 + mi;
     const int gst = __ldg(&goff[g]);
     if (gst < n0) continue;  // owned by the previous tile
     const int ms = s_mstart[mi];
     const int n = s_mstart[mi + 1] - ms;
-    const long long s = (long long)(gs + ms) - (long long)xb * 32;
+    const long long s = (long long)(gs + ms) - (long long)xo;
     for (int c = lane; c < NCH; c += 32) win[c] = extract_window_strided<NW>(s_pl + c, PS, nxw, s, n);
     __syncwarp();
     for (int rb = 0; rb < VQW; rb++) {
@@ -920,7 +973,7 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   // ---- write the GMCR bits and pair counts of the molecules starting here ----
   for (int mi = tid; mi < nmol; mi += NT) {
     const int g = g0 + mi;
-    if (gs + s_mstart[mi] < n0) continue;
+    if (!MOL && gs + s_mstart[mi] < n0) continue;
     long long np = 0;
     for (int qb = 0; qb < fp.NQW; qb++) {
       const uint32_t bits = s_gm[mi * fp.NQW + qb];
@@ -937,16 +990,17 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st) {
   if (num_tiles <= 0) return cudaSuccess;
   cudaError_t e = cudaSuccess;
-#define SIGMO_FILTER_CASE(K)                                                                         \
-  case K:                                                                                            \
-    e = cudaFuncSetAttribute(k_filter<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes); \
-    if (e != cudaSuccess) return e;                                                                  \
-    k_filter<K><<<num_tiles, kFilterThreads, p.smem_bytes, st>>>(p);                                 \
+#define SIGMO_FILTER_CASE(K, MOLF)                                                                              \
+  case K * 2 + MOLF:                                                                                            \
+    e = cudaFuncSetAttribute(k_filter<K, MOLF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem_bytes); \
+    if (e != cudaSuccess) return e;                                                                             \
+    k_filter<K, MOLF><<<num_tiles, kFilterThreads, p.smem_bytes, st>>>(p);                                      \
     break;
-  switch (NW) {
-    SIGMO_FILTER_CASE(1)
-    SIGMO_FILTER_CASE(2)
-    SIGMO_FILTER_CASE(4)
+  switch (NW * 2 + (p.cmol ? 1 : 0)) {
+    SIGMO_FILTER_CASE(1, 0)
+    SIGMO_FILTER_CASE(1, 1)
+    SIGMO_FILTER_CASE(2, 0)
+    SIGMO_FILTER_CASE(4, 0)
     default: return cudaErrorInvalidValue;
   }
 #undef SIGMO_FILTER_CASE
@@ -1689,10 +1743,10 @@ int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem) {
 // 32-query block.
 // ===========================================================================
 __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
-  extern __shared__ int4 s_q[];  // per query: {first query node, nq, root row word offset, -}
+  extern __shared__ int4 s_q[];  // per query: {first query node, nq, root row, -}
   for (int q = threadIdx.x; q < pp.NQ; q += blockDim.x) {
     const int qs = __ldg(&pp.qgoff[q]);
-    s_q[q] = make_int4(qs, __ldg(&pp.qgoff[q + 1]) - qs, __ldg(&pp.qp_row[qs]) * pp.Wpad, 0);
+    s_q[q] = make_int4(qs, __ldg(&pp.qgoff[q + 1]) - qs, __ldg(&pp.qp_row[qs]), 0);
   }
   __syncthreads();
   const int lane = threadIdx.x & 31;
@@ -1701,7 +1755,6 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
   const unsigned lt = (1u << lane) - 1u;
   long long o = pp.off[g].a;
   const int a = __ldg(&pp.goff[g]);
-  const int n = __ldg(&pp.goff[g + 1]) - a;
   for (int qb = 0; qb < pp.NQW; qb++) {
     const uint32_t bits = __ldg(&pp.gm[(size_t)g * pp.NQW + qb]);
     if ((bits >> lane) & 1u) {
@@ -1710,29 +1763,11 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
       const int4 qi = s_q[q];
       pp.pair_query[p] = q;
       if (pp.prec) {
-        pp.prec[p] = make_int4(a, q, qi.x, qi.y | (n << 8));
-        pp.pcm[p * pp.MQ] = extract_window<1>(pp.bitmap + (unsigned)qi.z, pp.Wpad, a, n).w[0];
+        pp.prec[p] = make_int4(a, q, g, qi.y | (qi.x << 8));
+        pp.pcm[p] = __ldg(&pp.cmol[(unsigned)g * (unsigned)pp.VQ + (unsigned)qi.z]);  // root (plan depth 0) candidates
       }
     }
     o += __popc(bits);
-  }
-}
-
-// candidate masks of plan depths >= 1: pcm[p * MQ + e] = molecule window of
-// the bitmap row of the query node at depth e.  One thread per (pair, depth).
-__global__ void __launch_bounds__(256) k_pair_masks(PairsParams pp) {
-  const unsigned M1 = (unsigned)pp.MQ - 1u;
-  const long long P = pp.off[pp.ND].a;  // GMCR pairs (device value)
-  const long long stride = (long long)gridDim.x * blockDim.x;
-  // (pair, depth) items; 32-bit division (P * M1 < 2^32 is a k_join_lane precondition)
-  const unsigned total = (unsigned)(P * M1);
-  for (unsigned t = blockIdx.x * blockDim.x + threadIdx.x; t < total; t += (unsigned)stride) {
-    const unsigned p = t / M1;
-    const int e = 1 + (int)(t - p * M1);
-    const int4 r = __ldg(&pp.prec[p]);
-    if (e >= (r.w & 0xff)) continue;
-    const int row = __ldg(&pp.qp_row[r.z + e]);
-    pp.pcm[(size_t)p * pp.MQ + e] = extract_window<1>(pp.bitmap + (size_t)row * pp.Wpad, pp.Wpad, r.x, r.w >> 8).w[0];
   }
 }
 
@@ -1743,9 +1778,29 @@ cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_pair_masks(const PairsParams &p, int grid, cudaStream_t st) {
-  if (p.MQ <= 1 || p.ND <= 0 || !p.prec) return cudaSuccess;
-  k_pair_masks<<<grid, 256, 0, st>>>(p);
+// Dense (row-major, LSB-first) view of the molecule-padded candidates for
+// sigmo_get_candidates: thread per (row, graph), OR the window into the rows.
+__global__ void k_unpad(const unsigned long long *cmol, const int32_t *goff, int ND, int VQ, int Wpad,
+                        uint32_t *dense) {
+  const long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= (long long)ND * VQ) return;
+  const int g = (int)(t / VQ), row = (int)(t - (long long)g * VQ);
+  const unsigned long long w = cmol[t];  // cmol[g][row]
+  if (!w) return;
+  const int a = goff[g];
+  uint32_t *r = dense + (size_t)row * Wpad;
+  const int wi = a >> 5, sh = a & 31;
+  const unsigned long long lo = w << sh;
+  atomicOr(&r[wi], (uint32_t)lo);
+  if ((uint32_t)(lo >> 32)) atomicOr(&r[wi + 1], (uint32_t)(lo >> 32));
+  if (sh && (uint32_t)(w >> (64 - sh))) atomicOr(&r[wi + 2], (uint32_t)(w >> (64 - sh)));
+}
+
+cudaError_t launch_unpad(const unsigned long long *cmol, const int32_t *goff, int ND, int VQ, int Wpad, uint32_t *dense,
+                         cudaStream_t st) {
+  const long long n = (long long)ND * VQ;
+  if (n <= 0) return cudaSuccess;
+  k_unpad<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(cmol, goff, ND, VQ, Wpad, dense);
   return cudaGetLastError();
 }
 
@@ -1849,7 +1904,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   const unsigned lt = (1u << lane) - 1u;
   unsigned long long *cursor = (unsigned long long *)jp.chunk_counter;
   const unsigned long long *adjb = jp.adjb;
-  const unsigned long long *pcm = jp.pcm;
+  const unsigned long long *cmol = jp.cmol;
   const int4 *qp_ent = jp.qp_ent;
   const unsigned ones = jp.ones_idx;
 
@@ -1863,7 +1918,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     const int cntq = (int)max(0ll, min(32ll, P - base));
     if (lane < cntq) {
       cp_async16(&q_rec[s * 32 + lane], &jp.prec[base + lane]);
-      cp_async8(&q_R0[s * 32 + lane], &jp.pcm[(base + lane) * MQ]);
+      cp_async8(&q_R0[s * 32 + lane], &jp.pcm[base + lane]);
     }
     cp_async_commit();
     if (s) {
@@ -1885,7 +1940,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   bool act = false, shared = false;
   long long cp = 0;
   int cq = 0, cnq = 0, leafd = -1;
-  unsigned ca = 0, cqb = 0, cmo = 0;  // molecule start node, plan base, pcm offset of the pair
+  unsigned ca = 0, cqb = 0, cgv = 0;  // molecule start node, plan base, data graph * VQ (cmol row base)
   uint32_t ne = 0;
   unsigned long long cnt = 0ull, steps = 0ull;
 
@@ -1916,7 +1971,8 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const int u1 = (j1 == d) ? v : (int)SM8(myM + 32u * (j1 & 31));
       const unsigned i0 = j0 == 0xff ? ones : (unsigned)en.y + ca + (unsigned)u0;
       const unsigned i1 = j1 == 0xff ? ones : (unsigned)en.z + ca + (unsigned)u1;
-      unsigned long long X = __ldg(&pcm[cmo + e]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
+      // cm[e] = the graph's window of the row of the query node at depth e
+      unsigned long long X = __ldg(&cmol[cgv + (unsigned)en.w]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
       const int nex = (en.x >> 16) & 0xff;
       if (nex) {  // > 2 back-edges at this depth (fused ring systems): rare
         const int k0 = __ldg(&jp.qp_beoff[cqb + e]) + 2;
@@ -1983,8 +2039,8 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         cq = r.y;
         cnq = r.w & 0xff;
         ca = (unsigned)r.x;
-        cqb = (unsigned)r.z;
-        cmo = (unsigned)(cp * MQ);
+        cqb = (unsigned)r.w >> 8;
+        cgv = (unsigned)r.z * (unsigned)jp.VQ;
         leafd = (cnq >= 3 && ((__ldg(&qp_ent[cqb + cnq - 1]).x >> 24) & 1)) ? cnq - 2 : -1;
         act = true;
         shared = false;
@@ -2017,7 +2073,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         const int s_leafd = __shfl_sync(FULL_MASK, leafd, src);
         const unsigned s_ca = __shfl_sync(FULL_MASK, ca, src);
         const unsigned s_cqb = __shfl_sync(FULL_MASK, cqb, src);
-        const unsigned s_cmo = __shfl_sync(FULL_MASK, cmo, src);
+        const unsigned s_cgv = __shfl_sync(FULL_MASK, cgv, src);
         if (give && !shared) {
           // the pair's result is accumulated from several lanes from now on
           jp.pair_result[cp] = 0ull;
@@ -2035,7 +2091,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
           leafd = s_leafd;
           ca = s_ca;
           cqb = s_cqb;
-          cmo = s_cmo;
+          cgv = s_cgv;
           ne = 1u << ds;
           cnt = 0ull;
           act = true;

@@ -1,6 +1,6 @@
 """Small driver for ncu: load configs[1] (or N molecules), run W warm-up
 steps then S profiled steps of filter + join.  Usage:
-    python tools/profile_step.py [molecules] [levels] [steps] [mode]"""
+    python tools/profile_step.py [molecules] [levels] [steps] [mode] [synth config id]"""
 import os
 import sys
 
@@ -14,8 +14,9 @@ n = int(sys.argv[1]) if len(sys.argv) > 1 else 100_000
 L = int(sys.argv[2]) if len(sys.argv) > 2 else 4
 S = int(sys.argv[3]) if len(sys.argv) > 3 else 2
 mode = int(sys.argv[4]) if len(sys.argv) > 4 else 0
+cid = int(sys.argv[5]) if len(sys.argv) > 5 else 2
 torch.cuda.set_device(0)
-Q, D = synth.config_queries(2), synth.config_data(2, count=n)
+Q, D = synth.config_queries(cid), synth.config_data(cid, count=n)
 ctx = sigmo.Context(0)
 ctx.load_batch(Q, D)
 for _ in range(2 + S):
