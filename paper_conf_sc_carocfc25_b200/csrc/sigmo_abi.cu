@@ -114,6 +114,7 @@ struct sigmo_ctx {
   uint16_t *qp_be = nullptr;
   uint32_t *qp_info = nullptr;
   const int4 *qp_ent = nullptr;
+  const uint32_t *qp_qinfo = nullptr;
   int32_t *tile_g0 = nullptr, *tile_g1 = nullptr;
   uint8_t *bclass = nullptr;
   // filter tile geometry per TW (32,16,8,4,2,1)
@@ -375,12 +376,73 @@ struct QPlan {
   std::vector<int32_t> beoff;   // [VQ+1]
   std::vector<uint16_t> be;     // (j << 8) | class
   std::vector<uint32_t> info;   // [VQ] two back-edges inline + #extra + leaf-sum flag (see plan_queries)
+  std::vector<uint32_t> qinfo;  // [NQ] nq | tail start t << 8 | first query node << 16 (k_join_lane)
 };
+
+// Independent tail of a query (k_join_lane): the largest set S of <= 4
+// pairwise non-adjacent nodes (|S| <= n-1) whose removal splits no connected
+// component.  Placed last in the matching order, the embeddings of S given a
+// prefix embedding are the injective choices from the per-node candidate
+// sets, counted in closed form (inclusion-exclusion over set partitions).
+// Ties: the larger data-label frequency (rare labels stay early to prune).
+uint32_t choose_tail(const HostGraphs &q, int64_t lo, int n, const std::vector<int64_t> &freq) {
+  if (n < 2 || n > kJoinLaneMaxQ) return 0u;
+  std::vector<uint32_t> adj(n, 0u);
+  for (int u = 0; u < n; u++)
+    for (int64_t e = q.roff[lo + u]; e < q.roff[lo + u + 1]; e++) adj[u] |= 1u << (q.col[e] - lo);
+  auto comps = [&](uint32_t keep) {
+    int c = 0;
+    uint32_t left = keep;
+    while (left) {
+      uint32_t fr = left & (0u - left), seen = 0u;
+      while (fr) {
+        seen |= fr;
+        uint32_t nx = 0u;
+        for (uint32_t f = fr; f; f &= f - 1u) nx |= adj[__builtin_ctz(f)];
+        fr = nx & keep & ~seen;
+      }
+      left &= ~seen;
+      c++;
+    }
+    return c;
+  };
+  const uint32_t all = (n == 32) ? 0xffffffffu : ((1u << n) - 1u);
+  const int c0 = comps(all);
+  int kmax = 1;
+  if (const char *e = getenv("SIGMO_TAIL_MAX")) kmax = std::max(1, std::min(4, atoi(e)));
+  for (int k = std::min(kmax, n - 1); k >= 2; k--) {
+    uint32_t best = 0u;
+    int64_t bf = -1;
+    // subsets of size k in increasing order (Gosper's hack)
+    for (uint32_t s = (1u << k) - 1u; s <= all && s != 0u;) {
+      bool indep = true;
+      int iso = 0;
+      int64_t f = 0;
+      for (uint32_t t = s; t && indep; t &= t - 1u) {
+        const int u = __builtin_ctz(t);
+        indep = (adj[u] & s) == 0u;
+        iso += adj[u] == 0u;
+        f += freq[q.nlab[lo + u]];
+      }
+      if (indep && comps(all & ~s) + iso == c0 && f > bf) {
+        best = s;
+        bf = f;
+      }
+      const uint32_t c = s & (0u - s), r = s + c;
+      if (r == 0u) break;
+      s = (((r ^ s) >> 2) / c) | r;
+    }
+    if (best) return best;
+  }
+  // k = 1: the last node of the greedy order (any node is a valid tail of one)
+  return 0u;
+}
 
 void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const uint8_t *bclass, QPlan &out) {
   out.row.assign((size_t)q.V, 0);
   out.beoff.assign((size_t)q.V + 1, 0);
   out.info.assign((size_t)q.V, 0x3fu | (0x3fu << 9));
+  out.qinfo.assign((size_t)q.G, 0u);
   out.be.clear();
   for (int64_t g = 0; g < q.G; g++) {
     const int64_t lo = q.goff[g];
@@ -388,10 +450,16 @@ void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const u
     std::vector<int> pos(n, -1), order;
     auto deg = [&](int u) { return (int)(q.roff[lo + u + 1] - q.roff[lo + u]); };
     auto fr = [&](int u) { return freq[q.nlab[lo + u]]; };
+    const uint32_t tail = choose_tail(q, lo, n, freq);
+    const int ntail = __builtin_popcount(tail);
+    // tail start: the closed form covers depths t..n-1 (t = n - max(|S|, 1))
+    const int t = n <= 1 ? n : n - std::max(ntail, 1);
+    out.qinfo[g] = (uint32_t)n | ((uint32_t)t << 8) | ((uint32_t)lo << 16);
     for (int i = 0; i < n; i++) {
       int best = -1, bc = -1;
       for (int u = 0; u < n; u++) {
         if (pos[u] >= 0) continue;
+        if (i < n - ntail && u < 32 && ((tail >> u) & 1u)) continue;  // the tail goes last
         int conn = 0;
         for (int64_t e = q.roff[lo + u]; e < q.roff[lo + u + 1]; e++)
           if (pos[q.col[e] - lo] >= 0) conn++;
@@ -908,10 +976,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     for (int64_t g = 0; g < hd.G; g++) maxn_h = std::max<int64_t>(maxn_h, hd.goff[g + 1] - hd.goff[g]);
     for (int64_t g = 0; g < hq.G; g++) maxq_h = std::max<int64_t>(maxq_h, hq.goff[g + 1] - hq.goff[g]);
     const char *legacy = getenv("SIGMO_JOIN_LEGACY");
-    lane_ok = maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) &&
+    lane_ok = maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
               (unsigned long long)std::max<int64_t>(hq.V, 1) * (unsigned long long)std::max<int64_t>(hd.G, 1) <
                   (1ull << 32) &&
-              (unsigned long long)c->NB * hd.V + 1 < (1ull << 31);
+              (unsigned long long)(c->NB + 1) * hd.V + 1 < (1ull << 31);
   }
   // ---- staging layout ----
   Layout L;
@@ -922,6 +990,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const size_t o_bc = L.take(256);
   const size_t o_info = L.take(4 * (size_t)hq.V + 4);
   const size_t o_ent = L.take(16 * (size_t)hq.V + 16);
+  const size_t o_qinfo = L.take(4 * (size_t)hq.G + 4);
   const PackedOffsets pd = plan_graphs(L, hd);
   const size_t o_tg0 = L.take(4 * tg0.size());
   const size_t o_tg1 = L.take(4 * tg1.size());
@@ -947,17 +1016,24 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     // per plan position: back-edge depths, bond-class offsets into adjb
     // (class * VD) and the extra back-edge start, for k_join_lane
     int4 *ent = (int4 *)(hb + o_ent);
+    int64_t qg = 0;
     for (int64_t i = 0; i < hq.V; i++) {
+      while (hq.goff[qg + 1] <= i) qg++;
       const uint32_t inf = plan.info[i];
-      const int j0 = inf & 0x3f, j1 = (inf >> 9) & 0x3f;
+      const uint32_t j0 = inf & 0x3f, j1 = (inf >> 9) & 0x3f;
+      // x: j0 | j1 << 4 (15 = none; map slot 15 reads 0) | #extra << 8 | query node << 12
+      // y, z: bond class of back-edge 0 / 1 (adjb[v * NB + class])
+      // w: first extra back-edge in qp_be
+      // (fields are only meaningful for queries of <= kJoinLaneMaxQ nodes)
       int4 e4;
-      e4.x = (j0 == 0x3f ? 0xff : j0) | ((j1 == 0x3f ? 0xff : j1) << 8) | (int)(((inf >> 18) & 0x3f) << 16) |
-             (int)(((inf >> 24) & 1u) << 24);
-      e4.y = j0 == 0x3f ? 0 : (int)(((inf >> 6) & 7) * hd.V);
-      e4.z = j1 == 0x3f ? 0 : (int)(((inf >> 15) & 7) * hd.V);
-      e4.w = plan.row[i];  // bitmap row (query node) of this plan position
+      e4.x = (int)((j0 == 0x3f ? 15u : (j0 & 15u)) | ((j1 == 0x3f ? 15u : (j1 & 15u)) << 4) |
+                   (((inf >> 18) & 15u) << 8) | ((uint32_t)((plan.row[i] - hq.goff[qg]) & 15) << 12));
+      e4.y = j0 == 0x3f ? 0 : (int)((inf >> 6) & 7u);
+      e4.z = j1 == 0x3f ? 0 : (int)((inf >> 15) & 7u);
+      e4.w = plan.beoff[i] + 2;
       ent[i] = e4;
     }
+    if (hq.G) memcpy(hb + o_qinfo, plan.qinfo.data(), 4 * (size_t)hq.G);
   }
   pack_graphs(hb, pd, hd);
   memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
@@ -979,6 +1055,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->tile_g1 = (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
   c->qp_ent = (const int4 *)(db + o_ent);
+  c->qp_qinfo = (const uint32_t *)(db + o_qinfo);
   c->NQ = (int)hq.G;
   c->VQ = (int)hq.V;
   c->EQ = (int)hq.E;
@@ -1050,11 +1127,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->mol_filter = false;
   if (c->lane_join) {
     SIGMO_TRY(dreserve(c, c->pair_rec, 16 * (size_t)std::max(pair_cap, 1ll), "pair records"));
-    SIGMO_TRY(dreserve(c, c->pair_cm, 8 * (size_t)std::max(pair_cap, 1ll), "pair root masks"));
     SIGMO_TRY(dreserve(c, c->adjb, 8 * ((size_t)c->NB * c->VD + 1), "bond-class adjacency"));
-    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, (unsigned long long *)c->adjb.p, c->stream));
-    // entry NB*VD = all ones: the target of absent back-edges
+    // entry VD * NB = all ones: the target of absent back-edges
     CUDA_TRY(c, cudaMemsetAsync((unsigned long long *)c->adjb.p + (size_t)c->NB * c->VD, 0xff, 8, c->stream));
+    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, (unsigned long long *)c->adjb.p, c->stream));
   }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
   SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 6), "join counters"));
@@ -1208,8 +1284,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     pp.bitmap = (const uint32_t *)c->bitmap.p;
     pp.pair_query = (int32_t *)c->pair_query.p;
     pp.prec = mol ? (int4 *)c->pair_rec.p : nullptr;
-    pp.pcm = mol ? (unsigned long long *)c->pair_cm.p : nullptr;
-    pp.cmol = mol ? (const unsigned long long *)c->bitmap.p : nullptr;
+    pp.qinfo = c->qp_qinfo;
     CUDA_TRY(c, launch_pairs(pp, c->stream));
     launches++;
     timing_mark(c, 4);
@@ -1262,11 +1337,9 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       jp.maxq = std::max(c->maxq, 2);
       jp.VD = c->VD;
       jp.prec = (const int4 *)c->pair_rec.p;
-      jp.pcm = (const unsigned long long *)c->pair_cm.p;
       jp.adjb = (const unsigned long long *)c->adjb.p;
       jp.qp_ent = c->qp_ent;
       jp.cmol = (const unsigned long long *)c->bitmap.p;
-      jp.ones_idx = (unsigned)(c->NB * c->VD);
       jp.batchK = 4;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
       const size_t smem = join_lane_smem_bytes(jp);

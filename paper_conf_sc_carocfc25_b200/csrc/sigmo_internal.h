@@ -135,12 +135,10 @@ struct JoinParams {
   size_t smem_bytes;
   // per-lane DFS kernel (k_join_lane)
   int VD;                      // data nodes
-  const int4 *prec;            // [P] pair records {graph start node, query, graph, nq | first query node << 8}
-  const unsigned long long *pcm;   // [P] root (plan depth 0) candidates of each pair
+  const int4 *prec;            // [P] pair records {graph start node, query, graph * VQ + first query node, qinfo[query]}
   const unsigned long long *cmol;  // [ND][VQ] molecule-padded candidate windows (filter output)
-  const unsigned long long *adjb;  // [NB][VD] bond-class adjacency masks (molecule-local bits) + all-ones entry
-  const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 8 | #extra << 16 | leaf-pair << 24, class0 * VD, class1 * VD, row}
-  unsigned ones_idx;           // index of the all-ones entry of adjb (= NB * VD)
+  const unsigned long long *adjb;  // [VD][NB] bond-class adjacency masks (molecule-local bits) + all-ones entry
+  const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 4 (15 none) | #extra << 8 | node << 12, class0, class1, extra back-edge start}
   int batchK;                  // finish/assign pairs when >= batchK lanes are free
 };
 
@@ -153,8 +151,7 @@ struct PairsParams {
   const uint32_t *bitmap;
   int32_t *pair_query;
   int4 *prec;                  // null: pair_query only
-  unsigned long long *pcm;     // [P] root candidates
-  const unsigned long long *cmol;
+  const uint32_t *qinfo;       // [NQ] nq | tail start << 8 | first query node << 16
 };
 
 struct SupportParams {
@@ -199,7 +196,7 @@ cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream
 size_t join_lane_smem_bytes(const JoinParams &p);
 int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem);
 constexpr int kJoinLaneThreads = 128;
-constexpr int kJoinLaneMaxQ = 16;  // k_join_lane handles queries <= 16 nodes in <= 64-node graphs
+constexpr int kJoinLaneMaxQ = 11;  // k_join_lane handles queries <= 11 nodes in <= 64-node graphs (map: 6 bits x 10 depths)
 size_t join_smem_bytes(int NW, const JoinParams &p);
 size_t join_gstack_bytes(int NW, const JoinParams &p, int grid);
 int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem);

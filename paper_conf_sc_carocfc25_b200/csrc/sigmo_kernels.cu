@@ -1737,18 +1737,12 @@ int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem) {
 
 // ===========================================================================
 // GMCR pair list (paper section 4.5, "mapping #2"): expand the
-// per-graph surviving-query bits into pair records at the scanned offsets,
-// with each pair's root candidates (the molecule window of the bitmap row of
-// its plan-depth-0 node).  One warp per data graph, lane = query of a
-// 32-query block.
+// per-graph surviving-query bits into pair records at the scanned offsets
+// (k_join_lane: molecule start node, query, cmol index of the pair's first
+// candidate row, query plan info).  One warp per data graph, lane = query of
+// a 32-query block.
 // ===========================================================================
 __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
-  extern __shared__ int4 s_q[];  // per query: {first query node, nq, root row, -}
-  for (int q = threadIdx.x; q < pp.NQ; q += blockDim.x) {
-    const int qs = __ldg(&pp.qgoff[q]);
-    s_q[q] = make_int4(qs, __ldg(&pp.qgoff[q + 1]) - qs, __ldg(&pp.qp_row[qs]), 0);
-  }
-  __syncthreads();
   const int lane = threadIdx.x & 31;
   const int g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (g >= pp.ND) return;
@@ -1760,11 +1754,10 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
     if ((bits >> lane) & 1u) {
       const int q = qb * 32 + lane;
       const long long p = o + __popc(bits & lt);
-      const int4 qi = s_q[q];
       pp.pair_query[p] = q;
       if (pp.prec) {
-        pp.prec[p] = make_int4(a, q, g, qi.y | (qi.x << 8));
-        pp.pcm[p] = __ldg(&pp.cmol[(unsigned)g * (unsigned)pp.VQ + (unsigned)qi.z]);  // root (plan depth 0) candidates
+        const uint32_t qi = __ldg(&pp.qinfo[q]);
+        pp.prec[p] = make_int4(a, q, (int)((unsigned)g * (unsigned)pp.VQ + (qi >> 16)), (int)qi);
       }
     }
     o += __popc(bits);
@@ -1774,7 +1767,7 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st) {
   if (p.ND <= 0) return cudaSuccess;
   const long long threads = 32ll * p.ND;
-  k_pairs<<<(unsigned)((threads + 255) / 256), 256, 16 * (size_t)(p.NQ > 0 ? p.NQ : 1), st>>>(p);
+  k_pairs<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(p);
   return cudaGetLastError();
 }
 
@@ -1805,7 +1798,7 @@ cudaError_t launch_unpad(const unsigned long long *cmol, const int32_t *goff, in
 }
 
 // ===========================================================================
-// Bond-class adjacency masks adjb[b][v] (molecule-local bits of the
+// Bond-class adjacency masks adjb[v * NB + b] (molecule-local bits of the
 // neighbours of v joined by a bond of class b), for <= 64-node graphs.
 // ===========================================================================
 __global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, unsigned long long *adjb) {
@@ -1824,7 +1817,7 @@ __global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, unsigned long
   }
 #pragma unroll
   for (int b = 0; b < 8; b++)
-    if (b < NB) adjb[(size_t)b * d.num_nodes + v] = m[b];
+    if (b < NB) adjb[(size_t)v * NB + b] = m[b];
 }
 
 cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsigned long long *adjb, cudaStream_t st) {
@@ -1835,43 +1828,52 @@ cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsig
 
 // ===========================================================================
 // k_join_lane: stack-based DFS (section 4.6) with ONE GMCR pair
-// per lane, for queries of <= 16 nodes in <= 64-node data graphs.
-//   * Each lane keeps its DFS stack in shared memory: per depth d the
-//     not-yet-tried candidates R_d and the used set U_d of f(pi_0..pi_{d-1});
-//     a bitmask `ne` of non-empty depths makes every step productive: a step
-//     pops the lowest candidate v of the deepest non-empty depth d
-//     (backtracking costs nothing) and builds the candidates of e = d+1:
-//       cm[e] & ~(U_d | {v}) & AND_{(j,b) in back(e)} adjb[b][f(j)]
-//     At the last depth they are counted with popc (Find All) or end the
-//     pair (Find First).
-//   * The candidate masks cm[e] of a pair were cut from the bitmap by
-//     k_pairs; a lane finishing its pair activates the next one it has
-//     prefetched, and lanes without a prefetched pair take new ones from a
-//     global cursor over the GMCR list (one atomic per warp).  Lanes of a
-//     warp thus run pairs of very different sizes without waiting for each
-//     other (the paper runs one work-item per query of a data graph and sits
-//     at ~48% occupancy, divergence-bound).
+// per lane, for queries of <= kJoinLaneMaxQ nodes in <= 64-node data graphs.
+//   * Per lane, in shared memory: the DFS stack {R_d, U_d} (untried
+//     candidates of depth d, used set of f(pi_0..pi_{d-1})), the map bytes
+//     f(pi_d), and two buffers of candidate windows cm[u] (one u64 per query
+//     node, cut by the filter into cmol[g][row]; a pair's rows are
+//     contiguous): the current pair's, and the next pair's, which is
+//     prefetched with cp.async while the current one runs.  A bitmask `ne`
+//     of open depths makes every step productive: a step pops the lowest
+//     candidate v of the deepest open depth d (backtracking is free) and
+//     builds the candidates of e = d + 1:
+//        X = cm[pi_e] & ~(U_d | {v}) & AND_{(j,b) in back(e)} adjb[b][f(pi_j)]
+//     pushed as {X, U_d | {v}}; at the last depth they are counted with popc
+//     (Find All) or end the pair (Find First).  Absent back-edges read the
+//     all-ones adjacency class, so the step has no selects.
+//   * The warp claims the GMCR list in chunks of 32 pair records (one atomic
+//     per chunk, issued a chunk ahead; the records are held in registers,
+//     one per lane, and handed to lanes by shuffles).  Lanes whose pair
+//     finished refill together (>= batchK at a time): write the result,
+//     activate the prefetched next pair, take a new next pair and start its
+//     prefetch.  Lanes of a warp thus run pairs of very different sizes
+//     without waiting for each other (the paper runs one work-item per query
+//     of a data graph and sits at ~48% occupancy, divergence-bound,
+//     P:1854-1884); when the list is drained, idle lanes take the shallowest
+//     open depth of a busy lane (heavy pairs).
+//   * Per-query totals are reduced in shared memory (one global atomic per
+//     query per CTA).
 // ===========================================================================
+constexpr int kJoinChunk = 32;  // GMCR pairs per warp claim (one record per lane)
+
 __host__ __device__ inline size_t join_lane_warp_bytes(int MQ) {
-  const int SD = MQ - 1;
-  // DFS stack (R, U per depth), map bytes, pair queue (2 batches x 32 x {record, root mask})
-  return align16(16 * (size_t)SD * 32) + align16((size_t)MQ * 32) + 2 * 32 * (16 + 8);
+  const int SD = MQ > 1 ? MQ - 1 : 1;  // pushed depths 0..n-2
+  // {R, U} [SD][32] 16 B | map [16][32] B
+  return 512 * (size_t)SD + 512;
 }
-__host__ __device__ inline size_t join_lane_smem(int NQ, int MQ) {
-  (void)NQ;
-  return join_lane_warp_bytes(MQ) * (kJoinLaneThreads / 32);
+// CTA: per-query totals [NQ] u64, then one region per warp
+__host__ __device__ inline size_t join_lane_cta_bytes(int VQ, int NQ) {
+  (void)VQ;
+  return align16(8 * (size_t)(NQ > 0 ? NQ : 1));
 }
-size_t join_lane_smem_bytes(const JoinParams &p) { return join_lane_smem(p.NQ, p.maxq); }
+__host__ __device__ inline size_t join_lane_smem(int VQ, int NQ, int MQ) {
+  return join_lane_cta_bytes(VQ, NQ) + join_lane_warp_bytes(MQ) * (kJoinLaneThreads / 32);
+}
+size_t join_lane_smem_bytes(const JoinParams &p) { return join_lane_smem(p.VQ, p.NQ, p.maxq); }
 
-__device__ __forceinline__ int ctz64(unsigned long long x) { return __ffsll((long long)x) - 1; }
-
-__device__ __forceinline__ void cp_async16(void *dst, const void *src) {
-  const unsigned s = (unsigned)__cvta_generic_to_shared(dst);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async8(void *dst, const void *src) {
-  const unsigned s = (unsigned)__cvta_generic_to_shared(dst);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(src) : "memory");
+__device__ __forceinline__ void cp_async8(unsigned dst_smem, const void *src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(dst_smem), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
@@ -1885,226 +1887,223 @@ __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
 template <int MODE>
 __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_constant__ JoinParams jp) {
   extern __shared__ __align__(16) unsigned char smem[];
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const int MQ = jp.maxq, SD = MQ - 1;
-  // per-warp shared memory (byte offsets): DFS stack R[d], U[d] (column = lane,
-  // 256 B per depth), map bytes f(pi_d) (32 B per depth), pair queue
-  const unsigned wbase = (unsigned)(wid * join_lane_warp_bytes(MQ));
-  const unsigned oR = wbase;
-  const unsigned oU = wbase + (unsigned)SD * 256u;
-  const unsigned oM = wbase + (unsigned)align16(16 * (size_t)SD * 32);
-  const unsigned oQ = oM + (unsigned)align16((size_t)MQ * 32);
-#define SM64(off) (*(unsigned long long *)(smem + (off)))
-#define SM8(off) (*(uint8_t *)(smem + (off)))
-  int4 *q_rec = (int4 *)(smem + oQ);                                 // [2][32]
-  unsigned long long *q_R0 = (unsigned long long *)(smem + oQ + 1024);  // [2][32]
-  const unsigned myR = oR + 8u * lane, myU = oU + 8u * lane, myM = oM + lane;
+#define LDS64(o) (*(const unsigned long long *)(smem + (o)))
+#define STS64(o) (*(unsigned long long *)(smem + (o)))
+#define LDS128(o) (*(const ulonglong2 *)(smem + (o)))
+#define STS128(o) (*(ulonglong2 *)(smem + (o)))
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int MQ = jp.maxq, SD = MQ > 1 ? MQ - 1 : 1;
+  // ---- CTA tables ----
+  const unsigned o_tot = 0u;
+  for (int i = threadIdx.x; i < jp.NQ; i += blockDim.x) ((unsigned long long *)(smem + o_tot))[i] = 0ull;
+  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.VQ, jp.NQ) + (size_t)wid * join_lane_warp_bytes(MQ));
+  const unsigned oRU = wbase + 16u * lane;                        // {R, U} of depth d: oRU + 512 d
+  const unsigned oM = wbase + 512u * SD + lane;                   // f(pi_d): oM + 32 d
+  smem[oM + 32 * 15] = 0;  // map slot 15 (absent back-edge) reads node 0 of the all-ones class
+  __syncthreads();
 
-  const long long P = jp.off[jp.ND].a;
   const unsigned lt = (1u << lane) - 1u;
-  unsigned long long *cursor = (unsigned long long *)jp.chunk_counter;
-  const unsigned long long *adjb = jp.adjb;
-  const unsigned long long *cmol = jp.cmol;
-  const int4 *qp_ent = jp.qp_ent;
-  const unsigned ones = jp.ones_idx;
+  const unsigned P = (unsigned)jp.off[jp.ND].a;
+  unsigned *const cursor = (unsigned *)jp.chunk_counter;
+  const unsigned long long *const adjb = jp.adjb;
+  const unsigned long long *const cmol = jp.cmol;
+  const unsigned NB = (unsigned)jp.NB;
+  const unsigned ones = (unsigned)jp.VD * NB;  // the all-ones entry (absent back-edge)
+  const int4 *const qp_ent = jp.qp_ent;
+  const int4 zero4 = make_int4(0, 0, 0, 0);
 
-  // warp-uniform pair queue: two batches of up to 32 consecutive GMCR pairs
-  long long qbase0 = 0, qbase1 = 0;
-  int qcnt0 = 0, qcnt1 = 0;
-  auto fetch = [&](int s) {  // claim the next 32 pairs, copy their records asynchronously
-    long long base = 0;
-    if (lane == 0) base = (long long)atomicAdd(cursor, 32ull);
-    base = __shfl_sync(FULL_MASK, base, 0);
-    const int cntq = (int)max(0ll, min(32ll, P - base));
-    if (lane < cntq) {
-      cp_async16(&q_rec[s * 32 + lane], &jp.prec[base + lane]);
-      cp_async8(&q_R0[s * 32 + lane], &jp.pcm[base + lane]);
-    }
-    cp_async_commit();
-    if (s) {
-      qbase1 = base;
-      qcnt1 = cntq;
-    } else {
-      qbase0 = base;
-      qcnt0 = cntq;
-    }
-  };
-  fetch(0);
-  cp_async_wait_all();
-  __syncwarp();
-  fetch(1);
-  int cur = 0, head = 0;
-  bool drained = false;  // warp-uniform: no pairs left in the queue
+  // ---- GMCR chunks: current (records of pairs cbase + i in lane i's crec), prefetched, claimed ----
+  unsigned cbase, pbase, nbase;
+  {
+    unsigned x = 0u;
+    if (lane == 0) x = atomicAdd(cursor, 3u * kJoinChunk);
+    x = __shfl_sync(FULL_MASK, x, 0);
+    cbase = x;
+    pbase = x + kJoinChunk;
+    nbase = x + 2u * kJoinChunk;
+  }
+  int4 crec = cbase + lane < P ? __ldg(&jp.prec[cbase + lane]) : zero4;
+  int4 prec = pbase + lane < P ? __ldg(&jp.prec[pbase + lane]) : zero4;
+  unsigned ccount = cbase < P ? min(P - cbase, (unsigned)kJoinChunk) : 0u, chead = 0u;
+  bool drained = ccount == 0u;
 
-  // lane state: the current pair (or a part of a pair received from another lane)
-  bool act = false, shared = false;
-  long long cp = 0;
-  int cq = 0, cnq = 0, leafd = -1;
-  unsigned ca = 0, cqb = 0, cgv = 0;  // molecule start node, plan base, data graph * VQ (cmol row base)
-  uint32_t ne = 0;
-  unsigned long long cnt = 0ull, steps = 0ull;
+  // ---- lane state ----
+  unsigned ne = 0u;  // open depths of the current pair (0: no work)
+  bool pend = false, shared = false;
+  unsigned cmb = 0u;  // cmol index of the current pair's first candidate row
+  unsigned cp = 0u, ca = 0u, cqb = 0u, cinfo = 0u;  // ca: adjb index of the molecule's first node
+  int cq = 0;
+  unsigned long long cnt = 0ull;
+  unsigned steps = 0u;
+  bool nv = false;  // next pair assigned (rows in flight into the other buffer)
+  unsigned np = 0u;
+  int4 nrec = zero4;
+  unsigned long long nR0 = 0ull;
 
   while (true) {
-    // ---- one DFS step: pop the lowest candidate v of the deepest non-empty
-    // depth d and build the candidates of depth e = d + 1.  A leaf-pair depth
-    // (the last node has no back-edge to it) is consumed whole instead:
-    // with Y = the last node's candidates, sum_{w in R} |Y \ {w}| = |R||Y| - |R & Y| ----
-    if (act && ne) {
+    // ---- one DFS step ----
+    if (ne) {
       const int d = 31 - __clz(ne);
-      const unsigned od = 256u * d;
-      const unsigned long long R = SM64(myR + od);
-      const unsigned long long U = SM64(myU + od);
-      const bool lp = d == leafd;
-      const unsigned lo = (unsigned)R, hi = (unsigned)(R >> 32);
+      const int e = d + 1;
+      const unsigned od = oRU + 512u * d;
+      // the plan entry of depth e and the map bytes of its back-edge targets
+      // depend on d only: loaded before v is known (j == d takes v below)
+      const int4 en = __ldg(&qp_ent[cqb + e]);
+      const ulonglong2 RU = LDS128(od);
+      const unsigned j0 = en.x & 15, j1 = (en.x >> 4) & 15;
+      const unsigned m0 = smem[oM + 32u * j0], m1 = smem[oM + 32u * j1];
+      const unsigned lo = (unsigned)RU.x, hi = (unsigned)(RU.x >> 32);
       const int v = lo ? __ffs(lo) - 1 : 31 + __ffs(hi);
       const unsigned long long bit = 1ull << v;
-      const unsigned long long Rn = lp ? 0ull : R ^ bit;
-      SM64(myR + od) = Rn;
+      const unsigned long long Rn = RU.x ^ bit;
+      STS64(od) = Rn;
+      smem[oM + 32u * d] = (unsigned char)v;
       if (!Rn) ne ^= 1u << d;
-      SM8(myM + 32u * d) = (uint8_t)v;
-      const unsigned long long used = lp ? U : (U | bit);
-      const int e = lp ? cnq - 1 : d + 1;
-      // candidates of depth e: cm[e] & ~used & AND_{(j,b) in back(e)} adjb[b][f(j)]
-      const int4 en = __ldg(&qp_ent[cqb + e]);
-      const int j0 = en.x & 0xff, j1 = (en.x >> 8) & 0xff;
-      const int u0 = (j0 == d) ? v : (int)SM8(myM + 32u * (j0 & 31));
-      const int u1 = (j1 == d) ? v : (int)SM8(myM + 32u * (j1 & 31));
-      const unsigned i0 = j0 == 0xff ? ones : (unsigned)en.y + ca + (unsigned)u0;
-      const unsigned i1 = j1 == 0xff ? ones : (unsigned)en.z + ca + (unsigned)u1;
-      // cm[e] = the graph's window of the row of the query node at depth e
-      unsigned long long X = __ldg(&cmol[cgv + (unsigned)en.w]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
-      const int nex = (en.x >> 16) & 0xff;
-      if (nex) {  // > 2 back-edges at this depth (fused ring systems): rare
-        const int k0 = __ldg(&jp.qp_beoff[cqb + e]) + 2;
+      const unsigned long long used = RU.y | bit;
+      // candidates of depth e
+      const unsigned u0 = j0 == (unsigned)d ? (unsigned)v : m0, u1 = j1 == (unsigned)d ? (unsigned)v : m1;
+      const unsigned i0 = j0 == 15u ? ones : ca + u0 * NB + (unsigned)en.y;
+      const unsigned i1 = j1 == 15u ? ones : ca + u1 * NB + (unsigned)en.z;
+      unsigned long long X = __ldg(&cmol[cmb + ((en.x >> 12) & 15)]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
+      if (en.x & 0xf00) {  // > 2 back-edges at this depth (fused rings): rare
+        const int nex = (en.x >> 8) & 15;
         for (int k = 0; k < nex; k++) {
-          const int be = __ldg(&jp.qp_be[k0 + k]);
-          const int j = be >> 8;
-          const int u = (j == d) ? v : (int)SM8(myM + 32u * j);
-          X &= __ldg(&adjb[(unsigned)(be & 255) * (unsigned)jp.VD + ca + (unsigned)u]);
+          const int be = __ldg(&jp.qp_be[en.w + k]);
+          X &= __ldg(&adjb[ca + smem[oM + 32u * (be >> 8)] * NB + (unsigned)(be & 255)]);
         }
       }
-      if (e == cnq - 1) {
-        const unsigned long long px = (unsigned long long)__popcll(X);
-        cnt += lp ? (unsigned long long)__popcll(R) * px - (unsigned long long)__popcll(R & X) : px;
+      if (e == (int)(cinfo & 0xff) - 1) {
+        cnt += (unsigned long long)__popcll(X);
+        if (MODE == 1 && cnt) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
-        SM64(myR + 256u * e) = X;
-        SM64(myU + 256u * e) = used;
+        STS128(oRU + 512u * e) = make_ulonglong2(X, used);
         ne |= 1u << e;
       }
-      if (MODE == 1 && cnt) ne = 0u;  // Find First: the pair (part) is decided
+      pend = ne == 0u;
       steps++;
     }
-    const bool done = act && ne == 0u;
-    const unsigned freem = __ballot_sync(FULL_MASK, !act || done);
-    if (__popc(freem) < (drained ? 1 : jp.batchK) && freem != FULL_MASK) continue;
+    const unsigned fm = __ballot_sync(FULL_MASK, ne == 0u);
+    if (drained ? fm == 0u : (__popc(fm) < jp.batchK && fm != FULL_MASK)) continue;
 
-    // ---- finished pairs (parts): result, per-query total (fire-and-forget reductions) ----
-    if (done) {
+    // ---- finished pairs (parts): result, per-query total in shared memory ----
+    if (pend) {
       if (MODE == 1) {
         if (!shared) {
           jp.pair_result[cp] = cnt ? 1ull : 0ull;
-          if (cnt) atomicAdd(&jp.totals[cq], 1ull);
+          if (cnt) atomicAdd((unsigned long long *)(smem + o_tot) + cq, 1ull);
         } else if (cnt) {
-          if (atomicOr(&jp.pair_result[cp], 1ull) == 0ull) atomicAdd(&jp.totals[cq], 1ull);
+          if (atomicOr(&jp.pair_result[cp], 1ull) == 0ull) atomicAdd((unsigned long long *)(smem + o_tot) + cq, 1ull);
         }
       } else {
         if (!shared) jp.pair_result[cp] = cnt;
         else if (cnt) atomicAdd(&jp.pair_result[cp], cnt);
-        if (cnt) atomicAdd(&jp.totals[cq], cnt);
+        if (cnt) atomicAdd((unsigned long long *)(smem + o_tot) + cq, cnt);
       }
-      act = false;
-      ne = 0u;
+      pend = false;
     }
-    // ---- free lanes take the next pairs of the queue ----
-    unsigned idle = freem;
-    while (idle && !drained) {
-      if (head == (cur ? qcnt1 : qcnt0)) {
-        if ((cur ? qcnt0 : qcnt1) == 0) {
+    // ---- free lanes activate their prefetched next pair ----
+    if (ne == 0u && nv) {
+      cp = np;
+      cmb = (unsigned)nrec.z;
+      ca = (unsigned)nrec.x * NB;
+      cq = nrec.y;
+      cinfo = (unsigned)nrec.w;
+      cqb = cinfo >> 16;
+      shared = false;
+      cnt = 0ull;
+      const int4 en0 = __ldg(&qp_ent[cqb]);
+      const unsigned long long R0 = nR0;
+      if ((cinfo & 0xff) == 1u) {
+        cnt = (unsigned long long)__popcll(R0);
+        pend = true;
+      } else {
+        STS128(oRU) = make_ulonglong2(R0, 0ull);
+        ne = R0 ? 1u : 0u;
+        pend = ne == 0u;
+      }
+      nv = false;
+    }
+    // ---- lanes without a next pair take one from the chunk and prefetch its rows ----
+    unsigned wm = __ballot_sync(FULL_MASK, !nv && !drained);
+    while (wm) {
+      const unsigned avail = ccount - chead;
+      const unsigned n = (unsigned)__popc(wm);
+      const unsigned take = min(n, avail);
+      const unsigned rank = (unsigned)__popc(wm & lt);
+      const bool mine = ((wm >> lane) & 1u) && rank < take;
+      const int src = (int)(chead + (mine ? rank : 0u));
+      int4 r;
+      r.x = __shfl_sync(FULL_MASK, crec.x, src);
+      r.y = __shfl_sync(FULL_MASK, crec.y, src);
+      r.z = __shfl_sync(FULL_MASK, crec.z, src);
+      r.w = __shfl_sync(FULL_MASK, crec.w, src);
+      if (mine) {
+        nrec = r;
+        np = cbase + (unsigned)src;
+        nv = true;
+        // root candidates of the next pair: the load completes while the current pair runs
+        nR0 = __ldg(&cmol[(unsigned)r.z + ((__ldg(&qp_ent[(unsigned)r.w >> 16]).x >> 12) & 15)]);
+      }
+      chead += take;
+      wm = __ballot_sync(FULL_MASK, !nv) & wm;
+      if (chead == ccount) {  // chunk exhausted: switch to the prefetched one, claim the one after
+        cbase = pbase;
+        crec = prec;
+        ccount = cbase < P ? min(P - cbase, (unsigned)kJoinChunk) : 0u;
+        chead = 0u;
+        if (ccount == 0u) {
           drained = true;
           break;
         }
-        cp_async_wait_all();
-        __syncwarp();
-        fetch(cur);  // refill the drained batch while the other one is consumed
-        cur ^= 1;
-        head = 0;
+        pbase = nbase;
+        prec = pbase + lane < P ? __ldg(&jp.prec[pbase + lane]) : zero4;
+        unsigned x = 0u;
+        if (lane == 0) x = atomicAdd(cursor, (unsigned)kJoinChunk);
+        nbase = __shfl_sync(FULL_MASK, x, 0);
       }
-      const int take = min(__popc(idle), (cur ? qcnt1 : qcnt0) - head);
-      const int rank = __popc(idle & lt);
-      if (!act && rank < take) {
-        const int ei = cur * 32 + head + rank;
-        const int4 r = q_rec[ei];
-        const unsigned long long R0 = q_R0[ei];
-        cp = (cur ? qbase1 : qbase0) + head + rank;
-        cq = r.y;
-        cnq = r.w & 0xff;
-        ca = (unsigned)r.x;
-        cqb = (unsigned)r.w >> 8;
-        cgv = (unsigned)r.z * (unsigned)jp.VQ;
-        leafd = (cnq >= 3 && ((__ldg(&qp_ent[cqb + cnq - 1]).x >> 24) & 1)) ? cnq - 2 : -1;
-        act = true;
-        shared = false;
-        cnt = 0ull;
-        if (cnq == 1) {
-          cnt = (unsigned long long)__popcll(R0);
-          ne = 0u;
-        } else {
-          SM64(myR) = R0;
-          SM64(myU) = 0ull;
-          ne = R0 ? 1u : 0u;
-        }
-      }
-      head += take;
-      idle = __ballot_sync(FULL_MASK, !act);
     }
-    // ---- tail: free lanes take the shallowest open depth of a busy lane ----
-    if (idle) {
-      const unsigned donors = __ballot_sync(FULL_MASK, act && (ne & (ne - 1u)) != 0u);
+    // ---- drained: idle lanes take the shallowest open depth of a busy lane ----
+    const unsigned idle = __ballot_sync(FULL_MASK, ne == 0u && !nv && !pend);
+    if (drained && idle) {
+      const unsigned donors = __ballot_sync(FULL_MASK, (ne & (ne - 1u)) != 0u);
       const int npair = min(__popc(idle), __popc(donors));
       if (npair > 0) {
-        const bool recv = !act && __popc(idle & lt) < npair;
-        const bool give = act && ((donors >> lane) & 1u) && __popc(donors & lt) < npair;
+        const bool recv = ((idle >> lane) & 1u) && __popc(idle & lt) < npair;
+        const bool give = ((donors >> lane) & 1u) && __popc(donors & lt) < npair;
         const int src = recv ? nth_set_bit(donors, __popc(idle & lt)) : lane;
-        const int ds_own = __ffs(ne) - 1;  // shallowest non-empty depth
+        const int ds_own = __ffs(ne) - 1;  // shallowest open depth
         const int ds = __shfl_sync(FULL_MASK, ds_own, src);
-        const long long s_cp = __shfl_sync(FULL_MASK, cp, src);
+        const unsigned s_cp = __shfl_sync(FULL_MASK, cp, src);
         const int s_cq = __shfl_sync(FULL_MASK, cq, src);
-        const int s_cnq = __shfl_sync(FULL_MASK, cnq, src);
-        const int s_leafd = __shfl_sync(FULL_MASK, leafd, src);
+        const unsigned s_info = __shfl_sync(FULL_MASK, cinfo, src);
         const unsigned s_ca = __shfl_sync(FULL_MASK, ca, src);
-        const unsigned s_cqb = __shfl_sync(FULL_MASK, cqb, src);
-        const unsigned s_cgv = __shfl_sync(FULL_MASK, cgv, src);
+        const unsigned s_cmb = __shfl_sync(FULL_MASK, cmb, src);
         if (give && !shared) {
-          // the pair's result is accumulated from several lanes from now on
-          jp.pair_result[cp] = 0ull;
+          jp.pair_result[cp] = 0ull;  // the pair's result is accumulated from several lanes from now on
           shared = true;
         }
         __syncwarp();
         if (recv) {
-          const unsigned dR = oR + 8u * src, dU = oU + 8u * src, dM = oM + src;
-          SM64(myR + 256u * ds) = SM64(dR + 256u * ds);
-          SM64(myU + 256u * ds) = SM64(dU + 256u * ds);
-          for (int j = 0; j < ds; j++) SM8(myM + 32u * j) = SM8(dM + 32u * j);
+          const unsigned dl = (unsigned)(src - lane);  // donor offsets = mine + dl * (8 | 16 | 1)
+          STS128(oRU + 512u * ds) = LDS128(oRU + 512u * ds + 16u * dl);
+          for (int j = 0; j < ds; j++) smem[oM + 32u * j] = smem[oM + 32u * j + dl];
+          cmb = s_cmb;
           cp = s_cp;
           cq = s_cq;
-          cnq = s_cnq;
-          leafd = s_leafd;
+          cinfo = s_info;
+          cqb = s_info >> 16;
           ca = s_ca;
-          cqb = s_cqb;
-          cgv = s_cgv;
           ne = 1u << ds;
           cnt = 0ull;
-          act = true;
           shared = true;
+          pend = false;
         }
         __syncwarp();
         if (give) ne &= ~(1u << ds_own);
       }
     }
-    if (__ballot_sync(FULL_MASK, act) == 0u) break;
+    if (drained && __ballot_sync(FULL_MASK, ne != 0u || nv || pend) == 0u) break;
   }
-#undef SM64
-#undef SM8
   cp_async_wait_all();
   if (jp.stats) {
     unsigned long long s2 = steps;
@@ -2112,6 +2111,15 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     for (int o = 16; o > 0; o >>= 1) s2 += __shfl_xor_sync(FULL_MASK, s2, o);
     if (lane == 0) atomicAdd(jp.stats, s2);
   }
+  __syncthreads();
+  for (int q = threadIdx.x; q < jp.NQ; q += blockDim.x) {
+    const unsigned long long t = ((const unsigned long long *)(smem + o_tot))[q];
+    if (t) atomicAdd(&jp.totals[q], t);
+  }
+#undef LDS64
+#undef STS64
+#undef LDS128
+#undef STS128
 }
 
 template <int MODE>
