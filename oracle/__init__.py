@@ -127,3 +127,12 @@ def count_pairs(Q, D, pq, pg, mode: int = FIND_ALL, nthreads: int | None = None,
     if ovf.value:
         raise OverflowError("oracle count exceeded 2^64-1")
     return OracleResult(out, work.value, ovf.value) if with_work else out
+
+
+def count_totals(Q, D, mode: int = FIND_ALL, nthreads: int | None = None, chunk: int = 100_000):
+    """Per-query sums over all data graphs of count_dense (uint64 [NQ]), in
+    chunks of data graphs so that large batches need no [NQ, ND] array."""
+    tot = np.zeros(Q.num_graphs, np.uint64)
+    for g0 in range(0, D.num_graphs, chunk):
+        tot += count_dense(Q, D.slice(g0, min(g0 + chunk, D.num_graphs)), mode, nthreads).sum(axis=1, dtype=np.uint64)
+    return tot

@@ -1878,6 +1878,23 @@ __device__ __forceinline__ void cp_async8(unsigned dst_smem, const void *src) {
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
+// Number of injective choices (x_0..x_{k-1}), x_i in A_i, 2 <= k <= 4: the
+// inclusion-exclusion over set partitions of {0..k-1}, each block B weighted
+// by (-1)^{|B|-1} (|B|-1)! |AND_{i in B} A_i|.
+__device__ __forceinline__ unsigned long long tail_injective_count(int k, const unsigned long long *A) {
+  const long long a = __popcll(A[0]), b = __popcll(A[1]), ab = __popcll(A[0] & A[1]);
+  if (k == 2) return (unsigned long long)(a * b - ab);
+  const long long c = __popcll(A[2]), ac = __popcll(A[0] & A[2]), bc = __popcll(A[1] & A[2]);
+  const unsigned long long m3 = A[0] & A[1] & A[2];
+  if (k == 3) return (unsigned long long)(a * b * c - ab * c - ac * b - bc * a + 2 * __popcll(m3));
+  const long long d = __popcll(A[3]), ad = __popcll(A[0] & A[3]), bd = __popcll(A[1] & A[3]),
+                  cd = __popcll(A[2] & A[3]);
+  const long long abc = __popcll(m3), abd = __popcll(A[0] & A[1] & A[3]), acd = __popcll(A[0] & A[2] & A[3]),
+                  bcd = __popcll(A[1] & A[2] & A[3]), abcd = __popcll(m3 & A[3]);
+  return (unsigned long long)(a * b * c * d - (ab * c * d + ac * b * d + ad * b * c + bc * a * d + bd * a * c + cd * a * b) +
+                              2 * (abc * d + abd * c + acd * b + bcd * a) + (ab * cd + ac * bd + ad * bc) - 6 * abcd);
+}
+
 // n-th (0-based) set bit of m (m has > n set bits)
 __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
   for (int i = 0; i < n; i++) m &= m - 1u;
@@ -1972,8 +1989,36 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
           X &= __ldg(&adjb[ca + smem[oM + 32u * (be >> 8)] * NB + (unsigned)(be & 255)]);
         }
       }
-      if (e == (int)(cinfo & 0xff) - 1) {
-        cnt += (unsigned long long)__popcll(X);
+      if (e == (int)((cinfo >> 8) & 0xff)) {
+        // tail start t: depths t..n-1 hold pairwise non-adjacent query nodes
+        // whose back-edges all end before t, so their embeddings given the
+        // prefix are the injective choices from their candidate sets A_i
+        const int k = (int)(cinfo & 0xff) - e;
+        if (k == 1) {
+          cnt += (unsigned long long)__popcll(X);
+        } else {
+          unsigned long long A[kJoinTailMax];
+          A[0] = X;
+#pragma unroll
+          for (int i = 1; i < kJoinTailMax; i++) {
+            A[i] = 0ull;
+            if (i < k) {
+              const int4 et = __ldg(&qp_ent[cqb + e + i]);
+              const unsigned t0 = et.x & 15, t1 = (et.x >> 4) & 15;
+              const unsigned k0 = t0 == 15u ? ones : ca + smem[oM + 32u * t0] * NB + (unsigned)et.y;
+              const unsigned k1 = t1 == 15u ? ones : ca + smem[oM + 32u * t1] * NB + (unsigned)et.z;
+              unsigned long long Y =
+                  __ldg(&cmol[cmb + ((et.x >> 12) & 15)]) & ~used & __ldg(&adjb[k0]) & __ldg(&adjb[k1]);
+              const int nex = (et.x >> 8) & 15;
+              for (int x = 0; x < nex; x++) {
+                const int be = __ldg(&jp.qp_be[et.w + x]);
+                Y &= __ldg(&adjb[ca + smem[oM + 32u * (be >> 8)] * NB + (unsigned)(be & 255)]);
+              }
+              A[i] = Y;
+            }
+          }
+          cnt += tail_injective_count(k, A);
+        }
         if (MODE == 1 && cnt) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
         STS128(oRU + 512u * e) = make_ulonglong2(X, used);

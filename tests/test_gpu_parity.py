@@ -214,6 +214,57 @@ def test_c2_full_size_parity(ctx, sigmo):
             assert np.array_equal((bm[:, w] >> b) & 1, (ref_bits[:, w] >> b) & 1), (g, v)
 
 
+def test_c3_bench_workload_parity(ctx, sigmo):
+    """configs[2] (the bench workload: 100 queries x 1M molecules, L=4) in the
+    bench's launch configuration: per-query Find All totals and Find First
+    positive-pair counts over all 1M molecules equal the oracle's; every pair
+    of three sampled 2,000-molecule windows (start, middle, ragged end) is
+    bit-exact."""
+    Q, D = synth.config_queries(3), synth.config_data(3)
+    ctx.load_batch(Q, D)
+    ctx.filter(4)
+    tot = ctx.join(sigmo.SIGMO_FIND_ALL)
+    qt = ctx.query_totals()
+    di, qi, r = ctx.pair_results()
+    ref_q = oracle.count_totals(Q, D)
+    assert np.array_equal(qt, ref_q)
+    assert tot == int(ref_q.sum())
+    ND = D.num_graphs
+    got = {}
+    for g0 in (0, ND // 2 - 1000, ND - 2000):
+        sel = (di >= g0) & (di < g0 + 2000)
+        dense = np.zeros((Q.num_graphs, 2000), np.uint64)
+        dense[qi[sel], di[sel] - g0] = r[sel]
+        ref = oracle.count_dense(Q, D.slice(g0, g0 + 2000))
+        assert np.array_equal(dense, ref), g0
+        got[g0] = ref
+    ctx.join(sigmo.SIGMO_FIND_FIRST)
+    ref_f = oracle.count_totals(Q, D, oracle.FIND_FIRST)
+    assert np.array_equal(ctx.query_totals(), ref_f)
+    di, qi, r = ctx.pair_results()
+    for g0, ref in got.items():
+        sel = (di >= g0) & (di < g0 + 2000)
+        dense = np.zeros((Q.num_graphs, 2000), np.uint64)
+        dense[qi[sel], di[sel] - g0] = r[sel]
+        assert np.array_equal(dense, (ref > 0).astype(np.uint64)), g0
+
+
+def test_join_tail_closed_form(sigmo, monkeypatch):
+    """Planner option SIGMO_TAIL_MAX=4 (independent tail of <= 4 query nodes
+    counted by inclusion-exclusion in k_join_lane): results unchanged."""
+    monkeypatch.setenv("SIGMO_TAIL_MAX", "4")
+    Q, D = synth.config_queries(2), synth.config_data(2, count=20000)
+    ref = oracle.count_dense(Q, D)
+    with sigmo.Context(0) as c:
+        c.load_batch(Q, D)
+        for L in (1, 4):
+            c.filter(L)
+            c.join(sigmo.SIGMO_FIND_ALL)
+            assert np.array_equal(c.dense_results(), ref), L
+            c.join(sigmo.SIGMO_FIND_FIRST)
+            assert np.array_equal(c.dense_results(), (ref > 0).astype(np.uint64)), L
+
+
 def test_join_stack_spill_path(sigmo, monkeypatch):
     """Force the smallest shared-memory DFS stack so that the global spill /
     restore path runs (deep 20-30-atom ring-system queries), results unchanged."""
