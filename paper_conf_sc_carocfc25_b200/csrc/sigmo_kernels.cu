@@ -454,10 +454,9 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   L.pl = o;       o = align16(o + 4 * (size_t)plane_stride(NLAB, P) * EXTW);
   L.fpl = o;      o = align16(o + 4 * (size_t)(NFU > 0 ? NFU : 1) * EXTW);
   L.memb = o;     o = align16(o + 4 * 32 * (size_t)EXTW);
-  // window path: per warp one molecule's channel windows; molecule tiles
-  // (mol): every channel window of the tile's 32 molecules, [channel][molecule]
-  L.win = o;      o = align16(o + mb * (size_t)(mol ? 32 : NWARP) * NCH);
-  L.nz = o;       o = align16(o + 4 * (size_t)NWARP * (VQW + 1));
+  // window path (dense tiles): per warp one molecule's channel windows
+  L.win = o;      o = align16(o + mb * (size_t)(mol ? 0 : NWARP) * NCH);
+  L.nz = o;       o = align16(o + (mol ? 0 : 4 * (size_t)NWARP * (VQW + 1)));
   L.gmb = o;      o = align16(o + 4 * (size_t)MOLCAP * (NQW > 0 ? NQW : 1));
   L.slotat = o;   o = align16(o + 2 * 32 * 32);
   L.endb = o;     o = align16(o + 4 * 32);
@@ -803,41 +802,79 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   }
 
   if (MOL) {
-    // ---- molecule tiles: channel windows of the 32 molecules, then rows with
-    // lane = molecule: the window of C_L = AND of the row's channel windows,
-    // written once to cmol[g][row]; GMCR: every row non-empty ----
-    const int NCHm = NLAB + 1 + fp.P;
-    M *win = s_win;  // [channel][32 molecules]
-    for (int t = tid; t < NCHm * 32; t += NT) {
-      const int c = t >> 5, mi = t & 31;
-      M w;
-      w.clear();
-      if (mi < nmol) {
-        const int ms = s_mstart[mi], n = s_mstart[mi + 1] - ms;
-        w = extract_window_strided<NW>(s_pl + c, PS, nxw, ms, n);
-      }
-      win[t] = w;
-    }
-    __syncthreads();
+    // ---- molecule tiles: rows in the word domain (lane = 32-node word k of
+    // the tile, C_L word = AND of the row's plane words, as in the dense
+    // path), then lane = molecule gathers its <= 3 words by shuffles and
+    // writes its window once to cmol[g][row]; GMCR: every row
+    // of the query non-empty ----
     const int mi = lane;
     const bool valid = mi < nmol;
-    const int RW = fp.RW;
+    const int ms = valid ? s_mstart[mi] : 0;
+    const int n = valid ? s_mstart[mi + 1] - ms : 0;
+    const unsigned long long nmask = n >= 64 ? ~0ull : ((1ull << n) - 1ull);
+    const int ws = ms >> 5, sh = ms & 31;
     const uint32_t *rowp = fp.rows_smem ? (const uint32_t *)(smem + L.rowp) : fp.rowp;
     unsigned long long *cm = fp.cmol + (size_t)(g0 + mi) * fp.VQ;  // molecule-major: cmol[g][row]
-    for (int q = wid; q < fp.NQ; q += NWARP) {
-      const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
-      bool all = valid;
-      for (int row = r0; row < r1; row++) {
-        const uint32_t *pr = rowp + (size_t)row * RW;
-        unsigned long long x = ~0ull;
-        for (int j = 0; j < RW; j++) {
-          const uint32_t two = pr[j];
-          x &= win[((two & 0xffffu) >> 2) * 32 + mi].w[0] & win[(two >> 18) * 32 + mi].w[0];
+    auto mol_rows = [&](auto RWc, auto HIc, const uint32_t *rowp) {
+      constexpr int RWk = decltype(RWc)::value;
+      constexpr bool HI = decltype(HIc)::value;  // the tile spans more than 32 words
+      const int RW = RWk ? RWk : fp.RW;
+      const unsigned char *pl0 = (const unsigned char *)(s_pl + (size_t)(lane < nxw ? lane : 0) * PS);
+      const unsigned char *pl1 = (const unsigned char *)(s_pl + (size_t)(lane + 32 < nxw ? lane + 32 : 0) * PS);
+      for (int q = wid; q < fp.NQ; q += NWARP) {
+        const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
+        bool all = valid;
+        const uint32_t *pr = rowp + (size_t)r0 * RW;
+        for (int row = r0; row < r1; row++, pr += RW) {
+          uint32_t x0 = 0xffffffffu, x1 = 0xffffffffu;
+#pragma unroll
+          for (int j = 0; j < (RWk ? RWk : 1); j++) {
+            const uint32_t two = pr[j];
+            x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
+            if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
+          }
+          for (int j = RWk; j < RW; j++) {
+            const uint32_t two = pr[j];
+            x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
+            if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
+          }
+          uint32_t w0, w1, w2;
+          if (HI) {
+            const uint32_t a0 = __shfl_sync(FULL_MASK, x0, ws & 31), b0 = __shfl_sync(FULL_MASK, x1, ws & 31);
+            const uint32_t a1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31), b1 = __shfl_sync(FULL_MASK, x1, (ws + 1) & 31);
+            const uint32_t a2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31), b2 = __shfl_sync(FULL_MASK, x1, (ws + 2) & 31);
+            w0 = ws < 32 ? a0 : b0;
+            w1 = ws + 1 < 32 ? a1 : b1;
+            w2 = ws + 2 < 32 ? a2 : b2;
+          } else {
+            w0 = __shfl_sync(FULL_MASK, x0, ws);
+            w1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31);
+            w2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31);
+          }
+          const unsigned long long x =
+              (((unsigned long long)__funnelshift_r(w1, w2, sh) << 32) | __funnelshift_r(w0, w1, sh)) & nmask;
+          if (valid) cm[row] = x;
+          all = all && x != 0ull;
         }
-        if (valid) cm[row] = x;
-        all = all && x != 0ull;
+        if (all) atomicOr(&s_gm[mi * fp.NQW + (q >> 5)], 1u << (q & 31));
       }
-      if (all) atomicOr(&s_gm[mi * fp.NQW + (q >> 5)], 1u << (q & 31));
+    };
+    const bool hi = nxw > 32;
+    if (fp.rows_smem) {
+      const uint32_t *rs = (const uint32_t *)(smem + L.rowp);
+      switch (hi ? 0 : fp.RW) {
+        case 1: mol_rows(std::integral_constant<int, 1>{}, std::false_type{}, rs); break;
+        case 2: mol_rows(std::integral_constant<int, 2>{}, std::false_type{}, rs); break;
+        case 3: mol_rows(std::integral_constant<int, 3>{}, std::false_type{}, rs); break;
+        case 4: mol_rows(std::integral_constant<int, 4>{}, std::false_type{}, rs); break;
+        default:
+          if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, rs);
+          else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, rs);
+          break;
+      }
+    } else {
+      if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, fp.rowp);
+      else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, fp.rowp);
     }
   }
 
