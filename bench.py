@@ -33,8 +33,11 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 BASELINE_METRIC = "matches/sec (Find All) and graph-pairs/sec (Find First) at 1/2/4/8 B200"
-# BASELINE.json configs[i] -> synth config id i+1, molecules per rank
-CONFIGS = {1: (2, 100_000), 2: (3, 1_000_000)}
+# BASELINE.json configs[i] -> synth config id i+1, molecules per rank.
+# configs[3]/[4] are 8-GPU configurations: the per-rank default is the 8-GPU
+# share (1M / 8 and 10M / 8), so `--gpus 8` processes the whole config.
+CONFIGS = {1: (2, 100_000), 2: (3, 1_000_000), 3: (4, 125_000), 4: (5, 1_250_000)}
+STREAM_BATCH = 250_000        # configs[4]: molecules per streamed batch per GPU
 LEVELS = 4
 CPU_SAMPLE_MOLS = 200_000     # cpu_baseline leg: oracle on the first 200k molecules (~100 core-seconds)
 REF_STEP_MOLS = 2_000         # --impl reference: molecules per step
@@ -228,13 +231,16 @@ def run_reference(args, world, rank):
 
 
 def config_dict(args, world, oracle_step=None):
-    nq = {2: 50, 3: 100}[args.cid]
+    nq = {2: 50, 3: 100, 4: 500, 5: 1000}[args.cid]
+    mode = "Find First" if args.cid == 4 else "Find All"
+    extra = f", streamed in batches of {STREAM_BATCH}" if args.cid == 5 else ""
     d = {"workload": f"configs[{args.config}]: {nq} queries x {args.molecules} ZINC-like molecules per GPU, "
-                     f"Find All, levels={args.levels}",
+                     f"{mode}, levels={args.levels}{extra}",
          "queries": nq, "molecules_per_gpu": args.molecules, "molecules_total": args.molecules * world,
-         "levels": args.levels, "mode": "find_all", "data_seed": hex(0x51C0_0000 + args.cid),
+         "levels": args.levels, "mode": "find_first" if args.cid == 4 else "find_all", "data_seed": hex(0x51C0_0000 + args.cid),
          "query_seed": hex(0x9E00_0000 + args.cid),
-         "l2": "flushed before every timed step (256 MiB device write, outside the events)",
+         "l2": ("flushed before every timed step (256 MiB device write, outside the events)" if args.cid in (2, 3)
+                else "no flush: per-step inputs and candidate arrays are larger than the 126 MB L2"),
          "parallelism": f"dp{world}: molecule shards, queries replicated, NCCL all-reduce of per-query totals"}
     if oracle_step:
         d["oracle_molecules_per_step"] = oracle_step
@@ -247,6 +253,9 @@ def main():
     world, rank, local = dist_setup(args)
     if args.impl == "reference":
         run_reference(args, world, rank)
+        return
+    if args.cid in (4, 5):
+        run_routed(args, world, rank, local)
         return
     import numpy as np
     import torch
@@ -405,6 +414,119 @@ def main():
         line["cpu_baseline"] = run_cpu_baseline(Q, args)
     print(json.dumps(line), flush=True)
     ctx.close()
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+def run_routed(args, world, rank, local):
+    """configs[3] (500 queries incl. 20-30-atom ring systems, Find First) and
+    configs[4] (1,000 queries, Find All, batches of 250k streamed through two
+    double-buffered contexts): queries routed by size (stream.split_queries).
+    configs[3]: data resident, a step = filter + join of both query groups,
+    device-timed.  configs[4]: a step = the whole stream (host pack + H2D of
+    every batch overlapped with the kernels of the previous one), wall clock
+    between device synchronisations."""
+    import numpy as np
+    import torch
+
+    import synth
+    import paper_conf_sc_carocfc25_b200 as sigmo
+    from paper_conf_sc_carocfc25_b200 import sharded, stream
+
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+    Q = synth.config_queries(args.cid)
+    first = rank * args.molecules
+    ff = args.cid == 4
+    mode = sigmo.SIGMO_FIND_FIRST if ff else sigmo.SIGMO_FIND_ALL
+    if args.cid == 5:
+        nb = (args.molecules + STREAM_BATCH - 1) // STREAM_BATCH
+        batches = [sigmo.as_c_batch(synth.config_data(5, first=first + i * STREAM_BATCH,
+                                                      count=min(STREAM_BATCH, args.molecules - i * STREAM_BATCH)))
+                   for i in range(nb)]
+    else:
+        batches = [sigmo.as_c_batch(synth.config_data(4, first=first, count=args.molecules))]
+    sr = stream.StreamRunner(Q, local, levels=args.levels, mode=mode)
+    totals_dev = torch.zeros(Q.num_graphs, dtype=torch.int64, device=dev)
+    if args.cid == 4:
+        for gi, (_, qb) in enumerate(sr.groups):
+            sr.ctx[0][gi].load_batch(qb, batches[0])
+
+    def step():
+        if args.cid == 5:
+            t = sr.run(batches)
+        else:
+            with torch.cuda.stream(sr.streams[0]):
+                for c in sr.ctx[0]:
+                    c.filter(args.levels)
+                    c.join(mode, total=False)
+            t = None
+        return t
+
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize(dev)
+    K = args.steps
+    sampler = ClockSampler(local)
+    if dist is not None:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    with sampler:
+        if args.cid == 5:
+            t0 = time.perf_counter()
+            for _ in range(K):
+                t = step()
+            torch.cuda.synchronize(dev)
+            ms = (time.perf_counter() - t0) * 1000
+        else:
+            s = sr.streams[0]
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            for _ in range(K):
+                step()
+            e1.record(s)
+            torch.cuda.synchronize(dev)
+            ms = e0.elapsed_time(e1)
+    clocks = sampler.summary()
+    if args.cid == 5:
+        local_tot = sr.run(batches)
+    else:
+        local_tot = np.zeros(Q.num_graphs, np.uint64)
+        for gi, (idx, _) in enumerate(sr.groups):
+            c = sr.ctx[0][gi]
+            c.join(mode, total=False)
+            local_tot[idx] = c.query_totals()
+    totals_dev.copy_(torch.from_numpy(local_tot.astype(np.int64)))
+    sharded.allreduce_totals(totals_dev)
+    nd_local = sum(b.num_graphs for b in batches)
+    vals = torch.tensor([ms], dtype=torch.float64, device=dev)
+    cnts = torch.tensor([nd_local], dtype=torch.int64, device=dev)
+    if dist is not None:
+        dist.all_reduce(vals, op=dist.ReduceOp.MAX)
+        dist.all_reduce(cnts)
+    ms = float(vals.item())
+    nd_all = int(cnts.item())
+    total = int(totals_dev.sum().item())
+    if rank == 0:
+        if ff:
+            value, unit = Q.num_graphs * nd_all * K / (ms / 1000.0), "graph-pairs/s"
+        else:
+            value, unit = total * K / (ms / 1000.0), "matches/s"
+        launches = sum(c.timings()["filter_launches"] + c.timings()["join_launches"] for c in sr.ctx[0])
+        line = {
+            "metric": BASELINE_METRIC, "value": value, "unit": unit, "n_gpus": world, "steps": K,
+            "warmup": max(args.warmup, 3), "ms_per_step": ms / K, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u64", "data": "synthetic", "config": config_dict(args, world),
+            "counts": {"matches" if not ff else "positive_pairs": total, "all_pairs": Q.num_graphs * nd_all},
+            "query_groups": [int(len(g)) for g, _ in sr.groups],
+            "timing": "wall clock incl. host pack + H2D of every batch" if args.cid == 5 else "device events",
+            "gpu_launches": int(K * launches * (len(batches) if args.cid == 5 else 1)),
+            "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    sr.close()
     if dist is not None:
         dist.destroy_process_group()
 

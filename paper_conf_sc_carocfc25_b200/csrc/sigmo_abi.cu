@@ -1343,7 +1343,9 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       jp.adjb = (const unsigned long long *)c->adjb.p;
       jp.qp_ent = c->qp_ent;
       jp.cmol = (const unsigned long long *)c->bitmap.p;
-      jp.batchK = 4;
+      // refill batch (lanes that must be free before a warp refills): swept on
+      // configs[2], FA 2/4/8/16 -> 11.2/10.3/9.7/9.9 ms, FF 10.4/9.8/9.2/9.0 ms
+      jp.batchK = mode == SIGMO_FIND_FIRST ? 16 : 8;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
       const size_t smem = join_lane_smem_bytes(jp);
       if (smem > c->max_smem) return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);

@@ -2209,6 +2209,10 @@ static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_
   cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)p.smem_bytes);
   if (e != cudaSuccess) return e;
+  if (const char *v = getenv("SIGMO_JOIN_CARVE")) {  // experiment: shared-memory carve-out (percent of L1+smem)
+    e = cudaFuncSetAttribute(k_join_lane<MODE>, cudaFuncAttributePreferredSharedMemoryCarveout, atoi(v));
+    if (e != cudaSuccess) return e;
+  }
   k_join_lane<MODE><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
