@@ -376,70 +376,8 @@ struct QPlan {
   std::vector<int32_t> beoff;   // [VQ+1]
   std::vector<uint16_t> be;     // (j << 8) | class
   std::vector<uint32_t> info;   // [VQ] two back-edges inline + #extra + leaf-sum flag (see plan_queries)
-  std::vector<uint32_t> qinfo;  // [NQ] nq | tail start t << 8 | first query node << 16 (k_join_lane)
+  std::vector<uint32_t> qinfo;  // [NQ] nq | last depth n-1 << 8 | first query node << 16 (k_join_lane)
 };
-
-// Independent tail of a query (k_join_lane): the largest set S of <= 4
-// pairwise non-adjacent nodes (|S| <= n-1) whose removal splits no connected
-// component.  Placed last in the matching order, the embeddings of S given a
-// prefix embedding are the injective choices from the per-node candidate
-// sets, counted in closed form (inclusion-exclusion over set partitions).
-// Ties: the larger data-label frequency (rare labels stay early to prune).
-uint32_t choose_tail(const HostGraphs &q, int64_t lo, int n, const std::vector<int64_t> &freq) {
-  if (n < 2 || n > kJoinLaneMaxQ) return 0u;
-  std::vector<uint32_t> adj(n, 0u);
-  for (int u = 0; u < n; u++)
-    for (int64_t e = q.roff[lo + u]; e < q.roff[lo + u + 1]; e++) adj[u] |= 1u << (q.col[e] - lo);
-  auto comps = [&](uint32_t keep) {
-    int c = 0;
-    uint32_t left = keep;
-    while (left) {
-      uint32_t fr = left & (0u - left), seen = 0u;
-      while (fr) {
-        seen |= fr;
-        uint32_t nx = 0u;
-        for (uint32_t f = fr; f; f &= f - 1u) nx |= adj[__builtin_ctz(f)];
-        fr = nx & keep & ~seen;
-      }
-      left &= ~seen;
-      c++;
-    }
-    return c;
-  };
-  const uint32_t all = (n == 32) ? 0xffffffffu : ((1u << n) - 1u);
-  const int c0 = comps(all);
-  // default off: measured on configs[2] (100 x 1M, L=4), k <= 2/3/4 cut DFS
-  // steps 1.11G -> 0.91/0.82/0.80G but the divergent tail evaluation raised
-  // the join 10.3 -> 12.1/13.5/14.3 ms
-  int kmax = 1;
-  if (const char *e = getenv("SIGMO_TAIL_MAX")) kmax = std::max(1, std::min(kJoinTailMax, atoi(e)));
-  for (int k = std::min(kmax, n - 1); k >= 2; k--) {
-    uint32_t best = 0u;
-    int64_t bf = -1;
-    // subsets of size k in increasing order (Gosper's hack)
-    for (uint32_t s = (1u << k) - 1u; s <= all && s != 0u;) {
-      bool indep = true;
-      int iso = 0;
-      int64_t f = 0;
-      for (uint32_t t = s; t && indep; t &= t - 1u) {
-        const int u = __builtin_ctz(t);
-        indep = (adj[u] & s) == 0u;
-        iso += adj[u] == 0u;
-        f += freq[q.nlab[lo + u]];
-      }
-      if (indep && comps(all & ~s) + iso == c0 && f > bf) {
-        best = s;
-        bf = f;
-      }
-      const uint32_t c = s & (0u - s), r = s + c;
-      if (r == 0u) break;
-      s = (((r ^ s) >> 2) / c) | r;
-    }
-    if (best) return best;
-  }
-  // k = 1: the last node of the greedy order (any node is a valid tail of one)
-  return 0u;
-}
 
 void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const uint8_t *bclass, QPlan &out) {
   out.row.assign((size_t)q.V, 0);
@@ -453,16 +391,13 @@ void plan_queries(const HostGraphs &q, const std::vector<int64_t> &freq, const u
     std::vector<int> pos(n, -1), order;
     auto deg = [&](int u) { return (int)(q.roff[lo + u + 1] - q.roff[lo + u]); };
     auto fr = [&](int u) { return freq[q.nlab[lo + u]]; };
-    const uint32_t tail = choose_tail(q, lo, n, freq);
-    const int ntail = __builtin_popcount(tail);
-    // tail start: the closed form covers depths t..n-1 (t = n - max(|S|, 1))
-    const int t = n <= 1 ? n : n - std::max(ntail, 1);
+    // qinfo: n | (n - 1) << 8 (the last depth, counted by popc) | first query node << 16
+    const int t = n <= 1 ? n : n - 1;
     out.qinfo[g] = (uint32_t)n | ((uint32_t)t << 8) | ((uint32_t)lo << 16);
     for (int i = 0; i < n; i++) {
       int best = -1, bc = -1;
       for (int u = 0; u < n; u++) {
         if (pos[u] >= 0) continue;
-        if (i < n - ntail && u < 32 && ((tail >> u) & 1u)) continue;  // the tail goes last
         int conn = 0;
         for (int64_t e = q.roff[lo + u]; e < q.roff[lo + u + 1]; e++)
           if (pos[q.col[e] - lo] >= 0) conn++;

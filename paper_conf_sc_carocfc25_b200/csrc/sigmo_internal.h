@@ -197,7 +197,6 @@ size_t join_lane_smem_bytes(const JoinParams &p);
 int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem);
 constexpr int kJoinLaneThreads = 128;
 constexpr int kJoinLaneMaxQ = 11;  // k_join_lane handles queries <= 11 nodes in <= 64-node graphs (map: 6 bits x 10 depths)
-constexpr int kJoinTailMax = 4;   // k_join_lane: closed-form independent tail of <= 4 query nodes (planner choose_tail)
 size_t join_smem_bytes(int NW, const JoinParams &p);
 size_t join_gstack_bytes(int NW, const JoinParams &p, int grid);
 int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem);

@@ -1793,7 +1793,8 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
       const long long p = o + __popc(bits & lt);
       pp.pair_query[p] = q;
       if (pp.prec) {
-        const uint32_t qi = __ldg(&pp.qinfo[q]);
+        // query info with the molecule size in bits 8-15 (class stride of adjb)
+        const uint32_t qi = (__ldg(&pp.qinfo[q]) & ~0xff00u) | ((uint32_t)(__ldg(&pp.goff[g + 1]) - a) << 8);
         pp.prec[p] = make_int4(a, q, (int)((unsigned)g * (unsigned)pp.VQ + (qi >> 16)), (int)qi);
       }
     }
@@ -1835,8 +1836,11 @@ cudaError_t launch_unpad(const unsigned long long *cmol, const int32_t *goff, in
 }
 
 // ===========================================================================
-// Bond-class adjacency masks adjb[v * NB + b] (molecule-local bits of the
-// neighbours of v joined by a bond of class b), for <= 64-node graphs.
+// Bond-class adjacency masks (molecule-local bits of the neighbours of v
+// joined by a bond of class b), for <= 64-node graphs, class-major inside
+// each molecule: adjb[a * NB + b * n + (v - a)] for the molecule [a, a + n)
+// holding v, so that lanes reading the same class of one molecule touch few
+// 32-B sectors.
 // ===========================================================================
 __global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, unsigned long long *adjb) {
   const int v = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1852,9 +1856,11 @@ __global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, unsigned long
     for (int b = 0; b < 8; b++)
       if (cls == b) m[b] |= 1ull << ((x >> 8) & 63);
   }
+  const int g = graph_of(d.goff, d.num_graphs, v);
+  const int a = d.goff[g], n = d.goff[g + 1] - a;
 #pragma unroll
   for (int b = 0; b < 8; b++)
-    if (b < NB) adjb[(size_t)v * NB + b] = m[b];
+    if (b < NB) adjb[(size_t)a * NB + (size_t)b * n + (v - a)] = m[b];
 }
 
 cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsigned long long *adjb, cudaStream_t st) {
@@ -1900,37 +1906,17 @@ __host__ __device__ inline size_t join_lane_warp_bytes(int MQ) {
   return 512 * (size_t)SD + 512;
 }
 // CTA: per-query totals [NQ] u64, then one region per warp
-__host__ __device__ inline size_t join_lane_cta_bytes(int VQ, int NQ) {
-  (void)VQ;
-  return align16(8 * (size_t)(NQ > 0 ? NQ : 1));
+__host__ __device__ inline size_t join_lane_cta_bytes(int NQ) { return align16(8 * (size_t)(NQ > 0 ? NQ : 1)); }
+__host__ __device__ inline size_t join_lane_smem(int NQ, int MQ) {
+  return join_lane_cta_bytes(NQ) + join_lane_warp_bytes(MQ) * (kJoinLaneThreads / 32);
 }
-__host__ __device__ inline size_t join_lane_smem(int VQ, int NQ, int MQ) {
-  return join_lane_cta_bytes(VQ, NQ) + join_lane_warp_bytes(MQ) * (kJoinLaneThreads / 32);
-}
-size_t join_lane_smem_bytes(const JoinParams &p) { return join_lane_smem(p.VQ, p.NQ, p.maxq); }
+size_t join_lane_smem_bytes(const JoinParams &p) { return join_lane_smem(p.NQ, p.maxq); }
 
 __device__ __forceinline__ void cp_async8(unsigned dst_smem, const void *src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(dst_smem), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
-
-// Number of injective choices (x_0..x_{k-1}), x_i in A_i, 2 <= k <= 4: the
-// inclusion-exclusion over set partitions of {0..k-1}, each block B weighted
-// by (-1)^{|B|-1} (|B|-1)! |AND_{i in B} A_i|.
-__device__ __forceinline__ unsigned long long tail_injective_count(int k, const unsigned long long *A) {
-  const long long a = __popcll(A[0]), b = __popcll(A[1]), ab = __popcll(A[0] & A[1]);
-  if (k == 2) return (unsigned long long)(a * b - ab);
-  const long long c = __popcll(A[2]), ac = __popcll(A[0] & A[2]), bc = __popcll(A[1] & A[2]);
-  const unsigned long long m3 = A[0] & A[1] & A[2];
-  if (k == 3) return (unsigned long long)(a * b * c - ab * c - ac * b - bc * a + 2 * __popcll(m3));
-  const long long d = __popcll(A[3]), ad = __popcll(A[0] & A[3]), bd = __popcll(A[1] & A[3]),
-                  cd = __popcll(A[2] & A[3]);
-  const long long abc = __popcll(m3), abd = __popcll(A[0] & A[1] & A[3]), acd = __popcll(A[0] & A[2] & A[3]),
-                  bcd = __popcll(A[1] & A[2] & A[3]), abcd = __popcll(m3 & A[3]);
-  return (unsigned long long)(a * b * c * d - (ab * c * d + ac * b * d + ad * b * c + bc * a * d + bd * a * c + cd * a * b) +
-                              2 * (abc * d + abd * c + acd * b + bcd * a) + (ab * cd + ac * bd + ad * bc) - 6 * abcd);
-}
 
 // n-th (0-based) set bit of m (m has > n set bits)
 __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
@@ -1950,7 +1936,10 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   // ---- CTA tables ----
   const unsigned o_tot = 0u;
   for (int i = threadIdx.x; i < jp.NQ; i += blockDim.x) ((unsigned long long *)(smem + o_tot))[i] = 0ull;
-  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.VQ, jp.NQ) + (size_t)wid * join_lane_warp_bytes(MQ));
+  // plan entry of plan position i, read through L1 (a shared-memory copy was
+  // measured slower: 15.5 vs 10.0 ms on configs[2])
+  const int4 *const qp_ent = jp.qp_ent;
+  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ) + (size_t)wid * join_lane_warp_bytes(MQ));
   const unsigned oRU = wbase + 16u * lane;                        // {R, U} of depth d: oRU + 512 d
   const unsigned oM = wbase + 512u * SD + lane;                   // f(pi_d): oM + 32 d
   smem[oM + 32 * 15] = 0;  // map slot 15 (absent back-edge) reads node 0 of the all-ones class
@@ -1963,7 +1952,6 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   const unsigned long long *const cmol = jp.cmol;
   const unsigned NB = (unsigned)jp.NB;
   const unsigned ones = (unsigned)jp.VD * NB;  // the all-ones entry (absent back-edge)
-  const int4 *const qp_ent = jp.qp_ent;
   const int4 zero4 = make_int4(0, 0, 0, 0);
 
   // ---- GMCR chunks: current (records of pairs cbase + i in lane i's crec), prefetched, claimed ----
@@ -2016,46 +2004,19 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const unsigned long long used = RU.y | bit;
       // candidates of depth e
       const unsigned u0 = j0 == (unsigned)d ? (unsigned)v : m0, u1 = j1 == (unsigned)d ? (unsigned)v : m1;
-      const unsigned i0 = j0 == 15u ? ones : ca + u0 * NB + (unsigned)en.y;
-      const unsigned i1 = j1 == 15u ? ones : ca + u1 * NB + (unsigned)en.z;
+      const unsigned ng = (cinfo >> 8) & 0xffu;  // molecule size: class stride of adjb
+      const unsigned i0 = j0 == 15u ? ones : ca + (unsigned)en.y * ng + u0;
+      const unsigned i1 = j1 == 15u ? ones : ca + (unsigned)en.z * ng + u1;
       unsigned long long X = __ldg(&cmol[cmb + ((en.x >> 12) & 15)]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
       if (en.x & 0xf00) {  // > 2 back-edges at this depth (fused rings): rare
         const int nex = (en.x >> 8) & 15;
         for (int k = 0; k < nex; k++) {
           const int be = __ldg(&jp.qp_be[en.w + k]);
-          X &= __ldg(&adjb[ca + smem[oM + 32u * (be >> 8)] * NB + (unsigned)(be & 255)]);
+          X &= __ldg(&adjb[ca + (unsigned)(be & 255) * ng + smem[oM + 32u * (be >> 8)]]);
         }
       }
-      if (e == (int)((cinfo >> 8) & 0xff)) {
-        // tail start t: depths t..n-1 hold pairwise non-adjacent query nodes
-        // whose back-edges all end before t, so their embeddings given the
-        // prefix are the injective choices from their candidate sets A_i
-        const int k = (int)(cinfo & 0xff) - e;
-        if (k == 1) {
-          cnt += (unsigned long long)__popcll(X);
-        } else {
-          unsigned long long A[kJoinTailMax];
-          A[0] = X;
-#pragma unroll
-          for (int i = 1; i < kJoinTailMax; i++) {
-            A[i] = 0ull;
-            if (i < k) {
-              const int4 et = __ldg(&qp_ent[cqb + e + i]);
-              const unsigned t0 = et.x & 15, t1 = (et.x >> 4) & 15;
-              const unsigned k0 = t0 == 15u ? ones : ca + smem[oM + 32u * t0] * NB + (unsigned)et.y;
-              const unsigned k1 = t1 == 15u ? ones : ca + smem[oM + 32u * t1] * NB + (unsigned)et.z;
-              unsigned long long Y =
-                  __ldg(&cmol[cmb + ((et.x >> 12) & 15)]) & ~used & __ldg(&adjb[k0]) & __ldg(&adjb[k1]);
-              const int nex = (et.x >> 8) & 15;
-              for (int x = 0; x < nex; x++) {
-                const int be = __ldg(&jp.qp_be[et.w + x]);
-                Y &= __ldg(&adjb[ca + smem[oM + 32u * (be >> 8)] * NB + (unsigned)(be & 255)]);
-              }
-              A[i] = Y;
-            }
-          }
-          cnt += tail_injective_count(k, A);
-        }
+      if (e == (int)(cinfo & 0xff) - 1) {
+        cnt += (unsigned long long)__popcll(X);
         if (MODE == 1 && cnt) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
         STS128(oRU + 512u * e) = make_ulonglong2(X, used);
@@ -2093,7 +2054,6 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       cqb = cinfo >> 16;
       shared = false;
       cnt = 0ull;
-      const int4 en0 = __ldg(&qp_ent[cqb]);
       const unsigned long long R0 = nR0;
       if ((cinfo & 0xff) == 1u) {
         cnt = (unsigned long long)__popcll(R0);
@@ -2209,10 +2169,6 @@ static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_
   cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)p.smem_bytes);
   if (e != cudaSuccess) return e;
-  if (const char *v = getenv("SIGMO_JOIN_CARVE")) {  // experiment: shared-memory carve-out (percent of L1+smem)
-    e = cudaFuncSetAttribute(k_join_lane<MODE>, cudaFuncAttributePreferredSharedMemoryCarveout, atoi(v));
-    if (e != cudaSuccess) return e;
-  }
   k_join_lane<MODE><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
@@ -2222,21 +2178,20 @@ cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream
   return mode == 1 ? launch_join_lane_t<1>(p, grid, st) : launch_join_lane_t<0>(p, grid, st);
 }
 
-int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem) {
+template <int MODE>
+static int join_lane_occ_t(size_t smem) {
   int n = 0;
-  cudaError_t e;
-  if (mode == 1) {
-    cudaFuncSetAttribute(k_join_lane<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<1>, kJoinLaneThreads, smem);
-  } else {
-    cudaFuncSetAttribute(k_join_lane<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<0>, kJoinLaneThreads, smem);
-  }
-  if (e != cudaSuccess) {
+  cudaFuncSetAttribute(k_join_lane<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE>, kJoinLaneThreads, smem) != cudaSuccess) {
     cudaGetLastError();
     return 1;
   }
   return n < 1 ? 1 : n;
+}
+
+int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem) {
+  (void)p;
+  return mode == 1 ? join_lane_occ_t<1>(smem) : join_lane_occ_t<0>(smem);
 }
 
 }  // namespace sigmo

@@ -249,22 +249,6 @@ def test_c3_bench_workload_parity(ctx, sigmo):
         assert np.array_equal(dense, (ref > 0).astype(np.uint64)), g0
 
 
-def test_join_tail_closed_form(sigmo, monkeypatch):
-    """Planner option SIGMO_TAIL_MAX=4 (independent tail of <= 4 query nodes
-    counted by inclusion-exclusion in k_join_lane): results unchanged."""
-    monkeypatch.setenv("SIGMO_TAIL_MAX", "4")
-    Q, D = synth.config_queries(2), synth.config_data(2, count=20000)
-    ref = oracle.count_dense(Q, D)
-    with sigmo.Context(0) as c:
-        c.load_batch(Q, D)
-        for L in (1, 4):
-            c.filter(L)
-            c.join(sigmo.SIGMO_FIND_ALL)
-            assert np.array_equal(c.dense_results(), ref), L
-            c.join(sigmo.SIGMO_FIND_FIRST)
-            assert np.array_equal(c.dense_results(), (ref > 0).astype(np.uint64)), L
-
-
 def test_join_stack_spill_path(sigmo, monkeypatch):
     """Force the smallest shared-memory DFS stack so that the global spill /
     restore path runs (deep 20-30-atom ring-system queries), results unchanged."""
