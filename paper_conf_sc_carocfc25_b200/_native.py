@@ -57,7 +57,7 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
     global _lib
     if _lib is not None:
         return _lib
-    path = path or LIB_PATH
+    path = path or os.environ.get("SIGMO_LIB") or LIB_PATH  # SIGMO_LIB: alternative in-tree build (experiments)
     if not os.path.exists(path):
         raise RuntimeError(f"libsigmo.so not found at {path}: build it with "
                            f"`python -c 'import __graft_entry__ as g; g.build()'` (there is no CPU fallback)")

@@ -813,7 +813,6 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
     const int n = valid ? s_mstart[mi + 1] - ms : 0;
     const unsigned long long nmask = n >= 64 ? ~0ull : ((1ull << n) - 1ull);
     const int ws = ms >> 5, sh = ms & 31;
-    const uint32_t *rowp = fp.rows_smem ? (const uint32_t *)(smem + L.rowp) : fp.rowp;
     unsigned long long *cm = fp.cmol + (size_t)(g0 + mi) * fp.VQ;  // molecule-major: cmol[g][row]
     auto mol_rows = [&](auto RWc, auto HIc, const uint32_t *rowp) {
       constexpr int RWk = decltype(RWc)::value;
@@ -1936,8 +1935,10 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   // ---- CTA tables ----
   const unsigned o_tot = 0u;
   for (int i = threadIdx.x; i < jp.NQ; i += blockDim.x) ((unsigned long long *)(smem + o_tot))[i] = 0ull;
-  // plan entry of plan position i, read through L1 (a shared-memory copy was
-  // measured slower: 15.5 vs 10.0 ms on configs[2])
+  // plan entry of plan position i, read through L1 (measured on configs[2]: a
+  // shared-memory copy of the entries 15.5 vs 10.0 ms; staging each pair's
+  // candidate rows in lane-private shared memory by cp.async, 10.6 vs 9.8 ms
+  // -- both lose to the occupancy they cost)
   const int4 *const qp_ent = jp.qp_ent;
   const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ) + (size_t)wid * join_lane_warp_bytes(MQ));
   const unsigned oRU = wbase + 16u * lane;                        // {R, U} of depth d: oRU + 512 d
