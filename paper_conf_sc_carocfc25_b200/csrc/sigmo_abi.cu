@@ -57,6 +57,7 @@ struct Timing {
 struct ProgCache {
   QueryProg prog;
   DBuf buf, pack;  // device program arrays; packed form for k_filter
+  std::vector<uint16_t> qdrow;  // host copy of prog.qdrow
   bool valid = false;
 };
 
@@ -134,6 +135,12 @@ struct sigmo_ctx {
   // jcnt u64 slots: [0] pair cursor / chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
   bool lane_join = false;  // per-lane join possible for this batch (<= 64-node graphs, <= 16-node queries)
   bool mol_filter = false; // last sigmo_filter used molecule tiles (candidates in cmol layout)
+  // plan entries as loaded (host) and the query node of each plan position;
+  // bits 12.. of .x are set to the distinct row of that node for the R whose
+  // program last ran (ent_R), re-uploaded when R changes
+  std::vector<int4> ent_host, ent_up;
+  std::vector<int32_t> ent_row;
+  int ent_R = -1;
   int mol_extn = 0, mol_extw = 0;  // molecule-tile geometry (32 graphs per tile)
   DBuf dense_tmp;          // dense view of cmol for sigmo_get_candidates
   int last_mode = 0;
@@ -601,6 +608,19 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
     }
   }
   rowp_off[VQ] = VQ * RW;
+  // distinct rows: query nodes with the same channel list (label + the same
+  // constraint planes) compute the same candidate row; the molecule-tile
+  // filter computes and stores each distinct row once per molecule
+  std::map<std::vector<int>, int> dmap;
+  std::vector<uint16_t> qdrow((size_t)VQ + 1, 0);
+  std::vector<uint32_t> drowp;
+  for (int v = 0; v < VQ; v++) {
+    auto ins = dmap.emplace(chans[v], (int)dmap.size());
+    qdrow[v] = (uint16_t)ins.first->second;
+    if (ins.second) drowp.insert(drowp.end(), rowp.begin() + (size_t)v * RW, rowp.begin() + (size_t)(v + 1) * RW);
+  }
+  const int NDR = (int)dmap.size();
+  if (NDR > 0xffff) return set_err(c, SIGMO_ERR_LIMIT, "%d distinct query rows", NDR);
   // upload
   Layout L;
   const size_t o_rec = L.take(sizeof(GroupRec) * (rec.size() + 1));
@@ -610,6 +630,8 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   const size_t o_bd = L.take(4 * bdone.size());
   const size_t o_po = L.take(4 * rowp_off.size());
   const size_t o_rp = L.take(4 * (rowp.size() + 1));
+  const size_t o_dp = L.take(4 * (drowp.size() + 1));
+  const size_t o_qd = L.take(2 * qdrow.size());
   std::vector<unsigned char> hb(L.off, 0);
   auto put = [&](size_t o, const void *src, size_t n) { if (n) memcpy(hb.data() + o, src, n); };
   put(o_rec, rec.data(), sizeof(GroupRec) * rec.size());
@@ -619,6 +641,8 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   put(o_bd, bdone.data(), 4 * bdone.size());
   put(o_po, rowp_off.data(), 4 * rowp_off.size());
   put(o_rp, rowp.data(), 4 * rowp.size());
+  put(o_dp, drowp.data(), 4 * drowp.size());
+  put(o_qd, qdrow.data(), 2 * qdrow.size());
   SIGMO_TRY(dreserve(c, pc.pack, L.off, "packed query program"));
   unsigned char *db = (unsigned char *)pc.pack.p;
   CUDA_TRY(c, cudaMemcpyAsync(db, hb.data(), L.off, cudaMemcpyHostToDevice, st));
@@ -630,6 +654,10 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   P.bdone = (int32_t *)(db + o_bd);
   P.rowp_off = (int32_t *)(db + o_po);
   P.rowp = (uint32_t *)(db + o_rp);
+  P.drowp = (uint32_t *)(db + o_dp);
+  P.qdrow = (uint16_t *)(db + o_qd);
+  P.meta.NDR = NDR;
+  pc.qdrow.assign(qdrow.begin(), qdrow.begin() + VQ);
   P.meta.NREC = (int)rec.size();
   P.meta.NRP = (int)rowp.size();
   P.meta.RW = RW;
@@ -972,6 +1000,9 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       ent[i] = e4;
     }
     if (hq.G) memcpy(hb + o_qinfo, plan.qinfo.data(), 4 * (size_t)hq.G);
+    c->ent_host.assign(ent, ent + hq.V);
+    c->ent_row.assign(plan.row.begin(), plan.row.end());
+    c->ent_R = -1;
   }
   pack_graphs(hb, pd, hd);
   memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
@@ -1100,12 +1131,12 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     int rows_smem = 1;
     if (mol) {
       rows_smem = 1;
-      smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NRP, 1, c->NQW,
-                               m.TS, 1);
+      smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NDR * m.RW, 1,
+                               c->NQW, m.TS, 1, m.NDR);
       if (smem > c->max_smem / 2) {
         rows_smem = 0;
-        smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NRP, 0,
-                                 c->NQW, m.TS, 1);
+        smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NDR * m.RW, 0,
+                                 c->NQW, m.TS, 1, m.NDR);
       }
       if (smem > c->max_smem) mol = false;  // fall back to dense tiles
     }
@@ -1135,7 +1166,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.NFU = m.NFU;
     fp.NLAB = m.NLAB;
     fp.NREC = m.NREC;
-    fp.NRP = m.NRP;
+    fp.NRP = mol ? m.NDR * m.RW : m.NRP;
     fp.NBATCH = m.NBATCH;
     fp.RW = m.RW;
     fp.TS = m.TS;
@@ -1147,7 +1178,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.fslot = prog->fslot;
     fp.lab_val = prog->lab_val;
     fp.rowp_off = prog->rowp_off;
-    fp.rowp = prog->rowp;
+    fp.rowp = mol ? prog->drowp : prog->rowp;  // molecule tiles: the distinct rows
     fp.qgoff = c->dq.goff;
     fp.bitmap = (uint32_t *)c->bitmap.p;
     fp.gm = (uint32_t *)c->gm.p;
@@ -1158,6 +1189,19 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.tile_g0 = (!mol && tws[k] == 32) ? c->tile_g0 : nullptr;
     fp.tile_g1 = (!mol && tws[k] == 32) ? c->tile_g1 : nullptr;
     fp.cmol = mol ? (unsigned long long *)c->bitmap.p : nullptr;
+    fp.qdrow = prog->qdrow;
+    fp.NDR = m.NDR;
+    if (mol && c->ent_R != R) {
+      // distinct-row index of each plan position's query node into the plan entries
+      const std::vector<uint16_t> &qd = c->progs[R].qdrow;
+      c->ent_up = c->ent_host;
+      for (size_t i = 0; i < c->ent_up.size(); i++)
+        c->ent_up[i].x = (c->ent_up[i].x & 0xfff) | ((int)qd[(size_t)c->ent_row[i]] << 12);
+      if (!c->ent_up.empty())
+        CUDA_TRY(c, cudaMemcpyAsync((void *)c->qp_ent, c->ent_up.data(), sizeof(int4) * c->ent_up.size(),
+                                    cudaMemcpyHostToDevice, c->stream));
+      c->ent_R = R;
+    }
     fp.rows_smem = rows_smem;
     fp.smem_bytes = smem;
     if (c->has_empty_graph) {
@@ -1222,6 +1266,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     pp.bitmap = (const uint32_t *)c->bitmap.p;
     pp.pair_query = (int32_t *)c->pair_query.p;
     pp.prec = mol ? (int4 *)c->pair_rec.p : nullptr;
+    pp.rowstride = m.NDR;
     pp.qinfo = c->qp_qinfo;
     CUDA_TRY(c, launch_pairs(pp, c->stream));
     launches++;
@@ -1401,8 +1446,9 @@ sigmo_status sigmo_get_candidates(sigmo_ctx *c, uint32_t *out) {
     const size_t bytes = 4 * (size_t)c->VQ * c->Wpad;
     SIGMO_TRY(dreserve(c, c->dense_tmp, bytes, "dense candidate view"));
     CUDA_TRY(c, cudaMemsetAsync(c->dense_tmp.p, 0, bytes, c->stream));
-    CUDA_TRY(c, launch_unpad((const unsigned long long *)c->bitmap.p, c->dd.goff, c->ND, c->VQ, c->Wpad,
-                             (uint32_t *)c->dense_tmp.p, c->stream));
+    const QueryProg &pg = c->progs[c->levels - 1].prog;  // the program of the last filter
+    CUDA_TRY(c, launch_unpad((const unsigned long long *)c->bitmap.p, pg.qdrow, pg.meta.NDR, c->dd.goff, c->ND, c->VQ,
+                             c->Wpad, (uint32_t *)c->dense_tmp.p, c->stream));
     src = c->dense_tmp.p;
   }
   CUDA_TRY(c, cudaMemcpy2DAsync(out, 4 * (size_t)c->W, src, 4 * (size_t)c->Wpad, 4 * (size_t)c->W,

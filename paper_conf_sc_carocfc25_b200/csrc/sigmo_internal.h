@@ -44,6 +44,7 @@ struct QueryProgMeta {
   int NBATCH;  // 32-plane batches
   int TS;      // threshold-table entries per record (64, or 256 for > 64-node graphs)
   int RW;      // row-program words per query node (padded)
+  int NDR;     // distinct rows (query nodes with the same label and constraint list share one)
 };
 
 // One part of a (radius, field) count group inside one 32-plane batch of the
@@ -76,6 +77,8 @@ struct QueryProg {
   uint32_t *tab = nullptr;     // [NREC * TS] thermometer tables
   int32_t *rowp_off = nullptr; // [VQ+1] row-program word range per query node
   uint32_t *rowp = nullptr;    // [NRP] channel byte offsets (lo | hi << 16), label channel first
+  uint32_t *drowp = nullptr;   // [NDR * RW] row programs of the distinct rows (molecule tiles)
+  uint16_t *qdrow = nullptr;   // [VQ] distinct row of each query node
   QueryProgMeta *d_meta = nullptr;
 };
 
@@ -96,7 +99,9 @@ struct FilterParams {
   const uint32_t *rowp;
   const int32_t *qgoff;        // [NQ+1] query node offsets (rows)
   uint32_t *bitmap;            // [VQ][Wpad] (dense tiles)
-  unsigned long long *cmol;    // [ND][VQ] molecule-padded windows (molecule tiles), else null
+  unsigned long long *cmol;    // [ND][NDR] molecule-padded windows of the distinct rows (molecule tiles), else null
+  const uint16_t *qdrow;       // [VQ] distinct row of each query node (molecule tiles)
+  int NDR;
   uint32_t *gm;                // [ND][NQW] surviving-query bits per data graph
   I64x2 *mol_cnt;              // [ND+1] (surviving pairs, candidate-mask entries)
   int EXTN, EXTW, MOLCAP;
@@ -145,6 +150,7 @@ struct JoinParams {
 // k_pairs: GMCR pair list + per-pair candidate masks
 struct PairsParams {
   int ND, NQ, NQW, MQ, Wpad, VQ;
+  int rowstride;               // cmol row stride per graph (distinct rows)
   const uint32_t *gm;
   const I64x2 *off;
   const int32_t *goff, *qgoff, *qp_row;
@@ -182,14 +188,15 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
                               cudaStream_t st);
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ,
-                         int NRP, int rows_smem, int NQW, int TS, int mol);
+                         int NRP, int rows_smem, int NQW, int TS, int mol, int NDR = 0);
 cudaError_t launch_support(int NW, const SupportParams &p, cudaStream_t st);
 size_t support_smem_bytes(int NW, int NB, int maxq, int NQW);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);
 cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
-cudaError_t launch_unpad(const unsigned long long *cmol, const int32_t *goff, int ND, int VQ, int Wpad, uint32_t *dense,
+cudaError_t launch_unpad(const unsigned long long *cmol, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
+                         int VQ, int Wpad, uint32_t *dense,
                          cudaStream_t st);
 cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsigned long long *adjb, cudaStream_t st);
 cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream_t st);

@@ -432,7 +432,7 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
 // ===========================================================================
 struct FilterSmem {
   size_t nb, ballA, ballB, fm, pl, fpl, memb, win, nz, gmb, slotat, endb, own, molstart, molslot, loc, fid, lab, mstart,
-      sos, grec, tab, bdone, rowpoff, rowp, total;
+      sos, grec, tab, bdone, rowpoff, rowp, dnz, qdr, total;
 };
 
 __host__ __device__ inline size_t align16(size_t x) { return (x + 15) & ~(size_t)15; }
@@ -440,7 +440,7 @@ __host__ __device__ inline int plane_stride(int NLAB, int P) { return (NLAB + 1 
 
 __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB,
                                                     int P, int NREC, int VQ, int NRP, int rows_smem, int NQW,
-                                                    int TS, int mol = 0) {
+                                                    int TS, int mol = 0, int NDR = 0) {
   FilterSmem L;
   const size_t mb = 8 * (size_t)NW;
   const int NWARP = kFilterThreads / 32;
@@ -471,15 +471,18 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   L.grec = o;     o = align16(o + sizeof(GroupRec) * (size_t)(NREC > 0 ? NREC : 1));
   L.tab = o;      o = align16(o + 4 * (size_t)TS * (NREC > 0 ? NREC : 1));
   L.bdone = o;    o = align16(o + (size_t)(P / 32 + 1));
-  L.rowpoff = o;  o = align16(o + (rows_smem ? 4 * (size_t)(VQ + 1) : 0));
+  L.rowpoff = o;  o = align16(o + (rows_smem && !mol ? 4 * (size_t)(VQ + 1) : 0));
   L.rowp = o;     o = align16(o + (rows_smem ? 4 * (size_t)NRP : 0));
+  // molecule tiles: non-empty bits of the distinct rows [NDR/32][32 molecules], distinct row per query node
+  L.dnz = o;      o = align16(o + (mol ? 4 * (size_t)32 * ((NDR + 31) / 32) : 0));
+  L.qdr = o;      o = align16(o + (mol ? 2 * (size_t)VQ : 0));
   L.total = o;
   return L;
 }
 
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ, int NRP,
-                         int rows_smem, int NQW, int TS, int mol) {
-  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, NREC, VQ, NRP, rows_smem, NQW, TS, mol).total;
+                         int rows_smem, int NQW, int TS, int mol, int NDR) {
+  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, NREC, VQ, NRP, rows_smem, NQW, TS, mol, NDR).total;
 }
 
 // 32x32 bit-matrix transpose across the warp: lane L holds row L (bit p =
@@ -533,7 +536,7 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   constexpr int NT = kFilterThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
   const FilterSmem L = filter_layout(NW, fp.EXTN, fp.EXTW, fp.MOLCAP, fp.NFU, fp.NLAB, fp.P, fp.NREC, fp.VQ, fp.NRP,
-                                     fp.rows_smem, fp.NQW, fp.TS, MOL ? 1 : 0);
+                                     fp.rows_smem, fp.NQW, fp.TS, MOL ? 1 : 0, fp.NDR);
   uint32_t *s_nb = (uint32_t *)(smem + L.nb);
   M *s_cur = (M *)(smem + L.ballA);
   M *s_nxt = (M *)(smem + L.ballB);
@@ -607,8 +610,15 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   if (fp.rows_smem) {
     int32_t *b = (int32_t *)(smem + L.rowpoff);
     uint32_t *c = (uint32_t *)(smem + L.rowp);
-    for (int i = tid; i <= fp.VQ; i += NT) b[i] = fp.rowp_off[i];
+    if (!MOL)
+      for (int i = tid; i <= fp.VQ; i += NT) b[i] = fp.rowp_off[i];
     for (int i = tid; i < fp.NRP; i += NT) c[i] = fp.rowp[i];
+  }
+  if (MOL) {
+    uint32_t *dnz = (uint32_t *)(smem + L.dnz);
+    uint16_t *qdr = (uint16_t *)(smem + L.qdr);
+    for (int i = tid; i < 32 * ((fp.NDR + 31) >> 5); i += NT) dnz[i] = 0u;
+    for (int i = tid; i < fp.VQ; i += NT) qdr[i] = __ldg(&fp.qdrow[i]);
   }
   if (tid < 32) {
     s_endb[tid] = 0u;
@@ -813,49 +823,47 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
     const int n = valid ? s_mstart[mi + 1] - ms : 0;
     const unsigned long long nmask = n >= 64 ? ~0ull : ((1ull << n) - 1ull);
     const int ws = ms >> 5, sh = ms & 31;
-    unsigned long long *cm = fp.cmol + (size_t)(g0 + mi) * fp.VQ;  // molecule-major: cmol[g][row]
+    unsigned long long *cm = fp.cmol + (size_t)(g0 + mi) * fp.NDR;  // molecule-major: cmol[g][distinct row]
+    uint32_t *dnz = (uint32_t *)(smem + L.dnz);                        // [NDR/32][32 molecules]
     auto mol_rows = [&](auto RWc, auto HIc, const uint32_t *rowp) {
       constexpr int RWk = decltype(RWc)::value;
       constexpr bool HI = decltype(HIc)::value;  // the tile spans more than 32 words
       const int RW = RWk ? RWk : fp.RW;
       const unsigned char *pl0 = (const unsigned char *)(s_pl + (size_t)(lane < nxw ? lane : 0) * PS);
       const unsigned char *pl1 = (const unsigned char *)(s_pl + (size_t)(lane + 32 < nxw ? lane + 32 : 0) * PS);
-      for (int q = wid; q < fp.NQ; q += NWARP) {
-        const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
-        bool all = valid;
-        const uint32_t *pr = rowp + (size_t)r0 * RW;
-        for (int row = r0; row < r1; row++, pr += RW) {
-          uint32_t x0 = 0xffffffffu, x1 = 0xffffffffu;
+      for (int row = wid; row < fp.NDR; row += NWARP) {
+        const uint32_t *pr = rowp + (size_t)row * RW;
+        uint32_t x0 = 0xffffffffu, x1 = 0xffffffffu;
 #pragma unroll
-          for (int j = 0; j < (RWk ? RWk : 1); j++) {
-            const uint32_t two = pr[j];
-            x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
-            if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
-          }
-          for (int j = RWk; j < RW; j++) {
-            const uint32_t two = pr[j];
-            x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
-            if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
-          }
-          uint32_t w0, w1, w2;
-          if (HI) {
-            const uint32_t a0 = __shfl_sync(FULL_MASK, x0, ws & 31), b0 = __shfl_sync(FULL_MASK, x1, ws & 31);
-            const uint32_t a1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31), b1 = __shfl_sync(FULL_MASK, x1, (ws + 1) & 31);
-            const uint32_t a2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31), b2 = __shfl_sync(FULL_MASK, x1, (ws + 2) & 31);
-            w0 = ws < 32 ? a0 : b0;
-            w1 = ws + 1 < 32 ? a1 : b1;
-            w2 = ws + 2 < 32 ? a2 : b2;
-          } else {
-            w0 = __shfl_sync(FULL_MASK, x0, ws);
-            w1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31);
-            w2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31);
-          }
-          const unsigned long long x =
-              (((unsigned long long)__funnelshift_r(w1, w2, sh) << 32) | __funnelshift_r(w0, w1, sh)) & nmask;
-          if (valid) cm[row] = x;
-          all = all && x != 0ull;
+        for (int j = 0; j < (RWk ? RWk : 1); j++) {
+          const uint32_t two = pr[j];
+          x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
+          if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
         }
-        if (all) atomicOr(&s_gm[mi * fp.NQW + (q >> 5)], 1u << (q & 31));
+        for (int j = RWk; j < RW; j++) {
+          const uint32_t two = pr[j];
+          x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
+          if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
+        }
+        uint32_t w0, w1, w2;
+        if (HI) {
+          const uint32_t a0 = __shfl_sync(FULL_MASK, x0, ws & 31), b0 = __shfl_sync(FULL_MASK, x1, ws & 31);
+          const uint32_t a1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31), b1 = __shfl_sync(FULL_MASK, x1, (ws + 1) & 31);
+          const uint32_t a2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31), b2 = __shfl_sync(FULL_MASK, x1, (ws + 2) & 31);
+          w0 = ws < 32 ? a0 : b0;
+          w1 = ws + 1 < 32 ? a1 : b1;
+          w2 = ws + 2 < 32 ? a2 : b2;
+        } else {
+          w0 = __shfl_sync(FULL_MASK, x0, ws);
+          w1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31);
+          w2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31);
+        }
+        const unsigned long long x =
+            (((unsigned long long)__funnelshift_r(w1, w2, sh) << 32) | __funnelshift_r(w0, w1, sh)) & nmask;
+        if (valid) {
+          cm[row] = x;
+          if (x) atomicOr(&dnz[(row >> 5) * 32 + mi], 1u << (row & 31));
+        }
       }
     };
     const bool hi = nxw > 32;
@@ -874,6 +882,18 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
     } else {
       if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, fp.rowp);
       else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, fp.rowp);
+    }
+    __syncthreads();
+    // GMCR: lane = molecule, warp per query: every node's distinct row non-empty
+    const uint16_t *qdr = (const uint16_t *)(smem + L.qdr);
+    for (int q = wid; q < fp.NQ && valid; q += NWARP) {
+      const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
+      bool all = true;
+      for (int v = r0; v < r1 && all; v++) {
+        const int dr = qdr[v];
+        all = (dnz[(dr >> 5) * 32 + mi] >> (dr & 31)) & 1u;
+      }
+      if (all) atomicOr(&s_gm[mi * fp.NQW + (q >> 5)], 1u << (q & 31));
     }
   }
 
@@ -1794,7 +1814,7 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
       if (pp.prec) {
         // query info with the molecule size in bits 8-15 (class stride of adjb)
         const uint32_t qi = (__ldg(&pp.qinfo[q]) & ~0xff00u) | ((uint32_t)(__ldg(&pp.goff[g + 1]) - a) << 8);
-        pp.prec[p] = make_int4(a, q, (int)((unsigned)g * (unsigned)pp.VQ + (qi >> 16)), (int)qi);
+        pp.prec[p] = make_int4(a, q, (int)((unsigned)g * (unsigned)pp.rowstride), (int)qi);
       }
     }
     o += __popc(bits);
@@ -1810,12 +1830,12 @@ cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st) {
 
 // Dense (row-major, LSB-first) view of the molecule-padded candidates for
 // sigmo_get_candidates: thread per (row, graph), OR the window into the rows.
-__global__ void k_unpad(const unsigned long long *cmol, const int32_t *goff, int ND, int VQ, int Wpad,
-                        uint32_t *dense) {
+__global__ void k_unpad(const unsigned long long *cmol, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
+                        int VQ, int Wpad, uint32_t *dense) {
   const long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (t >= (long long)ND * VQ) return;
   const int g = (int)(t / VQ), row = (int)(t - (long long)g * VQ);
-  const unsigned long long w = cmol[t];  // cmol[g][row]
+  const unsigned long long w = cmol[(size_t)g * NDR + qdrow[row]];  // cmol[g][distinct row of query node row]
   if (!w) return;
   const int a = goff[g];
   uint32_t *r = dense + (size_t)row * Wpad;
@@ -1826,11 +1846,11 @@ __global__ void k_unpad(const unsigned long long *cmol, const int32_t *goff, int
   if (sh && (uint32_t)(w >> (64 - sh))) atomicOr(&r[wi + 2], (uint32_t)(w >> (64 - sh)));
 }
 
-cudaError_t launch_unpad(const unsigned long long *cmol, const int32_t *goff, int ND, int VQ, int Wpad, uint32_t *dense,
-                         cudaStream_t st) {
+cudaError_t launch_unpad(const unsigned long long *cmol, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
+                         int VQ, int Wpad, uint32_t *dense, cudaStream_t st) {
   const long long n = (long long)ND * VQ;
   if (n <= 0) return cudaSuccess;
-  k_unpad<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(cmol, goff, ND, VQ, Wpad, dense);
+  k_unpad<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(cmol, qdrow, NDR, goff, ND, VQ, Wpad, dense);
   return cudaGetLastError();
 }
 
@@ -2008,7 +2028,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const unsigned ng = (cinfo >> 8) & 0xffu;  // molecule size: class stride of adjb
       const unsigned i0 = j0 == 15u ? ones : ca + (unsigned)en.y * ng + u0;
       const unsigned i1 = j1 == 15u ? ones : ca + (unsigned)en.z * ng + u1;
-      unsigned long long X = __ldg(&cmol[cmb + ((en.x >> 12) & 15)]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
+      unsigned long long X = __ldg(&cmol[cmb + ((unsigned)en.x >> 12)]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
       if (en.x & 0xf00) {  // > 2 back-edges at this depth (fused rings): rare
         const int nex = (en.x >> 8) & 15;
         for (int k = 0; k < nex; k++) {
@@ -2085,7 +2105,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         np = cbase + (unsigned)src;
         nv = true;
         // root candidates of the next pair: the load completes while the current pair runs
-        nR0 = __ldg(&cmol[(unsigned)r.z + ((__ldg(&qp_ent[(unsigned)r.w >> 16]).x >> 12) & 15)]);
+        nR0 = __ldg(&cmol[(unsigned)r.z + ((unsigned)__ldg(&qp_ent[(unsigned)r.w >> 16]).x >> 12)]);
       }
       chead += take;
       wm = __ballot_sync(FULL_MASK, !nv) & wm;
