@@ -140,6 +140,7 @@ struct sigmo_ctx {
   // program last ran (ent_R), re-uploaded when R changes
   std::vector<int4> ent_host, ent_up;
   std::vector<int32_t> ent_row;
+  std::vector<int64_t> qgoff_host;  // query graph offsets (host copy, for the per-query row-word lists)
   int ent_R = -1;
   int mol_extn = 0, mol_extw = 0;  // molecule-tile geometry (32 graphs per tile)
   DBuf dense_tmp;          // dense view of cmol for sigmo_get_candidates
@@ -621,6 +622,21 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   }
   const int NDR = (int)dmap.size();
   if (NDR > 0xffff) return set_err(c, SIGMO_ERR_LIMIT, "%d distinct query rows", NDR);
+  // GMCR lists of the molecule-tile filter: per query the (word, bits) pairs
+  // of its distinct rows in the per-molecule non-empty bit vector
+  const int NQ = c->NQ;
+  std::vector<int32_t> qw_off((size_t)NQ + 1, 0);
+  std::vector<uint32_t> qw;  // word, mask interleaved
+  for (int q = 0; q < NQ; q++) {
+    qw_off[q] = (int32_t)(qw.size() / 2);
+    std::map<int, uint32_t> wm;
+    for (int64_t v = c->qgoff_host[q]; v < c->qgoff_host[q + 1]; v++) wm[qdrow[v] >> 5] |= 1u << (qdrow[v] & 31);
+    for (const auto &kv : wm) {
+      qw.push_back((uint32_t)kv.first);
+      qw.push_back(kv.second);
+    }
+  }
+  qw_off[NQ] = (int32_t)(qw.size() / 2);
   // upload
   Layout L;
   const size_t o_rec = L.take(sizeof(GroupRec) * (rec.size() + 1));
@@ -632,6 +648,8 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   const size_t o_rp = L.take(4 * (rowp.size() + 1));
   const size_t o_dp = L.take(4 * (drowp.size() + 1));
   const size_t o_qd = L.take(2 * qdrow.size());
+  const size_t o_qwo = L.take(4 * qw_off.size());
+  const size_t o_qw = L.take(4 * (qw.size() + 2));
   std::vector<unsigned char> hb(L.off, 0);
   auto put = [&](size_t o, const void *src, size_t n) { if (n) memcpy(hb.data() + o, src, n); };
   put(o_rec, rec.data(), sizeof(GroupRec) * rec.size());
@@ -643,6 +661,8 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   put(o_rp, rowp.data(), 4 * rowp.size());
   put(o_dp, drowp.data(), 4 * drowp.size());
   put(o_qd, qdrow.data(), 2 * qdrow.size());
+  put(o_qwo, qw_off.data(), 4 * qw_off.size());
+  put(o_qw, qw.data(), 4 * qw.size());
   SIGMO_TRY(dreserve(c, pc.pack, L.off, "packed query program"));
   unsigned char *db = (unsigned char *)pc.pack.p;
   CUDA_TRY(c, cudaMemcpyAsync(db, hb.data(), L.off, cudaMemcpyHostToDevice, st));
@@ -657,6 +677,9 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   P.drowp = (uint32_t *)(db + o_dp);
   P.qdrow = (uint16_t *)(db + o_qd);
   P.meta.NDR = NDR;
+  P.qw_off = (int32_t *)(db + o_qwo);
+  P.qw = (uint32_t *)(db + o_qw);
+  P.meta.NQWL = (int)(qw.size() / 2);
   pc.qdrow.assign(qdrow.begin(), qdrow.begin() + VQ);
   P.meta.NREC = (int)rec.size();
   P.meta.NRP = (int)rowp.size();
@@ -1002,6 +1025,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     if (hq.G) memcpy(hb + o_qinfo, plan.qinfo.data(), 4 * (size_t)hq.G);
     c->ent_host.assign(ent, ent + hq.V);
     c->ent_row.assign(plan.row.begin(), plan.row.end());
+    c->qgoff_host.assign(hq.goff, hq.goff + hq.G + 1);
     c->ent_R = -1;
   }
   pack_graphs(hb, pd, hd);
@@ -1132,11 +1156,11 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     if (mol) {
       rows_smem = 1;
       smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NDR * m.RW, 1,
-                               c->NQW, m.TS, 1, m.NDR);
+                               c->NQW, m.TS, 1, m.NDR, c->NQ, m.NQWL);
       if (smem > c->max_smem / 2) {
         rows_smem = 0;
         smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NDR * m.RW, 0,
-                                 c->NQW, m.TS, 1, m.NDR);
+                                 c->NQW, m.TS, 1, m.NDR, c->NQ, m.NQWL);
       }
       if (smem > c->max_smem) mol = false;  // fall back to dense tiles
     }
@@ -1190,6 +1214,9 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.tile_g1 = (!mol && tws[k] == 32) ? c->tile_g1 : nullptr;
     fp.cmol = mol ? (unsigned long long *)c->bitmap.p : nullptr;
     fp.qdrow = prog->qdrow;
+    fp.qw_off = prog->qw_off;
+    fp.qw = prog->qw;
+    fp.NQWL = m.NQWL;
     fp.NDR = m.NDR;
     if (mol && c->ent_R != R) {
       // distinct-row index of each plan position's query node into the plan entries

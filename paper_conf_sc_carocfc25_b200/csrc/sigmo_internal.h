@@ -45,6 +45,7 @@ struct QueryProgMeta {
   int TS;      // threshold-table entries per record (64, or 256 for > 64-node graphs)
   int RW;      // row-program words per query node (padded)
   int NDR;     // distinct rows (query nodes with the same label and constraint list share one)
+  int NQWL;    // (word, bits) entries of the per-query GMCR lists over distinct rows
 };
 
 // One part of a (radius, field) count group inside one 32-plane batch of the
@@ -79,6 +80,8 @@ struct QueryProg {
   uint32_t *rowp = nullptr;    // [NRP] channel byte offsets (lo | hi << 16), label channel first
   uint32_t *drowp = nullptr;   // [NDR * RW] row programs of the distinct rows (molecule tiles)
   uint16_t *qdrow = nullptr;   // [VQ] distinct row of each query node
+  int32_t *qw_off = nullptr;   // [NQ+1] per-query range of (word, bits) entries
+  uint32_t *qw = nullptr;      // [NQWL][2] word of the distinct-row bit vector, bits of the query's rows in it
   QueryProgMeta *d_meta = nullptr;
 };
 
@@ -101,7 +104,9 @@ struct FilterParams {
   uint32_t *bitmap;            // [VQ][Wpad] (dense tiles)
   unsigned long long *cmol;    // [ND][NDR] molecule-padded windows of the distinct rows (molecule tiles), else null
   const uint16_t *qdrow;       // [VQ] distinct row of each query node (molecule tiles)
-  int NDR;
+  const int32_t *qw_off;       // [NQ+1] GMCR (word, bits) lists per query (molecule tiles)
+  const uint32_t *qw;
+  int NDR, NQWL;
   uint32_t *gm;                // [ND][NQW] surviving-query bits per data graph
   I64x2 *mol_cnt;              // [ND+1] (surviving pairs, candidate-mask entries)
   int EXTN, EXTW, MOLCAP;
@@ -188,7 +193,7 @@ cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts,
                               cudaStream_t st);
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ,
-                         int NRP, int rows_smem, int NQW, int TS, int mol, int NDR = 0);
+                         int NRP, int rows_smem, int NQW, int TS, int mol, int NDR = 0, int NQ = 0, int NQWL = 0);
 cudaError_t launch_support(int NW, const SupportParams &p, cudaStream_t st);
 size_t support_smem_bytes(int NW, int NB, int maxq, int NQW);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);

@@ -440,7 +440,7 @@ __host__ __device__ inline int plane_stride(int NLAB, int P) { return (NLAB + 1 
 
 __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB,
                                                     int P, int NREC, int VQ, int NRP, int rows_smem, int NQW,
-                                                    int TS, int mol = 0, int NDR = 0) {
+                                                    int TS, int mol = 0, int NDR = 0, int NQ = 0, int NQWL = 0) {
   FilterSmem L;
   const size_t mb = 8 * (size_t)NW;
   const int NWARP = kFilterThreads / 32;
@@ -475,14 +475,14 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   L.rowp = o;     o = align16(o + (rows_smem ? 4 * (size_t)NRP : 0));
   // molecule tiles: non-empty bits of the distinct rows [NDR/32][32 molecules], distinct row per query node
   L.dnz = o;      o = align16(o + (mol ? 4 * (size_t)32 * ((NDR + 31) / 32) : 0));
-  L.qdr = o;      o = align16(o + (mol ? 2 * (size_t)VQ : 0));
+  L.qdr = o;      o = align16(o + (mol ? align16(4 * (size_t)(NQ + 1)) + 8 * (size_t)NQWL : 0));  // GMCR lists
   L.total = o;
   return L;
 }
 
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ, int NRP,
-                         int rows_smem, int NQW, int TS, int mol, int NDR) {
-  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, NREC, VQ, NRP, rows_smem, NQW, TS, mol, NDR).total;
+                         int rows_smem, int NQW, int TS, int mol, int NDR, int NQ, int NQWL) {
+  return filter_layout(NW, EXTN, EXTW, MOLCAP, NFU, NLAB, P, NREC, VQ, NRP, rows_smem, NQW, TS, mol, NDR, NQ, NQWL).total;
 }
 
 // 32x32 bit-matrix transpose across the warp: lane L holds row L (bit p =
@@ -536,7 +536,7 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   constexpr int NT = kFilterThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
   const FilterSmem L = filter_layout(NW, fp.EXTN, fp.EXTW, fp.MOLCAP, fp.NFU, fp.NLAB, fp.P, fp.NREC, fp.VQ, fp.NRP,
-                                     fp.rows_smem, fp.NQW, fp.TS, MOL ? 1 : 0, fp.NDR);
+                                     fp.rows_smem, fp.NQW, fp.TS, MOL ? 1 : 0, fp.NDR, fp.NQ, fp.NQWL);
   uint32_t *s_nb = (uint32_t *)(smem + L.nb);
   M *s_cur = (M *)(smem + L.ballA);
   M *s_nxt = (M *)(smem + L.ballB);
@@ -616,9 +616,11 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   }
   if (MOL) {
     uint32_t *dnz = (uint32_t *)(smem + L.dnz);
-    uint16_t *qdr = (uint16_t *)(smem + L.qdr);
+    int32_t *qwo = (int32_t *)(smem + L.qdr);
+    uint2 *qw = (uint2 *)(smem + L.qdr + align16(4 * (size_t)(fp.NQ + 1)));
     for (int i = tid; i < 32 * ((fp.NDR + 31) >> 5); i += NT) dnz[i] = 0u;
-    for (int i = tid; i < fp.VQ; i += NT) qdr[i] = __ldg(&fp.qdrow[i]);
+    for (int i = tid; i <= fp.NQ; i += NT) qwo[i] = __ldg(&fp.qw_off[i]);
+    for (int i = tid; i < fp.NQWL; i += NT) qw[i] = make_uint2(__ldg(&fp.qw[2 * i]), __ldg(&fp.qw[2 * i + 1]));
   }
   if (tid < 32) {
     s_endb[tid] = 0u;
@@ -797,7 +799,8 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
             mb = 0u;
             cur_b = g.batch;
           }
-          const int c = min((ball & fmb[g.fslot]).popc(), TSm);
+          const int pc = (ball & fmb[g.fslot]).popc();
+          const int c = NW == 1 ? pc : min(pc, TSm);  // <= 64-node graphs: pc <= 63 < TS
           mb |= s_tab[g.toff + c];
         }
         if (s_bdone[cur_b] == r0) {
@@ -884,14 +887,16 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
       else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, fp.rowp);
     }
     __syncthreads();
-    // GMCR: lane = molecule, warp per query: every node's distinct row non-empty
-    const uint16_t *qdr = (const uint16_t *)(smem + L.qdr);
+    // GMCR: lane = molecule, warp per query: every node's distinct row
+    // non-empty = each (word, bits) entry of the query's list fully set
+    const int32_t *qwo = (const int32_t *)(smem + L.qdr);
+    const uint2 *qwl = (const uint2 *)(smem + L.qdr + align16(4 * (size_t)(fp.NQ + 1)));
     for (int q = wid; q < fp.NQ && valid; q += NWARP) {
-      const int r0 = __ldg(&fp.qgoff[q]), r1 = __ldg(&fp.qgoff[q + 1]);
       bool all = true;
-      for (int v = r0; v < r1 && all; v++) {
-        const int dr = qdr[v];
-        all = (dnz[(dr >> 5) * 32 + mi] >> (dr & 31)) & 1u;
+      const int k1 = qwo[q + 1];
+      for (int k = qwo[q]; k < k1; k++) {
+        const uint2 wm = qwl[k];
+        all = all && (dnz[wm.x * 32 + mi] & wm.y) == wm.y;
       }
       if (all) atomicOr(&s_gm[mi * fp.NQW + (q >> 5)], 1u << (q & 31));
     }
