@@ -142,7 +142,9 @@ struct sigmo_ctx {
   std::vector<int32_t> ent_row;
   std::vector<int64_t> qgoff_host;  // query graph offsets (host copy, for the per-query row-word lists)
   int ent_R = -1;
-  int mol_extn = 0, mol_extw = 0;  // molecule-tile geometry (32 graphs per tile)
+  int mol_extn = 0, mol_extw = 0;  // molecule-tile geometry (<= 32 graphs and <= 1,024 nodes per tile)
+  int n_mol_tiles = 0;
+  int32_t *mol_tiles = nullptr;     // [n_mol_tiles + 1] first graph of each molecule tile
   DBuf dense_tmp;          // dense view of cmol for sigmo_get_candidates
   int last_mode = 0;
   DBuf sig_tmp, gstack;
@@ -983,6 +985,22 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const PackedOffsets pd = plan_graphs(L, hd);
   const size_t o_tg0 = L.take(4 * tg0.size());
   const size_t o_tg1 = L.take(4 * tg1.size());
+  // molecule tiles of the lane-join filter: <= 32 graphs and <= 1,024 nodes
+  std::vector<int32_t> mt;
+  {
+    int64_t g = 0;
+    mt.push_back(0);
+    while (g < hd.G) {
+      int64_t k = 0, nodes = 0;
+      while (g < hd.G && k < 32 && (k == 0 || nodes + (hd.goff[g + 1] - hd.goff[g]) <= 1024)) {
+        nodes += hd.goff[g + 1] - hd.goff[g];
+        g++;
+        k++;
+      }
+      mt.push_back((int32_t)g);
+    }
+  }
+  const size_t o_mt = L.take(4 * mt.size());
   const size_t total = L.off;
   // wait until the previous upload no longer reads the staging buffer
   CUDA_TRY(c, cudaEventSynchronize(c->h2d_done));
@@ -1031,6 +1049,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   pack_graphs(hb, pd, hd);
   memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
   memcpy(hb + o_tg1, tg1.data(), 4 * tg1.size());
+  memcpy(hb + o_mt, mt.data(), 4 * mt.size());
 
   // ---- device arena + one H2D copy ----
   SIGMO_TRY(dreserve(c, c->arena, total, "input arena"));
@@ -1045,6 +1064,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->qp_be = (uint16_t *)(db + o_be);
   c->bclass = db + o_bc;
   c->tile_g0 = (int32_t *)(db + o_tg0);
+  c->mol_tiles = (int32_t *)(db + o_mt);
+  c->n_mol_tiles = (int)mt.size() - 1;
   c->tile_g1 = (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
   c->qp_ent = (const int4 *)(db + o_ent);
@@ -1067,8 +1088,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   tile_geometry(c, hd);
   {
     int extn = 1;
-    for (int64_t g0 = 0; g0 < hd.G; g0 += 32)
-      extn = std::max<int>(extn, (int)(hd.goff[std::min<int64_t>(g0 + 32, hd.G)] - hd.goff[g0]));
+    for (int t = 0; t < c->n_mol_tiles; t++) extn = std::max<int>(extn, (int)(hd.goff[mt[t + 1]] - hd.goff[mt[t]]));
     c->mol_extn = extn;
     c->mol_extw = (extn + 31) / 32;
   }
@@ -1235,7 +1255,8 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       CUDA_TRY(c, cudaMemsetAsync(c->gm.p, 0, 4 * (size_t)c->ND * c->NQW, c->stream));
       CUDA_TRY(c, cudaMemsetAsync(c->mol_cnt.p, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
     }
-    const int tiles = mol ? (c->ND + 31) / 32 : (c->W + fp.TW - 1) / fp.TW;
+    const int tiles = mol ? c->n_mol_tiles : (c->W + fp.TW - 1) / fp.TW;
+    fp.mtile = c->mol_tiles;
     timing_mark(c, 2);
     CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));
     launches++;

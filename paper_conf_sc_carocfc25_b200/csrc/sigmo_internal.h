@@ -107,6 +107,7 @@ struct FilterParams {
   const int32_t *qw_off;       // [NQ+1] GMCR (word, bits) lists per query (molecule tiles)
   const uint32_t *qw;
   int NDR, NQWL;
+  const int32_t *mtile;        // [tiles+1] first graph of each molecule tile (<= 32 graphs, <= 1,024 nodes)
   uint32_t *gm;                // [ND][NQW] surviving-query bits per data graph
   I64x2 *mol_cnt;              // [ND+1] (surviving pairs, candidate-mask entries)
   int EXTN, EXTW, MOLCAP;

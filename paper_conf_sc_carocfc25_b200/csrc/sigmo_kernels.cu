@@ -579,8 +579,8 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   const int PS = plane_stride(NLAB, fp.P);
   if (tid == 0) {
     if (MOL) {
-      s_g0 = blockIdx.x * 32;
-      s_g1 = min(s_g0 + 32, ND);
+      s_g0 = __ldg(&fp.mtile[blockIdx.x]);
+      s_g1 = __ldg(&fp.mtile[blockIdx.x + 1]);
     } else if (fp.tile_g0) {
       s_g0 = __ldg(&fp.tile_g0[blockIdx.x]);
       s_g1 = __ldg(&fp.tile_g1[blockIdx.x]);
@@ -749,8 +749,8 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
   for (int r = 1; r <= fp.R; r++) {
     if (NW == 1) {
       // in place: all new balls are computed into registers before any is written
-      // EXTN <= 32 * TW + 2 * 63 (dense) or 32 * 64 (molecule tiles) for <= 64-node graphs
-      constexpr int kIt = MOL ? (2048 + NT - 1) / NT : (1024 + 2 * 63 + NT - 1) / NT;
+      // EXTN <= 32 * TW + 2 * 63 (dense) or 1,024 (molecule tiles) for <= 64-node graphs
+      constexpr int kIt = MOL ? (1024 + NT - 1) / NT : (1024 + 2 * 63 + NT - 1) / NT;
       M tmp[kIt];
 #pragma unroll
       for (int it = 0; it < kIt; it++) {
