@@ -458,7 +458,7 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   L.win = o;      o = align16(o + mb * (size_t)(mol ? 0 : NWARP) * NCH);
   L.nz = o;       o = align16(o + (mol ? 0 : 4 * (size_t)NWARP * (VQW + 1)));
   L.gmb = o;      o = align16(o + 4 * (size_t)MOLCAP * (NQW > 0 ? NQW : 1));
-  L.slotat = o;   o = align16(o + 2 * 32 * 32);
+  L.slotat = o;   o = align16(o + (mol ? 0 : 2 * 32 * 32));
   L.endb = o;     o = align16(o + 4 * 32);
   L.own = o;      o = align16(o + 4 * 32);
   L.molstart = o; o = align16(o + 2 * (size_t)EXTN);
@@ -476,7 +476,7 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   // molecule tiles: non-empty bits of the distinct rows [NDR/32][32 molecules], distinct row per query node
   L.dnz = o;      o = align16(o + (mol ? 4 * (size_t)32 * ((NDR + 31) / 32) : 0));
   L.qdr = o;      o = align16(o + (mol ? align16(4 * (size_t)(NQ + 1)) + 8 * (size_t)NQWL : 0));  // GMCR lists
-  L.stg = o;      o = align16(o + (mol ? 8 * (size_t)NWARP * 8 * 33 : 0));  // store staging (8 rows x 33 per warp)
+  L.stg = o;      o = align16(o + (mol ? 8 * (size_t)NWARP * 4 * 33 : 0));  // store staging (4 rows x 33 per warp)
   L.total = o;
   return L;
 }
@@ -828,17 +828,17 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
     const unsigned long long nmask = n >= 64 ? ~0ull : ((1ull << n) - 1ull);
     const int ws = ms >> 5, sh = ms & 31;
     uint32_t *dnz = (uint32_t *)(smem + L.dnz);  // [NDR/32][32 molecules]
-    // per warp: 8 rows x 32 molecules of windows, staged so that the stores
-    // to cmol[g][row] (molecule-major) go out as 64-B runs per molecule
-    unsigned long long *stg = (unsigned long long *)(smem + L.stg) + (size_t)wid * (8 * 33);
+    // per warp: 4 rows x 32 molecules of windows, staged so that the stores
+    // to cmol[g][row] (molecule-major) go out as 32-B sectors per molecule
+    unsigned long long *stg = (unsigned long long *)(smem + L.stg) + (size_t)wid * (4 * 33);
     auto mol_rows = [&](auto RWc, auto HIc, const uint32_t *rowp) {
       constexpr int RWk = decltype(RWc)::value;
       constexpr bool HI = decltype(HIc)::value;  // the tile spans more than 32 words
       const int RW = RWk ? RWk : fp.RW;
       const unsigned char *pl0 = (const unsigned char *)(s_pl + (size_t)(lane < nxw ? lane : 0) * PS);
       const unsigned char *pl1 = (const unsigned char *)(s_pl + (size_t)(lane + 32 < nxw ? lane + 32 : 0) * PS);
-      for (int rb = 8 * wid; rb < fp.NDR; rb += 8 * NWARP) {  // blocks of 8 rows per warp
-      const int nr = min(8, fp.NDR - rb);
+      for (int rb = 4 * wid; rb < fp.NDR; rb += 4 * NWARP) {  // blocks of 4 rows per warp
+      const int nr = min(4, fp.NDR - rb);
       uint32_t nzb = 0u;
       for (int r = 0; r < nr; r++) {
         const int row = rb + r;
@@ -873,11 +873,11 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
         stg[r * 33 + mi] = x;
         nzb |= (x != 0ull ? 1u : 0u) << r;
       }
-      if (valid && nzb) atomicOr(&dnz[(rb >> 5) * 32 + mi], nzb << (rb & 31));  // rb % 8 == 0: one word
+      if (valid && nzb) atomicOr(&dnz[(rb >> 5) * 32 + mi], nzb << (rb & 31));  // rb % 4 == 0: one word
       __syncwarp();
 #pragma unroll
-      for (int k = 0; k < 8; k++) {  // lane = (molecule, row): 4 molecules x 8 rows per store
-        const int e = k * 32 + lane, m = e >> 3, r = e & 7;
+      for (int k = 0; k < 4; k++) {  // lane = (molecule, row): 8 molecules x 4 rows per store
+        const int e = k * 32 + lane, m = e >> 2, r = e & 3;
         if (m < nmol && r < nr) fp.cmol[(size_t)(g0 + m) * fp.NDR + rb + r] = stg[r * 33 + m];
       }
       __syncwarp();
