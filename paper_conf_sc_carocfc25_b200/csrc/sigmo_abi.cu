@@ -1256,6 +1256,9 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       CUDA_TRY(c, cudaMemsetAsync(c->mol_cnt.p, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
     }
     const int tiles = mol ? c->n_mol_tiles : (c->W + fp.TW - 1) / fp.TW;
+    if (getenv("SIGMO_DEBUG_FILTER"))
+      fprintf(stderr, "sigmo filter: mol=%d smem=%zu EXTN=%d EXTW=%d NFU=%d NLAB=%d P=%d NREC=%d TS=%d NDR=%d RW=%d NQWL=%d tiles=%d\n",
+              (int)mol, smem, fp.EXTN, fp.EXTW, m.NFU, m.NLAB, m.P, m.NREC, m.TS, m.NDR, m.RW, m.NQWL, tiles);
     fp.mtile = c->mol_tiles;
     timing_mark(c, 2);
     CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));

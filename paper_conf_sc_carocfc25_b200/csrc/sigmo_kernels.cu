@@ -473,10 +473,29 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   L.bdone = o;    o = align16(o + (size_t)(P / 32 + 1));
   L.rowpoff = o;  o = align16(o + (rows_smem && !mol ? 4 * (size_t)(VQ + 1) : 0));
   L.rowp = o;     o = align16(o + (rows_smem ? 4 * (size_t)NRP : 0));
-  // molecule tiles: non-empty bits of the distinct rows [NDR/32][32 molecules], distinct row per query node
-  L.dnz = o;      o = align16(o + (mol ? 4 * (size_t)32 * ((NDR + 31) / 32) : 0));
-  L.qdr = o;      o = align16(o + (mol ? align16(4 * (size_t)(NQ + 1)) + 8 * (size_t)NQWL : 0));  // GMCR lists
-  L.stg = o;      o = align16(o + (mol ? 8 * (size_t)NWARP * 4 * 33 : 0));  // store staging (4 rows x 33 per warp)
+  // molecule tiles, rows phase only: non-empty bits of the distinct rows
+  // [NDR/32][32 molecules], the per-query GMCR lists, the store staging (4
+  // rows x 33 per warp).  They live after the plane phase, so they alias the
+  // BFS arrays (nb, balls) and the plane-batch carry words (memb) when they fit
+  if (mol) {
+    const size_t dnz_b = align16(4 * (size_t)32 * ((NDR + 31) / 32));
+    const size_t qdr_b = align16(align16(4 * (size_t)(NQ + 1)) + 8 * (size_t)NQWL);
+    const size_t stg_b = align16(8 * (size_t)NWARP * 4 * 33);
+    if (stg_b <= L.fm - L.nb) {  // nb + ballA (+ ballB) are contiguous
+      L.stg = L.nb;
+    } else {
+      L.stg = o; o = align16(o + stg_b);
+    }
+    if (dnz_b + qdr_b <= 4 * 32 * (size_t)EXTW) {
+      L.dnz = L.memb;
+      L.qdr = L.memb + dnz_b;
+    } else {
+      L.dnz = o; o = align16(o + dnz_b);
+      L.qdr = o; o = align16(o + qdr_b);
+    }
+  } else {
+    L.dnz = L.qdr = L.stg = o;
+  }
   L.total = o;
   return L;
 }
@@ -532,7 +551,7 @@ __device__ __forceinline__ Mask<NW> extract_window_strided(const uint32_t *words
 // by k_join_lane.  Otherwise
 // dense tiles of TW words writing the row-major bitmap.
 template <int NW, bool MOL>
-__global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_constant__ FilterParams fp) {
+__global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __grid_constant__ FilterParams fp) {
   using M = Mask<NW>;
   constexpr int NT = kFilterThreads, NWARP = NT / 32;
   extern __shared__ __align__(16) unsigned char smem[];
@@ -614,14 +633,6 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
     if (!MOL)
       for (int i = tid; i <= fp.VQ; i += NT) b[i] = fp.rowp_off[i];
     for (int i = tid; i < fp.NRP; i += NT) c[i] = fp.rowp[i];
-  }
-  if (MOL) {
-    uint32_t *dnz = (uint32_t *)(smem + L.dnz);
-    int32_t *qwo = (int32_t *)(smem + L.qdr);
-    uint2 *qw = (uint2 *)(smem + L.qdr + align16(4 * (size_t)(fp.NQ + 1)));
-    for (int i = tid; i < 32 * ((fp.NDR + 31) >> 5); i += NT) dnz[i] = 0u;
-    for (int i = tid; i <= fp.NQ; i += NT) qwo[i] = __ldg(&fp.qw_off[i]);
-    for (int i = tid; i < fp.NQWL; i += NT) qw[i] = make_uint2(__ldg(&fp.qw[2 * i]), __ldg(&fp.qw[2 * i + 1]));
   }
   if (tid < 32) {
     s_endb[tid] = 0u;
@@ -828,6 +839,14 @@ __global__ void __launch_bounds__(kFilterThreads, 4) k_filter(const __grid_const
     const unsigned long long nmask = n >= 64 ? ~0ull : ((1ull << n) - 1ull);
     const int ws = ms >> 5, sh = ms & 31;
     uint32_t *dnz = (uint32_t *)(smem + L.dnz);  // [NDR/32][32 molecules]
+    {  // these regions alias the BFS / plane-carry arrays, dead from here on
+      int32_t *qwo = (int32_t *)(smem + L.qdr);
+      uint2 *qw = (uint2 *)(smem + L.qdr + align16(4 * (size_t)(fp.NQ + 1)));
+      for (int i = tid; i < 32 * ((fp.NDR + 31) >> 5); i += NT) dnz[i] = 0u;
+      for (int i = tid; i <= fp.NQ; i += NT) qwo[i] = __ldg(&fp.qw_off[i]);
+      for (int i = tid; i < fp.NQWL; i += NT) qw[i] = make_uint2(__ldg(&fp.qw[2 * i]), __ldg(&fp.qw[2 * i + 1]));
+    }
+    __syncthreads();
     // per warp: 4 rows x 32 molecules of windows, staged so that the stores
     // to cmol[g][row] (molecule-major) go out as 32-B sectors per molecule
     unsigned long long *stg = (unsigned long long *)(smem + L.stg) + (size_t)wid * (4 * 33);
