@@ -1177,7 +1177,8 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       rows_smem = 1;
       smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NDR * m.RW, 1,
                                c->NQW, m.TS, 1, m.NDR, c->NQ, m.NQWL);
-      if (smem > c->max_smem / 2) {
+      const char *rg = getenv("SIGMO_FILTER_ROWS_GLOBAL");
+      if (smem > c->max_smem / 2 || (rg && atoi(rg))) {
         rows_smem = 0;
         smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NDR * m.RW, 0,
                                  c->NQW, m.TS, 1, m.NDR, c->NQ, m.NQWL);

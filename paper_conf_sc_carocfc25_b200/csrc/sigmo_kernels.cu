@@ -467,7 +467,13 @@ __host__ __device__ inline FilterSmem filter_layout(int NW, int EXTN, int EXTW, 
   L.fid = o;      o = align16(o + (size_t)EXTN);
   L.lab = o;      o = align16(o + (size_t)EXTN);
   L.mstart = o;   o = align16(o + 4 * (size_t)(MOLCAP + 1));
-  L.sos = o;      o = align16(o + 2 * (size_t)EXTN);
+  // start-of-segment slots: used while loading the tile, before the plane
+  // phase writes memb (molecule tiles: alias memb)
+  if (mol && 2 * (size_t)EXTN <= 4 * 32 * (size_t)EXTW) {
+    L.sos = L.memb;
+  } else {
+    L.sos = o; o = align16(o + 2 * (size_t)EXTN);
+  }
   L.grec = o;     o = align16(o + sizeof(GroupRec) * (size_t)(NREC > 0 ? NREC : 1));
   L.tab = o;      o = align16(o + 4 * (size_t)TS * (NREC > 0 ? NREC : 1));
   L.bdone = o;    o = align16(o + (size_t)(P / 32 + 1));
@@ -850,8 +856,9 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
     // per warp: 4 rows x 32 molecules of windows, staged so that the stores
     // to cmol[g][row] (molecule-major) go out as 32-B sectors per molecule
     unsigned long long *stg = (unsigned long long *)(smem + L.stg) + (size_t)wid * (4 * 33);
-    auto mol_rows = [&](auto RWc, auto HIc, const uint32_t *rowp) {
+    auto mol_rows = [&](auto RWc, auto HIc, const uint32_t *rowp, auto GLc) {
       constexpr int RWk = decltype(RWc)::value;
+      constexpr bool GL = decltype(GLc)::value;  // row programs in global memory (read-only path)
       constexpr bool HI = decltype(HIc)::value;  // the tile spans more than 32 words
       const int RW = RWk ? RWk : fp.RW;
       const unsigned char *pl0 = (const unsigned char *)(s_pl + (size_t)(lane < nxw ? lane : 0) * PS);
@@ -865,12 +872,12 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
         uint32_t x0 = 0xffffffffu, x1 = 0xffffffffu;
 #pragma unroll
         for (int j = 0; j < (RWk ? RWk : 1); j++) {
-          const uint32_t two = pr[j];
+          const uint32_t two = GL ? __ldg(&pr[j]) : pr[j];
           x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
           if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
         }
         for (int j = RWk; j < RW; j++) {
-          const uint32_t two = pr[j];
+          const uint32_t two = GL ? __ldg(&pr[j]) : pr[j];
           x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
           if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
         }
@@ -906,18 +913,26 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
     if (fp.rows_smem) {
       const uint32_t *rs = (const uint32_t *)(smem + L.rowp);
       switch (hi ? 0 : fp.RW) {
-        case 1: mol_rows(std::integral_constant<int, 1>{}, std::false_type{}, rs); break;
-        case 2: mol_rows(std::integral_constant<int, 2>{}, std::false_type{}, rs); break;
-        case 3: mol_rows(std::integral_constant<int, 3>{}, std::false_type{}, rs); break;
-        case 4: mol_rows(std::integral_constant<int, 4>{}, std::false_type{}, rs); break;
+        case 1: mol_rows(std::integral_constant<int, 1>{}, std::false_type{}, rs, std::false_type{}); break;
+        case 2: mol_rows(std::integral_constant<int, 2>{}, std::false_type{}, rs, std::false_type{}); break;
+        case 3: mol_rows(std::integral_constant<int, 3>{}, std::false_type{}, rs, std::false_type{}); break;
+        case 4: mol_rows(std::integral_constant<int, 4>{}, std::false_type{}, rs, std::false_type{}); break;
         default:
-          if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, rs);
-          else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, rs);
+          if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, rs, std::false_type{});
+          else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, rs, std::false_type{});
           break;
       }
-    } else {
-      if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, fp.rowp);
-      else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, fp.rowp);
+    } else {  // row programs read through the read-only cache (warp-uniform loads)
+      const uint32_t *rg = fp.rowp;
+      switch (hi ? 0 : fp.RW) {
+        case 2: mol_rows(std::integral_constant<int, 2>{}, std::false_type{}, rg, std::true_type{}); break;
+        case 3: mol_rows(std::integral_constant<int, 3>{}, std::false_type{}, rg, std::true_type{}); break;
+        case 4: mol_rows(std::integral_constant<int, 4>{}, std::false_type{}, rg, std::true_type{}); break;
+        default:
+          if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, rg, std::true_type{});
+          else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, rg, std::true_type{});
+          break;
+      }
     }
     __syncthreads();
     // GMCR: lane = molecule, warp per query: every node's distinct row
