@@ -131,14 +131,15 @@ struct sigmo_ctx {
   int PC = 512, AC = 512, CMC = 2048, MC = 128;
 
   // ---- join ----
-  DBuf pair_query, pair_rec, pair_cm, pair_result, jcnt, adjb;
+  DBuf pair_query, pair_rec, pair_cm, pair_result, jcnt, adjb, ent2;
   // jcnt u64 slots: [0] pair cursor / chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
   bool lane_join = false;  // per-lane join possible for this batch (<= 64-node graphs, <= 16-node queries)
   bool mol_filter = false; // last sigmo_filter used molecule tiles (candidates in cmol layout)
   // plan entries as loaded (host) and the query node of each plan position;
   // bits 12.. of .x are set to the distinct row of that node for the R whose
   // program last ran (ent_R), re-uploaded when R changes
-  std::vector<int4> ent_host, ent_up;
+  std::vector<int4> ent_host;
+  std::vector<uint2> ent_up;  // compact entries for k_join_lane (8 B): see JoinParams::qp_ent2
   std::vector<int32_t> ent_row;
   std::vector<int64_t> qgoff_host;  // query graph offsets (host copy, for the per-query row-word lists)
   int ent_R = -1;
@@ -771,7 +772,7 @@ void free_all(sigmo_ctx *c) {
   c->progs.clear();
   DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
                   &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_rec, &c->pair_cm, &c->pair_result, &c->jcnt,
-                  &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp};
+                  &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp, &c->ent2};
   for (DBuf *b : bufs) dfree(c, *b);
 }
 
@@ -970,7 +971,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     lane_ok = maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
               (unsigned long long)std::max<int64_t>(hq.V, 1) * (unsigned long long)std::max<int64_t>(hd.G, 1) <
                   (1ull << 32) &&
-              (unsigned long long)(c->NB + 1) * hd.V + 1 < (1ull << 31);
+              (unsigned long long)(c->NB + 1) * hd.V + 1 < (1ull << 31) &&
+              plan.be.size() + 2 < 0xffff;  // compact plan entries: 16-bit extra back-edge offsets
   }
   // ---- staging layout ----
   Layout L;
@@ -1242,11 +1244,15 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     if (mol && c->ent_R != R) {
       // distinct-row index of each plan position's query node into the plan entries
       const std::vector<uint16_t> &qd = c->progs[R].qdrow;
-      c->ent_up = c->ent_host;
-      for (size_t i = 0; i < c->ent_up.size(); i++)
-        c->ent_up[i].x = (c->ent_up[i].x & 0xfff) | ((int)qd[(size_t)c->ent_row[i]] << 12);
+      c->ent_up.resize(c->ent_host.size());
+      for (size_t i = 0; i < c->ent_up.size(); i++) {
+        const int4 e = c->ent_host[i];
+        c->ent_up[i].x = ((unsigned)e.x & 0xfffu) | ((unsigned)qd[(size_t)c->ent_row[i]] << 12);
+        c->ent_up[i].y = ((unsigned)e.w & 0xffffu) | ((unsigned)e.y << 16) | ((unsigned)e.z << 19);
+      }
+      SIGMO_TRY(dreserve(c, c->ent2, sizeof(uint2) * (c->ent_up.size() + 1), "plan entries"));
       if (!c->ent_up.empty())
-        CUDA_TRY(c, cudaMemcpyAsync((void *)c->qp_ent, c->ent_up.data(), sizeof(int4) * c->ent_up.size(),
+        CUDA_TRY(c, cudaMemcpyAsync(c->ent2.p, c->ent_up.data(), sizeof(uint2) * c->ent_up.size(),
                                     cudaMemcpyHostToDevice, c->stream));
       c->ent_R = R;
     }
@@ -1374,6 +1380,7 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       jp.prec = (const int4 *)c->pair_rec.p;
       jp.adjb = (const unsigned long long *)c->adjb.p;
       jp.qp_ent = c->qp_ent;
+      jp.qp_ent2 = (const uint2 *)c->ent2.p;
       jp.cmol = (const unsigned long long *)c->bitmap.p;
       // refill batch (lanes that must be free before a warp refills): swept on
       // configs[2], FA 2/4/8/16 -> 11.2/10.3/9.7/9.9 ms, FF 10.4/9.8/9.2/9.0 ms

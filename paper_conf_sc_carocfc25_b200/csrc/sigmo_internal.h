@@ -150,6 +150,8 @@ struct JoinParams {
   const unsigned long long *cmol;  // [ND][VQ] molecule-padded candidate windows (filter output)
   const unsigned long long *adjb;  // [VD][NB] bond-class adjacency masks (molecule-local bits) + all-ones entry
   const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 4 (15 none) | #extra << 8 | node << 12, class0, class1, extra back-edge start}
+  const uint2 *qp_ent2;        // [VQ] compact, k_join_lane: x = j0 | j1 << 4 | #extra << 8 | distinct row << 12,
+                               // y = extra back-edge start (16 b) | class0 << 16 | class1 << 19
   int batchK;                  // finish/assign pairs when >= batchK lanes are free
 };
 

@@ -2013,7 +2013,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   // candidate rows in lane-private shared memory by cp.async, 10.6 vs 9.8 ms
   // -- both lose to the occupancy they cost; so did taking two leaf-level
   // candidates per step, 9.60 vs 9.49 ms)
-  const int4 *const qp_ent = jp.qp_ent;
+  const uint2 *const qp_ent = jp.qp_ent2;  // 8-B entries: more lanes share a sector
   const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ) + (size_t)wid * join_lane_warp_bytes(MQ));
   const unsigned oRU = wbase + 16u * lane;                        // {R, U} of depth d: oRU + 512 d
   const unsigned oM = wbase + 512u * SD + lane;                   // f(pi_d): oM + 32 d
@@ -2065,7 +2065,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const unsigned od = oRU + 512u * d;
       // the plan entry of depth e and the map bytes of its back-edge targets
       // depend on d only: loaded before v is known (j == d takes v below)
-      const int4 en = __ldg(&qp_ent[cqb + e]);
+      const uint2 en = __ldg(&qp_ent[cqb + e]);
       const ulonglong2 RU = LDS128(od);
       const unsigned j0 = en.x & 15, j1 = (en.x >> 4) & 15;
       const unsigned m0 = smem[oM + 32u * j0], m1 = smem[oM + 32u * j1];
@@ -2080,13 +2080,13 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       // candidates of depth e
       const unsigned u0 = j0 == (unsigned)d ? (unsigned)v : m0, u1 = j1 == (unsigned)d ? (unsigned)v : m1;
       const unsigned ng = (cinfo >> 8) & 0xffu;  // molecule size: class stride of adjb
-      const unsigned i0 = j0 == 15u ? ones : ca + (unsigned)en.y * ng + u0;
-      const unsigned i1 = j1 == 15u ? ones : ca + (unsigned)en.z * ng + u1;
+      const unsigned i0 = j0 == 15u ? ones : ca + ((en.y >> 16) & 7u) * ng + u0;
+      const unsigned i1 = j1 == 15u ? ones : ca + ((en.y >> 19) & 7u) * ng + u1;
       unsigned long long X = __ldg(&cmol[cmb + ((unsigned)en.x >> 12)]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
       if (en.x & 0xf00) {  // > 2 back-edges at this depth (fused rings): rare
         const int nex = (en.x >> 8) & 15;
         for (int k = 0; k < nex; k++) {
-          const int be = __ldg(&jp.qp_be[en.w + k]);
+          const int be = __ldg(&jp.qp_be[(en.y & 0xffffu) + k]);
           X &= __ldg(&adjb[ca + (unsigned)(be & 255) * ng + smem[oM + 32u * (be >> 8)]]);
         }
       }
