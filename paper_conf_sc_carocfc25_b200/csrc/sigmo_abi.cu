@@ -1169,7 +1169,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     const QueryProgMeta &m = prog->meta;
     // molecule tiles (cmol layout for the per-lane join) unless the
     // neighbour-support pass (dense bitmap) is requested
-    bool mol = c->lane_join && !(flags & SIGMO_FILTER_NEIGHBOR_SUPPORT);
+    bool mol = c->lane_join && !(flags & SIGMO_FILTER_NEIGHBOR_SUPPORT) && c->mol_extn <= 1024;  // one word per lane
     // tile width: largest TW whose shared memory fits
     const int tws[6] = {32, 16, 8, 4, 2, 1};
     int k = 0;

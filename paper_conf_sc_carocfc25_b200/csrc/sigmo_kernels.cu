@@ -856,44 +856,31 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
     // per warp: 4 rows x 32 molecules of windows, staged so that the stores
     // to cmol[g][row] (molecule-major) go out as 32-B sectors per molecule
     unsigned long long *stg = (unsigned long long *)(smem + L.stg) + (size_t)wid * (4 * 33);
-    auto mol_rows = [&](auto RWc, auto HIc, const uint32_t *rowp, auto GLc) {
+    // tiles hold <= 1,024 nodes: nxw <= 32 words, one per lane
+    auto mol_rows = [&](auto RWc, const uint32_t *rowp, auto GLc) {
       constexpr int RWk = decltype(RWc)::value;
       constexpr bool GL = decltype(GLc)::value;  // row programs in global memory (read-only path)
-      constexpr bool HI = decltype(HIc)::value;  // the tile spans more than 32 words
       const int RW = RWk ? RWk : fp.RW;
       const unsigned char *pl0 = (const unsigned char *)(s_pl + (size_t)(lane < nxw ? lane : 0) * PS);
-      const unsigned char *pl1 = (const unsigned char *)(s_pl + (size_t)(lane + 32 < nxw ? lane + 32 : 0) * PS);
       for (int rb = 4 * wid; rb < fp.NDR; rb += 4 * NWARP) {  // blocks of 4 rows per warp
       const int nr = min(4, fp.NDR - rb);
       uint32_t nzb = 0u;
       for (int r = 0; r < nr; r++) {
         const int row = rb + r;
         const uint32_t *pr = rowp + (size_t)row * RW;
-        uint32_t x0 = 0xffffffffu, x1 = 0xffffffffu;
+        uint32_t x0 = 0xffffffffu;
 #pragma unroll
         for (int j = 0; j < (RWk ? RWk : 1); j++) {
           const uint32_t two = GL ? __ldg(&pr[j]) : pr[j];
           x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
-          if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
         }
         for (int j = RWk; j < RW; j++) {
           const uint32_t two = GL ? __ldg(&pr[j]) : pr[j];
           x0 &= *(const uint32_t *)(pl0 + (two & 0xffffu)) & *(const uint32_t *)(pl0 + (two >> 16));
-          if (HI) x1 &= *(const uint32_t *)(pl1 + (two & 0xffffu)) & *(const uint32_t *)(pl1 + (two >> 16));
         }
-        uint32_t w0, w1, w2;
-        if (HI) {
-          const uint32_t a0 = __shfl_sync(FULL_MASK, x0, ws & 31), b0 = __shfl_sync(FULL_MASK, x1, ws & 31);
-          const uint32_t a1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31), b1 = __shfl_sync(FULL_MASK, x1, (ws + 1) & 31);
-          const uint32_t a2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31), b2 = __shfl_sync(FULL_MASK, x1, (ws + 2) & 31);
-          w0 = ws < 32 ? a0 : b0;
-          w1 = ws + 1 < 32 ? a1 : b1;
-          w2 = ws + 2 < 32 ? a2 : b2;
-        } else {
-          w0 = __shfl_sync(FULL_MASK, x0, ws);
-          w1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31);
-          w2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31);
-        }
+        const uint32_t w0 = __shfl_sync(FULL_MASK, x0, ws);
+        const uint32_t w1 = __shfl_sync(FULL_MASK, x0, (ws + 1) & 31);
+        const uint32_t w2 = __shfl_sync(FULL_MASK, x0, (ws + 2) & 31);
         const unsigned long long x =
             (((unsigned long long)__funnelshift_r(w1, w2, sh) << 32) | __funnelshift_r(w0, w1, sh)) & nmask;
         stg[r * 33 + mi] = x;
@@ -909,29 +896,22 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
       __syncwarp();
       }
     };
-    const bool hi = nxw > 32;
     if (fp.rows_smem) {
       const uint32_t *rs = (const uint32_t *)(smem + L.rowp);
-      switch (hi ? 0 : fp.RW) {
-        case 1: mol_rows(std::integral_constant<int, 1>{}, std::false_type{}, rs, std::false_type{}); break;
-        case 2: mol_rows(std::integral_constant<int, 2>{}, std::false_type{}, rs, std::false_type{}); break;
-        case 3: mol_rows(std::integral_constant<int, 3>{}, std::false_type{}, rs, std::false_type{}); break;
-        case 4: mol_rows(std::integral_constant<int, 4>{}, std::false_type{}, rs, std::false_type{}); break;
-        default:
-          if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, rs, std::false_type{});
-          else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, rs, std::false_type{});
-          break;
+      switch (fp.RW) {
+        case 1: mol_rows(std::integral_constant<int, 1>{}, rs, std::false_type{}); break;
+        case 2: mol_rows(std::integral_constant<int, 2>{}, rs, std::false_type{}); break;
+        case 3: mol_rows(std::integral_constant<int, 3>{}, rs, std::false_type{}); break;
+        case 4: mol_rows(std::integral_constant<int, 4>{}, rs, std::false_type{}); break;
+        default: mol_rows(std::integral_constant<int, 0>{}, rs, std::false_type{}); break;
       }
     } else {  // row programs read through the read-only cache (warp-uniform loads)
       const uint32_t *rg = fp.rowp;
-      switch (hi ? 0 : fp.RW) {
-        case 2: mol_rows(std::integral_constant<int, 2>{}, std::false_type{}, rg, std::true_type{}); break;
-        case 3: mol_rows(std::integral_constant<int, 3>{}, std::false_type{}, rg, std::true_type{}); break;
-        case 4: mol_rows(std::integral_constant<int, 4>{}, std::false_type{}, rg, std::true_type{}); break;
-        default:
-          if (hi) mol_rows(std::integral_constant<int, 0>{}, std::true_type{}, rg, std::true_type{});
-          else mol_rows(std::integral_constant<int, 0>{}, std::false_type{}, rg, std::true_type{});
-          break;
+      switch (fp.RW) {
+        case 2: mol_rows(std::integral_constant<int, 2>{}, rg, std::true_type{}); break;
+        case 3: mol_rows(std::integral_constant<int, 3>{}, rg, std::true_type{}); break;
+        case 4: mol_rows(std::integral_constant<int, 4>{}, rg, std::true_type{}); break;
+        default: mol_rows(std::integral_constant<int, 0>{}, rg, std::true_type{}); break;
       }
     }
     __syncthreads();

@@ -249,6 +249,28 @@ def test_c3_bench_workload_parity(ctx, sigmo):
         assert np.array_equal(dense, (ref > 0).astype(np.uint64)), g0
 
 
+def test_filter_rows_from_global(sigmo, monkeypatch):
+    """Row programs read from global memory (the fallback when shared memory is
+    short, forced by SIGMO_FILTER_ROWS_GLOBAL): same bitmap and counts."""
+    monkeypatch.setenv("SIGMO_FILTER_ROWS_GLOBAL", "1")
+    Q, D = synth.config_queries(2), synth.config_data(2, count=3000)
+    ref = oracle.count_dense(Q, D)
+    with sigmo.Context(0) as c:
+        c.load_batch(Q, D)
+        for L in (1, 3, 4):
+            c.filter(L)
+            c.join(sigmo.SIGMO_FIND_ALL)
+            assert np.array_equal(c.dense_results(), ref), L
+        Cb = fr.candidates_bool(Q, D, 4, data_graphs=list(range(0, 3000, 97)))
+        ref_bits = fr.to_bitmap(Cb)
+        bm = c.candidates()
+        for g in range(0, 3000, 97):
+            lo, hi = int(D.graph_offsets[g]), int(D.graph_offsets[g + 1])
+            for v in range(lo, hi):
+                w, b = v >> 5, v & 31
+                assert np.array_equal((bm[:, w] >> b) & 1, (ref_bits[:, w] >> b) & 1), (g, v)
+
+
 def test_join_stack_spill_path(sigmo, monkeypatch):
     """Force the smallest shared-memory DFS stack so that the global spill /
     restore path runs (deep 20-30-atom ring-system queries), results unchanged."""
