@@ -146,6 +146,8 @@ struct sigmo_ctx {
   int mol_extn = 0, mol_extw = 0;  // molecule-tile geometry (<= 32 graphs and <= 1,024 nodes per tile)
   int n_mol_tiles = 0;
   int32_t *mol_tiles = nullptr;     // [n_mol_tiles + 1] first graph of each molecule tile
+  uint32_t *adj_off = nullptr;      // [ND + 1] 32-bit word offset of each molecule's bond-class adjacency
+  uint32_t adj_words = 0;           // adjacency words (the all-ones entry follows)
   DBuf dense_tmp;          // dense view of cmol for sigmo_get_candidates
   int last_mode = 0;
   DBuf sig_tmp, gstack;
@@ -1003,6 +1005,22 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     }
   }
   const size_t o_mt = L.take(4 * mt.size());
+  // bond-class adjacency layout (k_join_lane): per molecule class-major,
+  // 32-bit masks for <= 32-node molecules, 64-bit (even word offset) otherwise
+  std::vector<uint32_t> aoff((size_t)hd.G + 1, 0);
+  {
+    uint64_t w = 0;
+    for (int64_t g = 0; g < hd.G; g++) {
+      const int64_t n = hd.goff[g + 1] - hd.goff[g];
+      if (n > 32) w = (w + 1) & ~1ull;
+      aoff[g] = (uint32_t)std::min<uint64_t>(w, 0xffffffffull);
+      w += (uint64_t)n * (uint64_t)std::max(c->NB, 1) * (n > 32 ? 2 : 1);
+    }
+    w = (w + 1) & ~1ull;
+    aoff[hd.G] = (uint32_t)std::min<uint64_t>(w, 0xffffffffull);
+    if (w + 2 >= (1ull << 32)) lane_ok = false;
+  }
+  const size_t o_ao = L.take(4 * aoff.size());
   const size_t total = L.off;
   // wait until the previous upload no longer reads the staging buffer
   CUDA_TRY(c, cudaEventSynchronize(c->h2d_done));
@@ -1052,6 +1070,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
   memcpy(hb + o_tg1, tg1.data(), 4 * tg1.size());
   memcpy(hb + o_mt, mt.data(), 4 * mt.size());
+  memcpy(hb + o_ao, aoff.data(), 4 * aoff.size());
 
   // ---- device arena + one H2D copy ----
   SIGMO_TRY(dreserve(c, c->arena, total, "input arena"));
@@ -1067,6 +1086,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->bclass = db + o_bc;
   c->tile_g0 = (int32_t *)(db + o_tg0);
   c->mol_tiles = (int32_t *)(db + o_mt);
+  c->adj_off = (uint32_t *)(db + o_ao);
+  c->adj_words = aoff[hd.G];
   c->n_mol_tiles = (int)mt.size() - 1;
   c->tile_g1 = (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
@@ -1142,10 +1163,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->mol_filter = false;
   if (c->lane_join) {
     SIGMO_TRY(dreserve(c, c->pair_rec, 16 * (size_t)std::max(pair_cap, 1ll), "pair records"));
-    SIGMO_TRY(dreserve(c, c->adjb, 8 * ((size_t)c->NB * c->VD + 1), "bond-class adjacency"));
-    // entry VD * NB = all ones: the target of absent back-edges
-    CUDA_TRY(c, cudaMemsetAsync((unsigned long long *)c->adjb.p + (size_t)c->NB * c->VD, 0xff, 8, c->stream));
-    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, (unsigned long long *)c->adjb.p, c->stream));
+    SIGMO_TRY(dreserve(c, c->adjb, 4 * ((size_t)c->adj_words + 2), "bond-class adjacency"));
+    // words adj_words, adj_words + 1 = all ones: the target of absent back-edges
+    CUDA_TRY(c, cudaMemsetAsync((uint32_t *)c->adjb.p + c->adj_words, 0xff, 8, c->stream));
+    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, c->adj_off, (uint32_t *)c->adjb.p, c->stream));
   }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
   SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 6), "join counters"));
@@ -1319,6 +1340,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     pp.gm = (const uint32_t *)c->gm.p;
     pp.off = (const I64x2 *)c->off.p;
     pp.goff = c->dd.goff;
+    pp.adj_off = c->adj_off;
     pp.qgoff = c->dq.goff;
     pp.qp_row = c->qp_row;
     pp.bitmap = (const uint32_t *)c->bitmap.p;
@@ -1378,7 +1400,8 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       jp.maxq = std::max(c->maxq, 2);
       jp.VD = c->VD;
       jp.prec = (const int4 *)c->pair_rec.p;
-      jp.adjb = (const unsigned long long *)c->adjb.p;
+      jp.adjw = (const uint32_t *)c->adjb.p;
+      jp.adj_ones = c->adj_words;
       jp.qp_ent = c->qp_ent;
       jp.qp_ent2 = (const uint2 *)c->ent2.p;
       jp.cmol = (const unsigned long long *)c->bitmap.p;

@@ -148,7 +148,9 @@ struct JoinParams {
   int VD;                      // data nodes
   const int4 *prec;            // [P] pair records {graph start node, query, graph * VQ + first query node, qinfo[query]}
   const unsigned long long *cmol;  // [ND][VQ] molecule-padded candidate windows (filter output)
-  const unsigned long long *adjb;  // [VD][NB] bond-class adjacency masks (molecule-local bits) + all-ones entry
+  const uint32_t *adjw;        // bond-class adjacency masks (molecule-local bits), per molecule at word adj_off[g]:
+                               // class-major [NB][n], u32 masks (n <= 32) or u64 (n > 32); all ones at word adj_ones
+  unsigned adj_ones;
   const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 4 (15 none) | #extra << 8 | node << 12, class0, class1, extra back-edge start}
   const uint2 *qp_ent2;        // [VQ] compact, k_join_lane: x = j0 | j1 << 4 | #extra << 8 | distinct row << 12,
                                // y = extra back-edge start (16 b) | class0 << 16 | class1 << 19
@@ -159,6 +161,7 @@ struct JoinParams {
 struct PairsParams {
   int ND, NQ, NQW, MQ, Wpad, VQ;
   int rowstride;               // cmol row stride per graph (distinct rows)
+  const uint32_t *adj_off;     // [ND+1] adjacency word offset per graph (pair record .x)
   const uint32_t *gm;
   const I64x2 *off;
   const int32_t *goff, *qgoff, *qp_row;
@@ -206,7 +209,8 @@ cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
 cudaError_t launch_unpad(const unsigned long long *cmol, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
                          int VQ, int Wpad, uint32_t *dense,
                          cudaStream_t st);
-cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsigned long long *adjb, cudaStream_t st);
+cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
+                        cudaStream_t st);
 cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream_t st);
 size_t join_lane_smem_bytes(const JoinParams &p);
 int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem);

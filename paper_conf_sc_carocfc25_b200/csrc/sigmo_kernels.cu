@@ -1838,6 +1838,7 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
   const unsigned lt = (1u << lane) - 1u;
   long long o = pp.off[g].a;
   const int a = __ldg(&pp.goff[g]);
+  const int aw = pp.prec ? (int)__ldg(&pp.adj_off[g]) : 0;  // adjacency word offset (pair record .x)
   for (int qb = 0; qb < pp.NQW; qb++) {
     const uint32_t bits = __ldg(&pp.gm[(size_t)g * pp.NQW + qb]);
     if ((bits >> lane) & 1u) {
@@ -1847,7 +1848,7 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
       if (pp.prec) {
         // query info with the molecule size in bits 8-15 (class stride of adjb)
         const uint32_t qi = (__ldg(&pp.qinfo[q]) & ~0xff00u) | ((uint32_t)(__ldg(&pp.goff[g + 1]) - a) << 8);
-        pp.prec[p] = make_int4(a, q, (int)((unsigned)g * (unsigned)pp.rowstride), (int)qi);
+        pp.prec[p] = make_int4(aw, q, (int)((unsigned)g * (unsigned)pp.rowstride), (int)qi);
       }
     }
     o += __popc(bits);
@@ -1894,7 +1895,7 @@ cudaError_t launch_unpad(const unsigned long long *cmol, const uint16_t *qdrow, 
 // holding v, so that lanes reading the same class of one molecule touch few
 // 32-B sectors.
 // ===========================================================================
-__global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, unsigned long long *adjb) {
+__global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw) {
   const int v = blockIdx.x * blockDim.x + threadIdx.x;
   if (v >= d.num_nodes) return;
   unsigned long long m[8];
@@ -1910,14 +1911,19 @@ __global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, unsigned long
   }
   const int g = graph_of(d.goff, d.num_graphs, v);
   const int a = d.goff[g], n = d.goff[g + 1] - a;
+  const uint32_t base = adj_off[g];
 #pragma unroll
   for (int b = 0; b < 8; b++)
-    if (b < NB) adjb[(size_t)a * NB + (size_t)b * n + (v - a)] = m[b];
+    if (b < NB) {
+      if (n <= 32) adjw[base + (uint32_t)(b * n + (v - a))] = (uint32_t)m[b];
+      else *(unsigned long long *)(adjw + base + 2u * (uint32_t)(b * n + (v - a))) = m[b];
+    }
 }
 
-cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, unsigned long long *adjb, cudaStream_t st) {
+cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
+                        cudaStream_t st) {
   if (d.num_nodes <= 0 || NB <= 0) return cudaSuccess;
-  k_adjb<<<(d.num_nodes + 255) / 256, 256, 0, st>>>(d, bclass, NB, adjb);
+  k_adjb<<<(d.num_nodes + 255) / 256, 256, 0, st>>>(d, bclass, NB, adj_off, adjw);
   return cudaGetLastError();
 }
 
@@ -2004,10 +2010,13 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   const unsigned lt = (1u << lane) - 1u;
   const unsigned P = (unsigned)jp.off[jp.ND].a;
   unsigned *const cursor = (unsigned *)jp.chunk_counter;
-  const unsigned long long *const adjb = jp.adjb;
+  const uint32_t *const adjw = jp.adjw;
+  // mask of adjacency word index i: 32-bit for <= 32-node molecules, else 64-bit
+  auto adj = [&](bool wide, unsigned i) -> unsigned long long {
+    return wide ? __ldg((const unsigned long long *)(adjw + i)) : (unsigned long long)__ldg(adjw + i);
+  };
   const unsigned long long *const cmol = jp.cmol;
-  const unsigned NB = (unsigned)jp.NB;
-  const unsigned ones = (unsigned)jp.VD * NB;  // the all-ones entry (absent back-edge)
+  const unsigned ones = jp.adj_ones;  // the all-ones entry (absent back-edge)
   const int4 zero4 = make_int4(0, 0, 0, 0);
 
   // ---- GMCR chunks: current (records of pairs cbase + i in lane i's crec), prefetched, claimed ----
@@ -2060,15 +2069,17 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const unsigned long long used = RU.y | bit;
       // candidates of depth e
       const unsigned u0 = j0 == (unsigned)d ? (unsigned)v : m0, u1 = j1 == (unsigned)d ? (unsigned)v : m1;
-      const unsigned ng = (cinfo >> 8) & 0xffu;  // molecule size: class stride of adjb
-      const unsigned i0 = j0 == 15u ? ones : ca + ((en.y >> 16) & 7u) * ng + u0;
-      const unsigned i1 = j1 == 15u ? ones : ca + ((en.y >> 19) & 7u) * ng + u1;
-      unsigned long long X = __ldg(&cmol[cmb + ((unsigned)en.x >> 12)]) & ~used & __ldg(&adjb[i0]) & __ldg(&adjb[i1]);
+      const unsigned ng = (cinfo >> 8) & 0xffu;  // molecule size: class stride of the adjacency
+      const bool wide = ng > 32u;
+      const unsigned sw = wide ? 1u : 0u;  // word shift of an entry
+      const unsigned i0 = j0 == 15u ? ones : ca + ((((en.y >> 16) & 7u) * ng + u0) << sw);
+      const unsigned i1 = j1 == 15u ? ones : ca + ((((en.y >> 19) & 7u) * ng + u1) << sw);
+      unsigned long long X = __ldg(&cmol[cmb + ((unsigned)en.x >> 12)]) & ~used & adj(wide, i0) & adj(wide, i1);
       if (en.x & 0xf00) {  // > 2 back-edges at this depth (fused rings): rare
         const int nex = (en.x >> 8) & 15;
         for (int k = 0; k < nex; k++) {
           const int be = __ldg(&jp.qp_be[(en.y & 0xffffu) + k]);
-          X &= __ldg(&adjb[ca + (unsigned)(be & 255) * ng + smem[oM + 32u * (be >> 8)]]);
+          X &= adj(wide, ca + (((unsigned)(be & 255) * ng + smem[oM + 32u * (be >> 8)]) << sw));
         }
       }
       if (e == (int)(cinfo & 0xff) - 1) {
@@ -2104,7 +2115,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     if (ne == 0u && nv) {
       cp = np;
       cmb = (unsigned)nrec.z;
-      ca = (unsigned)nrec.x * NB;
+      ca = (unsigned)nrec.x;  // adjacency word offset of the molecule
       cq = nrec.y;
       cinfo = (unsigned)nrec.w;
       cqb = cinfo >> 16;
