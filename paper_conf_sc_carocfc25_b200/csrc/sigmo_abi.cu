@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <atomic>
 #include <cstdarg>
 #include <cstdio>
@@ -135,6 +136,8 @@ struct sigmo_ctx {
   // jcnt u64 slots: [0] pair cursor / chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
   bool lane_join = false;  // per-lane join possible for this batch (<= 64-node graphs, <= 16-node queries)
   bool mol_filter = false; // last sigmo_filter used molecule tiles (candidates in cmol layout)
+  bool dense_pad_zero = false;  // padding words >= W of the dense bitmap rows (and the tail) are zero
+  size_t bm_bytes = 0;
   // plan entries as loaded (host) and the query node of each plan position;
   // bits 12.. of .x are set to the distinct row of that node for the R whose
   // program last ran (ent_R), re-uploaded when R changes
@@ -238,8 +241,18 @@ sigmo_status validate(const sigmo_graph_batch *b, int is_query, std::string &msg
   }
   if (go[G] != V) return fail(SIGMO_ERR_INVALID_GRAPH, "graph_offsets[num_graphs] = %lld != num_nodes %lld", go[G], V);
   if (ro[0] != 0) return fail(SIGMO_ERR_INVALID_GRAPH, "row_offsets[0] = %lld, expected 0", ro[0], 0);
-  for (int64_t v = 0; v < V; v++)
-    if (ro[v + 1] < ro[v]) return fail(SIGMO_ERR_INVALID_GRAPH, "row_offsets decreasing at node %lld (%lld)", v, ro[v + 1]);
+  {
+    std::vector<int64_t> bad(64, -1);
+    parallel_for_graphs(V, V, [&](int th, int64_t a, int64_t b) {
+      for (int64_t v = a; v < b; v++)
+        if (ro[v + 1] < ro[v]) {
+          bad[th] = v;
+          return;
+        }
+    });
+    for (int64_t v : bad)
+      if (v >= 0) return fail(SIGMO_ERR_INVALID_GRAPH, "row_offsets decreasing at node %lld (%lld)", v, ro[v + 1]);
+  }
   const int64_t E = ro[V];
   if (E >= (1ll << 31) - 1) return fail(SIGMO_ERR_LIMIT, "adjacency entries %lld >= 2^31-1", E, 0);
   if (V > 0 && !b->node_labels) return fail(SIGMO_ERR_INVALID_ARG, "node_labels NULL", 0, 0);
@@ -746,15 +759,19 @@ sigmo_status ensure_prog(sigmo_ctx *c, int R, QueryProg *&out) {
 
 // per-TW tile geometry (EXTN, EXTW, MOLCAP) of the data batch
 void tile_geometry(sigmo_ctx *c, const HostGraphs &d) {
+  // one monotone sweep per tile width (the graph of a node only moves forward)
   const int tws[6] = {32, 16, 8, 4, 2, 1};
   for (int k = 0; k < 6; k++) {
     const int TW = tws[k];
     int extn = 1, extw = 1, molcap = 1;
     const int64_t W = c->W;
+    int64_t ga = 0, gb = 0;  // graph of the tile's first / last node
     for (int64_t w0 = 0; w0 < W; w0 += TW) {
       const int64_t n0 = w0 * 32, n1 = std::min<int64_t>(n0 + 32ll * TW, d.V);
-      const int g0 = graph_of_host(d.goff, d.G, n0);
-      const int g1 = graph_of_host(d.goff, d.G, n1 - 1) + 1;
+      while (ga + 1 <= d.G && d.goff[ga + 1] <= n0) ga++;
+      if (gb < ga) gb = ga;
+      while (gb + 1 <= d.G && d.goff[gb + 1] <= n1 - 1) gb++;
+      const int g0 = (int)ga, g1 = (int)gb + 1;
       const int64_t gs = d.goff[g0], ge = d.goff[g1];
       extn = std::max<int>(extn, (int)(ge - gs));
       extw = std::max<int>(extw, (int)(((ge - 1) >> 5) - (gs >> 5) + 1));
@@ -925,10 +942,12 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   CUDA_TRY(c, cudaSetDevice(c->device));
   HostGraphs hq, hd;
   std::string msg;
+  const auto t0 = std::chrono::steady_clock::now();
   sigmo_status s = validate(queries, 1, msg, hq);
   if (s != SIGMO_OK) return set_err(c, s, "query batch: %s", msg.c_str());
   s = validate(data, 0, msg, hd);
   if (s != SIGMO_OK) return set_err(c, s, "data batch: %s", msg.c_str());
+  const auto t1 = std::chrono::steady_clock::now();
   // bond classes = distinct query bond labels
   uint8_t bclass[256];
   memset(bclass, 255, sizeof(bclass));
@@ -947,7 +966,15 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->state = 0;
   // label frequencies of the data batch (planner heuristic)
   std::vector<int64_t> freq(256, 0);
-  for (int64_t v = 0; v < hd.V; v++) freq[hd.nlab[v]]++;
+  {
+    std::vector<std::vector<int64_t>> part(64, std::vector<int64_t>(256, 0));
+    parallel_for_graphs(hd.V, hd.V, [&](int th, int64_t a, int64_t b) {
+      int64_t *f = part[th].data();
+      for (int64_t v = a; v < b; v++) f[hd.nlab[v]]++;
+    });
+    for (const auto &p : part)
+      for (int l = 0; l < 256; l++) freq[l] += p[l];
+  }
   QPlan plan;
   plan_queries(hq, freq, bclass, plan);
 
@@ -976,6 +1003,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
               (unsigned long long)(c->NB + 1) * hd.V + 1 < (1ull << 31) &&
               plan.be.size() + 2 < 0xffff;  // compact plan entries: 16-bit extra back-edge offsets
   }
+  const auto t2 = std::chrono::steady_clock::now();
   // ---- staging layout ----
   Layout L;
   const PackedOffsets pq = plan_graphs(L, hq);
@@ -1022,6 +1050,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   }
   const size_t o_ao = L.take(4 * aoff.size());
   const size_t total = L.off;
+  const auto t3 = std::chrono::steady_clock::now();
   // wait until the previous upload no longer reads the staging buffer
   CUDA_TRY(c, cudaEventSynchronize(c->h2d_done));
   if (c->staging.cap < total) {
@@ -1072,6 +1101,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   memcpy(hb + o_mt, mt.data(), 4 * mt.size());
   memcpy(hb + o_ao, aoff.data(), 4 * aoff.size());
 
+  const auto t4 = std::chrono::steady_clock::now();
   // ---- device arena + one H2D copy ----
   SIGMO_TRY(dreserve(c, c->arena, total, "input arena"));
   unsigned char *db = (unsigned char *)c->arena.p;
@@ -1141,10 +1171,9 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   // (+64 B: the join reads up to two words past a molecule window)
   size_t bm_bytes = 4 * (size_t)std::max(c->VQ, 1) * c->Wpad + 64;
   if (lane_ok) bm_bytes = std::max(bm_bytes, 8 * (size_t)std::max(c->VQ, 1) * std::max(c->ND, 1));  // cmol layout
-  const bool bm_grow = c->bitmap.cap < bm_bytes;
   SIGMO_TRY(dreserve(c, c->bitmap, bm_bytes, "candidate bitmap"));
-  // padding words (>= W) are never written by the filter: zero once
-  if (bm_grow || true) CUDA_TRY(c, cudaMemsetAsync(c->bitmap.p, 0, bm_bytes, c->stream));
+  c->dense_pad_zero = false;  // zeroed before the first dense-tile filter (sigmo_filter)
+  c->bm_bytes = bm_bytes;
   SIGMO_TRY(dreserve(c, c->gm, 4 * (size_t)std::max(c->ND, 1) * std::max(c->NQW, 1), "gmcr bits"));
   SIGMO_TRY(dreserve(c, c->mol_cnt, sizeof(I64x2) * ((size_t)c->ND + 1), "gmcr counts"));
   CUDA_TRY(c, cudaMemsetAsync(c->mol_cnt.p, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
@@ -1170,6 +1199,14 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
   SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 6), "join counters"));
+  if (getenv("SIGMO_DEBUG_LOAD")) {
+    const auto t5 = std::chrono::steady_clock::now();
+    auto ms = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
+      return std::chrono::duration<double, std::milli>(b - a).count();
+    };
+    fprintf(stderr, "sigmo load: validate %.1f  plan %.1f  layout %.1f  pack %.1f  h2d+device %.1f  (%.1f) ms\n",
+            ms(t0, t1), ms(t1, t2), ms(t2, t3), ms(t3, t4), ms(t4, t5), 0.0);
+  }
   c->state = 1;
   c->err.clear();
   return SIGMO_OK;
@@ -1221,6 +1258,18 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       k = k % 6;
     }
     c->mol_filter = mol;
+    if (mol) {
+      c->dense_pad_zero = false;  // the molecule-padded layout overwrites the dense padding
+    } else if (!c->dense_pad_zero) {
+      // the dense filter writes words [0, W) of every row; the padding words
+      // (read past molecule windows by the general join) and the tail are zero
+      if (c->Wpad > c->W)
+        CUDA_TRY(c, cudaMemset2DAsync((uint32_t *)c->bitmap.p + c->W, 4 * (size_t)c->Wpad, 0, 4 * (size_t)(c->Wpad - c->W),
+                                      (size_t)std::max(c->VQ, 1), c->stream));
+      const size_t used = 4 * (size_t)std::max(c->VQ, 1) * c->Wpad;
+      if (c->bm_bytes > used) CUDA_TRY(c, cudaMemsetAsync((char *)c->bitmap.p + used, 0, c->bm_bytes - used, c->stream));
+      c->dense_pad_zero = true;
+    }
     FilterParams fp{};
     fp.D = c->dd;
     fp.TW = tws[k];
