@@ -121,6 +121,8 @@ struct sigmo_ctx {
   uint8_t *bclass = nullptr;
   // filter tile geometry per TW (32,16,8,4,2,1)
   int tile_extn[6] = {}, tile_extw[6] = {}, tile_molcap[6] = {};
+  bool tile_geom_ok = false;         // dense-tile geometry computed (lazily, first dense-tile filter)
+  std::vector<int64_t> goff_host;    // data graph offsets (host copy for the lazy geometry)
 
   // ---- filter ----
   std::map<int, ProgCache> progs;  // keyed by R = levels-1
@@ -265,42 +267,55 @@ sigmo_status validate(const sigmo_graph_batch *b, int is_query, std::string &msg
   std::vector<sigmo_status> bad_st(64, SIGMO_OK);
   parallel_for_graphs(G, E + V, [&](int t, int64_t ga, int64_t gb) {
     char buf[256];
+    // graphs of <= 64 nodes: neighbour bitmasks and a local label matrix
+    // replace the per-edge row scans (duplicate / symmetry checks)
+    std::vector<uint64_t> nbm(64);
+    std::vector<uint8_t> elm(64 * 64);
+    auto report = [&](int64_t g, const char *why, long long a1, long long a2) {
+      snprintf(buf, sizeof(buf), why, a1, a2);
+      bad_graph[t] = g;
+      bad_msg[t] = buf;
+      bad_st[t] = SIGMO_ERR_INVALID_GRAPH;
+    };
     for (int64_t g = ga; g < gb; g++) {
       const int64_t lo = go[g], hi = go[g + 1];
+      if (hi - lo <= 64) {
+        const int n = (int)(hi - lo);
+        for (int i = 0; i < n; i++) nbm[i] = 0ull;
+        for (int64_t u = lo; u < hi; u++) {
+          const int ul = (int)(u - lo);
+          for (int64_t e = ro[u]; e < ro[u + 1]; e++) {
+            const int64_t v = col[e];
+            if (v < lo || v >= hi) return report(g, "column %lld of node %lld outside its graph", v, u);
+            if (v == u) return report(g, "self-loop at node %lld", u, 0);
+            const int vl = (int)(v - lo);
+            if ((nbm[ul] >> vl) & 1ull) return report(g, "duplicate edge %lld -> %lld", u, v);
+            nbm[ul] |= 1ull << vl;
+            elm[ul * 64 + vl] = el[e];
+          }
+        }
+        for (int64_t u = lo; u < hi; u++) {
+          const int ul = (int)(u - lo);
+          for (int64_t e = ro[u]; e < ro[u + 1]; e++) {
+            const int vl = (int)(col[e] - lo);
+            if (!((nbm[vl] >> ul) & 1ull) || elm[vl * 64 + ul] != el[e])
+              return report(g, "asymmetric edge or edge label %lld -> %lld", u, (long long)col[e]);
+          }
+        }
+        continue;
+      }
       for (int64_t u = lo; u < hi; u++) {
         for (int64_t e = ro[u]; e < ro[u + 1]; e++) {
           const int64_t v = col[e];
-          const char *why = nullptr;
-          long long a1 = 0, a2 = 0;
-          if (v < lo || v >= hi) {
-            why = "column %lld of node %lld outside its graph";
-            a1 = v; a2 = u;
-          } else if (v == u) {
-            why = "self-loop at node %lld";
-            a1 = u;
-          } else {
-            int dup = 0;
-            for (int64_t f = ro[u]; f < ro[u + 1]; f++) dup += (col[f] == v);
-            if (dup > 1) {
-              why = "duplicate edge %lld -> %lld";
-              a1 = u; a2 = v;
-            } else {
-              bool sym = false;
-              for (int64_t f = ro[v]; f < ro[v + 1] && !sym; f++)
-                if (col[f] == u && el[f] == el[e]) sym = true;
-              if (!sym) {
-                why = "asymmetric edge or edge label %lld -> %lld";
-                a1 = u; a2 = v;
-              }
-            }
-          }
-          if (why) {
-            snprintf(buf, sizeof(buf), why, a1, a2);
-            bad_graph[t] = g;
-            bad_msg[t] = buf;
-            bad_st[t] = SIGMO_ERR_INVALID_GRAPH;
-            return;
-          }
+          if (v < lo || v >= hi) return report(g, "column %lld of node %lld outside its graph", v, u);
+          if (v == u) return report(g, "self-loop at node %lld", u, 0);
+          int dup = 0;
+          for (int64_t f = ro[u]; f < ro[u + 1]; f++) dup += (col[f] == v);
+          if (dup > 1) return report(g, "duplicate edge %lld -> %lld", u, v);
+          bool sym = false;
+          for (int64_t f = ro[v]; f < ro[v + 1] && !sym; f++)
+            if (col[f] == u && el[f] == el[e]) sym = true;
+          if (!sym) return report(g, "asymmetric edge or edge label %lld -> %lld", u, v);
         }
       }
     }
@@ -1138,7 +1153,13 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->W = (c->VD + 31) / 32;
   c->Wpad = ((c->W + 31) / 32) * 32;
   if (c->Wpad == 0) c->Wpad = 32;
-  tile_geometry(c, hd);
+  // dense-tile geometry: now if the dense path is the only one, else lazily
+  c->goff_host.assign(hd.goff, hd.goff + hd.G + 1);
+  c->tile_geom_ok = false;
+  if (!lane_ok) {
+    tile_geometry(c, hd);
+    c->tile_geom_ok = true;
+  }
   {
     int extn = 1;
     for (int t = 0; t < c->n_mol_tiles; t++) extn = std::max<int>(extn, (int)(hd.goff[mt[t + 1]] - hd.goff[mt[t]]));
@@ -1244,6 +1265,14 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
                                  c->NQW, m.TS, 1, m.NDR, c->NQ, m.NQWL);
       }
       if (smem > c->max_smem) mol = false;  // fall back to dense tiles
+    }
+    if (!mol && !c->tile_geom_ok) {
+      HostGraphs hg;
+      hg.G = c->ND;
+      hg.V = c->VD;
+      hg.goff = c->goff_host.data();
+      tile_geometry(c, hg);
+      c->tile_geom_ok = true;
     }
     if (!mol) {
       for (k = 0; k < 12; k++) {
