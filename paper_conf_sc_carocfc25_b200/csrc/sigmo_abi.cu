@@ -152,6 +152,8 @@ struct sigmo_ctx {
   int n_mol_tiles = 0;
   int32_t *mol_tiles = nullptr;     // [n_mol_tiles + 1] first graph of each molecule tile
   uint32_t *adj_off = nullptr;      // [ND + 1] 32-bit word offset of each molecule's bond-class adjacency
+  uint32_t *cand_units = nullptr;   // [ND + 1] candidate-window units before each molecule (x NDR = its cmol word offset)
+  uint32_t cand_total = 0;
   uint32_t adj_words = 0;           // adjacency words (the all-ones entry follows)
   DBuf dense_tmp;          // dense view of cmol for sigmo_get_candidates
   int last_mode = 0;
@@ -1064,6 +1066,22 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     if (w + 2 >= (1ull << 32)) lane_ok = false;
   }
   const size_t o_ao = L.take(4 * aoff.size());
+  // molecule-padded candidate windows (filter output, join input): per
+  // molecule NDR windows of one 32-bit word (<= 32 nodes) or two (64-bit,
+  // even unit offset); molecule g starts at word NDR * cu[g]
+  std::vector<uint32_t> cu((size_t)hd.G + 1, 0);
+  {
+    uint64_t u = 0;
+    for (int64_t g = 0; g < hd.G; g++) {
+      const int64_t n = hd.goff[g + 1] - hd.goff[g];
+      if (n > 32) u = (u + 1) & ~1ull;
+      cu[g] = (uint32_t)std::min<uint64_t>(u, 0xffffffffull);
+      u += n > 32 ? 2 : 1;
+    }
+    cu[hd.G] = (uint32_t)std::min<uint64_t>(u, 0xffffffffull);
+    if ((unsigned long long)std::max<int64_t>(hq.V, 1) * (u + 2) >= (1ull << 32)) lane_ok = false;
+  }
+  const size_t o_cu = L.take(4 * cu.size());
   const size_t total = L.off;
   const auto t3 = std::chrono::steady_clock::now();
   // wait until the previous upload no longer reads the staging buffer
@@ -1115,6 +1133,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   memcpy(hb + o_tg1, tg1.data(), 4 * tg1.size());
   memcpy(hb + o_mt, mt.data(), 4 * mt.size());
   memcpy(hb + o_ao, aoff.data(), 4 * aoff.size());
+  memcpy(hb + o_cu, cu.data(), 4 * cu.size());
 
   const auto t4 = std::chrono::steady_clock::now();
   // ---- device arena + one H2D copy ----
@@ -1133,6 +1152,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->mol_tiles = (int32_t *)(db + o_mt);
   c->adj_off = (uint32_t *)(db + o_ao);
   c->adj_words = aoff[hd.G];
+  c->cand_units = (uint32_t *)(db + o_cu);
+  c->cand_total = cu[hd.G];
   c->n_mol_tiles = (int)mt.size() - 1;
   c->tile_g1 = (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
@@ -1191,7 +1212,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   // ---- per-batch device buffers ----
   // (+64 B: the join reads up to two words past a molecule window)
   size_t bm_bytes = 4 * (size_t)std::max(c->VQ, 1) * c->Wpad + 64;
-  if (lane_ok) bm_bytes = std::max(bm_bytes, 8 * (size_t)std::max(c->VQ, 1) * std::max(c->ND, 1));  // cmol layout
+  if (lane_ok) bm_bytes = std::max(bm_bytes, 4 * (size_t)std::max(c->VQ, 1) * (c->cand_total + 2));  // cmol layout
   SIGMO_TRY(dreserve(c, c->bitmap, bm_bytes, "candidate bitmap"));
   c->dense_pad_zero = false;  // zeroed before the first dense-tile filter (sigmo_filter)
   c->bm_bytes = bm_bytes;
@@ -1334,7 +1355,8 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     fp.MOLCAP = mol ? 32 : c->tile_molcap[k];
     fp.tile_g0 = (!mol && tws[k] == 32) ? c->tile_g0 : nullptr;
     fp.tile_g1 = (!mol && tws[k] == 32) ? c->tile_g1 : nullptr;
-    fp.cmol = mol ? (unsigned long long *)c->bitmap.p : nullptr;
+    fp.cmol = mol ? (uint32_t *)c->bitmap.p : nullptr;
+    fp.cand_units = c->cand_units;
     fp.qdrow = prog->qdrow;
     fp.qw_off = prog->qw_off;
     fp.qw = prog->qw;
@@ -1419,6 +1441,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     pp.off = (const I64x2 *)c->off.p;
     pp.goff = c->dd.goff;
     pp.adj_off = c->adj_off;
+    pp.cand_units = c->cand_units;
     pp.qgoff = c->dq.goff;
     pp.qp_row = c->qp_row;
     pp.bitmap = (const uint32_t *)c->bitmap.p;
@@ -1482,7 +1505,7 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       jp.adj_ones = c->adj_words;
       jp.qp_ent = c->qp_ent;
       jp.qp_ent2 = (const uint2 *)c->ent2.p;
-      jp.cmol = (const unsigned long long *)c->bitmap.p;
+      jp.cmol = (const uint32_t *)c->bitmap.p;
       // refill batch (lanes that must be free before a warp refills): swept on
       // configs[2], FA 2/4/8/16 -> 11.2/10.3/9.7/9.9 ms, FF 10.4/9.8/9.2/9.0 ms
       jp.batchK = mode == SIGMO_FIND_FIRST ? 16 : 8;
@@ -1607,8 +1630,8 @@ sigmo_status sigmo_get_candidates(sigmo_ctx *c, uint32_t *out) {
     SIGMO_TRY(dreserve(c, c->dense_tmp, bytes, "dense candidate view"));
     CUDA_TRY(c, cudaMemsetAsync(c->dense_tmp.p, 0, bytes, c->stream));
     const QueryProg &pg = c->progs[c->levels - 1].prog;  // the program of the last filter
-    CUDA_TRY(c, launch_unpad((const unsigned long long *)c->bitmap.p, pg.qdrow, pg.meta.NDR, c->dd.goff, c->ND, c->VQ,
-                             c->Wpad, (uint32_t *)c->dense_tmp.p, c->stream));
+    CUDA_TRY(c, launch_unpad((const uint32_t *)c->bitmap.p, c->cand_units, pg.qdrow, pg.meta.NDR, c->dd.goff, c->ND,
+                             c->VQ, c->Wpad, (uint32_t *)c->dense_tmp.p, c->stream));
     src = c->dense_tmp.p;
   }
   CUDA_TRY(c, cudaMemcpy2DAsync(out, 4 * (size_t)c->W, src, 4 * (size_t)c->Wpad, 4 * (size_t)c->W,

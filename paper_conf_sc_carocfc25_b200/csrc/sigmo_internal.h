@@ -102,7 +102,9 @@ struct FilterParams {
   const uint32_t *rowp;
   const int32_t *qgoff;        // [NQ+1] query node offsets (rows)
   uint32_t *bitmap;            // [VQ][Wpad] (dense tiles)
-  unsigned long long *cmol;    // [ND][NDR] molecule-padded windows of the distinct rows (molecule tiles), else null
+  uint32_t *cmol;              // molecule-padded windows of the distinct rows (molecule tiles), else null: molecule g
+                               // at word NDR * cand_units[g], NDR u32 windows (<= 32 nodes) or u64 (> 32 nodes)
+  const uint32_t *cand_units;
   const uint16_t *qdrow;       // [VQ] distinct row of each query node (molecule tiles)
   const int32_t *qw_off;       // [NQ+1] GMCR (word, bits) lists per query (molecule tiles)
   const uint32_t *qw;
@@ -147,7 +149,7 @@ struct JoinParams {
   // per-lane DFS kernel (k_join_lane)
   int VD;                      // data nodes
   const int4 *prec;            // [P] pair records {graph start node, query, graph * VQ + first query node, qinfo[query]}
-  const unsigned long long *cmol;  // [ND][VQ] molecule-padded candidate windows (filter output)
+  const uint32_t *cmol;        // molecule-padded candidate windows (filter output, see FilterParams::cmol)
   const uint32_t *adjw;        // bond-class adjacency masks (molecule-local bits), per molecule at word adj_off[g]:
                                // class-major [NB][n], u32 masks (n <= 32) or u64 (n > 32); all ones at word adj_ones
   unsigned adj_ones;
@@ -162,6 +164,7 @@ struct PairsParams {
   int ND, NQ, NQW, MQ, Wpad, VQ;
   int rowstride;               // cmol row stride per graph (distinct rows)
   const uint32_t *adj_off;     // [ND+1] adjacency word offset per graph (pair record .x)
+  const uint32_t *cand_units;  // [ND+1] candidate-window units per graph (pair record .z = rowstride * units)
   const uint32_t *gm;
   const I64x2 *off;
   const int32_t *goff, *qgoff, *qp_row;
@@ -206,7 +209,7 @@ cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *
 cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
-cudaError_t launch_unpad(const unsigned long long *cmol, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
+cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
                          int VQ, int Wpad, uint32_t *dense,
                          cudaStream_t st);
 cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,

@@ -587,6 +587,7 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
   uint32_t *s_tab = (uint32_t *)(smem + L.tab);
   uint8_t *s_bdone = smem + L.bdone;
   __shared__ int s_g0, s_g1, s_strad;
+  __shared__ unsigned s_cwb[33];  // molecule tiles: cmol word base of each molecule (bit 31: 64-bit windows)
   __shared__ int s_rrec[kMaxRadius + 1];
   __shared__ int s_rcarry[kMaxRadius];
   __shared__ uint8_t s_fused[kNumFields];
@@ -662,6 +663,10 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
   for (int i = tid; i <= nmol; i += NT) {
     const int st = __ldg(&goff[g0 + i]) - gs;
     s_mstart[i] = st;
+    if (MOL && i < nmol) {
+      const int n = __ldg(&goff[g0 + i + 1]) - gs - st;
+      s_cwb[i] = ((unsigned)fp.NDR * __ldg(&fp.cand_units[g0 + i])) | (n > 32 ? 0x80000000u : 0u);
+    }
     if (i < nmol) {
       const int n = __ldg(&goff[g0 + i + 1]) - gs - st;
       const int tb = gs + st - n0;  // tile bit of the molecule's first node
@@ -891,7 +896,13 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
 #pragma unroll
       for (int k = 0; k < 4; k++) {  // lane = (molecule, row): 8 molecules x 4 rows per store
         const int e = k * 32 + lane, m = e >> 2, r = e & 3;
-        if (m < nmol && r < nr) fp.cmol[(size_t)(g0 + m) * fp.NDR + rb + r] = stg[r * 33 + m];
+        if (m < nmol && r < nr) {
+          const unsigned b = s_cwb[m];
+          if (b & 0x80000000u)
+            *(unsigned long long *)(fp.cmol + (b & 0x7fffffffu) + 2u * (unsigned)(rb + r)) = stg[r * 33 + m];
+          else
+            fp.cmol[b + (unsigned)(rb + r)] = (uint32_t)stg[r * 33 + m];
+        }
       }
       __syncwarp();
       }
@@ -1839,6 +1850,7 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
   long long o = pp.off[g].a;
   const int a = __ldg(&pp.goff[g]);
   const int aw = pp.prec ? (int)__ldg(&pp.adj_off[g]) : 0;  // adjacency word offset (pair record .x)
+  const int cw = pp.prec ? (int)((unsigned)pp.rowstride * __ldg(&pp.cand_units[g])) : 0;  // cmol word base (.z)
   for (int qb = 0; qb < pp.NQW; qb++) {
     const uint32_t bits = __ldg(&pp.gm[(size_t)g * pp.NQW + qb]);
     if ((bits >> lane) & 1u) {
@@ -1848,7 +1860,7 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
       if (pp.prec) {
         // query info with the molecule size in bits 8-15 (class stride of adjb)
         const uint32_t qi = (__ldg(&pp.qinfo[q]) & ~0xff00u) | ((uint32_t)(__ldg(&pp.goff[g + 1]) - a) << 8);
-        pp.prec[p] = make_int4(aw, q, (int)((unsigned)g * (unsigned)pp.rowstride), (int)qi);
+        pp.prec[p] = make_int4(aw, q, cw, (int)qi);
       }
     }
     o += __popc(bits);
@@ -1864,14 +1876,16 @@ cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st) {
 
 // Dense (row-major, LSB-first) view of the molecule-padded candidates for
 // sigmo_get_candidates: thread per (row, graph), OR the window into the rows.
-__global__ void k_unpad(const unsigned long long *cmol, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
-                        int VQ, int Wpad, uint32_t *dense) {
+__global__ void k_unpad(const uint32_t *cmol, const uint32_t *cand_units, const uint16_t *qdrow, int NDR,
+                        const int32_t *goff, int ND, int VQ, int Wpad, uint32_t *dense) {
   const long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (t >= (long long)ND * VQ) return;
   const int g = (int)(t / VQ), row = (int)(t - (long long)g * VQ);
-  const unsigned long long w = cmol[(size_t)g * NDR + qdrow[row]];  // cmol[g][distinct row of query node row]
-  if (!w) return;
   const int a = goff[g];
+  const size_t base = (size_t)NDR * cand_units[g];  // window of the distinct row of query node `row`
+  const unsigned long long w = goff[g + 1] - a > 32 ? *(const unsigned long long *)(cmol + base + 2 * (size_t)qdrow[row])
+                                                    : (unsigned long long)cmol[base + qdrow[row]];
+  if (!w) return;
   uint32_t *r = dense + (size_t)row * Wpad;
   const int wi = a >> 5, sh = a & 31;
   const unsigned long long lo = w << sh;
@@ -1880,11 +1894,11 @@ __global__ void k_unpad(const unsigned long long *cmol, const uint16_t *qdrow, i
   if (sh && (uint32_t)(w >> (64 - sh))) atomicOr(&r[wi + 2], (uint32_t)(w >> (64 - sh)));
 }
 
-cudaError_t launch_unpad(const unsigned long long *cmol, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
-                         int VQ, int Wpad, uint32_t *dense, cudaStream_t st) {
+cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const uint16_t *qdrow, int NDR,
+                         const int32_t *goff, int ND, int VQ, int Wpad, uint32_t *dense, cudaStream_t st) {
   const long long n = (long long)ND * VQ;
   if (n <= 0) return cudaSuccess;
-  k_unpad<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(cmol, qdrow, NDR, goff, ND, VQ, Wpad, dense);
+  k_unpad<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(cmol, cand_units, qdrow, NDR, goff, ND, VQ, Wpad, dense);
   return cudaGetLastError();
 }
 
@@ -2015,7 +2029,11 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   auto adj = [&](bool wide, unsigned i) -> unsigned long long {
     return wide ? __ldg((const unsigned long long *)(adjw + i)) : (unsigned long long)__ldg(adjw + i);
   };
-  const unsigned long long *const cmol = jp.cmol;
+  const uint32_t *const cmol = jp.cmol;
+  // candidate window of distinct row r of the pair's molecule (cmol word base cb)
+  auto cand = [&](bool wide, unsigned cb, unsigned r) -> unsigned long long {
+    return wide ? __ldg((const unsigned long long *)(cmol + cb + 2u * r)) : (unsigned long long)__ldg(cmol + cb + r);
+  };
   const unsigned ones = jp.adj_ones;  // the all-ones entry (absent back-edge)
   const int4 zero4 = make_int4(0, 0, 0, 0);
 
@@ -2074,7 +2092,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const unsigned sw = wide ? 1u : 0u;  // word shift of an entry
       const unsigned i0 = j0 == 15u ? ones : ca + ((((en.y >> 16) & 7u) * ng + u0) << sw);
       const unsigned i1 = j1 == 15u ? ones : ca + ((((en.y >> 19) & 7u) * ng + u1) << sw);
-      unsigned long long X = __ldg(&cmol[cmb + ((unsigned)en.x >> 12)]) & ~used & adj(wide, i0) & adj(wide, i1);
+      unsigned long long X = cand(wide, cmb, (unsigned)en.x >> 12) & ~used & adj(wide, i0) & adj(wide, i1);
       if (en.x & 0xf00) {  // > 2 back-edges at this depth (fused rings): rare
         const int nex = (en.x >> 8) & 15;
         for (int k = 0; k < nex; k++) {
@@ -2151,7 +2169,8 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         np = cbase + (unsigned)src;
         nv = true;
         // root candidates of the next pair: the load completes while the current pair runs
-        nR0 = __ldg(&cmol[(unsigned)r.z + ((unsigned)__ldg(&qp_ent[(unsigned)r.w >> 16]).x >> 12)]);
+        nR0 = cand((((unsigned)r.w >> 8) & 0xffu) > 32u, (unsigned)r.z,
+                   (unsigned)__ldg(&qp_ent[(unsigned)r.w >> 16]).x >> 12);
       }
       chead += take;
       wm = __ballot_sync(FULL_MASK, !nv) & wm;
