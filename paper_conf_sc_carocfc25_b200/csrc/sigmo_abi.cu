@@ -1575,8 +1575,13 @@ sigmo_status sigmo_get_pair_results(sigmo_ctx *c, int64_t cap, int64_t *n, int64
   *n = P;
   if (cap < P) return set_err(c, SIGMO_ERR_INVALID_ARG, "capacity %lld < %lld pairs", (long long)cap, (long long)P);
   if (P == 0) return SIGMO_OK;
-  if (query_idx)
-    CUDA_TRY(c, cudaMemcpyAsync(query_idx, c->pair_query.p, 4 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
+  if (query_idx) {
+    if (c->mol_filter)  // lane-join path: the query is field .y of the int4 pair records
+      CUDA_TRY(c, cudaMemcpy2DAsync(query_idx, 4, (const char *)c->pair_rec.p + 4, 16, 4, (size_t)P,
+                                    cudaMemcpyDeviceToHost, c->stream));
+    else
+      CUDA_TRY(c, cudaMemcpyAsync(query_idx, c->pair_query.p, 4 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
+  }
   if (result)
     CUDA_TRY(c, cudaMemcpyAsync(result, c->pair_result.p, 8 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
   std::vector<I64x2> off;

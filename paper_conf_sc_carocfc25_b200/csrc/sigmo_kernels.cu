@@ -1849,6 +1849,7 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
   const unsigned lt = (1u << lane) - 1u;
   long long o = pp.off[g].a;
   const int a = __ldg(&pp.goff[g]);
+  const uint32_t ng8 = (uint32_t)(__ldg(&pp.goff[g + 1]) - a) << 8;  // molecule size, bits 8-15 of the query info
   const int aw = pp.prec ? (int)__ldg(&pp.adj_off[g]) : 0;  // adjacency word offset (pair record .x)
   const int cw = pp.prec ? (int)((unsigned)pp.rowstride * __ldg(&pp.cand_units[g])) : 0;  // cmol word base (.z)
   for (int qb = 0; qb < pp.NQW; qb++) {
@@ -1856,10 +1857,10 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
     if ((bits >> lane) & 1u) {
       const int q = qb * 32 + lane;
       const long long p = o + __popc(bits & lt);
-      pp.pair_query[p] = q;
-      if (pp.prec) {
-        // query info with the molecule size in bits 8-15 (class stride of adjb)
-        const uint32_t qi = (__ldg(&pp.qinfo[q]) & ~0xff00u) | ((uint32_t)(__ldg(&pp.goff[g + 1]) - a) << 8);
+      if (!pp.prec) {
+        pp.pair_query[p] = q;
+      } else {  // the lane join reads the records only (queries from .y)
+        const uint32_t qi = (__ldg(&pp.qinfo[q]) & ~0xff00u) | ng8;
         pp.prec[p] = make_int4(aw, q, cw, (int)qi);
       }
     }
