@@ -1507,8 +1507,9 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       jp.qp_ent2 = (const uint2 *)c->ent2.p;
       jp.cmol = (const uint32_t *)c->bitmap.p;
       // refill batch (lanes that must be free before a warp refills): swept on
-      // configs[2], FA 2/4/8/16 -> 11.2/10.3/9.7/9.9 ms, FF 10.4/9.8/9.2/9.0 ms
-      jp.batchK = mode == SIGMO_FIND_FIRST ? 16 : 8;
+      // configs[2] (r1 final kernel), FA 6/8/12/16 -> 8.70/8.61/8.81/9.42 ms,
+      // FF 7.43/7.27/7.18/7.29 ms
+      jp.batchK = mode == SIGMO_FIND_FIRST ? 12 : 8;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
       const size_t smem = join_lane_smem_bytes(jp);
       if (smem > c->max_smem) return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
