@@ -1240,7 +1240,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, c->adj_off, (uint32_t *)c->adjb.p, c->stream));
   }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
-  SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 6), "join counters"));
+  SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 8), "join counters"));  // + the second claim counter
   if (getenv("SIGMO_DEBUG_LOAD")) {
     const auto t5 = std::chrono::steady_clock::now();
     auto ms = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
@@ -1465,7 +1465,7 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
   if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_join before sigmo_filter");
   if (mode != SIGMO_FIND_ALL && mode != SIGMO_FIND_FIRST) return set_err(c, SIGMO_ERR_INVALID_ARG, "bad mode %d", (int)mode);
   CUDA_TRY(c, cudaSetDevice(c->device));
-  CUDA_TRY(c, cudaMemsetAsync(c->jcnt.p, 0, 8 * ((size_t)c->NQ + 6), c->stream));
+  CUDA_TRY(c, cudaMemsetAsync(c->jcnt.p, 0, 8 * ((size_t)c->NQ + 8), c->stream));
   int launches = 0;
   if (c->ND > 0 && c->VD > 0 && c->NQ > 0) {
     JoinParams jp{};
@@ -1511,15 +1511,23 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       // FF 7.43/7.27/7.18/7.29 ms
       jp.batchK = mode == SIGMO_FIND_FIRST ? 12 : 8;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
-      const size_t smem = join_lane_smem_bytes(jp);
-      if (smem > c->max_smem) return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
-      jp.smem_bytes = smem;
-      int bps = join_lane_blocks_per_sm((int)mode, jp, smem);
-      if (const char *e = getenv("SIGMO_JOIN_BPS")) bps = std::max(1, std::min(bps, atoi(e)));
-      const int grid = bps * c->sm_count;
+      // two launches: pairs of <= 32-node molecules with 32-bit masks, then
+      // the others with 64-bit masks (each finds its range in off[ND])
       timing_join(c, 0);
-      CUDA_TRY(c, launch_join_lane((int)mode, jp, grid, c->stream));
-      launches++;
+      for (int w = 0; w < 2; w++) {
+        const bool w64 = w == 1;
+        if (w64 && c->maxn <= 32) break;
+        const size_t smem = join_lane_smem_bytes(jp, w64);
+        if (smem > c->max_smem)
+          return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
+        jp.smem_bytes = smem;
+        jp.chunk_counter = (int *)((unsigned long long *)c->jcnt.p + (w64 ? 6 + (size_t)c->NQ : 0));
+        int bps = join_lane_blocks_per_sm((int)mode, w64, jp, smem);
+        if (const char *e = getenv("SIGMO_JOIN_BPS")) bps = std::max(1, std::min(bps, atoi(e)));
+        const int grid = bps * c->sm_count;
+        CUDA_TRY(c, launch_join_lane((int)mode, w64, jp, grid, c->stream));
+        launches++;
+      }
       timing_join(c, 1);
     } else {
       const size_t smem = join_smem_bytes(c->NW, jp);
@@ -1562,7 +1570,7 @@ sigmo_status sigmo_num_pairs(sigmo_ctx *c, int64_t *n) {
   I64x2 t;
   CUDA_TRY(c, cudaMemcpyAsync(&t, (I64x2 *)c->off.p + c->ND, sizeof(I64x2), cudaMemcpyDeviceToHost, c->stream));
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-  *n = t.a;
+  *n = t.a + t.b;  // .b: pairs of > 32-node molecules on the lane-join path (else 0)
   return SIGMO_OK;
 }
 
@@ -1576,24 +1584,44 @@ sigmo_status sigmo_get_pair_results(sigmo_ctx *c, int64_t cap, int64_t *n, int64
   *n = P;
   if (cap < P) return set_err(c, SIGMO_ERR_INVALID_ARG, "capacity %lld < %lld pairs", (long long)cap, (long long)P);
   if (P == 0) return SIGMO_OK;
-  if (query_idx) {
-    if (c->mol_filter)  // lane-join path: the query is field .y of the int4 pair records
-      CUDA_TRY(c, cudaMemcpy2DAsync(query_idx, 4, (const char *)c->pair_rec.p + 4, 16, 4, (size_t)P,
-                                    cudaMemcpyDeviceToHost, c->stream));
-    else
+  std::vector<I64x2> off((size_t)c->ND + 1);
+  CUDA_TRY(c, cudaMemcpyAsync(off.data(), c->off.p, sizeof(I64x2) * off.size(), cudaMemcpyDeviceToHost, c->stream));
+  if (!c->mol_filter) {
+    if (query_idx)
       CUDA_TRY(c, cudaMemcpyAsync(query_idx, c->pair_query.p, 4 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
+    if (result)
+      CUDA_TRY(c, cudaMemcpyAsync(result, c->pair_result.p, 8 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    if (data_idx)
+      for (int g = 0; g < c->ND; g++)
+        for (long long p = off[g].a; p < off[g + 1].a; p++) data_idx[p] = g;
+    return SIGMO_OK;
   }
-  if (result)
-    CUDA_TRY(c, cudaMemcpyAsync(result, c->pair_result.p, 8 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
-  std::vector<I64x2> off;
-  if (data_idx) {
-    off.resize((size_t)c->ND + 1);
-    CUDA_TRY(c, cudaMemcpyAsync(off.data(), c->off.p, sizeof(I64x2) * off.size(), cudaMemcpyDeviceToHost, c->stream));
-  }
+  // lane-join path: records of <= 32-node molecules first, then the others;
+  // the query is field .y of the int4 records.  Merge back to graph order.
+  std::vector<int32_t> q((size_t)P);
+  std::vector<uint64_t> r((size_t)P);
+  CUDA_TRY(c, cudaMemcpy2DAsync(q.data(), 4, (const char *)c->pair_rec.p + 4, 16, 4, (size_t)P, cudaMemcpyDeviceToHost,
+                                c->stream));
+  CUDA_TRY(c, cudaMemcpyAsync(r.data(), c->pair_result.p, 8 * (size_t)P, cudaMemcpyDeviceToHost, c->stream));
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
-  if (data_idx)
-    for (int g = 0; g < c->ND; g++)
-      for (long long p = off[g].a; p < off[g + 1].a; p++) data_idx[p] = g;
+  const long long Pn = off[c->ND].a;
+  long long o = 0;
+  for (int g = 0; g < c->ND; g++) {
+    long long s0, s1;
+    if (off[g + 1].a > off[g].a) {
+      s0 = off[g].a;
+      s1 = off[g + 1].a;
+    } else {
+      s0 = Pn + off[g].b;
+      s1 = Pn + off[g + 1].b;
+    }
+    for (long long p = s0; p < s1; p++, o++) {
+      if (data_idx) data_idx[o] = g;
+      if (query_idx) query_idx[o] = q[(size_t)p];
+      if (result) result[o] = r[(size_t)p];
+    }
+  }
   return SIGMO_OK;
 }
 

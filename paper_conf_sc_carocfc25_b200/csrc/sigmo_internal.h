@@ -148,7 +148,7 @@ struct JoinParams {
   size_t smem_bytes;
   // per-lane DFS kernel (k_join_lane)
   int VD;                      // data nodes
-  const int4 *prec;            // [P] pair records {graph start node, query, graph * VQ + first query node, qinfo[query]}
+  const int4 *prec;            // [P] pair records {adjacency word offset, query, cmol word base, qinfo | size << 8}
   const uint32_t *cmol;        // molecule-padded candidate windows (filter output, see FilterParams::cmol)
   const uint32_t *adjw;        // bond-class adjacency masks (molecule-local bits), per molecule at word adj_off[g]:
                                // class-major [NB][n], u32 masks (n <= 32) or u64 (n > 32); all ones at word adj_ones
@@ -214,9 +214,9 @@ cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const
                          cudaStream_t st);
 cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
                         cudaStream_t st);
-cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream_t st);
-size_t join_lane_smem_bytes(const JoinParams &p);
-int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem);
+cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, cudaStream_t st);
+size_t join_lane_smem_bytes(const JoinParams &p, bool w64);
+int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem);
 constexpr int kJoinLaneThreads = 128;
 constexpr int kJoinLaneMaxQ = 11;  // k_join_lane handles queries <= 11 nodes in <= 64-node graphs (map: 6 bits x 10 depths)
 size_t join_smem_bytes(int NW, const JoinParams &p);

@@ -1081,8 +1081,11 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
       np += __popc(bits);
     }
     I64x2 v;
-    v.a = np;
-    v.b = 0;
+    // molecule tiles: pairs of <= 32-node molecules counted in .a, of larger
+    // ones in .b (the lane join runs the two classes as separate launches)
+    const bool wide = MOL && s_mstart[mi + 1] - s_mstart[mi] > 32;
+    v.a = wide ? 0 : np;
+    v.b = wide ? np : 0;
     fp.mol_cnt[g] = v;
   }
 }
@@ -1847,7 +1850,10 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
   const int g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (g >= pp.ND) return;
   const unsigned lt = (1u << lane) - 1u;
+  // lane join: records of <= 32-node molecules first (off.a), then the others
+  // at P_narrow + off.b; the general path only uses .a
   long long o = pp.off[g].a;
+  if (pp.prec && pp.off[g + 1].b > pp.off[g].b) o = pp.off[pp.ND].a + pp.off[g].b;
   const int a = __ldg(&pp.goff[g]);
   const uint32_t ng8 = (uint32_t)(__ldg(&pp.goff[g + 1]) - a) << 8;  // molecule size, bits 8-15 of the query info
   const int aw = pp.prec ? (int)__ldg(&pp.adj_off[g]) : 0;  // adjacency word offset (pair record .x)
@@ -1973,17 +1979,18 @@ cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const
 // ===========================================================================
 constexpr int kJoinChunk = 32;  // GMCR pairs per warp claim (one record per lane)
 
-__host__ __device__ inline size_t join_lane_warp_bytes(int MQ) {
+// stack entry {R, U}: 2 x 32-bit masks (<= 32-node molecules) or 2 x 64-bit
+__host__ __device__ inline size_t join_lane_warp_bytes(int MQ, bool w64) {
   const int SD = MQ > 1 ? MQ - 1 : 1;  // pushed depths 0..n-2
-  // {R, U} [SD][32] 16 B | map [16][32] B
-  return 512 * (size_t)SD + 512;
+  // {R, U} [SD][32] (8 or 16 B) | map [16][32] B
+  return 32 * (size_t)(w64 ? 16 : 8) * SD + 512;
 }
 // CTA: per-query totals [NQ] u64, then one region per warp
 __host__ __device__ inline size_t join_lane_cta_bytes(int NQ) { return align16(8 * (size_t)(NQ > 0 ? NQ : 1)); }
-__host__ __device__ inline size_t join_lane_smem(int NQ, int MQ) {
-  return join_lane_cta_bytes(NQ) + join_lane_warp_bytes(MQ) * (kJoinLaneThreads / 32);
+__host__ __device__ inline size_t join_lane_smem(int NQ, int MQ, bool w64) {
+  return join_lane_cta_bytes(NQ) + join_lane_warp_bytes(MQ, w64) * (kJoinLaneThreads / 32);
 }
-size_t join_lane_smem_bytes(const JoinParams &p) { return join_lane_smem(p.NQ, p.maxq); }
+size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_smem(p.NQ, p.maxq, w64); }
 
 __device__ __forceinline__ void cp_async8(unsigned dst_smem, const void *src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(dst_smem), "l"(src) : "memory");
@@ -1997,8 +2004,12 @@ __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
   return __ffs(m) - 1;
 }
 
-template <int MODE>
+// W64: the launch's pairs are on > 32-node molecules (64-bit masks); else all
+// masks, stack entries and loads are 32-bit
+template <int MODE, bool W64>
 __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_constant__ JoinParams jp) {
+  using MT = typename std::conditional<W64, unsigned long long, unsigned>::type;
+  constexpr unsigned ES = W64 ? 16u : 8u;  // stack entry bytes
   extern __shared__ __align__(16) unsigned char smem[];
 #define LDS64(o) (*(const unsigned long long *)(smem + (o)))
 #define STS64(o) (*(unsigned long long *)(smem + (o)))
@@ -2016,24 +2027,54 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   // candidates per step, 9.60 vs 9.49 ms, and caching the top stack entry in
   // registers, 8.92 vs 8.80 ms)
   const uint2 *const qp_ent = jp.qp_ent2;  // 8-B entries: more lanes share a sector
-  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ) + (size_t)wid * join_lane_warp_bytes(MQ));
-  const unsigned oRU = wbase + 16u * lane;                        // {R, U} of depth d: oRU + 512 d
-  const unsigned oM = wbase + 512u * SD + lane;                   // f(pi_d): oM + 32 d
+  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
+  const unsigned oRU = wbase + ES * lane;                         // {R, U} of depth d: oRU + 32 ES d
+  const unsigned oM = wbase + 32u * ES * SD + lane;               // f(pi_d): oM + 32 d
+  auto ldRU = [&](unsigned o, MT &r, MT &u) {
+    if (W64) {
+      const ulonglong2 x = *(const ulonglong2 *)(smem + o);
+      r = (MT)x.x;
+      u = (MT)x.y;
+    } else {
+      const uint2 x = *(const uint2 *)(smem + o);
+      r = (MT)x.x;
+      u = (MT)x.y;
+    }
+  };
+  auto stRU = [&](unsigned o, MT r, MT u) {
+    if (W64) *(ulonglong2 *)(smem + o) = make_ulonglong2((unsigned long long)r, (unsigned long long)u);
+    else *(uint2 *)(smem + o) = make_uint2((unsigned)r, (unsigned)u);
+  };
+  auto popc = [](MT x) -> int { return W64 ? __popcll((unsigned long long)x) : __popc((unsigned)x); };
+  auto lowest = [](MT x) -> int {  // index of the lowest set bit (x != 0)
+    if (W64) {
+      const unsigned lo = (unsigned)x, hi = (unsigned)((unsigned long long)x >> 32);
+      return lo ? __ffs(lo) - 1 : 31 + __ffs(hi);
+    }
+    return __ffs((unsigned)x) - 1;
+  };
   smem[oM + 32 * 15] = 0;  // map slot 15 (absent back-edge) reads node 0 of the all-ones class
   __syncthreads();
 
   const unsigned lt = (1u << lane) - 1u;
-  const unsigned P = (unsigned)jp.off[jp.ND].a;
+  // this launch's pairs: records / results [pair_base, pair_base + pair_count)
+  const I64x2 ptot = jp.off[jp.ND];  // (pairs of <= 32-node molecules, pairs of larger ones)
+  const unsigned P = (unsigned)(W64 ? ptot.b : ptot.a);
+  const long long pbase0 = W64 ? ptot.a : 0;
+  const int4 *const recs = jp.prec + pbase0;
+  unsigned long long *const presult = jp.pair_result + pbase0;
   unsigned *const cursor = (unsigned *)jp.chunk_counter;
   const uint32_t *const adjw = jp.adjw;
-  // mask of adjacency word index i: 32-bit for <= 32-node molecules, else 64-bit
-  auto adj = [&](bool wide, unsigned i) -> unsigned long long {
-    return wide ? __ldg((const unsigned long long *)(adjw + i)) : (unsigned long long)__ldg(adjw + i);
+  // mask of adjacency word index i (entries of 1 or 2 words)
+  auto adj = [&](unsigned i) -> MT {
+    if (W64) return (MT)__ldg((const unsigned long long *)(adjw + i));
+    return (MT)__ldg(adjw + i);
   };
   const uint32_t *const cmol = jp.cmol;
   // candidate window of distinct row r of the pair's molecule (cmol word base cb)
-  auto cand = [&](bool wide, unsigned cb, unsigned r) -> unsigned long long {
-    return wide ? __ldg((const unsigned long long *)(cmol + cb + 2u * r)) : (unsigned long long)__ldg(cmol + cb + r);
+  auto cand = [&](unsigned cb, unsigned r) -> MT {
+    if (W64) return (MT)__ldg((const unsigned long long *)(cmol + cb + 2u * r));
+    return (MT)__ldg(cmol + cb + r);
   };
   const unsigned ones = jp.adj_ones;  // the all-ones entry (absent back-edge)
   const int4 zero4 = make_int4(0, 0, 0, 0);
@@ -2048,8 +2089,8 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     pbase = x + kJoinChunk;
     nbase = x + 2u * kJoinChunk;
   }
-  int4 crec = cbase + lane < P ? __ldg(&jp.prec[cbase + lane]) : zero4;
-  int4 prec = pbase + lane < P ? __ldg(&jp.prec[pbase + lane]) : zero4;
+  int4 crec = cbase + lane < P ? __ldg(&recs[cbase + lane]) : zero4;
+  int4 prec = pbase + lane < P ? __ldg(&recs[pbase + lane]) : zero4;
   unsigned ccount = cbase < P ? min(P - cbase, (unsigned)kJoinChunk) : 0u, chead = 0u;
   bool drained = ccount == 0u;
 
@@ -2064,48 +2105,47 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   bool nv = false;  // next pair assigned (rows in flight into the other buffer)
   unsigned np = 0u;
   int4 nrec = zero4;
-  unsigned long long nR0 = 0ull;
+  MT nR0 = 0;
 
   while (true) {
     // ---- one DFS step ----
     if (ne) {
       const int d = 31 - __clz(ne);
       const int e = d + 1;
-      const unsigned od = oRU + 512u * d;
+      const unsigned od = oRU + 32u * ES * d;
       // the plan entry of depth e and the map bytes of its back-edge targets
       // depend on d only: loaded before v is known (j == d takes v below)
       const uint2 en = __ldg(&qp_ent[cqb + e]);
-      const ulonglong2 RU = LDS128(od);
+      MT R, U;
+      ldRU(od, R, U);
       const unsigned j0 = en.x & 15, j1 = (en.x >> 4) & 15;
       const unsigned m0 = smem[oM + 32u * j0], m1 = smem[oM + 32u * j1];
-      const unsigned lo = (unsigned)RU.x, hi = (unsigned)(RU.x >> 32);
-      const int v = lo ? __ffs(lo) - 1 : 31 + __ffs(hi);
-      const unsigned long long bit = 1ull << v;
-      const unsigned long long Rn = RU.x ^ bit;
-      STS64(od) = Rn;
+      const int v = lowest(R);
+      const MT bit = (MT)1 << v;
+      const MT Rn = R ^ bit;
+      *(MT *)(smem + od) = Rn;
       smem[oM + 32u * d] = (unsigned char)v;
       if (!Rn) ne ^= 1u << d;
-      const unsigned long long used = RU.y | bit;
+      const MT used = U | bit;
       // candidates of depth e
       const unsigned u0 = j0 == (unsigned)d ? (unsigned)v : m0, u1 = j1 == (unsigned)d ? (unsigned)v : m1;
       const unsigned ng = (cinfo >> 8) & 0xffu;  // molecule size: class stride of the adjacency
-      const bool wide = ng > 32u;
-      const unsigned sw = wide ? 1u : 0u;  // word shift of an entry
+      constexpr unsigned sw = W64 ? 1u : 0u;  // word shift of an entry
       const unsigned i0 = j0 == 15u ? ones : ca + ((((en.y >> 16) & 7u) * ng + u0) << sw);
       const unsigned i1 = j1 == 15u ? ones : ca + ((((en.y >> 19) & 7u) * ng + u1) << sw);
-      unsigned long long X = cand(wide, cmb, (unsigned)en.x >> 12) & ~used & adj(wide, i0) & adj(wide, i1);
+      MT X = cand(cmb, (unsigned)en.x >> 12) & ~used & adj(i0) & adj(i1);
       if (en.x & 0xf00) {  // > 2 back-edges at this depth (fused rings): rare
         const int nex = (en.x >> 8) & 15;
         for (int k = 0; k < nex; k++) {
           const int be = __ldg(&jp.qp_be[(en.y & 0xffffu) + k]);
-          X &= adj(wide, ca + (((unsigned)(be & 255) * ng + smem[oM + 32u * (be >> 8)]) << sw));
+          X &= adj(ca + (((unsigned)(be & 255) * ng + smem[oM + 32u * (be >> 8)]) << sw));
         }
       }
       if (e == (int)(cinfo & 0xff) - 1) {
-        cnt += (unsigned long long)__popcll(X);
+        cnt += (unsigned long long)popc(X);
         if (MODE == 1 && cnt) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
-        STS128(oRU + 512u * e) = make_ulonglong2(X, used);
+        stRU(oRU + 32u * ES * e, X, used);
         ne |= 1u << e;
       }
       pend = ne == 0u;
@@ -2118,14 +2158,14 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     if (pend) {
       if (MODE == 1) {
         if (!shared) {
-          jp.pair_result[cp] = cnt ? 1ull : 0ull;
+          presult[cp] = cnt ? 1ull : 0ull;
           if (cnt) atomicAdd((unsigned long long *)(smem + o_tot) + cq, 1ull);
         } else if (cnt) {
-          if (atomicOr(&jp.pair_result[cp], 1ull) == 0ull) atomicAdd((unsigned long long *)(smem + o_tot) + cq, 1ull);
+          if (atomicOr(&presult[cp], 1ull) == 0ull) atomicAdd((unsigned long long *)(smem + o_tot) + cq, 1ull);
         }
       } else {
-        if (!shared) jp.pair_result[cp] = cnt;
-        else if (cnt) atomicAdd(&jp.pair_result[cp], cnt);
+        if (!shared) presult[cp] = cnt;
+        else if (cnt) atomicAdd(&presult[cp], cnt);
         if (cnt) atomicAdd((unsigned long long *)(smem + o_tot) + cq, cnt);
       }
       pend = false;
@@ -2140,12 +2180,12 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       cqb = cinfo >> 16;
       shared = false;
       cnt = 0ull;
-      const unsigned long long R0 = nR0;
+      const MT R0 = nR0;
       if ((cinfo & 0xff) == 1u) {
-        cnt = (unsigned long long)__popcll(R0);
+        cnt = (unsigned long long)popc(R0);
         pend = true;
       } else {
-        STS128(oRU) = make_ulonglong2(R0, 0ull);
+        stRU(oRU, R0, (MT)0);
         ne = R0 ? 1u : 0u;
         pend = ne == 0u;
       }
@@ -2170,8 +2210,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         np = cbase + (unsigned)src;
         nv = true;
         // root candidates of the next pair: the load completes while the current pair runs
-        nR0 = cand((((unsigned)r.w >> 8) & 0xffu) > 32u, (unsigned)r.z,
-                   (unsigned)__ldg(&qp_ent[(unsigned)r.w >> 16]).x >> 12);
+        nR0 = cand((unsigned)r.z, (unsigned)__ldg(&qp_ent[(unsigned)r.w >> 16]).x >> 12);
       }
       chead += take;
       wm = __ballot_sync(FULL_MASK, !nv) & wm;
@@ -2185,7 +2224,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
           break;
         }
         pbase = nbase;
-        prec = pbase + lane < P ? __ldg(&jp.prec[pbase + lane]) : zero4;
+        prec = pbase + lane < P ? __ldg(&recs[pbase + lane]) : zero4;
         unsigned x = 0u;
         if (lane == 0) x = atomicAdd(cursor, (unsigned)kJoinChunk);
         nbase = __shfl_sync(FULL_MASK, x, 0);
@@ -2208,13 +2247,17 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         const unsigned s_ca = __shfl_sync(FULL_MASK, ca, src);
         const unsigned s_cmb = __shfl_sync(FULL_MASK, cmb, src);
         if (give && !shared) {
-          jp.pair_result[cp] = 0ull;  // the pair's result is accumulated from several lanes from now on
+          presult[cp] = 0ull;  // the pair's result is accumulated from several lanes from now on
           shared = true;
         }
         __syncwarp();
         if (recv) {
           const unsigned dl = (unsigned)(src - lane);  // donor offsets = mine + dl * (8 | 16 | 1)
-          STS128(oRU + 512u * ds) = LDS128(oRU + 512u * ds + 16u * dl);
+          {
+            MT r, u;
+            ldRU(oRU + 32u * ES * ds + ES * dl, r, u);
+            stRU(oRU + 32u * ES * ds, r, u);
+          }
           for (int j = 0; j < ds; j++) smem[oM + 32u * j] = smem[oM + 32u * j + dl];
           cmb = s_cmb;
           cp = s_cp;
@@ -2251,34 +2294,37 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
 #undef STS128
 }
 
-template <int MODE>
+template <int MODE, bool W64>
 static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_t st) {
-  cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE, W64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)p.smem_bytes);
   if (e != cudaSuccess) return e;
-  k_join_lane<MODE><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
+  k_join_lane<MODE, W64><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-cudaError_t launch_join_lane(int mode, const JoinParams &p, int grid, cudaStream_t st) {
+cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, cudaStream_t st) {
   if (grid <= 0) return cudaSuccess;
-  return mode == 1 ? launch_join_lane_t<1>(p, grid, st) : launch_join_lane_t<0>(p, grid, st);
+  if (w64) return mode == 1 ? launch_join_lane_t<1, true>(p, grid, st) : launch_join_lane_t<0, true>(p, grid, st);
+  return mode == 1 ? launch_join_lane_t<1, false>(p, grid, st) : launch_join_lane_t<0, false>(p, grid, st);
 }
 
-template <int MODE>
+template <int MODE, bool W64>
 static int join_lane_occ_t(size_t smem) {
   int n = 0;
-  cudaFuncSetAttribute(k_join_lane<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE>, kJoinLaneThreads, smem) != cudaSuccess) {
+  cudaFuncSetAttribute(k_join_lane<MODE, W64>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE, W64>, kJoinLaneThreads, smem) !=
+      cudaSuccess) {
     cudaGetLastError();
     return 1;
   }
   return n < 1 ? 1 : n;
 }
 
-int join_lane_blocks_per_sm(int mode, const JoinParams &p, size_t smem) {
+int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem) {
   (void)p;
-  return mode == 1 ? join_lane_occ_t<1>(smem) : join_lane_occ_t<0>(smem);
+  if (w64) return mode == 1 ? join_lane_occ_t<1, true>(smem) : join_lane_occ_t<0, true>(smem);
+  return mode == 1 ? join_lane_occ_t<1, false>(smem) : join_lane_occ_t<0, false>(smem);
 }
 
 }  // namespace sigmo
