@@ -106,6 +106,8 @@ struct sigmo_ctx {
   // ---- load ----
   Pinned staging;
   cudaEvent_t h2d_done = nullptr;
+  cudaStream_t aux = nullptr;                        // the wide-molecule join launch runs beside the narrow one
+  cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
   DBuf arena;
   DevGraphs dq, dd;
   int NQ = 0, VQ = 0, EQ = 0, NQW = 0, maxq = 0, NB = 0, NBE = 0, plan_smem = 0;
@@ -897,7 +899,10 @@ sigmo_status sigmo_create(int device, void *cuda_stream, const sigmo_allocator *
   int smem = 0;
   cudaDeviceGetAttribute(&smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
   if (smem > 0) c->max_smem = (size_t)smem;
-  if (cudaEventCreateWithFlags(&c->h2d_done, cudaEventDisableTiming) != cudaSuccess) {
+  if (cudaEventCreateWithFlags(&c->h2d_done, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->fork_ev, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->join_ev, cudaEventDisableTiming) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking) != cudaSuccess) {
     delete c;
     return SIGMO_ERR_CUDA;
   }
@@ -917,6 +922,12 @@ sigmo_status sigmo_destroy(sigmo_ctx *c) {
   cudaStreamSynchronize(c->stream);
   if (c->staging.p) cudaFreeHost(c->staging.p);
   if (c->h2d_done) cudaEventDestroy(c->h2d_done);
+  if (c->aux) {
+    cudaStreamSynchronize(c->aux);
+    cudaStreamDestroy(c->aux);
+  }
+  if (c->fork_ev) cudaEventDestroy(c->fork_ev);
+  if (c->join_ev) cudaEventDestroy(c->join_ev);
   for (int r = 0; r < Timing::RING; r++) {
     for (int k = 0; k < 5; k++) cudaEventDestroy(c->timing.fev[r][k]);
     for (int k = 0; k < 2; k++) cudaEventDestroy(c->timing.jev[r][k]);
@@ -1511,12 +1522,19 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       // FF 7.43/7.27/7.18/7.29 ms
       jp.batchK = mode == SIGMO_FIND_FIRST ? 12 : 8;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
-      // two launches: pairs of <= 32-node molecules with 32-bit masks, then
-      // the others with 64-bit masks (each finds its range in off[ND])
+      // two launches: pairs of <= 32-node molecules with 32-bit masks, and
+      // the others with 64-bit masks (each finds its range in off[ND]); the
+      // wide one on the auxiliary stream, so its CTAs fill the SMs the narrow
+      // launch frees at its tail
       timing_join(c, 0);
+      const bool two = c->maxn > 32;
+      if (two) {
+        CUDA_TRY(c, cudaEventRecord(c->fork_ev, c->stream));
+        CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->fork_ev, 0));
+      }
       for (int w = 0; w < 2; w++) {
         const bool w64 = w == 1;
-        if (w64 && c->maxn <= 32) break;
+        if (w64 && !two) break;
         const size_t smem = join_lane_smem_bytes(jp, w64);
         if (smem > c->max_smem)
           return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
@@ -1525,8 +1543,12 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
         int bps = join_lane_blocks_per_sm((int)mode, w64, jp, smem);
         if (const char *e = getenv("SIGMO_JOIN_BPS")) bps = std::max(1, std::min(bps, atoi(e)));
         const int grid = bps * c->sm_count;
-        CUDA_TRY(c, launch_join_lane((int)mode, w64, jp, grid, c->stream));
+        CUDA_TRY(c, launch_join_lane((int)mode, w64, jp, grid, w64 ? c->aux : c->stream));
         launches++;
+      }
+      if (two) {
+        CUDA_TRY(c, cudaEventRecord(c->join_ev, c->aux));
+        CUDA_TRY(c, cudaStreamWaitEvent(c->stream, c->join_ev, 0));
       }
       timing_join(c, 1);
     } else {
