@@ -10,7 +10,14 @@ from __future__ import annotations
 import itertools
 
 
-def brute_embeddings(qgraph, dgraph):
+def _induced_ok(f, qedges, bond, nq):
+    """Condition (3) of the induced reading (G_D[X]; R20):
+    non-adjacent query nodes map to non-adjacent data nodes."""
+    qadj = {(u, v) for (u, v, _) in qedges} | {(v, u) for (u, v, _) in qedges}
+    return all((f[u], f[v]) not in bond for u in range(nq) for v in range(nq) if u != v and (u, v) not in qadj)
+
+
+def brute_embeddings(qgraph, dgraph, induced: bool = False):
     """Yield every embedding f (tuple, f[i] = data node of query node i)."""
     qlab, qedges = qgraph
     dlab, dedges = dgraph
@@ -24,10 +31,12 @@ def brute_embeddings(qgraph, dgraph):
             continue
         if any(bond.get((f[u], f[v])) != b for (u, v, b) in qedges):  # condition (2) + bond labels
             continue
+        if induced and not _induced_ok(f, qedges, bond, nq):
+            continue
         yield f
 
 
-def brute_count(qgraph, dgraph) -> int:
+def brute_count(qgraph, dgraph, induced: bool = False) -> int:
     """qgraph/dgraph: (labels, [(u, v, bond), ...]) with local ids."""
     qlab, qedges = qgraph
     dlab, dedges = dgraph
@@ -42,12 +51,14 @@ def brute_count(qgraph, dgraph) -> int:
             continue
         if any(bond.get((f[u], f[v])) != b for (u, v, b) in qedges):  # condition (2) + bond labels
             continue
+        if induced and not _induced_ok(f, qedges, bond, nq):
+            continue
         total += 1
     return total
 
 
-def brute_dense(qgraphs, dgraphs, find_first: bool = False):
-    out = [[brute_count(q, d) for d in dgraphs] for q in qgraphs]
+def brute_dense(qgraphs, dgraphs, find_first: bool = False, induced: bool = False):
+    out = [[brute_count(q, d, induced) for d in dgraphs] for q in qgraphs]
     if find_first:
         out = [[1 if c else 0 for c in row] for row in out]
     return out

@@ -28,6 +28,13 @@
  *      (f(pi_j), v) with bond label b; assign, recurse, unassign
  *   5. at depth n_q count one embedding; Find First returns at the first leaf.
  *
+ * Induced mode (mode bit 1, the literal G_D[X] reading of
+ * Def. 2.1): additionally
+ *                   for all u != v in V_q with (u,v) not in E_q:
+ *                         (f(u),f(v)) not in E_g (any bond label)       (3)
+ *   step 3b: non[i] = {j < i : (pi_j, pi_i) not in E_q}
+ *   step 4b: require no data edge between f(pi_j) and v for j in non[i].
+ *
  * Threads (std pthreads) split the data graphs into static contiguous chunks
  * and write independent per-pair slots, so results are deterministic.
  * Counts are u64; an addition that would overflow sets *overflow (R19).
@@ -54,6 +61,8 @@ typedef struct {
   int nback[64];
   int back_j[64][64];    /* depth index j < i */
   int back_b[64][64];    /* bond label */
+  int nnon[64];
+  int non_j[64][64];     /* depth index j < i with (pi_j, pi_i) NOT in E_q (induced mode) */
 } qplan;
 
 static int build_plan(const oracle_batch *Q, int64_t q, qplan *P) {
@@ -95,6 +104,14 @@ static int build_plan(const oracle_batch *Q, int64_t q, qplan *P) {
         P->nback[i]++;
       }
     }
+    /* step 3b (induced mode): earlier depths not adjacent to pi_i */
+    P->nnon[i] = 0;
+    for (int j = 0; j < i; j++) {
+      int adj = 0;
+      for (int k = 0; k < P->nback[i]; k++)
+        if (P->back_j[i][k] == j) adj = 1;
+      if (!adj) P->non_j[i][P->nnon[i]++] = j;
+    }
   }
   return 0;
 }
@@ -108,6 +125,7 @@ typedef struct {
   int map[64];
   uint8_t used[256];
   int find_first;
+  int induced;
   int overflow;
   uint64_t work;        /* search-tree nodes visited (informational) */
 } search;
@@ -123,6 +141,10 @@ static uint64_t rec(search *S, int depth) {
       int u = S->map[S->P->back_j[depth][k]];
       if (S->adjm[u * S->ng + v] != S->P->back_b[depth][k]) { ok = 0; break; }
     }
+    if (!ok) continue;
+    if (S->induced)  /* step 4b: no data edge (any bond) between v and f(pi_j) for j in non[i] */
+      for (int k = 0; k < S->P->nnon[depth]; k++)
+        if (S->adjm[S->map[S->P->non_j[depth][k]] * S->ng + v] >= 0) { ok = 0; break; }
     if (!ok) continue;
     S->used[v] = 1;
     S->map[depth] = v;
@@ -176,14 +198,15 @@ static uint64_t count_one(job *J, const qplan *P, int ng, const uint8_t *glab, c
   S.ng = ng;
   S.glab = glab;
   S.adjm = adjm;
-  S.find_first = J->find_first;
+  S.find_first = J->find_first & 1;
+  S.induced = (J->find_first >> 1) & 1;
   S.overflow = 0;
   S.work = 0;
   memset(S.used, 0, sizeof(S.used));
   uint64_t c = rec(&S, 0);
   J->work += S.work;
   if (S.overflow) J->overflow = 1;
-  return J->find_first ? (c ? 1u : 0u) : c;
+  return (J->find_first & 1) ? (c ? 1u : 0u) : c;
 }
 
 static void *dense_worker(void *arg) {
@@ -245,7 +268,9 @@ static int run_jobs(job *jobs, int nthreads, void *(*fn)(void *), uint64_t *work
 }
 
 /* Dense results out[q*ND + g] for every (query, data graph) pair.
- * mode 0 = Find All (counts), 1 = Find First (0/1).  Returns 0 on success. */
+ * mode bit 0: 0 = Find All (counts), 1 = Find First (0/1); mode bit 1
+ * (value 2): induced-subgraph mode (Def. 2.1 read literally as G_D[X],
+ * P:427-440, R20).  Returns 0 on success. */
 int oracle_count_dense(const oracle_batch *Q, const oracle_batch *D, int mode, int nthreads,
                        uint64_t *out, uint64_t *work_out, int *overflow_out) {
   if (nthreads < 1) nthreads = 1;

@@ -207,3 +207,64 @@ def test_pair_list_matches_dense():
     assert np.array_equal(out.reshape(full.shape), full)
     out1 = oracle.count_pairs(Q, D, pq.ravel(), pg.ravel(), nthreads=1)
     assert np.array_equal(out1, out)
+
+
+# ---------------------------------------------------------------- N4 induced mode (R20)
+IND = oracle.INDUCED
+
+
+def test_induced_closed_forms():
+    assert count([path(3)], [ring(3)], IND)[0, 0] == 0         # P3 needs a non-edge; K3 has none
+    assert count([path(3)], [ring(3)])[0, 0] == 6              # vs monomorphism (R1)
+    assert count([path(3, C, 4)], [ring(6, C, 4)], IND)[0, 0] == 12   # C6 has no chords
+    assert count([ring(4)], [complete(4)], IND)[0, 0] == 0     # K4 has both diagonals
+    assert count([ring(4)], [complete(4)])[0, 0] == 24
+    for n in range(1, 6):
+        assert count([complete(n)], [complete(n + 1)], IND)[0, 0] == math.factorial(n + 1)  # cliques induce
+    # two isolated C in P4 (C-C-C-C): ordered non-adjacent pairs = 2 * (C(4,2) - 3)
+    assert count([([C, C], [])], [path(4)], IND)[0, 0] == 6
+    assert count([([C, C], [])], [path(4)], IND | oracle.FIND_FIRST)[0, 0] == 1
+    # a non-edge with a bond of another label still counts as an edge (any bond)
+    q = ([C, C, C], [(0, 1, 1), (1, 2, 1)])
+    d = ([C, C, C], [(0, 1, 1), (1, 2, 1), (0, 2, 2)])
+    assert count([q], [d])[0, 0] == 2 and count([q], [d], IND)[0, 0] == 0
+
+
+def test_induced_vs_brute_force_and_subset():
+    rng = np.random.default_rng(777)
+    qs = [synth.random_labelled_graph(rng, int(rng.integers(1, 6)), float(rng.uniform(0.3, 1.0)),
+                                      labels=(C, N), bonds=(1, 2)) for _ in range(60)]
+    ds = [synth.random_labelled_graph(rng, int(rng.integers(1, 9)), float(rng.uniform(0.2, 0.8)),
+                                      labels=(C, N), bonds=(1, 2)) for _ in range(80)]
+    ind = count(qs, ds, IND)
+    ff = count(qs, ds, IND | oracle.FIND_FIRST)
+    mono = count(qs, ds)
+    n_pos = n_strict = 0
+    for i, q in enumerate(qs):
+        for j, d in enumerate(ds):
+            b = brute_count(q, d, induced=True)
+            assert ind[i, j] == b, (i, j)
+            assert ff[i, j] == (1 if b else 0)
+            assert ind[i, j] <= mono[i, j]
+            n_pos += b > 0
+            n_strict += ind[i, j] < mono[i, j]
+    assert n_pos > 40 and n_strict > 40  # both matching and induced-pruned pairs are exercised
+
+
+def test_induced_vs_networkx_molecules():
+    pytest.importorskip("networkx")
+    from networkx.algorithms import isomorphism as iso
+    D = synth.molecules(synth.DATA_SEED_BASE + 98, 0, 30)
+    qs = synth.library() + synth.random_subgraph_queries(8, 10)
+    res = oracle.count_dense(GraphBatch.from_graphs(qs), D, IND)
+    nm = iso.categorical_node_match("l", None)
+    em = iso.categorical_edge_match("b", None)
+    total = 0
+    for g in range(D.num_graphs):
+        G = _nx(D.graph(g))
+        for qi, q in enumerate(qs):
+            GM = iso.GraphMatcher(G, _nx(q), node_match=nm, edge_match=em)
+            c = sum(1 for _ in GM.subgraph_isomorphisms_iter())  # induced (node-induced subgraph isomorphism)
+            assert res[qi, g] == c, (qi, g)
+            total += c
+    assert total > 0
