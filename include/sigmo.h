@@ -13,7 +13,7 @@
  *              filter (Alg. 1; section 4.2-4.4) ->
  *              GMCR mapping (section 4.5) -> DFS join
  *              (section 4.6).
- * Readings of the paper (R1-R20) are listed in DESIGN.md.
+ * Readings of the paper (R1-R21) are listed in DESIGN.md.
  *
  * Conventions (all calls):
  *   * Every call returns sigmo_status; 0 = SIGMO_OK.  On error the context
@@ -182,6 +182,15 @@ SIGMO_API sigmo_status sigmo_get_candidates(sigmo_ctx *ctx, uint32_t *out);
 SIGMO_API sigmo_status sigmo_get_signatures(sigmo_ctx *ctx, int which, int radius, uint64_t *out);
 
 /* Enable/disable per-stage CUDA-event timing (default off) and read it. */
+/* Induced-subgraph mode (the literal G_D[X] reading of
+ * Def. 2.1; R21): an embedding must also map every
+ * NON-adjacent query node pair to a non-adjacent data node pair (a data bond
+ * of any label counts as adjacency).  enable = 0 (default, monomorphism,
+ * reading R1) or 1.  Takes effect at the next sigmo_load_batch, which then
+ * routes the batch to the general join kernel; the filter is unchanged
+ * (induced embeddings are a subset of the monomorphisms, so its candidate
+ * sets stay sound).  Never fails for a valid ctx. */
+SIGMO_API sigmo_status sigmo_set_induced(sigmo_ctx *ctx, int enable);
 SIGMO_API sigmo_status sigmo_set_timing(sigmo_ctx *ctx, int enable);
 SIGMO_API sigmo_status sigmo_get_timings(sigmo_ctx *ctx, sigmo_timings *out);
 

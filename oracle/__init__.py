@@ -30,7 +30,7 @@ _lib = None
 
 FIND_ALL = 0
 FIND_FIRST = 1
-INDUCED = 2  # mode bit: induced-subgraph embeddings (R20)
+INDUCED = 2  # mode bit: induced-subgraph embeddings (R21)
 
 
 class _Batch(ctypes.Structure):

@@ -11,7 +11,7 @@ import itertools
 
 
 def _induced_ok(f, qedges, bond, nq):
-    """Condition (3) of the induced reading (G_D[X]; R20):
+    """Condition (3) of the induced reading (G_D[X]; R21):
     non-adjacent query nodes map to non-adjacent data nodes."""
     qadj = {(u, v) for (u, v, _) in qedges} | {(v, u) for (u, v, _) in qedges}
     return all((f[u], f[v]) not in bond for u in range(nq) for v in range(nq) if u != v and (u, v) not in qadj)

@@ -270,7 +270,7 @@ static int run_jobs(job *jobs, int nthreads, void *(*fn)(void *), uint64_t *work
 /* Dense results out[q*ND + g] for every (query, data graph) pair.
  * mode bit 0: 0 = Find All (counts), 1 = Find First (0/1); mode bit 1
  * (value 2): induced-subgraph mode (Def. 2.1 read literally as G_D[X],
- * P:427-440, R20).  Returns 0 on success. */
+ * P:427-440, R21).  Returns 0 on success. */
 int oracle_count_dense(const oracle_batch *Q, const oracle_batch *D, int mode, int nthreads,
                        uint64_t *out, uint64_t *work_out, int *overflow_out) {
   if (nthreads < 1) nthreads = 1;

@@ -186,6 +186,10 @@ class Context:
                     "sigmo_get_signatures")
         return out
 
+    def set_induced(self, enable: bool = True):
+        """Induced-subgraph mode for the next load_batch (include/sigmo.h sigmo_set_induced)."""
+        self._check(self._lib.sigmo_set_induced(self._handle, 1 if enable else 0), "sigmo_set_induced")
+
     def set_timing(self, enable: bool = True):
         self._check(self._lib.sigmo_set_timing(self._handle, 1 if enable else 0), "sigmo_set_timing")
 

@@ -138,6 +138,8 @@ struct sigmo_ctx {
   // ---- join ----
   DBuf pair_query, pair_rec, pair_cm, pair_result, jcnt, adjb, ent2;
   // jcnt u64 slots: [0] pair cursor / chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
+  int induced = 0;         // sigmo_set_induced (applies to the next sigmo_load_batch)
+  int induced_loaded = 0;  // induced mode of the loaded batch (routes it to k_join)
   bool lane_join = false;  // per-lane join possible for this batch (<= 64-node graphs, <= 16-node queries)
   bool mol_filter = false; // last sigmo_filter used molecule tiles (candidates in cmol layout)
   bool dense_pad_zero = false;  // padding words >= W of the dense bitmap rows (and the tail) are zero
@@ -820,6 +822,7 @@ void fill_join_caps(sigmo_ctx *c, JoinParams &jp) {
   jp.NQW = c->NQW;
   jp.VQ = c->VQ;
   jp.NB = c->NB;
+  jp.induced = c->induced_loaded;
   jp.maxq = std::max(c->maxq, 2);
   jp.PCAP = c->PC;
   jp.ACAP = c->AC + c->maxn;
@@ -936,6 +939,12 @@ sigmo_status sigmo_destroy(sigmo_ctx *c) {
   return SIGMO_OK;
 }
 
+sigmo_status sigmo_set_induced(sigmo_ctx *c, int enable) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  c->induced = enable != 0;
+  return SIGMO_OK;
+}
+
 sigmo_status sigmo_set_timing(sigmo_ctx *c, int enable) {
   if (!c) return SIGMO_ERR_INVALID_ARG;
   c->timing.enabled = enable != 0;
@@ -1020,12 +1029,13 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   }
   // per-lane join + molecule-tile filter possible for this batch?
   bool lane_ok = false;
+  c->induced_loaded = c->induced;
   {
     int64_t maxn_h = 0, maxq_h = 0;
     for (int64_t g = 0; g < hd.G; g++) maxn_h = std::max<int64_t>(maxn_h, hd.goff[g + 1] - hd.goff[g]);
     for (int64_t g = 0; g < hq.G; g++) maxq_h = std::max<int64_t>(maxq_h, hq.goff[g + 1] - hq.goff[g]);
     const char *legacy = getenv("SIGMO_JOIN_LEGACY");
-    lane_ok = maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
+    lane_ok = !c->induced && maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
               (unsigned long long)std::max<int64_t>(hq.V, 1) * (unsigned long long)std::max<int64_t>(hd.G, 1) <
                   (1ull << 32) &&
               (unsigned long long)(c->NB + 1) * hd.V + 1 < (1ull << 31) &&

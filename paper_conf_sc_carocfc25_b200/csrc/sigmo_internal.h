@@ -157,6 +157,8 @@ struct JoinParams {
   const uint2 *qp_ent2;        // [VQ] compact, k_join_lane: x = j0 | j1 << 4 | #extra << 8 | distinct row << 12,
                                // y = extra back-edge start (16 b) | class0 << 16 | class1 << 19
   int batchK;                  // finish/assign pairs when >= batchK lanes are free
+  int induced;                 // 1 = induced-subgraph embeddings (k_join only, R21):
+                               // the union of all bonds is staged as adjacency class NB
 };
 
 // k_pairs: GMCR pair list + per-pair candidate masks

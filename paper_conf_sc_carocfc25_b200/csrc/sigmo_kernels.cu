@@ -1380,7 +1380,7 @@ __host__ __device__ inline JoinSmem join_layout(const JoinParams &p, int NW, int
   L.tot = o;   o = align16(o + 8 * (size_t)p.NQ);
   L.warps = o;
   size_t w = 0;
-  L.w.adj = w;     w = align16(w + mb * (size_t)p.NB * p.ACAP);
+  L.w.adj = w;     w = align16(w + mb * (size_t)(p.NB + (p.induced ? 1 : 0)) * p.ACAP);
   L.w.cm = w;      w = align16(w + mb * (size_t)p.CMCAP);
   L.w.cinfo = w;   w = align16(w + 4 * (size_t)p.CMCAP);
   L.w.pinfo = w;   w = align16(w + 16 * (size_t)p.PCAP);
@@ -1501,19 +1501,22 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
     for (int i = lane; i < na; i += 32) {
       const int v = a0 + i;
       const int e0 = __ldg(&jp.roff[v]), e1 = __ldg(&jp.roff[v + 1]);
-      M m[8];
+      M m[8], mall;
 #pragma unroll
       for (int b = 0; b < 8; b++) m[b].clear();
+      mall.clear();
       for (int e = e0; e < e1; e++) {
         const int x = __ldg(&jp.nbr[e]);
         const int cls = jp.bclass[x & 255];
 #pragma unroll
         for (int b = 0; b < 8; b++)
           if (cls == b) m[b].set(x >> 8);
+        mall.set(x >> 8);
       }
 #pragma unroll
       for (int b = 0; b < 8; b++)
         if (b < jp.NB) s_adj[b * ACAP + i] = m[b];
+      if (jp.induced) s_adj[jp.NB * ACAP + i] = mall;  // every bond, whatever its label
     }
     __syncwarp();
     // The chunk's pairs are processed in passes that fit the warp's pair /
@@ -1679,12 +1682,30 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
           x &= s_adj[(be & 255) * ACAP + mbase + map_get<MQ>(mp, be >> 8)];
         }
       }
+      if (jp.induced && e < nq) {
+        // induced mode (condition (3), R21): v' must not be adjacent
+        // (any bond) to f(j) for every mapped depth j that is not a back-edge
+        unsigned long long bm = 0ull;
+        {
+          const int j0 = info & 0x3f, j1 = (info >> 9) & 0x3f;
+          if (j0 != 0x3f) bm |= 1ull << j0;
+          if (j1 != 0x3f) bm |= 1ull << j1;
+          if (nex) {
+            const int k0 = __ldg(&jp.qp_beoff[pinf.y + ec]) + 2;
+#pragma unroll 1
+            for (int k = 0; k < nex; k++) bm |= 1ull << (__ldg(&jp.qp_be[k0 + k]) >> 8);
+          }
+        }
+#pragma unroll 1
+        for (int j = 0; j < e; j++)
+          if (!((bm >> j) & 1ull)) x = x.andnot(s_adj[jp.NB * ACAP + mbase + map_get<MQ>(mp, j)]);
+      }
       // leaf sum (e == nq-2 and the last node is not adjacent to depth nq-2):
       // X = candidates of the last depth given f(0..e-1) and v; then
       // sum_{w in x} |X \ {w}| = |x||X| - |x & X|
       const int lastd = max(nq - 1, 0);
       const uint32_t li = s_cinfo[pinf.x + lastd];
-      const bool lsum = (e == nq - 2) && ((li >> 24) & 1u);
+      const bool lsum = !jp.induced && (e == nq - 2) && ((li >> 24) & 1u);
       unsigned long long cnt = 0ull;
       if (__any_sync(FULL_MASK, lsum && alive)) {
         M X = s_cm[pinf.x + lastd].andnot(u2);

@@ -209,7 +209,7 @@ def test_pair_list_matches_dense():
     assert np.array_equal(out1, out)
 
 
-# ---------------------------------------------------------------- N4 induced mode (R20)
+# ---------------------------------------------------------------- N4 induced mode (R21)
 IND = oracle.INDUCED
 
 
