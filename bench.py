@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--induced", action="store_true",
+                    help="induced-subgraph embeddings (sigmo_set_induced; SURVEY 8(f) N4, DESIGN.md R21)")
     a = ap.parse_args()
     a.cid = CONFIGS[a.config][0]
     if a.molecules is None:
@@ -180,16 +182,17 @@ def run_cpu_baseline(Q, args):
     nmol = min(CPU_SAMPLE_MOLS, args.molecules)
     D = synth.config_data(args.cid, first=0, count=nmol)
     th = host_cores()
+    im = oracle.INDUCED if getattr(args, "induced", False) else 0
     t0 = time.perf_counter()
-    res = oracle.count_dense(Q, D, oracle.FIND_ALL, nthreads=th)
+    res = oracle.count_dense(Q, D, oracle.FIND_ALL | im, nthreads=th)
     dt = time.perf_counter() - t0
     t1 = time.perf_counter()
-    oracle.count_dense(Q, D, oracle.FIND_FIRST, nthreads=th)
+    oracle.count_dense(Q, D, oracle.FIND_FIRST | im, nthreads=th)
     dt_ff = time.perf_counter() - t1
     # single-thread rate on a 1 % deterministic subsample (every 100th molecule)
     sub = synth.GraphBatch.from_graphs([D.graph(g) for g in range(0, D.num_graphs, 100)])
     t2 = time.perf_counter()
-    r1 = oracle.count_dense(Q, sub, oracle.FIND_ALL, nthreads=1)
+    r1 = oracle.count_dense(Q, sub, oracle.FIND_ALL | im, nthreads=1)
     dt1 = time.perf_counter() - t2
     return {"value": float(res.sum()) / dt, "unit": "matches/s", "cores": th, "kind": "oracle",
             "single_thread": {"value": float(r1.sum()) / dt1, "unit": "matches/s",
@@ -208,6 +211,7 @@ def run_reference(args, world, rank):
     import synth
     Q = synth.config_queries(args.cid)
     th = host_cores()
+    im = oracle.INDUCED if args.induced else 0
     n_total = args.molecules
     step_mols = min(REF_STEP_MOLS, n_total)
 
@@ -216,13 +220,13 @@ def run_reference(args, world, rank):
         return synth.config_data(args.cid, first=first, count=step_mols)
 
     for i in range(args.warmup):
-        oracle.count_dense(Q, batch(i), oracle.FIND_ALL, nthreads=th)
+        oracle.count_dense(Q, batch(i), oracle.FIND_ALL | im, nthreads=th)
     batches = [batch(args.warmup + i) for i in range(args.steps)]
     matches = 0
     t = 0.0
     for D in batches:
         t0 = time.perf_counter()
-        r = oracle.count_dense(Q, D, oracle.FIND_ALL, nthreads=th)
+        r = oracle.count_dense(Q, D, oracle.FIND_ALL | im, nthreads=th)
         t += time.perf_counter() - t0
         matches += int(r.sum())
     value = matches / t
@@ -249,6 +253,9 @@ def config_dict(args, world, oracle_step=None):
          "l2": ("flushed before every timed step (256 MiB device write, outside the events)" if args.cid in (2, 3)
                 else "no flush: per-step inputs and candidate arrays are larger than the 126 MB L2"),
          "parallelism": f"dp{world}: molecule shards, queries replicated, NCCL all-reduce of per-query totals"}
+    if getattr(args, "induced", False):
+        d["workload"] += ", induced-subgraph mode (N4)"
+        d["induced"] = True
     if oracle_step:
         d["oracle_molecules_per_step"] = oracle_step
     return d
@@ -262,6 +269,8 @@ def main():
         run_reference(args, world, rank)
         return
     if args.cid in (4, 5):
+        if args.induced:
+            raise SystemExit("--induced applies to configs[0..2] (the routed runs use the lane join)")
         run_routed(args, world, rank, local)
         return
     import numpy as np
@@ -278,6 +287,8 @@ def main():
     D = synth.config_data(args.cid, first=rank * args.molecules, count=args.molecules)
     stream = torch.cuda.current_stream(dev)
     ctx = sigmo.Context(local, stream)
+    if args.induced:
+        ctx.set_induced(True)
     ctx.load_batch(Q, D)
     totals = torch.zeros(Q.num_graphs, dtype=torch.int64, device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
