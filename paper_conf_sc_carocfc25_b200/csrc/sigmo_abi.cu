@@ -118,6 +118,7 @@ struct sigmo_ctx {
   uint16_t *qp_be = nullptr;
   uint32_t *qp_info = nullptr;
   const int4 *qp_ent = nullptr;
+  const uint32_t *qp_non = nullptr;
   const uint32_t *qp_qinfo = nullptr;
   int32_t *tile_g0 = nullptr, *tile_g1 = nullptr;
   uint8_t *bclass = nullptr;
@@ -823,6 +824,7 @@ void fill_join_caps(sigmo_ctx *c, JoinParams &jp) {
   jp.VQ = c->VQ;
   jp.NB = c->NB;
   jp.induced = c->induced_loaded;
+  jp.qp_non = c->qp_non;
   jp.maxq = std::max(c->maxq, 2);
   jp.PCAP = c->PC;
   jp.ACAP = c->AC + c->maxn;
@@ -1035,10 +1037,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     for (int64_t g = 0; g < hd.G; g++) maxn_h = std::max<int64_t>(maxn_h, hd.goff[g + 1] - hd.goff[g]);
     for (int64_t g = 0; g < hq.G; g++) maxq_h = std::max<int64_t>(maxq_h, hq.goff[g + 1] - hq.goff[g]);
     const char *legacy = getenv("SIGMO_JOIN_LEGACY");
-    lane_ok = !c->induced && maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
+    lane_ok = maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
               (unsigned long long)std::max<int64_t>(hq.V, 1) * (unsigned long long)std::max<int64_t>(hd.G, 1) <
                   (1ull << 32) &&
-              (unsigned long long)(c->NB + 1) * hd.V + 1 < (1ull << 31) &&
+              (unsigned long long)(c->NB + 2) * hd.V + 1 < (1ull << 31) &&
               plan.be.size() + 2 < 0xffff;  // compact plan entries: 16-bit extra back-edge offsets
   }
   const auto t2 = std::chrono::steady_clock::now();
@@ -1051,6 +1053,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const size_t o_bc = L.take(256);
   const size_t o_info = L.take(4 * (size_t)hq.V + 4);
   const size_t o_ent = L.take(16 * (size_t)hq.V + 16);
+  const size_t o_non = L.take(4 * (size_t)hq.V + 4);  // induced mode: non-adjacent earlier depths per plan position
   const size_t o_qinfo = L.take(4 * (size_t)hq.G + 4);
   const PackedOffsets pd = plan_graphs(L, hd);
   const size_t o_tg0 = L.take(4 * tg0.size());
@@ -1080,7 +1083,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       const int64_t n = hd.goff[g + 1] - hd.goff[g];
       if (n > 32) w = (w + 1) & ~1ull;
       aoff[g] = (uint32_t)std::min<uint64_t>(w, 0xffffffffull);
-      w += (uint64_t)n * (uint64_t)std::max(c->NB, 1) * (n > 32 ? 2 : 1);
+      w += (uint64_t)n * (uint64_t)(std::max(c->NB, 1) + c->induced_loaded) * (n > 32 ? 2 : 1);  // + the all-bonds class
     }
     w = (w + 1) & ~1ull;
     aoff[hd.G] = (uint32_t)std::min<uint64_t>(w, 0xffffffffull);
@@ -1144,6 +1147,16 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       ent[i] = e4;
     }
     if (hq.G) memcpy(hb + o_qinfo, plan.qinfo.data(), 4 * (size_t)hq.G);
+    // induced mode (R21): bit j of non[i] = earlier depth j < e not adjacent to depth e
+    uint32_t *non = (uint32_t *)(hb + o_non);
+    int64_t qn = 0;
+    for (int64_t i = 0; i < hq.V; i++) {
+      while (hq.goff[qn + 1] <= i) qn++;
+      const int e = (int)(i - hq.goff[qn]);
+      uint64_t m = e >= 32 ? 0xffffffffull : ((1ull << e) - 1ull);
+      for (int k = plan.beoff[i]; k < plan.beoff[i + 1]; k++) m &= ~(1ull << (plan.be[k] >> 8));
+      non[i] = (uint32_t)m;
+    }
     c->ent_host.assign(ent, ent + hq.V);
     c->ent_row.assign(plan.row.begin(), plan.row.end());
     c->qgoff_host.assign(hq.goff, hq.goff + hq.G + 1);
@@ -1179,6 +1192,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->tile_g1 = (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
   c->qp_ent = (const int4 *)(db + o_ent);
+  c->qp_non = (const uint32_t *)(db + o_non);
   c->qp_qinfo = (const uint32_t *)(db + o_qinfo);
   c->NQ = (int)hq.G;
   c->VQ = (int)hq.V;
@@ -1258,7 +1272,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     SIGMO_TRY(dreserve(c, c->adjb, 4 * ((size_t)c->adj_words + 2), "bond-class adjacency"));
     // words adj_words, adj_words + 1 = all ones: the target of absent back-edges
     CUDA_TRY(c, cudaMemsetAsync((uint32_t *)c->adjb.p + c->adj_words, 0xff, 8, c->stream));
-    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, c->adj_off, (uint32_t *)c->adjb.p, c->stream));
+    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, c->induced_loaded, c->adj_off, (uint32_t *)c->adjb.p, c->stream));
   }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
   SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 8), "join counters"));  // + the second claim counter

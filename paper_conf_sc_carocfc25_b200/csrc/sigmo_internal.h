@@ -159,6 +159,7 @@ struct JoinParams {
   int batchK;                  // finish/assign pairs when >= batchK lanes are free
   int induced;                 // 1 = induced-subgraph embeddings (k_join only, R21):
                                // the union of all bonds is staged as adjacency class NB
+  const uint32_t *qp_non;      // [VQ] induced mode: mask of the earlier plan depths NOT adjacent to depth e
 };
 
 // k_pairs: GMCR pair list + per-pair candidate masks
@@ -214,7 +215,7 @@ cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
 cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
                          int VQ, int Wpad, uint32_t *dense,
                          cudaStream_t st);
-cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
+cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, int induced, const uint32_t *adj_off, uint32_t *adjw,
                         cudaStream_t st);
 cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, cudaStream_t st);
 size_t join_lane_smem_bytes(const JoinParams &p, bool w64);

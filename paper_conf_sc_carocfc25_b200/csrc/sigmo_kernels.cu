@@ -1937,10 +1937,11 @@ cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const
 // holding v, so that lanes reading the same class of one molecule touch few
 // 32-B sectors.
 // ===========================================================================
-__global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw) {
+__global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, int induced, const uint32_t *adj_off,
+                       uint32_t *adjw) {
   const int v = blockIdx.x * blockDim.x + threadIdx.x;
   if (v >= d.num_nodes) return;
-  unsigned long long m[8];
+  unsigned long long m[8], mall = 0ull;
 #pragma unroll
   for (int b = 0; b < 8; b++) m[b] = 0ull;
   const int e1 = d.roff[v + 1];
@@ -1950,6 +1951,7 @@ __global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, const uint32_
 #pragma unroll
     for (int b = 0; b < 8; b++)
       if (cls == b) m[b] |= 1ull << ((x >> 8) & 63);
+    mall |= 1ull << ((x >> 8) & 63);
   }
   const int g = graph_of(d.goff, d.num_graphs, v);
   const int a = d.goff[g], n = d.goff[g + 1] - a;
@@ -1960,12 +1962,16 @@ __global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, const uint32_
       if (n <= 32) adjw[base + (uint32_t)(b * n + (v - a))] = (uint32_t)m[b];
       else *(unsigned long long *)(adjw + base + 2u * (uint32_t)(b * n + (v - a))) = m[b];
     }
+  if (induced) {  // class NB: every bond, whatever its label (induced mode, R21)
+    if (n <= 32) adjw[base + (uint32_t)(NB * n + (v - a))] = (uint32_t)mall;
+    else *(unsigned long long *)(adjw + base + 2u * (uint32_t)(NB * n + (v - a))) = mall;
+  }
 }
 
-cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
-                        cudaStream_t st) {
+cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, int induced, const uint32_t *adj_off,
+                        uint32_t *adjw, cudaStream_t st) {
   if (d.num_nodes <= 0 || NB <= 0) return cudaSuccess;
-  k_adjb<<<(d.num_nodes + 255) / 256, 256, 0, st>>>(d, bclass, NB, adj_off, adjw);
+  k_adjb<<<(d.num_nodes + 255) / 256, 256, 0, st>>>(d, bclass, NB, induced, adj_off, adjw);
   return cudaGetLastError();
 }
 
@@ -2162,9 +2168,14 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
           X &= adj(ca + (((unsigned)(be & 255) * ng + smem[oM + 32u * (be >> 8)]) << sw));
         }
       }
+      if (MODE & 2) {  // induced mode (R21): drop neighbours (any bond) of mapped non-adjacent depths
+        const unsigned cn = (unsigned)jp.NB * ng;
+        for (unsigned nm = __ldg(&jp.qp_non[cqb + e]); nm; nm &= nm - 1u)
+          X &= ~adj(ca + ((cn + smem[oM + 32u * (unsigned)(__ffs(nm) - 1)]) << sw));
+      }
       if (e == (int)(cinfo & 0xff) - 1) {
         cnt += (unsigned long long)popc(X);
-        if (MODE == 1 && cnt) ne = 0u;  // Find First: the pair (part) is decided
+        if ((MODE & 1) && cnt) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
         stRU(oRU + 32u * ES * e, X, used);
         ne |= 1u << e;
@@ -2177,7 +2188,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
 
     // ---- finished pairs (parts): result, per-query total in shared memory ----
     if (pend) {
-      if (MODE == 1) {
+      if (MODE & 1) {
         if (!shared) {
           presult[cp] = cnt ? 1ull : 0ull;
           if (cnt) atomicAdd((unsigned long long *)(smem + o_tot) + cq, 1ull);
@@ -2326,8 +2337,22 @@ static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_
 
 cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, cudaStream_t st) {
   if (grid <= 0) return cudaSuccess;
-  if (w64) return mode == 1 ? launch_join_lane_t<1, true>(p, grid, st) : launch_join_lane_t<0, true>(p, grid, st);
-  return mode == 1 ? launch_join_lane_t<1, false>(p, grid, st) : launch_join_lane_t<0, false>(p, grid, st);
+  // mode bit 0: Find First; bit 1: induced (p.induced)
+  const int m = (mode & 1) | (p.induced ? 2 : 0);
+  if (w64) {
+    switch (m) {
+      case 0: return launch_join_lane_t<0, true>(p, grid, st);
+      case 1: return launch_join_lane_t<1, true>(p, grid, st);
+      case 2: return launch_join_lane_t<2, true>(p, grid, st);
+      default: return launch_join_lane_t<3, true>(p, grid, st);
+    }
+  }
+  switch (m) {
+    case 0: return launch_join_lane_t<0, false>(p, grid, st);
+    case 1: return launch_join_lane_t<1, false>(p, grid, st);
+    case 2: return launch_join_lane_t<2, false>(p, grid, st);
+    default: return launch_join_lane_t<3, false>(p, grid, st);
+  }
 }
 
 template <int MODE, bool W64>

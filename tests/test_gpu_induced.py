@@ -88,3 +88,17 @@ def test_induced_toggle_restores_monomorphism(ctx, sigmo):
     ctx.filter(4)
     ctx.join(sigmo.SIGMO_FIND_ALL)
     assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D))
+
+
+def test_induced_general_path_forced(sigmo, monkeypatch):
+    """the same batches through the general k_join (SIGMO_JOIN_LEGACY routes
+    the load away from the lane join) -- both induced implementations agree
+    with the oracle."""
+    monkeypatch.setenv("SIGMO_JOIN_LEGACY", "1")
+    c = sigmo.Context(0)
+    c.set_induced(True)
+    try:
+        check(c, sigmo, synth.config_queries(1), synth.config_data(1))
+        check(c, sigmo, synth.config_queries(2), synth.config_data(2, count=5000))
+    finally:
+        c.close()
