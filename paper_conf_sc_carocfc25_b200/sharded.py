@@ -40,6 +40,65 @@ def equal_count_range(n_total: int, rank: int, world: int) -> Tuple[int, int]:
     return n_total * rank // world, n_total * (rank + 1) // world
 
 
+# ---------------------------------------------------------------------------
+# Cost-model partitioning.  The paper's static
+# equal-molecule split leaves a 4-8 % runtime CV across GPUs and names
+# adaptive load balancing as the remedy.  Here the per-molecule
+# cost of a batch is modelled from what the filter already produced -- its
+# atom count (filter bytes) plus its GMCR pairs (join work, section 4.5
+# P:1240-1282) -- gathered over ranks once, and the next batch of the same
+# molecules (streaming, repeated queries) is split at equal modelled cost.
+# ---------------------------------------------------------------------------
+def cost_bounds(costs, world: int) -> np.ndarray:
+    """Molecule boundaries b[0..world] splitting a per-molecule cost vector into
+    `world` contiguous shards of nearly equal summed cost (each shard's excess
+    over the ideal share is below the largest single-molecule cost)."""
+    c = np.asarray(costs, dtype=np.float64)
+    if world <= 0:
+        raise ValueError("world must be >= 1")
+    if c.ndim != 1 or (c.size and c.min() < 0):
+        raise ValueError("costs must be a 1-D non-negative vector")
+    G = c.shape[0]
+    pref = np.concatenate([[0.0], np.cumsum(c)])
+    targets = np.arange(world + 1, dtype=np.float64) * pref[-1] / world
+    b = np.searchsorted(pref[:-1], targets, side="left").astype(np.int64) if G > 0 else np.zeros(world + 1, np.int64)
+    b[0], b[-1] = 0, G
+    return np.maximum.accumulate(np.minimum(b, G))
+
+
+def molecule_costs(graph_offsets, pair_data_idx, w_atom: float = 1.0, w_pair: float = 4.0) -> np.ndarray:
+    """Per-molecule cost model: w_atom * atoms + w_pair * GMCR pairs of the
+    molecule.  pair_data_idx: data-graph index of every surviving pair
+    (Context.pair_results()[0], local indices)."""
+    goff = np.asarray(graph_offsets, dtype=np.int64)
+    G = goff.shape[0] - 1
+    pairs = np.bincount(np.asarray(pair_data_idx, dtype=np.int64), minlength=G)[:G] if G > 0 else np.zeros(0)
+    return w_atom * np.diff(goff).astype(np.float64) + w_pair * pairs.astype(np.float64)
+
+
+def gather_costs(local_costs, group=None) -> np.ndarray:
+    """Concatenate every rank's per-molecule costs in rank order (the ranks'
+    shards are contiguous and ordered).  All-gathers the lengths, then the
+    zero-padded vectors (float64; CPU tensors on gloo, device tensors on NCCL)."""
+    import torch
+    import torch.distributed as dist
+    loc = np.asarray(local_costs, dtype=np.float64)
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
+        return loc.copy()
+    world = dist.get_world_size(group)
+    dev = torch.device("cuda", torch.cuda.current_device()) if dist.get_backend(group) == "nccl" else torch.device("cpu")
+    n = torch.tensor([loc.shape[0]], dtype=torch.int64, device=dev)
+    ns = [torch.zeros_like(n) for _ in range(world)]
+    dist.all_gather(ns, n, group=group)
+    ns = [int(x.item()) for x in ns]
+    m = max(max(ns), 1)
+    buf = torch.zeros(m, dtype=torch.float64, device=dev)
+    buf[:loc.shape[0]] = torch.from_numpy(loc).to(dev)
+    outs = [torch.zeros_like(buf) for _ in range(world)]
+    dist.all_gather(outs, buf, group=group)
+    return np.concatenate([o[:k].cpu().numpy() for o, k in zip(outs, ns)])
+
+
 def allreduce_totals(totals, group=None):
     """Sum per-query totals over ranks (torch int64 tensor, in place).  On the
     NCCL backend the tensor is on the rank's GPU (NVLink); on gloo it is CPU."""

@@ -339,3 +339,24 @@ def test_neighbour_support_edge_cases(ctx, sigmo):
     assert np.array_equal(ctx.candidates(), fr.to_bitmap(Cb))
     ctx.join(sigmo.SIGMO_FIND_ALL)
     assert np.array_equal(ctx.dense_results(), oracle.count_dense(Q, D))
+
+
+def test_cost_model_from_device_gmcr(ctx, sigmo):
+    """N2 cost model (sharded.molecule_costs) fed by the device GMCR pair list
+    equals the model fed by the reference GMCR; the rebalanced split covers
+    the batch and is at least as balanced in modelled cost as the atom split."""
+    from paper_conf_sc_carocfc25_b200 import sharded
+    Q, D = synth.config_queries(1), synth.config_data(1)
+    ctx.load_batch(Q, D)
+    ctx.filter(4)
+    ctx.join(sigmo.SIGMO_FIND_ALL)
+    di, _, _ = ctx.pair_results()
+    c = sharded.molecule_costs(D.graph_offsets, di)
+    G = fr.gmcr(Q, D, fr.candidates_bool(Q, D, 4))
+    assert np.array_equal(c, sharded.molecule_costs(D.graph_offsets, np.nonzero(G)[1]))
+    for world in (2, 4, 8):
+        b = sharded.cost_bounds(c, world)
+        a = sharded.shard_bounds(D.graph_offsets, world)
+        cb = max(c[b[r]:b[r + 1]].sum() for r in range(world))
+        ca = max(c[a[r]:a[r + 1]].sum() for r in range(world))
+        assert b[-1] == D.num_graphs and cb <= ca + c.max()

@@ -68,3 +68,60 @@ def test_gloo_world2_allreduce_equals_unsharded(tmp_path):
         for r in range(world):
             got = np.load(os.path.join(tmp_path, f"r{r}_m{mode}.npy"))
             assert np.array_equal(got, ref), (r, mode)
+
+
+# ---------------------------------------------------------------- N2 cost-model partitioning
+def test_cost_bounds_balance():
+    rng = np.random.default_rng(3)
+    for G in (0, 1, 5, 1000):
+        c = rng.pareto(1.5, G) + 0.1  # heavy-tailed per-molecule cost
+        for world in (1, 2, 3, 8):
+            b = sharded.cost_bounds(c, world)
+            assert b[0] == 0 and b[-1] == G and np.all(np.diff(b) >= 0)
+            if G:
+                shard = [c[b[r]:b[r + 1]].sum() for r in range(world)]
+                assert abs(sum(shard) - c.sum()) < 1e-9 * c.sum()
+                assert max(shard) <= c.sum() / world + c.max() + 1e-9
+    # unit costs reduce to the equal-count split; atom costs to shard_bounds
+    assert np.array_equal(sharded.cost_bounds(np.ones(10), 2), [0, 5, 10])
+    D = synth.molecules(123, 0, 500)
+    for world in (2, 4):
+        assert np.array_equal(sharded.cost_bounds(D.sizes(), world), sharded.shard_bounds(D.graph_offsets, world))
+    with pytest.raises(ValueError):
+        sharded.cost_bounds([1.0, -1.0], 2)
+
+
+def test_molecule_costs_model():
+    goff = np.array([0, 3, 3, 10], np.int64)
+    c = sharded.molecule_costs(goff, [0, 2, 2, 2], w_atom=1.0, w_pair=4.0)
+    assert np.array_equal(c, [3 + 4, 0, 7 + 12])
+
+
+def _cost_worker(rank, world, port, out_dir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    Q = synth.config_queries(1)
+    D = synth.config_data(1, count=150)
+    g0, g1 = sharded.shard_range(D.graph_offsets, rank, world)
+    part = D.slice(g0, g1)
+    # GMCR-pair proxy on CPU: the oracle's positive pairs of the shard (local indices)
+    dense = oracle.count_dense(Q, part, oracle.FIND_FIRST, nthreads=2)
+    local = sharded.molecule_costs(part.graph_offsets, np.nonzero(dense)[1])
+    glob = sharded.gather_costs(local)
+    np.save(os.path.join(out_dir, f"c{rank}.npy"), glob)
+    np.save(os.path.join(out_dir, f"b{rank}.npy"), sharded.cost_bounds(glob, world))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_gathered_costs_equal_unsharded(tmp_path):
+    world = 2
+    mp.spawn(_cost_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    Q = synth.config_queries(1)
+    D = synth.config_data(1, count=150)
+    dense = oracle.count_dense(Q, D, oracle.FIND_FIRST)
+    ref = sharded.molecule_costs(D.graph_offsets, np.nonzero(dense)[1])
+    for r in range(world):
+        assert np.array_equal(np.load(os.path.join(tmp_path, f"c{r}.npy")), ref)
+        assert np.array_equal(np.load(os.path.join(tmp_path, f"b{r}.npy")), sharded.cost_bounds(ref, world))
