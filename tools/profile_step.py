@@ -18,6 +18,8 @@ cid = int(sys.argv[5]) if len(sys.argv) > 5 else 2
 torch.cuda.set_device(0)
 Q, D = synth.config_queries(cid), synth.config_data(cid, count=n)
 ctx = sigmo.Context(0)
+if os.environ.get("SIGMO_PROFILE_INDUCED") == "1":
+    ctx.set_induced(True)
 ctx.load_batch(Q, D)
 for _ in range(2 + S):
     ctx.filter(L)
