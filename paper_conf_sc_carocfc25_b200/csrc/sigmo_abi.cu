@@ -1269,9 +1269,11 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->mol_filter = false;
   if (c->lane_join) {
     SIGMO_TRY(dreserve(c, c->pair_rec, 16 * (size_t)std::max(pair_cap, 1ll), "pair records"));
-    SIGMO_TRY(dreserve(c, c->adjb, 4 * ((size_t)c->adj_words + 2), "bond-class adjacency"));
-    // words adj_words, adj_words + 1 = all ones: the target of absent back-edges
+    SIGMO_TRY(dreserve(c, c->adjb, 4 * ((size_t)c->adj_words + 4), "bond-class adjacency"));
+    // words adj_words, adj_words + 1 = all ones: the target of absent back-edges;
+    // adj_words + 2, + 3 = all zeros (absent non-edge in the induced lane join)
     CUDA_TRY(c, cudaMemsetAsync((uint32_t *)c->adjb.p + c->adj_words, 0xff, 8, c->stream));
+    CUDA_TRY(c, cudaMemsetAsync((uint32_t *)c->adjb.p + c->adj_words + 2, 0, 8, c->stream));
     CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, c->induced_loaded, c->adj_off, (uint32_t *)c->adjb.p, c->stream));
   }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));

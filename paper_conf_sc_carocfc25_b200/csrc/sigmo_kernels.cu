@@ -2170,8 +2170,14 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       }
       if (MODE & 2) {  // induced mode (R21): drop neighbours (any bond) of mapped non-adjacent depths
         const unsigned cn = (unsigned)jp.NB * ng;
-        for (unsigned nm = __ldg(&jp.qp_non[cqb + e]); nm; nm &= nm - 1u)
-          X &= ~adj(ca + ((cn + smem[oM + 32u * (unsigned)(__ffs(nm) - 1)]) << sw));
+        // two depths per iteration (the second reads the all-zeros entry when absent)
+        for (unsigned nm = __ldg(&jp.qp_non[cqb + e]); nm;) {
+          const unsigned ia = ca + ((cn + smem[oM + 32u * (unsigned)(__ffs(nm) - 1)]) << sw);
+          nm &= nm - 1u;
+          const unsigned ib = nm ? ca + ((cn + smem[oM + 32u * (unsigned)(__ffs(nm) - 1)]) << sw) : ones + 2u;
+          nm &= nm - 1u;
+          X &= ~(adj(ia) | adj(ib));
+        }
       }
       if (e == (int)(cinfo & 0xff) - 1) {
         cnt += (unsigned long long)popc(X);
