@@ -8,7 +8,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libsigmo.so")
-SOURCES = ["sigmo_abi.cu", "sigmo_kernels.cu"]
+SOURCES = ["sigmo_abi.cu", "sigmo_kernels.cu", "sigmo_filter_lane.cu"]
 HEADERS = ["sigmo_internal.h", os.path.join("..", "..", "include", "sigmo.h")]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",

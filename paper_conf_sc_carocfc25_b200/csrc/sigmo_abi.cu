@@ -155,6 +155,9 @@ struct sigmo_ctx {
   int ent_R = -1;
   int mol_extn = 0, mol_extw = 0;  // molecule-tile geometry (<= 32 graphs and <= 1,024 nodes per tile)
   int n_mol_tiles = 0;
+  int32_t *grp_narrow = nullptr, *grp_wide = nullptr;  // k_filter_lane groups (input arena)
+  int NGN = 0, NGW = 0;
+  DBuf nb4, mrec;                   // k_filter_lane: packed neighbours [VD], molecule records [ND]
   int32_t *mol_tiles = nullptr;     // [n_mol_tiles + 1] first graph of each molecule tile
   uint32_t *adj_off = nullptr;      // [ND + 1] 32-bit word offset of each molecule's bond-class adjacency
   uint32_t *cand_units = nullptr;   // [ND + 1] candidate-window units before each molecule (x NDR = its cmol word offset)
@@ -650,15 +653,23 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   }
   rowp_off[VQ] = VQ * RW;
   // distinct rows: query nodes with the same channel list (label + the same
-  // constraint planes) compute the same candidate row; the molecule-tile
-  // filter computes and stores each distinct row once per molecule
+  // constraint planes) compute the same candidate row; the lane-path filter
+  // computes and stores each distinct row once per molecule.  Distinct rows
+  // are numbered by channel count (then content), so a 32-row group of
+  // k_filter_lane has nearly uniform program lengths.
   std::map<std::vector<int>, int> dmap;
+  for (int v = 0; v < VQ; v++) dmap.emplace(chans[v], 0);
+  std::vector<const std::vector<int> *> drows;
+  for (auto &kv : dmap) drows.push_back(&kv.first);
+  std::stable_sort(drows.begin(), drows.end(),
+                   [](const std::vector<int> *a, const std::vector<int> *b) { return a->size() < b->size(); });
+  for (size_t i = 0; i < drows.size(); i++) dmap[*drows[i]] = (int)i;
   std::vector<uint16_t> qdrow((size_t)VQ + 1, 0);
-  std::vector<uint32_t> drowp;
+  std::vector<uint32_t> drowp((size_t)dmap.size() * RW);
   for (int v = 0; v < VQ; v++) {
-    auto ins = dmap.emplace(chans[v], (int)dmap.size());
-    qdrow[v] = (uint16_t)ins.first->second;
-    if (ins.second) drowp.insert(drowp.end(), rowp.begin() + (size_t)v * RW, rowp.begin() + (size_t)(v + 1) * RW);
+    const int d = dmap[chans[v]];
+    qdrow[v] = (uint16_t)d;
+    std::copy(rowp.begin() + (size_t)v * RW, rowp.begin() + (size_t)(v + 1) * RW, drowp.begin() + (size_t)d * RW);
   }
   const int NDR = (int)dmap.size();
   if (NDR > 0xffff) return set_err(c, SIGMO_ERR_LIMIT, "%d distinct query rows", NDR);
@@ -677,6 +688,72 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
     }
   }
   qw_off[NQ] = (int32_t)(qw.size() / 2);
+  // ---- k_filter_lane program (FilterLaneParams) ----
+  // plane records: per (radius, field) group, chunks of <= 4 planes
+  std::vector<uint2> lrec;
+  std::vector<int32_t> lrrec((size_t)R + 1, 0);
+  for (int r0 = 0; r0 < R; r0++) {
+    lrrec[r0] = (int)lrec.size();
+    for (int g = rg_off[r0]; g < rg_off[r0 + 1]; g++)
+      for (int p = grp_poff[g]; p < grp_poff[g + 1]; p += 4) {
+        const int np = std::min(4, grp_poff[g + 1] - p);
+        uint2 e;
+        e.x = (uint32_t)(uint8_t)fslot[grp_f[g]] | ((uint32_t)np << 8) | ((uint32_t)(NLAB + 1 + p) << 16);
+        e.y = 0;
+        for (int j = 0; j < np; j++) e.y |= (uint32_t)p_t[p + j] << (8 * j);
+        lrec.push_back(e);
+      }
+  }
+  lrrec[R] = (int)lrec.size();
+  // row programs: channel byte offsets (x16: [channel][4 slots] u32), pairs
+  // per u32, 4 u32 per uint4, padded with the all-ones channel
+  int maxch = 1;
+  for (const auto *d : drows) maxch = std::max<int>(maxch, (int)d->size());
+  const int LRWV = (maxch + 7) / 8;
+  const int NCH = NLAB + 1 + NP;
+  if (16 * NCH > 0xffff) return set_err(c, SIGMO_ERR_LIMIT, "plane program too large (%d planes)", NP);
+  const uint32_t pad2 = (uint32_t)(16 * NLAB) | ((uint32_t)(16 * NLAB) << 16);
+  std::vector<uint32_t> lrowp((size_t)NDR * LRWV * 4, pad2);
+  const int NDRW = (NDR + 31) / 32;
+  std::vector<int32_t> lrgn((size_t)NDRW + 1, 0);
+  for (int d = 0; d < NDR; d++) {
+    const std::vector<int> &ch = *drows[d];
+    for (size_t j = 0; j < ch.size(); j++) {
+      uint32_t &w = lrowp[(size_t)d * LRWV * 4 + j / 2];
+      const uint32_t o = (uint32_t)(16 * ch[j]);
+      w = (j & 1) ? ((w & 0xffffu) | (o << 16)) : ((w & 0xffff0000u) | o);
+    }
+    lrgn[d / 32] = std::max<int32_t>(lrgn[d / 32], (int32_t)((ch.size() + 1) / 2));
+  }
+  // label -> label channel | field slot << 8
+  std::vector<uint16_t> llut(256);
+  {
+    std::vector<uint8_t> lab_val(NLAB > 0 ? NLAB : 1);
+    if (NLAB) CUDA_TRY(c, cudaMemcpy(lab_val.data(), P.lab_val, NLAB, cudaMemcpyDeviceToHost));
+    for (int l = 0; l < 256; l++) {
+      uint32_t lc = 0xff;
+      for (int k = 0; k < NLAB; k++)
+        if (lab_val[k] == l) lc = (uint32_t)k;
+      const int fs = fslot[field_of_label(l)];
+      llut[l] = (uint16_t)(lc | ((uint32_t)(fs >= 0 ? fs : 0xff) << 8));
+    }
+  }
+  // GMCR lists per 32-query group: [entry][lane] (word, bits), padded (0, 0)
+  const int NQG = (NQ + 31) / 32;
+  std::vector<int2> lqwh((size_t)NQG + 1);
+  std::vector<uint2> lqwl;
+  for (int qg = 0; qg < NQG; qg++) {
+    int mx = 0;
+    for (int q = 32 * qg; q < std::min(NQ, 32 * qg + 32); q++) mx = std::max(mx, qw_off[q + 1] - qw_off[q]);
+    lqwh[qg] = make_int2((int)(lqwl.size() / 32), mx);
+    for (int j = 0; j < mx; j++)
+      for (int l = 0; l < 32; l++) {
+        const int q = 32 * qg + l;
+        uint2 e = make_uint2(0u, 0u);
+        if (q < NQ && j < qw_off[q + 1] - qw_off[q]) e = make_uint2(qw[2 * (qw_off[q] + j)], qw[2 * (qw_off[q] + j) + 1]);
+        lqwl.push_back(e);
+      }
+  }
   // upload
   Layout L;
   const size_t o_rec = L.take(sizeof(GroupRec) * (rec.size() + 1));
@@ -690,6 +767,13 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   const size_t o_qd = L.take(2 * qdrow.size());
   const size_t o_qwo = L.take(4 * qw_off.size());
   const size_t o_qw = L.take(4 * (qw.size() + 2));
+  const size_t o_lrec = L.take(8 * (lrec.size() + 1));
+  const size_t o_lrr = L.take(4 * lrrec.size());
+  const size_t o_lrp = L.take(4 * (lrowp.size() + 4));
+  const size_t o_lrg = L.take(4 * lrgn.size());
+  const size_t o_lqh = L.take(8 * lqwh.size());
+  const size_t o_lql = L.take(8 * (lqwl.size() + 1));
+  const size_t o_llu = L.take(2 * llut.size());
   std::vector<unsigned char> hb(L.off, 0);
   auto put = [&](size_t o, const void *src, size_t n) { if (n) memcpy(hb.data() + o, src, n); };
   put(o_rec, rec.data(), sizeof(GroupRec) * rec.size());
@@ -703,10 +787,28 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   put(o_qd, qdrow.data(), 2 * qdrow.size());
   put(o_qwo, qw_off.data(), 4 * qw_off.size());
   put(o_qw, qw.data(), 4 * qw.size());
+  put(o_lrec, lrec.data(), 8 * lrec.size());
+  put(o_lrr, lrrec.data(), 4 * lrrec.size());
+  put(o_lrp, lrowp.data(), 4 * lrowp.size());
+  put(o_lrg, lrgn.data(), 4 * lrgn.size());
+  put(o_lqh, lqwh.data(), 8 * lqwh.size());
+  put(o_lql, lqwl.data(), 8 * lqwl.size());
+  put(o_llu, llut.data(), 2 * llut.size());
   SIGMO_TRY(dreserve(c, pc.pack, L.off, "packed query program"));
   unsigned char *db = (unsigned char *)pc.pack.p;
   CUDA_TRY(c, cudaMemcpyAsync(db, hb.data(), L.off, cudaMemcpyHostToDevice, st));
   CUDA_TRY(c, cudaStreamSynchronize(st));  // hb is pageable and goes out of scope
+  P.l_grec = (uint2 *)(db + o_lrec);
+  P.l_rrec = (int32_t *)(db + o_lrr);
+  P.l_rowp = (uint4 *)(db + o_lrp);
+  P.l_rgn = (int32_t *)(db + o_lrg);
+  P.l_qwh = (int2 *)(db + o_lqh);
+  P.l_qwl = (uint2 *)(db + o_lql);
+  P.l_lut = (uint16_t *)(db + o_llu);
+  P.meta.L_NREC = (int)lrec.size();
+  P.meta.L_RWV = LRWV;
+  P.meta.L_NQWE = (int)lqwl.size();
+  P.meta.L_NQG = NQG;
   P.grec = (GroupRec *)(db + o_rec);
   P.tab = (uint32_t *)(db + o_tab);
   P.rrec_off = (int32_t *)(db + o_rr);
@@ -813,7 +915,7 @@ void free_all(sigmo_ctx *c) {
   c->progs.clear();
   DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
                   &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_rec, &c->pair_cm, &c->pair_result, &c->jcnt,
-                  &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp, &c->ent2};
+                  &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp, &c->ent2, &c->nb4, &c->mrec};
   for (DBuf *b : bufs) dfree(c, *b);
 }
 
@@ -1083,11 +1185,11 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       const int64_t n = hd.goff[g + 1] - hd.goff[g];
       if (n > 32) w = (w + 1) & ~1ull;
       aoff[g] = (uint32_t)std::min<uint64_t>(w, 0xffffffffull);
-      w += (uint64_t)n * (uint64_t)(std::max(c->NB, 1) + c->induced_loaded) * (n > 32 ? 2 : 1);  // + the all-bonds class
+      w += (uint64_t)n * (uint64_t)(c->NB + 1) * (n > 32 ? 2 : 1);  // + the all-bonds class (index NB)
     }
     w = (w + 1) & ~1ull;
     aoff[hd.G] = (uint32_t)std::min<uint64_t>(w, 0xffffffffull);
-    if (w + 2 >= (1ull << 32)) lane_ok = false;
+    if (w + 4 >= (1ull << 32)) lane_ok = false;  // + the all-ones and all-zeros sentinel entries
   }
   const size_t o_ao = L.take(4 * aoff.size());
   // molecule-padded candidate windows (filter output, join input): per
@@ -1106,6 +1208,16 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     if ((unsigned long long)std::max<int64_t>(hq.V, 1) * (u + 2) >= (1ull << 32)) lane_ok = false;
   }
   const size_t o_cu = L.take(4 * cu.size());
+  // k_filter_lane groups: 4 molecules of <= 32 atoms / 2 of 33-64 atoms (-1 = empty slot)
+  std::vector<int32_t> grpn, grpw;
+  for (int64_t g = 0; g < hd.G; g++) {
+    const int64_t n = hd.goff[g + 1] - hd.goff[g];
+    (n > 32 ? grpw : grpn).push_back((int32_t)g);
+  }
+  while (grpn.size() % 4) grpn.push_back(-1);
+  while (grpw.size() % 2) grpw.push_back(-1);
+  const size_t o_grpn = L.take(4 * grpn.size() + 16);
+  const size_t o_grpw = L.take(4 * grpw.size() + 16);
   const size_t total = L.off;
   const auto t3 = std::chrono::steady_clock::now();
   // wait until the previous upload no longer reads the staging buffer
@@ -1168,6 +1280,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   memcpy(hb + o_mt, mt.data(), 4 * mt.size());
   memcpy(hb + o_ao, aoff.data(), 4 * aoff.size());
   memcpy(hb + o_cu, cu.data(), 4 * cu.size());
+  if (!grpn.empty()) memcpy(hb + o_grpn, grpn.data(), 4 * grpn.size());
+  if (!grpw.empty()) memcpy(hb + o_grpw, grpw.data(), 4 * grpw.size());
 
   const auto t4 = std::chrono::steady_clock::now();
   // ---- device arena + one H2D copy ----
@@ -1189,6 +1303,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->cand_units = (uint32_t *)(db + o_cu);
   c->cand_total = cu[hd.G];
   c->n_mol_tiles = (int)mt.size() - 1;
+  c->grp_narrow = (int32_t *)(db + o_grpn);
+  c->grp_wide = (int32_t *)(db + o_grpw);
+  c->NGN = (int)(grpn.size() / 4);
+  c->NGW = (int)(grpw.size() / 2);
   c->tile_g1 = (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
   c->qp_ent = (const int4 *)(db + o_ent);
@@ -1274,7 +1392,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     // adj_words + 2, + 3 = all zeros (absent non-edge in the induced lane join)
     CUDA_TRY(c, cudaMemsetAsync((uint32_t *)c->adjb.p + c->adj_words, 0xff, 8, c->stream));
     CUDA_TRY(c, cudaMemsetAsync((uint32_t *)c->adjb.p + c->adj_words + 2, 0, 8, c->stream));
-    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, c->induced_loaded, c->adj_off, (uint32_t *)c->adjb.p, c->stream));
+    SIGMO_TRY(dreserve(c, c->nb4, 4 * (size_t)std::max(c->VD, 1), "packed neighbours"));
+    SIGMO_TRY(dreserve(c, c->mrec, 16 * (size_t)std::max(c->ND, 1), "molecule records"));
+    CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, c->adj_off, (uint32_t *)c->adjb.p, (uint32_t *)c->nb4.p, c->stream));
+    CUDA_TRY(c, launch_mrec(c->dd.goff, c->adj_off, c->cand_units, c->ND, (uint4 *)c->mrec.p, c->stream));
   }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
   SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 8), "join counters"));  // + the second claim counter
@@ -1304,26 +1425,13 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
   int launches = 0;
   if (c->ND > 0 && c->VD > 0) {
     const QueryProgMeta &m = prog->meta;
-    // molecule tiles (cmol layout for the per-lane join) unless the
+    // lane path (cmol layout for the per-lane join, k_filter_lane) unless the
     // neighbour-support pass (dense bitmap) is requested
-    bool mol = c->lane_join && !(flags & SIGMO_FILTER_NEIGHBOR_SUPPORT) && c->mol_extn <= 1024;  // one word per lane
-    // tile width: largest TW whose shared memory fits
+    bool mol = c->lane_join && !(flags & SIGMO_FILTER_NEIGHBOR_SUPPORT);
     const int tws[6] = {32, 16, 8, 4, 2, 1};
     int k = 0;
     size_t smem = 0;
     int rows_smem = 1;
-    if (mol) {
-      rows_smem = 1;
-      smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NDR * m.RW, 1,
-                               c->NQW, m.TS, 1, m.NDR, c->NQ, m.NQWL);
-      const char *rg = getenv("SIGMO_FILTER_ROWS_GLOBAL");
-      if (smem > c->max_smem / 2 || (rg && atoi(rg))) {
-        rows_smem = 0;
-        smem = filter_smem_bytes(1, c->mol_extn, c->mol_extw, 32, m.NFU, m.NLAB, m.P, m.NREC, c->VQ, m.NDR * m.RW, 0,
-                                 c->NQW, m.TS, 1, m.NDR, c->NQ, m.NQWL);
-      }
-      if (smem > c->max_smem) mol = false;  // fall back to dense tiles
-    }
     if (!mol && !c->tile_geom_ok) {
       HostGraphs hg;
       hg.G = c->ND;
@@ -1357,48 +1465,6 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       if (c->bm_bytes > used) CUDA_TRY(c, cudaMemsetAsync((char *)c->bitmap.p + used, 0, c->bm_bytes - used, c->stream));
       c->dense_pad_zero = true;
     }
-    FilterParams fp{};
-    fp.D = c->dd;
-    fp.TW = tws[k];
-    fp.W = c->W;
-    fp.Wpad = c->Wpad;
-    fp.VQ = c->VQ;
-    fp.NQ = c->NQ;
-    fp.NQW = c->NQW;
-    fp.R = R;
-    fp.P = m.P;
-    fp.NFU = m.NFU;
-    fp.NLAB = m.NLAB;
-    fp.NREC = m.NREC;
-    fp.NRP = mol ? m.NDR * m.RW : m.NRP;
-    fp.NBATCH = m.NBATCH;
-    fp.RW = m.RW;
-    fp.TS = m.TS;
-    fp.grec = prog->grec;
-    fp.rrec_off = prog->rrec_off;
-    fp.rcarry = prog->rcarry;
-    fp.bdone = prog->bdone;
-    fp.tab = prog->tab;
-    fp.fslot = prog->fslot;
-    fp.lab_val = prog->lab_val;
-    fp.rowp_off = prog->rowp_off;
-    fp.rowp = mol ? prog->drowp : prog->rowp;  // molecule tiles: the distinct rows
-    fp.qgoff = c->dq.goff;
-    fp.bitmap = (uint32_t *)c->bitmap.p;
-    fp.gm = (uint32_t *)c->gm.p;
-    fp.mol_cnt = (I64x2 *)c->mol_cnt.p;
-    fp.EXTN = mol ? c->mol_extn : c->tile_extn[k];
-    fp.EXTW = mol ? c->mol_extw : c->tile_extw[k];
-    fp.MOLCAP = mol ? 32 : c->tile_molcap[k];
-    fp.tile_g0 = (!mol && tws[k] == 32) ? c->tile_g0 : nullptr;
-    fp.tile_g1 = (!mol && tws[k] == 32) ? c->tile_g1 : nullptr;
-    fp.cmol = mol ? (uint32_t *)c->bitmap.p : nullptr;
-    fp.cand_units = c->cand_units;
-    fp.qdrow = prog->qdrow;
-    fp.qw_off = prog->qw_off;
-    fp.qw = prog->qw;
-    fp.NQWL = m.NQWL;
-    fp.NDR = m.NDR;
     if (mol && c->ent_R != R) {
       // distinct-row index of each plan position's query node into the plan entries
       const std::vector<uint16_t> &qd = c->progs[R].qdrow;
@@ -1414,20 +1480,107 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
                                     cudaMemcpyHostToDevice, c->stream));
       c->ent_R = R;
     }
-    fp.rows_smem = rows_smem;
-    fp.smem_bytes = smem;
     if (c->has_empty_graph) {
       CUDA_TRY(c, cudaMemsetAsync(c->gm.p, 0, 4 * (size_t)c->ND * c->NQW, c->stream));
       CUDA_TRY(c, cudaMemsetAsync(c->mol_cnt.p, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
     }
-    const int tiles = mol ? c->n_mol_tiles : (c->W + fp.TW - 1) / fp.TW;
+    if (mol) {
+      FilterLaneParams lp{};
+      lp.NGN = c->NGN;
+      lp.NGW = c->NGW;
+      lp.grp_narrow = c->grp_narrow;
+      lp.grp_wide = c->grp_wide;
+      lp.mrec = (const uint4 *)c->mrec.p;
+      lp.label = c->dd.label;
+      lp.nb4 = (const uint32_t *)c->nb4.p;
+      lp.adjw = (const uint32_t *)c->adjb.p;
+      lp.NB = c->NB;
+      lp.R = R;
+      lp.NLAB = m.NLAB;
+      lp.NFU = m.NFU;
+      lp.NCH = m.NLAB + 1 + m.P;
+      lp.lut = prog->l_lut;
+      lp.grec = prog->l_grec;
+      lp.NREC = m.L_NREC;
+      lp.rrec = prog->l_rrec;
+      lp.rowp = prog->l_rowp;
+      lp.rgn = prog->l_rgn;
+      lp.NDR = m.NDR;
+      lp.RWV = m.L_RWV;
+      lp.qwl = prog->l_qwl;
+      lp.NQWE = m.L_NQWE;
+      lp.qwh = prog->l_qwh;
+      lp.NQG = m.L_NQG;
+      lp.NQ = c->NQ;
+      lp.NQW = c->NQW;
+      lp.cmol = (uint32_t *)c->bitmap.p;
+      lp.gm = (uint32_t *)c->gm.p;
+      lp.mol_cnt = (I64x2 *)c->mol_cnt.p;
+      lp.tables_global = 0;
+      lp.smem_bytes = filter_lane_smem_bytes(lp);
+      const char *tg = getenv("SIGMO_FILTER_TABLES_GLOBAL");  // test knob: tables from global memory
+      if (lp.smem_bytes > c->max_smem / 3 || (tg && atoi(tg))) {
+        lp.tables_global = 1;
+        lp.smem_bytes = filter_lane_smem_bytes(lp);
+      }
+      if (lp.smem_bytes > c->max_smem)
+        return set_err(c, SIGMO_ERR_LIMIT, "lane filter shared memory %zu exceeds %zu", lp.smem_bytes, c->max_smem);
+      const int bps = filter_lane_blocks_per_sm(lp);
+      const int ngroups = c->NGN + c->NGW;
+      const int grid = std::max(1, std::min(bps * c->sm_count, (ngroups + kFilterLaneThreads / 32 - 1) / (kFilterLaneThreads / 32)));
+      if (getenv("SIGMO_DEBUG_FILTER"))
+        fprintf(stderr, "sigmo filter (lane): smem=%zu global=%d NCH=%d NFU=%d NREC=%d NDR=%d RWV=%d NQG=%d NQWE=%d groups=%d+%d grid=%d\n",
+                lp.smem_bytes, lp.tables_global, lp.NCH, lp.NFU, lp.NREC, lp.NDR, lp.RWV, lp.NQG, lp.NQWE, c->NGN, c->NGW, grid);
+      timing_mark(c, 2);
+      CUDA_TRY(c, launch_filter_lane(lp, grid, c->stream));
+      launches++;
+    } else {
+    FilterParams fp{};
+    fp.D = c->dd;
+    fp.TW = tws[k];
+    fp.W = c->W;
+    fp.Wpad = c->Wpad;
+    fp.VQ = c->VQ;
+    fp.NQ = c->NQ;
+    fp.NQW = c->NQW;
+    fp.R = R;
+    fp.P = m.P;
+    fp.NFU = m.NFU;
+    fp.NLAB = m.NLAB;
+    fp.NREC = m.NREC;
+    fp.NRP = m.NRP;
+    fp.NBATCH = m.NBATCH;
+    fp.RW = m.RW;
+    fp.TS = m.TS;
+    fp.grec = prog->grec;
+    fp.rrec_off = prog->rrec_off;
+    fp.rcarry = prog->rcarry;
+    fp.bdone = prog->bdone;
+    fp.tab = prog->tab;
+    fp.fslot = prog->fslot;
+    fp.lab_val = prog->lab_val;
+    fp.rowp_off = prog->rowp_off;
+    fp.rowp = prog->rowp;
+    fp.qgoff = c->dq.goff;
+    fp.bitmap = (uint32_t *)c->bitmap.p;
+    fp.gm = (uint32_t *)c->gm.p;
+    fp.mol_cnt = (I64x2 *)c->mol_cnt.p;
+    fp.EXTN = c->tile_extn[k];
+    fp.EXTW = c->tile_extw[k];
+    fp.MOLCAP = c->tile_molcap[k];
+    fp.tile_g0 = tws[k] == 32 ? c->tile_g0 : nullptr;
+    fp.tile_g1 = tws[k] == 32 ? c->tile_g1 : nullptr;
+    fp.cmol = nullptr;
+    fp.rows_smem = rows_smem;
+    fp.smem_bytes = smem;
+    const int tiles = (c->W + fp.TW - 1) / fp.TW;
     if (getenv("SIGMO_DEBUG_FILTER"))
-      fprintf(stderr, "sigmo filter: mol=%d smem=%zu EXTN=%d EXTW=%d NFU=%d NLAB=%d P=%d NREC=%d TS=%d NDR=%d RW=%d NQWL=%d tiles=%d\n",
-              (int)mol, smem, fp.EXTN, fp.EXTW, m.NFU, m.NLAB, m.P, m.NREC, m.TS, m.NDR, m.RW, m.NQWL, tiles);
-    fp.mtile = c->mol_tiles;
+      fprintf(stderr, "sigmo filter (dense): smem=%zu EXTN=%d EXTW=%d NFU=%d NLAB=%d P=%d NREC=%d TS=%d RW=%d tiles=%d\n",
+              smem, fp.EXTN, fp.EXTW, m.NFU, m.NLAB, m.P, m.NREC, m.TS, m.RW, tiles);
     timing_mark(c, 2);
     CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));
     launches++;
+    }
     if (flags & SIGMO_FILTER_NEIGHBOR_SUPPORT) {
       SupportParams sp{};
       sp.ND = c->ND;

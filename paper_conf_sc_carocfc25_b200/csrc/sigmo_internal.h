@@ -19,6 +19,25 @@ struct I64x2 {
   long long a, b;
 };
 
+// R7 field of an atom label (atomic number): C N O S F Cl Br I P H B Si, other
+__host__ __device__ inline int field_of_label(int lab) {
+  switch (lab) {
+    case 6: return 0;
+    case 7: return 1;
+    case 8: return 2;
+    case 16: return 3;
+    case 9: return 4;
+    case 17: return 5;
+    case 35: return 6;
+    case 53: return 7;
+    case 15: return 8;
+    case 1: return 9;
+    case 5: return 10;
+    case 14: return 11;
+    default: return 12;
+  }
+}
+
 // Packed CSR-GO batch on the device (produced by sigmo_load_batch).
 //   nbr[e] = (molecule-local index of the neighbour << 8) | bond label
 struct DevGraphs {
@@ -46,6 +65,11 @@ struct QueryProgMeta {
   int RW;      // row-program words per query node (padded)
   int NDR;     // distinct rows (query nodes with the same label and constraint list share one)
   int NQWL;    // (word, bits) entries of the per-query GMCR lists over distinct rows
+  // k_filter_lane program (FilterLaneParams)
+  int L_NREC;  // plane records (<= 4 planes each)
+  int L_RWV;   // uint4 words per distinct row program
+  int L_NQWE;  // GMCR list entries x 32
+  int L_NQG;   // 32-query groups
 };
 
 // One part of a (radius, field) count group inside one 32-plane batch of the
@@ -83,6 +107,14 @@ struct QueryProg {
   int32_t *qw_off = nullptr;   // [NQ+1] per-query range of (word, bits) entries
   uint32_t *qw = nullptr;      // [NQWL][2] word of the distinct-row bit vector, bits of the query's rows in it
   QueryProgMeta *d_meta = nullptr;
+  // k_filter_lane program (see FilterLaneParams)
+  uint2 *l_grec = nullptr;
+  int32_t *l_rrec = nullptr;
+  uint4 *l_rowp = nullptr;
+  int32_t *l_rgn = nullptr;
+  uint2 *l_qwl = nullptr;
+  int2 *l_qwh = nullptr;
+  uint16_t *l_lut = nullptr;
 };
 
 struct FilterParams {
@@ -198,6 +230,38 @@ struct ChunkParams {
   int32_t *nchunks;
 };
 
+// k_filter_lane (sigmo_filter_lane.cu): the filter of the lane-join path.
+// Groups of 4 slots of 32 nodes: narrow groups = 4 molecules of <= 32 atoms,
+// wide groups = 2 molecules of 33-64 atoms.  Channels of the per-warp plane
+// array: 0..NLAB-1 label planes, NLAB all ones, NLAB+1+p constraint plane p.
+constexpr int kFilterLaneThreads = 256;
+struct FilterLaneParams {
+  int NGN, NGW;                 // narrow / wide groups
+  const int32_t *grp_narrow;    // [4 NGN] molecule ids (-1 = empty slot)
+  const int32_t *grp_wide;      // [2 NGW]
+  const uint4 *mrec;            // [ND] {first node, atoms, adjacency word offset, candidate units}
+  const uint8_t *label;         // [VD]
+  const uint32_t *nb4;          // [VD] first <= 4 neighbours (molecule-local ids, filler = self; bit 7: degree > 4)
+  const uint32_t *adjw;         // bond-class adjacency, class NB = all bonds (slow path of degree > 4 nodes)
+  int NB, R, NLAB, NFU, NCH;
+  const uint16_t *lut;          // [256] label -> label channel (0xff none) | field slot << 8 (0xff unused)
+  const uint2 *grec;            // [NREC] plane records: x = field slot | #planes (<= 4) << 8 | first channel << 16,
+  int NREC;                     //        y = thresholds (bytes), sorted by radius
+  const int32_t *rrec;          // [R+1] record range per radius
+  const uint4 *rowp;            // [NDR][RWV] row programs: pairs of 16-bit channel byte offsets (x16), all-ones padded
+  const int32_t *rgn;           // [ceil(NDR/32)] channel-pair words needed by each 32-row group (rows sorted by length)
+  int NDR, RWV;
+  const uint2 *qwl;             // GMCR lists [entries][32 lanes] (word, bits), (0, 0) padded
+  int NQWE;                     // entries x 32
+  const int2 *qwh;              // [NQG] {first entry, entries} per 32-query group
+  int NQG, NQ, NQW;
+  uint32_t *cmol;               // molecule-padded windows (FilterParams::cmol)
+  uint32_t *gm;                 // [ND][NQW]
+  I64x2 *mol_cnt;               // [ND+1]
+  int tables_global;            // 1: row programs and GMCR lists read from global memory (too large for smem)
+  size_t smem_bytes;
+};
+
 // ---- launchers (sigmo_kernels.cu); all enqueue on `st` ----
 cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, cudaStream_t st);
 cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *out, cudaStream_t st);
@@ -215,7 +279,12 @@ cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
 cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
                          int VQ, int Wpad, uint32_t *dense,
                          cudaStream_t st);
-cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, int induced, const uint32_t *adj_off, uint32_t *adjw,
+cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
+                        uint32_t *nb4, cudaStream_t st);
+cudaError_t launch_filter_lane(const FilterLaneParams &p, int grid, cudaStream_t st);
+size_t filter_lane_smem_bytes(const FilterLaneParams &p);
+int filter_lane_blocks_per_sm(const FilterLaneParams &p);
+cudaError_t launch_mrec(const int32_t *goff, const uint32_t *adj_off, const uint32_t *cand_units, int ND, uint4 *mrec,
                         cudaStream_t st);
 cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, cudaStream_t st);
 size_t join_lane_smem_bytes(const JoinParams &p, bool w64);

@@ -1101,7 +1101,6 @@ cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStre
     break;
   switch (NW * 2 + (p.cmol ? 1 : 0)) {
     SIGMO_FILTER_CASE(1, 0)
-    SIGMO_FILTER_CASE(1, 1)
     SIGMO_FILTER_CASE(2, 0)
     SIGMO_FILTER_CASE(4, 0)
     default: return cudaErrorInvalidValue;
@@ -1937,15 +1936,15 @@ cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const
 // holding v, so that lanes reading the same class of one molecule touch few
 // 32-B sectors.
 // ===========================================================================
-__global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, int induced, const uint32_t *adj_off,
-                       uint32_t *adjw) {
+__global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
+                       uint32_t *nb4) {
   const int v = blockIdx.x * blockDim.x + threadIdx.x;
   if (v >= d.num_nodes) return;
   unsigned long long m[8], mall = 0ull;
 #pragma unroll
   for (int b = 0; b < 8; b++) m[b] = 0ull;
-  const int e1 = d.roff[v + 1];
-  for (int e = d.roff[v]; e < e1; e++) {
+  const int e0 = d.roff[v], e1 = d.roff[v + 1];
+  for (int e = e0; e < e1; e++) {
     const int x = d.nbr[e];
     const int cls = bclass[x & 255];
 #pragma unroll
@@ -1962,16 +1961,28 @@ __global__ void k_adjb(DevGraphs d, const uint8_t *bclass, int NB, int induced, 
       if (n <= 32) adjw[base + (uint32_t)(b * n + (v - a))] = (uint32_t)m[b];
       else *(unsigned long long *)(adjw + base + 2u * (uint32_t)(b * n + (v - a))) = m[b];
     }
-  if (induced) {  // class NB: every bond, whatever its label (induced mode, R21)
-    if (n <= 32) adjw[base + (uint32_t)(NB * n + (v - a))] = (uint32_t)mall;
-    else *(unsigned long long *)(adjw + base + 2u * (uint32_t)(NB * n + (v - a))) = mall;
+  // class NB: every bond, whatever its label (k_filter_lane's slow path for
+  // degree > 4, the induced lane join, R21)
+  if (n <= 32) adjw[base + (uint32_t)(NB * n + (v - a))] = (uint32_t)mall;
+  else *(unsigned long long *)(adjw + base + 2u * (uint32_t)(NB * n + (v - a))) = mall;
+  // nb4: the first <= 4 neighbours (molecule-local ids, byte k), unused bytes
+  // = the node itself, bit 7 of byte 0 set when the degree exceeds 4
+  const uint32_t self = (uint32_t)(v - a) & 63u;
+  uint32_t w = self * 0x01010101u;
+  unsigned long long rest = mall;
+  for (int k = 0; k < 4 && rest; k++) {
+    const uint32_t u = (uint32_t)(__ffsll((long long)rest) - 1);
+    rest &= rest - 1ull;
+    w = (w & ~(0xffu << (8 * k))) | (u << (8 * k));
   }
+  if (rest) w |= 0x80u;
+  nb4[v] = w;
 }
 
-cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, int induced, const uint32_t *adj_off,
-                        uint32_t *adjw, cudaStream_t st) {
-  if (d.num_nodes <= 0 || NB <= 0) return cudaSuccess;
-  k_adjb<<<(d.num_nodes + 255) / 256, 256, 0, st>>>(d, bclass, NB, induced, adj_off, adjw);
+cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
+                        uint32_t *nb4, cudaStream_t st) {
+  if (d.num_nodes <= 0) return cudaSuccess;
+  k_adjb<<<(d.num_nodes + 255) / 256, 256, 0, st>>>(d, bclass, NB, adj_off, adjw, nb4);
   return cudaGetLastError();
 }
 
