@@ -689,11 +689,13 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   }
   qw_off[NQ] = (int32_t)(qw.size() / 2);
   // ---- k_filter_lane program (FilterLaneParams) ----
-  // plane records: per (radius, field) group, chunks of <= 4 planes
+  // plane records: per (radius, field) group, chunks of <= 4 planes; per
+  // radius sorted by plane count (k_filter_lane runs the four counts as
+  // separate loops): lrrec[4 r0 + k] = first record of radius r0 with k + 1 planes
   std::vector<uint2> lrec;
-  std::vector<int32_t> lrrec((size_t)R + 1, 0);
+  std::vector<int32_t> lrrec((size_t)4 * R + 1, 0);
   for (int r0 = 0; r0 < R; r0++) {
-    lrrec[r0] = (int)lrec.size();
+    std::vector<uint2> byn[4];
     for (int g = rg_off[r0]; g < rg_off[r0 + 1]; g++)
       for (int p = grp_poff[g]; p < grp_poff[g + 1]; p += 4) {
         const int np = std::min(4, grp_poff[g + 1] - p);
@@ -701,10 +703,14 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
         e.x = (uint32_t)(uint8_t)fslot[grp_f[g]] | ((uint32_t)np << 8) | ((uint32_t)(NLAB + 1 + p) << 16);
         e.y = 0;
         for (int j = 0; j < np; j++) e.y |= (uint32_t)p_t[p + j] << (8 * j);
-        lrec.push_back(e);
+        byn[np - 1].push_back(e);
       }
+    for (int k = 0; k < 4; k++) {
+      lrrec[4 * r0 + k] = (int)lrec.size();
+      lrec.insert(lrec.end(), byn[k].begin(), byn[k].end());
+    }
   }
-  lrrec[R] = (int)lrec.size();
+  lrrec[4 * R] = (int)lrec.size();
   // row programs: channel byte offsets (x16: [channel][4 slots] u32), pairs
   // per u32, 4 u32 per uint4, padded with the all-ones channel
   int maxch = 1;

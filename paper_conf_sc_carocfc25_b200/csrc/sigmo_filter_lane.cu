@@ -53,7 +53,7 @@ __host__ __device__ inline LaneFilterLayout lane_filter_layout(const FilterLaneP
   L.qwl = o;  o = lf_align16(o + (p.tables_global ? 0 : 8 * (size_t)p.NQWE));
   L.qwh = o;  o = lf_align16(o + 8 * (size_t)(p.NQG > 0 ? p.NQG : 1));
   L.lut = o;  o = lf_align16(o + 2 * 256);
-  L.rrec = o; o = lf_align16(o + 4 * (size_t)(kMaxRadius + 1));
+  L.rrec = o; o = lf_align16(o + 4 * (size_t)(4 * kMaxRadius + 1));
   L.warps = o;
   size_t w = 0;
   L.w_planes = w; w = lf_align16(w + 16 * (size_t)p.NCH);
@@ -73,6 +73,60 @@ __device__ __forceinline__ void and4(uint4 &a, const uint4 b) {
   a.y &= b.y;
   a.z &= b.z;
   a.w &= b.w;
+}
+
+// threshold planes of the records [e0, e1), each with exactly NP planes:
+// c = |ball_r(v) \ {v}| in the record's field, plane word = ballot(c >= t)
+// per slot, stored as [channel][4 slots] (every lane stores the same value:
+// one unpredicated 128-bit shared store)
+template <bool WIDE, int NP, typename BT>
+__device__ __forceinline__ void plane_records(int e0, int e1, const uint2 *grec, const unsigned char *wfm,
+                                              unsigned char *wpl, const BT (&bx)[4]) {
+  for (int e = e0; e < e1; e++) {
+    // record: x = field slot | #planes << 8 | first plane channel << 16, y = thresholds (bytes)
+    const uint2 g = grec[e];
+    const uint4 fm = lds128(wfm + 16 * (g.x & 0xffu));
+    int c[4];
+    if constexpr (WIDE) {
+      const unsigned long long f0 = (unsigned long long)fm.x | ((unsigned long long)fm.y << 32);
+      const unsigned long long f1 = (unsigned long long)fm.z | ((unsigned long long)fm.w << 32);
+      c[0] = __popcll((unsigned long long)bx[0] & f0);
+      c[1] = __popcll((unsigned long long)bx[1] & f0);
+      c[2] = __popcll((unsigned long long)bx[2] & f1);
+      c[3] = __popcll((unsigned long long)bx[3] & f1);
+    } else {
+      c[0] = __popc((unsigned)bx[0] & fm.x);
+      c[1] = __popc((unsigned)bx[1] & fm.y);
+      c[2] = __popc((unsigned)bx[2] & fm.z);
+      c[3] = __popc((unsigned)bx[3] & fm.w);
+    }
+    unsigned char *pp = wpl + 16 * (g.x >> 16);
+#pragma unroll
+    for (int j = 0; j < NP; j++) {
+      const int t = (int)((g.y >> (8 * j)) & 0xffu);
+      uint4 w;
+      w.x = __ballot_sync(LF_FULL, c[0] >= t);
+      w.y = __ballot_sync(LF_FULL, c[1] >= t);
+      w.z = __ballot_sync(LF_FULL, c[2] >= t);
+      w.w = __ballot_sync(LF_FULL, c[3] >= t);
+      *(uint4 *)(pp + 16 * j) = w;
+    }
+  }
+}
+
+// 32x32 bit-matrix transpose across the warp: lane L holds row L (bit p =
+// element (L, p)); returns column `lane` (bit L = element (L, lane))
+__device__ __forceinline__ unsigned lf_transpose32(unsigned x, int lane) {
+#pragma unroll
+  for (int j = 16; j >= 1; j >>= 1) {
+    const unsigned m = j == 16 ? 0x0000ffffu : j == 8 ? 0x00ff00ffu : j == 4 ? 0x0f0f0f0fu : j == 2 ? 0x33333333u
+                                                                                               : 0x55555555u;
+    const unsigned sw = ((x << j) & ~m) | ((x >> j) & m);
+    const unsigned y = __shfl_xor_sync(LF_FULL, sw, j);
+    const unsigned K = (lane & j) ? ~m : m;
+    x = (x & K) | (y & ~K);
+  }
+  return x;
 }
 
 // one group of 4 slots.  WIDE: 2 molecules of 33-64 atoms (slots 2m + h =
@@ -128,23 +182,40 @@ __device__ __forceinline__ void lane_filter_group(const FilterLaneParams &fp, in
       nb[k] = __ldg(fp.nb4 + mr[m].x + v);
     }
   }
-  // label planes (channels 0..NLAB-1) and field masks, one ballot per slot
-  for (int c = 0; c < fp.NLAB; c++) {
-    uint4 w;
-    w.x = __ballot_sync(LF_FULL, (lt[0] & 0xffu) == (unsigned)c);
-    w.y = __ballot_sync(LF_FULL, (lt[1] & 0xffu) == (unsigned)c);
-    w.z = __ballot_sync(LF_FULL, (lt[2] & 0xffu) == (unsigned)c);
-    w.w = __ballot_sync(LF_FULL, (lt[3] & 0xffu) == (unsigned)c);
-    if (lane == 0) *(uint4 *)(wpl + 16 * c) = w;
+  // label planes (channels 0..NLAB-1) and field masks [NFU][4 slots]
+  if (fp.NLAB + fp.NFU <= 32) {
+    // per slot, lane = node builds its one-hot word (bit c: label channel c,
+    // bit NLAB + f: field slot f); a warp transpose turns it into lane = channel
+    unsigned tw[4];
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const unsigned lc = lt[k] & 0xffu, fs = lt[k] >> 8;
+      unsigned mb = lc < 32u ? 1u << lc : 0u;
+      mb |= fs < 32u ? 1u << ((unsigned)fp.NLAB + fs) : 0u;
+      tw[k] = lf_transpose32(mb, lane);
+    }
+    const uint4 w = make_uint4(tw[0], tw[1], tw[2], tw[3]);
+    if (lane < fp.NLAB) *(uint4 *)(wpl + 16 * lane) = w;
+    else if (lane < fp.NLAB + fp.NFU) *(uint4 *)(wfm + 16 * (lane - fp.NLAB)) = w;
+  } else {
+    for (int c = 0; c < fp.NLAB; c++) {
+      uint4 w;
+      w.x = __ballot_sync(LF_FULL, (lt[0] & 0xffu) == (unsigned)c);
+      w.y = __ballot_sync(LF_FULL, (lt[1] & 0xffu) == (unsigned)c);
+      w.z = __ballot_sync(LF_FULL, (lt[2] & 0xffu) == (unsigned)c);
+      w.w = __ballot_sync(LF_FULL, (lt[3] & 0xffu) == (unsigned)c);
+      *(uint4 *)(wpl + 16 * c) = w;
+    }
+    for (int f = 0; f < fp.NFU; f++) {
+      uint4 w;
+      w.x = __ballot_sync(LF_FULL, (lt[0] >> 8) == (unsigned)f);
+      w.y = __ballot_sync(LF_FULL, (lt[1] >> 8) == (unsigned)f);
+      w.z = __ballot_sync(LF_FULL, (lt[2] >> 8) == (unsigned)f);
+      w.w = __ballot_sync(LF_FULL, (lt[3] >> 8) == (unsigned)f);
+      *(uint4 *)(wfm + 16 * f) = w;
+    }
   }
-  for (int f = 0; f < fp.NFU; f++) {
-    uint4 w;
-    w.x = __ballot_sync(LF_FULL, (lt[0] >> 8) == (unsigned)f);
-    w.y = __ballot_sync(LF_FULL, (lt[1] >> 8) == (unsigned)f);
-    w.z = __ballot_sync(LF_FULL, (lt[2] >> 8) == (unsigned)f);
-    w.w = __ballot_sync(LF_FULL, (lt[3] >> 8) == (unsigned)f);
-    if (lane == 0) *(uint4 *)(wfm + 16 * f) = w;
-  }
+  __syncwarp();
 
   // ---- radii 1..R: BFS + threshold planes ----
   // balls: narrow u32 (bit = node of the molecule), wide u64
@@ -233,40 +304,12 @@ __device__ __forceinline__ void lane_filter_group(const FilterLaneParams &fp, in
       bx[k] = ball[k] & ~((BT)1 << v);
     }
     __syncwarp();
-    const int e1 = rrec[r];
-    for (int e = rrec[r - 1]; e < e1; e++) {
-      // record: x = field slot | #planes << 8 | first plane channel << 16, y = thresholds (bytes)
-      const uint2 g = grec[e];
-      const uint4 fm = lds128(wfm + 16 * (g.x & 0xffu));
-      int c[4];
-      if constexpr (WIDE) {
-        const unsigned long long f0 = (unsigned long long)fm.x | ((unsigned long long)fm.y << 32);
-        const unsigned long long f1 = (unsigned long long)fm.z | ((unsigned long long)fm.w << 32);
-        c[0] = __popcll((unsigned long long)bx[0] & f0);
-        c[1] = __popcll((unsigned long long)bx[1] & f0);
-        c[2] = __popcll((unsigned long long)bx[2] & f1);
-        c[3] = __popcll((unsigned long long)bx[3] & f1);
-      } else {
-        c[0] = __popc((unsigned)bx[0] & fm.x);
-        c[1] = __popc((unsigned)bx[1] & fm.y);
-        c[2] = __popc((unsigned)bx[2] & fm.z);
-        c[3] = __popc((unsigned)bx[3] & fm.w);
-      }
-      const int np = (int)((g.x >> 8) & 0xffu);
-      unsigned char *pp = wpl + 16 * (g.x >> 16);
-#pragma unroll
-      for (int j = 0; j < 4; j++) {
-        if (j < np) {
-          const int t = (int)((g.y >> (8 * j)) & 0xffu);
-          uint4 w;
-          w.x = __ballot_sync(LF_FULL, c[0] >= t);
-          w.y = __ballot_sync(LF_FULL, c[1] >= t);
-          w.z = __ballot_sync(LF_FULL, c[2] >= t);
-          w.w = __ballot_sync(LF_FULL, c[3] >= t);
-          if (lane == 0) *(uint4 *)(pp + 16 * j) = w;
-        }
-      }
-    }
+    // records of radius r, in four runs of 1, 2, 3, 4 planes (no per-plane branches)
+    const int *rr = rrec + 4 * (r - 1);
+    plane_records<WIDE, 1>(rr[0], rr[1], grec, wfm, wpl, bx);
+    plane_records<WIDE, 2>(rr[1], rr[2], grec, wfm, wpl, bx);
+    plane_records<WIDE, 3>(rr[2], rr[3], grec, wfm, wpl, bx);
+    plane_records<WIDE, 4>(rr[3], rr[4], grec, wfm, wpl, bx);
   }
   __syncwarp();
 
@@ -291,19 +334,22 @@ __device__ __forceinline__ void lane_filter_group(const FilterLaneParams &fp, in
       const uint4 *pr = rowp + (size_t)row * RWV;
       for (int q = 0; q < nw; q += 4) {
         const uint4 pw = pr[q >> 2];
-        and4(acc, lds128(wpl + (pw.x & 0xffffu)));
-        and4(acc, lds128(wpl + (pw.x >> 16)));
-        if (q + 1 < nw) {
-          and4(acc, lds128(wpl + (pw.y & 0xffffu)));
-          and4(acc, lds128(wpl + (pw.y >> 16)));
-        }
-        if (q + 2 < nw) {
-          and4(acc, lds128(wpl + (pw.z & 0xffffu)));
-          and4(acc, lds128(wpl + (pw.z >> 16)));
-        }
-        if (q + 3 < nw) {
-          and4(acc, lds128(wpl + (pw.w & 0xffffu)));
-          and4(acc, lds128(wpl + (pw.w >> 16)));
+        switch (nw - q) {  // uniform across the warp: rows are sorted by length
+          default:
+            and4(acc, lds128(wpl + (pw.w & 0xffffu)));
+            and4(acc, lds128(wpl + (pw.w >> 16)));
+            [[fallthrough]];
+          case 3:
+            and4(acc, lds128(wpl + (pw.z & 0xffffu)));
+            and4(acc, lds128(wpl + (pw.z >> 16)));
+            [[fallthrough]];
+          case 2:
+            and4(acc, lds128(wpl + (pw.y & 0xffffu)));
+            and4(acc, lds128(wpl + (pw.y >> 16)));
+            [[fallthrough]];
+          case 1:
+            and4(acc, lds128(wpl + (pw.x & 0xffffu)));
+            and4(acc, lds128(wpl + (pw.x >> 16)));
         }
       }
       const unsigned ro = OS * (unsigned)row;
@@ -323,7 +369,7 @@ __device__ __forceinline__ void lane_filter_group(const FilterLaneParams &fp, in
       ne.z |= ne.w;
       ne.w = ne.z;
     }
-    if (lane == 0) *(uint4 *)(wdz + 16 * rg) = ne;
+    *(uint4 *)(wdz + 16 * rg) = ne;
   }
   __syncwarp();
 
@@ -391,7 +437,7 @@ __global__ void __launch_bounds__(kFilterLaneThreads) k_filter_lane(const __grid
     uint16_t *lu = (uint16_t *)(smem + L.lut);
     for (int i = tid; i < 256; i += kFilterLaneThreads) lu[i] = __ldg(&fp.lut[i]);
     int32_t *rr = (int32_t *)(smem + L.rrec);
-    for (int i = tid; i <= fp.R; i += kFilterLaneThreads) rr[i] = __ldg(&fp.rrec[i]);
+    for (int i = tid; i <= 4 * fp.R; i += kFilterLaneThreads) rr[i] = __ldg(&fp.rrec[i]);
   }
   unsigned char *wsm = smem + L.warps + (size_t)wid * L.w_total;
   // the all-ones channel NLAB (row padding and label-less rows never read it otherwise)

@@ -247,7 +247,7 @@ struct FilterLaneParams {
   const uint16_t *lut;          // [256] label -> label channel (0xff none) | field slot << 8 (0xff unused)
   const uint2 *grec;            // [NREC] plane records: x = field slot | #planes (<= 4) << 8 | first channel << 16,
   int NREC;                     //        y = thresholds (bytes), sorted by radius
-  const int32_t *rrec;          // [R+1] record range per radius
+  const int32_t *rrec;          // [4R+1] record ranges: radius r, k+1 planes at [rrec[4(r-1)+k], rrec[4(r-1)+k+1])
   const uint4 *rowp;            // [NDR][RWV] row programs: pairs of 16-bit channel byte offsets (x16), all-ones padded
   const int32_t *rgn;           // [ceil(NDR/32)] channel-pair words needed by each 32-row group (rows sorted by length)
   int NDR, RWV;
