@@ -117,6 +117,8 @@ typedef struct {
   int64_t filter_calls, join_calls;        /* calls averaged */
   int64_t dfs_steps;    /* DFS iterator steps (search-tree nodes) of the last join */
   int64_t dfs_iters, dfs_tail_iters, dfs_max_stack;  /* warp iterations, of which after the last pair claim; max stack */
+  int64_t filter_jit;   /* 1 if the last lane-path filter ran the kernel specialised for the query program (NVRTC) */
+  double jit_compile_ms; /* wall time of the last specialisation compile (0 if served from the process cache) */
 } sigmo_timings;
 
 /* Create a context on `device` (CUDA ordinal) enqueuing on `cuda_stream`

@@ -46,7 +46,8 @@ class sigmo_timings(ctypes.Structure):
                 ("filter_launches", ctypes.c_int64), ("join_launches", ctypes.c_int64),
                 ("h2d_bytes", ctypes.c_int64), ("filter_calls", ctypes.c_int64),
                 ("join_calls", ctypes.c_int64), ("dfs_steps", ctypes.c_int64),
-                ("dfs_iters", ctypes.c_int64), ("dfs_tail_iters", ctypes.c_int64), ("dfs_max_stack", ctypes.c_int64)]
+                ("dfs_iters", ctypes.c_int64), ("dfs_tail_iters", ctypes.c_int64), ("dfs_max_stack", ctypes.c_int64),
+                ("filter_jit", ctypes.c_int64), ("jit_compile_ms", ctypes.c_double)]
 
 
 _lib = None

@@ -8,8 +8,21 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libsigmo.so")
-SOURCES = ["sigmo_abi.cu", "sigmo_kernels.cu", "sigmo_filter_lane.cu"]
-HEADERS = ["sigmo_internal.h", os.path.join("..", "..", "include", "sigmo.h")]
+SOURCES = ["sigmo_abi.cu", "sigmo_kernels.cu", "sigmo_filter_lane.cu", "sigmo_jit.cu"]
+HEADERS = ["sigmo_internal.h", "lane_filter_types.h", "lane_filter_body.cuh", os.path.join("..", "..", "include", "sigmo.h")]
+# headers embedded as raw strings for the NVRTC-specialised filter (sigmo_jit.cu)
+EMBED = ["lane_filter_types.h", "lane_filter_body.cuh"]
+
+
+def _embed() -> None:
+    for h in EMBED:
+        src = open(os.path.join(CSRC, h)).read()
+        assert ")SIGMOSRC" not in src
+        inc = os.path.join(CSRC, h.rsplit(".", 1)[0] + ".inc")
+        body = 'R"SIGMOSRC(' + src + ')SIGMOSRC"\n'
+        if not os.path.exists(inc) or open(inc).read() != body:
+            with open(inc, "w") as f:
+                f.write(body)
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
               "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-shared", "-cudart", "static",
@@ -27,6 +40,7 @@ def _stale() -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not _stale():
         return LIB
+    _embed()
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
     objs = []
     for src in SOURCES:
@@ -38,7 +52,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         objs.append(obj)
     tmp = LIB + ".tmp"
     subprocess.check_call([nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-cudart", "static",
-                           "-Xcompiler", "-fPIC", *objs, "-o", tmp])
+                           "-Xcompiler", "-fPIC", *objs, "-o", tmp, "-ldl"])
     os.replace(tmp, LIB)
     return LIB
 

@@ -59,6 +59,7 @@ struct ProgCache {
   QueryProg prog;
   DBuf buf, pack;  // device program arrays; packed form for k_filter
   std::vector<uint16_t> qdrow;  // host copy of prog.qdrow
+  LaneJitSpec jit;              // the k_filter_lane program (host copy) for the NVRTC-specialised kernel
   bool valid = false;
 };
 
@@ -169,6 +170,7 @@ struct sigmo_ctx {
 
   Timing timing;
   sigmo_timings last{};
+  std::string jit_note;  // last lane-filter specialisation outcome ("compiled", "cached" or why not)
 };
 
 namespace {
@@ -811,6 +813,19 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
   P.l_qwh = (int2 *)(db + o_lqh);
   P.l_qwl = (uint2 *)(db + o_lql);
   P.l_lut = (uint16_t *)(db + o_llu);
+  pc.jit = LaneJitSpec();
+  pc.jit.NLAB = NLAB;
+  pc.jit.NFU = m.NFU;
+  pc.jit.R = R;
+  pc.jit.NDR = NDR;
+  pc.jit.RWV = LRWV;
+  pc.jit.NQG = NQG;
+  pc.jit.NQ = NQ;
+  pc.jit.NQW = c->NQW;
+  pc.jit.recs.resize((size_t)R);
+  for (int r0 = 0; r0 < R; r0++) pc.jit.recs[r0].assign(lrec.begin() + lrrec[4 * r0], lrec.begin() + lrrec[4 * r0 + 4]);
+  pc.jit.rgn.assign(lrgn.begin(), lrgn.begin() + NDRW);
+  pc.jit.qwh.assign(lqwh.begin(), lqwh.begin() + NQG);
   P.meta.L_NREC = (int)lrec.size();
   P.meta.L_RWV = LRWV;
   P.meta.L_NQWE = (int)lqwl.size();
@@ -1531,14 +1546,31 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       }
       if (lp.smem_bytes > c->max_smem)
         return set_err(c, SIGMO_ERR_LIMIT, "lane filter shared memory %zu exceeds %zu", lp.smem_bytes, c->max_smem);
-      const int bps = filter_lane_blocks_per_sm(lp);
+      // the program-specialised kernel (NVRTC, cached per process) unless
+      // disabled (SIGMO_FILTER_JIT=0) or unavailable; the generic one otherwise
+      cudaKernel_t jk = nullptr;
+      const char *je = getenv("SIGMO_FILTER_JIT");
+      if (!(je && atoi(je) == 0)) {
+        LaneJitSpec &js = c->progs[R].jit;
+        js.GL = lp.tables_global != 0;
+        std::string why;
+        double cms = 0.0;
+        jk = lane_jit_kernel(js, &why, &cms);
+        c->jit_note = jk ? (cms > 0.0 ? "compiled" : "cached") : why;
+        if (cms > 0.0) c->last.jit_compile_ms = cms;
+        if (!jk && getenv("SIGMO_DEBUG_FILTER")) fprintf(stderr, "sigmo filter: JIT unavailable: %s\n", why.c_str());
+      }
+      c->last.filter_jit = jk ? 1 : 0;
+      const int bps = jk ? filter_lane_jit_blocks_per_sm(jk, lp) : filter_lane_blocks_per_sm(lp);
       const int ngroups = c->NGN + c->NGW;
       const int grid = std::max(1, std::min(bps * c->sm_count, (ngroups + kFilterLaneThreads / 32 - 1) / (kFilterLaneThreads / 32)));
       if (getenv("SIGMO_DEBUG_FILTER"))
-        fprintf(stderr, "sigmo filter (lane): smem=%zu global=%d NCH=%d NFU=%d NREC=%d NDR=%d RWV=%d NQG=%d NQWE=%d groups=%d+%d grid=%d\n",
-                lp.smem_bytes, lp.tables_global, lp.NCH, lp.NFU, lp.NREC, lp.NDR, lp.RWV, lp.NQG, lp.NQWE, c->NGN, c->NGW, grid);
+        fprintf(stderr, "sigmo filter (lane%s): smem=%zu global=%d NCH=%d NFU=%d NREC=%d NDR=%d RWV=%d NQG=%d NQWE=%d groups=%d+%d grid=%d\n",
+                jk ? ", specialised" : "", lp.smem_bytes, lp.tables_global, lp.NCH, lp.NFU, lp.NREC, lp.NDR, lp.RWV, lp.NQG,
+                lp.NQWE, c->NGN, c->NGW, grid);
       timing_mark(c, 2);
-      CUDA_TRY(c, launch_filter_lane(lp, grid, c->stream));
+      if (jk) CUDA_TRY(c, launch_filter_lane_jit(jk, lp, grid, c->stream));
+      else CUDA_TRY(c, launch_filter_lane(lp, grid, c->stream));
       launches++;
     } else {
     FilterParams fp{};

@@ -1,456 +1,12 @@
-// sigmo_filter_lane.cu -- the filter of the lane-join path (every data graph
-// <= 64 atoms, every query <= kJoinLaneMaxQ nodes): InitializeCandidates
-// (Alg. 1 l.29-37), GenerateSignatures (l.11-18, read
-// as cumulative counts R4, saturated R8), RefineCandidates (l.19-28,
-// P:580-591, per field R5) for every level at once, and the GMCR mapping test
-// (section 4.5), writing each candidate window once.
-//
-// B200 design ("k_filter_lane"):
-//   * one warp per GROUP of 4 slots, persistent CTAs.  A slot is 32 data
-//     nodes: a narrow group holds 4 molecules of <= 32 atoms (slot k =
-//     molecule k), a wide group 2 molecules of 33-64 atoms (slots 2m, 2m+1 =
-//     nodes 0-31 / 32-63 of molecule m).  Lane = node inside the slot.  The
-//     4 slots run as SIMD lanes of one instruction stream: every decode of
-//     the query program (plane records, row programs, GMCR lists) is paid
-//     once per 4 slots.
-//   * signatures: bitset BFS, ball_r(v) = ball_{r-1}(v) | OR_{u in N(v)}
-//     ball_{r-1}(u), gathered with warp shuffles over the <= 4 packed
-//     neighbour ids of the node (nb4, written at load); count of field f at
-//     radius r = popc(ball_r(v) \ {v} & fieldmask_f).
-//   * planes: plane p = (r, f, t) is the 32-bit word [count_{r,f}(v) >= t]
-//     of a slot, one ballot per (plane, slot); label planes likewise; kept in
-//     the warp's shared memory as [channel][4 slots].
-//   * rows (lane = distinct row): window = AND of the row's channels, one
-//     128-bit shared load per channel for the 4 slots; stored once to
-//     cmol[g][row] (coalesced: lanes = consecutive rows of one molecule).
-//   * GMCR (lane = query): a query survives in molecule g iff each of its
-//     distinct rows has a non-empty window, tested from the per-slot
-//     non-empty ballots through the query's (word, bits) list.
-#include <type_traits>
-
+// sigmo_filter_lane.cu -- the generic (table-driven) build of the lane-path
+// filter kernel (device code in lane_filter_body.cuh) and its launchers.  The
+// NVRTC-specialised build of the same body is in sigmo_jit.cu.
 #include "sigmo_internal.h"
+#include "lane_filter_body.cuh"
 
 namespace sigmo {
 
-#define LF_FULL 0xffffffffu
-
-__host__ __device__ inline size_t lf_align16(size_t x) { return (x + 15) & ~(size_t)15; }
-
-// shared-memory layout: CTA tables, then one region per warp
-struct LaneFilterLayout {
-  size_t rowp, rgn, grec, qwl, qwh, lut, rrec, warps;
-  size_t w_planes, w_fm, w_dnz, w_ball, w_total;
-  size_t total;
-};
-
-__host__ __device__ inline LaneFilterLayout lane_filter_layout(const FilterLaneParams &p) {
-  LaneFilterLayout L;
-  const int NDRW = (p.NDR + 31) / 32;
-  size_t o = 0;
-  L.rowp = o; o = lf_align16(o + (p.tables_global ? 0 : 16 * (size_t)p.NDR * p.RWV));
-  L.rgn = o;  o = lf_align16(o + 4 * (size_t)NDRW);
-  L.grec = o; o = lf_align16(o + 8 * (size_t)(p.NREC > 0 ? p.NREC : 1));
-  L.qwl = o;  o = lf_align16(o + (p.tables_global ? 0 : 8 * (size_t)p.NQWE));
-  L.qwh = o;  o = lf_align16(o + 8 * (size_t)(p.NQG > 0 ? p.NQG : 1));
-  L.lut = o;  o = lf_align16(o + 2 * 256);
-  L.rrec = o; o = lf_align16(o + 4 * (size_t)(4 * kMaxRadius + 1));
-  L.warps = o;
-  size_t w = 0;
-  L.w_planes = w; w = lf_align16(w + 16 * (size_t)p.NCH);
-  L.w_fm = w;     w = lf_align16(w + 16 * (size_t)(p.NFU > 0 ? p.NFU : 1));
-  L.w_dnz = w;    w = lf_align16(w + 16 * (size_t)NDRW);
-  L.w_ball = w;   w = lf_align16(w + 8 * 64 * 2);
-  L.w_total = w;
-  L.total = o + w * (kFilterLaneThreads / 32);
-  return L;
-}
-
 size_t filter_lane_smem_bytes(const FilterLaneParams &p) { return lane_filter_layout(p).total; }
-
-__device__ __forceinline__ uint4 lds128(const unsigned char *p) { return *(const uint4 *)p; }
-__device__ __forceinline__ void and4(uint4 &a, const uint4 b) {
-  a.x &= b.x;
-  a.y &= b.y;
-  a.z &= b.z;
-  a.w &= b.w;
-}
-
-// threshold planes of the records [e0, e1), each with exactly NP planes:
-// c = |ball_r(v) \ {v}| in the record's field, plane word = ballot(c >= t)
-// per slot, stored as [channel][4 slots] (every lane stores the same value:
-// one unpredicated 128-bit shared store)
-template <bool WIDE, int NP, typename BT>
-__device__ __forceinline__ void plane_records(int e0, int e1, const uint2 *grec, const unsigned char *wfm,
-                                              unsigned char *wpl, const BT (&bx)[4]) {
-  for (int e = e0; e < e1; e++) {
-    // record: x = field slot | #planes << 8 | first plane channel << 16, y = thresholds (bytes)
-    const uint2 g = grec[e];
-    const uint4 fm = lds128(wfm + 16 * (g.x & 0xffu));
-    int c[4];
-    if constexpr (WIDE) {
-      const unsigned long long f0 = (unsigned long long)fm.x | ((unsigned long long)fm.y << 32);
-      const unsigned long long f1 = (unsigned long long)fm.z | ((unsigned long long)fm.w << 32);
-      c[0] = __popcll((unsigned long long)bx[0] & f0);
-      c[1] = __popcll((unsigned long long)bx[1] & f0);
-      c[2] = __popcll((unsigned long long)bx[2] & f1);
-      c[3] = __popcll((unsigned long long)bx[3] & f1);
-    } else {
-      c[0] = __popc((unsigned)bx[0] & fm.x);
-      c[1] = __popc((unsigned)bx[1] & fm.y);
-      c[2] = __popc((unsigned)bx[2] & fm.z);
-      c[3] = __popc((unsigned)bx[3] & fm.w);
-    }
-    unsigned char *pp = wpl + 16 * (g.x >> 16);
-#pragma unroll
-    for (int j = 0; j < NP; j++) {
-      const int t = (int)((g.y >> (8 * j)) & 0xffu);
-      uint4 w;
-      w.x = __ballot_sync(LF_FULL, c[0] >= t);
-      w.y = __ballot_sync(LF_FULL, c[1] >= t);
-      w.z = __ballot_sync(LF_FULL, c[2] >= t);
-      w.w = __ballot_sync(LF_FULL, c[3] >= t);
-      *(uint4 *)(pp + 16 * j) = w;
-    }
-  }
-}
-
-// 32x32 bit-matrix transpose across the warp: lane L holds row L (bit p =
-// element (L, p)); returns column `lane` (bit L = element (L, lane))
-__device__ __forceinline__ unsigned lf_transpose32(unsigned x, int lane) {
-#pragma unroll
-  for (int j = 16; j >= 1; j >>= 1) {
-    const unsigned m = j == 16 ? 0x0000ffffu : j == 8 ? 0x00ff00ffu : j == 4 ? 0x0f0f0f0fu : j == 2 ? 0x33333333u
-                                                                                               : 0x55555555u;
-    const unsigned sw = ((x << j) & ~m) | ((x >> j) & m);
-    const unsigned y = __shfl_xor_sync(LF_FULL, sw, j);
-    const unsigned K = (lane & j) ? ~m : m;
-    x = (x & K) | (y & ~K);
-  }
-  return x;
-}
-
-// one group of 4 slots.  WIDE: 2 molecules of 33-64 atoms (slots 2m + h =
-// nodes 32h .. 32h+31 of molecule m), else 4 molecules of <= 32 atoms.
-template <bool WIDE>
-__device__ __forceinline__ void lane_filter_group(const FilterLaneParams &fp, int gi, int lane,
-                                                  unsigned char *wsm, const LaneFilterLayout &L,
-                                                  const unsigned char *smem, const uint4 *rowp,
-                                                  const uint2 *qwl) {
-  constexpr int NM = WIDE ? 2 : 4;  // molecules in the group
-  unsigned char *wpl = wsm + L.w_planes;
-  unsigned char *wfm = wsm + L.w_fm;
-  unsigned char *wdz = wsm + L.w_dnz;
-  unsigned long long *wball = (unsigned long long *)(wsm + L.w_ball);
-  const uint16_t *lut = (const uint16_t *)(smem + L.lut);
-  const uint2 *grec = (const uint2 *)(smem + L.grec);
-  const int32_t *rrec = (const int32_t *)(smem + L.rrec);
-  const int32_t *rgn = (const int32_t *)(smem + L.rgn);
-  const int2 *qwh = (const int2 *)(smem + L.qwh);
-
-  // ---- molecules of the group: {first node, n, adjacency word offset, candidate units} ----
-  int mol[NM];
-  if constexpr (WIDE) {
-    const int2 m2 = __ldg((const int2 *)fp.grp_wide + gi);
-    mol[0] = m2.x;
-    mol[1] = m2.y;
-  } else {
-    const int4 m4 = __ldg((const int4 *)fp.grp_narrow + gi);
-    mol[0] = m4.x;
-    mol[1] = m4.y;
-    mol[2] = m4.z;
-    mol[3] = m4.w;
-  }
-  int my_mol = -1;  // lane m < NM: molecule m (GMCR words and pair counts)
-#pragma unroll
-  for (int m = 0; m < NM; m++)
-    if (lane == m) my_mol = mol[m];
-  uint4 mr[NM];
-#pragma unroll
-  for (int m = 0; m < NM; m++) mr[m] = mol[m] >= 0 ? __ldg(&fp.mrec[mol[m]]) : make_uint4(0u, 0u, 0u, 0u);
-
-  // ---- nodes: slot k holds node v = 32 h + lane of molecule m ----
-  unsigned lt[4], nb[4];
-#pragma unroll
-  for (int k = 0; k < 4; k++) {
-    const int m = WIDE ? k >> 1 : k;
-    const unsigned v = (WIDE ? 32u * (k & 1) : 0u) + (unsigned)lane;
-    const bool ok = v < mr[m].y;
-    lt[k] = 0xffffu;
-    nb[k] = v * 0x01010101u;  // filler = the node itself (OR-neutral in the BFS)
-    if (ok) {
-      lt[k] = lut[__ldg(fp.label + mr[m].x + v)];
-      nb[k] = __ldg(fp.nb4 + mr[m].x + v);
-    }
-  }
-  // label planes (channels 0..NLAB-1) and field masks [NFU][4 slots]
-  if (fp.NLAB + fp.NFU <= 32) {
-    // per slot, lane = node builds its one-hot word (bit c: label channel c,
-    // bit NLAB + f: field slot f); a warp transpose turns it into lane = channel
-    unsigned tw[4];
-#pragma unroll
-    for (int k = 0; k < 4; k++) {
-      const unsigned lc = lt[k] & 0xffu, fs = lt[k] >> 8;
-      unsigned mb = lc < 32u ? 1u << lc : 0u;
-      mb |= fs < 32u ? 1u << ((unsigned)fp.NLAB + fs) : 0u;
-      tw[k] = lf_transpose32(mb, lane);
-    }
-    const uint4 w = make_uint4(tw[0], tw[1], tw[2], tw[3]);
-    if (lane < fp.NLAB) *(uint4 *)(wpl + 16 * lane) = w;
-    else if (lane < fp.NLAB + fp.NFU) *(uint4 *)(wfm + 16 * (lane - fp.NLAB)) = w;
-  } else {
-    for (int c = 0; c < fp.NLAB; c++) {
-      uint4 w;
-      w.x = __ballot_sync(LF_FULL, (lt[0] & 0xffu) == (unsigned)c);
-      w.y = __ballot_sync(LF_FULL, (lt[1] & 0xffu) == (unsigned)c);
-      w.z = __ballot_sync(LF_FULL, (lt[2] & 0xffu) == (unsigned)c);
-      w.w = __ballot_sync(LF_FULL, (lt[3] & 0xffu) == (unsigned)c);
-      *(uint4 *)(wpl + 16 * c) = w;
-    }
-    for (int f = 0; f < fp.NFU; f++) {
-      uint4 w;
-      w.x = __ballot_sync(LF_FULL, (lt[0] >> 8) == (unsigned)f);
-      w.y = __ballot_sync(LF_FULL, (lt[1] >> 8) == (unsigned)f);
-      w.z = __ballot_sync(LF_FULL, (lt[2] >> 8) == (unsigned)f);
-      w.w = __ballot_sync(LF_FULL, (lt[3] >> 8) == (unsigned)f);
-      *(uint4 *)(wfm + 16 * f) = w;
-    }
-  }
-  __syncwarp();
-
-  // ---- radii 1..R: BFS + threshold planes ----
-  // balls: narrow u32 (bit = node of the molecule), wide u64
-  using BT = typename std::conditional<WIDE, unsigned long long, unsigned>::type;
-  BT ball[4];
-#pragma unroll
-  for (int k = 0; k < 4; k++) {
-    const int m = WIDE ? k >> 1 : k;
-    const unsigned v = (WIDE ? 32u * (k & 1) : 0u) + (unsigned)lane;
-    ball[k] = v < mr[m].y ? (BT)1 << v : (BT)0;
-  }
-  // nodes with > 4 neighbours (flag bit 7 of nb byte 0): slow path over the all-bonds adjacency mask
-  bool slow[4];
-#pragma unroll
-  for (int k = 0; k < 4; k++) slow[k] = __any_sync(LF_FULL, (nb[k] & 0x80u) != 0u);
-
-  for (int r = 1; r <= fp.R; r++) {
-    if constexpr (!WIDE) {
-      BT nx[4];
-#pragma unroll
-      for (int k = 0; k < 4; k++) {
-        BT x = ball[k];
-        x |= __shfl_sync(LF_FULL, ball[k], (int)(nb[k] & 31u));
-        x |= __shfl_sync(LF_FULL, ball[k], (int)((nb[k] >> 8) & 31u));
-        x |= __shfl_sync(LF_FULL, ball[k], (int)((nb[k] >> 16) & 31u));
-        x |= __shfl_sync(LF_FULL, ball[k], (int)((nb[k] >> 24) & 31u));
-        if (slow[k]) {  // rare: the 5th.. neighbours from the all-bonds adjacency mask
-          const int m = k;
-          const unsigned v = (unsigned)lane;
-          unsigned rest = 0u;
-          if ((nb[k] & 0x80u) && v < mr[m].y)
-            rest = __ldg(fp.adjw + mr[m].z + (unsigned)fp.NB * mr[m].y + v);
-          // drop the 4 neighbours already gathered
-          rest &= ~((1u << (nb[k] & 31u)) | (1u << ((nb[k] >> 8) & 31u)) | (1u << ((nb[k] >> 16) & 31u)) |
-                    (1u << ((nb[k] >> 24) & 31u)));
-          unsigned any = __ballot_sync(LF_FULL, rest != 0u);
-          while (any) {
-            const int u = rest ? __ffs(rest) - 1 : lane;
-            const unsigned y = __shfl_sync(LF_FULL, ball[k], u);
-            if (rest) x |= y;
-            rest &= rest - 1u;
-            any = __ballot_sync(LF_FULL, rest != 0u);
-          }
-        }
-        nx[k] = x;
-      }
-#pragma unroll
-      for (int k = 0; k < 4; k++) ball[k] = nx[k];
-    } else {
-      // wide: balls of molecule m at wball[64 m + v]
-#pragma unroll
-      for (int k = 0; k < 4; k++) wball[64 * (k >> 1) + 32 * (k & 1) + lane] = ball[k];
-      __syncwarp();
-      BT nx[4];
-#pragma unroll
-      for (int k = 0; k < 4; k++) {
-        const unsigned long long *bm = wball + 64 * (k >> 1);
-        BT x = ball[k];
-        x |= bm[nb[k] & 63u];
-        x |= bm[(nb[k] >> 8) & 63u];
-        x |= bm[(nb[k] >> 16) & 63u];
-        x |= bm[(nb[k] >> 24) & 63u];
-        const int m = k >> 1;
-        const unsigned v = 32u * (k & 1) + (unsigned)lane;
-        if (slow[k] && (nb[k] & 0x80u) && v < mr[m].y) {
-          unsigned long long rest =
-              __ldg((const unsigned long long *)(fp.adjw + mr[m].z + 2u * ((unsigned)fp.NB * mr[m].y + v)));
-          rest &= ~((1ull << (nb[k] & 63u)) | (1ull << ((nb[k] >> 8) & 63u)) | (1ull << ((nb[k] >> 16) & 63u)) |
-                    (1ull << ((nb[k] >> 24) & 63u)));
-          while (rest) {
-            x |= bm[__ffsll((long long)rest) - 1];
-            rest &= rest - 1ull;
-          }
-        }
-        nx[k] = x;
-      }
-      __syncwarp();
-#pragma unroll
-      for (int k = 0; k < 4; k++) ball[k] = nx[k];
-    }
-    // the node itself is not counted (u != v, R4)
-    BT bx[4];
-#pragma unroll
-    for (int k = 0; k < 4; k++) {
-      const unsigned v = (WIDE ? 32u * (k & 1) : 0u) + (unsigned)lane;
-      bx[k] = ball[k] & ~((BT)1 << v);
-    }
-    __syncwarp();
-    // records of radius r, in four runs of 1, 2, 3, 4 planes (no per-plane branches)
-    const int *rr = rrec + 4 * (r - 1);
-    plane_records<WIDE, 1>(rr[0], rr[1], grec, wfm, wpl, bx);
-    plane_records<WIDE, 2>(rr[1], rr[2], grec, wfm, wpl, bx);
-    plane_records<WIDE, 3>(rr[2], rr[3], grec, wfm, wpl, bx);
-    plane_records<WIDE, 4>(rr[3], rr[4], grec, wfm, wpl, bx);
-  }
-  __syncwarp();
-
-  // ---- rows: lane = distinct row; window = AND of the row's channels ----
-  unsigned obase[4];  // cmol word of row 0 of each slot (narrow: u32 windows; wide: u64, lo/hi words)
-  bool sval[4];
-#pragma unroll
-  for (int k = 0; k < 4; k++) {
-    const int m = WIDE ? k >> 1 : k;
-    sval[k] = mol[m] >= 0;
-    obase[k] = (unsigned)fp.NDR * mr[m].w + (WIDE ? (unsigned)(k & 1) : 0u);
-  }
-  constexpr unsigned OS = WIDE ? 2u : 1u;  // words per window
-  const int NDRW = (fp.NDR + 31) >> 5;
-  const int RWV = fp.RWV;
-  for (int rg = 0; rg < NDRW; rg++) {
-    const int row = 32 * rg + lane;
-    uint4 acc = make_uint4(0u, 0u, 0u, 0u);
-    if (row < fp.NDR) {
-      acc = make_uint4(LF_FULL, LF_FULL, LF_FULL, LF_FULL);
-      const int nw = rgn[rg];  // channel-pair words of this row group (rows sorted by length)
-      const uint4 *pr = rowp + (size_t)row * RWV;
-      for (int q = 0; q < nw; q += 4) {
-        const uint4 pw = pr[q >> 2];
-        switch (nw - q) {  // uniform across the warp: rows are sorted by length
-          default:
-            and4(acc, lds128(wpl + (pw.w & 0xffffu)));
-            and4(acc, lds128(wpl + (pw.w >> 16)));
-            [[fallthrough]];
-          case 3:
-            and4(acc, lds128(wpl + (pw.z & 0xffffu)));
-            and4(acc, lds128(wpl + (pw.z >> 16)));
-            [[fallthrough]];
-          case 2:
-            and4(acc, lds128(wpl + (pw.y & 0xffffu)));
-            and4(acc, lds128(wpl + (pw.y >> 16)));
-            [[fallthrough]];
-          case 1:
-            and4(acc, lds128(wpl + (pw.x & 0xffffu)));
-            and4(acc, lds128(wpl + (pw.x >> 16)));
-        }
-      }
-      const unsigned ro = OS * (unsigned)row;
-      if (sval[0]) fp.cmol[obase[0] + ro] = acc.x;
-      if (sval[1]) fp.cmol[obase[1] + ro] = acc.y;
-      if (sval[2]) fp.cmol[obase[2] + ro] = acc.z;
-      if (sval[3]) fp.cmol[obase[3] + ro] = acc.w;
-    }
-    uint4 ne;
-    ne.x = __ballot_sync(LF_FULL, acc.x != 0u);
-    ne.y = __ballot_sync(LF_FULL, acc.y != 0u);
-    ne.z = __ballot_sync(LF_FULL, acc.z != 0u);
-    ne.w = __ballot_sync(LF_FULL, acc.w != 0u);
-    if (WIDE) {  // a molecule's row is non-empty if either half is
-      ne.x |= ne.y;
-      ne.y = ne.x;
-      ne.z |= ne.w;
-      ne.w = ne.z;
-    }
-    *(uint4 *)(wdz + 16 * rg) = ne;
-  }
-  __syncwarp();
-
-  // ---- GMCR: lane = query; its (word, bits) list over the
-  // distinct-row non-empty bits, padded per 32-query group with (0, 0) ----
-  long long cnt = 0;     // lane m < NM: surviving pairs of molecule m
-  for (int qg = 0; qg < fp.NQG; qg++) {
-    const int2 h = qwh[qg];  // entry offset (x 32), entries
-    unsigned f0 = 0u, f1 = 0u, f2 = 0u, f3 = 0u;
-    for (int j = 0; j < h.y; j++) {
-      const uint2 e = qwl[(size_t)(h.x + j) * 32 + lane];
-      const uint4 d = lds128(wdz + 16 * e.x);
-      f0 |= e.y & ~d.x;
-      f1 |= e.y & ~d.y;
-      f2 |= e.y & ~d.z;
-      f3 |= e.y & ~d.w;
-    }
-    const bool qv = 32 * qg + lane < fp.NQ;
-    unsigned w[4];
-    w[0] = __ballot_sync(LF_FULL, qv && f0 == 0u);
-    w[1] = __ballot_sync(LF_FULL, qv && f1 == 0u);
-    w[2] = __ballot_sync(LF_FULL, qv && f2 == 0u);
-    w[3] = __ballot_sync(LF_FULL, qv && f3 == 0u);
-    // molecule m's word: slot m (narrow) or slot 2m (wide; both halves carry it)
-    unsigned gmw = 0u;
-#pragma unroll
-    for (int m = 0; m < NM; m++)
-      if (lane == m) gmw = w[WIDE ? 2 * m : m];
-    if (my_mol >= 0) {
-      fp.gm[(size_t)my_mol * fp.NQW + qg] = gmw;
-      cnt += __popc(gmw);
-    }
-  }
-  if (my_mol >= 0) {
-    I64x2 v;
-    v.a = WIDE ? 0 : cnt;
-    v.b = WIDE ? cnt : 0;
-    fp.mol_cnt[my_mol] = v;
-  }
-  __syncwarp();
-}
-
-template <bool GL>
-__global__ void __launch_bounds__(kFilterLaneThreads) k_filter_lane(const __grid_constant__ FilterLaneParams fp) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  constexpr int NWARP = kFilterLaneThreads / 32;
-  const LaneFilterLayout L = lane_filter_layout(fp);
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  // ---- CTA tables ----
-  if (!GL) {
-    const uint4 *src = fp.rowp;
-    uint4 *dst = (uint4 *)(smem + L.rowp);
-    for (int i = tid; i < fp.NDR * fp.RWV; i += kFilterLaneThreads) dst[i] = __ldg(&src[i]);
-    const uint2 *qs = fp.qwl;
-    uint2 *qd = (uint2 *)(smem + L.qwl);
-    for (int i = tid; i < fp.NQWE; i += kFilterLaneThreads) qd[i] = __ldg(&qs[i]);
-  }
-  {
-    int32_t *rg = (int32_t *)(smem + L.rgn);
-    for (int i = tid; i < (fp.NDR + 31) / 32; i += kFilterLaneThreads) rg[i] = __ldg(&fp.rgn[i]);
-    uint2 *gr = (uint2 *)(smem + L.grec);
-    for (int i = tid; i < fp.NREC; i += kFilterLaneThreads) gr[i] = __ldg(&fp.grec[i]);
-    int2 *qh = (int2 *)(smem + L.qwh);
-    for (int i = tid; i < fp.NQG; i += kFilterLaneThreads) qh[i] = __ldg(&fp.qwh[i]);
-    uint16_t *lu = (uint16_t *)(smem + L.lut);
-    for (int i = tid; i < 256; i += kFilterLaneThreads) lu[i] = __ldg(&fp.lut[i]);
-    int32_t *rr = (int32_t *)(smem + L.rrec);
-    for (int i = tid; i <= 4 * fp.R; i += kFilterLaneThreads) rr[i] = __ldg(&fp.rrec[i]);
-  }
-  unsigned char *wsm = smem + L.warps + (size_t)wid * L.w_total;
-  // the all-ones channel NLAB (row padding and label-less rows never read it otherwise)
-  if (lane == 0) *(uint4 *)(wsm + L.w_planes + 16 * fp.NLAB) = make_uint4(LF_FULL, LF_FULL, LF_FULL, LF_FULL);
-  __syncthreads();
-  const uint4 *rowp = GL ? fp.rowp : (const uint4 *)(smem + L.rowp);
-  const uint2 *qwl = GL ? fp.qwl : (const uint2 *)(smem + L.qwl);
-  const int ng = fp.NGN + fp.NGW;
-  for (int gi = blockIdx.x * NWARP + wid; gi < ng; gi += gridDim.x * NWARP) {
-    if (gi < fp.NGN) lane_filter_group<false>(fp, gi, lane, wsm, L, smem, rowp, qwl);
-    else lane_filter_group<true>(fp, gi - fp.NGN, lane, wsm, L, smem, rowp, qwl);
-  }
-}
 
 cudaError_t launch_filter_lane(const FilterLaneParams &p, int grid, cudaStream_t st) {
   if (grid <= 0 || p.NGN + p.NGW <= 0) return cudaSuccess;

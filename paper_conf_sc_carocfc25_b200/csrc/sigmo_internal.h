@@ -5,19 +5,18 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <string>
 #include <vector>
+
+#include "lane_filter_types.h"
 
 namespace sigmo {
 
 constexpr int kNumFields = 13;   // R7 field table (see sigmo_kernels.cu kFieldWidth)
-constexpr int kMaxRadius = 15;   // levels <= 16
 constexpr int kFilterThreads = 256;
 constexpr int kJoinThreads = 128;
 constexpr int kQueryPrepThreads = 1024;
 
-struct I64x2 {
-  long long a, b;
-};
 
 // R7 field of an atom label (atomic number): C N O S F Cl Br I P H B Si, other
 __host__ __device__ inline int field_of_label(int lab) {
@@ -230,37 +229,6 @@ struct ChunkParams {
   int32_t *nchunks;
 };
 
-// k_filter_lane (sigmo_filter_lane.cu): the filter of the lane-join path.
-// Groups of 4 slots of 32 nodes: narrow groups = 4 molecules of <= 32 atoms,
-// wide groups = 2 molecules of 33-64 atoms.  Channels of the per-warp plane
-// array: 0..NLAB-1 label planes, NLAB all ones, NLAB+1+p constraint plane p.
-constexpr int kFilterLaneThreads = 256;
-struct FilterLaneParams {
-  int NGN, NGW;                 // narrow / wide groups
-  const int32_t *grp_narrow;    // [4 NGN] molecule ids (-1 = empty slot)
-  const int32_t *grp_wide;      // [2 NGW]
-  const uint4 *mrec;            // [ND] {first node, atoms, adjacency word offset, candidate units}
-  const uint8_t *label;         // [VD]
-  const uint32_t *nb4;          // [VD] first <= 4 neighbours (molecule-local ids, filler = self; bit 7: degree > 4)
-  const uint32_t *adjw;         // bond-class adjacency, class NB = all bonds (slow path of degree > 4 nodes)
-  int NB, R, NLAB, NFU, NCH;
-  const uint16_t *lut;          // [256] label -> label channel (0xff none) | field slot << 8 (0xff unused)
-  const uint2 *grec;            // [NREC] plane records: x = field slot | #planes (<= 4) << 8 | first channel << 16,
-  int NREC;                     //        y = thresholds (bytes), sorted by radius
-  const int32_t *rrec;          // [4R+1] record ranges: radius r, k+1 planes at [rrec[4(r-1)+k], rrec[4(r-1)+k+1])
-  const uint4 *rowp;            // [NDR][RWV] row programs: pairs of 16-bit channel byte offsets (x16), all-ones padded
-  const int32_t *rgn;           // [ceil(NDR/32)] channel-pair words needed by each 32-row group (rows sorted by length)
-  int NDR, RWV;
-  const uint2 *qwl;             // GMCR lists [entries][32 lanes] (word, bits), (0, 0) padded
-  int NQWE;                     // entries x 32
-  const int2 *qwh;              // [NQG] {first entry, entries} per 32-query group
-  int NQG, NQ, NQW;
-  uint32_t *cmol;               // molecule-padded windows (FilterParams::cmol)
-  uint32_t *gm;                 // [ND][NQW]
-  I64x2 *mol_cnt;               // [ND+1]
-  int tables_global;            // 1: row programs and GMCR lists read from global memory (too large for smem)
-  size_t smem_bytes;
-};
 
 // ---- launchers (sigmo_kernels.cu); all enqueue on `st` ----
 cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, cudaStream_t st);
@@ -282,6 +250,18 @@ cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const
 cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const uint32_t *adj_off, uint32_t *adjw,
                         uint32_t *nb4, cudaStream_t st);
 cudaError_t launch_filter_lane(const FilterLaneParams &p, int grid, cudaStream_t st);
+// run-time specialised lane filter (sigmo_jit.cu)
+struct LaneJitSpec {
+  int NLAB = 0, NFU = 0, R = 0, NDR = 0, RWV = 1, NQG = 0, NQ = 0, NQW = 0;
+  bool GL = false;
+  std::vector<std::vector<uint2>> recs;  // [R] plane records of each radius (FilterLaneParams::grec format)
+  std::vector<int> rgn;                  // channel-pair words per 32-row group
+  std::vector<int2> qwh;                 // {first entry, entries} per 32-query group
+};
+std::string lane_jit_header(const LaneJitSpec &s);
+cudaKernel_t lane_jit_kernel(const LaneJitSpec &s, std::string *why, double *compile_ms);
+cudaError_t launch_filter_lane_jit(cudaKernel_t k, const FilterLaneParams &p, int grid, cudaStream_t st);
+int filter_lane_jit_blocks_per_sm(cudaKernel_t k, const FilterLaneParams &p);
 size_t filter_lane_smem_bytes(const FilterLaneParams &p);
 int filter_lane_blocks_per_sm(const FilterLaneParams &p);
 cudaError_t launch_mrec(const int32_t *goff, const uint32_t *adj_off, const uint32_t *cand_units, int ND, uint4 *mrec,

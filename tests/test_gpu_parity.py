@@ -249,19 +249,28 @@ def test_c3_bench_workload_parity(ctx, sigmo):
         assert np.array_equal(dense, (ref > 0).astype(np.uint64)), g0
 
 
-def test_filter_rows_from_global(sigmo, monkeypatch):
-    """Row programs read from global memory (the fallback when shared memory is
-    short, forced by SIGMO_FILTER_ROWS_GLOBAL): same bitmap and counts."""
-    monkeypatch.setenv("SIGMO_FILTER_ROWS_GLOBAL", "1")
+@pytest.mark.parametrize("env", [{"SIGMO_FILTER_JIT": "0"}, {"SIGMO_FILTER_JIT": "0", "SIGMO_FILTER_TABLES_GLOBAL": "1"},
+                                 {"SIGMO_FILTER_TABLES_GLOBAL": "1"}, {}],
+                         ids=["generic", "generic-global", "jit-global", "jit"])
+def test_lane_filter_variants(sigmo, monkeypatch, env):
+    """Every build of the lane-path filter (the table-driven generic kernel and
+    the NVRTC-specialised one; query tables in shared or global memory) gives
+    the same bitmap, GMCR pairs and counts as the references."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
     Q, D = synth.config_queries(2), synth.config_data(2, count=3000)
     ref = oracle.count_dense(Q, D)
     with sigmo.Context(0) as c:
         c.load_batch(Q, D)
         for L in (1, 3, 4):
             c.filter(L)
+            c.set_timing(True)
             c.join(sigmo.SIGMO_FIND_ALL)
             assert np.array_equal(c.dense_results(), ref), L
+            assert c.timings()["filter_jit"] == (0 if env.get("SIGMO_FILTER_JIT") == "0" else 1), L
         Cb = fr.candidates_bool(Q, D, 4, data_graphs=list(range(0, 3000, 97)))
+        G = fr.gmcr(Q, D, fr.candidates_bool(Q, D, 4))
+        assert c.num_pairs() == int(G.sum())
         ref_bits = fr.to_bitmap(Cb)
         bm = c.candidates()
         for g in range(0, 3000, 97):
