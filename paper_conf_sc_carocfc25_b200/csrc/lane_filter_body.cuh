@@ -48,6 +48,15 @@ namespace sigmo {
 #define LF_C(x) fp.x
 #endif
 
+// 128-bit shared store by lane 0 only (a store of the same value by all 32
+// lanes still costs 4 shared wavefronts); a = shared-window address
+__device__ __forceinline__ void lf_sts128_lane0(unsigned a, const uint4 v, int lane) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.eq.s32 p, %5, 0;\n @p st.shared.v4.u32 [%0], {%1, %2, %3, %4};\n}\n" ::"r"(a),
+      "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"(lane)
+      : "memory");
+}
+
 template <bool W> struct LfBall { typedef unsigned T; };
 template <> struct LfBall<true> { typedef unsigned long long T; };
 
@@ -95,7 +104,7 @@ __device__ __forceinline__ void and4(uint4 &a, const uint4 b) {
 // per slot, stored as [channel][4 slots] (every lane stores the same value:
 // one unpredicated 128-bit shared store)
 template <bool WIDE, int NP, typename BT>
-__device__ __forceinline__ void lf_record(const BT (&bx)[4], const uint4 fm, unsigned char *pp, unsigned thr) {
+__device__ __forceinline__ void lf_record(const BT (&bx)[4], const uint4 fm, unsigned pp, unsigned thr, int lane) {
   int c[4];
   if constexpr (WIDE) {
     const unsigned long long f0 = (unsigned long long)fm.x | ((unsigned long long)fm.y << 32);
@@ -118,18 +127,18 @@ __device__ __forceinline__ void lf_record(const BT (&bx)[4], const uint4 fm, uns
     w.y = __ballot_sync(LF_FULL, c[1] >= t);
     w.z = __ballot_sync(LF_FULL, c[2] >= t);
     w.w = __ballot_sync(LF_FULL, c[3] >= t);
-    *(uint4 *)(pp + 16 * j) = w;
+    lf_sts128_lane0(pp + 16u * j, w, lane);
   }
 }
 
 // threshold planes of the records [e0, e1), each with exactly NP planes
 template <bool WIDE, int NP, typename BT>
 __device__ __forceinline__ void plane_records(int e0, int e1, const uint2 *grec, const unsigned char *wfm,
-                                              unsigned char *wpl, const BT (&bx)[4]) {
+                                              unsigned wpl_s, const BT (&bx)[4], int lane) {
   for (int e = e0; e < e1; e++) {
     // record: x = field slot | #planes << 8 | first plane channel << 16, y = thresholds (bytes)
     const uint2 g = grec[e];
-    lf_record<WIDE, NP>(bx, lds128(wfm + 16 * (g.x & 0xffu)), wpl + 16 * (g.x >> 16), g.y);
+    lf_record<WIDE, NP>(bx, lds128(wfm + 16 * (g.x & 0xffu)), wpl_s + 16u * (g.x >> 16), g.y, lane);
   }
 }
 
@@ -218,7 +227,7 @@ __device__ __forceinline__ void lf_row_group(int rg, int nw, int NDR, int RWV, c
     ne.z |= ne.w;
     ne.w = ne.z;
   }
-  *(uint4 *)(c.wdz + 16 * rg) = ne;
+  lf_sts128_lane0((unsigned)__cvta_generic_to_shared(c.wdz) + 16u * rg, ne, c.lane);
 }
 
 // one 32-query group of the GMCR test: lane = query; a query
@@ -279,6 +288,7 @@ __device__ __forceinline__ void lane_filter_group(const FilterLaneParams &fp, in
                                                   const uint2 *qwl) {
   constexpr int NM = WIDE ? 2 : 4;  // molecules in the group
   unsigned char *wpl = wsm + L.w_planes;
+  const unsigned wpl_s = (unsigned)__cvta_generic_to_shared(wpl);
   unsigned char *wfm = wsm + L.w_fm;
   unsigned char *wdz = wsm + L.w_dnz;
   unsigned long long *wball = (unsigned long long *)(wsm + L.w_ball);
@@ -446,14 +456,14 @@ __device__ __forceinline__ void lane_filter_group(const FilterLaneParams &fp, in
     }
     __syncwarp();
 #ifdef SIGMO_LF_JIT
-    jit_records<WIDE>(r, bx, wfm, wpl);  // generated: the query program's records of radius r, constants inlined
+    jit_records<WIDE>(r, bx, wfm, wpl_s, lane);  // generated: the query program's records of radius r, constants inlined
 #else
     // records of radius r, in four runs of 1, 2, 3, 4 planes (no per-plane branches)
     const int *rr = rrec + 4 * (r - 1);
-    plane_records<WIDE, 1>(rr[0], rr[1], grec, wfm, wpl, bx);
-    plane_records<WIDE, 2>(rr[1], rr[2], grec, wfm, wpl, bx);
-    plane_records<WIDE, 3>(rr[2], rr[3], grec, wfm, wpl, bx);
-    plane_records<WIDE, 4>(rr[3], rr[4], grec, wfm, wpl, bx);
+    plane_records<WIDE, 1>(rr[0], rr[1], grec, wfm, wpl_s, bx, lane);
+    plane_records<WIDE, 2>(rr[1], rr[2], grec, wfm, wpl_s, bx, lane);
+    plane_records<WIDE, 3>(rr[2], rr[3], grec, wfm, wpl_s, bx, lane);
+    plane_records<WIDE, 4>(rr[3], rr[4], grec, wfm, wpl_s, bx, lane);
 #endif
   }
   __syncwarp();

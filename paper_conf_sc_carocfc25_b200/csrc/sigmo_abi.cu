@@ -1553,6 +1553,8 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       if (!(je && atoi(je) == 0)) {
         LaneJitSpec &js = c->progs[R].jit;
         js.GL = lp.tables_global != 0;
+        js.min_blocks = 3;  // 80 registers, 24 warps/SM (configs[2]: 0.93 ms at the unbounded 110 registers)
+        if (const char *mb = getenv("SIGMO_FILTER_JIT_MINB")) js.min_blocks = std::max(1, std::min(8, atoi(mb)));
         std::string why;
         double cms = 0.0;
         jk = lane_jit_kernel(js, &why, &cms);

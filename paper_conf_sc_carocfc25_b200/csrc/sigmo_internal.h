@@ -254,6 +254,7 @@ cudaError_t launch_filter_lane(const FilterLaneParams &p, int grid, cudaStream_t
 struct LaneJitSpec {
   int NLAB = 0, NFU = 0, R = 0, NDR = 0, RWV = 1, NQG = 0, NQ = 0, NQW = 0;
   bool GL = false;
+  int min_blocks = 3;                    // __launch_bounds__ min CTAs per SM (register cap)
   std::vector<std::vector<uint2>> recs;  // [R] plane records of each radius (FilterLaneParams::grec format)
   std::vector<int> rgn;                  // channel-pair words per 32-row group
   std::vector<int2> qwh;                 // {first entry, entries} per 32-query group
