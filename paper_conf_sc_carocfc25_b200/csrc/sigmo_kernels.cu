@@ -2024,11 +2024,16 @@ __host__ __device__ inline size_t join_lane_warp_bytes(int MQ, bool w64) {
   return 32 * (size_t)(w64 ? 16 : 8) * SD + 512;
 }
 // CTA: per-query totals [NQ] u64, then one region per warp
-__host__ __device__ inline size_t join_lane_cta_bytes(int NQ) { return align16(8 * (size_t)(NQ > 0 ? NQ : 1)); }
-__host__ __device__ inline size_t join_lane_smem(int NQ, int MQ, bool w64) {
-  return join_lane_cta_bytes(NQ) + join_lane_warp_bytes(MQ, w64) * (kJoinLaneThreads / 32);
+// CTA: per-query totals [NQ] u64, then (optionally) the plan entries [VQ] uint2
+constexpr int kJoinLanePlanSmemMax = 2048;  // plan positions copied to shared memory (16 KB)
+__host__ __device__ inline size_t join_lane_plan_bytes(int VQ) { return VQ <= kJoinLanePlanSmemMax ? align16(8 * (size_t)VQ) : 0; }
+__host__ __device__ inline size_t join_lane_cta_bytes(int NQ, int VQ) {
+  return align16(8 * (size_t)(NQ > 0 ? NQ : 1)) + join_lane_plan_bytes(VQ);
 }
-size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_smem(p.NQ, p.maxq, w64); }
+__host__ __device__ inline size_t join_lane_smem(int NQ, int VQ, int MQ, bool w64) {
+  return join_lane_cta_bytes(NQ, VQ) + join_lane_warp_bytes(MQ, w64) * (kJoinLaneThreads / 32);
+}
+size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_smem(p.NQ, p.VQ, p.maxq, w64); }
 
 __device__ __forceinline__ void cp_async8(unsigned dst_smem, const void *src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(dst_smem), "l"(src) : "memory");
@@ -2064,8 +2069,13 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   // -- both lose to the occupancy they cost; so did taking two leaf-level
   // candidates per step, 9.60 vs 9.49 ms, and caching the top stack entry in
   // registers, 8.92 vs 8.80 ms)
-  const uint2 *const qp_ent = jp.qp_ent2;  // 8-B entries: more lanes share a sector
-  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
+  // plan entries (8 B): a shared-memory copy when they fit, else through the read-only cache
+  const unsigned o_plan = (unsigned)align16(8 * (size_t)(jp.NQ > 0 ? jp.NQ : 1));
+  const bool plan_s = join_lane_plan_bytes(jp.VQ) > 0;
+  if (plan_s)
+    for (int i = threadIdx.x; i < jp.VQ; i += blockDim.x) ((uint2 *)(smem + o_plan))[i] = __ldg(&jp.qp_ent2[i]);
+  auto plan = [&](unsigned i) -> uint2 { return plan_s ? ((const uint2 *)(smem + o_plan))[i] : __ldg(&jp.qp_ent2[i]); };
+  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ, jp.VQ) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
   const unsigned oRU = wbase + ES * lane;                         // {R, U} of depth d: oRU + 32 ES d
   const unsigned oM = wbase + 32u * ES * SD + lane;               // f(pi_d): oM + 32 d
   auto ldRU = [&](unsigned o, MT &r, MT &u) {
@@ -2111,8 +2121,8 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   const uint32_t *const cmol = jp.cmol;
   // candidate window of distinct row r of the pair's molecule (cmol word base cb)
   auto cand = [&](unsigned cb, unsigned r) -> MT {
-    if (W64) return (MT)__ldg((const unsigned long long *)(cmol + cb + 2u * r));
-    return (MT)__ldg(cmol + cb + r);
+    if (W64) return (MT)__ldg((const unsigned long long *)(cmol + (cb + 2u * r)));
+    return (MT)__ldg(cmol + (cb + r));
   };
   const unsigned ones = jp.adj_ones;  // the all-ones entry (absent back-edge)
   const int4 zero4 = make_int4(0, 0, 0, 0);
@@ -2153,7 +2163,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const unsigned od = oRU + 32u * ES * d;
       // the plan entry of depth e and the map bytes of its back-edge targets
       // depend on d only: loaded before v is known (j == d takes v below)
-      const uint2 en = __ldg(&qp_ent[cqb + e]);
+      const uint2 en = plan(cqb + e);
       MT R, U;
       ldRU(od, R, U);
       const unsigned j0 = en.x & 15, j1 = (en.x >> 4) & 15;
@@ -2259,7 +2269,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         np = cbase + (unsigned)src;
         nv = true;
         // root candidates of the next pair: the load completes while the current pair runs
-        nR0 = cand((unsigned)r.z, (unsigned)__ldg(&qp_ent[(unsigned)r.w >> 16]).x >> 12);
+        nR0 = cand((unsigned)r.z, plan((unsigned)r.w >> 16).x >> 12);
       }
       chead += take;
       wm = __ballot_sync(FULL_MASK, !nv) & wm;
@@ -2385,9 +2395,22 @@ static int join_lane_occ_t(size_t smem) {
 }
 
 int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem) {
-  (void)p;
-  if (w64) return mode == 1 ? join_lane_occ_t<1, true>(smem) : join_lane_occ_t<0, true>(smem);
-  return mode == 1 ? join_lane_occ_t<1, false>(smem) : join_lane_occ_t<0, false>(smem);
+  // the instantiation launch_join_lane picks: bit 0 Find First, bit 1 induced
+  const int m = (mode & 1) | (p.induced ? 2 : 0);
+  if (w64) {
+    switch (m) {
+      case 0: return join_lane_occ_t<0, true>(smem);
+      case 1: return join_lane_occ_t<1, true>(smem);
+      case 2: return join_lane_occ_t<2, true>(smem);
+      default: return join_lane_occ_t<3, true>(smem);
+    }
+  }
+  switch (m) {
+    case 0: return join_lane_occ_t<0, false>(smem);
+    case 1: return join_lane_occ_t<1, false>(smem);
+    case 2: return join_lane_occ_t<2, false>(smem);
+    default: return join_lane_occ_t<3, false>(smem);
+  }
 }
 
 }  // namespace sigmo
