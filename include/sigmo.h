@@ -183,16 +183,36 @@ SIGMO_API sigmo_status sigmo_get_candidates(sigmo_ctx *ctx, uint32_t *out);
  * Host out[V] u64.  Requires load_batch only. */
 SIGMO_API sigmo_status sigmo_get_signatures(sigmo_ctx *ctx, int which, int radius, uint64_t *out);
 
-/* Enable/disable per-stage CUDA-event timing (default off) and read it. */
+/* Read back the CSR-GO batch as the library packed it on the device
+ * (section 4.1; Fig. 3): which = 0 queries, 1 data.
+ * sizes: *num_graphs, *num_nodes, *num_adj (adjacency entries, both
+ * directions).  Pass NULL arrays to query the sizes only; otherwise
+ * caller-allocated host arrays graph_offsets[G+1], row_offsets[V+1],
+ * col_indices[E2] (global node ids), node_labels[V], edge_labels[E2] are
+ * filled from the device arrays (a test hook that pins the packer against
+ * the paper's worked example).  Requires load_batch.  Synchronizes. */
+SIGMO_API sigmo_status sigmo_get_packed_batch(sigmo_ctx *ctx, int which, int64_t *num_graphs, int64_t *num_nodes,
+                                              int64_t *num_adj, int64_t *graph_offsets, int64_t *row_offsets,
+                                              int32_t *col_indices, uint8_t *node_labels, uint8_t *edge_labels);
+
+/* SIGMO_OK if the last sigmo_join completed within the kernels' internal
+ * capacities, else SIGMO_ERR_LIMIT (the results are then incomplete).  The
+ * device-pointer path of sigmo_get_query_totals does not synchronize, so
+ * callers that only read totals on the device (multi-GPU all-reduce,
+ * streaming) check this once per run.  Synchronizes. */
+SIGMO_API sigmo_status sigmo_check_join(sigmo_ctx *ctx);
+
 /* Induced-subgraph mode (the literal G_D[X] reading of
  * Def. 2.1; R21): an embedding must also map every
  * NON-adjacent query node pair to a non-adjacent data node pair (a data bond
  * of any label counts as adjacency).  enable = 0 (default, monomorphism,
- * reading R1) or 1.  Takes effect at the next sigmo_load_batch, which then
- * routes the batch to the general join kernel; the filter is unchanged
- * (induced embeddings are a subset of the monomorphisms, so its candidate
- * sets stay sound).  Never fails for a valid ctx. */
+ * reading R1) or 1.  Takes effect at the next sigmo_load_batch; both join
+ * kernels (the per-lane k_join_lane and the general k_join) apply the
+ * non-edge constraints; the filter is unchanged (induced embeddings are a
+ * subset of the monomorphisms, so its candidate sets stay sound).  Never
+ * fails for a valid ctx. */
 SIGMO_API sigmo_status sigmo_set_induced(sigmo_ctx *ctx, int enable);
+/* Enable/disable per-stage CUDA-event timing (default off) and read it. */
 SIGMO_API sigmo_status sigmo_set_timing(sigmo_ctx *ctx, int enable);
 SIGMO_API sigmo_status sigmo_get_timings(sigmo_ctx *ctx, sigmo_timings *out);
 

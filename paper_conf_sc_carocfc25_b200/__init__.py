@@ -76,15 +76,47 @@ def _stream_handle(stream) -> int:
     return int(stream.cuda_stream)
 
 
-class Context:
-    """One sigmo_ctx: a device, a stream and the device state of one batch."""
+def _torch_allocator(device: int):
+    """sigmo_allocator backed by PyTorch's caching allocator (include/sigmo.h
+    sigmo_create; SURVEY 8(b) ownership): the library's device buffers come
+    from, and return to, torch's pool on the ctx stream."""
+    import torch
 
-    def __init__(self, device: int = 0, stream=None):
+    def alloc(nbytes, stream, user):
+        try:
+            return int(torch.cuda.caching_allocator_alloc(int(nbytes), device, int(stream or 0)))
+        except Exception:  # out of memory: the library reports SIGMO_ERR_OOM
+            return None
+
+    def free(ptr, stream, user):
+        try:
+            torch.cuda.caching_allocator_delete(int(ptr))
+        except Exception:  # interpreter teardown: the process is exiting anyway
+            pass
+
+    a = _native.sigmo_allocator()
+    a.alloc = _native.ALLOC_FN(alloc)
+    a.free = _native.FREE_FN(free)
+    a.user = None
+    return a
+
+
+class Context:
+    """One sigmo_ctx: a device, a stream and the device state of one batch.
+
+    ``allocator="torch"`` (default) routes the library's device buffers through
+    PyTorch's caching allocator; ``"cuda"`` uses the library's own
+    cudaMallocAsync pool."""
+
+    def __init__(self, device: int = 0, stream=None, allocator: str = "torch"):
         self._lib = load_library()
         self.device = device
         self._handle = ctypes.c_void_p()
         self._stream = _stream_handle(stream)
-        st = self._lib.sigmo_create(device, ctypes.c_void_p(self._stream), None, ctypes.byref(self._handle))
+        self._alloc = _torch_allocator(device) if allocator == "torch" else None
+        st = self._lib.sigmo_create(device, ctypes.c_void_p(self._stream),
+                                    ctypes.byref(self._alloc) if self._alloc is not None else None,
+                                    ctypes.byref(self._handle))
         if st != 0:
             raise SigmoError(st, f"sigmo_create(device={device}) failed")
         self.nq = self.nd = self.vq = self.vd = 0
@@ -185,6 +217,26 @@ class Context:
                                                    out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))),
                     "sigmo_get_signatures")
         return out
+
+    def packed_batch(self, which: int):
+        """sigmo_get_packed_batch: the CSR-GO arrays as packed on the device
+        (graph_offsets, row_offsets, col_indices, node_labels, edge_labels)."""
+        G, V, E = ctypes.c_int64(0), ctypes.c_int64(0), ctypes.c_int64(0)
+        self._check(self._lib.sigmo_get_packed_batch(self._handle, int(which), ctypes.byref(G), ctypes.byref(V),
+                                                     ctypes.byref(E), None, None, None, None, None),
+                    "sigmo_get_packed_batch")
+        go, ro = np.zeros(G.value + 1, np.int64), np.zeros(V.value + 1, np.int64)
+        co, nl, el = np.zeros(E.value, np.int32), np.zeros(V.value, np.uint8), np.zeros(E.value, np.uint8)
+        P = ctypes.POINTER
+        self._check(self._lib.sigmo_get_packed_batch(
+            self._handle, int(which), None, None, None, go.ctypes.data_as(P(ctypes.c_int64)),
+            ro.ctypes.data_as(P(ctypes.c_int64)), co.ctypes.data_as(P(ctypes.c_int32)),
+            nl.ctypes.data_as(P(ctypes.c_uint8)), el.ctypes.data_as(P(ctypes.c_uint8))), "sigmo_get_packed_batch")
+        return go, ro, co, nl, el
+
+    def check(self):
+        """sigmo_check_join: raise if the last join exceeded an internal capacity."""
+        self._check(self._lib.sigmo_check_join(self._handle), "sigmo_check_join")
 
     def set_induced(self, enable: bool = True):
         """Induced-subgraph mode for the next load_batch (include/sigmo.h sigmo_set_induced)."""

@@ -19,7 +19,8 @@ SIGMO_FILTER_NEIGHBOR_SUPPORT = 1
 # every symbol declared in include/sigmo.h
 EXPORTS = ["sigmo_create", "sigmo_load_batch", "sigmo_filter", "sigmo_join", "sigmo_num_pairs",
            "sigmo_get_pair_results", "sigmo_get_dense_results", "sigmo_get_query_totals", "sigmo_get_candidates",
-           "sigmo_get_signatures", "sigmo_set_induced", "sigmo_set_timing", "sigmo_get_timings", "sigmo_validate_batch",
+           "sigmo_get_signatures", "sigmo_get_packed_batch", "sigmo_check_join", "sigmo_set_induced", "sigmo_set_timing",
+           "sigmo_get_timings", "sigmo_validate_batch",
            "sigmo_last_error", "sigmo_version", "sigmo_destroy"]
 
 
@@ -77,6 +78,10 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
     lib.sigmo_get_query_totals.argtypes = [vp, vp, ctypes.c_int]
     lib.sigmo_get_candidates.argtypes = [vp, P(ctypes.c_uint32)]
     lib.sigmo_get_signatures.argtypes = [vp, ctypes.c_int, ctypes.c_int, P(ctypes.c_uint64)]
+    lib.sigmo_get_packed_batch.argtypes = [vp, ctypes.c_int, P(ctypes.c_int64), P(ctypes.c_int64), P(ctypes.c_int64),
+                                           P(ctypes.c_int64), P(ctypes.c_int64), P(ctypes.c_int32),
+                                           P(ctypes.c_uint8), P(ctypes.c_uint8)]
+    lib.sigmo_check_join.argtypes = [vp]
     lib.sigmo_set_timing.argtypes = [vp, ctypes.c_int]
     lib.sigmo_set_induced.argtypes = [vp, ctypes.c_int]
     lib.sigmo_get_timings.argtypes = [vp, P(sigmo_timings)]

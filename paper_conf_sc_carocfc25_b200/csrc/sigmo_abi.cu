@@ -1915,6 +1915,47 @@ sigmo_status sigmo_get_candidates(sigmo_ctx *c, uint32_t *out) {
   return SIGMO_OK;
 }
 
+sigmo_status sigmo_get_packed_batch(sigmo_ctx *c, int which, int64_t *num_graphs, int64_t *num_nodes, int64_t *num_adj,
+                                    int64_t *graph_offsets, int64_t *row_offsets, int32_t *col_indices,
+                                    uint8_t *node_labels, uint8_t *edge_labels) {
+  if (!c || (which != 0 && which != 1)) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 1) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_packed_batch before sigmo_load_batch");
+  const DevGraphs &d = which ? c->dd : c->dq;
+  if (num_graphs) *num_graphs = d.num_graphs;
+  if (num_nodes) *num_nodes = d.num_nodes;
+  if (num_adj) *num_adj = d.num_adj;
+  if (!graph_offsets && !row_offsets && !col_indices && !node_labels && !edge_labels) return SIGMO_OK;
+  if (!graph_offsets || !row_offsets || !col_indices || !node_labels || !edge_labels)
+    return set_err(c, SIGMO_ERR_INVALID_ARG, "sigmo_get_packed_batch: NULL output array");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  std::vector<int32_t> goff((size_t)d.num_graphs + 1), roff((size_t)d.num_nodes + 1);
+  std::vector<uint16_t> nbr((size_t)d.num_adj + 1);
+  std::vector<uint8_t> lab((size_t)d.num_nodes + 1);
+  CUDA_TRY(c, cudaMemcpyAsync(goff.data(), d.goff, 4 * goff.size(), cudaMemcpyDeviceToHost, c->stream));
+  CUDA_TRY(c, cudaMemcpyAsync(roff.data(), d.roff, 4 * roff.size(), cudaMemcpyDeviceToHost, c->stream));
+  if (d.num_adj) CUDA_TRY(c, cudaMemcpyAsync(nbr.data(), d.nbr, 2 * (size_t)d.num_adj, cudaMemcpyDeviceToHost, c->stream));
+  if (d.num_nodes) CUDA_TRY(c, cudaMemcpyAsync(lab.data(), d.label, (size_t)d.num_nodes, cudaMemcpyDeviceToHost, c->stream));
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  for (int g = 0; g <= d.num_graphs; g++) graph_offsets[g] = goff[g];
+  for (int v = 0; v <= d.num_nodes; v++) row_offsets[v] = roff[v];
+  for (int v = 0; v < d.num_nodes; v++) node_labels[v] = lab[v];
+  // packed neighbour = molecule-local index << 8 | bond label -> global id
+  for (int g = 0; g < d.num_graphs; g++)
+    for (int v = goff[g]; v < goff[g + 1]; v++)
+      for (int e = roff[v]; e < roff[v + 1]; e++) {
+        col_indices[e] = goff[g] + (nbr[e] >> 8);
+        edge_labels[e] = (uint8_t)(nbr[e] & 0xffu);
+      }
+  return SIGMO_OK;
+}
+
+sigmo_status sigmo_check_join(sigmo_ctx *c) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 3) return set_err(c, SIGMO_ERR_STATE, "sigmo_check_join before sigmo_join");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  return read_join_flags(c);
+}
+
 sigmo_status sigmo_get_signatures(sigmo_ctx *c, int which, int radius, uint64_t *out) {
   if (!c || !out || (which != 0 && which != 1)) return SIGMO_ERR_INVALID_ARG;
   if (radius < 1 || radius > 255) return set_err(c, SIGMO_ERR_INVALID_ARG, "radius %d not in 1..255", radius);

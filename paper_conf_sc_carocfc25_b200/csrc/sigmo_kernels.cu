@@ -1990,11 +1990,10 @@ cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const
 // k_join_lane: stack-based DFS (section 4.6) with ONE GMCR pair
 // per lane, for queries of <= kJoinLaneMaxQ nodes in <= 64-node data graphs.
 //   * Per lane, in shared memory: the DFS stack {R_d, U_d} (untried
-//     candidates of depth d, used set of f(pi_0..pi_{d-1})), the map bytes
-//     f(pi_d), and two buffers of candidate windows cm[u] (one u64 per query
-//     node, cut by the filter into cmol[g][row]; a pair's rows are
-//     contiguous): the current pair's, and the next pair's, which is
-//     prefetched with cp.async while the current one runs.  A bitmask `ne`
+//     candidates of depth d, used set of f(pi_0..pi_{d-1})) and the map
+//     bytes f(pi_d); the candidate windows cm[u] are read from the filter's
+//     cmol[g][row] layout (a pair's rows are contiguous), the next pair's
+//     root window is loaded while the current pair runs.  A bitmask `ne`
 //     of open depths makes every step productive: a step pops the lowest
 //     candidate v of the deepest open depth d (backtracking is free) and
 //     builds the candidates of e = d + 1:
@@ -2034,12 +2033,6 @@ __host__ __device__ inline size_t join_lane_smem(int NQ, int VQ, int MQ, bool w6
   return join_lane_cta_bytes(NQ, VQ) + join_lane_warp_bytes(MQ, w64) * (kJoinLaneThreads / 32);
 }
 size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_smem(p.NQ, p.VQ, p.maxq, w64); }
-
-__device__ __forceinline__ void cp_async8(unsigned dst_smem, const void *src) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(dst_smem), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
 // n-th (0-based) set bit of m (m has > n set bits)
 __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
@@ -2335,7 +2328,6 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     }
     if (drained && __ballot_sync(FULL_MASK, ne != 0u || nv || pend) == 0u) break;
   }
-  cp_async_wait_all();
   if (jp.stats) {
     unsigned long long s2 = steps;
 #pragma unroll

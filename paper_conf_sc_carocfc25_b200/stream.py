@@ -128,6 +128,14 @@ class StreamRunner:
         torch = self.torch
         for s in self.streams:
             s.synchronize()
+        for row in self.ctx:  # the device-pointer totals path never synchronized: check capacities once
+            for c in row:
+                if c.nq and self.batches_done:
+                    try:
+                        c.check()
+                    except Exception as e:
+                        if "before sigmo_join" not in str(e):
+                            raise
         out = np.zeros(self.nq, np.uint64)
         for gi, (idx, _) in enumerate(self.groups):
             out[idx] = (self.acc[0][gi] + self.acc[1][gi]).cpu().numpy().astype(np.uint64)

@@ -176,3 +176,48 @@ def test_bitmap_view_bit_order():
     bm = fr.to_bitmap(Cb)
     assert bm.shape == (2, 3)
     assert bm[0, 0] == 1 and bm[0, 1] == 2 and bm[1, 2] == 1 << 5
+
+
+def test_gmcr_rule_hand_computed():
+    """GMCR: a pair survives iff EVERY query node has a
+    candidate in the data graph.  Hand-built candidate matrix where the
+    'any node' and 'every node' readings differ."""
+    from synth import GraphBatch
+    Q = GraphBatch.from_graphs([([C, O], [(0, 1, 1)]),       # q0: C-O
+                                ([C, C], [(0, 1, 1)])])      # q1: C-C
+    D = GraphBatch.from_graphs([([C, C, C], [(0, 1, 1), (1, 2, 1)]),  # g0: propane (no O)
+                                ([C, O], [(0, 1, 1)])])               # g1: methanol-like
+    Cb = np.zeros((4, 5), bool)
+    Cb[0, [0, 1, 2, 3]] = True   # q0 node C: candidates in g0 and g1
+    Cb[1, 4] = True              # q0 node O: only g1's O
+    Cb[2, [0, 1, 2, 3]] = True   # q1 nodes: every C
+    Cb[3, [0, 1, 2, 3]] = True
+    expect = np.array([[False, True],    # q0 survives only where its O has a candidate
+                       [True, True]])    # q1: both nodes have candidates in g0 and g1
+    assert np.array_equal(fr.gmcr(Q, D, Cb), expect)
+    Cb[3, 3] = False                      # q1's second node loses its only candidate in g1
+    expect[1, 1] = False
+    assert np.array_equal(fr.gmcr(Q, D, Cb), expect)
+
+
+def test_neighbour_support_bond_labels_hand_computed():
+    """Neighbour support (R9) with bond labels: a query C=C (double bond) on
+    all-single-bond data has no support at all, so the fixed point is empty,
+    although every data C has a C neighbour (a rule ignoring the bond label
+    would keep them); on C=C-C only the double-bonded pair survives."""
+    from synth import GraphBatch
+    Q = GraphBatch.from_graphs([([C, C], [(0, 1, 2)])])
+    D = GraphBatch.from_graphs([([C, C, C], [(0, 1, 1), (1, 2, 1)])])
+    C0 = fr.candidates_bool(Q, D, 1)
+    assert C0.all()
+    assert not fr.neighbour_support(Q, D, C0).any()
+    D2 = GraphBatch.from_graphs([([C, C, C], [(0, 1, 2), (1, 2, 1)])])
+    F = fr.neighbour_support(Q, D2, fr.candidates_bool(Q, D2, 1))
+    assert np.array_equal(F, np.array([[True, True, False], [True, True, False]]))
+    # the support must come from a CANDIDATE neighbour: drop node 1 from C(q1)
+    Cb = fr.candidates_bool(Q, D2, 1)
+    Cb[1, 1] = False
+    F = fr.neighbour_support(Q, D2, Cb)
+    # q0 needs a double-bond neighbour in C(q1) = {0, 2}: only node 1 has one (node 0);
+    # q1 then needs a double-bond neighbour in C(q0) = {1}: only node 0 has one
+    assert np.array_equal(F, np.array([[False, True, False], [True, False, False]]))

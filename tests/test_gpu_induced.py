@@ -102,26 +102,3 @@ def test_induced_general_path_forced(sigmo, monkeypatch):
         check(c, sigmo, synth.config_queries(2), synth.config_data(2, count=5000))
     finally:
         c.close()
-
-
-def test_induced_bench_workload_parity(ctx, sigmo):
-    """configs[2] (the `bench.py --induced` workload: 100 queries x 1M
-    molecules, L=4) in the bench's launch configuration: per-query induced
-    Find All totals and Find First positive-pair counts over all 1M molecules
-    equal the oracle's induced mode; every pair of a ragged-end
-    2,000-molecule window is bit-exact."""
-    Q, D = synth.config_queries(3), synth.config_data(3)
-    ctx.load_batch(Q, D)
-    ctx.filter(4)
-    tot = ctx.join(sigmo.SIGMO_FIND_ALL)
-    ref_q = oracle.count_totals(Q, D, IND)
-    assert np.array_equal(ctx.query_totals(), ref_q)
-    assert tot == int(ref_q.sum())
-    di, qi, r = ctx.pair_results()
-    g0 = D.num_graphs - 2000
-    sel = di >= g0
-    dense = np.zeros((Q.num_graphs, 2000), np.uint64)
-    dense[qi[sel], di[sel] - g0] = r[sel]
-    assert np.array_equal(dense, oracle.count_dense(Q, D.slice(g0, g0 + 2000), IND))
-    ctx.join(sigmo.SIGMO_FIND_FIRST)
-    assert np.array_equal(ctx.query_totals(), oracle.count_totals(Q, D, IND | oracle.FIND_FIRST))

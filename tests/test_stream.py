@@ -58,24 +58,3 @@ def test_stream_runner_matches_oracle():
         assert np.array_equal(got2, got)
     with stream.StreamRunner(Q, 0, levels=2, mode=oracle.FIND_FIRST) as sr:
         assert np.array_equal(sr.run(batches), oracle.count_totals(Q, D, oracle.FIND_FIRST))
-
-
-@pytest.mark.gpu
-def test_config3_share_and_config4_stream_vs_oracle():
-    """The bench's routed launch configurations: configs[3] per-GPU share
-    (500 queries incl. ring systems x 125k molecules, Find First, one batch)
-    and configs[4] streaming (1,000 queries, several batches; a 60k-molecule
-    sample in 3 batches) -- per-query totals equal to the oracle's."""
-    import torch
-    import __graft_entry__
-    __graft_entry__.build()
-    torch.cuda.set_device(0)
-    Q3 = synth.config_queries(4)
-    D3 = synth.config_data(4, count=125_000)
-    with stream.StreamRunner(Q3, 0, levels=4, mode=oracle.FIND_FIRST) as sr:
-        assert np.array_equal(sr.run([D3]), oracle.count_totals(Q3, D3, oracle.FIND_FIRST))
-    Q5 = synth.config_queries(5)
-    batches = [synth.config_data(5, first=20_000 * i, count=20_000) for i in range(3)]
-    with stream.StreamRunner(Q5, 0, levels=4) as sr:
-        got = sr.run(batches)
-    assert np.array_equal(got, oracle.count_totals(Q5, synth.GraphBatch.concat(batches)))
