@@ -61,6 +61,8 @@ def _load():
         lib.oracle_count_dense.argtypes = [bp, bp, ctypes.c_int, ctypes.c_int, u64p, u64p, ip]
         lib.oracle_count_pairs.argtypes = [bp, bp, ctypes.c_int, ctypes.c_int, ctypes.c_int64, i64p, i64p, u64p,
                                            u64p, ip]
+        lib.oracle_enumerate_pair.argtypes = [bp, bp, ctypes.c_int64, ctypes.c_int64, ctypes.c_int,
+                                              ctypes.POINTER(ctypes.c_int32), ctypes.c_int64, i64p]
         _lib = lib
     return _lib
 
@@ -128,6 +130,33 @@ def count_pairs(Q, D, pq, pg, mode: int = FIND_ALL, nthreads: int | None = None,
     if ovf.value:
         raise OverflowError("oracle count exceeded 2^64-1")
     return OracleResult(out, work.value, ovf.value) if with_work else out
+
+
+def enumerate_pair(Q, D, q: int, g: int, mode: int = FIND_ALL) -> np.ndarray:
+    """Every embedding of query q in data graph g (enumerate mode, SURVEY
+    8(f) N1): int32 [n, n_q], row k = the molecule-local data node of each
+    query node (query node order) in the k-th embedding.  mode: FIND_ALL or
+    INDUCED (Find First is meaningless here)."""
+    lib = _load()
+    qs, ds = _as_struct(Q), _as_struct(D)
+    nq = int(Q.graph_offsets[q + 1] - Q.graph_offsets[q])
+    cap = 64
+    while True:
+        out = np.zeros((cap, max(nq, 1)), np.int32)
+        n = ctypes.c_int64(0)
+        rc = lib.oracle_enumerate_pair(ctypes.byref(qs), ctypes.byref(ds), int(q), int(g), int(mode) & ~FIND_FIRST,
+                                       out.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)), cap, ctypes.byref(n))
+        if rc != 0:
+            raise RuntimeError(f"oracle_enumerate_pair failed rc={rc}")
+        if n.value <= cap:
+            return out[:n.value, :nq]
+        cap = int(n.value)
+
+
+def node_sets(emb: np.ndarray) -> list:
+    """NLSM's output: the distinct node SETS X = f(V_q) of a
+    pair's embeddings, as sorted tuples, in sorted order."""
+    return sorted({tuple(sorted(int(x) for x in row)) for row in emb})
 
 
 def count_totals(Q, D, mode: int = FIND_ALL, nthreads: int | None = None, chunk: int = 100_000):

@@ -35,6 +35,11 @@
  *   step 3b: non[i] = {j < i : (pi_j, pi_i) not in E_q}
  *   step 4b: require no data edge between f(pi_j) and v for j in non[i].
  *
+ * Enumerate mode (NLSM outputs the embeddings themselves,
+ * P:446-453, and atom typing needs every isomorphism): the same
+ * search, but step 5 appends the leaf's mapping f, written in query node
+ * order (f[pi_i] = map[i]), to the caller's buffer instead of counting it.
+ *
  * Threads (std pthreads) split the data graphs into static contiguous chunks
  * and write independent per-pair slots, so results are deterministic.
  * Counts are u64; an addition that would overflow sets *overflow (R19).
@@ -120,6 +125,8 @@ static int build_plan(const oracle_batch *Q, int64_t q, qplan *P) {
 typedef struct {
   const qplan *P;
   int ng;
+  int32_t *emb;         /* enumerate mode: embeddings [cap][n] (query node order), else NULL */
+  int64_t emb_cap, emb_n;
   const uint8_t *glab;  /* [ng] */
   const int16_t *adjm;  /* [ng*ng], -1 = no edge, else bond label */
   int map[64];
@@ -132,7 +139,14 @@ typedef struct {
 
 static uint64_t rec(search *S, int depth) {
   S->work++;
-  if (depth == S->P->n) return 1;
+  if (depth == S->P->n) {
+    if (S->emb) { /* enumerate mode: record f in query node order */
+      if (S->emb_n < S->emb_cap)
+        for (int i = 0; i < S->P->n; i++) S->emb[S->emb_n * S->P->n + S->P->order[i]] = S->map[i];
+      S->emb_n++;
+    }
+    return 1;
+  }
   uint64_t total = 0;
   for (int v = 0; v < S->ng; v++) {
     if (S->used[v] || S->glab[v] != S->P->label[depth]) continue;
@@ -202,6 +216,8 @@ static uint64_t count_one(job *J, const qplan *P, int ng, const uint8_t *glab, c
   S.induced = (J->find_first >> 1) & 1;
   S.overflow = 0;
   S.work = 0;
+  S.emb = NULL;
+  S.emb_cap = S.emb_n = 0;
   memset(S.used, 0, sizeof(S.used));
   uint64_t c = rec(&S, 0);
   J->work += S.work;
@@ -310,5 +326,42 @@ int oracle_count_pairs(const oracle_batch *Q, const oracle_batch *D, int mode, i
   int rc = run_jobs(jobs, nthreads, pair_worker, work_out, overflow_out);
   free(jobs);
   free(plans);
+  return rc;
+}
+
+/* Enumerate mode: every embedding f of query q in data graph g (Find All;
+ * mode bit 1 = induced).  out[k * n_q + i] = molecule-local data node of
+ * query node i in the k-th embedding, for k < cap; *n = the number of
+ * embeddings (may exceed cap: call again with a larger buffer).  Returns 0
+ * on success. */
+int oracle_enumerate_pair(const oracle_batch *Q, const oracle_batch *D, int64_t q, int64_t g, int mode,
+                          int32_t *out, int64_t cap, int64_t *n) {
+  if (q < 0 || q >= Q->num_graphs || g < 0 || g >= D->num_graphs) return -1;
+  qplan *P = (qplan *)malloc(sizeof(qplan));
+  if (build_plan(Q, q, P)) { free(P); return -1; }
+  uint8_t glab[256];
+  int16_t *adjm = (int16_t *)malloc(sizeof(int16_t) * 256 * 256);
+  int ng = 0;
+  int rc = load_graph(D, g, glab, adjm, &ng);
+  *n = 0;
+  if (rc == 0 && P->n <= ng) { /* step 1 */
+    search S;
+    S.P = P;
+    S.ng = ng;
+    S.glab = glab;
+    S.adjm = adjm;
+    S.find_first = 0;
+    S.induced = (mode >> 1) & 1;
+    S.overflow = 0;
+    S.work = 0;
+    S.emb = out;
+    S.emb_cap = cap;
+    S.emb_n = 0;
+    memset(S.used, 0, sizeof(S.used));
+    rec(&S, 0);
+    *n = S.emb_n;
+  }
+  free(adjm);
+  free(P);
   return rc;
 }

@@ -17,7 +17,7 @@ from paper_conf_sc_carocfc25_b200 import stream
 pytestmark = pytest.mark.gpu
 
 CHUNK = 100_000
-IND = 4  # oracle mode bit 2: induced-subgraph embeddings (R21)
+IND = oracle.INDUCED  # induced-subgraph embeddings (R21)
 
 
 @pytest.fixture(scope="module")

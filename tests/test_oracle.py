@@ -268,3 +268,52 @@ def test_induced_vs_networkx_molecules():
             assert res[qi, g] == c, (qi, g)
             total += c
     assert total > 0
+
+
+# ---------------------------------------------------------------- N1 enumerate mode
+def test_enumerate_vs_brute_force_random_tiny():
+    """Enumerate mode (NLSM P:446-453): the set of mappings
+    equals brute-force enumeration of injective tuples (Def. 2.1 conditions
+    (1)-(2), bond labels), monomorphic and induced, on random tiny graphs."""
+    from oracle.brute import brute_embeddings
+    rng = np.random.default_rng(777)
+    n_emb = 0
+    for it in range(400):
+        d = synth.random_labelled_graph(rng, int(rng.integers(1, 8)), float(rng.uniform(0.2, 0.8)),
+                                        labels=(C, N), bonds=(1, 2))
+        q = synth.random_labelled_graph(rng, int(rng.integers(1, 5)), float(rng.uniform(0.3, 1.0)),
+                                        labels=(C, N), bonds=(1, 2))
+        Q, D = GraphBatch.from_graphs([q]), GraphBatch.from_graphs([d])
+        for induced in (False, True):
+            got = oracle.enumerate_pair(Q, D, 0, 0, oracle.INDUCED if induced else oracle.FIND_ALL)
+            ref = sorted(brute_embeddings(q, d, induced))
+            assert sorted(map(tuple, got.tolist())) == ref, (it, induced)
+            assert len(got) == len(set(map(tuple, got.tolist())))  # no mapping twice
+            n_emb += len(ref)
+    assert n_emb > 300
+
+
+def test_enumerate_closed_forms():
+    """Benzene: the 12 embeddings of the aromatic 6-ring are the 12
+    automorphisms of C6 and form ONE node set (NLSM's X); naphthalene: 24
+    embeddings, 2 node sets (the two rings); a single bond C-C in propane:
+    2|E| = 4 mappings, 2 node sets."""
+    benzene = ring(6, C, 4)
+    got = oracle.enumerate_pair(GraphBatch.from_graphs([benzene]), GraphBatch.from_graphs([benzene]), 0, 0)
+    assert len(got) == 12 and oracle.node_sets(got) == [(0, 1, 2, 3, 4, 5)]
+    # every embedding is a rotation or reflection of the ring
+    for f in got.tolist():
+        step = (f[1] - f[0]) % 6
+        assert step in (1, 5) and all((f[i + 1] - f[i]) % 6 == step for i in range(5))
+    naph = naphthalene()
+    got = oracle.enumerate_pair(GraphBatch.from_graphs([benzene]), GraphBatch.from_graphs([naph]), 0, 0)
+    assert len(got) == 24 and len(oracle.node_sets(got)) == 2
+    got = oracle.enumerate_pair(GraphBatch.from_graphs([path(2)]), GraphBatch.from_graphs([path(3)]), 0, 0)
+    assert sorted(map(tuple, got.tolist())) == [(0, 1), (1, 0), (1, 2), (2, 1)]
+    assert oracle.node_sets(got) == [(0, 1), (1, 2)]
+    # consistent with the counting mode on a molecule sample
+    Q, D = synth.config_queries(1), synth.config_data(1, count=20)
+    dense = oracle.count_dense(Q, D)
+    for q in range(Q.num_graphs):
+        for g in range(D.num_graphs):
+            assert len(oracle.enumerate_pair(Q, D, q, g)) == dense[q, g]
