@@ -183,6 +183,37 @@ SIGMO_API sigmo_status sigmo_get_candidates(sigmo_ctx *ctx, uint32_t *out);
  * Host out[V] u64.  Requires load_batch only. */
 SIGMO_API sigmo_status sigmo_get_signatures(sigmo_ctx *ctx, int which, int radius, uint64_t *out);
 
+/* ---- Embedding enumeration ----
+ * NLSM's literal output is the set of embeddings X and atom typing
+ * needs every isomorphism, not a count.  sigmo_enumerate runs, on
+ * the device, a Find All count pass of the join, a prefix sum of the per-pair
+ * counts (each pair's first slot) and a write pass in which every leaf of the
+ * DFS writes its mapping f.  flags SIGMO_ENUM_NODE_SETS also forms, per pair,
+ * the distinct node sets f(V_q) (automorphic images collapse to one set) as
+ * molecule-local 64-bit masks.  Requires sigmo_filter (levels of the caller's
+ * choice, without the neighbour-support flag) on the lane path: every data
+ * graph <= 64 atoms and every query <= 11 nodes; else SIGMO_ERR_LIMIT.  The
+ * per-pair results of the last join are the Find All counts afterwards.
+ * *num_embeddings (nullable) = the total.  Device memory: stride (8 bytes for
+ * queries <= 8 nodes, else 16) per embedding, + 8 with node sets. */
+enum { SIGMO_ENUM_NODE_SETS = 1u << 0 };
+SIGMO_API sigmo_status sigmo_enumerate(sigmo_ctx *ctx, uint32_t flags, int64_t *num_embeddings);
+/* Copy the embeddings of the last sigmo_enumerate to the host, pairs in the
+ * order of sigmo_get_pair_results (data graph, then query).  Call with NULL
+ * arrays to get *num_pairs, *num_embeddings and *stride.  Then
+ * data_idx/query_idx[num_pairs], emb_offsets[num_pairs+1] (embeddings of pair
+ * k are [emb_offsets[k], emb_offsets[k+1])), maps[num_embeddings * stride]:
+ * byte i of an embedding = molecule-local index of the data node that query
+ * node i maps to (0xff.. padding beyond the query's size is 0). */
+SIGMO_API sigmo_status sigmo_get_embeddings(sigmo_ctx *ctx, int64_t pair_cap, int64_t *num_pairs, int64_t *data_idx,
+                                            int32_t *query_idx, int64_t *emb_offsets, int64_t emb_cap, uint8_t *maps,
+                                            int64_t *num_embeddings, int32_t *stride);
+/* The distinct node sets (SIGMO_ENUM_NODE_SETS), same pair order: bit j of a
+ * set = molecule-local data node j; sets of a pair ascending.  NULL arrays:
+ * sizes only. */
+SIGMO_API sigmo_status sigmo_get_node_sets(sigmo_ctx *ctx, int64_t pair_cap, int64_t *num_pairs, int64_t *set_offsets,
+                                           int64_t set_cap, uint64_t *sets, int64_t *num_sets);
+
 /* Read back the CSR-GO batch as the library packed it on the device
  * (section 4.1; Fig. 3): which = 0 queries, 1 data.
  * sizes: *num_graphs, *num_nodes, *num_adj (adjacency entries, both

@@ -234,6 +234,44 @@ class Context:
             nl.ctypes.data_as(P(ctypes.c_uint8)), el.ctypes.data_as(P(ctypes.c_uint8))), "sigmo_get_packed_batch")
         return go, ro, co, nl, el
 
+    def enumerate(self, node_sets: bool = False) -> int:
+        """sigmo_enumerate: every embedding of every GMCR
+        pair, written on the device; returns the total."""
+        n = ctypes.c_int64(0)
+        self._check(self._lib.sigmo_enumerate(self._handle, _native.SIGMO_ENUM_NODE_SETS if node_sets else 0,
+                                              ctypes.byref(n)), "sigmo_enumerate")
+        return int(n.value)
+
+    def embeddings(self):
+        """(data_idx [P], query_idx [P], offsets [P+1], maps uint8 [n, stride]): pair k's
+        embeddings are maps[offsets[k]:offsets[k+1]], column i = data node of query node i."""
+        P, n, st = ctypes.c_int64(0), ctypes.c_int64(0), ctypes.c_int32(0)
+        null = None
+        self._check(self._lib.sigmo_get_embeddings(self._handle, 0, ctypes.byref(P), null, null, null, 0, null,
+                                                   ctypes.byref(n), ctypes.byref(st)), "sigmo_get_embeddings")
+        di, qi = np.zeros(P.value, np.int64), np.zeros(P.value, np.int32)
+        off, maps = np.zeros(P.value + 1, np.int64), np.zeros((n.value, st.value), np.uint8)
+        Pt = ctypes.POINTER
+        self._check(self._lib.sigmo_get_embeddings(
+            self._handle, P.value, ctypes.byref(P), di.ctypes.data_as(Pt(ctypes.c_int64)),
+            qi.ctypes.data_as(Pt(ctypes.c_int32)), off.ctypes.data_as(Pt(ctypes.c_int64)), n.value,
+            maps.ctypes.data_as(Pt(ctypes.c_uint8)), ctypes.byref(n), ctypes.byref(st)), "sigmo_get_embeddings")
+        return di, qi, off, maps
+
+    def node_sets(self):
+        """(offsets [P+1], sets uint64 [n]) of the distinct node sets per pair
+        (bit j = molecule-local data node j), pairs in embeddings() order."""
+        P, n = ctypes.c_int64(0), ctypes.c_int64(0)
+        self._check(self._lib.sigmo_get_node_sets(self._handle, 0, ctypes.byref(P), None, 0, None, ctypes.byref(n)),
+                    "sigmo_get_node_sets")
+        off, sets = np.zeros(P.value + 1, np.int64), np.zeros(n.value, np.uint64)
+        Pt = ctypes.POINTER
+        self._check(self._lib.sigmo_get_node_sets(self._handle, P.value, ctypes.byref(P),
+                                                  off.ctypes.data_as(Pt(ctypes.c_int64)), n.value,
+                                                  sets.ctypes.data_as(Pt(ctypes.c_uint64)), ctypes.byref(n)),
+                    "sigmo_get_node_sets")
+        return off, sets
+
     def check(self):
         """sigmo_check_join: raise if the last join exceeded an internal capacity."""
         self._check(self._lib.sigmo_check_join(self._handle), "sigmo_check_join")

@@ -14,12 +14,14 @@ STATUS_NAMES = {0: "SIGMO_OK", -1: "SIGMO_ERR_INVALID_ARG", -2: "SIGMO_ERR_INVAL
                 -4: "SIGMO_ERR_STATE", -5: "SIGMO_ERR_OOM", -6: "SIGMO_ERR_CUDA"}
 SIGMO_FIND_ALL = 0
 SIGMO_FIND_FIRST = 1
+SIGMO_ENUM_NODE_SETS = 1
 SIGMO_FILTER_NEIGHBOR_SUPPORT = 1
 
 # every symbol declared in include/sigmo.h
 EXPORTS = ["sigmo_create", "sigmo_load_batch", "sigmo_filter", "sigmo_join", "sigmo_num_pairs",
            "sigmo_get_pair_results", "sigmo_get_dense_results", "sigmo_get_query_totals", "sigmo_get_candidates",
-           "sigmo_get_signatures", "sigmo_get_packed_batch", "sigmo_check_join", "sigmo_set_induced", "sigmo_set_timing",
+           "sigmo_get_signatures", "sigmo_get_packed_batch", "sigmo_check_join", "sigmo_enumerate",
+           "sigmo_get_embeddings", "sigmo_get_node_sets", "sigmo_set_induced", "sigmo_set_timing",
            "sigmo_get_timings", "sigmo_validate_batch",
            "sigmo_last_error", "sigmo_version", "sigmo_destroy"]
 
@@ -82,6 +84,11 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
                                            P(ctypes.c_int64), P(ctypes.c_int64), P(ctypes.c_int32),
                                            P(ctypes.c_uint8), P(ctypes.c_uint8)]
     lib.sigmo_check_join.argtypes = [vp]
+    i64p, i32p = P(ctypes.c_int64), P(ctypes.c_int32)
+    lib.sigmo_enumerate.argtypes = [vp, ctypes.c_uint32, i64p]
+    lib.sigmo_get_embeddings.argtypes = [vp, ctypes.c_int64, i64p, i64p, i32p, i64p, ctypes.c_int64,
+                                         P(ctypes.c_uint8), i64p, i32p]
+    lib.sigmo_get_node_sets.argtypes = [vp, ctypes.c_int64, i64p, i64p, ctypes.c_int64, P(ctypes.c_uint64), i64p]
     lib.sigmo_set_timing.argtypes = [vp, ctypes.c_int]
     lib.sigmo_set_induced.argtypes = [vp, ctypes.c_int]
     lib.sigmo_get_timings.argtypes = [vp, P(sigmo_timings)]

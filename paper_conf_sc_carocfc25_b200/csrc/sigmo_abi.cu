@@ -171,6 +171,11 @@ struct sigmo_ctx {
   Timing timing;
   sigmo_timings last{};
   std::string jit_note;  // last lane-filter specialisation outcome ("compiled", "cached" or why not)
+  // enumerate mode
+  const uint8_t *qp_qn = nullptr;  // [VQ] local query node of each plan position (input arena)
+  DBuf eoff, ecur, emaps, esets, ucnt, uoff, uniq, etmp;
+  int64_t enum_P = -1, enum_total = 0, enum_uniq = -1;
+  int enum_stride = 8;
 };
 
 namespace {
@@ -936,7 +941,8 @@ void free_all(sigmo_ctx *c) {
   c->progs.clear();
   DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
                   &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_rec, &c->pair_cm, &c->pair_result, &c->jcnt,
-                  &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp, &c->ent2, &c->nb4, &c->mrec};
+                  &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp, &c->ent2, &c->nb4, &c->mrec,
+                  &c->eoff, &c->ecur, &c->emaps, &c->esets, &c->ucnt, &c->uoff, &c->uniq, &c->etmp};
   for (DBuf *b : bufs) dfree(c, *b);
 }
 
@@ -1178,6 +1184,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const size_t o_ent = L.take(16 * (size_t)hq.V + 16);
   const size_t o_non = L.take(4 * (size_t)hq.V + 4);  // induced mode: non-adjacent earlier depths per plan position
   const size_t o_qinfo = L.take(4 * (size_t)hq.G + 4);
+  const size_t o_qn = L.take((size_t)hq.V + 16);  // enumerate mode: local query node of each plan position
   const PackedOffsets pd = plan_graphs(L, hd);
   const size_t o_tg0 = L.take(4 * tg0.size());
   const size_t o_tg1 = L.take(4 * tg1.size());
@@ -1280,6 +1287,14 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       ent[i] = e4;
     }
     if (hq.G) memcpy(hb + o_qinfo, plan.qinfo.data(), 4 * (size_t)hq.G);
+    {
+      uint8_t *qn = hb + o_qn;
+      int64_t qq = 0;
+      for (int64_t i = 0; i < hq.V; i++) {
+        while (hq.goff[qq + 1] <= i) qq++;
+        qn[i] = (uint8_t)(plan.row[i] - hq.goff[qq]);
+      }
+    }
     // induced mode (R21): bit j of non[i] = earlier depth j < e not adjacent to depth e
     uint32_t *non = (uint32_t *)(hb + o_non);
     int64_t qn = 0;
@@ -1333,6 +1348,8 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->qp_ent = (const int4 *)(db + o_ent);
   c->qp_non = (const uint32_t *)(db + o_non);
   c->qp_qinfo = (const uint32_t *)(db + o_qinfo);
+  c->qp_qn = (const uint8_t *)(db + o_qn);
+  c->enum_P = -1;
   c->NQ = (int)hq.G;
   c->VQ = (int)hq.V;
   c->EQ = (int)hq.E;
@@ -1684,16 +1701,32 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     timing_mark(c, 4);
   }
   c->last.filter_launches = launches;
+  c->enum_P = -1;
   c->levels = levels;
   c->flags = flags;
   c->state = 2;
   return SIGMO_OK;
 }
 
+namespace {
+// enumerate-mode outputs of the lane join; all null: counting
+struct EnumOut {
+  unsigned char *emaps = nullptr;
+  int estride = 8;
+  unsigned long long *esets = nullptr, *ecur = nullptr;
+};
+sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_out, const EnumOut &eo);
+}  // namespace
+
 sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_out) {
   if (!c) return SIGMO_ERR_INVALID_ARG;
   if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_join before sigmo_filter");
   if (mode != SIGMO_FIND_ALL && mode != SIGMO_FIND_FIRST) return set_err(c, SIGMO_ERR_INVALID_ARG, "bad mode %d", (int)mode);
+  return join_impl(c, mode, total_matches_out, EnumOut());
+}
+
+namespace {
+sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_out, const EnumOut &eo) {
   CUDA_TRY(c, cudaSetDevice(c->device));
   CUDA_TRY(c, cudaMemsetAsync(c->jcnt.p, 0, 8 * ((size_t)c->NQ + 8), c->stream));
   int launches = 0;
@@ -1740,6 +1773,11 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
       // configs[2] (r1 final kernel), FA 6/8/12/16 -> 8.70/8.61/8.81/9.42 ms,
       // FF 7.43/7.27/7.18/7.29 ms
       jp.batchK = mode == SIGMO_FIND_FIRST ? 12 : 8;
+      jp.emaps = eo.emaps;
+      jp.estride = eo.estride;
+      jp.esets = eo.esets;
+      jp.ecur = eo.ecur;
+      jp.qp_qn = c->qp_qn;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
       // two launches: pairs of <= 32-node molecules with 32-bit masks, and
       // the others with 64-bit masks (each finds its range in off[ND]); the
@@ -1799,6 +1837,181 @@ sigmo_status sigmo_join(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_o
     *total_matches_out = s;
   }
   return SIGMO_OK;
+}
+}  // namespace
+
+sigmo_status sigmo_enumerate(sigmo_ctx *c, uint32_t flags, int64_t *num_embeddings) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_enumerate before sigmo_filter");
+  if (flags & ~(uint32_t)SIGMO_ENUM_NODE_SETS) return set_err(c, SIGMO_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
+  if (c->ND > 0 && c->VD > 0 && c->NQ > 0 && !c->mol_filter)
+    return set_err(c, SIGMO_ERR_LIMIT,
+                   "embedding enumeration runs on the lane path: data graphs <= 64 atoms, queries <= %d nodes, "
+                   "filter without the neighbour-support flag",
+                   kJoinLaneMaxQ);
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  // count pass (Find All) -> per-pair counts -> scan -> first slot per pair
+  SIGMO_TRY(join_impl(c, SIGMO_FIND_ALL, nullptr, EnumOut()));
+  SIGMO_TRY(read_join_flags(c));
+  int64_t P = 0;
+  SIGMO_TRY(sigmo_num_pairs(c, &P));
+  SIGMO_TRY(dreserve(c, c->eoff, 8 * ((size_t)P + 1), "embedding offsets"));
+  CUDA_TRY(c, cudaMemsetAsync(c->eoff.p, 0, 8, c->stream));
+  unsigned long long total = 0;
+  if (P > 0) {
+    size_t tb = 0;
+    CUDA_TRY(c, launch_u64_inclusive_sum(nullptr, nullptr, P, nullptr, &tb, c->stream));
+    SIGMO_TRY(dreserve(c, c->etmp, tb, "scan temp"));
+    CUDA_TRY(c, launch_u64_inclusive_sum((const unsigned long long *)c->pair_result.p,
+                                         (unsigned long long *)c->eoff.p + 1, P, c->etmp.p, &tb, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(&total, (unsigned long long *)c->eoff.p + P, 8, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  }
+  const int stride = c->maxq <= 8 ? 8 : 16;
+  const bool sets = (flags & SIGMO_ENUM_NODE_SETS) != 0;
+  if (total > 0) {
+    SIGMO_TRY(dreserve(c, c->emaps, (size_t)stride * total, "embeddings"));
+    SIGMO_TRY(dreserve(c, c->ecur, 8 * (size_t)P, "embedding cursors"));
+    if (sets) SIGMO_TRY(dreserve(c, c->esets, 8 * (size_t)total, "embedding node sets"));
+    CUDA_TRY(c, cudaMemcpyAsync(c->ecur.p, c->eoff.p, 8 * (size_t)P, cudaMemcpyDeviceToDevice, c->stream));
+    // write pass
+    EnumOut eo;
+    eo.emaps = (unsigned char *)c->emaps.p;
+    eo.estride = stride;
+    eo.esets = sets ? (unsigned long long *)c->esets.p : nullptr;
+    eo.ecur = (unsigned long long *)c->ecur.p;
+    SIGMO_TRY(join_impl(c, SIGMO_FIND_ALL, nullptr, eo));
+    SIGMO_TRY(read_join_flags(c));
+  }
+  c->enum_uniq = -1;
+  if (sets && P > 0) {
+    // distinct node sets per pair (NLSM's X)
+    SIGMO_TRY(dreserve(c, c->ucnt, 8 * (size_t)P, "node-set counts"));
+    SIGMO_TRY(dreserve(c, c->uoff, 8 * ((size_t)P + 1), "node-set offsets"));
+    CUDA_TRY(c, launch_nodesets((const unsigned long long *)c->eoff.p, P, (unsigned long long *)c->esets.p,
+                                (unsigned long long *)c->ucnt.p, nullptr, nullptr, c->stream));
+    size_t tb = 0;
+    CUDA_TRY(c, launch_u64_inclusive_sum(nullptr, nullptr, P, nullptr, &tb, c->stream));
+    SIGMO_TRY(dreserve(c, c->etmp, tb, "scan temp"));
+    CUDA_TRY(c, cudaMemsetAsync(c->uoff.p, 0, 8, c->stream));
+    CUDA_TRY(c, launch_u64_inclusive_sum((const unsigned long long *)c->ucnt.p, (unsigned long long *)c->uoff.p + 1,
+                                         P, c->etmp.p, &tb, c->stream));
+    unsigned long long nu = 0;
+    CUDA_TRY(c, cudaMemcpyAsync(&nu, (unsigned long long *)c->uoff.p + P, 8, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    SIGMO_TRY(dreserve(c, c->uniq, 8 * (size_t)std::max<unsigned long long>(nu, 1), "distinct node sets"));
+    CUDA_TRY(c, launch_nodesets((const unsigned long long *)c->eoff.p, P, (unsigned long long *)c->esets.p, nullptr,
+                                (const unsigned long long *)c->uoff.p, (unsigned long long *)c->uniq.p, c->stream));
+    c->enum_uniq = (int64_t)nu;
+  } else if (sets) {
+    c->enum_uniq = 0;
+  }
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  c->enum_P = P;
+  c->enum_total = (int64_t)total;
+  c->enum_stride = stride;
+  if (num_embeddings) *num_embeddings = (int64_t)total;
+  return SIGMO_OK;
+}
+
+namespace {
+// pairs of the lane path in getter order (graph, then query): the internal
+// position of each, as in sigmo_get_pair_results
+sigmo_status lane_pair_order(sigmo_ctx *c, int64_t P, std::vector<int64_t> &pos, std::vector<int64_t> &gidx,
+                             std::vector<int32_t> &qidx) {
+  std::vector<I64x2> off((size_t)c->ND + 1);
+  CUDA_TRY(c, cudaMemcpyAsync(off.data(), c->off.p, sizeof(I64x2) * off.size(), cudaMemcpyDeviceToHost, c->stream));
+  std::vector<int32_t> q((size_t)P + 1);
+  if (P)
+    CUDA_TRY(c, cudaMemcpy2DAsync(q.data(), 4, (const char *)c->pair_rec.p + 4, 16, 4, (size_t)P, cudaMemcpyDeviceToHost,
+                                  c->stream));
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  pos.clear();
+  gidx.clear();
+  qidx.clear();
+  const long long Pn = off[c->ND].a;
+  for (int g = 0; g < c->ND; g++) {
+    long long s0, s1;
+    if (off[g + 1].a > off[g].a) {
+      s0 = off[g].a;
+      s1 = off[g + 1].a;
+    } else {
+      s0 = Pn + off[g].b;
+      s1 = Pn + off[g + 1].b;
+    }
+    for (long long p = s0; p < s1; p++) {
+      pos.push_back(p);
+      gidx.push_back(g);
+      qidx.push_back(q[(size_t)p]);
+    }
+  }
+  return SIGMO_OK;
+}
+
+// copy per-pair segments [seg[p], seg[p+1]) of a device array of `esize`-byte
+// elements to the host in getter order
+sigmo_status copy_segments(sigmo_ctx *c, const DBuf &segs, const DBuf &data, size_t esize, int64_t P,
+                           const std::vector<int64_t> &pos, int64_t cap, int64_t *offsets, void *out,
+                           int64_t *n_out) {
+  std::vector<unsigned long long> seg((size_t)P + 1, 0);
+  if (P) CUDA_TRY(c, cudaMemcpyAsync(seg.data(), segs.p, 8 * ((size_t)P + 1), cudaMemcpyDeviceToHost, c->stream));
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  const int64_t total = P ? (int64_t)seg[(size_t)P] : 0;
+  if (n_out) *n_out = total;
+  if (!out) return SIGMO_OK;
+  if (cap < total) return set_err(c, SIGMO_ERR_INVALID_ARG, "capacity %lld < %lld", (long long)cap, (long long)total);
+  std::vector<unsigned char> h(esize * (size_t)total + 1);
+  if (total) CUDA_TRY(c, cudaMemcpyAsync(h.data(), data.p, esize * (size_t)total, cudaMemcpyDeviceToHost, c->stream));
+  CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+  int64_t o = 0;
+  for (size_t k = 0; k < pos.size(); k++) {
+    const unsigned long long a = seg[(size_t)pos[k]], b = seg[(size_t)pos[k] + 1];
+    if (offsets) offsets[k] = o;
+    memcpy((unsigned char *)out + esize * (size_t)o, h.data() + esize * a, esize * (size_t)(b - a));
+    o += (int64_t)(b - a);
+  }
+  if (offsets) offsets[pos.size()] = o;
+  return SIGMO_OK;
+}
+}  // namespace
+
+sigmo_status sigmo_get_embeddings(sigmo_ctx *c, int64_t pair_cap, int64_t *num_pairs, int64_t *data_idx,
+                                  int32_t *query_idx, int64_t *emb_offsets, int64_t emb_cap, uint8_t *maps,
+                                  int64_t *num_embeddings, int32_t *stride) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  if (c->enum_P < 0 || c->state < 3) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_embeddings before sigmo_enumerate");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  const int64_t P = c->enum_P;
+  if (num_pairs) *num_pairs = P;
+  if (stride) *stride = c->enum_stride;
+  if (num_embeddings) *num_embeddings = c->enum_total;
+  if (!data_idx && !query_idx && !emb_offsets && !maps) return SIGMO_OK;
+  if (pair_cap < P) return set_err(c, SIGMO_ERR_INVALID_ARG, "pair capacity %lld < %lld", (long long)pair_cap, (long long)P);
+  std::vector<int64_t> pos, gi;
+  std::vector<int32_t> qi;
+  SIGMO_TRY(lane_pair_order(c, P, pos, gi, qi));
+  for (size_t k = 0; k < pos.size(); k++) {
+    if (data_idx) data_idx[k] = gi[k];
+    if (query_idx) query_idx[k] = qi[k];
+  }
+  return copy_segments(c, c->eoff, c->emaps, (size_t)c->enum_stride, P, pos, emb_cap, emb_offsets, maps, nullptr);
+}
+
+sigmo_status sigmo_get_node_sets(sigmo_ctx *c, int64_t pair_cap, int64_t *num_pairs, int64_t *set_offsets,
+                                 int64_t set_cap, uint64_t *sets, int64_t *num_sets) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  if (c->enum_P < 0 || c->state < 3 || c->enum_uniq < 0)
+    return set_err(c, SIGMO_ERR_STATE, "sigmo_get_node_sets before sigmo_enumerate(SIGMO_ENUM_NODE_SETS)");
+  CUDA_TRY(c, cudaSetDevice(c->device));
+  const int64_t P = c->enum_P;
+  if (num_pairs) *num_pairs = P;
+  if (num_sets) *num_sets = c->enum_uniq;
+  if (!set_offsets && !sets) return SIGMO_OK;
+  if (pair_cap < P) return set_err(c, SIGMO_ERR_INVALID_ARG, "pair capacity %lld < %lld", (long long)pair_cap, (long long)P);
+  std::vector<int64_t> pos, gi;
+  std::vector<int32_t> qi;
+  SIGMO_TRY(lane_pair_order(c, P, pos, gi, qi));
+  return copy_segments(c, c->uoff, c->uniq, 8, P, pos, set_cap, set_offsets, sets, nullptr);
 }
 
 sigmo_status sigmo_num_pairs(sigmo_ctx *c, int64_t *n) {

@@ -191,6 +191,12 @@ struct JoinParams {
   int induced;                 // 1 = induced-subgraph embeddings (k_join only, R21):
                                // the union of all bonds is staged as adjacency class NB
   const uint32_t *qp_non;      // [VQ] induced mode: mask of the earlier plan depths NOT adjacent to depth e
+  // enumerate mode (k_join_lane); emaps == nullptr: counting
+  unsigned char *emaps;        // [embeddings][estride] molecule-local data node per query node (query node order)
+  int estride;                 // 8 (queries <= 8 nodes) or 16 bytes per embedding
+  unsigned long long *esets;   // [embeddings] node set f(V_q) as a molecule-local bit mask (nullable)
+  unsigned long long *ecur;    // [P] write cursor per pair (= its first embedding slot after the scan)
+  const uint8_t *qp_qn;        // [VQ] local query node of each plan position
 };
 
 // k_pairs: GMCR pair list + per-pair candidate masks
@@ -242,6 +248,13 @@ cudaError_t launch_support(int NW, const SupportParams &p, cudaStream_t st);
 size_t support_smem_bytes(int NW, int NB, int maxq, int NQW);
 cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *temp_bytes, cudaStream_t st);
 cudaError_t launch_chunks(const ChunkParams &p, cudaStream_t st);
+cudaError_t launch_u64_inclusive_sum(const unsigned long long *in, unsigned long long *out, long long n, void *temp,
+                                     size_t *temp_bytes, cudaStream_t st);
+// enumerate mode: uoff == nullptr -> sort each pair's node masks and count the distinct ones (ucnt);
+// else write them at uoff
+cudaError_t launch_nodesets(const unsigned long long *eoff, long long P, unsigned long long *sets,
+                            unsigned long long *ucnt, const unsigned long long *uoff, unsigned long long *uniq,
+                            cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
 cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,

@@ -1300,6 +1300,57 @@ cudaError_t launch_scan(const I64x2 *in, I64x2 *out, int n, void *temp, size_t *
 }
 
 // ===========================================================================
+// Enumerate mode helpers: inclusive sum of the per-pair
+// embedding counts (u64), and the distinct node sets of every pair (NLSM's
+// X = f(V_q)) from its embeddings' molecule-local node masks.
+// ===========================================================================
+cudaError_t launch_u64_inclusive_sum(const unsigned long long *in, unsigned long long *out, long long n, void *temp,
+                                     size_t *temp_bytes, cudaStream_t st) {
+  return cub::DeviceScan::InclusiveSum(temp, *temp_bytes, in, out, n, st);
+}
+
+// one thread per pair: sort its node masks (insertion sort, segments are
+// short; the shared-lane join writes them in any order) and count the distinct
+__global__ void k_nodeset_count(const unsigned long long *eoff, long long P, unsigned long long *sets,
+                                unsigned long long *ucnt) {
+  const long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= P) return;
+  const unsigned long long a = eoff[p], b = eoff[p + 1];
+  for (unsigned long long i = a + 1; i < b; i++) {
+    const unsigned long long x = sets[i];
+    unsigned long long j = i;
+    while (j > a && sets[j - 1] > x) {
+      sets[j] = sets[j - 1];
+      j--;
+    }
+    sets[j] = x;
+  }
+  unsigned long long u = 0;
+  for (unsigned long long i = a; i < b; i++) u += (i == a || sets[i] != sets[i - 1]) ? 1ull : 0ull;
+  ucnt[p] = u;
+}
+
+__global__ void k_nodeset_write(const unsigned long long *eoff, const unsigned long long *uoff, long long P,
+                                const unsigned long long *sets, unsigned long long *uniq) {
+  const long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= P) return;
+  const unsigned long long a = eoff[p], b = eoff[p + 1];
+  unsigned long long o = uoff[p];
+  for (unsigned long long i = a; i < b; i++)
+    if (i == a || sets[i] != sets[i - 1]) uniq[o++] = sets[i];
+}
+
+cudaError_t launch_nodesets(const unsigned long long *eoff, long long P, unsigned long long *sets,
+                            unsigned long long *ucnt, const unsigned long long *uoff, unsigned long long *uniq,
+                            cudaStream_t st) {
+  if (P <= 0) return cudaSuccess;
+  const unsigned blocks = (unsigned)((P + 255) / 256);
+  if (!uoff) k_nodeset_count<<<blocks, 256, 0, st>>>(eoff, P, sets, ucnt);
+  else k_nodeset_write<<<blocks, 256, 0, st>>>(eoff, uoff, P, sets, uniq);
+  return cudaGetLastError();
+}
+
+// ===========================================================================
 // k_chunks: chunk key(g) = floor(pairs_before/PC) + floor(atoms_before/AC)
 // + floor(cm_before/CMC) + floor(g/MC) is non-decreasing; chunk k is the run
 // of graphs with key == k, so every chunk fits the join's smem capacities
@@ -2148,6 +2199,36 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   int4 nrec = zero4;
   MT nR0 = 0;
 
+  // enumerate mode: the embeddings of a leaf step -- the
+  // mapped depths 0..d (map bytes) plus each candidate w of the last depth --
+  // written in query node order at the pair's cursor (count pass + scan set
+  // it to the pair's first slot; several lanes may share a donated pair), and
+  // the node set f(V_q) as a molecule-local bit mask
+  auto emit = [&](MT X, int d, MT used) {
+    unsigned long long r0 = 0ull, r1 = 0ull;
+    for (int j = 0; j <= d; j++) {
+      const unsigned qn = __ldg(&jp.qp_qn[cqb + (unsigned)j]);
+      const unsigned long long b = smem[oM + 32u * (unsigned)j];
+      if (qn < 8u) r0 |= b << (8u * qn);
+      else r1 |= b << (8u * (qn - 8u));
+    }
+    const unsigned qe = __ldg(&jp.qp_qn[cqb + (unsigned)(d + 1)]);
+    unsigned long long pos = atomicAdd(jp.ecur + pbase0 + cp, (unsigned long long)popc(X));
+    while (X) {
+      const unsigned w = (unsigned)lowest(X);
+      X &= X - (MT)1;
+      const unsigned long long a0 = r0 | (qe < 8u ? (unsigned long long)w << (8u * qe) : 0ull);
+      const unsigned long long a1 = r1 | (qe >= 8u ? (unsigned long long)w << (8u * (qe - 8u)) : 0ull);
+      if (jp.estride == 8) {
+        ((unsigned long long *)jp.emaps)[pos] = a0;
+      } else {
+        ((ulonglong2 *)jp.emaps)[pos] = make_ulonglong2(a0, a1);
+      }
+      if (jp.esets) jp.esets[pos] = (unsigned long long)used | (1ull << w);
+      pos++;
+    }
+  };
+
   while (true) {
     // ---- one DFS step ----
     if (ne) {
@@ -2195,6 +2276,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       }
       if (e == (int)(cinfo & 0xff) - 1) {
         cnt += (unsigned long long)popc(X);
+        if ((MODE & 4) && X) emit(X, d, used);  // enumerate mode: write the embeddings
         if ((MODE & 1) && cnt) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
         stRU(oRU + 32u * ES * e, X, used);
@@ -2235,6 +2317,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const MT R0 = nR0;
       if ((cinfo & 0xff) == 1u) {
         cnt = (unsigned long long)popc(R0);
+        if ((MODE & 4) && R0) emit(R0, -1, (MT)0);
         pend = true;
       } else {
         stRU(oRU, R0, (MT)0);
@@ -2356,8 +2439,12 @@ static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_
 
 cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, cudaStream_t st) {
   if (grid <= 0) return cudaSuccess;
-  // mode bit 0: Find First; bit 1: induced (p.induced)
+  // mode bit 0: Find First; bit 1: induced (p.induced); p.emaps: enumerate (Find All semantics)
   const int m = (mode & 1) | (p.induced ? 2 : 0);
+  if (p.emaps) {
+    if (w64) return p.induced ? launch_join_lane_t<6, true>(p, grid, st) : launch_join_lane_t<4, true>(p, grid, st);
+    return p.induced ? launch_join_lane_t<6, false>(p, grid, st) : launch_join_lane_t<4, false>(p, grid, st);
+  }
   if (w64) {
     switch (m) {
       case 0: return launch_join_lane_t<0, true>(p, grid, st);
@@ -2387,8 +2474,12 @@ static int join_lane_occ_t(size_t smem) {
 }
 
 int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem) {
-  // the instantiation launch_join_lane picks: bit 0 Find First, bit 1 induced
+  // the instantiation launch_join_lane picks: bit 0 Find First, bit 1 induced, enumerate
   const int m = (mode & 1) | (p.induced ? 2 : 0);
+  if (p.emaps) {
+    if (w64) return p.induced ? join_lane_occ_t<6, true>(smem) : join_lane_occ_t<4, true>(smem);
+    return p.induced ? join_lane_occ_t<6, false>(smem) : join_lane_occ_t<4, false>(smem);
+  }
   if (w64) {
     switch (m) {
       case 0: return join_lane_occ_t<0, true>(smem);
