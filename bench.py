@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--ns", action="store_true",
+                    help="neighbour-support fixed point in the filter (SIGMO_FILTER_NEIGHBOR_SUPPORT; DESIGN.md R9)")
     ap.add_argument("--induced", action="store_true",
                     help="induced-subgraph embeddings (sigmo_set_induced; SURVEY 8(f) N4, DESIGN.md R21)")
     a = ap.parse_args()
@@ -296,14 +298,16 @@ def main():
     from paper_conf_sc_carocfc25_b200 import sharded
 
     def step(mode=sigmo.SIGMO_FIND_ALL):
-        ctx.filter(args.levels)
+        ctx.filter(args.levels, neighbor_support=args.ns)
         ctx.join(mode, total=False)
         ctx.query_totals(device_tensor=totals)
         sharded.allreduce_totals(totals)  # the only collective: NCCL sum of per-query totals
 
-    # ---- warm-up ----
+    # ---- warm-up (both join modes: the first launch of a kernel instantiation
+    # loads its module, which must not land in a timed step) ----
     for _ in range(max(args.warmup, 3)):
         step()
+    step(sigmo.SIGMO_FIND_FIRST)
     torch.cuda.synchronize(dev)
 
     def timed_loop(mode, K, with_timing):
@@ -345,7 +349,7 @@ def main():
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
         ctx.load_batch(cq, cd)
-        ctx.filter(args.levels)
+        ctx.filter(args.levels, neighbor_support=args.ns)
         tot = ctx.join(sigmo.SIGMO_FIND_ALL, total=True)  # D2H of the per-query totals
         dt = (time.perf_counter() - t0) * 1000
         if i > 0:

@@ -143,9 +143,14 @@ SIGMO_API sigmo_status sigmo_load_batch(sigmo_ctx *ctx, const sigmo_graph_batch 
  * Alg.1 l.29-37); L>=2 also applies signature dominance at radii 1..L-1
  * (GenerateSignatures l.11-18 cumulative per R4, RefineCandidates l.19-28 on
  * every field per R5, saturating fields per R7/R8).  flags: 0 or
- * SIGMO_FILTER_NEIGHBOR_SUPPORT.  Asynchronous, except that the first call
- * for a given `levels` after load_batch synchronizes once to size the
- * query-side plane program. */
+ * SIGMO_FILTER_NEIGHBOR_SUPPORT.  With the flag, the lane path (graphs <= 64
+ * atoms, queries <= 11 nodes) refines the candidate windows of every GMCR
+ * pair to the fixed point (k_support_lane) and the join reads the refined
+ * windows; the general path runs k_support over the dense bitmap.
+ * Asynchronous, except that the first call for a given `levels` after
+ * load_batch synchronizes once to size the query-side plane program, and
+ * the lane-path neighbour-support pass synchronizes once to size its
+ * per-pair window arrays. */
 SIGMO_API sigmo_status sigmo_filter(sigmo_ctx *ctx, int levels, uint32_t flags);
 
 /* Stack-based DFS join over the GMCR pairs (section 4.6).
@@ -190,8 +195,8 @@ SIGMO_API sigmo_status sigmo_get_signatures(sigmo_ctx *ctx, int which, int radiu
  * counts (each pair's first slot) and a write pass in which every leaf of the
  * DFS writes its mapping f.  flags SIGMO_ENUM_NODE_SETS also forms, per pair,
  * the distinct node sets f(V_q) (automorphic images collapse to one set) as
- * molecule-local 64-bit masks.  Requires sigmo_filter (levels of the caller's
- * choice, without the neighbour-support flag) on the lane path: every data
+ * molecule-local 64-bit masks.  Requires sigmo_filter (any levels and flags)
+ * on the lane path: every data
  * graph <= 64 atoms and every query <= 11 nodes; else SIGMO_ERR_LIMIT.  The
  * per-pair results of the last join are the Find All counts afterwards.
  * *num_embeddings (nullable) = the total.  Device memory: stride (8 bytes for

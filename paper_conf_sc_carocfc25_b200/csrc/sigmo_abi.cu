@@ -176,6 +176,12 @@ struct sigmo_ctx {
   DBuf eoff, ecur, emaps, esets, ucnt, uoff, uniq, etmp;
   int64_t enum_P = -1, enum_total = 0, enum_uniq = -1;
   int enum_stride = 8;
+  // neighbour support on the lane path (k_support_lane)
+  bool lane_ns = false;            // the last filter refined per-pair windows (join reads ns_win*)
+  bool ns_lane_ok = true;          // every query node has <= 8 neighbours (k_support_lane's lists)
+  const uint2 *qp_nbr = nullptr;   // [VQ] query neighbours per plan position (input arena)
+  DBuf ns_win32, ns_win64, ns_alive, gm_old, off_old, ent_ns, ns_bitmap, ns_gm, ns_cnt;
+  std::vector<uint2> ent_ns_up;    // plan entries whose row field is the plan depth (windows per pair)
 };
 
 namespace {
@@ -942,7 +948,9 @@ void free_all(sigmo_ctx *c) {
   DBuf *bufs[] = {&c->arena, &c->qcounts, &c->bitmap, &c->gm, &c->mol_cnt, &c->off, &c->scan_tmp,
                   &c->chunk_start, &c->nchunks, &c->pair_query, &c->pair_rec, &c->pair_cm, &c->pair_result, &c->jcnt,
                   &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp, &c->ent2, &c->nb4, &c->mrec,
-                  &c->eoff, &c->ecur, &c->emaps, &c->esets, &c->ucnt, &c->uoff, &c->uniq, &c->etmp};
+                  &c->eoff, &c->ecur, &c->emaps, &c->esets, &c->ucnt, &c->uoff, &c->uniq, &c->etmp,
+                  &c->ns_win32, &c->ns_win64, &c->ns_alive, &c->gm_old, &c->off_old, &c->ent_ns, &c->ns_bitmap,
+                  &c->ns_gm, &c->ns_cnt};
   for (DBuf *b : bufs) dfree(c, *b);
 }
 
@@ -978,6 +986,109 @@ sigmo_status read_join_flags(sigmo_ctx *c) {
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
   c->last.dfs_steps = (int64_t)f[2];
   if ((int)f[1] != 0) return set_err(c, SIGMO_ERR_LIMIT, "join DFS stack capacity exceeded (internal limit)");
+  return SIGMO_OK;
+}
+
+// Dense-tile filter (general path: > 64-atom graphs or > 11-node queries)
+// into `bitmap` [VQ][Wpad] with its GMCR bits and counts, plus the
+// neighbour-support pass on it (flag).  Also the dense view of the
+// neighbour-support bitmap for sigmo_get_candidates on the lane path.
+sigmo_status launch_dense(sigmo_ctx *c, int R, const QueryProg &P, uint32_t *bitmap, uint32_t *gm, I64x2 *mol_cnt,
+                          bool ns, int &launches) {
+  const QueryProgMeta &m = P.meta;
+  if (!c->tile_geom_ok) {
+    HostGraphs hg;
+    hg.G = c->ND;
+    hg.V = c->VD;
+    hg.goff = c->goff_host.data();
+    tile_geometry(c, hg);
+    c->tile_geom_ok = true;
+  }
+  const int tws[6] = {32, 16, 8, 4, 2, 1};
+  int k = 0, rows_smem = 1;
+  size_t smem = 0;
+  for (k = 0; k < 12; k++) {
+    rows_smem = k < 6 ? 1 : 0;
+    const int kk = k % 6;
+    smem = filter_smem_bytes(c->NW, c->tile_extn[kk], c->tile_extw[kk], c->tile_molcap[kk], m.NFU, m.NLAB, m.P, m.NREC,
+                             c->VQ, m.NRP, rows_smem, c->NQW, m.TS, 0);
+    // prefer >= 2 CTAs per SM with row programs in shared memory
+    if (smem <= (rows_smem ? c->max_smem / 2 : c->max_smem)) break;
+  }
+  if (k == 12) return set_err(c, SIGMO_ERR_LIMIT, "filter shared memory %zu exceeds %zu (P=%d)", smem, c->max_smem, m.P);
+  k = k % 6;
+  if (c->has_empty_graph) {
+    CUDA_TRY(c, cudaMemsetAsync(gm, 0, 4 * (size_t)c->ND * c->NQW, c->stream));
+    CUDA_TRY(c, cudaMemsetAsync(mol_cnt, 0, sizeof(I64x2) * ((size_t)c->ND + 1), c->stream));
+  }
+    FilterParams fp{};
+    fp.D = c->dd;
+    fp.TW = tws[k];
+    fp.W = c->W;
+    fp.Wpad = c->Wpad;
+    fp.VQ = c->VQ;
+    fp.NQ = c->NQ;
+    fp.NQW = c->NQW;
+    fp.R = R;
+    fp.P = m.P;
+    fp.NFU = m.NFU;
+    fp.NLAB = m.NLAB;
+    fp.NREC = m.NREC;
+    fp.NRP = m.NRP;
+    fp.NBATCH = m.NBATCH;
+    fp.RW = m.RW;
+    fp.TS = m.TS;
+    fp.grec = P.grec;
+    fp.rrec_off = P.rrec_off;
+    fp.rcarry = P.rcarry;
+    fp.bdone = P.bdone;
+    fp.tab = P.tab;
+    fp.fslot = P.fslot;
+    fp.lab_val = P.lab_val;
+    fp.rowp_off = P.rowp_off;
+    fp.rowp = P.rowp;
+    fp.qgoff = c->dq.goff;
+    fp.bitmap = bitmap;
+    fp.gm = gm;
+    fp.mol_cnt = mol_cnt;
+    fp.EXTN = c->tile_extn[k];
+    fp.EXTW = c->tile_extw[k];
+    fp.MOLCAP = c->tile_molcap[k];
+    fp.tile_g0 = tws[k] == 32 ? c->tile_g0 : nullptr;
+    fp.tile_g1 = tws[k] == 32 ? c->tile_g1 : nullptr;
+    fp.cmol = nullptr;
+    fp.rows_smem = rows_smem;
+    fp.smem_bytes = smem;
+    const int tiles = (c->W + fp.TW - 1) / fp.TW;
+    if (getenv("SIGMO_DEBUG_FILTER"))
+      fprintf(stderr, "sigmo filter (dense): smem=%zu EXTN=%d EXTW=%d NFU=%d NLAB=%d P=%d NREC=%d TS=%d RW=%d tiles=%d\n",
+              smem, fp.EXTN, fp.EXTW, m.NFU, m.NLAB, m.P, m.NREC, m.TS, m.RW, tiles);
+    timing_mark(c, 2);
+    CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));
+    launches++;
+    if (ns) {
+      SupportParams sp{};
+      sp.ND = c->ND;
+      sp.NQ = c->NQ;
+      sp.NQW = c->NQW;
+      sp.NB = c->NB;
+      sp.maxq = std::max(c->maxq, 1);
+      sp.Wpad = c->Wpad;
+      sp.goff = c->dd.goff;
+      sp.roff = c->dd.roff;
+      sp.nbr = c->dd.nbr;
+      sp.bclass = c->bclass;
+      sp.qgoff = c->dq.goff;
+      sp.qroff = c->dq.roff;
+      sp.qnbr = c->dq.nbr;
+      sp.bitmap = bitmap;
+      sp.gm = gm;
+      sp.mol_cnt = mol_cnt;
+      if (support_smem_bytes(c->NW, c->NB, sp.maxq, c->NQW) > c->max_smem)
+        return set_err(c, SIGMO_ERR_LIMIT, "neighbour-support shared memory exceeds the device limit");
+      CUDA_TRY(c, launch_support(c->NW, sp, c->stream));
+      launches++;
+    }
   return SIGMO_OK;
 }
 
@@ -1185,6 +1296,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const size_t o_non = L.take(4 * (size_t)hq.V + 4);  // induced mode: non-adjacent earlier depths per plan position
   const size_t o_qinfo = L.take(4 * (size_t)hq.G + 4);
   const size_t o_qn = L.take((size_t)hq.V + 16);  // enumerate mode: local query node of each plan position
+  const size_t o_qnb = L.take(8 * (size_t)hq.V + 16);  // lane neighbour support: query neighbours per plan position
   const PackedOffsets pd = plan_graphs(L, hd);
   const size_t o_tg0 = L.take(4 * tg0.size());
   const size_t o_tg1 = L.take(4 * tg1.size());
@@ -1288,6 +1400,33 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     }
     if (hq.G) memcpy(hb + o_qinfo, plan.qinfo.data(), 4 * (size_t)hq.G);
     {
+      // neighbours (plan depth | bond class << 4 | 0x80) of each plan position, <= 8
+      uint2 *qnb = (uint2 *)(hb + o_qnb);
+      std::vector<uint8_t> cnt((size_t)hq.V, 0);
+      c->ns_lane_ok = true;
+      for (int64_t i = 0; i < hq.V; i++) qnb[i] = make_uint2(0u, 0u);
+      auto put = [&](int64_t pos, uint32_t depth, uint32_t cls) {
+        const int k = cnt[(size_t)pos]++;
+        if (k >= 8) {
+          c->ns_lane_ok = false;
+          return;
+        }
+        const uint32_t b = (depth & 15u) | ((cls & 7u) << 4) | 0x80u;
+        if (k < 4) qnb[pos].x |= b << (8 * k);
+        else qnb[pos].y |= b << (8 * (k - 4));
+      };
+      int64_t qq = 0;
+      for (int64_t i = 0; i < hq.V; i++) {
+        while (hq.goff[qq + 1] <= i) qq++;
+        const int64_t lo = hq.goff[qq];
+        for (int k = plan.beoff[i]; k < plan.beoff[i + 1]; k++) {
+          const uint32_t j = plan.be[k] >> 8, cls = plan.be[k] & 255u;
+          put(i, j, cls);                                        // i's back-edge to depth j
+          put(lo + j, (uint32_t)(i - lo), cls);                  // and the forward edge of depth j
+        }
+      }
+    }
+    {
       uint8_t *qn = hb + o_qn;
       int64_t qq = 0;
       for (int64_t i = 0; i < hq.V; i++) {
@@ -1349,6 +1488,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->qp_non = (const uint32_t *)(db + o_non);
   c->qp_qinfo = (const uint32_t *)(db + o_qinfo);
   c->qp_qn = (const uint8_t *)(db + o_qn);
+  c->qp_nbr = (const uint2 *)(db + o_qnb);
   c->enum_P = -1;
   c->NQ = (int)hq.G;
   c->VQ = (int)hq.V;
@@ -1463,33 +1603,14 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
   int launches = 0;
   if (c->ND > 0 && c->VD > 0) {
     const QueryProgMeta &m = prog->meta;
-    // lane path (cmol layout for the per-lane join, k_filter_lane) unless the
-    // neighbour-support pass (dense bitmap) is requested
-    bool mol = c->lane_join && !(flags & SIGMO_FILTER_NEIGHBOR_SUPPORT);
-    const int tws[6] = {32, 16, 8, 4, 2, 1};
-    int k = 0;
-    size_t smem = 0;
-    int rows_smem = 1;
-    if (!mol && !c->tile_geom_ok) {
-      HostGraphs hg;
-      hg.G = c->ND;
-      hg.V = c->VD;
-      hg.goff = c->goff_host.data();
-      tile_geometry(c, hg);
-      c->tile_geom_ok = true;
-    }
-    if (!mol) {
-      for (k = 0; k < 12; k++) {
-        rows_smem = k < 6 ? 1 : 0;
-        const int kk = k % 6;
-        smem = filter_smem_bytes(c->NW, c->tile_extn[kk], c->tile_extw[kk], c->tile_molcap[kk], m.NFU, m.NLAB, m.P,
-                                 m.NREC, c->VQ, m.NRP, rows_smem, c->NQW, m.TS, 0);
-        // prefer >= 2 CTAs per SM with row programs in shared memory
-        if (smem <= (rows_smem ? c->max_smem / 2 : c->max_smem)) break;
-      }
-      if (k == 12) return set_err(c, SIGMO_ERR_LIMIT, "filter shared memory %zu exceeds %zu (P=%d)", smem, c->max_smem, m.P);
-      k = k % 6;
-    }
+    // lane path (cmol layout for the per-lane join, k_filter_lane; the
+    // neighbour-support pass on it refines per-pair windows, k_support_lane)
+    // or the dense tiles of the general path
+    const bool mol = c->lane_join;
+    const bool lane_ns = mol && (flags & SIGMO_FILTER_NEIGHBOR_SUPPORT) != 0;
+    c->lane_ns = false;
+    if (lane_ns && !c->ns_lane_ok)
+      return set_err(c, SIGMO_ERR_LIMIT, "neighbour support on the lane path: a query node has more than 8 neighbours");
     c->mol_filter = mol;
     if (mol) {
       c->dense_pad_zero = false;  // the molecule-padded layout overwrites the dense padding
@@ -1516,6 +1637,20 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       if (!c->ent_up.empty())
         CUDA_TRY(c, cudaMemcpyAsync(c->ent2.p, c->ent_up.data(), sizeof(uint2) * c->ent_up.size(),
                                     cudaMemcpyHostToDevice, c->stream));
+      // neighbour-support mode: the join reads per-pair windows in plan-depth order
+      c->ent_ns_up = c->ent_up;
+      {
+        int64_t q = 0;
+        for (size_t i = 0; i < c->ent_ns_up.size(); i++) {
+          while (c->qgoff_host[q + 1] <= (int64_t)i) q++;
+          c->ent_ns_up[i].x = (c->ent_ns_up[i].x & 0xfffu) | ((unsigned)(i - c->qgoff_host[q]) << 12);
+        }
+      }
+      SIGMO_TRY(dreserve(c, c->ent_ns, sizeof(uint2) * (c->ent_ns_up.size() + 1), "plan entries (support)"));
+      if (!c->ent_ns_up.empty())
+        CUDA_TRY(c, cudaMemcpyAsync(c->ent_ns.p, c->ent_ns_up.data(), sizeof(uint2) * c->ent_ns_up.size(),
+                                    cudaMemcpyHostToDevice, c->stream));
+      CUDA_TRY(c, cudaStreamSynchronize(c->stream));  // the host vectors may change before the copies ran
       c->ent_R = R;
     }
     if (c->has_empty_graph) {
@@ -1592,74 +1727,8 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       else CUDA_TRY(c, launch_filter_lane(lp, grid, c->stream));
       launches++;
     } else {
-    FilterParams fp{};
-    fp.D = c->dd;
-    fp.TW = tws[k];
-    fp.W = c->W;
-    fp.Wpad = c->Wpad;
-    fp.VQ = c->VQ;
-    fp.NQ = c->NQ;
-    fp.NQW = c->NQW;
-    fp.R = R;
-    fp.P = m.P;
-    fp.NFU = m.NFU;
-    fp.NLAB = m.NLAB;
-    fp.NREC = m.NREC;
-    fp.NRP = m.NRP;
-    fp.NBATCH = m.NBATCH;
-    fp.RW = m.RW;
-    fp.TS = m.TS;
-    fp.grec = prog->grec;
-    fp.rrec_off = prog->rrec_off;
-    fp.rcarry = prog->rcarry;
-    fp.bdone = prog->bdone;
-    fp.tab = prog->tab;
-    fp.fslot = prog->fslot;
-    fp.lab_val = prog->lab_val;
-    fp.rowp_off = prog->rowp_off;
-    fp.rowp = prog->rowp;
-    fp.qgoff = c->dq.goff;
-    fp.bitmap = (uint32_t *)c->bitmap.p;
-    fp.gm = (uint32_t *)c->gm.p;
-    fp.mol_cnt = (I64x2 *)c->mol_cnt.p;
-    fp.EXTN = c->tile_extn[k];
-    fp.EXTW = c->tile_extw[k];
-    fp.MOLCAP = c->tile_molcap[k];
-    fp.tile_g0 = tws[k] == 32 ? c->tile_g0 : nullptr;
-    fp.tile_g1 = tws[k] == 32 ? c->tile_g1 : nullptr;
-    fp.cmol = nullptr;
-    fp.rows_smem = rows_smem;
-    fp.smem_bytes = smem;
-    const int tiles = (c->W + fp.TW - 1) / fp.TW;
-    if (getenv("SIGMO_DEBUG_FILTER"))
-      fprintf(stderr, "sigmo filter (dense): smem=%zu EXTN=%d EXTW=%d NFU=%d NLAB=%d P=%d NREC=%d TS=%d RW=%d tiles=%d\n",
-              smem, fp.EXTN, fp.EXTW, m.NFU, m.NLAB, m.P, m.NREC, m.TS, m.RW, tiles);
-    timing_mark(c, 2);
-    CUDA_TRY(c, launch_filter(c->NW, fp, tiles, c->stream));
-    launches++;
-    }
-    if (flags & SIGMO_FILTER_NEIGHBOR_SUPPORT) {
-      SupportParams sp{};
-      sp.ND = c->ND;
-      sp.NQ = c->NQ;
-      sp.NQW = c->NQW;
-      sp.NB = c->NB;
-      sp.maxq = std::max(c->maxq, 1);
-      sp.Wpad = c->Wpad;
-      sp.goff = c->dd.goff;
-      sp.roff = c->dd.roff;
-      sp.nbr = c->dd.nbr;
-      sp.bclass = c->bclass;
-      sp.qgoff = c->dq.goff;
-      sp.qroff = c->dq.roff;
-      sp.qnbr = c->dq.nbr;
-      sp.bitmap = (uint32_t *)c->bitmap.p;
-      sp.gm = (uint32_t *)c->gm.p;
-      sp.mol_cnt = (I64x2 *)c->mol_cnt.p;
-      if (support_smem_bytes(c->NW, c->NB, sp.maxq, c->NQW) > c->max_smem)
-        return set_err(c, SIGMO_ERR_LIMIT, "neighbour-support shared memory exceeds the device limit");
-      CUDA_TRY(c, launch_support(c->NW, sp, c->stream));
-      launches++;
+      SIGMO_TRY(launch_dense(c, R, *prog, (uint32_t *)c->bitmap.p, (uint32_t *)c->gm.p, (I64x2 *)c->mol_cnt.p,
+                             (flags & SIGMO_FILTER_NEIGHBOR_SUPPORT) != 0, launches));
     }
     timing_mark(c, 3);
     size_t tb = c->scan_tmp_bytes;
@@ -1698,6 +1767,47 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
     pp.qinfo = c->qp_qinfo;
     CUDA_TRY(c, launch_pairs(pp, c->stream));
     launches++;
+    if (lane_ns) {
+      // neighbour support on the pre-support pair list: refined windows per
+      // pair + alive flags, then the GMCR bits, counts and records again
+      const size_t gmb = 4 * (size_t)c->ND * c->NQW, offb = sizeof(I64x2) * ((size_t)c->ND + 1);
+      SIGMO_TRY(dreserve(c, c->gm_old, gmb, "pre-support gmcr bits"));
+      SIGMO_TRY(dreserve(c, c->off_old, offb, "pre-support offsets"));
+      CUDA_TRY(c, cudaMemcpyAsync(c->gm_old.p, c->gm.p, gmb, cudaMemcpyDeviceToDevice, c->stream));
+      CUDA_TRY(c, cudaMemcpyAsync(c->off_old.p, c->off.p, offb, cudaMemcpyDeviceToDevice, c->stream));
+      I64x2 pt{};
+      CUDA_TRY(c, cudaMemcpyAsync(&pt, (const I64x2 *)c->off.p + c->ND, sizeof(I64x2), cudaMemcpyDeviceToHost, c->stream));
+      CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+      const int MQ = std::max(c->maxq, 1);
+      SIGMO_TRY(dreserve(c, c->ns_win32, 4 * (size_t)std::max<long long>(pt.a, 1) * MQ, "support windows"));
+      SIGMO_TRY(dreserve(c, c->ns_win64, 8 * (size_t)std::max<long long>(pt.b, 1) * MQ, "support windows (wide)"));
+      SIGMO_TRY(dreserve(c, c->ns_alive, (size_t)(pt.a + pt.b + 1), "support flags"));
+      SupportLaneParams sl{};
+      sl.Pn = pt.a;
+      sl.Pw = pt.b;
+      sl.prec = (const int4 *)c->pair_rec.p;
+      sl.cmol = (const uint32_t *)c->bitmap.p;
+      sl.adjw = (const uint32_t *)c->adjb.p;
+      sl.qp_ent2 = (const uint2 *)c->ent2.p;
+      sl.qp_be = c->qp_be;
+      sl.qp_nbr = c->qp_nbr;
+      sl.MQ = MQ;
+      sl.win32 = (uint32_t *)c->ns_win32.p;
+      sl.win64 = (unsigned long long *)c->ns_win64.p;
+      sl.alive = (uint8_t *)c->ns_alive.p;
+      CUDA_TRY(c, launch_support_lane(sl, c->stream));
+      CUDA_TRY(c, launch_gmcr_update(c->ND, c->NQW, (const uint32_t *)c->gm_old.p, (const I64x2 *)c->off_old.p,
+                                     c->dd.goff, (const uint8_t *)c->ns_alive.p, (uint32_t *)c->gm.p,
+                                     (I64x2 *)c->mol_cnt.p, c->stream));
+      size_t tb2 = c->scan_tmp_bytes;
+      CUDA_TRY(c, launch_scan((const I64x2 *)c->mol_cnt.p, (I64x2 *)c->off.p, c->ND + 1, c->scan_tmp.p, &tb2, c->stream));
+      pp.gm_old = (const uint32_t *)c->gm_old.p;
+      pp.off_old = (const I64x2 *)c->off_old.p;
+      pp.ns_mq = MQ;
+      CUDA_TRY(c, launch_pairs(pp, c->stream));
+      launches += 4;
+      c->lane_ns = true;
+    }
     timing_mark(c, 4);
   }
   c->last.filter_launches = launches;
@@ -1767,7 +1877,7 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
       jp.adjw = (const uint32_t *)c->adjb.p;
       jp.adj_ones = c->adj_words;
       jp.qp_ent = c->qp_ent;
-      jp.qp_ent2 = (const uint2 *)c->ent2.p;
+      jp.qp_ent2 = (const uint2 *)(c->lane_ns ? c->ent_ns.p : c->ent2.p);
       jp.cmol = (const uint32_t *)c->bitmap.p;
       // refill batch (lanes that must be free before a warp refills): swept on
       // configs[2] (r1 final kernel), FA 6/8/12/16 -> 8.70/8.61/8.81/9.42 ms,
@@ -1797,6 +1907,8 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
           return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
         jp.smem_bytes = smem;
         jp.chunk_counter = (int *)((unsigned long long *)c->jcnt.p + (w64 ? 6 + (size_t)c->NQ : 0));
+        // neighbour-support mode: the refined windows of each pair (plan-depth order)
+        if (c->lane_ns) jp.cmol = (const uint32_t *)(w64 ? c->ns_win64.p : c->ns_win32.p);
         int bps = join_lane_blocks_per_sm((int)mode, w64, jp, smem);
         if (const char *e = getenv("SIGMO_JOIN_BPS")) bps = std::max(1, std::min(bps, atoi(e)));
         const int grid = bps * c->sm_count;
@@ -1846,8 +1958,7 @@ sigmo_status sigmo_enumerate(sigmo_ctx *c, uint32_t flags, int64_t *num_embeddin
   if (flags & ~(uint32_t)SIGMO_ENUM_NODE_SETS) return set_err(c, SIGMO_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
   if (c->ND > 0 && c->VD > 0 && c->NQ > 0 && !c->mol_filter)
     return set_err(c, SIGMO_ERR_LIMIT,
-                   "embedding enumeration runs on the lane path: data graphs <= 64 atoms, queries <= %d nodes, "
-                   "filter without the neighbour-support flag",
+                   "embedding enumeration runs on the lane path: data graphs <= 64 atoms, queries <= %d nodes",
                    kJoinLaneMaxQ);
   CUDA_TRY(c, cudaSetDevice(c->device));
   // count pass (Find All) -> per-pair counts -> scan -> first slot per pair
@@ -2113,7 +2224,19 @@ sigmo_status sigmo_get_candidates(sigmo_ctx *c, uint32_t *out) {
   if (c->state < 2) return set_err(c, SIGMO_ERR_STATE, "sigmo_get_candidates before sigmo_filter");
   if (c->VQ == 0 || c->W == 0) return SIGMO_OK;
   const void *src = c->bitmap.p;
-  if (c->mol_filter) {  // dense view of the molecule-padded layout
+  if (c->lane_ns) {
+    // the neighbour-support fixed point over the whole bitmap (pairs the GMCR
+    // pruned included), by the dense-tile filter + k_support into scratch
+    const size_t bytes = 4 * (size_t)c->VQ * c->Wpad + 64;
+    SIGMO_TRY(dreserve(c, c->ns_bitmap, bytes, "candidate view (support)"));
+    SIGMO_TRY(dreserve(c, c->ns_gm, 4 * (size_t)c->ND * std::max(c->NQW, 1), "scratch gmcr bits"));
+    SIGMO_TRY(dreserve(c, c->ns_cnt, sizeof(I64x2) * ((size_t)c->ND + 1), "scratch gmcr counts"));
+    CUDA_TRY(c, cudaMemsetAsync(c->ns_bitmap.p, 0, bytes, c->stream));
+    int nl = 0;
+    SIGMO_TRY(launch_dense(c, c->levels - 1, c->progs[c->levels - 1].prog, (uint32_t *)c->ns_bitmap.p,
+                           (uint32_t *)c->ns_gm.p, (I64x2 *)c->ns_cnt.p, true, nl));
+    src = c->ns_bitmap.p;
+  } else if (c->mol_filter) {  // dense view of the molecule-padded layout
     const size_t bytes = 4 * (size_t)c->VQ * c->Wpad;
     SIGMO_TRY(dreserve(c, c->dense_tmp, bytes, "dense candidate view"));
     CUDA_TRY(c, cudaMemsetAsync(c->dense_tmp.p, 0, bytes, c->stream));

@@ -212,6 +212,27 @@ struct PairsParams {
   int32_t *pair_query;
   int4 *prec;                  // null: pair_query only
   const uint32_t *qinfo;       // [NQ] nq | tail start << 8 | first query node << 16
+  // neighbour-support mode of the lane path: records of the surviving pairs point
+  // (.z) at the refined windows k_support_lane wrote for the pre-support pair list
+  const uint32_t *gm_old;      // pre-support GMCR bits (null: normal mode)
+  const I64x2 *off_old;        // pre-support pair offsets
+  int ns_mq;                   // windows per pair in the refined arrays
+};
+
+// k_support_lane: neighbour support (R9) on the lane path, one thread per
+// pre-support GMCR pair
+struct SupportLaneParams {
+  long long Pn, Pw;            // pre-support pairs on <= 32-node / larger molecules
+  const int4 *prec;            // pre-support pair records
+  const uint32_t *cmol;        // filter windows (distinct rows)
+  const uint32_t *adjw;        // bond-class adjacency (as JoinParams::adjw)
+  const uint2 *qp_ent2;        // plan entries with distinct rows (JoinParams::qp_ent2)
+  const uint16_t *qp_be;       // back-edge lists
+  const uint2 *qp_nbr;         // [VQ] query neighbours of each plan position (depth | class << 4 | 0x80, 8 bytes)
+  int MQ;                      // max query nodes (window slots per pair)
+  uint32_t *win32;             // [Pn][MQ] refined windows (<= 32-node molecules)
+  unsigned long long *win64;   // [Pw][MQ] refined windows (larger molecules)
+  uint8_t *alive;              // [Pn + Pw] 0 = the fixed point emptied a node of the pair
 };
 
 struct SupportParams {
@@ -257,6 +278,9 @@ cudaError_t launch_nodesets(const unsigned long long *eoff, long long P, unsigne
                             cudaStream_t st);
 cudaError_t launch_join(int NW, int mode, const JoinParams &p, int grid, cudaStream_t st);
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st);
+cudaError_t launch_support_lane(const SupportLaneParams &p, cudaStream_t st);
+cudaError_t launch_gmcr_update(int ND, int NQW, const uint32_t *gm_old, const I64x2 *off_old, const int32_t *goff,
+                               const uint8_t *alive, uint32_t *gm, I64x2 *mol_cnt, cudaStream_t st);
 cudaError_t launch_unpad(const uint32_t *cmol, const uint32_t *cand_units, const uint16_t *qdrow, int NDR, const int32_t *goff, int ND,
                          int VQ, int Wpad, uint32_t *dense,
                          cudaStream_t st);

@@ -1929,8 +1929,14 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
   const uint32_t ng8 = (uint32_t)(__ldg(&pp.goff[g + 1]) - a) << 8;  // molecule size, bits 8-15 of the query info
   const int aw = pp.prec ? (int)__ldg(&pp.adj_off[g]) : 0;  // adjacency word offset (pair record .x)
   const int cw = pp.prec ? (int)((unsigned)pp.rowstride * __ldg(&pp.cand_units[g])) : 0;  // cmol word base (.z)
+  // neighbour-support mode: the pair's pre-support index (its refined windows)
+  long long oo = 0;
+  const bool ns = pp.gm_old != nullptr;
+  const bool wide_g = (ng8 >> 8) > 32u;
+  if (ns) oo = wide_g ? pp.off_old[g].b : pp.off_old[g].a;
   for (int qb = 0; qb < pp.NQW; qb++) {
     const uint32_t bits = __ldg(&pp.gm[(size_t)g * pp.NQW + qb]);
+    const uint32_t obits = ns ? __ldg(&pp.gm_old[(size_t)g * pp.NQW + qb]) : 0u;
     if ((bits >> lane) & 1u) {
       const int q = qb * 32 + lane;
       const long long p = o + __popc(bits & lt);
@@ -1938,11 +1944,167 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
         pp.pair_query[p] = q;
       } else {  // the lane join reads the records only (queries from .y)
         const uint32_t qi = (__ldg(&pp.qinfo[q]) & ~0xff00u) | ng8;
-        pp.prec[p] = make_int4(aw, q, cw, (int)qi);
+        const int z = ns ? (int)((unsigned long long)(oo + __popc(obits & lt)) * (unsigned)pp.ns_mq * (wide_g ? 2u : 1u))
+                         : cw;
+        pp.prec[p] = make_int4(aw, q, z, (int)qi);
       }
     }
     o += __popc(bits);
+    oo += __popc(obits);
   }
+}
+
+// ===========================================================================
+// k_support_lane: neighbour support to the greatest fixed point (north_star;
+// DESIGN.md R9) on the lane path.  One thread per pre-support GMCR pair: the
+// windows of its query nodes (plan-depth order) are refined by
+//   C(w) &= OR_{u in C(v)} adj_b[u]   for every query edge (v, w, b)
+// until nothing changes (an AC-3 worklist; the fixed point is unique, so the
+// order is free); the refined windows are written per
+// pair for the join, and a pair with an emptied node leaves the GMCR
+// (k_gmcr_update rebuilds the GMCR bits and pair counts from the alive flags,
+// then the pair records are rebuilt from the remaining bits).
+// ===========================================================================
+constexpr int kSupportLaneThreads = 128;
+
+template <bool W64>
+__global__ void __launch_bounds__(kSupportLaneThreads) k_support_lane(const __grid_constant__ SupportLaneParams sp) {
+  using MT = typename std::conditional<W64, unsigned long long, unsigned>::type;
+  constexpr unsigned sw = W64 ? 1u : 0u;
+  extern __shared__ __align__(16) unsigned char smem[];
+  MT *const wv = (MT *)smem + threadIdx.x;  // window of depth e at wv[e * blockDim.x]
+  const long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+  const long long P = W64 ? sp.Pw : sp.Pn;
+  if (p >= P) return;
+  const int4 r = __ldg(&sp.prec[(W64 ? sp.Pn : 0) + p]);
+  const unsigned ca = (unsigned)r.x, cmb = (unsigned)r.z, info = (unsigned)r.w;
+  const unsigned nq = info & 0xffu, ng = (info >> 8) & 0xffu, qb = info >> 16;
+  const unsigned T = blockDim.x;
+  auto adj = [&](unsigned i) -> MT {
+    if (W64) return (MT)__ldg((const unsigned long long *)(sp.adjw + i));
+    return (MT)__ldg(sp.adjw + i);
+  };
+  auto low = [](MT x) -> unsigned {
+    return W64 ? (unsigned)(__ffsll((long long)x) - 1) : (unsigned)(__ffs((unsigned)x) - 1);
+  };
+  bool empty = false;
+  for (unsigned e = 0; e < nq; e++) {
+    const unsigned row = __ldg(&sp.qp_ent2[qb + e]).x >> 12;
+    const MT w = W64 ? (MT)__ldg((const unsigned long long *)(sp.cmol + (cmb + 2u * row))) : (MT)__ldg(sp.cmol + (cmb + row));
+    wv[e * T] = w;
+    empty |= w == (MT)0;
+  }
+  // support of S along the bond-class row base a: the nodes with a b-neighbour
+  // in S (up to four independent adjacency loads per round)
+  auto supp = [&](MT S, unsigned a) -> MT {
+    MT x = 0;
+    while (S) {
+      const unsigned u0 = low(S);
+      S &= S - (MT)1;
+      const bool h1 = S != (MT)0;
+      const unsigned u1 = h1 ? low(S) : 0u;
+      S &= S - (MT)(h1 ? 1 : 0);
+      const bool h2 = S != (MT)0;
+      const unsigned u2 = h2 ? low(S) : 0u;
+      S &= S - (MT)(h2 ? 1 : 0);
+      const bool h3 = S != (MT)0;
+      const unsigned u3 = h3 ? low(S) : 0u;
+      S &= S - (MT)(h3 ? 1 : 0);
+      const MT y0 = adj(a + (u0 << sw));
+      const MT y1 = h1 ? adj(a + (u1 << sw)) : (MT)0;
+      const MT y2 = h2 ? adj(a + (u2 << sw)) : (MT)0;
+      const MT y3 = h3 ? adj(a + (u3 << sw)) : (MT)0;
+      x |= (y0 | y1) | (y2 | y3);
+    }
+    return x;
+  };
+  // AC-3 worklist over query nodes: revising every neighbour w of a dirty
+  // node u against C(u) (C(w) &= supp(C(u), b)) and marking w dirty when it
+  // shrinks reaches the greatest fixed point with no confirmation pass
+  unsigned dirty = empty ? 0u : (nq >= 32 ? 0xffffffffu : (1u << nq) - 1u);
+  while (dirty) {
+    const unsigned u = (unsigned)(__ffs(dirty) - 1);
+    dirty &= dirty - 1u;
+    const uint2 nb = __ldg(&sp.qp_nbr[qb + u]);  // up to 8 neighbours: depth | class << 4 | 0x80
+    const MT cu = wv[u * T];
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+      const unsigned byte = ((k < 4 ? nb.x : nb.y) >> (8 * (k & 3))) & 0xffu;
+      if (!(byte & 0x80u)) break;
+      const unsigned w = byte & 15u, cls = (byte >> 4) & 7u;
+      const MT cw = wv[w * T];
+      const MT nw = cw & supp(cu, ca + ((cls * ng) << sw));
+      if (nw != cw) {
+        wv[w * T] = nw;
+        if (!nw) {
+          empty = true;
+          dirty = 0u;
+          break;
+        }
+        dirty |= 1u << w;
+      }
+    }
+  }
+  sp.alive[(W64 ? sp.Pn : 0) + p] = empty ? 0 : 1;  // k_gmcr_update rebuilds the GMCR bits from these
+  if (empty) return;
+  for (unsigned e = 0; e < nq; e++) {
+    if (W64) sp.win64[(size_t)p * sp.MQ + e] = (unsigned long long)wv[e * T];
+    else sp.win32[(size_t)p * sp.MQ + e] = (uint32_t)wv[e * T];
+  }
+}
+
+cudaError_t launch_support_lane(const SupportLaneParams &p, cudaStream_t st) {
+  const size_t s32 = 4 * (size_t)p.MQ * kSupportLaneThreads, s64 = 8 * (size_t)p.MQ * kSupportLaneThreads;
+  if (p.Pn > 0) {
+    k_support_lane<false><<<(unsigned)((p.Pn + kSupportLaneThreads - 1) / kSupportLaneThreads), kSupportLaneThreads, s32,
+                            st>>>(p);
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+  }
+  if (p.Pw > 0) {
+    k_support_lane<true><<<(unsigned)((p.Pw + kSupportLaneThreads - 1) / kSupportLaneThreads), kSupportLaneThreads, s64,
+                           st>>>(p);
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+// GMCR bits and pair counts after neighbour support: warp per data graph,
+// lane = query of a 32-query block; a pre-support pair survives iff its
+// alive flag is set (pre-support index = the graph's offset + rank of the bit)
+__global__ void __launch_bounds__(256) k_gmcr_update(int ND, int NQW, const uint32_t *gm_old, const I64x2 *off_old,
+                                                      const int32_t *goff, const uint8_t *alive, uint32_t *gm,
+                                                      I64x2 *mol_cnt) {
+  const int lane = threadIdx.x & 31;
+  const int g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (g >= ND) return;
+  const unsigned lt = (1u << lane) - 1u;
+  const bool wide = __ldg(&goff[g + 1]) - __ldg(&goff[g]) > 32;
+  long long oo = wide ? off_old[ND].a + off_old[g].b : off_old[g].a;  // alive[] index of the graph's first pair
+  long long np = 0;
+  for (int qb = 0; qb < NQW; qb++) {
+    const uint32_t obits = __ldg(&gm_old[(size_t)g * NQW + qb]);
+    const bool mine = (obits >> lane) & 1u;
+    const bool keep = mine && alive[oo + __popc(obits & lt)];
+    const uint32_t nb = __ballot_sync(0xffffffffu, keep);
+    if (lane == 0) gm[(size_t)g * NQW + qb] = nb;
+    np += __popc(nb);
+    oo += __popc(obits);
+  }
+  if (lane == 0) {
+    I64x2 v;
+    v.a = wide ? 0 : np;
+    v.b = wide ? np : 0;
+    mol_cnt[g] = v;
+  }
+}
+
+cudaError_t launch_gmcr_update(int ND, int NQW, const uint32_t *gm_old, const I64x2 *off_old, const int32_t *goff,
+                               const uint8_t *alive, uint32_t *gm, I64x2 *mol_cnt, cudaStream_t st) {
+  if (ND <= 0) return cudaSuccess;
+  k_gmcr_update<<<(unsigned)((32ll * ND + 255) / 256), 256, 0, st>>>(ND, NQW, gm_old, off_old, goff, alive, gm, mol_cnt);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st) {

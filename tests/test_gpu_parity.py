@@ -351,3 +351,30 @@ def test_cost_model_from_device_gmcr(ctx, sigmo):
         cb = max(c[b[r]:b[r + 1]].sum() for r in range(world))
         ca = max(c[a[r]:a[r + 1]].sum() for r in range(world))
         assert b[-1] == D.num_graphs and cb <= ca + c.max()
+
+
+def test_neighbour_support_lane_path_c2(sigmo):
+    """Neighbour support on the lane path (k_support_lane: per-pair refined
+    windows, GMCR rebuilt) on a 20k-molecule configs[1] slice incl. > 32-atom
+    molecules: GMCR pairs = the reference GMCR of the fixed point on sampled
+    molecules, every pair's Find All / Find First result = the oracle's."""
+    Q, D = synth.config_queries(2), synth.config_data(2, first=60_000, count=20_000)
+    ref = oracle.count_dense(Q, D)
+    with sigmo.Context(0) as c:
+        c.load_batch(Q, D)
+        c.filter(4)
+        n_plain = c.num_pairs()
+        c.filter(4, neighbor_support=True)
+        n_ns = c.num_pairs()
+        assert n_ns < n_plain
+        c.join(sigmo.SIGMO_FIND_ALL)
+        assert np.array_equal(c.dense_results(), ref)
+        c.join(sigmo.SIGMO_FIND_FIRST)
+        assert np.array_equal(c.dense_results(), (ref > 0).astype(np.uint64))
+        di, qi, _ = c.pair_results()
+    gs = list(range(0, 20_000, 97))
+    for g in gs[:40]:
+        Dg = D.slice(g, g + 1)
+        F = fr.neighbour_support(Q, Dg, fr.candidates_bool(Q, Dg, 4))
+        want = set(np.nonzero(fr.gmcr(Q, Dg, F)[:, 0])[0].tolist())
+        assert set(qi[di == g].tolist()) == want, g

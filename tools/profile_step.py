@@ -21,8 +21,9 @@ ctx = sigmo.Context(0)
 if os.environ.get("SIGMO_PROFILE_INDUCED") == "1":
     ctx.set_induced(True)
 ctx.load_batch(Q, D)
+ns = os.environ.get("SIGMO_PROFILE_NS") == "1"  # neighbour-support flag
 for _ in range(2 + S):
-    ctx.filter(L)
+    ctx.filter(L, neighbor_support=ns)
     ctx.join(mode, total=False)
 torch.cuda.synchronize()
 print("matches", ctx.join(mode))
