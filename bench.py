@@ -55,6 +55,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-flush", action="store_true")
+    ap.add_argument("--balance", default="atoms", choices=["count", "atoms", "cost"],
+                    help="molecule shards at N>1: equal count (the paper's static split), equal atoms (default), "
+                         "or equal modelled cost (SURVEY 8(f) N2: a first filter pass feeds sharded.molecule_costs)")
     ap.add_argument("--ns", action="store_true",
                     help="neighbour-support fixed point in the filter (SIGMO_FILTER_NEIGHBOR_SUPPORT; DESIGN.md R9)")
     ap.add_argument("--induced", action="store_true",
@@ -254,7 +257,8 @@ def config_dict(args, world, oracle_step=None):
          "query_seed": hex(0x9E00_0000 + args.cid),
          "l2": ("flushed before every timed step (256 MiB device write, outside the events)" if args.cid in (2, 3)
                 else "no flush: per-step inputs and candidate arrays are larger than the 126 MB L2"),
-         "parallelism": f"dp{world}: molecule shards, queries replicated, NCCL all-reduce of per-query totals"}
+         "parallelism": f"dp{world}: molecule shards, queries replicated, NCCL all-reduce of per-query totals",
+         "shards": getattr(args, "balance", "atoms") if world > 1 else "whole batch"}
     if getattr(args, "induced", False):
         d["workload"] += ", induced-subgraph mode (N4)"
         d["induced"] = True
@@ -285,17 +289,33 @@ def main():
     dist = None
     if world > 1:
         import torch.distributed as dist
+    from paper_conf_sc_carocfc25_b200 import sharded
     Q = synth.config_queries(args.cid)
-    D = synth.config_data(args.cid, first=rank * args.molecules, count=args.molecules)
     stream = torch.cuda.current_stream(dev)
     ctx = sigmo.Context(local, stream)
     if args.induced:
         ctx.set_induced(True)
+    # this rank's molecules of the world x M stream (weak scaling): contiguous
+    # shards balanced by atoms (default), count, or modelled cost (N2)
+    M_total = args.molecules * world
+    if world > 1:
+        sizes = synth.molecule_sizes(synth.DATA_SEED_BASE + args.cid, 0, M_total)
+        bounds = sharded.stream_shard_bounds(sizes, world, "count" if args.balance == "count" else "atoms")
+        if args.balance == "cost":
+            # first pass on the atom shards: per-molecule cost = atoms + w_pair x GMCR pairs, gathered over ranks
+            D0 = synth.config_data(args.cid, first=int(bounds[rank]), count=int(bounds[rank + 1] - bounds[rank]))
+            ctx.load_batch(Q, D0)
+            ctx.filter(args.levels, neighbor_support=args.ns)
+            ctx.join(sigmo.SIGMO_FIND_ALL, total=False)
+            costs = sharded.gather_costs(sharded.molecule_costs(D0.graph_offsets, ctx.pair_results()[0]))
+            bounds = sharded.stream_shard_bounds(sizes, world, "cost", costs=costs)
+            del D0
+    else:
+        bounds = np.array([0, args.molecules], np.int64)
+    D = synth.config_data(args.cid, first=int(bounds[rank]), count=int(bounds[rank + 1] - bounds[rank]))
     ctx.load_batch(Q, D)
     totals = torch.zeros(Q.num_graphs, dtype=torch.int64, device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device=dev)
-
-    from paper_conf_sc_carocfc25_b200 import sharded
 
     def step(mode=sigmo.SIGMO_FIND_ALL):
         ctx.filter(args.levels, neighbor_support=args.ns)
@@ -357,15 +377,10 @@ def main():
         assert tot == matches_local
     h2d = ctx.timings()["h2d_bytes"]
 
-    # ---- reduce over ranks ----
-    vals = torch.tensor([ms_all, ms_ff, sum(e2e_ms)], dtype=torch.float64, device=dev)
-    cnts = torch.tensor([matches_local, pairs_local, positive_local, Q.num_graphs * D.num_graphs],
-                        dtype=torch.int64, device=dev)
-    if dist is not None:
-        dist.all_reduce(vals, op=dist.ReduceOp.MAX)
-        dist.all_reduce(cnts)
-    ms_all, ms_ff, e2e_total = vals.tolist()
-    matches, pairs, positive, all_pairs = [int(x) for x in cnts.tolist()]
+    # ---- reduce over ranks (sharded.rank_reduce: times MAX, counts SUM) ----
+    ctx.check()  # the device-pointer totals path never synchronized: check the join's capacities once
+    (ms_all, ms_ff, e2e_total), (matches, pairs, positive, all_pairs) = sharded.rank_reduce(
+        [ms_all, ms_ff, sum(e2e_ms)], [matches_local, pairs_local, positive_local, Q.num_graphs * D.num_graphs], dev)
     if rank != 0:
         ctx.close()
         if dist is not None:
@@ -373,7 +388,7 @@ def main():
         return
 
     K = args.steps
-    value = matches * K / (ms_all / 1000.0)
+    value = sharded.throughput(matches, K, ms_all)
     ms_per_step = ms_all / K
     # ---- roofline of the dominant kernel (per-launch CUDA events over the timed region) ----
     import json as _json

@@ -36,8 +36,58 @@ def shard_range(graph_offsets: np.ndarray, rank: int, world: int) -> Tuple[int, 
 
 
 def equal_count_range(n_total: int, rank: int, world: int) -> Tuple[int, int]:
-    """Equal-molecule-count shard (used when molecules are generated per rank)."""
+    """Equal-molecule-count shard (the paper's static split)."""
     return n_total * rank // world, n_total * (rank + 1) // world
+
+
+def stream_shard_bounds(natoms, world: int, balance: str = "atoms", costs=None) -> np.ndarray:
+    """Shard boundaries over a molecule stream of known atom counts:
+    balance = "count" (equal molecules, the paper's static split), "atoms"
+    (equal atoms: filter bytes scale with atoms; the default) or "cost"
+    (equal modelled cost, N2: `costs` per molecule, see molecule_costs)."""
+    natoms = np.asarray(natoms, dtype=np.int64)
+    G = natoms.shape[0]
+    if balance == "count":
+        return np.array([G * r // world for r in range(world + 1)], np.int64)
+    if balance == "atoms":
+        goff = np.concatenate([[0], np.cumsum(natoms)])
+        return shard_bounds(goff, world)
+    if balance == "cost":
+        if costs is None:
+            raise ValueError("balance='cost' needs the per-molecule costs")
+        return cost_bounds(costs, world)
+    raise ValueError(f"unknown balance {balance!r}")
+
+
+# ---------------------------------------------------------------------------
+# Rank bookkeeping of a timed multi-GPU run (bench.py): per-rank device
+# times reduce with MAX (the job ends when the slowest rank ends), counts
+# with SUM (whole-job throughput = all ranks' units / max time).
+# ---------------------------------------------------------------------------
+def rank_reduce(max_vals, sum_vals, device=None):
+    """All-reduce a list of float64 per-rank times with MAX and a list of
+    int64 per-rank counts with SUM (one collective each; NCCL on the rank's
+    GPU, gloo on the CPU); identity without a process group."""
+    import torch
+    import torch.distributed as dist
+    dev = device if device is not None else torch.device("cpu")
+    mx = torch.tensor(list(max_vals), dtype=torch.float64, device=dev)
+    sm = torch.tensor([int(x) for x in sum_vals], dtype=torch.int64, device=dev)
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size() > 1:
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+    return [float(x) for x in mx.tolist()], [int(x) for x in sm.tolist()]
+
+
+def barrier():
+    import torch.distributed as dist
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size() > 1:
+        dist.barrier()
+
+
+def throughput(units_total: int, steps: int, max_ms: float) -> float:
+    """Whole-job rate: units of all ranks over the slowest rank's time."""
+    return units_total * steps / (max_ms / 1000.0) if max_ms > 0 else 0.0
 
 
 # ---------------------------------------------------------------------------

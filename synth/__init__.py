@@ -174,6 +174,18 @@ class GraphBatch:
 # molecules
 # ----------------------------------------------------------------------------
 
+def molecule_sizes(seed: int, first: int, count: int, mode: int = 0, nthreads: int | None = None) -> np.ndarray:
+    """Atom counts of molecules first..first+count-1 of the stream (no graphs
+    built): what a shard planner needs to balance ranks by atoms."""
+    lib = _load()
+    nthreads = nthreads or min(32, os.cpu_count() or 1)
+    natoms = np.zeros(count, np.int32)
+    nadj = np.zeros(count, np.int32)
+    if count:
+        lib.synth_sizes(seed, first, count, mode, nthreads, _ptr(natoms, ctypes.c_int32), _ptr(nadj, ctypes.c_int32))
+    return natoms
+
+
 def molecules(seed: int, first: int, count: int, mode: int = 0, nthreads: int | None = None) -> GraphBatch:
     """Molecules first..first+count-1 of the stream (seed, mode) as one batch."""
     lib = _load()

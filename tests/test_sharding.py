@@ -125,3 +125,56 @@ def test_gloo_world2_gathered_costs_equal_unsharded(tmp_path):
     for r in range(world):
         assert np.array_equal(np.load(os.path.join(tmp_path, f"c{r}.npy")), ref)
         assert np.array_equal(np.load(os.path.join(tmp_path, f"b{r}.npy")), sharded.cost_bounds(ref, world))
+
+
+# ---------------------------------------------------------------- bench rank logic (gloo world 2)
+def _rank_worker(rank, world, port, out_dir):
+    """What bench.py does at N>1 minus the GPU: each rank takes its shard of the
+    world x M molecule stream (atom-balanced bounds computed from the stream's
+    atom counts, identically on every rank), times its 'steps', and the ranks
+    reduce times with MAX and counts with SUM (sharded.rank_reduce)."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    M = 150
+    sizes = synth.molecule_sizes(synth.DATA_SEED_BASE + 1, 0, M * world)
+    out = {}
+    for bal in ("count", "atoms"):
+        b = sharded.stream_shard_bounds(sizes, world, bal)
+        Q = synth.config_queries(1)
+        D = synth.config_data(1, first=int(b[rank]), count=int(b[rank + 1] - b[rank]))
+        sharded.barrier()
+        counts = oracle.count_dense(Q, D, nthreads=2)
+        fake_ms = 10.0 + rank  # a per-rank device time
+        (mx,), (matches, pairs) = sharded.rank_reduce([fake_ms], [int(counts.sum()), Q.num_graphs * D.num_graphs])
+        out[bal] = (b.tolist(), mx, matches, pairs, sharded.throughput(matches, 1, mx))
+    # the cost split (N2): gathered per-molecule costs, identical bounds on all ranks
+    b = sharded.stream_shard_bounds(sizes, world, "atoms")
+    D = synth.config_data(1, first=int(b[rank]), count=int(b[rank + 1] - b[rank]))
+    local = sharded.molecule_costs(D.graph_offsets, np.repeat(np.arange(D.num_graphs), 2))
+    costs = sharded.gather_costs(local)
+    out["cost"] = sharded.stream_shard_bounds(sizes, world, "cost", costs=costs).tolist()
+    np.save(os.path.join(out_dir, f"rank{rank}.npy"), np.array([out], dtype=object), allow_pickle=True)
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_bench_rank_logic(tmp_path):
+    world = 2
+    mp.spawn(_rank_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    outs = [np.load(os.path.join(tmp_path, f"rank{r}.npy"), allow_pickle=True)[0] for r in range(world)]
+    M = 150
+    Q = synth.config_queries(1)
+    D = synth.config_data(1, count=M * world)
+    total = int(oracle.count_dense(Q, D).sum())
+    sizes = synth.molecule_sizes(synth.DATA_SEED_BASE + 1, 0, M * world)
+    for bal in ("count", "atoms"):
+        b0, mx0, m0, p0, v0 = outs[0][bal]
+        b1, mx1, m1, p1, v1 = outs[1][bal]
+        assert b0 == b1 and b0[0] == 0 and b0[-1] == M * world   # identical, covering bounds
+        assert mx0 == mx1 == 11.0                                # MAX of the per-rank times
+        assert m0 == m1 == total                                  # SUM of the per-rank matches
+        assert p0 == Q.num_graphs * M * world
+        assert v0 == total / 0.011
+    atoms = [int(sizes[outs[0]["atoms"][0][r]:outs[0]["atoms"][0][r + 1]].sum()) for r in range(world)]
+    assert abs(atoms[0] - atoms[1]) <= int(sizes.max())            # atom-balanced within one molecule
+    assert outs[0]["cost"] == outs[1]["cost"]
