@@ -302,12 +302,19 @@ def main():
         sizes = synth.molecule_sizes(synth.DATA_SEED_BASE + args.cid, 0, M_total)
         bounds = sharded.stream_shard_bounds(sizes, world, "count" if args.balance == "count" else "atoms")
         if args.balance == "cost":
-            # first pass on the atom shards: per-molecule cost = atoms + w_pair x GMCR pairs, gathered over ranks
+            # adaptive (N2): a timed first pass on the atom shards; each rank's
+            # device time spread over its molecules by atoms, gathered over
+            # ranks, split at equal cost (sharded.measured_costs)
             D0 = synth.config_data(args.cid, first=int(bounds[rank]), count=int(bounds[rank + 1] - bounds[rank]))
             ctx.load_batch(Q, D0)
-            ctx.filter(args.levels, neighbor_support=args.ns)
-            ctx.join(sigmo.SIGMO_FIND_ALL, total=False)
-            costs = sharded.gather_costs(sharded.molecule_costs(D0.graph_offsets, ctx.pair_results()[0]))
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            for i in range(2):
+                ev0.record(stream)
+                ctx.filter(args.levels, neighbor_support=args.ns)
+                ctx.join(sigmo.SIGMO_FIND_ALL, total=False)
+                ev1.record(stream)
+            torch.cuda.synchronize(dev)
+            costs = sharded.gather_costs(sharded.measured_costs(D0.graph_offsets, ev0.elapsed_time(ev1)))
             bounds = sharded.stream_shard_bounds(sizes, world, "cost", costs=costs)
             del D0
     else:

@@ -126,6 +126,17 @@ def molecule_costs(graph_offsets, pair_data_idx, w_atom: float = 1.0, w_pair: fl
     return w_atom * np.diff(goff).astype(np.float64) + w_pair * pairs.astype(np.float64)
 
 
+def measured_costs(graph_offsets, ms: float) -> np.ndarray:
+    """Feedback cost model (adaptive balancing, N2): the rank's measured device
+    time of its previous batch spread over its molecules by atoms -- every
+    molecule of a shard costs atoms x (ms / atoms of the shard).  Gathered over
+    ranks and split with cost_bounds, shards that ran slow per atom (e.g.
+    ring-rich regions of a library) shrink for the next batch."""
+    natoms = np.diff(np.asarray(graph_offsets, dtype=np.int64)).astype(np.float64)
+    tot = natoms.sum()
+    return natoms * (float(ms) / tot) if tot > 0 else natoms
+
+
 def gather_costs(local_costs, group=None) -> np.ndarray:
     """Concatenate every rank's per-molecule costs in rank order (the ranks'
     shards are contiguous and ordered).  All-gathers the lengths, then the
