@@ -7,7 +7,10 @@
 Workload (N=1): BASELINE.json configs[2] -- the configuration the metric is
 quoted on at 1/2/4/8 B200 -- = 100 queries (35 library functional groups +
 65 random 3-8-atom subgraphs) x 1M synthetic ZINC-like molecules per GPU,
-Find All, filter levels 4; `--config 1` selects configs[1]
+Find All, filter levels 2 = the best of the configs[1] levels sweep (SURVEY.md
+8(d) C3 "L = best from C2"; profiles/r2/levels_sweep_c1.jsonl: Find All
+L=1..7 -> 1.14/0.74/0.75/0.77/0.78/0.79/0.79 ms, Find First best at L=2 too,
+and the same on configs[2] itself, levels_sweep_c2.jsonl); `--config 1` selects configs[1]
 (50 queries x 100k molecules, the levels-sweep / Find First config).  Weak
 scaling: rank r owns molecules [r*M, (r+1)*M) of the same counter-based
 stream; queries are replicated; the only collective is an NCCL all-reduce of
@@ -38,7 +41,7 @@ BASELINE_METRIC = "matches/sec (Find All) and graph-pairs/sec (Find First) at 1/
 # share (1M / 8 and 10M / 8), so `--gpus 8` processes the whole config.
 CONFIGS = {1: (2, 100_000), 2: (3, 1_000_000), 3: (4, 125_000), 4: (5, 1_250_000)}
 STREAM_BATCH = 250_000        # configs[4]: molecules per streamed batch per GPU
-LEVELS = 4
+LEVELS = 2  # best of the configs[1] sweep (profiles/r2/levels_sweep_c1.jsonl)
 CPU_SAMPLE_MOLS = 200_000     # cpu_baseline leg: oracle on the first 200k molecules (~100 core-seconds)
 REF_STEP_MOLS = 2_000         # --impl reference: molecules per step
 

@@ -41,6 +41,18 @@ def main():
         if n <= 200_000:
             bm = ctx.candidates()
             row["candidate_bits"] = int(np.unpackbits(bm.view(np.uint8)).sum())
+        # the neighbour-support flag (R9) at this level, Find All
+        ctx.filter(L, neighbor_support=True)
+        ctx.join(sigmo.SIGMO_FIND_ALL)
+        ctx.set_timing(True)
+        for _ in range(max(reps // 4, 2)):
+            ctx.filter(L, neighbor_support=True)
+            ctx.join(sigmo.SIGMO_FIND_ALL, total=False)
+        t = ctx.timings()
+        ctx.set_timing(False)
+        row["all_ns"] = {"filter_ms": t["filter_ms"], "mapping_ms": t["mapping_ms"], "join_ms": t["join_ms"],
+                         "total_ms": t["filter_ms"] + t["mapping_ms"] + t["join_ms"],
+                         "result": ctx.join(sigmo.SIGMO_FIND_ALL), "gmcr_pairs": ctx.num_pairs()}
         print(json.dumps(row), flush=True)
 
 
