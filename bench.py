@@ -402,38 +402,58 @@ def main():
     ms_per_step = ms_all / K
     # ---- roofline of the dominant kernel (per-launch CUDA events over the timed region) ----
     import json as _json
-    peaks = {}
-    try:
-        peaks = _json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
-    except Exception:
-        pass
+
+    def _load(rel):
+        try:
+            return _json.load(open(os.path.join(ROOT, rel)))
+        except Exception:
+            return {}
+
+    peaks = _load("MEASURED_PEAKS.json")
     hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
     peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s"
+    # ncu --set full of the same kernels at the bench's levels (profiles/r2/ncu_traffic.json, tools/ncu_traffic.py):
+    # DRAM bytes per launch and instruction counts; cold-cache and serialised, so only shares/ratios are used
+    ncu = _load("profiles/r2/ncu_traffic.json")
+    nk = ncu.get("kernels", {}) if ncu.get("levels") == args.levels else {}
     VQ, VD, ND, NQ = Q.num_nodes, D.num_nodes, D.num_graphs, Q.num_graphs
     W = (VD + 31) // 32
+    # the method must produce C_L -- VQ x VD bits written once -- plus the GMCR bits / counts,
+    # reading the packed CSR-GO once (the kernel writes the distinct-row windows instead: fewer DRAM bytes)
     filter_bytes = (4 * VQ * W                       # bitmap written once
                     + 4 * ND * ((NQ + 31) // 32) + 16 * ND  # GMCR bits + counts
                     + 4 * (ND + 1) + 2 * VD + 4 * (VD + 1) + 2 * D.num_adj)  # packed CSR-GO read once
     f_ms, j_ms, m_ms = tim["filter_ms"], tim["join_ms"], tim["mapping_ms"]
+    fk = nk.get("sigmo_filter_lane_jit", {})
+    f_dram = fk.get("dram_bytes")
     filter_roof = {"bound": "hbm", "achieved": filter_bytes / (f_ms * 1e-3) / 1e9, "peak": hbm_peak,
-                   "unit": "GB/s", "frac": filter_bytes / (f_ms * 1e-3) / 1e9 / hbm_peak, "traffic": None,
-                   "kernel": "k_filter", "ms": f_ms, "algorithmic_bytes": filter_bytes, "peak_source": peak_src}
-    # join: ALU bound: algorithmic work = DFS iterator
-    # steps x 12 lane-ops; peak = 148 SMs x 128 lanes x SM clock
+                   "unit": "GB/s", "frac": filter_bytes / (f_ms * 1e-3) / 1e9 / hbm_peak, "traffic": f_dram,
+                   "kernel": "sigmo_filter_lane_jit" if tim.get("filter_jit") else "k_filter_lane", "ms": f_ms,
+                   "algorithmic_bytes": filter_bytes, "peak_source": peak_src,
+                   "algorithmic_bytes_model": "SURVEY 8(d): VQ*VD/8 candidate bits + GMCR bits/counts + packed CSR-GO",
+                   "frac_dram": (f_dram / (f_ms * 1e-3) / 1e9 / hbm_peak) if f_dram else None,
+                   "frac_dram_note": "ncu DRAM bytes of one launch (distinct-row windows, profiles/r2/ncu_traffic.json) "
+                                     "/ this run's kernel time / peak"}
+    # join: integer-issue bound.  Peak = the measured mixed LOP3 + IMAD rate of this
+    # B200 model (tools/microbench/int_peak.cu -> profiles/r2/int_peak.json: 122 lanes/SM/clk) at the run's
+    # clock; algorithmic work = DFS steps x 12 lane-ops (the minimum a step needs); the measured cost per
+    # step (thread-instructions) comes from the ncu capture
     sm_mhz = float(clocks.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0))
-    traffic = {}
-    try:
-        traffic = _json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-    except Exception:
-        pass
+    ip = _load("profiles/r2/int_peak.json")
+    lanes = float(ip.get("mixed_lanes_per_sm_per_clk", 128.0))
     steps = tim.get("dfs_steps", 0)
-    alu_peak = 148 * 128 * sm_mhz * 1e6 / 1e12
+    alu_peak = 148 * lanes * sm_mhz * 1e6 / 1e12
     join_ach = 12.0 * steps / (j_ms * 1e-3) / 1e12 if j_ms > 0 else 0.0
+    jn, jw = nk.get("k_join_lane_narrow", {}), nk.get("k_join_lane_wide", {})
+    thr_instr = sum(k.get("warp_instructions", 0) * k.get("threads_per_instruction", 0) for k in (jn, jw))
     join_roof = {"bound": "alu", "achieved": join_ach, "peak": alu_peak, "unit": "Tops/s", "frac": join_ach / alu_peak,
-                 "traffic": traffic.get("k_join"), "kernel": "k_join", "ms": j_ms, "dfs_steps_per_launch": steps,
-                 "ops_per_step": 12, "peak_source": f"148 SM x 128 int lanes x {sm_mhz:.0f} MHz (measured clock)",
+                 "traffic": (jn.get("dram_bytes", 0) + jw.get("dram_bytes", 0)) or None,
+                 "kernel": "k_join_lane", "ms": j_ms, "dfs_steps_per_launch": steps, "ops_per_step": 12,
+                 "peak_source": f"measured: 148 SM x {lanes:.1f} int lanes/clk (mixed LOP3+IMAD, profiles/r2/"
+                                f"int_peak.json) x {sm_mhz:.0f} MHz (this run's clock)",
+                 "thread_instructions_per_step": (thr_instr / steps) if (steps and thr_instr) else None,
+                 "issue_utilization": (jn.get("ipc", 0) / 4.0) if jn else None,
                  "pairs_per_launch": pairs_local, "matches_per_launch": matches_local}
-    filter_roof["traffic"] = traffic.get("k_filter")
     dominant = "join" if j_ms >= f_ms else "filter"
     roofline = dict(join_roof) if dominant == "join" else dict(filter_roof)
 
