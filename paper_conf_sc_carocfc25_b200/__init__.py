@@ -32,15 +32,32 @@ def _arr(a, dt):
     return np.ascontiguousarray(a, dtype=dt)
 
 
-class _CBatch:
-    """Keeps the numpy arrays alive while the C struct points at them."""
+def _pinned(a, dt):
+    """A copy of `a` in page-locked host memory (torch's pinned allocator), so
+    that sigmo_load_batch's copies of it are plain DMA."""
+    import torch
+    t = torch.from_numpy(np.ascontiguousarray(a, dtype=dt)).pin_memory()
+    return t.numpy(), t
 
-    def __init__(self, b):
-        self.goff = _arr(b.graph_offsets, np.int64)
-        self.roff = _arr(b.row_offsets, np.int64)
-        self.col = _arr(b.col_indices, np.int32)
-        self.nlab = _arr(b.node_labels, np.uint8)
-        self.elab = _arr(b.edge_labels, np.uint8)
+
+class _CBatch:
+    """Keeps the numpy arrays alive while the C struct points at them.
+    pinned=True: the arrays are copied once into page-locked memory (what a
+    data loader feeding the GPU holds)."""
+
+    def __init__(self, b, pinned: bool = False):
+        self._keep = []
+        conv = _arr
+        if pinned:
+            def conv(a, dt):
+                x, t = _pinned(a, dt)
+                self._keep.append(t)
+                return x
+        self.goff = conv(b.graph_offsets, np.int64)
+        self.roff = conv(b.row_offsets, np.int64)
+        self.col = conv(b.col_indices, np.int32)
+        self.nlab = conv(b.node_labels, np.uint8)
+        self.elab = conv(b.edge_labels, np.uint8)
         s = _native.sigmo_graph_batch()
         s.num_graphs = int(self.goff.shape[0] - 1)
         s.num_nodes = int(self.nlab.shape[0])
@@ -54,8 +71,8 @@ class _CBatch:
         self.num_nodes = s.num_nodes
 
 
-def as_c_batch(b) -> _CBatch:
-    return b if isinstance(b, _CBatch) else _CBatch(b)
+def as_c_batch(b, pinned: bool = False) -> _CBatch:
+    return b if isinstance(b, _CBatch) else _CBatch(b, pinned)
 
 
 def validate_batch(batch, is_query: bool):

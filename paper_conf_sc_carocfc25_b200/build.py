@@ -8,7 +8,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libsigmo.so")
-SOURCES = ["sigmo_abi.cu", "sigmo_kernels.cu", "sigmo_filter_lane.cu", "sigmo_jit.cu"]
+SOURCES = ["sigmo_abi.cu", "sigmo_kernels.cu", "sigmo_filter_lane.cu", "sigmo_jit.cu", "sigmo_load.cu"]
 HEADERS = ["sigmo_internal.h", "lane_filter_types.h", "lane_filter_body.cuh", os.path.join("..", "..", "include", "sigmo.h")]
 # headers embedded as raw strings for the NVRTC-specialised filter (sigmo_jit.cu)
 EMBED = ["lane_filter_types.h", "lane_filter_body.cuh"]

@@ -176,6 +176,9 @@ struct sigmo_ctx {
   DBuf eoff, ecur, emaps, esets, ucnt, uoff, uniq, etmp;
   int64_t enum_P = -1, enum_total = 0, enum_uniq = -1;
   int enum_stride = 8;
+  // device-side load of large data batches (k_load_data)
+  DBuf raw, dpk, ldinfo;
+  Pinned ldhost;                    // histogram + error words read back
   // neighbour support on the lane path (k_support_lane)
   bool lane_ns = false;            // the last filter refined per-pair windows (join reads ns_win*)
   bool ns_lane_ok = true;          // every query node has <= 8 neighbours (k_support_lane's lists)
@@ -362,6 +365,44 @@ sigmo_status validate(const sigmo_graph_batch *b, int is_query, std::string &msg
   out.col = col;
   out.nlab = b->node_labels;
   out.elab = el;
+  return SIGMO_OK;
+}
+
+// O(#graphs) checks of a large data batch; the per-entry checks run on the
+// device (k_load_data) with the same error classes
+sigmo_status validate_light(const sigmo_graph_batch *b, std::string &msg, HostGraphs &out) {
+  auto fail = [&](sigmo_status s, const char *fmt, long long x, long long y) {
+    char buf[256];
+    snprintf(buf, sizeof(buf), fmt, x, y);
+    msg = buf;
+    return s;
+  };
+  if (b->num_graphs < 0 || b->num_nodes < 0) return fail(SIGMO_ERR_INVALID_ARG, "negative num_graphs %lld / num_nodes %lld", b->num_graphs, b->num_nodes);
+  if (!b->graph_offsets || !b->row_offsets) return fail(SIGMO_ERR_INVALID_ARG, "graph_offsets/row_offsets NULL", 0, 0);
+  if (b->num_nodes >= (1ll << 31) - 1) return fail(SIGMO_ERR_LIMIT, "num_nodes %lld >= 2^31-1", b->num_nodes, 0);
+  if (b->num_graphs >= (1ll << 31) - 1) return fail(SIGMO_ERR_LIMIT, "num_graphs %lld >= 2^31-1", b->num_graphs, 0);
+  const int64_t G = b->num_graphs, V = b->num_nodes;
+  const int64_t *go = b->graph_offsets, *ro = b->row_offsets;
+  if (go[0] != 0) return fail(SIGMO_ERR_INVALID_GRAPH, "graph_offsets[0] = %lld, expected 0", go[0], 0);
+  for (int64_t g = 0; g < G; g++) {
+    if (go[g + 1] < go[g]) return fail(SIGMO_ERR_INVALID_GRAPH, "graph_offsets decreasing at graph %lld (%lld)", g, go[g + 1]);
+    if (go[g + 1] - go[g] > SIGMO_MAX_DATA_NODES)
+      return fail(SIGMO_ERR_LIMIT, "data graph %lld has %lld nodes > 256", g, go[g + 1] - go[g]);
+  }
+  if (go[G] != V) return fail(SIGMO_ERR_INVALID_GRAPH, "graph_offsets[num_graphs] = %lld != num_nodes %lld", go[G], V);
+  if (ro[0] != 0) return fail(SIGMO_ERR_INVALID_GRAPH, "row_offsets[0] = %lld, expected 0", ro[0], 0);
+  const int64_t E = ro[V];
+  if (E < 0 || E >= (1ll << 31) - 1) return fail(SIGMO_ERR_LIMIT, "adjacency entries %lld not in [0, 2^31-1)", E, 0);
+  if (V > 0 && !b->node_labels) return fail(SIGMO_ERR_INVALID_ARG, "node_labels NULL", 0, 0);
+  if (E > 0 && (!b->col_indices || !b->edge_labels)) return fail(SIGMO_ERR_INVALID_ARG, "col_indices/edge_labels NULL", 0, 0);
+  out.G = G;
+  out.V = V;
+  out.E = E;
+  out.goff = go;
+  out.roff = ro;
+  out.col = b->col_indices;
+  out.nlab = b->node_labels;
+  out.elab = b->edge_labels;
   return SIGMO_OK;
 }
 
@@ -950,7 +991,7 @@ void free_all(sigmo_ctx *c) {
                   &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp, &c->ent2, &c->nb4, &c->mrec,
                   &c->eoff, &c->ecur, &c->emaps, &c->esets, &c->ucnt, &c->uoff, &c->uniq, &c->etmp,
                   &c->ns_win32, &c->ns_win64, &c->ns_alive, &c->gm_old, &c->off_old, &c->ent_ns, &c->ns_bitmap,
-                  &c->ns_gm, &c->ns_cnt};
+                  &c->ns_gm, &c->ns_cnt, &c->raw, &c->dpk, &c->ldinfo};
   for (DBuf *b : bufs) dfree(c, *b);
 }
 
@@ -1166,6 +1207,7 @@ sigmo_status sigmo_destroy(sigmo_ctx *c) {
   free_all(c);
   cudaStreamSynchronize(c->stream);
   if (c->staging.p) cudaFreeHost(c->staging.p);
+  if (c->ldhost.p) cudaFreeHost(c->ldhost.p);
   if (c->h2d_done) cudaEventDestroy(c->h2d_done);
   if (c->aux) {
     cudaStreamSynchronize(c->aux);
@@ -1224,8 +1266,72 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const auto t0 = std::chrono::steady_clock::now();
   sigmo_status s = validate(queries, 1, msg, hq);
   if (s != SIGMO_OK) return set_err(c, s, "query batch: %s", msg.c_str());
-  s = validate(data, 0, msg, hd);
+  // large data batches: O(#graphs) checks here, the per-entry checks and the
+  // packing on the device (k_load_data) from the raw arrays
+  const char *hl = getenv("SIGMO_HOST_LOAD");  // test knob: host validation + packing at any size
+  const bool dev_load = data->num_nodes >= kDeviceLoadMinNodes && !(hl && atoi(hl));
+  s = dev_load ? validate_light(data, msg, hd) : validate(data, 0, msg, hd);
   if (s != SIGMO_OK) return set_err(c, s, "data batch: %s", msg.c_str());
+  size_t raw_bytes = 0;
+  PackedOffsets pdd{};
+  if (dev_load) {
+    CUDA_TRY(c, cudaEventSynchronize(c->h2d_done));  // the previous load's copies no longer read our buffers
+    Layout R;
+    const size_t r_go = R.take(8 * (size_t)(hd.G + 1)), r_ro = R.take(8 * (size_t)(hd.V + 1));
+    const size_t r_co = R.take(4 * (size_t)hd.E + 4), r_nl = R.take((size_t)hd.V + 1), r_el = R.take((size_t)hd.E + 1);
+    SIGMO_TRY(dreserve(c, c->raw, R.off, "raw data batch"));
+    unsigned char *rb = (unsigned char *)c->raw.p;
+    // from the caller's buffers: DMA when they are pinned, else the driver stages them
+    CUDA_TRY(c, cudaMemcpyAsync(rb + r_go, hd.goff, 8 * (size_t)(hd.G + 1), cudaMemcpyHostToDevice, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(rb + r_ro, hd.roff, 8 * (size_t)(hd.V + 1), cudaMemcpyHostToDevice, c->stream));
+    if (hd.E) CUDA_TRY(c, cudaMemcpyAsync(rb + r_co, hd.col, 4 * (size_t)hd.E, cudaMemcpyHostToDevice, c->stream));
+    if (hd.V) CUDA_TRY(c, cudaMemcpyAsync(rb + r_nl, hd.nlab, (size_t)hd.V, cudaMemcpyHostToDevice, c->stream));
+    if (hd.E) CUDA_TRY(c, cudaMemcpyAsync(rb + r_el, hd.elab, (size_t)hd.E, cudaMemcpyHostToDevice, c->stream));
+    raw_bytes = 8 * (size_t)(hd.G + 1) + 8 * (size_t)(hd.V + 1) + 5 * (size_t)hd.E + (size_t)hd.V;
+    Layout Ld;
+    pdd = plan_graphs(Ld, hd);
+    SIGMO_TRY(dreserve(c, c->dpk, Ld.off, "packed data batch"));
+    SIGMO_TRY(dreserve(c, c->ldinfo, 8 * 256 + 8 * 8, "load info"));
+    CUDA_TRY(c, cudaMemsetAsync(c->ldinfo.p, 0, 8 * 256, c->stream));
+    CUDA_TRY(c, cudaMemsetAsync((char *)c->ldinfo.p + 8 * 256, 0x7f, 8 * 8, c->stream));
+    unsigned char *pk = (unsigned char *)c->dpk.p;
+    DataLoadParams lp;
+    lp.G = hd.G;
+    lp.goff = (const int64_t *)(rb + r_go);
+    lp.roff = (const int64_t *)(rb + r_ro);
+    lp.col = (const int32_t *)(rb + r_co);
+    lp.nlab = rb + r_nl;
+    lp.elab = rb + r_el;
+    lp.goff32 = (int32_t *)(pk + pdd.goff);
+    lp.roff32 = (int32_t *)(pk + pdd.roff);
+    lp.label = pk + pdd.label;
+    lp.local = pk + pdd.local;
+    lp.nbr = (uint16_t *)(pk + pdd.nbr);
+    lp.hist = (unsigned long long *)c->ldinfo.p;
+    lp.err_graph = (long long *)((char *)c->ldinfo.p + 8 * 256);
+    if (hd.G == 0) CUDA_TRY(c, cudaMemsetAsync(pk + pdd.goff, 0, 4, c->stream));
+    if (hd.G == 0) CUDA_TRY(c, cudaMemsetAsync(pk + pdd.roff, 0, 4, c->stream));
+    CUDA_TRY(c, launch_load_data(lp, c->stream));
+    if (c->ldhost.cap < 8 * 264) {
+      if (c->ldhost.p) cudaFreeHost(c->ldhost.p);
+      c->ldhost.p = nullptr;
+      CUDA_TRY(c, cudaHostAlloc(&c->ldhost.p, 8 * 264, cudaHostAllocDefault));
+      c->ldhost.cap = 8 * 264;
+    }
+    CUDA_TRY(c, cudaMemcpyAsync(c->ldhost.p, c->ldinfo.p, 8 * 264, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    const long long *eg = (const long long *)c->ldhost.p + 256;
+    const char *why[5] = {"row_offsets decreasing", "column outside its graph", "self-loop", "duplicate edge",
+                          "asymmetric edge or edge label"};
+    long long first = -1;
+    int cls = -1;
+    for (int k = 0; k < 5; k++)
+      if (eg[k] < (long long)hd.G && (first < 0 || eg[k] < first)) {
+        first = eg[k];
+        cls = k;
+      }
+    if (cls >= 0) return set_err(c, SIGMO_ERR_INVALID_GRAPH, "data batch: data graph %lld: %s", first, why[cls]);
+  }
   const auto t1 = std::chrono::steady_clock::now();
   // bond classes = distinct query bond labels
   uint8_t bclass[256];
@@ -1245,7 +1351,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->state = 0;
   // label frequencies of the data batch (planner heuristic)
   std::vector<int64_t> freq(256, 0);
-  {
+  if (dev_load) {
+    const unsigned long long *h = (const unsigned long long *)c->ldhost.p;
+    for (int l = 0; l < 256; l++) freq[l] = (int64_t)h[l];
+  } else {
     std::vector<std::vector<int64_t>> part(64, std::vector<int64_t>(256, 0));
     parallel_for_graphs(hd.V, hd.V, [&](int th, int64_t a, int64_t b) {
       int64_t *f = part[th].data();
@@ -1297,7 +1406,9 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const size_t o_qinfo = L.take(4 * (size_t)hq.G + 4);
   const size_t o_qn = L.take((size_t)hq.V + 16);  // enumerate mode: local query node of each plan position
   const size_t o_qnb = L.take(8 * (size_t)hq.V + 16);  // lane neighbour support: query neighbours per plan position
-  const PackedOffsets pd = plan_graphs(L, hd);
+  HostGraphs hd_arena = hd;  // the data batch's packed arrays travel in the arena only when packed on the host
+  if (dev_load) hd_arena.G = hd_arena.V = hd_arena.E = 0;
+  const PackedOffsets pd = plan_graphs(L, hd_arena);
   const size_t o_tg0 = L.take(4 * tg0.size());
   const size_t o_tg1 = L.take(4 * tg1.size());
   // molecule tiles of the lane-join filter: <= 32 graphs and <= 1,024 nodes
@@ -1449,7 +1560,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     c->qgoff_host.assign(hq.goff, hq.goff + hq.G + 1);
     c->ent_R = -1;
   }
-  pack_graphs(hb, pd, hd);
+  if (!dev_load) pack_graphs(hb, pd, hd);
   memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
   memcpy(hb + o_tg1, tg1.data(), 4 * tg1.size());
   memcpy(hb + o_mt, mt.data(), 4 * mt.size());
@@ -1463,10 +1574,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   SIGMO_TRY(dreserve(c, c->arena, total, "input arena"));
   unsigned char *db = (unsigned char *)c->arena.p;
   CUDA_TRY(c, cudaMemcpyAsync(db, hb, total, cudaMemcpyHostToDevice, c->stream));
-  c->last.h2d_bytes = (int64_t)total;
+  c->last.h2d_bytes = (int64_t)(total + raw_bytes);
   CUDA_TRY(c, cudaEventRecord(c->h2d_done, c->stream));
   c->dq = dev_view(db, pq, hq);
-  c->dd = dev_view(db, pd, hd);
+  c->dd = dev_load ? dev_view((unsigned char *)c->dpk.p, pdd, hd) : dev_view(db, pd, hd);
   c->qp_row = (int32_t *)(db + o_row);
   c->qp_beoff = (int32_t *)(db + o_beoff);
   c->qp_be = (uint16_t *)(db + o_be);

@@ -257,6 +257,22 @@ struct ChunkParams {
 };
 
 
+// k_load_data (sigmo_load.cu): device-side validation + packing of a large data batch
+struct DataLoadParams {
+  long long G;
+  const int64_t *goff, *roff;  // raw CSR-GO (caller's layout, on the device)
+  const int32_t *col;
+  const uint8_t *nlab, *elab;
+  int32_t *goff32, *roff32;    // packed (DevGraphs)
+  uint8_t *label, *local;
+  uint16_t *nbr;
+  unsigned long long *hist;    // [256] node label histogram (query planner)
+  long long *err_graph;        // [5] first offending graph per error class (LLONG_MAX-ish = none):
+                               //     row offsets decreasing, column outside graph, self-loop, duplicate, asymmetric
+};
+constexpr long long kDeviceLoadMinNodes = 65536;  // smaller data batches are validated and packed on the host
+cudaError_t launch_load_data(const DataLoadParams &p, cudaStream_t st);
+
 // ---- launchers (sigmo_kernels.cu); all enqueue on `st` ----
 cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, cudaStream_t st);
 cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *out, cudaStream_t st);
