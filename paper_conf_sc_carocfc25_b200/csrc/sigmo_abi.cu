@@ -154,12 +154,9 @@ struct sigmo_ctx {
   std::vector<int32_t> ent_row;
   std::vector<int64_t> qgoff_host;  // query graph offsets (host copy, for the per-query row-word lists)
   int ent_R = -1;
-  int mol_extn = 0, mol_extw = 0;  // molecule-tile geometry (<= 32 graphs and <= 1,024 nodes per tile)
-  int n_mol_tiles = 0;
   int32_t *grp_narrow = nullptr, *grp_wide = nullptr;  // k_filter_lane groups (input arena)
   int NGN = 0, NGW = 0;
   DBuf nb4, mrec;                   // k_filter_lane: packed neighbours [VD], molecule records [ND]
-  int32_t *mol_tiles = nullptr;     // [n_mol_tiles + 1] first graph of each molecule tile
   uint32_t *adj_off = nullptr;      // [ND + 1] 32-bit word offset of each molecule's bond-class adjacency
   uint32_t *cand_units = nullptr;   // [ND + 1] candidate-window units before each molecule (x NDR = its cmol word offset)
   uint32_t cand_total = 0;
@@ -177,7 +174,7 @@ struct sigmo_ctx {
   int64_t enum_P = -1, enum_total = 0, enum_uniq = -1;
   int enum_stride = 8;
   // device-side load of large data batches (k_load_data)
-  DBuf raw, dpk, ldinfo;
+  DBuf raw, dpk, ldinfo, lay;
   Pinned ldhost;                    // histogram + error words read back
   // neighbour support on the lane path (k_support_lane)
   bool lane_ns = false;            // the last filter refined per-pair windows (join reads ns_win*)
@@ -991,7 +988,7 @@ void free_all(sigmo_ctx *c) {
                   &c->sig_tmp, &c->gstack, &c->adjb, &c->dense_tmp, &c->ent2, &c->nb4, &c->mrec,
                   &c->eoff, &c->ecur, &c->emaps, &c->esets, &c->ucnt, &c->uoff, &c->uniq, &c->etmp,
                   &c->ns_win32, &c->ns_win64, &c->ns_alive, &c->gm_old, &c->off_old, &c->ent_ns, &c->ns_bitmap,
-                  &c->ns_gm, &c->ns_cnt, &c->raw, &c->dpk, &c->ldinfo};
+                  &c->ns_gm, &c->ns_cnt, &c->raw, &c->dpk, &c->ldinfo, &c->lay};
   for (DBuf *b : bufs) dfree(c, *b);
 }
 
@@ -1038,6 +1035,12 @@ sigmo_status launch_dense(sigmo_ctx *c, int R, const QueryProg &P, uint32_t *bit
                           bool ns, int &launches) {
   const QueryProgMeta &m = P.meta;
   if (!c->tile_geom_ok) {
+    if ((int64_t)c->goff_host.size() != (int64_t)c->ND + 1) {  // device-loaded batch: read the offsets back
+      std::vector<int32_t> g32((size_t)c->ND + 1);
+      CUDA_TRY(c, cudaMemcpyAsync(g32.data(), c->dd.goff, 4 * g32.size(), cudaMemcpyDeviceToHost, c->stream));
+      CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+      c->goff_host.assign(g32.begin(), g32.end());
+    }
     HostGraphs hg;
     hg.G = c->ND;
     hg.V = c->VD;
@@ -1272,8 +1275,27 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const bool dev_load = data->num_nodes >= kDeviceLoadMinNodes && !(hl && atoi(hl));
   s = dev_load ? validate_light(data, msg, hd) : validate(data, 0, msg, hd);
   if (s != SIGMO_OK) return set_err(c, s, "data batch: %s", msg.c_str());
+  // bond classes = distinct query bond labels
+  uint8_t bclass[256];
+  memset(bclass, 255, sizeof(bclass));
+  {
+    bool seen[256] = {};
+    for (int64_t e = 0; e < hq.E; e++) seen[hq.elab[e]] = true;
+    int nb = 0;
+    for (int l = 0; l < 256; l++)
+      if (seen[l]) {
+        if (nb >= SIGMO_MAX_BOND_CLASSES)
+          return set_err(c, SIGMO_ERR_LIMIT, "more than %d distinct query bond labels", SIGMO_MAX_BOND_CLASSES);
+        bclass[l] = (uint8_t)nb++;
+      }
+    c->NB = nb;
+  }
   size_t raw_bytes = 0;
   PackedOffsets pdd{};
+  struct {
+    long long an, aw;
+    int cn, cw, maxn, nempty;
+  } lay{};
   if (dev_load) {
     CUDA_TRY(c, cudaEventSynchronize(c->h2d_done));  // the previous load's copies no longer read our buffers
     Layout R;
@@ -1291,7 +1313,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     Layout Ld;
     pdd = plan_graphs(Ld, hd);
     SIGMO_TRY(dreserve(c, c->dpk, Ld.off, "packed data batch"));
-    SIGMO_TRY(dreserve(c, c->ldinfo, 8 * 256 + 8 * 8, "load info"));
+    SIGMO_TRY(dreserve(c, c->ldinfo, 8 * 272, "load info"));
     CUDA_TRY(c, cudaMemsetAsync(c->ldinfo.p, 0, 8 * 256, c->stream));
     CUDA_TRY(c, cudaMemsetAsync((char *)c->ldinfo.p + 8 * 256, 0x7f, 8 * 8, c->stream));
     unsigned char *pk = (unsigned char *)c->dpk.p;
@@ -1312,14 +1334,36 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     if (hd.G == 0) CUDA_TRY(c, cudaMemsetAsync(pk + pdd.goff, 0, 4, c->stream));
     if (hd.G == 0) CUDA_TRY(c, cudaMemsetAsync(pk + pdd.roff, 0, 4, c->stream));
     CUDA_TRY(c, launch_load_data(lp, c->stream));
-    if (c->ldhost.cap < 8 * 264) {
+    // per-molecule layout (adjacency blocks, candidate units, group lists,
+    // molecule records) from the packed offsets, on the device
+    {
+      const size_t G1 = (size_t)hd.G + 1;
+      Layout LL;
+      const size_t l_ao = LL.take(4 * G1), l_cu = LL.take(4 * G1), l_gn = LL.take(4 * (G1 + 8)),
+                   l_gw = LL.take(4 * (G1 + 8)), l_sc = LL.take(layout_scan_bytes((int)hd.G));
+      SIGMO_TRY(dreserve(c, c->lay, LL.off, "molecule layout"));
+      SIGMO_TRY(dreserve(c, c->mrec, 16 * std::max<size_t>(G1, 2), "molecule records"));
+      unsigned char *lb = (unsigned char *)c->lay.p;
+      CUDA_TRY(c, cudaMemsetAsync(lb + l_gn, 0xff, 4 * (G1 + 8), c->stream));  // -1: empty group slots
+      CUDA_TRY(c, cudaMemsetAsync(lb + l_gw, 0xff, 4 * (G1 + 8), c->stream));
+      CUDA_TRY(c, launch_layout((const int32_t *)(pk + pdd.goff), (int)hd.G, std::max(c->NB, 0), lb + l_sc,
+                                (uint32_t *)(lb + l_ao), (uint32_t *)(lb + l_cu), (int32_t *)(lb + l_gn),
+                                (int32_t *)(lb + l_gw), (uint4 *)c->mrec.p,
+                                (long long *)((char *)c->ldinfo.p + 8 * 264), c->stream));
+      c->adj_off = (uint32_t *)(lb + l_ao);
+      c->cand_units = (uint32_t *)(lb + l_cu);
+      c->grp_narrow = (int32_t *)(lb + l_gn);
+      c->grp_wide = (int32_t *)(lb + l_gw);
+    }
+    if (c->ldhost.cap < 8 * 272) {
       if (c->ldhost.p) cudaFreeHost(c->ldhost.p);
       c->ldhost.p = nullptr;
-      CUDA_TRY(c, cudaHostAlloc(&c->ldhost.p, 8 * 264, cudaHostAllocDefault));
-      c->ldhost.cap = 8 * 264;
+      CUDA_TRY(c, cudaHostAlloc(&c->ldhost.p, 8 * 272, cudaHostAllocDefault));
+      c->ldhost.cap = 8 * 272;
     }
-    CUDA_TRY(c, cudaMemcpyAsync(c->ldhost.p, c->ldinfo.p, 8 * 264, cudaMemcpyDeviceToHost, c->stream));
+    CUDA_TRY(c, cudaMemcpyAsync(c->ldhost.p, c->ldinfo.p, 8 * 272, cudaMemcpyDeviceToHost, c->stream));
     CUDA_TRY(c, cudaStreamSynchronize(c->stream));
+    memcpy(&lay, (const char *)c->ldhost.p + 8 * 264, sizeof(lay));
     const long long *eg = (const long long *)c->ldhost.p + 256;
     const char *why[5] = {"row_offsets decreasing", "column outside its graph", "self-loop", "duplicate edge",
                           "asymmetric edge or edge label"};
@@ -1333,21 +1377,6 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     if (cls >= 0) return set_err(c, SIGMO_ERR_INVALID_GRAPH, "data batch: data graph %lld: %s", first, why[cls]);
   }
   const auto t1 = std::chrono::steady_clock::now();
-  // bond classes = distinct query bond labels
-  uint8_t bclass[256];
-  memset(bclass, 255, sizeof(bclass));
-  {
-    bool seen[256] = {};
-    for (int64_t e = 0; e < hq.E; e++) seen[hq.elab[e]] = true;
-    int nb = 0;
-    for (int l = 0; l < 256; l++)
-      if (seen[l]) {
-        if (nb >= SIGMO_MAX_BOND_CLASSES)
-          return set_err(c, SIGMO_ERR_LIMIT, "more than %d distinct query bond labels", SIGMO_MAX_BOND_CLASSES);
-        bclass[l] = (uint8_t)nb++;
-      }
-    c->NB = nb;
-  }
   c->state = 0;
   // label frequencies of the data batch (planner heuristic)
   std::vector<int64_t> freq(256, 0);
@@ -1368,7 +1397,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
 
   // per-tile graph ranges of the filter for TW = 32 (1,024 nodes per tile)
   std::vector<int32_t> tg0, tg1;
-  {
+  if (!dev_load) {  // device-loaded batches: the dense filter finds its tiles' graphs by binary search
     const int64_t W = (hd.V + 31) / 32, tiles = (W + 31) / 32;
     tg0.resize((size_t)tiles + 1);
     tg1.resize((size_t)tiles + 1);
@@ -1383,7 +1412,9 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->induced_loaded = c->induced;
   {
     int64_t maxn_h = 0, maxq_h = 0;
-    for (int64_t g = 0; g < hd.G; g++) maxn_h = std::max<int64_t>(maxn_h, hd.goff[g + 1] - hd.goff[g]);
+    if (dev_load) maxn_h = lay.maxn;
+    else
+      for (int64_t g = 0; g < hd.G; g++) maxn_h = std::max<int64_t>(maxn_h, hd.goff[g + 1] - hd.goff[g]);
     for (int64_t g = 0; g < hq.G; g++) maxq_h = std::max<int64_t>(maxq_h, hq.goff[g + 1] - hq.goff[g]);
     const char *legacy = getenv("SIGMO_JOIN_LEGACY");
     lane_ok = maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
@@ -1411,26 +1442,18 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const PackedOffsets pd = plan_graphs(L, hd_arena);
   const size_t o_tg0 = L.take(4 * tg0.size());
   const size_t o_tg1 = L.take(4 * tg1.size());
-  // molecule tiles of the lane-join filter: <= 32 graphs and <= 1,024 nodes
-  std::vector<int32_t> mt;
-  {
-    int64_t g = 0;
-    mt.push_back(0);
-    while (g < hd.G) {
-      int64_t k = 0, nodes = 0;
-      while (g < hd.G && k < 32 && (k == 0 || nodes + (hd.goff[g + 1] - hd.goff[g]) <= 1024)) {
-        nodes += hd.goff[g + 1] - hd.goff[g];
-        g++;
-        k++;
-      }
-      mt.push_back((int32_t)g);
-    }
-  }
-  const size_t o_mt = L.take(4 * mt.size());
   // bond-class adjacency layout (k_join_lane): per molecule class-major,
   // 32-bit masks for <= 32-node molecules, 64-bit (even word offset) otherwise
-  std::vector<uint32_t> aoff((size_t)hd.G + 1, 0);
-  {
+  std::vector<uint32_t> aoff(dev_load ? 1 : (size_t)hd.G + 1, 0), cu(dev_load ? 1 : (size_t)hd.G + 1, 0);
+  std::vector<int32_t> grpn, grpw;
+  uint64_t adj_words_total = 0, cand_units_total = 0;
+  if (dev_load) {
+    // computed on the device (launch_layout): narrow molecules first, wide ones from an even offset
+    adj_words_total = (((uint64_t)lay.an + 1) & ~1ull) + (uint64_t)lay.aw;
+    cand_units_total = (((uint64_t)lay.cn + 1) & ~1ull) + 2ull * (uint64_t)lay.cw;
+    if (adj_words_total + 4 >= (1ull << 32)) lane_ok = false;
+    if ((unsigned long long)std::max<int64_t>(hq.V, 1) * (cand_units_total + 2) >= (1ull << 32)) lane_ok = false;
+  } else {
     uint64_t w = 0;
     for (int64_t g = 0; g < hd.G; g++) {
       const int64_t n = hd.goff[g + 1] - hd.goff[g];
@@ -1440,14 +1463,11 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     }
     w = (w + 1) & ~1ull;
     aoff[hd.G] = (uint32_t)std::min<uint64_t>(w, 0xffffffffull);
+    adj_words_total = w;
     if (w + 4 >= (1ull << 32)) lane_ok = false;  // + the all-ones and all-zeros sentinel entries
-  }
-  const size_t o_ao = L.take(4 * aoff.size());
-  // molecule-padded candidate windows (filter output, join input): per
-  // molecule NDR windows of one 32-bit word (<= 32 nodes) or two (64-bit,
-  // even unit offset); molecule g starts at word NDR * cu[g]
-  std::vector<uint32_t> cu((size_t)hd.G + 1, 0);
-  {
+    // molecule-padded candidate windows (filter output, join input): per
+    // molecule NDR windows of one 32-bit word (<= 32 nodes) or two (64-bit,
+    // even unit offset); molecule g starts at word NDR * cu[g]
     uint64_t u = 0;
     for (int64_t g = 0; g < hd.G; g++) {
       const int64_t n = hd.goff[g + 1] - hd.goff[g];
@@ -1456,17 +1476,18 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       u += n > 32 ? 2 : 1;
     }
     cu[hd.G] = (uint32_t)std::min<uint64_t>(u, 0xffffffffull);
+    cand_units_total = u;
     if ((unsigned long long)std::max<int64_t>(hq.V, 1) * (u + 2) >= (1ull << 32)) lane_ok = false;
+    // k_filter_lane groups: 4 molecules of <= 32 atoms / 2 of 33-64 atoms (-1 = empty slot)
+    for (int64_t g = 0; g < hd.G; g++) {
+      const int64_t n = hd.goff[g + 1] - hd.goff[g];
+      (n > 32 ? grpw : grpn).push_back((int32_t)g);
+    }
+    while (grpn.size() % 4) grpn.push_back(-1);
+    while (grpw.size() % 2) grpw.push_back(-1);
   }
+  const size_t o_ao = L.take(4 * aoff.size());
   const size_t o_cu = L.take(4 * cu.size());
-  // k_filter_lane groups: 4 molecules of <= 32 atoms / 2 of 33-64 atoms (-1 = empty slot)
-  std::vector<int32_t> grpn, grpw;
-  for (int64_t g = 0; g < hd.G; g++) {
-    const int64_t n = hd.goff[g + 1] - hd.goff[g];
-    (n > 32 ? grpw : grpn).push_back((int32_t)g);
-  }
-  while (grpn.size() % 4) grpn.push_back(-1);
-  while (grpw.size() % 2) grpw.push_back(-1);
   const size_t o_grpn = L.take(4 * grpn.size() + 16);
   const size_t o_grpw = L.take(4 * grpw.size() + 16);
   const size_t total = L.off;
@@ -1563,7 +1584,6 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   if (!dev_load) pack_graphs(hb, pd, hd);
   memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
   memcpy(hb + o_tg1, tg1.data(), 4 * tg1.size());
-  memcpy(hb + o_mt, mt.data(), 4 * mt.size());
   memcpy(hb + o_ao, aoff.data(), 4 * aoff.size());
   memcpy(hb + o_cu, cu.data(), 4 * cu.size());
   if (!grpn.empty()) memcpy(hb + o_grpn, grpn.data(), 4 * grpn.size());
@@ -1577,23 +1597,35 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->last.h2d_bytes = (int64_t)(total + raw_bytes);
   CUDA_TRY(c, cudaEventRecord(c->h2d_done, c->stream));
   c->dq = dev_view(db, pq, hq);
-  c->dd = dev_load ? dev_view((unsigned char *)c->dpk.p, pdd, hd) : dev_view(db, pd, hd);
+  if (dev_load) {
+    HostGraphs hd0 = hd;
+    hd0.G = 0;  // dev_view's O(#graphs) maximum: known from the device layout pass
+    c->dd = dev_view((unsigned char *)c->dpk.p, pdd, hd0);
+    c->dd.num_graphs = (int)hd.G;
+    c->dd.max_nodes = lay.maxn;
+  } else {
+    c->dd = dev_view(db, pd, hd);
+  }
   c->qp_row = (int32_t *)(db + o_row);
   c->qp_beoff = (int32_t *)(db + o_beoff);
   c->qp_be = (uint16_t *)(db + o_be);
   c->bclass = db + o_bc;
-  c->tile_g0 = (int32_t *)(db + o_tg0);
-  c->mol_tiles = (int32_t *)(db + o_mt);
-  c->adj_off = (uint32_t *)(db + o_ao);
-  c->adj_words = aoff[hd.G];
-  c->cand_units = (uint32_t *)(db + o_cu);
-  c->cand_total = cu[hd.G];
-  c->n_mol_tiles = (int)mt.size() - 1;
-  c->grp_narrow = (int32_t *)(db + o_grpn);
-  c->grp_wide = (int32_t *)(db + o_grpw);
-  c->NGN = (int)(grpn.size() / 4);
-  c->NGW = (int)(grpw.size() / 2);
-  c->tile_g1 = (int32_t *)(db + o_tg1);
+  c->tile_g0 = dev_load ? nullptr : (int32_t *)(db + o_tg0);
+  if (!dev_load) {
+    c->adj_off = (uint32_t *)(db + o_ao);
+    c->cand_units = (uint32_t *)(db + o_cu);
+    c->grp_narrow = (int32_t *)(db + o_grpn);
+    c->grp_wide = (int32_t *)(db + o_grpw);
+    c->NGN = (int)(grpn.size() / 4);
+    c->NGW = (int)(grpw.size() / 2);
+  } else {
+    c->NGN = (lay.cn + 3) / 4;
+    c->NGW = (lay.cw + 1) / 2;
+  }
+  c->adj_words = (uint32_t)std::min<uint64_t>(adj_words_total, 0xffffffffull);
+  c->cand_total = (uint32_t)std::min<uint64_t>(cand_units_total, 0xffffffffull);
+
+  c->tile_g1 = dev_load ? nullptr : (int32_t *)(db + o_tg1);
   c->qp_info = (uint32_t *)(db + o_info);
   c->qp_ent = (const int4 *)(db + o_ent);
   c->qp_non = (const uint32_t *)(db + o_non);
@@ -1612,22 +1644,19 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   c->maxn = c->dd.max_nodes;
   c->NW = c->maxn <= 64 ? 1 : (c->maxn <= 128 ? 2 : 4);
   c->has_empty_graph = false;
-  for (int64_t g = 0; g < hd.G && !c->has_empty_graph; g++) c->has_empty_graph = hd.goff[g + 1] == hd.goff[g];
+  if (dev_load) c->has_empty_graph = lay.nempty > 0;
+  else
+    for (int64_t g = 0; g < hd.G && !c->has_empty_graph; g++) c->has_empty_graph = hd.goff[g + 1] == hd.goff[g];
   c->W = (c->VD + 31) / 32;
   c->Wpad = ((c->W + 31) / 32) * 32;
   if (c->Wpad == 0) c->Wpad = 32;
   // dense-tile geometry: now if the dense path is the only one, else lazily
-  c->goff_host.assign(hd.goff, hd.goff + hd.G + 1);
+  if (dev_load) c->goff_host.clear();  // read back from the device if the dense path ever needs it
+  else c->goff_host.assign(hd.goff, hd.goff + hd.G + 1);
   c->tile_geom_ok = false;
   if (!lane_ok) {
     tile_geometry(c, hd);
     c->tile_geom_ok = true;
-  }
-  {
-    int extn = 1;
-    for (int t = 0; t < c->n_mol_tiles; t++) extn = std::max<int>(extn, (int)(hd.goff[mt[t + 1]] - hd.goff[mt[t]]));
-    c->mol_extn = extn;
-    c->mol_extw = (extn + 31) / 32;
   }
   c->NBE = (int)plan.be.size();
   c->plan_smem = 0;  // plans are read through the read-only cache
@@ -1682,9 +1711,9 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     CUDA_TRY(c, cudaMemsetAsync((uint32_t *)c->adjb.p + c->adj_words, 0xff, 8, c->stream));
     CUDA_TRY(c, cudaMemsetAsync((uint32_t *)c->adjb.p + c->adj_words + 2, 0, 8, c->stream));
     SIGMO_TRY(dreserve(c, c->nb4, 4 * (size_t)std::max(c->VD, 1), "packed neighbours"));
-    SIGMO_TRY(dreserve(c, c->mrec, 16 * (size_t)std::max(c->ND, 1), "molecule records"));
+    if (!dev_load) SIGMO_TRY(dreserve(c, c->mrec, 16 * (size_t)std::max(c->ND, 1), "molecule records"));
     CUDA_TRY(c, launch_adjb(c->dd, c->bclass, c->NB, c->adj_off, (uint32_t *)c->adjb.p, (uint32_t *)c->nb4.p, c->stream));
-    CUDA_TRY(c, launch_mrec(c->dd.goff, c->adj_off, c->cand_units, c->ND, (uint4 *)c->mrec.p, c->stream));
+    if (!dev_load) CUDA_TRY(c, launch_mrec(c->dd.goff, c->adj_off, c->cand_units, c->ND, (uint4 *)c->mrec.p, c->stream));
   }
   SIGMO_TRY(dreserve(c, c->pair_result, 8 * (size_t)std::max(pair_cap, 1ll), "pair results"));
   SIGMO_TRY(dreserve(c, c->jcnt, 8 * ((size_t)c->NQ + 8), "join counters"));  // + the second claim counter
@@ -1693,8 +1722,10 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     auto ms = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
       return std::chrono::duration<double, std::milli>(b - a).count();
     };
-    fprintf(stderr, "sigmo load: validate %.1f  plan %.1f  layout %.1f  pack %.1f  h2d+device %.1f  (%.1f) ms\n",
-            ms(t0, t1), ms(t1, t2), ms(t2, t3), ms(t3, t4), ms(t4, t5), 0.0);
+    cudaStreamSynchronize(c->stream);
+    const auto t6 = std::chrono::steady_clock::now();
+    fprintf(stderr, "sigmo load: validate(+device pass) %.1f  plan %.1f  layout %.1f  pack %.1f  h2d+device enqueue %.1f  "
+            "drain %.1f ms\n", ms(t0, t1), ms(t1, t2), ms(t2, t3), ms(t3, t4), ms(t4, t5), ms(t5, t6));
   }
   c->state = 1;
   c->err.clear();

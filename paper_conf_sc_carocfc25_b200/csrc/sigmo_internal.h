@@ -272,6 +272,10 @@ struct DataLoadParams {
 };
 constexpr long long kDeviceLoadMinNodes = 65536;  // smaller data batches are validated and packed on the host
 cudaError_t launch_load_data(const DataLoadParams &p, cudaStream_t st);
+// per-molecule adjacency / candidate layout of a device-loaded batch (sigmo_load.cu)
+size_t layout_scan_bytes(int G);
+cudaError_t launch_layout(const int32_t *goff, int G, int NB, void *scratch, uint32_t *aoff, uint32_t *cu,
+                          int32_t *grpn, int32_t *grpw, uint4 *mrec, long long *info_out, cudaStream_t st);
 
 // ---- launchers (sigmo_kernels.cu); all enqueue on `st` ----
 cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, cudaStream_t st);

@@ -8,6 +8,8 @@
 // the packed device form (int32 offsets, molecule-local neighbour | bond
 // label, local index) and the label histogram the query planner uses.
 // One thread per graph (graphs are <= 256 atoms and sparse).
+#include <cub/cub.cuh>
+
 #include "sigmo_internal.h"
 
 namespace sigmo {
@@ -68,6 +70,111 @@ cudaError_t launch_load_data(const DataLoadParams &p, cudaStream_t st) {
   if (p.G <= 0) return cudaSuccess;
   k_load_data<<<(unsigned)((p.G + 255) / 256), 256, 0, st>>>(p);
   return cudaGetLastError();
+}
+
+}  // namespace sigmo
+
+// ---------------------------------------------------------------------------
+// Per-molecule layout of a device-loaded batch, from the packed offsets:
+// bond-class adjacency blocks ([NB+1][n] words, u64 for > 32 atoms) and
+// candidate-window units (NDR x 1 word, or 2 for > 32 atoms), narrow
+// molecules first, then the wide ones from an even word / unit offset; the
+// k_filter_lane group lists (narrow / wide molecule ids); the molecule records
+// of the lane filter; the batch maxima.  One exclusive scan of per-molecule
+// sizes, then a scatter.
+// ---------------------------------------------------------------------------
+namespace sigmo {
+namespace {
+struct LayAcc {
+  long long an, aw;  // adjacency words of narrow / wide molecules
+  int cn, cw;        // narrow / wide molecules
+  int maxn, nempty;  // largest molecule, empty molecules
+};
+struct LayOp {
+  __host__ __device__ __forceinline__ LayAcc operator()(const LayAcc &x, const LayAcc &y) const {
+    LayAcc r;
+    r.an = x.an + y.an;
+    r.aw = x.aw + y.aw;
+    r.cn = x.cn + y.cn;
+    r.cw = x.cw + y.cw;
+    r.maxn = x.maxn > y.maxn ? x.maxn : y.maxn;
+    r.nempty = x.nempty + y.nempty;
+    return r;
+  }
+};
+
+__global__ void k_layout_sizes(const int32_t *goff, int G, int NB, LayAcc *acc) {
+  const int g = blockIdx.x * blockDim.x + threadIdx.x;
+  if (g > G) return;
+  LayAcc a{0, 0, 0, 0, 0, 0};
+  if (g < G) {
+    const int n = goff[g + 1] - goff[g];
+    const bool wide = n > 32;
+    a.an = wide ? 0 : (long long)n * (NB + 1);
+    a.aw = wide ? 2ll * n * (NB + 1) : 0;
+    a.cn = wide ? 0 : 1;
+    a.cw = wide ? 1 : 0;
+    a.maxn = n;
+    a.nempty = n == 0;
+  }
+  acc[g] = a;
+}
+
+__global__ void k_layout_scatter(const int32_t *goff, int G, const LayAcc *pre, uint32_t *aoff, uint32_t *cu,
+                                 int32_t *grpn, int32_t *grpw, uint4 *mrec) {
+  const int g = blockIdx.x * blockDim.x + threadIdx.x;
+  if (g > G) return;
+  const LayAcc tot = pre[G];
+  const unsigned long long an_even = ((unsigned long long)tot.an + 1ull) & ~1ull;
+  const unsigned long long cn_even = ((unsigned long long)tot.cn + 1ull) & ~1ull;
+  if (g == G) {
+    aoff[G] = (uint32_t)(an_even + (unsigned long long)tot.aw);
+    cu[G] = (uint32_t)(cn_even + 2ull * (unsigned long long)tot.cw);
+    return;
+  }
+  const LayAcc p = pre[g];
+  const int a = goff[g], n = goff[g + 1] - a;
+  uint32_t ao, c;
+  if (n > 32) {
+    ao = (uint32_t)(an_even + (unsigned long long)p.aw);
+    c = (uint32_t)(cn_even + 2ull * (unsigned long long)p.cw);
+    grpw[p.cw] = g;
+  } else {
+    ao = (uint32_t)p.an;
+    c = (uint32_t)p.cn;
+    grpn[p.cn] = g;
+  }
+  aoff[g] = ao;
+  cu[g] = c;
+  mrec[g] = make_uint4((unsigned)a, (unsigned)n, ao, c);
+}
+}  // namespace
+
+size_t layout_scan_bytes(int G) {
+  size_t tb = 0;
+  cub::DeviceScan::ExclusiveScan(nullptr, tb, (const LayAcc *)nullptr, (LayAcc *)nullptr, LayOp(),
+                                 LayAcc{0, 0, 0, 0, 0, 0}, G + 1, (cudaStream_t)0);
+  return tb + 2 * sizeof(LayAcc) * ((size_t)G + 1) + 256;
+}
+
+// scratch: layout_scan_bytes(G) bytes; info_out (device, 32 B): {int64 an, aw; int32 cn, cw, maxn, nempty} totals
+cudaError_t launch_layout(const int32_t *goff, int G, int NB, void *scratch, uint32_t *aoff, uint32_t *cu,
+                          int32_t *grpn, int32_t *grpw, uint4 *mrec, long long *info_out, cudaStream_t st) {
+  LayAcc *acc = (LayAcc *)scratch;
+  LayAcc *pre = acc + (G + 1);
+  void *tmp = (void *)(pre + (G + 1));
+  size_t tb = 0;
+  cudaError_t e = cub::DeviceScan::ExclusiveScan(nullptr, tb, acc, pre, LayOp(), LayAcc{0, 0, 0, 0, 0, 0}, G + 1, st);
+  if (e != cudaSuccess) return e;
+  const unsigned blocks = (unsigned)((G + 1 + 255) / 256);
+  k_layout_sizes<<<blocks, 256, 0, st>>>(goff, G, NB, acc);
+  e = cub::DeviceScan::ExclusiveScan(tmp, tb, acc, pre, LayOp(), LayAcc{0, 0, 0, 0, 0, 0}, G + 1, st);
+  if (e != cudaSuccess) return e;
+  k_layout_scatter<<<blocks, 256, 0, st>>>(goff, G, pre, aoff, cu, grpn, grpw, mrec);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  // the totals pre[G] for the host: {int64 an, aw; int32 cn, cw, maxn, nempty}
+  return cudaMemcpyAsync(info_out, pre + G, sizeof(LayAcc), cudaMemcpyDeviceToDevice, st);
 }
 
 }  // namespace sigmo
