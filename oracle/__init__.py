@@ -31,6 +31,7 @@ _lib = None
 FIND_ALL = 0
 FIND_FIRST = 1
 INDUCED = 2  # mode bit: induced-subgraph embeddings (R21)
+WILDCARD = 4  # mode bit: query atom label 0 = any atom, bond label 0 = any bond (R22)
 
 
 class _Batch(ctypes.Structure):
@@ -136,7 +137,7 @@ def enumerate_pair(Q, D, q: int, g: int, mode: int = FIND_ALL) -> np.ndarray:
     """Every embedding of query q in data graph g (enumerate mode, SURVEY
     8(f) N1): int32 [n, n_q], row k = the molecule-local data node of each
     query node (query node order) in the k-th embedding.  mode: FIND_ALL or
-    INDUCED (Find First is meaningless here)."""
+    INDUCED and/or WILDCARD (Find First is meaningless here)."""
     lib = _load()
     qs, ds = _as_struct(Q), _as_struct(D)
     nq = int(Q.graph_offsets[q + 1] - Q.graph_offsets[q])

@@ -17,7 +17,15 @@ def _induced_ok(f, qedges, bond, nq):
     return all((f[u], f[v]) not in bond for u in range(nq) for v in range(nq) if u != v and (u, v) not in qadj)
 
 
-def brute_embeddings(qgraph, dgraph, induced: bool = False):
+def _label_ok(ql, dl, wildcard):
+    return ql == dl or (wildcard and ql == 0)          # (1); wildcard '*' = label 0 (R22)
+
+
+def _bond_ok(db, qb, wildcard):
+    return db is not None and (db == qb or (wildcard and qb == 0))  # (2); wildcard '~' = bond 0
+
+
+def brute_embeddings(qgraph, dgraph, induced: bool = False, wildcard: bool = False):
     """Yield every embedding f (tuple, f[i] = data node of query node i)."""
     qlab, qedges = qgraph
     dlab, dedges = dgraph
@@ -27,38 +35,22 @@ def brute_embeddings(qgraph, dgraph, induced: bool = False):
         bond[(u, v)] = b
         bond[(v, u)] = b
     for f in itertools.permutations(range(nd), nq):
-        if any(qlab[i] != dlab[f[i]] for i in range(nq)):           # condition (1)
+        if any(not _label_ok(qlab[i], dlab[f[i]], wildcard) for i in range(nq)):           # condition (1)
             continue
-        if any(bond.get((f[u], f[v])) != b for (u, v, b) in qedges):  # condition (2) + bond labels
+        if any(not _bond_ok(bond.get((f[u], f[v])), b, wildcard) for (u, v, b) in qedges):  # condition (2)
             continue
         if induced and not _induced_ok(f, qedges, bond, nq):
             continue
         yield f
 
 
-def brute_count(qgraph, dgraph, induced: bool = False) -> int:
+def brute_count(qgraph, dgraph, induced: bool = False, wildcard: bool = False) -> int:
     """qgraph/dgraph: (labels, [(u, v, bond), ...]) with local ids."""
-    qlab, qedges = qgraph
-    dlab, dedges = dgraph
-    nq, nd = len(qlab), len(dlab)
-    bond = {}
-    for (u, v, b) in dedges:
-        bond[(u, v)] = b
-        bond[(v, u)] = b
-    total = 0
-    for f in itertools.permutations(range(nd), nq):
-        if any(qlab[i] != dlab[f[i]] for i in range(nq)):           # condition (1)
-            continue
-        if any(bond.get((f[u], f[v])) != b for (u, v, b) in qedges):  # condition (2) + bond labels
-            continue
-        if induced and not _induced_ok(f, qedges, bond, nq):
-            continue
-        total += 1
-    return total
+    return sum(1 for _ in brute_embeddings(qgraph, dgraph, induced, wildcard))
 
 
-def brute_dense(qgraphs, dgraphs, find_first: bool = False, induced: bool = False):
-    out = [[brute_count(q, d, induced) for d in dgraphs] for q in qgraphs]
+def brute_dense(qgraphs, dgraphs, find_first: bool = False, induced: bool = False, wildcard: bool = False):
+    out = [[brute_count(q, d, induced, wildcard) for d in dgraphs] for q in qgraphs]
     if find_first:
         out = [[1 if c else 0 for c in row] for row in out]
     return out

@@ -35,6 +35,12 @@
  *   step 3b: non[i] = {j < i : (pi_j, pi_i) not in E_q}
  *   step 4b: require no data edge between f(pi_j) and v for j in non[i].
  *
+ * Wildcard mode (mode bit 2, value 4, the paper's stated
+ * next step P:2639-2645; R22): a query atom label 0 is the SMARTS
+ * '*' (any atom) and a query bond label 0 the SMARTS '~' (any bond):
+ *                   (1') L_q(v) == 0  or  L_q(v) == L_g(f(v))
+ *                   (2') (f(u),f(v)) in E_g and (b == 0 or bond_g(f(u),f(v)) == b)
+ *
  * Enumerate mode (NLSM outputs the embeddings themselves,
  * P:446-453, and atom typing needs every isomorphism): the same
  * search, but step 5 appends the leaf's mapping f, written in query node
@@ -133,6 +139,7 @@ typedef struct {
   uint8_t used[256];
   int find_first;
   int induced;
+  int wildcard;         /* mode bit 2: query label 0 = any atom, bond 0 = any bond */
   int overflow;
   uint64_t work;        /* search-tree nodes visited (informational) */
 } search;
@@ -149,11 +156,13 @@ static uint64_t rec(search *S, int depth) {
   }
   uint64_t total = 0;
   for (int v = 0; v < S->ng; v++) {
-    if (S->used[v] || S->glab[v] != S->P->label[depth]) continue;
+    if (S->used[v]) continue;
+    if (S->glab[v] != S->P->label[depth] && !(S->wildcard && S->P->label[depth] == 0)) continue; /* (1), (1') */
     int ok = 1;
     for (int k = 0; k < S->P->nback[depth]; k++) {
       int u = S->map[S->P->back_j[depth][k]];
-      if (S->adjm[u * S->ng + v] != S->P->back_b[depth][k]) { ok = 0; break; }
+      const int16_t b = S->adjm[u * S->ng + v];
+      if (b < 0 || (b != S->P->back_b[depth][k] && !(S->wildcard && S->P->back_b[depth][k] == 0))) { ok = 0; break; }
     }
     if (!ok) continue;
     if (S->induced)  /* step 4b: no data edge (any bond) between v and f(pi_j) for j in non[i] */
@@ -214,6 +223,7 @@ static uint64_t count_one(job *J, const qplan *P, int ng, const uint8_t *glab, c
   S.adjm = adjm;
   S.find_first = J->find_first & 1;
   S.induced = (J->find_first >> 1) & 1;
+  S.wildcard = (J->find_first >> 2) & 1;
   S.overflow = 0;
   S.work = 0;
   S.emb = NULL;
@@ -352,6 +362,7 @@ int oracle_enumerate_pair(const oracle_batch *Q, const oracle_batch *D, int64_t 
     S.adjm = adjm;
     S.find_first = 0;
     S.induced = (mode >> 1) & 1;
+    S.wildcard = (mode >> 2) & 1;
     S.overflow = 0;
     S.work = 0;
     S.emb = out;

@@ -317,3 +317,59 @@ def test_enumerate_closed_forms():
     for q in range(Q.num_graphs):
         for g in range(D.num_graphs):
             assert len(oracle.enumerate_pair(Q, D, q, g)) == dense[q, g]
+
+
+# ---------------------------------------------------------------- N3 wildcard mode
+WC = oracle.WILDCARD
+ANY = 0  # query atom label 0 = SMARTS '*', query bond label 0 = SMARTS '~' (R22)
+
+
+def test_wildcard_closed_forms():
+    """'*' matches every atom; '*~*' every bond twice (2|E|); 'C~C' any C-C
+    bond, 'C-C' only single ones; a 6-ring of '*' atoms and '~' bonds has the
+    12 automorphic embeddings in benzene AND in cyclohexane, while the
+    aromatic-bond ring has none in cyclohexane (R22)."""
+    benzene, cyclohexane = ring(6, C, 4), ring(6, C, 1)
+    mol = ([C, C, C, O], [(0, 1, 2), (1, 2, 1), (2, 3, 1)])  # C=C-C-O
+    assert count([([ANY], [])], [benzene, mol], WC).tolist() == [[6, 4]]
+    assert count([([ANY, ANY], [(0, 1, ANY)])], [benzene, mol], WC).tolist() == [[12, 6]]
+    assert count([([C, C], [(0, 1, ANY)])], [mol], WC).tolist() == [[4]]
+    assert count([([C, C], [(0, 1, 1)])], [mol], WC).tolist() == [[2]]
+    assert count([([C, ANY], [(0, 1, 1)])], [mol], WC).tolist() == [[3]]  # C1-C2 both ways, C2-O3
+    wring = ([ANY] * 6, [(i, (i + 1) % 6, ANY) for i in range(6)])
+    assert count([wring, benzene], [benzene, cyclohexane], WC).tolist() == [[12, 12], [12, 0]]
+    # without the wildcard bit, label 0 / bond 0 are literal values (nothing in these molecules)
+    assert count([([ANY], [])], [benzene], oracle.FIND_ALL).tolist() == [[0]]
+
+
+def test_wildcard_vs_brute_force_random_tiny():
+    """Wildcard mode vs brute force (conditions (1') and (2')), monomorphic and
+    induced, Find All and Find First, on random tiny graphs whose queries have
+    wildcard atoms and bonds; with no label-0 atom or bond the mode equals the
+    exact one."""
+    from oracle.brute import brute_count
+    rng = np.random.default_rng(4242)
+    qs, ds = [], []
+    for _ in range(80):
+        ds.append(synth.random_labelled_graph(rng, int(rng.integers(1, 8)), float(rng.uniform(0.2, 0.8)),
+                                              labels=(C, N, O), bonds=(1, 2)))
+    for _ in range(60):
+        lab, edges = synth.random_labelled_graph(rng, int(rng.integers(1, 5)), float(rng.uniform(0.3, 1.0)),
+                                                 labels=(C, N), bonds=(1, 2))
+        lab = [ANY if rng.random() < 0.3 else x for x in lab]
+        edges = [(u, v, ANY if rng.random() < 0.3 else b) for (u, v, b) in edges]
+        qs.append((lab, edges))
+    n_pos = 0
+    for induced in (False, True):
+        im = oracle.INDUCED if induced else 0
+        res = count(qs, ds, WC | im)
+        ff = count(qs, ds, WC | im | oracle.FIND_FIRST)
+        for i, q in enumerate(qs):
+            for j, d in enumerate(ds):
+                b = brute_count(q, d, induced=induced, wildcard=True)
+                assert res[i, j] == b, (i, j, induced)
+                assert ff[i, j] == (1 if b else 0)
+                n_pos += b > 0
+    assert n_pos > 200
+    exact = [q for q in qs if ANY not in q[0] and all(b != ANY for (_, _, b) in q[1])]
+    assert np.array_equal(count(exact, ds, WC), count(exact, ds))
