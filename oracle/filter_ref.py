@@ -62,7 +62,7 @@ def _bfs_dist(adj, src, lo, hi):
     return dist
 
 
-def raw_signatures(B, max_radius: int, graphs=None):
+def raw_signatures(B, max_radius: int, graphs=None, skip_wildcards: bool = False):
     """Raw (unsaturated) counts S[k][v, f] for k = 1..max_radius, following
     GenerateSignatures (Alg. 1 l.11-18): for each node v and each k, add one to
     S(v, field(L(u))) for every u in the ring R_k(v) = N^k(v) \\ N^{k-1}(v).
@@ -71,6 +71,10 @@ def raw_signatures(B, max_radius: int, graphs=None):
     adj = _adjacency(B)
     V = B.num_nodes
     fld = np.array([field_of(int(x)) for x in B.node_labels], np.int64)
+    # wildcard mode (R22): a '*' query atom (label 0) has no known label, so it
+    # adds to no field of its neighbours' signatures (sound: the data
+    # signature then dominates on the known labels only)
+    wild = (B.node_labels == 0) if skip_wildcards else np.zeros(V, bool)
     S = np.zeros((V, NF), np.int64)
     out = {}
     dists = {}
@@ -83,7 +87,8 @@ def raw_signatures(B, max_radius: int, graphs=None):
         for v, (lo, dist) in dists.items():
             ring = np.nonzero(dist == k)[0] + lo          # R_k(v)
             for u in ring:
-                S[v, fld[u]] += 1                          # S(v, L(u)) <- S(v, L(u)) + 1
+                if not wild[u]:
+                    S[v, fld[u]] += 1                      # S(v, L(u)) <- S(v, L(u)) + 1
         out[k] = S.copy()
     return out
 
@@ -106,7 +111,7 @@ def signatures(B, radius: int, graphs=None):
     return pack(saturate(raw_signatures(B, radius, graphs)[radius]))
 
 
-def candidates_bool(Q, D, levels: int, data_graphs=None, q_rows=None):
+def candidates_bool(Q, D, levels: int, data_graphs=None, q_rows=None, wildcard: bool = False):
     """Boolean candidate matrix C_L [VQ, VD] (Alg. 1 Filter):
     C_1 = InitializeCandidates (label equality, l.29-37); then for
     k = 1..L-1 RefineCandidates (l.19-28) keeps v_d in C(v_q) iff it was in
@@ -115,7 +120,7 @@ def candidates_bool(Q, D, levels: int, data_graphs=None, q_rows=None):
     False); ``q_rows`` restricts the query rows (others False)."""
     VQ, VD = Q.num_nodes, D.num_nodes
     rows = range(VQ) if q_rows is None else q_rows
-    SQ = raw_signatures(Q, max(levels - 1, 0))
+    SQ = raw_signatures(Q, max(levels - 1, 0), skip_wildcards=wildcard)
     SD = raw_signatures(D, max(levels - 1, 0), data_graphs)
     if data_graphs is None:
         cols = np.ones(VD, bool)
@@ -125,7 +130,10 @@ def candidates_bool(Q, D, levels: int, data_graphs=None, q_rows=None):
             cols[int(D.graph_offsets[g]):int(D.graph_offsets[g + 1])] = True
     C = np.zeros((VQ, VD), bool)
     for vq in rows:
-        C[vq] = (D.node_labels == Q.node_labels[vq]) & cols          # InitializeCandidates
+        if wildcard and Q.node_labels[vq] == 0:                       # '*': every atom (R22)
+            C[vq] = cols.copy()
+        else:
+            C[vq] = (D.node_labels == Q.node_labels[vq]) & cols      # InitializeCandidates
     for k in range(1, levels):                                        # k = 1 .. s-1
         sq, sd = saturate(SQ[k]), saturate(SD[k])
         for vq in rows:
@@ -133,7 +141,7 @@ def candidates_bool(Q, D, levels: int, data_graphs=None, q_rows=None):
     return C
 
 
-def neighbour_support(Q, D, C):
+def neighbour_support(Q, D, C, wildcard: bool = False):
     """Greatest fixed point of the neighbour-support rule (north_star; R9):
     remove v_d from C(v_q) if some query edge (v_q, u_q, b) has no data edge
     (v_d, u_d, b) with u_d in C(u_q).  Naive iteration until nothing changes."""
@@ -149,7 +157,7 @@ def neighbour_support(Q, D, C):
         changed = False
         for e in range(qsrc.shape[0]):
             vq, uq, b = int(qsrc[e]), int(qdst[e]), int(qlab[e])
-            m = (dlab == b) & C[uq, ddst]
+            m = ((dlab == b) | (wildcard and b == 0)) & C[uq, ddst]  # '~' bond: any label (R22)
             support = np.zeros(D.num_nodes, bool)
             support[dsrc[m]] = True
             new = C[vq] & support
@@ -169,10 +177,10 @@ def to_bitmap(C):
     return np.ascontiguousarray(by).view(np.uint32).reshape(VQ, W) if VQ else np.zeros((0, W), np.uint32)
 
 
-def candidates(Q, D, levels: int, neighbour: bool = False):
-    C = candidates_bool(Q, D, levels)
+def candidates(Q, D, levels: int, neighbour: bool = False, wildcard: bool = False):
+    C = candidates_bool(Q, D, levels, wildcard=wildcard)
     if neighbour:
-        C = neighbour_support(Q, D, C)
+        C = neighbour_support(Q, D, C, wildcard=wildcard)
     return to_bitmap(C)
 
 

@@ -221,3 +221,30 @@ def test_neighbour_support_bond_labels_hand_computed():
     # q0 needs a double-bond neighbour in C(q1) = {0, 2}: only node 1 has one (node 0);
     # q1 then needs a double-bond neighbour in C(q0) = {1}: only node 0 has one
     assert np.array_equal(F, np.array([[False, True, False], [True, False, False]]))
+
+
+def test_wildcard_filter_soundness():
+    """Wildcard mode (R22): a '*' query atom's candidates start from every
+    atom and it adds to no signature field; the filter (with and without the
+    neighbour-support fixed point, '~' bonds matching any label) keeps every
+    embedding image of the oracle's wildcard mode at every level."""
+    from synth import GraphBatch
+    rng = np.random.default_rng(91)
+    D = synth.molecules(synth.DATA_SEED_BASE + 5, 0, 25)
+    qs = []
+    for lab, edges in synth.library(synth.C1_NAMES) + synth.random_subgraph_queries(synth.QUERY_SEED_BASE + 5, 8):
+        lab = [0 if rng.random() < 0.35 else x for x in lab]
+        edges = [(u, v, 0 if rng.random() < 0.35 else b) for (u, v, b) in edges]
+        qs.append((lab, edges))
+    Q = GraphBatch.from_graphs(qs)
+    imgs = set()
+    for q in range(Q.num_graphs):
+        for g in range(D.num_graphs):
+            for f in oracle.enumerate_pair(Q, D, q, g, oracle.WILDCARD).tolist():
+                imgs.update((int(Q.graph_offsets[q]) + i, int(D.graph_offsets[g]) + v) for i, v in enumerate(f))
+    assert len(imgs) > 50
+    for L in (1, 2, 4):
+        Cb = fr.candidates_bool(Q, D, L, wildcard=True)
+        F = fr.neighbour_support(Q, D, Cb, wildcard=True)
+        for (vq, vd) in imgs:
+            assert Cb[vq, vd] and F[vq, vd], (L, vq, vd)
