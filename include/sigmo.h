@@ -248,6 +248,18 @@ SIGMO_API sigmo_status sigmo_check_join(sigmo_ctx *ctx);
  * subset of the monomorphisms, so its candidate sets stay sound).  Never
  * fails for a valid ctx. */
 SIGMO_API sigmo_status sigmo_set_induced(sigmo_ctx *ctx, int enable);
+/* Wildcard atoms and bonds (the paper's stated next step,
+ * P:2639-2645; R22): with enable = 1, a QUERY atom label 0 is the
+ * SMARTS '*' (matches an atom of any label) and a query bond label 0 the
+ * SMARTS '~' (matches a bond of any label); data labels stay literal.  Takes
+ * effect at the next sigmo_load_batch.  The filter stays sound: a '*' atom's
+ * candidates start from every atom and it adds to no signature field of the
+ * other query atoms; '~' bonds use the all-bond adjacency in the join and in
+ * the neighbour-support pass.  With '~' bonds at most 7 distinct concrete
+ * query bond labels (SIGMO_ERR_LIMIT).  The query side of
+ * sigmo_get_signatures leaves '*' atoms out of every field.  Never fails for a
+ * valid ctx. */
+SIGMO_API sigmo_status sigmo_set_wildcards(sigmo_ctx *ctx, int enable);
 /* Enable/disable per-stage CUDA-event timing (default off) and read it. */
 SIGMO_API sigmo_status sigmo_set_timing(sigmo_ctx *ctx, int enable);
 SIGMO_API sigmo_status sigmo_get_timings(sigmo_ctx *ctx, sigmo_timings *out);

@@ -297,6 +297,11 @@ class Context:
         """Induced-subgraph mode for the next load_batch (include/sigmo.h sigmo_set_induced)."""
         self._check(self._lib.sigmo_set_induced(self._handle, 1 if enable else 0), "sigmo_set_induced")
 
+    def set_wildcards(self, enable: bool = True):
+        """Wildcard atoms / bonds for the next load_batch: query label 0 = '*', bond 0 = '~'
+        (include/sigmo.h sigmo_set_wildcards)."""
+        self._check(self._lib.sigmo_set_wildcards(self._handle, 1 if enable else 0), "sigmo_set_wildcards")
+
     def set_timing(self, enable: bool = True):
         self._check(self._lib.sigmo_set_timing(self._handle, 1 if enable else 0), "sigmo_set_timing")
 

@@ -21,7 +21,7 @@ SIGMO_FILTER_NEIGHBOR_SUPPORT = 1
 EXPORTS = ["sigmo_create", "sigmo_load_batch", "sigmo_filter", "sigmo_join", "sigmo_num_pairs",
            "sigmo_get_pair_results", "sigmo_get_dense_results", "sigmo_get_query_totals", "sigmo_get_candidates",
            "sigmo_get_signatures", "sigmo_get_packed_batch", "sigmo_check_join", "sigmo_enumerate",
-           "sigmo_get_embeddings", "sigmo_get_node_sets", "sigmo_set_induced", "sigmo_set_timing",
+           "sigmo_get_embeddings", "sigmo_get_node_sets", "sigmo_set_wildcards", "sigmo_set_induced", "sigmo_set_timing",
            "sigmo_get_timings", "sigmo_validate_batch",
            "sigmo_last_error", "sigmo_version", "sigmo_destroy"]
 
@@ -91,6 +91,7 @@ def load_library(path: str | None = None) -> ctypes.CDLL:
     lib.sigmo_get_node_sets.argtypes = [vp, ctypes.c_int64, i64p, i64p, ctypes.c_int64, P(ctypes.c_uint64), i64p]
     lib.sigmo_set_timing.argtypes = [vp, ctypes.c_int]
     lib.sigmo_set_induced.argtypes = [vp, ctypes.c_int]
+    lib.sigmo_set_wildcards.argtypes = [vp, ctypes.c_int]
     lib.sigmo_get_timings.argtypes = [vp, P(sigmo_timings)]
     lib.sigmo_validate_batch.argtypes = [P(sigmo_graph_batch), ctypes.c_int, ctypes.c_char_p, ctypes.c_size_t]
     lib.sigmo_last_error.argtypes = [vp]

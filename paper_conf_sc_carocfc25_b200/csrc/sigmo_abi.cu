@@ -142,6 +142,9 @@ struct sigmo_ctx {
   // jcnt u64 slots: [0] pair cursor / chunk counter, [1] error flag, [2..5] DFS stats, [6..] totals
   int induced = 0;         // sigmo_set_induced (applies to the next sigmo_load_batch)
   int induced_loaded = 0;  // induced mode of the loaded batch (routes it to k_join)
+  int wildcard = 0;        // sigmo_set_wildcards (applies to the next sigmo_load_batch)
+  int wildcard_loaded = 0; // wildcard mode of the loaded batch (R22)
+  int any_bond = 0;        // the loaded queries use '~' bonds: label 0 -> adjacency class NB (all bonds)
   bool lane_join = false;  // per-lane join possible for this batch (<= 64-node graphs, <= 16-node queries)
   bool mol_filter = false; // last sigmo_filter used molecule tiles (candidates in cmol layout)
   bool dense_pad_zero = false;  // padding words >= W of the dense bitmap rows (and the tail) are zero
@@ -938,9 +941,9 @@ sigmo_status ensure_prog(sigmo_ctx *c, int R, QueryProg *&out) {
   timing_mark(c, 0);
   if (R > 0) {
     SIGMO_TRY(dreserve(c, c->qcounts, (size_t)VQ * R * kNumFields, "query counts"));
-    CUDA_TRY(c, launch_sig_counts(c->dq, R, (uint8_t *)c->qcounts.p, c->stream));
+    CUDA_TRY(c, launch_sig_counts(c->dq, R, (uint8_t *)c->qcounts.p, c->wildcard_loaded, c->stream));
   }
-  CUDA_TRY(c, launch_query_prep(c->dq, R, (const uint8_t *)c->qcounts.p, P, c->stream));
+  CUDA_TRY(c, launch_query_prep(c->dq, R, (const uint8_t *)c->qcounts.p, P, c->wildcard_loaded, c->stream));
   timing_mark(c, 1);
   CUDA_TRY(c, cudaMemcpyAsync(&P.meta, P.d_meta, sizeof(QueryProgMeta), cudaMemcpyDeviceToHost, c->stream));
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
@@ -999,6 +1002,7 @@ void fill_join_caps(sigmo_ctx *c, JoinParams &jp) {
   jp.VQ = c->VQ;
   jp.NB = c->NB;
   jp.induced = c->induced_loaded;
+  jp.any_bond = c->any_bond;
   jp.qp_non = c->qp_non;
   jp.maxq = std::max(c->maxq, 2);
   jp.PCAP = c->PC;
@@ -1116,6 +1120,7 @@ sigmo_status launch_dense(sigmo_ctx *c, int R, const QueryProg &P, uint32_t *bit
       sp.NQ = c->NQ;
       sp.NQW = c->NQW;
       sp.NB = c->NB;
+      sp.any_bond = c->any_bond;
       sp.maxq = std::max(c->maxq, 1);
       sp.Wpad = c->Wpad;
       sp.goff = c->dd.goff;
@@ -1232,6 +1237,12 @@ sigmo_status sigmo_set_induced(sigmo_ctx *c, int enable) {
   return SIGMO_OK;
 }
 
+sigmo_status sigmo_set_wildcards(sigmo_ctx *c, int enable) {
+  if (!c) return SIGMO_ERR_INVALID_ARG;
+  c->wildcard = enable != 0;
+  return SIGMO_OK;
+}
+
 sigmo_status sigmo_set_timing(sigmo_ctx *c, int enable) {
   if (!c) return SIGMO_ERR_INVALID_ARG;
   c->timing.enabled = enable != 0;
@@ -1275,20 +1286,27 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const bool dev_load = data->num_nodes >= kDeviceLoadMinNodes && !(hl && atoi(hl));
   s = dev_load ? validate_light(data, msg, hd) : validate(data, 0, msg, hd);
   if (s != SIGMO_OK) return set_err(c, s, "data batch: %s", msg.c_str());
-  // bond classes = distinct query bond labels
+  // bond classes = distinct query bond labels; in wildcard mode (R22) the
+  // '~' label 0 is no class of its own: it reads class NB, the union of all
+  // bonds (the all-bonds adjacency every kernel builds)
+  c->wildcard_loaded = c->wildcard;
   uint8_t bclass[256];
   memset(bclass, 255, sizeof(bclass));
   {
     bool seen[256] = {};
     for (int64_t e = 0; e < hq.E; e++) seen[hq.elab[e]] = true;
+    c->any_bond = c->wildcard_loaded && seen[0];
+    if (c->any_bond) seen[0] = false;
     int nb = 0;
     for (int l = 0; l < 256; l++)
       if (seen[l]) {
-        if (nb >= SIGMO_MAX_BOND_CLASSES)
-          return set_err(c, SIGMO_ERR_LIMIT, "more than %d distinct query bond labels", SIGMO_MAX_BOND_CLASSES);
+        if (nb >= SIGMO_MAX_BOND_CLASSES - (c->any_bond ? 1 : 0))
+          return set_err(c, SIGMO_ERR_LIMIT, "more than %d distinct query bond labels",
+                         SIGMO_MAX_BOND_CLASSES - (c->any_bond ? 1 : 0));
         bclass[l] = (uint8_t)nb++;
       }
     c->NB = nb;
+    if (c->any_bond) bclass[0] = (uint8_t)nb;
   }
   size_t raw_bytes = 0;
   PackedOffsets pdd{};
@@ -1392,6 +1410,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
     for (const auto &p : part)
       for (int l = 0; l < 256; l++) freq[l] += p[l];
   }
+  if (c->wildcard_loaded) freq[0] = std::max<int64_t>(hd.V, 1);  // '*' matches every atom: the least selective
   QPlan plan;
   plan_queries(hq, freq, bclass, plan);
 
@@ -1417,7 +1436,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       for (int64_t g = 0; g < hd.G; g++) maxn_h = std::max<int64_t>(maxn_h, hd.goff[g + 1] - hd.goff[g]);
     for (int64_t g = 0; g < hq.G; g++) maxq_h = std::max<int64_t>(maxq_h, hq.goff[g + 1] - hq.goff[g]);
     const char *legacy = getenv("SIGMO_JOIN_LEGACY");
-    lane_ok = maxn_h <= 64 && c->NB > 0 && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
+    lane_ok = maxn_h <= 64 && (c->NB > 0 || c->any_bond) && maxq_h <= kJoinLaneMaxQ && !(legacy && atoi(legacy)) && hq.V < 65536 &&
               (unsigned long long)std::max<int64_t>(hq.V, 1) * (unsigned long long)std::max<int64_t>(hd.G, 1) <
                   (1ull << 32) &&
               (unsigned long long)(c->NB + 2) * hd.V + 1 < (1ull << 31) &&
@@ -2442,7 +2461,8 @@ sigmo_status sigmo_get_signatures(sigmo_ctx *c, int which, int radius, uint64_t 
   const DevGraphs &g = which == 0 ? c->dq : c->dd;
   if (g.num_nodes == 0) return SIGMO_OK;
   SIGMO_TRY(dreserve(c, c->sig_tmp, 8 * (size_t)g.num_nodes, "signature export"));
-  CUDA_TRY(c, launch_sig_pack(g, radius, (unsigned long long *)c->sig_tmp.p, c->stream));
+  CUDA_TRY(c, launch_sig_pack(g, radius, (unsigned long long *)c->sig_tmp.p, which == 0 ? c->wildcard_loaded : 0,
+                              c->stream));
   CUDA_TRY(c, cudaMemcpyAsync(out, c->sig_tmp.p, 8 * (size_t)g.num_nodes, cudaMemcpyDeviceToHost, c->stream));
   CUDA_TRY(c, cudaStreamSynchronize(c->stream));
   return SIGMO_OK;

@@ -191,6 +191,7 @@ struct JoinParams {
   int induced;                 // 1 = induced-subgraph embeddings (k_join only, R21):
                                // the union of all bonds is staged as adjacency class NB
   const uint32_t *qp_non;      // [VQ] induced mode: mask of the earlier plan depths NOT adjacent to depth e
+  int any_bond;                // wildcard query bonds ('~', label 0; R22) map to adjacency class NB (all bonds)
   // enumerate mode (k_join_lane); emaps == nullptr: counting
   unsigned char *emaps;        // [embeddings][estride] molecule-local data node per query node (query node order)
   int estride;                 // 8 (queries <= 8 nodes) or 16 bytes per embedding
@@ -237,6 +238,7 @@ struct SupportLaneParams {
 
 struct SupportParams {
   int ND, NQ, NQW, NB, maxq, Wpad;
+  int any_bond;                  // wildcard query bonds map to class NB (all bonds)
   const int32_t *goff, *roff;
   const uint16_t *nbr;
   const uint8_t *bclass;
@@ -278,9 +280,9 @@ cudaError_t launch_layout(const int32_t *goff, int G, int NB, void *scratch, uin
                           int32_t *grpn, int32_t *grpw, uint4 *mrec, long long *info_out, cudaStream_t st);
 
 // ---- launchers (sigmo_kernels.cu); all enqueue on `st` ----
-cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, cudaStream_t st);
-cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *out, cudaStream_t st);
-cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts, QueryProg &prog,
+cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, int skip0, cudaStream_t st);
+cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *out, int skip0, cudaStream_t st);
+cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts, QueryProg &prog, int wild,
                               cudaStream_t st);
 cudaError_t launch_filter(int NW, const FilterParams &p, int num_tiles, cudaStream_t st);
 size_t filter_smem_bytes(int NW, int EXTN, int EXTW, int MOLCAP, int NFU, int NLAB, int P, int NREC, int VQ,

@@ -222,8 +222,10 @@ __device__ int block_exclusive_scan(T *data, int n, int *s_warp) {
 // r = 1..R, saturated per field (R8), optionally packed at one radius.
 // One CTA per graph (<= 256 nodes, NW = 4); not on the data hot path.
 // ===========================================================================
+// skip0: wildcard query batches (R22) -- a label-0 atom ('*') adds
+// to no field of the other atoms' counts
 __global__ void __launch_bounds__(128) k_sig_counts(DevGraphs g, int R, uint8_t *counts,
-                                                    unsigned long long *packed, int pack_radius) {
+                                                    unsigned long long *packed, int pack_radius, int skip0) {
   using M = Mask<4>;
   __shared__ M s_ballA[256], s_ballB[256], s_adj[256], s_fm[kNumFields];
   __shared__ uint8_t s_fid[256];
@@ -241,7 +243,7 @@ __global__ void __launch_bounds__(128) k_sig_counts(DevGraphs g, int R, uint8_t 
   for (int f = threadIdx.x; f < kNumFields; f += blockDim.x) s_fm[f].clear();
   __syncthreads();
   for (int i = threadIdx.x; i < n; i += blockDim.x)
-    atomicOr(&s_fm[s_fid[i]].w[i >> 6], 1ull << (i & 63));
+    if (!(skip0 && g.label[base + i] == 0)) atomicOr(&s_fm[s_fid[i]].w[i >> 6], 1ull << (i & 63));
   __syncthreads();
   M *cur = s_ballA, *nxt = s_ballB;
   for (int r = 1; r <= R; r++) {
@@ -258,7 +260,8 @@ __global__ void __launch_bounds__(128) k_sig_counts(DevGraphs g, int R, uint8_t 
     for (int i = threadIdx.x; i < n; i += blockDim.x) {
       unsigned long long pk = 0;
       for (int f = 0; f < kNumFields; f++) {
-        int c = (cur[i] & s_fm[f]).popc() - (s_fid[i] == f ? 1 : 0);
+        // the node itself is not counted (u != v); a skipped wildcard is in no field mask
+        int c = (cur[i] & s_fm[f]).popc() - ((s_fid[i] == f && !(skip0 && g.label[base + i] == 0)) ? 1 : 0);
         int mx = (1 << c_field_width[f]) - 1;
         if (c > mx) c = mx;  // R8: saturate, never wrap
         if (counts) counts[((size_t)(base + i) * R + (r - 1)) * kNumFields + f] = (uint8_t)c;
@@ -270,15 +273,15 @@ __global__ void __launch_bounds__(128) k_sig_counts(DevGraphs g, int R, uint8_t 
   }
 }
 
-cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, cudaStream_t st) {
+cudaError_t launch_sig_counts(const DevGraphs &g, int R, uint8_t *counts, int skip0, cudaStream_t st) {
   if (g.num_graphs == 0 || R <= 0) return cudaSuccess;
-  k_sig_counts<<<g.num_graphs, 128, 0, st>>>(g, R, counts, nullptr, 0);
+  k_sig_counts<<<g.num_graphs, 128, 0, st>>>(g, R, counts, nullptr, 0, skip0);
   return cudaGetLastError();
 }
 
-cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *out, cudaStream_t st) {
+cudaError_t launch_sig_pack(const DevGraphs &g, int radius, unsigned long long *out, int skip0, cudaStream_t st) {
   if (g.num_graphs == 0) return cudaSuccess;
-  k_sig_counts<<<g.num_graphs, 128, 0, st>>>(g, radius, nullptr, out, radius);
+  k_sig_counts<<<g.num_graphs, 128, 0, st>>>(g, radius, nullptr, out, radius, skip0);
   return cudaGetLastError();
 }
 
@@ -298,7 +301,7 @@ constexpr int kKeyWords = (kMaxRadius * kNumFields * 256) / 32;  // 1560
 constexpr int kRF = kMaxRadius * kNumFields;                     // 195
 
 __global__ void __launch_bounds__(kQueryPrepThreads) k_query_prep(int VQ, int R, const uint8_t *qlabel,
-                                                                   const uint8_t *qc, QueryProg prog) {
+                                                                   const uint8_t *qc, QueryProg prog, int wild) {
   constexpr int NT = kQueryPrepThreads;
   __shared__ uint32_t s_key[kKeyWords];
   __shared__ int s_rank[kKeyWords];
@@ -323,7 +326,10 @@ __global__ void __launch_bounds__(kQueryPrepThreads) k_query_prep(int VQ, int R,
       atomicOr(&s_key[key >> 5], 1u << (key & 31));
     }
   }
-  for (int v = tid; v < VQ; v += NT) atomicOr(&s_lab[qlabel[v] >> 5], 1u << (qlabel[v] & 31));
+  // label planes of the query labels; a wildcard atom ('*', label 0; R22) has
+  // none -- its row starts from the all-ones channel NLAB
+  for (int v = tid; v < VQ; v += NT)
+    if (!(wild && qlabel[v] == 0)) atomicOr(&s_lab[qlabel[v] >> 5], 1u << (qlabel[v] & 31));
   __syncthreads();
   for (int i = tid; i < kKeyWords; i += NT) s_rank[i] = __popc(s_key[i]);
   __syncthreads();
@@ -395,7 +401,8 @@ __global__ void __launch_bounds__(kQueryPrepThreads) k_query_prep(int VQ, int R,
       }
     prog.row_off[v] = c;
     int l = qlabel[v];
-    prog.row_lab[v] = (uint8_t)(s_labrank[l >> 5] + __popc(s_lab[l >> 5] & ((1u << (l & 31)) - 1u)));
+    prog.row_lab[v] = (wild && l == 0) ? (uint8_t)prog.d_meta->NLAB
+                                       : (uint8_t)(s_labrank[l >> 5] + __popc(s_lab[l >> 5] & ((1u << (l & 31)) - 1u)));
   }
   __syncthreads();
   const int RE = block_exclusive_scan<NT>(prog.row_off, VQ, s_warp);
@@ -418,9 +425,9 @@ __global__ void __launch_bounds__(kQueryPrepThreads) k_query_prep(int VQ, int R,
   }
 }
 
-cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts, QueryProg &prog,
+cudaError_t launch_query_prep(const DevGraphs &q, int R, const uint8_t *qcounts, QueryProg &prog, int wild,
                               cudaStream_t st) {
-  k_query_prep<<<1, kQueryPrepThreads, 0, st>>>(q.num_nodes, R, q.label, qcounts, prog);
+  k_query_prep<<<1, kQueryPrepThreads, 0, st>>>(q.num_nodes, R, q.label, qcounts, prog, wild);
   return cudaGetLastError();
 }
 
@@ -1134,7 +1141,7 @@ __global__ void __launch_bounds__(SupportCfg<NW>::kThreads) k_support(SupportPar
   const int NB = sp.NB;
   const int ACAP = kSupportMols * 64 * NW;
   M *s_adj = (M *)smem;                                              // [NB][ACAP]
-  M *s_cm = s_adj + (size_t)NB * ACAP;                               // [threads][maxq]
+  M *s_cm = s_adj + (size_t)(NB + sp.any_bond) * ACAP;              // [threads][maxq]
   uint32_t *s_gm = (uint32_t *)(s_cm + (size_t)kSupportThreads * sp.maxq);  // [mols][NQW]
   __shared__ int s_mstart[kSupportMols + 1];
   const int tid = threadIdx.x;
@@ -1149,19 +1156,22 @@ __global__ void __launch_bounds__(SupportCfg<NW>::kThreads) k_support(SupportPar
   for (int i = tid; i < na; i += kSupportThreads) {
     const int v = a0 + i;
     const int e0 = __ldg(&sp.roff[v]), e1 = __ldg(&sp.roff[v + 1]);
-    M m[8];
+    M m[8], mall;
 #pragma unroll
     for (int b = 0; b < 8; b++) m[b].clear();
+    mall.clear();
     for (int e = e0; e < e1; e++) {
       const int x = __ldg(&sp.nbr[e]);
       const int cls = sp.bclass[x & 255];
 #pragma unroll
       for (int b = 0; b < 8; b++)
         if (cls == b) m[b].set(x >> 8);
+      mall.set(x >> 8);
     }
 #pragma unroll
     for (int b = 0; b < 8; b++)
       if (b < NB) s_adj[b * ACAP + i] = m[b];
+    if (sp.any_bond) s_adj[NB * ACAP + i] = mall;  // '~' query bonds (R22): class NB = every bond
   }
   __syncthreads();
   M *cm = s_cm + (size_t)tid * sp.maxq;
@@ -1251,7 +1261,7 @@ __global__ void __launch_bounds__(SupportCfg<NW>::kThreads) k_support(SupportPar
 template <int NW>
 static size_t support_smem_t(int NB, int maxq, int NQW) {
   constexpr int mols = SupportCfg<NW>::kMols, thr = SupportCfg<NW>::kThreads;
-  return (size_t)8 * NW * ((size_t)NB * mols * 64 * NW + (size_t)thr * maxq) + 4 * (size_t)mols * NQW;
+  return (size_t)8 * NW * ((size_t)(NB + 1) * mols * 64 * NW + (size_t)thr * maxq) + 4 * (size_t)mols * NQW;
 }
 
 size_t support_smem_bytes(int NW, int NB, int maxq, int NQW) {
@@ -1430,7 +1440,7 @@ __host__ __device__ inline JoinSmem join_layout(const JoinParams &p, int NW, int
   L.tot = o;   o = align16(o + 8 * (size_t)p.NQ);
   L.warps = o;
   size_t w = 0;
-  L.w.adj = w;     w = align16(w + mb * (size_t)(p.NB + (p.induced ? 1 : 0)) * p.ACAP);
+  L.w.adj = w;     w = align16(w + mb * (size_t)(p.NB + ((p.induced || p.any_bond) ? 1 : 0)) * p.ACAP);
   L.w.cm = w;      w = align16(w + mb * (size_t)p.CMCAP);
   L.w.cinfo = w;   w = align16(w + 4 * (size_t)p.CMCAP);
   L.w.pinfo = w;   w = align16(w + 16 * (size_t)p.PCAP);
@@ -1566,7 +1576,7 @@ __global__ void __launch_bounds__(kJoinThreads) k_join(JoinParams jp) {
 #pragma unroll
       for (int b = 0; b < 8; b++)
         if (b < jp.NB) s_adj[b * ACAP + i] = m[b];
-      if (jp.induced) s_adj[jp.NB * ACAP + i] = mall;  // every bond, whatever its label
+      if (jp.induced || jp.any_bond) s_adj[jp.NB * ACAP + i] = mall;  // every bond, whatever its label
     }
     __syncwarp();
     // The chunk's pairs are processed in passes that fit the warp's pair /
