@@ -333,6 +333,19 @@ __device__ __forceinline__ void lane_filter_group(const FilterLaneParams &fp, in
       nb[k] = __ldg(fp.nb4 + mr[m].x + v);
     }
   }
+  // channel NLAB: the slot's existing atoms (row padding, and the start of a
+  // wildcard '*' row, R22)
+  {
+    unsigned vm[4];
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const int m = WIDE ? k >> 1 : k;
+      const int lo = WIDE ? 32 * (k & 1) : 0;
+      const int nk = (int)mr[m].y - lo;
+      vm[k] = nk >= 32 ? LF_FULL : (nk <= 0 ? 0u : (1u << nk) - 1u);
+    }
+    lf_sts128_lane0(wpl_s + 16u * (unsigned)LF_C(NLAB), make_uint4(vm[0], vm[1], vm[2], vm[3]), lane);
+  }
   // label planes (channels 0..NLAB-1) and field masks [NFU][4 slots]
   if (LF_C(NLAB) + LF_C(NFU) <= 32) {
     // per slot, lane = node builds its one-hot word (bit c: label channel c,
@@ -538,8 +551,6 @@ __device__ __forceinline__ void lf_kernel_body(const FilterLaneParams &fp) {
     for (int i = tid; i <= 4 * fp.R; i += kFilterLaneThreads) rr[i] = __ldg(&fp.rrec[i]);
   }
   unsigned char *wsm = smem + L.warps + (size_t)wid * L.w_total;
-  // the all-ones channel NLAB (row padding and label-less rows never read it otherwise)
-  if (lane == 0) *(uint4 *)(wsm + L.w_planes + 16 * fp.NLAB) = make_uint4(LF_FULL, LF_FULL, LF_FULL, LF_FULL);
   __syncthreads();
   const uint4 *rowp = GL ? fp.rowp : (const uint4 *)(smem + L.rowp);
   const uint2 *qwl = GL ? fp.qwl : (const uint2 *)(smem + L.qwl);

@@ -734,15 +734,17 @@ __global__ void __launch_bounds__(kFilterThreads, MOL ? 5 : 4) k_filter(const __
         if (fs >= 0) mb |= 1u << (NLAB + 1 + fs);
       }
       const uint32_t T = transpose32(mb, lane);
+      const uint32_t vw = __ballot_sync(FULL_MASK, valid);  // channel NLAB: existing nodes (wildcard rows, R22)
       if (lane < NLAB) plw[lane] = T;
-      else if (lane == NLAB) plw[NLAB] = 0xffffffffu;
+      else if (lane == NLAB) plw[NLAB] = vw;
       else if (lane < NLAB + 1 + NFU) s_fpl[(lane - NLAB - 1) * EXTW + k] = T;
     } else {
       for (int c = 0; c < NLAB; c++) {
         const unsigned b = __ballot_sync(FULL_MASK, lab == (int)s_labval[c]);
         if (lane == 0) plw[c] = b;
       }
-      if (lane == 0) plw[NLAB] = 0xffffffffu;
+      const uint32_t vw = __ballot_sync(FULL_MASK, valid);
+      if (lane == 0) plw[NLAB] = vw;
       for (int fs = 0; fs < NFU; fs++) {
         const unsigned b = __ballot_sync(FULL_MASK, fid == (int)s_fused[fs]);
         if (lane == 0) s_fpl[fs * EXTW + k] = b;
