@@ -2267,7 +2267,8 @@ __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
 
 // W64: the launch's pairs are on > 32-node molecules (64-bit masks); else all
 // masks, stack entries and loads are 32-bit
-template <int MODE, bool W64>
+// PS: the plan entries are copied to shared memory (VQ <= kJoinLanePlanSmemMax)
+template <int MODE, bool W64, bool PS>
 __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_constant__ JoinParams jp) {
   using MT = typename std::conditional<W64, unsigned long long, unsigned>::type;
   constexpr unsigned ES = W64 ? 16u : 8u;  // stack entry bytes
@@ -2289,28 +2290,32 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   // registers, 8.92 vs 8.80 ms)
   // plan entries (8 B): a shared-memory copy when they fit, else through the read-only cache
   const unsigned o_plan = (unsigned)align16(8 * (size_t)(jp.NQ > 0 ? jp.NQ : 1));
-  const bool plan_s = join_lane_plan_bytes(jp.VQ) > 0;
-  if (plan_s)
+  if (PS)
     for (int i = threadIdx.x; i < jp.VQ; i += blockDim.x) ((uint2 *)(smem + o_plan))[i] = __ldg(&jp.qp_ent2[i]);
-  auto plan = [&](unsigned i) -> uint2 { return plan_s ? ((const uint2 *)(smem + o_plan))[i] : __ldg(&jp.qp_ent2[i]); };
+#define JL_PLAN(i) (PS ? ((const uint2 *)(smem + o_plan))[(i)] : __ldg(&jp.qp_ent2[(i)]))
   const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ, jp.VQ) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
   const unsigned oRU = wbase + ES * lane;                         // {R, U} of depth d: oRU + 32 ES d
   const unsigned oM = wbase + 32u * ES * SD + lane;               // f(pi_d): oM + 32 d
-  auto ldRU = [&](unsigned o, MT &r, MT &u) {
-    if (W64) {
-      const ulonglong2 x = *(const ulonglong2 *)(smem + o);
-      r = (MT)x.x;
-      u = (MT)x.y;
-    } else {
-      const uint2 x = *(const uint2 *)(smem + o);
-      r = (MT)x.x;
-      u = (MT)x.y;
-    }
-  };
-  auto stRU = [&](unsigned o, MT r, MT u) {
-    if (W64) *(ulonglong2 *)(smem + o) = make_ulonglong2((unsigned long long)r, (unsigned long long)u);
-    else *(uint2 *)(smem + o) = make_uint2((unsigned)r, (unsigned)u);
-  };
+  // stack entry {R, U} at byte offset o of the kernel's shared memory (macros,
+  // not lambdas: a captured `smem` loses its address space and every access
+  // would re-derive the shared window)
+#define JL_LDRU(o, r, u)                                           \
+  do {                                                             \
+    if (W64) {                                                     \
+      const ulonglong2 x_ = *(const ulonglong2 *)(smem + (o));     \
+      r = (MT)x_.x;                                                \
+      u = (MT)x_.y;                                                \
+    } else {                                                       \
+      const uint2 x_ = *(const uint2 *)(smem + (o));               \
+      r = (MT)x_.x;                                                \
+      u = (MT)x_.y;                                                \
+    }                                                              \
+  } while (0)
+#define JL_STRU(o, r, u)                                                                                           \
+  do {                                                                                                             \
+    if (W64) *(ulonglong2 *)(smem + (o)) = make_ulonglong2((unsigned long long)(r), (unsigned long long)(u));      \
+    else *(uint2 *)(smem + (o)) = make_uint2((unsigned)(r), (unsigned)(u));                                        \
+  } while (0)
   auto popc = [](MT x) -> int { return W64 ? __popcll((unsigned long long)x) : __popc((unsigned)x); };
   auto lowest = [](MT x) -> int {  // index of the lowest set bit (x != 0)
     if (W64) {
@@ -2411,9 +2416,9 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const unsigned od = oRU + 32u * ES * d;
       // the plan entry of depth e and the map bytes of its back-edge targets
       // depend on d only: loaded before v is known (j == d takes v below)
-      const uint2 en = plan(cqb + e);
+      const uint2 en = JL_PLAN(cqb + e);
       MT R, U;
-      ldRU(od, R, U);
+      JL_LDRU(od, R, U);
       const unsigned j0 = en.x & 15, j1 = (en.x >> 4) & 15;
       const unsigned m0 = smem[oM + 32u * j0], m1 = smem[oM + 32u * j1];
       const int v = lowest(R);
@@ -2453,7 +2458,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         if ((MODE & 4) && X) emit(X, d, used);  // enumerate mode: write the embeddings
         if ((MODE & 1) && cnt) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
-        stRU(oRU + 32u * ES * e, X, used);
+        JL_STRU(oRU + 32u * ES * e, X, used);
         ne |= 1u << e;
       }
       pend = ne == 0u;
@@ -2494,7 +2499,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         if ((MODE & 4) && R0) emit(R0, -1, (MT)0);
         pend = true;
       } else {
-        stRU(oRU, R0, (MT)0);
+        JL_STRU(oRU, R0, (MT)0);
         ne = R0 ? 1u : 0u;
         pend = ne == 0u;
       }
@@ -2519,7 +2524,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         np = cbase + (unsigned)src;
         nv = true;
         // root candidates of the next pair: the load completes while the current pair runs
-        nR0 = cand((unsigned)r.z, plan((unsigned)r.w >> 16).x >> 12);
+        nR0 = cand((unsigned)r.z, JL_PLAN((unsigned)r.w >> 16).x >> 12);
       }
       chead += take;
       wm = __ballot_sync(FULL_MASK, !nv) & wm;
@@ -2564,8 +2569,8 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
           const unsigned dl = (unsigned)(src - lane);  // donor offsets = mine + dl * (8 | 16 | 1)
           {
             MT r, u;
-            ldRU(oRU + 32u * ES * ds + ES * dl, r, u);
-            stRU(oRU + 32u * ES * ds, r, u);
+            JL_LDRU(oRU + 32u * ES * ds + ES * dl, r, u);
+            JL_STRU(oRU + 32u * ES * ds, r, u);
           }
           for (int j = 0; j < ds; j++) smem[oM + 32u * j] = smem[oM + 32u * j + dl];
           cmb = s_cmb;
@@ -2600,14 +2605,25 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
 #undef STS64
 #undef LDS128
 #undef STS128
+#undef JL_LDRU
+#undef JL_STRU
+#undef JL_PLAN
 }
 
 template <int MODE, bool W64>
 static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_t st) {
-  cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE, W64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       (int)p.smem_bytes);
-  if (e != cudaSuccess) return e;
-  k_join_lane<MODE, W64><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
+  // plan entries in shared memory when they fit (join_lane_plan_bytes)
+  if (join_lane_plan_bytes(p.VQ) > 0) {
+    cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE, W64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)p.smem_bytes);
+    if (e != cudaSuccess) return e;
+    k_join_lane<MODE, W64, true><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
+  } else {
+    cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE, W64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)p.smem_bytes);
+    if (e != cudaSuccess) return e;
+    k_join_lane<MODE, W64, false><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
+  }
   return cudaGetLastError();
 }
 
@@ -2636,11 +2652,17 @@ cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, 
 }
 
 template <int MODE, bool W64>
-static int join_lane_occ_t(size_t smem) {
+static int join_lane_occ_t(size_t smem, bool ps) {
   int n = 0;
-  cudaFuncSetAttribute(k_join_lane<MODE, W64>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE, W64>, kJoinLaneThreads, smem) !=
-      cudaSuccess) {
+  cudaError_t e;
+  if (ps) {
+    cudaFuncSetAttribute(k_join_lane<MODE, W64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE, W64, true>, kJoinLaneThreads, smem);
+  } else {
+    cudaFuncSetAttribute(k_join_lane<MODE, W64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE, W64, false>, kJoinLaneThreads, smem);
+  }
+  if (e != cudaSuccess) {
     cudaGetLastError();
     return 1;
   }
@@ -2650,23 +2672,24 @@ static int join_lane_occ_t(size_t smem) {
 int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem) {
   // the instantiation launch_join_lane picks: bit 0 Find First, bit 1 induced, enumerate
   const int m = (mode & 1) | (p.induced ? 2 : 0);
+  const bool ps = join_lane_plan_bytes(p.VQ) > 0;
   if (p.emaps) {
-    if (w64) return p.induced ? join_lane_occ_t<6, true>(smem) : join_lane_occ_t<4, true>(smem);
-    return p.induced ? join_lane_occ_t<6, false>(smem) : join_lane_occ_t<4, false>(smem);
+    if (w64) return p.induced ? join_lane_occ_t<6, true>(smem, ps) : join_lane_occ_t<4, true>(smem, ps);
+    return p.induced ? join_lane_occ_t<6, false>(smem, ps) : join_lane_occ_t<4, false>(smem, ps);
   }
   if (w64) {
     switch (m) {
-      case 0: return join_lane_occ_t<0, true>(smem);
-      case 1: return join_lane_occ_t<1, true>(smem);
-      case 2: return join_lane_occ_t<2, true>(smem);
-      default: return join_lane_occ_t<3, true>(smem);
+      case 0: return join_lane_occ_t<0, true>(smem, ps);
+      case 1: return join_lane_occ_t<1, true>(smem, ps);
+      case 2: return join_lane_occ_t<2, true>(smem, ps);
+      default: return join_lane_occ_t<3, true>(smem, ps);
     }
   }
   switch (m) {
-    case 0: return join_lane_occ_t<0, false>(smem);
-    case 1: return join_lane_occ_t<1, false>(smem);
-    case 2: return join_lane_occ_t<2, false>(smem);
-    default: return join_lane_occ_t<3, false>(smem);
+    case 0: return join_lane_occ_t<0, false>(smem, ps);
+    case 1: return join_lane_occ_t<1, false>(smem, ps);
+    case 2: return join_lane_occ_t<2, false>(smem, ps);
+    default: return join_lane_occ_t<3, false>(smem, ps);
   }
 }
 

@@ -115,3 +115,13 @@ def test_validate_limits(lib):
     assert _ok(lib, big_d)[0] == LIMIT
     ok_d = GraphBatch.from_graphs([([6] * 256, [(i, i + 1, 1) for i in range(255)])])
     assert _ok(lib, ok_d)[0] == 0
+
+
+def test_library_has_no_unresolved_internal_symbols():
+    """Every internal (namespace sigmo) function the library calls is defined
+    in it: a missing launcher would only surface at dlopen on the GPU box."""
+    import subprocess
+    from paper_conf_sc_carocfc25_b200 import build as B
+    out = subprocess.run(["nm", "-D", "--undefined-only", B.LIB], capture_output=True, text=True).stdout
+    missing = [l.split()[-1] for l in out.splitlines() if "_ZN5sigmo" in l]
+    assert missing == [], missing
