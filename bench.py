@@ -53,6 +53,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="sigmo", choices=["sigmo", "reference"])
     ap.add_argument("--levels", type=int, default=LEVELS)
+    ap.add_argument("--levels-large", type=int, default=4,
+                    help="configs[3]/[4]: levels of the 20-30-atom ring-system query group (general join)")
     ap.add_argument("--config", type=int, default=2, choices=sorted(CONFIGS), help="BASELINE.json configs[i]")
     ap.add_argument("--molecules", type=int, default=None, help="molecules per rank (default: the config's)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -262,6 +264,9 @@ def config_dict(args, world, oracle_step=None):
                 else "no flush: per-step inputs and candidate arrays are larger than the 126 MB L2"),
          "parallelism": f"dp{world}: molecule shards, queries replicated, NCCL all-reduce of per-query totals",
          "shards": getattr(args, "balance", "atoms") if world > 1 else "whole batch"}
+    if args.cid in (4, 5):
+        d["levels_ring_systems"] = args.levels_large
+        d["workload"] += f" (ring-system query group: levels={args.levels_large})"
     if getattr(args, "induced", False):
         d["workload"] += ", induced-subgraph mode (N4)"
         d["induced"] = True
@@ -518,7 +523,7 @@ def run_routed(args, world, rank, local):
                    for i in range(nb)]
     else:
         batches = [sigmo.as_c_batch(synth.config_data(4, first=first, count=args.molecules))]
-    sr = stream.StreamRunner(Q, local, levels=args.levels, mode=mode)
+    sr = stream.StreamRunner(Q, local, levels=args.levels, mode=mode, levels_large=args.levels_large)
     totals_dev = torch.zeros(Q.num_graphs, dtype=torch.int64, device=dev)
     if args.cid == 4:
         for gi, (_, qb) in enumerate(sr.groups):
@@ -529,8 +534,8 @@ def run_routed(args, world, rank, local):
             t = sr.run(batches)
         else:
             with torch.cuda.stream(sr.streams[0]):
-                for c in sr.ctx[0]:
-                    c.filter(args.levels)
+                for gi, c in enumerate(sr.ctx[0]):
+                    c.filter(sr.group_levels(gi))
                     c.join(mode, total=False)
             t = None
         return t
@@ -539,6 +544,9 @@ def run_routed(args, world, rank, local):
         step()
     torch.cuda.synchronize(dev)
     K = args.steps
+    if args.cid == 4:  # per-group stage times (the ring-system group runs the general k_join)
+        for c in sr.ctx[0]:
+            c.set_timing(True)
     sampler = ClockSampler(local)
     if dist is not None:
         dist.barrier()
@@ -584,13 +592,17 @@ def run_routed(args, world, rank, local):
             value, unit = Q.num_graphs * nd_all * K / (ms / 1000.0), "graph-pairs/s"
         else:
             value, unit = total * K / (ms / 1000.0), "matches/s"
-        launches = sum(c.timings()["filter_launches"] + c.timings()["join_launches"] for c in sr.ctx[0])
+        tims = [c.timings() for c in sr.ctx[0]]
+        launches = sum(t["filter_launches"] + t["join_launches"] for t in tims)
         line = {
             "metric": BASELINE_METRIC, "value": value, "unit": unit, "n_gpus": world, "steps": K,
             "warmup": max(args.warmup, 3), "ms_per_step": ms / K, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u64", "data": "synthetic", "config": config_dict(args, world),
             "counts": {"matches" if not ff else "positive_pairs": total, "all_pairs": Q.num_graphs * nd_all},
             "query_groups": [int(len(g)) for g, _ in sr.groups],
+            "group_stage_ms": ([{"queries": int(len(g)), "join_kernel": "k_join_lane" if len(g) and gi == 0 else "k_join",
+                                 "filter": t["filter_ms"], "mapping": t["mapping_ms"], "join": t["join_ms"]}
+                                for gi, ((g, _), t) in enumerate(zip(sr.groups, tims))] if args.cid == 4 else None),
             "timing": "wall clock incl. host pack + H2D of every batch" if args.cid == 5 else "device events",
             "gpu_launches": int(K * launches * (len(batches) if args.cid == 5 else 1)),
             "clocks": clocks,

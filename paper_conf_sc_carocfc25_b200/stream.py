@@ -76,11 +76,14 @@ class StreamRunner:
     query order) summed over all batches."""
 
     def __init__(self, queries, device: int = 0, levels: int = 4, mode: int = SIGMO_FIND_ALL,
-                 split: bool = True):
+                 split: bool = True, levels_large: Optional[int] = None):
         import torch
         self.torch = torch
         self.device = device
         self.levels = levels
+        # the group of large queries (general join) may filter deeper: its DFS is
+        # expensive and pruning pays more (levels sweep, DESIGN.md section 9)
+        self.levels_large = levels if levels_large is None else levels_large
         self.mode = mode
         self.nq = queries.num_graphs
         groups = split_queries(queries) if split else [np.arange(self.nq)]
@@ -101,6 +104,10 @@ class StreamRunner:
         for st in self.streams:  # the buffers above were zeroed on the current stream
             st.wait_stream(cur)
 
+    def group_levels(self, gi: int) -> int:
+        """Filter levels of query group gi (the large-query group is the second)."""
+        return self.levels_large if (len(self.groups) > 1 and gi == 1) else self.levels
+
     def reset(self):
         for s, row in zip(self.streams, self.acc):
             with self.torch.cuda.stream(s):
@@ -116,7 +123,7 @@ class StreamRunner:
         for gi, (_, qb) in enumerate(self.groups):
             c = self.ctx[b][gi]
             c.load_batch(qb, data)  # waits only for this buffer's previous H2D
-            c.filter(self.levels)
+            c.filter(self.group_levels(gi))
             c.join(self.mode, total=False)
             c.query_totals(device_tensor=self.tmp[b][gi])
             with torch.cuda.stream(s):
