@@ -422,7 +422,10 @@ def main():
     # ncu --set full of the same kernels at the bench's levels (profiles/r2/ncu_traffic.json, tools/ncu_traffic.py):
     # DRAM bytes per launch and instruction counts; cold-cache and serialised, so only shares/ratios are used
     ncu = _load("profiles/r2/ncu_traffic.json")
-    nk = ncu.get("kernels", {}) if ncu.get("levels") == args.levels else {}
+    # the capture is of the default workload only (configs[2], 1M molecules, monomorphic, no neighbour support)
+    same = (ncu.get("levels") == args.levels and ncu.get("workload") == f"configs[{args.config}]"
+            and args.molecules == 1_000_000 and not args.induced and not args.ns)
+    nk = ncu.get("kernels", {}) if same else {}
     VQ, VD, ND, NQ = Q.num_nodes, D.num_nodes, D.num_graphs, Q.num_graphs
     W = (VD + 31) // 32
     # the method must produce C_L -- VQ x VD bits written once -- plus the GMCR bits / counts,

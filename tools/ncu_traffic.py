@@ -4,6 +4,7 @@ Usage: python tools/ncu_traffic.py report.ncu-rep levels > profiles/r2/ncu_traff
 import csv
 import io
 import json
+import re
 import subprocess
 import sys
 
@@ -22,11 +23,12 @@ def val(r, k):
     return x * scale
 
 
-res = {"source": rep.rsplit("/", 1)[-1], "levels": levels, "kernels": {}}
+res = {"source": rep.rsplit("/", 1)[-1], "levels": levels, "workload": "configs[2]", "kernels": {}}
 for r in rows[2:]:
     name = r[hdr.index("Kernel Name")]
+    m = re.search(r"k_join_lane<0, (\d)", name)  # <MODE, W64, PS>: Find All launches, narrow / wide masks
     key = "sigmo_filter_lane_jit" if "filter_lane" in name else (
-        "k_join_lane_narrow" if "k_join_lane<0, 0>" in name else "k_join_lane_wide" if "k_join_lane<0, 1>" in name else name)
+        ("k_join_lane_wide" if m.group(1) == "1" else "k_join_lane_narrow") if m else name)
     res["kernels"][key] = {
         "ms": val(r, "gpu__time_duration.sum"),
         "dram_bytes": val(r, "dram__bytes_read.sum") + val(r, "dram__bytes_write.sum"),
