@@ -1789,10 +1789,19 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
       // distinct-row index of each plan position's query node into the plan entries
       const std::vector<uint16_t> &qd = c->progs[R].qdrow;
       c->ent_up.resize(c->ent_host.size());
+      // k_join_lane entry of plan position i (JoinParams::qp_ent2): byte offsets of the two
+      // back-edge map slots (slot maxq - 1 = absent), leaf flag, #extra back-edges;
+      // bond classes and the distinct row
+      int64_t q = 0;
       for (size_t i = 0; i < c->ent_up.size(); i++) {
+        while (c->qgoff_host[q + 1] <= (int64_t)i) q++;
         const int4 e = c->ent_host[i];
-        c->ent_up[i].x = ((unsigned)e.x & 0xfffu) | ((unsigned)qd[(size_t)c->ent_row[i]] << 12);
-        c->ent_up[i].y = ((unsigned)e.w & 0xffffu) | ((unsigned)e.y << 16) | ((unsigned)e.z << 19);
+        const unsigned j0 = (unsigned)e.x & 15u, j1 = ((unsigned)e.x >> 4) & 15u, nex = ((unsigned)e.x >> 8) & 15u;
+        const unsigned absent = (unsigned)std::max(c->maxq, 2) - 1u;  // = JoinParams::maxq - 1
+        const unsigned s0 = j0 == 15u ? absent : j0, s1 = j1 == 15u ? absent : j1;
+        const unsigned leaf = (int64_t)i == c->qgoff_host[q + 1] - 1 ? 1u : 0u;
+        c->ent_up[i].x = (s0 << 7) | (leaf << 11) | (nex << 12) | ((s1 << 7) << 16);
+        c->ent_up[i].y = ((unsigned)e.y & 7u) | (((unsigned)e.z & 7u) << 3) | ((unsigned)qd[(size_t)c->ent_row[i]] << 12);
       }
       SIGMO_TRY(dreserve(c, c->ent2, sizeof(uint2) * (c->ent_up.size() + 1), "plan entries"));
       if (!c->ent_up.empty())
@@ -1804,7 +1813,7 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
         int64_t q = 0;
         for (size_t i = 0; i < c->ent_ns_up.size(); i++) {
           while (c->qgoff_host[q + 1] <= (int64_t)i) q++;
-          c->ent_ns_up[i].x = (c->ent_ns_up[i].x & 0xfffu) | ((unsigned)(i - c->qgoff_host[q]) << 12);
+          c->ent_ns_up[i].y = (c->ent_ns_up[i].y & 0xfffu) | ((unsigned)(i - c->qgoff_host[q]) << 12);
         }
       }
       SIGMO_TRY(dreserve(c, c->ent_ns, sizeof(uint2) * (c->ent_ns_up.size() + 1), "plan entries (support)"));
@@ -2050,6 +2059,10 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
       jp.ecur = eo.ecur;
       jp.qp_qn = c->qp_qn;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
+      jp.plan_smem_max = kJoinLanePlanSmemMax;
+      if (const char *e = getenv("SIGMO_JOIN_PLAN_SMEM")) jp.plan_smem_max = atoi(e);  // test knob: 0 = plan through L1
+      jp.carveout = -1;
+      if (const char *e = getenv("SIGMO_JOIN_CARVEOUT")) jp.carveout = atoi(e);  // test knob (percent)
       // two launches: pairs of <= 32-node molecules with 32-bit masks, and
       // the others with 64-bit masks (each finds its range in off[ND]); the
       // wide one on the auxiliary stream, so its CTAs fill the SMs the narrow
@@ -2063,6 +2076,9 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
       for (int w = 0; w < 2; w++) {
         const bool w64 = w == 1;
         if (w64 && !two) break;
+        jp.lane_threads = jl_threads(w64);
+        if (const char *e = getenv(w64 ? "SIGMO_JOIN_WARPS_WIDE" : "SIGMO_JOIN_WARPS"))  // test knob: warps per CTA
+          jp.lane_threads = 32 * std::max(1, std::min(jl_threads(w64) / 32, atoi(e)));
         const size_t smem = join_lane_smem_bytes(jp, w64);
         if (smem > c->max_smem)
           return set_err(c, SIGMO_ERR_LIMIT, "join shared memory %zu exceeds %zu", smem, c->max_smem);
@@ -2073,6 +2089,9 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
         int bps = join_lane_blocks_per_sm((int)mode, w64, jp, smem);
         if (const char *e = getenv("SIGMO_JOIN_BPS")) bps = std::max(1, std::min(bps, atoi(e)));
         const int grid = bps * c->sm_count;
+        if (getenv("SIGMO_DEBUG_JOIN"))
+          fprintf(stderr, "sigmo join: lane %s mode %d threads %d smem %zu blocks/SM %d grid %d\n", w64 ? "wide" : "narrow",
+                  (int)mode, jp.lane_threads, smem, bps, grid);
         CUDA_TRY(c, launch_join_lane((int)mode, w64, jp, grid, w64 ? c->aux : c->stream));
         launches++;
       }

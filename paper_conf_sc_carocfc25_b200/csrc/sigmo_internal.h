@@ -185,8 +185,9 @@ struct JoinParams {
                                // class-major [NB][n], u32 masks (n <= 32) or u64 (n > 32); all ones at word adj_ones
   unsigned adj_ones;
   const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 4 (15 none) | #extra << 8 | node << 12, class0, class1, extra back-edge start}
-  const uint2 *qp_ent2;        // [VQ] compact, k_join_lane: x = j0 | j1 << 4 | #extra << 8 | distinct row << 12,
-                               // y = extra back-edge start (16 b) | class0 << 16 | class1 << 19
+  const uint2 *qp_ent2;        // [VQ] compact, k_join_lane: x = slot0 * 128 | leaf << 11 | #extra back-edges << 12 |
+                               // slot1 * 128 << 16 (slot = back-edge depth, maxq - 1 = none: the map slot
+                               // holding the all-ones index); y = class0 | class1 << 3 | distinct row << 12
   int batchK;                  // finish/assign pairs when >= batchK lanes are free
   int induced;                 // 1 = induced-subgraph embeddings (k_join only, R21):
                                // the union of all bonds is staged as adjacency class NB
@@ -198,6 +199,9 @@ struct JoinParams {
   unsigned long long *esets;   // [embeddings] node set f(V_q) as a molecule-local bit mask (nullable)
   unsigned long long *ecur;    // [P] write cursor per pair (= its first embedding slot after the scan)
   const uint8_t *qp_qn;        // [VQ] local query node of each plan position
+  int plan_smem_max;           // k_join_lane: plan entries copied to shared memory when VQ <= this
+  int carveout;                // k_join_lane: preferred shared-memory carveout in percent (-1: driver default)
+  int lane_threads;            // k_join_lane: threads per CTA of this launch (<= jl_threads(w64))
 };
 
 // k_pairs: GMCR pair list + per-pair candidate masks
@@ -330,6 +334,11 @@ cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, 
 size_t join_lane_smem_bytes(const JoinParams &p, bool w64);
 int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem);
 constexpr int kJoinLaneThreads = 128;
+constexpr int kJoinLanePlanSmemMax = 2048;  // k_join_lane: plan positions copied to shared memory (16 KB)
+// k_join_lane CTA size (the launch-bounds maximum; JoinParams::lane_threads is the launched size): 6 warps for
+// 32-bit masks (7 CTAs x 6 warps at <= 48 registers and ~30 KB of shared memory; the plan copy and the per-query
+// totals are per CTA), 4 for 64-bit masks
+__host__ __device__ constexpr int jl_threads(bool w64) { return w64 ? 128 : 192; }
 constexpr int kJoinLaneMaxQ = 11;  // k_join_lane handles queries <= 11 nodes in <= 64-node graphs (map: 6 bits x 10 depths)
 size_t join_smem_bytes(int NW, const JoinParams &p);
 size_t join_gstack_bytes(int NW, const JoinParams &p, int grid);

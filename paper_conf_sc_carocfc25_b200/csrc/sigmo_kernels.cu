@@ -2001,7 +2001,7 @@ __global__ void __launch_bounds__(kSupportLaneThreads) k_support_lane(const __gr
   };
   bool empty = false;
   for (unsigned e = 0; e < nq; e++) {
-    const unsigned row = __ldg(&sp.qp_ent2[qb + e]).x >> 12;
+    const unsigned row = __ldg(&sp.qp_ent2[qb + e]).y >> 12;
     const MT w = W64 ? (MT)__ldg((const unsigned long long *)(sp.cmol + (cmb + 2u * row))) : (MT)__ldg(sp.cmol + (cmb + row));
     wv[e * T] = w;
     empty |= w == (MT)0;
@@ -2239,25 +2239,26 @@ cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const
 //   * Per-query totals are reduced in shared memory (one global atomic per
 //     query per CTA).
 // ===========================================================================
-constexpr int kJoinChunk = 32;  // GMCR pairs per warp claim (one record per lane)
+constexpr int kJoinChunk = 16;    // GMCR pair records per warp buffer (copied to shared memory by lanes 0..15)
+constexpr int kJoinClaim = 128;   // GMCR pairs per warp claim (atomic on the launch's pair counter)
 
 // stack entry {R, U}: 2 x 32-bit masks (<= 32-node molecules) or 2 x 64-bit
 __host__ __device__ inline size_t join_lane_warp_bytes(int MQ, bool w64) {
   const int SD = MQ > 1 ? MQ - 1 : 1;  // pushed depths 0..n-2
-  // {R, U} [SD][32] (8 or 16 B) | map [16][32] B
-  return 32 * (size_t)(w64 ? 16 : 8) * SD + 512;
+  // pair records [2][kJoinChunk] (current and next chunk) | next pair per lane: record [32] int4, index [32] |
+  // {R, U} [SD][32] (8 or 16 B) | map words [SD + 1][32] (u32: adjacency index of f(pi_d); slot SD: all ones)
+  return 2 * 16 * (size_t)kJoinChunk + 16 * 32 + 4 * 32 + 32 * (size_t)(w64 ? 16 : 8) * SD + 128 * (size_t)(SD + 1);
 }
 // CTA: per-query totals [NQ] u64, then one region per warp
 // CTA: per-query totals [NQ] u64, then (optionally) the plan entries [VQ] uint2
-constexpr int kJoinLanePlanSmemMax = 2048;  // plan positions copied to shared memory (16 KB)
-__host__ __device__ inline size_t join_lane_plan_bytes(int VQ) { return VQ <= kJoinLanePlanSmemMax ? align16(8 * (size_t)VQ) : 0; }
-__host__ __device__ inline size_t join_lane_cta_bytes(int NQ, int VQ) {
-  return align16(8 * (size_t)(NQ > 0 ? NQ : 1)) + join_lane_plan_bytes(VQ);
+__host__ __device__ inline size_t join_lane_plan_bytes(int VQ, int pmax) { return VQ <= pmax ? align16(8 * (size_t)VQ) : 0; }
+__host__ __device__ inline size_t join_lane_cta_bytes(int NQ, int VQ, int pmax) {
+  return align16(8 * (size_t)(NQ > 0 ? NQ : 1)) + join_lane_plan_bytes(VQ, pmax);
 }
-__host__ __device__ inline size_t join_lane_smem(int NQ, int VQ, int MQ, bool w64) {
-  return join_lane_cta_bytes(NQ, VQ) + join_lane_warp_bytes(MQ, w64) * (kJoinLaneThreads / 32);
+__host__ __device__ inline size_t join_lane_smem(int NQ, int VQ, int MQ, bool w64, int pmax, int threads) {
+  return join_lane_cta_bytes(NQ, VQ, pmax) + join_lane_warp_bytes(MQ, w64) * (size_t)(threads / 32);
 }
-size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_smem(p.NQ, p.VQ, p.maxq, w64); }
+size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_smem(p.NQ, p.VQ, p.maxq, w64, p.plan_smem_max, p.lane_threads); }
 
 // n-th (0-based) set bit of m (m has > n set bits)
 __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
@@ -2265,37 +2266,43 @@ __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
   return __ffs(m) - 1;
 }
 
+__device__ __forceinline__ uint2 lds_u2(unsigned a) {
+  uint2 v;
+  asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
+  return v;
+}
+
 // W64: the launch's pairs are on > 32-node molecules (64-bit masks); else all
 // masks, stack entries and loads are 32-bit
 // PS: the plan entries are copied to shared memory (VQ <= kJoinLanePlanSmemMax)
+#ifndef SIGMO_JL_MAXNREG
+#define SIGMO_JL_MAXNREG 56
+#endif
 template <int MODE, bool W64, bool PS>
-__global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_constant__ JoinParams jp) {
+__global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_JL_MAXNREG) k_join_lane(const __grid_constant__ JoinParams jp) {
   using MT = typename std::conditional<W64, unsigned long long, unsigned>::type;
   constexpr unsigned ES = W64 ? 16u : 8u;  // stack entry bytes
+  constexpr unsigned sw = W64 ? 1u : 0u;   // word shift of an adjacency / window entry
   extern __shared__ __align__(16) unsigned char smem[];
-#define LDS64(o) (*(const unsigned long long *)(smem + (o)))
-#define STS64(o) (*(unsigned long long *)(smem + (o)))
-#define LDS128(o) (*(const ulonglong2 *)(smem + (o)))
-#define STS128(o) (*(ulonglong2 *)(smem + (o)))
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int MQ = jp.maxq, SD = MQ > 1 ? MQ - 1 : 1;
   // ---- CTA tables ----
   const unsigned o_tot = 0u;
   for (int i = threadIdx.x; i < jp.NQ; i += blockDim.x) ((unsigned long long *)(smem + o_tot))[i] = 0ull;
-  // plan entry of plan position i, read through L1 (measured on configs[2]: a
-  // shared-memory copy of the entries 15.5 vs 10.0 ms; staging each pair's
-  // candidate rows in lane-private shared memory by cp.async, 10.6 vs 9.8 ms
-  // -- both lose to the occupancy they cost; so did taking two leaf-level
-  // candidates per step, 9.60 vs 9.49 ms, and caching the top stack entry in
-  // registers, 8.92 vs 8.80 ms)
-  // plan entries (8 B): a shared-memory copy when they fit, else through the read-only cache
+  // plan entries (8 B, JoinParams::qp_ent2): a shared-memory copy when they fit, else through the read-only cache
   const unsigned o_plan = (unsigned)align16(8 * (size_t)(jp.NQ > 0 ? jp.NQ : 1));
   if (PS)
     for (int i = threadIdx.x; i < jp.VQ; i += blockDim.x) ((uint2 *)(smem + o_plan))[i] = __ldg(&jp.qp_ent2[i]);
-#define JL_PLAN(i) (PS ? ((const uint2 *)(smem + o_plan))[(i)] : __ldg(&jp.qp_ent2[(i)]))
-  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ, jp.VQ) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
-  const unsigned oRU = wbase + ES * lane;                         // {R, U} of depth d: oRU + 32 ES d
-  const unsigned oM = wbase + 32u * ES * SD + lane;               // f(pi_d): oM + 32 d
+  // plan entry at shared-space address / global index p (an explicit ld.shared:
+  // a generic smem + offset re-derives the shared window every step)
+  const unsigned sbase = (unsigned)__cvta_generic_to_shared(smem);
+#define JL_PLAN(p) (PS ? lds_u2(p) : __ldg(&jp.qp_ent2[(p)]))
+  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ, jp.VQ, jp.plan_smem_max) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
+  const unsigned oRec = wbase;                              // pair records of chunk buffer b: oRec + 16 kJoinChunk b
+  const unsigned oNx = wbase + 32u * kJoinChunk + 16u * lane;  // record of the lane's next pair
+  const unsigned oNp = wbase + 32u * kJoinChunk + 512u + 4u * lane;  // its index
+  const unsigned oRU = wbase + 32u * kJoinChunk + 640u + ES * lane;  // {R, U} of depth d: oRU + 32 ES d
+  const unsigned mA = oRU - ES * lane + 32u * ES * SD + 4u * lane;  // map word of depth d: mA + 128 d (slot SD: absent)
   // stack entry {R, U} at byte offset o of the kernel's shared memory (macros,
   // not lambdas: a captured `smem` loses its address space and every access
   // would re-derive the shared window)
@@ -2316,15 +2323,23 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     if (W64) *(ulonglong2 *)(smem + (o)) = make_ulonglong2((unsigned long long)(r), (unsigned long long)(u));      \
     else *(uint2 *)(smem + (o)) = make_uint2((unsigned)(r), (unsigned)(u));                                        \
   } while (0)
+#define JL_MAP(d) (*(unsigned *)(smem + mA + 128u * (unsigned)(d)))
   auto popc = [](MT x) -> int { return W64 ? __popcll((unsigned long long)x) : __popc((unsigned)x); };
-  auto lowest = [](MT x) -> int {  // index of the lowest set bit (x != 0)
-    if (W64) {
-      const unsigned lo = (unsigned)x, hi = (unsigned)((unsigned long long)x >> 32);
-      return lo ? __ffs(lo) - 1 : 31 + __ffs(hi);
-    }
-    return __ffs((unsigned)x) - 1;
+  auto highest = [](MT x) -> unsigned {  // index of the highest set bit (x != 0)
+    unsigned r;
+    if (W64) asm("bfind.u64 %0, %1;" : "=r"(r) : "l"((unsigned long long)x));
+    else asm("bfind.u32 %0, %1;" : "=r"(r) : "r"((unsigned)x));
+    return r;
   };
-  smem[oM + 32 * 15] = 0;  // map slot 15 (absent back-edge) reads node 0 of the all-ones class
+  auto bfind32 = [](unsigned x) -> unsigned {
+    unsigned r;
+    asm("bfind.u32 %0, %1;" : "=r"(r) : "r"(x));
+    return r;
+  };
+  auto lowest = [](MT x) -> unsigned {  // index of the lowest set bit (x != 0)
+    return W64 ? (unsigned)(__ffsll((long long)x) - 1) : (unsigned)(__ffs((unsigned)x) - 1);
+  };
+  JL_MAP(SD) = jp.adj_ones;  // absent back-edges read the all-ones entry (class field 0)
   __syncthreads();
 
   const unsigned lt = (1u << lane) - 1u;
@@ -2342,59 +2357,80 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     return (MT)__ldg(adjw + i);
   };
   const uint32_t *const cmol = jp.cmol;
-  // candidate window of distinct row r of the pair's molecule (cmol word base cb)
-  auto cand = [&](unsigned cb, unsigned r) -> MT {
-    if (W64) return (MT)__ldg((const unsigned long long *)(cmol + (cb + 2u * r)));
-    return (MT)__ldg(cmol + (cb + r));
+  // candidate window at cmol word index i
+  auto cand = [&](unsigned i) -> MT {
+    if (W64) return (MT)__ldg((const unsigned long long *)(cmol + i));
+    return (MT)__ldg(cmol + i);
   };
-  const unsigned ones = jp.adj_ones;  // the all-ones entry (absent back-edge)
-  const int4 zero4 = make_int4(0, 0, 0, 0);
+  // plan address (smem byte offset, or global index) of plan position i
+  auto paddr = [&](unsigned i) -> unsigned { return PS ? sbase + o_plan + 8u * i : i; };
+  constexpr unsigned PSTEP = PS ? 8u : 1u;
+  // plan position of depth 0 of the pair whose depth-1 plan address is a
+  auto cqb_of = [&](unsigned a) -> unsigned { return PS ? (a - sbase - o_plan) / 8u - 1u : a - 1u; };
 
-  // ---- GMCR chunks: current (records of pairs cbase + i in lane i's crec), prefetched, claimed ----
-  unsigned cbase, pbase, nbase;
+  // ---- GMCR chunks of kJoinChunk pairs: the current one (cbase, chead taken) and the next, claimed a
+  // chunk ahead; their records are copied into the warp's two record buffers by cp.async (no registers,
+  // no stall: a buffer is waited for one chunk after its copy was issued) ----
+  const unsigned srec = sbase + oRec + 16u * lane;
+  auto fetch_chunk = [&](unsigned base, unsigned buf) {
+    if (lane < kJoinChunk && base + lane < P)
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(srec + 16u * kJoinChunk * buf), "l"(recs + base + lane)
+                   : "memory");
+    asm volatile("cp.async.commit_group;\n" ::: "memory");
+  };
+  // the warp claims blocks of kJoinClaim pairs (one same-address atomic per block: at one atomic per chunk the
+  // counter serialised the launch), a block ahead; lane 0 holds the next block's start until it is needed
+  unsigned cbase, pbase, pnext, bend, cbuf = 0u, bnext0 = 0u;
   {
     unsigned x = 0u;
-    if (lane == 0) x = atomicAdd(cursor, 3u * kJoinChunk);
+    if (lane == 0) x = atomicAdd(cursor, 2u * kJoinClaim);
     x = __shfl_sync(FULL_MASK, x, 0);
     cbase = x;
     pbase = x + kJoinChunk;
-    nbase = x + 2u * kJoinChunk;
+    pnext = x + 2u * kJoinChunk;
+    bend = x + kJoinClaim;
+    bnext0 = x + kJoinClaim;
+    fetch_chunk(cbase, 0u);
+    fetch_chunk(pbase, 1u);
+    asm volatile("cp.async.wait_group 1;\n" ::: "memory");  // the current chunk
+    __syncwarp();
   }
-  int4 crec = cbase + lane < P ? __ldg(&recs[cbase + lane]) : zero4;
-  int4 prec = pbase + lane < P ? __ldg(&recs[pbase + lane]) : zero4;
   unsigned ccount = cbase < P ? min(P - cbase, (unsigned)kJoinChunk) : 0u, chead = 0u;
   bool drained = ccount == 0u;
+  int keff = jp.batchK;  // free lanes that end a stepping phase (1 once the list is drained)
+  if (drained) keff = 1;
 
   // ---- lane state ----
   unsigned ne = 0u;  // open depths of the current pair (0: no work)
-  bool pend = false, shared = false;
-  unsigned cmb = 0u;  // cmol index of the current pair's first candidate row
-  unsigned cp = 0u, ca = 0u, cqb = 0u, cinfo = 0u;  // ca: adjb index of the molecule's first node
+  bool pend = false;  // holds a pair (part) whose result is not yet written
+  bool shared = false;
+  unsigned cmb = 0u;  // cmol index of the current pair's first candidate window
+  unsigned ca = 0u, ngs = 0u, pe = 0u;  // ca: adjacency index of the molecule's node 0; pe: plan address of depth 1
+  unsigned cp = 0u;
   int cq = 0;
   unsigned long long cnt = 0ull;
   unsigned steps = 0u;
-  bool nv = false;  // next pair assigned (rows in flight into the other buffer)
-  unsigned np = 0u;
-  int4 nrec = zero4;
+  bool nv = false;  // next pair assigned (record and index in the lane's slots, root window in flight)
   MT nR0 = 0;
 
   // enumerate mode: the embeddings of a leaf step -- the
-  // mapped depths 0..d (map bytes) plus each candidate w of the last depth --
+  // mapped depths 0..d (map words) plus each candidate w of the last depth --
   // written in query node order at the pair's cursor (count pass + scan set
   // it to the pair's first slot; several lanes may share a donated pair), and
   // the node set f(V_q) as a molecule-local bit mask
   auto emit = [&](MT X, int d, MT used) {
+    const unsigned cqb = cqb_of(pe);
     unsigned long long r0 = 0ull, r1 = 0ull;
     for (int j = 0; j <= d; j++) {
       const unsigned qn = __ldg(&jp.qp_qn[cqb + (unsigned)j]);
-      const unsigned long long b = smem[oM + 32u * (unsigned)j];
+      const unsigned long long b = (JL_MAP(j) - ca) >> sw;
       if (qn < 8u) r0 |= b << (8u * qn);
       else r1 |= b << (8u * (qn - 8u));
     }
     const unsigned qe = __ldg(&jp.qp_qn[cqb + (unsigned)(d + 1)]);
     unsigned long long pos = atomicAdd(jp.ecur + pbase0 + cp, (unsigned long long)popc(X));
     while (X) {
-      const unsigned w = (unsigned)lowest(X);
+      const unsigned w = lowest(X);
       X &= X - (MT)1;
       const unsigned long long a0 = r0 | (qe < 8u ? (unsigned long long)w << (8u * qe) : 0ull);
       const unsigned long long a1 = r1 | (qe >= 8u ? (unsigned long long)w << (8u * (qe - 8u)) : 0ull);
@@ -2411,64 +2447,61 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
   while (true) {
     // ---- one DFS step ----
     if (ne) {
-      const int d = 31 - __clz(ne);
-      const int e = d + 1;
+      const unsigned d = bfind32(ne);  // deepest open depth
       const unsigned od = oRU + 32u * ES * d;
-      // the plan entry of depth e and the map bytes of its back-edge targets
-      // depend on d only: loaded before v is known (j == d takes v below)
-      const uint2 en = JL_PLAN(cqb + e);
+      // plan entry of depth e = d + 1 (x: back-edge map slots, leaf, #extra;
+      // y: bond classes, distinct row)
+      const uint2 en = JL_PLAN(pe + PSTEP * d);
       MT R, U;
       JL_LDRU(od, R, U);
-      const unsigned j0 = en.x & 15, j1 = (en.x >> 4) & 15;
-      const unsigned m0 = smem[oM + 32u * j0], m1 = smem[oM + 32u * j1];
-      const int v = lowest(R);
+      const unsigned v = highest(R);
       const MT bit = (MT)1 << v;
       const MT Rn = R ^ bit;
       *(MT *)(smem + od) = Rn;
-      smem[oM + 32u * d] = (unsigned char)v;
       if (!Rn) ne ^= 1u << d;
+      // map word of depth d = the adjacency index of f(pi_d); stored before the
+      // back-edge slots are read, so a back-edge to d reads it
+      JL_MAP(d) = ca + (v << sw);
+      const unsigned a0 = *(const unsigned *)(smem + mA + (en.x & 0x7ffu));
+      const unsigned a1 = *(const unsigned *)(smem + mA + (en.x >> 16));
+      const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
       const MT used = U | bit;
-      // candidates of depth e
-      const unsigned u0 = j0 == (unsigned)d ? (unsigned)v : m0, u1 = j1 == (unsigned)d ? (unsigned)v : m1;
-      const unsigned ng = (cinfo >> 8) & 0xffu;  // molecule size: class stride of the adjacency
-      constexpr unsigned sw = W64 ? 1u : 0u;  // word shift of an entry
-      const unsigned i0 = j0 == 15u ? ones : ca + ((((en.y >> 16) & 7u) * ng + u0) << sw);
-      const unsigned i1 = j1 == 15u ? ones : ca + ((((en.y >> 19) & 7u) * ng + u1) << sw);
-      MT X = cand(cmb, (unsigned)en.x >> 12) & ~used & adj(i0) & adj(i1);
-      if (en.x & 0xf00) {  // > 2 back-edges at this depth (fused rings): rare
-        const int nex = (en.x >> 8) & 15;
-        for (int k = 0; k < nex; k++) {
-          const int be = __ldg(&jp.qp_be[(en.y & 0xffffu) + k]);
-          X &= adj(ca + (((unsigned)(be & 255) * ng + smem[oM + 32u * (be >> 8)]) << sw));
+      MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0) & adj(i1);
+      if (en.x & 0xf000u) {  // > 2 back-edges at this depth (fused rings): rare
+        const unsigned nex = (en.x >> 12) & 15u;
+        const unsigned b0 = (unsigned)__ldg(&jp.qp_ent[cqb_of(pe) + d + 1u]).w;
+#pragma unroll 1
+        for (unsigned k = 0; k < nex; k++) {
+          const unsigned be = __ldg(&jp.qp_be[b0 + k]);
+          X &= adj((be & 255u) * ngs + JL_MAP(be >> 8));
         }
       }
       if (MODE & 2) {  // induced mode (R21): drop neighbours (any bond) of mapped non-adjacent depths
-        const unsigned cn = (unsigned)jp.NB * ng;
+        const unsigned cn = (unsigned)jp.NB * ngs;
         // two depths per iteration (the second reads the all-zeros entry when absent)
-        for (unsigned nm = __ldg(&jp.qp_non[cqb + e]); nm;) {
-          const unsigned ia = ca + ((cn + smem[oM + 32u * (unsigned)(__ffs(nm) - 1)]) << sw);
+#pragma unroll 1
+        for (unsigned nm = __ldg(&jp.qp_non[cqb_of(pe) + d + 1u]); nm;) {
+          const unsigned ia = cn + JL_MAP(__ffs(nm) - 1);
           nm &= nm - 1u;
-          const unsigned ib = nm ? ca + ((cn + smem[oM + 32u * (unsigned)(__ffs(nm) - 1)]) << sw) : ones + 2u;
+          const unsigned ib = nm ? cn + JL_MAP(__ffs(nm) - 1) : jp.adj_ones + 2u;
           nm &= nm - 1u;
           X &= ~(adj(ia) | adj(ib));
         }
       }
-      if (e == (int)(cinfo & 0xff) - 1) {
+      if (en.x & 0x800u) {  // depth e is the last: count (or decide) its candidates
         cnt += (unsigned long long)popc(X);
-        if ((MODE & 4) && X) emit(X, d, used);  // enumerate mode: write the embeddings
-        if ((MODE & 1) && cnt) ne = 0u;  // Find First: the pair (part) is decided
+        if ((MODE & 4) && X) emit(X, (int)d, used);  // enumerate mode: write the embeddings
+        if ((MODE & 1) && X) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
-        JL_STRU(oRU + 32u * ES * e, X, used);
-        ne |= 1u << e;
+        JL_STRU(od + 32u * ES, X, used);
+        ne += 2u << d;  // bit d + 1 is clear: d is the deepest open depth
       }
-      pend = ne == 0u;
       steps++;
     }
-    const unsigned fm = __ballot_sync(FULL_MASK, ne == 0u);
-    if (drained ? fm == 0u : (__popc(fm) < jp.batchK && fm != FULL_MASK)) continue;
+    if (__popc(__ballot_sync(FULL_MASK, ne == 0u)) < keff) continue;
 
     // ---- finished pairs (parts): result, per-query total in shared memory ----
-    if (pend) {
+    if (pend && ne == 0u) {
       if (MODE & 1) {
         if (!shared) {
           presult[cp] = cnt ? 1ull : 0ull;
@@ -2485,27 +2518,27 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     }
     // ---- free lanes activate their prefetched next pair ----
     if (ne == 0u && nv) {
-      cp = np;
+      const int4 nrec = *(const int4 *)(smem + oNx);
+      cp = *(const unsigned *)(smem + oNp);
       cmb = (unsigned)nrec.z;
       ca = (unsigned)nrec.x;  // adjacency word offset of the molecule
       cq = nrec.y;
-      cinfo = (unsigned)nrec.w;
-      cqb = cinfo >> 16;
+      ngs = (((unsigned)nrec.w >> 8) & 0xffu) << sw;  // molecule size: class stride of the adjacency
+      pe = paddr(((unsigned)nrec.w >> 16) + 1u);
       shared = false;
+      pend = true;
       cnt = 0ull;
       const MT R0 = nR0;
-      if ((cinfo & 0xff) == 1u) {
+      if ((nrec.w & 0xff) == 1) {
         cnt = (unsigned long long)popc(R0);
         if ((MODE & 4) && R0) emit(R0, -1, (MT)0);
-        pend = true;
       } else {
         JL_STRU(oRU, R0, (MT)0);
         ne = R0 ? 1u : 0u;
-        pend = ne == 0u;
       }
       nv = false;
     }
-    // ---- lanes without a next pair take one from the chunk and prefetch its rows ----
+    // ---- lanes without a next pair take one from the chunk and prefetch its root window ----
     unsigned wm = __ballot_sync(FULL_MASK, !nv && !drained);
     while (wm) {
       const unsigned avail = ccount - chead;
@@ -2513,35 +2546,36 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
       const unsigned take = min(n, avail);
       const unsigned rank = (unsigned)__popc(wm & lt);
       const bool mine = ((wm >> lane) & 1u) && rank < take;
-      const int src = (int)(chead + (mine ? rank : 0u));
-      int4 r;
-      r.x = __shfl_sync(FULL_MASK, crec.x, src);
-      r.y = __shfl_sync(FULL_MASK, crec.y, src);
-      r.z = __shfl_sync(FULL_MASK, crec.z, src);
-      r.w = __shfl_sync(FULL_MASK, crec.w, src);
       if (mine) {
-        nrec = r;
-        np = cbase + (unsigned)src;
+        const int4 nrec = *(const int4 *)(smem + oRec + 16u * kJoinChunk * cbuf + 16u * (chead + rank));
+        *(int4 *)(smem + oNx) = nrec;
+        *(unsigned *)(smem + oNp) = cbase + chead + rank;
         nv = true;
-        // root candidates of the next pair: the load completes while the current pair runs
-        nR0 = cand((unsigned)r.z, JL_PLAN((unsigned)r.w >> 16).x >> 12);
+        // root candidates of the next pair: the loads complete while the current pair runs
+        nR0 = cand((unsigned)nrec.z + ((JL_PLAN(paddr((unsigned)nrec.w >> 16)).y >> 12) << sw));
       }
       chead += take;
       wm = __ballot_sync(FULL_MASK, !nv) & wm;
       if (chead == ccount) {  // chunk exhausted: switch to the prefetched one, claim the one after
         cbase = pbase;
-        crec = prec;
         ccount = cbase < P ? min(P - cbase, (unsigned)kJoinChunk) : 0u;
         chead = 0u;
         if (ccount == 0u) {
           drained = true;
+          keff = 1;
           break;
         }
-        pbase = nbase;
-        prec = pbase + lane < P ? __ldg(&recs[pbase + lane]) : zero4;
-        unsigned x = 0u;
-        if (lane == 0) x = atomicAdd(cursor, (unsigned)kJoinChunk);
-        nbase = __shfl_sync(FULL_MASK, x, 0);
+        asm volatile("cp.async.wait_all;\n" ::: "memory");  // the next chunk (issued a chunk ago)
+        __syncwarp();
+        cbuf ^= 1u;
+        if (pnext == bend) {  // the block is scheduled: continue with the claimed one, claim the one after
+          pnext = __shfl_sync(FULL_MASK, bnext0, 0);
+          bend = pnext + kJoinClaim;
+          if (lane == 0) bnext0 = atomicAdd(cursor, (unsigned)kJoinClaim);
+        }
+        pbase = pnext;
+        pnext += kJoinChunk;
+        fetch_chunk(pbase, cbuf ^ 1u);  // into the buffer just emptied
       }
     }
     // ---- drained: idle lanes take the shallowest open depth of a busy lane ----
@@ -2557,7 +2591,8 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         const int ds = __shfl_sync(FULL_MASK, ds_own, src);
         const unsigned s_cp = __shfl_sync(FULL_MASK, cp, src);
         const int s_cq = __shfl_sync(FULL_MASK, cq, src);
-        const unsigned s_info = __shfl_sync(FULL_MASK, cinfo, src);
+        const unsigned s_ngs = __shfl_sync(FULL_MASK, ngs, src);
+        const unsigned s_pe = __shfl_sync(FULL_MASK, pe, src);
         const unsigned s_ca = __shfl_sync(FULL_MASK, ca, src);
         const unsigned s_cmb = __shfl_sync(FULL_MASK, cmb, src);
         if (give && !shared) {
@@ -2566,23 +2601,23 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
         }
         __syncwarp();
         if (recv) {
-          const unsigned dl = (unsigned)(src - lane);  // donor offsets = mine + dl * (8 | 16 | 1)
+          const unsigned dl = (unsigned)(src - lane);  // donor offsets = mine + dl * (ES | 4)
           {
             MT r, u;
             JL_LDRU(oRU + 32u * ES * ds + ES * dl, r, u);
             JL_STRU(oRU + 32u * ES * ds, r, u);
           }
-          for (int j = 0; j < ds; j++) smem[oM + 32u * j] = smem[oM + 32u * j + dl];
+          for (int j = 0; j < ds; j++) JL_MAP(j) = *(const unsigned *)(smem + mA + 128u * j + 4u * dl);
           cmb = s_cmb;
           cp = s_cp;
           cq = s_cq;
-          cinfo = s_info;
-          cqb = s_info >> 16;
+          ngs = s_ngs;
+          pe = s_pe;
           ca = s_ca;
           ne = 1u << ds;
           cnt = 0ull;
           shared = true;
-          pend = false;
+          pend = true;
         }
         __syncwarp();
         if (give) ne &= ~(1u << ds_own);
@@ -2590,6 +2625,7 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     }
     if (drained && __ballot_sync(FULL_MASK, ne != 0u || nv || pend) == 0u) break;
   }
+  asm volatile("cp.async.wait_all;\n" ::: "memory");  // no copy in flight into the CTA's shared memory at exit
   if (jp.stats) {
     unsigned long long s2 = steps;
 #pragma unroll
@@ -2601,28 +2637,32 @@ __global__ void __launch_bounds__(kJoinLaneThreads) k_join_lane(const __grid_con
     const unsigned long long t = ((const unsigned long long *)(smem + o_tot))[q];
     if (t) atomicAdd(&jp.totals[q], t);
   }
-#undef LDS64
-#undef STS64
-#undef LDS128
-#undef STS128
 #undef JL_LDRU
 #undef JL_STRU
 #undef JL_PLAN
+#undef JL_MAP
+}
+
+// dynamic shared memory size and (optionally) the preferred shared-memory carveout of a k_join_lane instantiation
+template <typename K>
+static cudaError_t jl_attrs(K k, size_t smem, int carveout) {
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess && carveout >= 0)
+    e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, carveout);
+  return e;
 }
 
 template <int MODE, bool W64>
 static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_t st) {
   // plan entries in shared memory when they fit (join_lane_plan_bytes)
-  if (join_lane_plan_bytes(p.VQ) > 0) {
-    cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE, W64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)p.smem_bytes);
+  if (join_lane_plan_bytes(p.VQ, p.plan_smem_max) > 0) {
+    cudaError_t e = jl_attrs(k_join_lane<MODE, W64, true>, p.smem_bytes, p.carveout);
     if (e != cudaSuccess) return e;
-    k_join_lane<MODE, W64, true><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
+    k_join_lane<MODE, W64, true><<<grid, p.lane_threads, p.smem_bytes, st>>>(p);
   } else {
-    cudaError_t e = cudaFuncSetAttribute(k_join_lane<MODE, W64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)p.smem_bytes);
+    cudaError_t e = jl_attrs(k_join_lane<MODE, W64, false>, p.smem_bytes, p.carveout);
     if (e != cudaSuccess) return e;
-    k_join_lane<MODE, W64, false><<<grid, kJoinLaneThreads, p.smem_bytes, st>>>(p);
+    k_join_lane<MODE, W64, false><<<grid, p.lane_threads, p.smem_bytes, st>>>(p);
   }
   return cudaGetLastError();
 }
@@ -2652,15 +2692,15 @@ cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, 
 }
 
 template <int MODE, bool W64>
-static int join_lane_occ_t(size_t smem, bool ps) {
+static int join_lane_occ_t(size_t smem, bool ps, int carveout, int threads) {
   int n = 0;
   cudaError_t e;
   if (ps) {
-    cudaFuncSetAttribute(k_join_lane<MODE, W64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE, W64, true>, kJoinLaneThreads, smem);
+    jl_attrs(k_join_lane<MODE, W64, true>, smem, carveout);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE, W64, true>, threads, smem);
   } else {
-    cudaFuncSetAttribute(k_join_lane<MODE, W64, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE, W64, false>, kJoinLaneThreads, smem);
+    jl_attrs(k_join_lane<MODE, W64, false>, smem, carveout);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_join_lane<MODE, W64, false>, threads, smem);
   }
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -2672,24 +2712,24 @@ static int join_lane_occ_t(size_t smem, bool ps) {
 int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem) {
   // the instantiation launch_join_lane picks: bit 0 Find First, bit 1 induced, enumerate
   const int m = (mode & 1) | (p.induced ? 2 : 0);
-  const bool ps = join_lane_plan_bytes(p.VQ) > 0;
+  const bool ps = join_lane_plan_bytes(p.VQ, p.plan_smem_max) > 0;
   if (p.emaps) {
-    if (w64) return p.induced ? join_lane_occ_t<6, true>(smem, ps) : join_lane_occ_t<4, true>(smem, ps);
-    return p.induced ? join_lane_occ_t<6, false>(smem, ps) : join_lane_occ_t<4, false>(smem, ps);
+    if (w64) return p.induced ? join_lane_occ_t<6, true>(smem, ps, p.carveout, p.lane_threads) : join_lane_occ_t<4, true>(smem, ps, p.carveout, p.lane_threads);
+    return p.induced ? join_lane_occ_t<6, false>(smem, ps, p.carveout, p.lane_threads) : join_lane_occ_t<4, false>(smem, ps, p.carveout, p.lane_threads);
   }
   if (w64) {
     switch (m) {
-      case 0: return join_lane_occ_t<0, true>(smem, ps);
-      case 1: return join_lane_occ_t<1, true>(smem, ps);
-      case 2: return join_lane_occ_t<2, true>(smem, ps);
-      default: return join_lane_occ_t<3, true>(smem, ps);
+      case 0: return join_lane_occ_t<0, true>(smem, ps, p.carveout, p.lane_threads);
+      case 1: return join_lane_occ_t<1, true>(smem, ps, p.carveout, p.lane_threads);
+      case 2: return join_lane_occ_t<2, true>(smem, ps, p.carveout, p.lane_threads);
+      default: return join_lane_occ_t<3, true>(smem, ps, p.carveout, p.lane_threads);
     }
   }
   switch (m) {
-    case 0: return join_lane_occ_t<0, false>(smem, ps);
-    case 1: return join_lane_occ_t<1, false>(smem, ps);
-    case 2: return join_lane_occ_t<2, false>(smem, ps);
-    default: return join_lane_occ_t<3, false>(smem, ps);
+    case 0: return join_lane_occ_t<0, false>(smem, ps, p.carveout, p.lane_threads);
+    case 1: return join_lane_occ_t<1, false>(smem, ps, p.carveout, p.lane_threads);
+    case 2: return join_lane_occ_t<2, false>(smem, ps, p.carveout, p.lane_threads);
+    default: return join_lane_occ_t<3, false>(smem, ps, p.carveout, p.lane_threads);
   }
 }
 
