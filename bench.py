@@ -40,6 +40,7 @@ BASELINE_METRIC = "matches/sec (Find All) and graph-pairs/sec (Find First) at 1/
 # configs[3]/[4] are 8-GPU configurations: the per-rank default is the 8-GPU
 # share (1M / 8 and 10M / 8), so `--gpus 8` processes the whole config.
 CONFIGS = {1: (2, 100_000), 2: (3, 1_000_000), 3: (4, 125_000), 4: (5, 1_250_000)}
+E2E_BATCH = 250_000  # molecules per host batch of the e2e measurement (StreamRunner)
 STREAM_BATCH = 250_000        # configs[4]: molecules per streamed batch per GPU
 LEVELS = 2  # best of the configs[1] sweep (profiles/r2/levels_sweep_c1.jsonl)
 CPU_SAMPLE_MOLS = 200_000     # cpu_baseline leg: oracle on the first 200k molecules (~100 core-seconds)
@@ -376,23 +377,32 @@ def main():
     positive_local = int(ctx.join(sigmo.SIGMO_FIND_FIRST))
 
     # ---- e2e through the public API from host buffers ----
-    # the inputs sit in page-locked host memory (as a loader feeding the GPU
-    # holds them); sigmo_load_batch copies them every step inside the timed region
-    cq, cd = sigmo.as_c_batch(Q, pinned=True), sigmo.as_c_batch(D, pinned=True)
+    # the inputs sit in page-locked host memory as a loader feeding the GPU holds
+    # them: the step's molecules in batches of E2E_BATCH, run by the double-buffered
+    # StreamRunner (stream.py; each batch's host-to-device copy overlaps the previous
+    # batch's filter + join); the copies and the D2H of the per-query totals are
+    # inside the timed region
+    from paper_conf_sc_carocfc25_b200.stream import StreamRunner
+    n_local = D.num_graphs
+    nb_e2e = max(1, (n_local + E2E_BATCH - 1) // E2E_BATCH)
+    parts = [D.slice(i * n_local // nb_e2e, (i + 1) * n_local // nb_e2e) for i in range(nb_e2e)]
+    h2d = sum(p.nbytes() for p in parts) + nb_e2e * Q.nbytes()  # every batch also loads the (small) queries
+    subs = [sigmo.as_c_batch(p, pinned=True) for p in parts]
+    del parts
+    runner = StreamRunner(Q, local, levels=args.levels, mode=sigmo.SIGMO_FIND_ALL, split=False,
+                          induced=args.induced, neighbor_support=args.ns)
     e2e_ms = []
     for i in range(args.e2e_steps + 1):
         if dist is not None:
             dist.barrier()
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
-        ctx.load_batch(cq, cd)
-        ctx.filter(args.levels, neighbor_support=args.ns)
-        tot = ctx.join(sigmo.SIGMO_FIND_ALL, total=True)  # D2H of the per-query totals
+        tot = runner.run(subs)  # D2H of the per-query totals
         dt = (time.perf_counter() - t0) * 1000
         if i > 0:
             e2e_ms.append(dt)
-        assert tot == matches_local
-    h2d = ctx.timings()["h2d_bytes"]
+        assert int(tot.sum()) == matches_local
+    runner.close()
 
     # ---- reduce over ranks (sharded.rank_reduce: times MAX, counts SUM) ----
     ctx.check()  # the device-pointer totals path never synchronized: check the join's capacities once
@@ -482,8 +492,11 @@ def main():
         "e2e": {"value": matches * args.e2e_steps / (e2e_total / 1000.0), "unit": "matches/s",
                 "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": 8 * NQ,
                 "ms_per_step": e2e_total / args.e2e_steps,
-                "note": "sigmo_load_batch from pinned host arrays (H2D of the raw CSR-GO arrays, validation + packing "
-                        "on the device) + filter + join + D2H of the totals, wall clock"},
+                "batches_per_step": nb_e2e,
+                "note": f"StreamRunner.run over the step's molecules in {nb_e2e} pinned host batches: per batch "
+                        "sigmo_load_batch (H2D of the raw CSR-GO arrays, validation + packing on the device) + "
+                        "filter + join on one of two double-buffered contexts (the next batch's copy overlaps), "
+                        "then the D2H of the per-query totals; wall clock"},
         "gpu_launches": int(K * (tim["filter_launches"] + tim["join_launches"])),
         "clocks": clocks,
         "roofline": roofline,

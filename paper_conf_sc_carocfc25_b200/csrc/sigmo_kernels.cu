@@ -2278,6 +2278,12 @@ __device__ __forceinline__ uint2 lds_u2(unsigned a) {
 #ifndef SIGMO_JL_MAXNREG
 #define SIGMO_JL_MAXNREG 56
 #endif
+#ifndef JL_PRED
+#define JL_PRED 0
+#endif
+#ifndef JL_SPLIT
+#define JL_SPLIT 0
+#endif
 template <int MODE, bool W64, bool PS>
 __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_JL_MAXNREG) k_join_lane(const __grid_constant__ JoinParams jp) {
   using MT = typename std::conditional<W64, unsigned long long, unsigned>::type;
@@ -2301,11 +2307,29 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   const unsigned oRec = wbase;                              // pair records of chunk buffer b: oRec + 16 kJoinChunk b
   const unsigned oNx = wbase + 32u * kJoinChunk + 16u * lane;  // record of the lane's next pair
   const unsigned oNp = wbase + 32u * kJoinChunk + 512u + 4u * lane;  // its index
-  const unsigned oRU = wbase + 32u * kJoinChunk + 640u + ES * lane;  // {R, U} of depth d: oRU + 32 ES d
-  const unsigned mA = oRU - ES * lane + 32u * ES * SD + 4u * lane;  // map word of depth d: mA + 128 d (slot SD: absent)
+#if JL_SPLIT
+  // stack depth d: R_d of the 32 lanes, then U_d of the 32 lanes (one wavefront per 32-bit access)
+  constexpr unsigned LS = sizeof(MT);  // lane stride of a stack array
+#else
+  constexpr unsigned LS = ES;  // {R, U} interleaved per lane
+#endif
+  const unsigned oRU = wbase + 32u * kJoinChunk + 640u + LS * lane;  // stack entry of depth d: oRU + 32 ES d
+  const unsigned mA = oRU - LS * lane + 32u * ES * SD + 4u * lane;  // map word of depth d: mA + 128 d (slot SD: absent)
   // stack entry {R, U} at byte offset o of the kernel's shared memory (macros,
   // not lambdas: a captured `smem` loses its address space and every access
   // would re-derive the shared window)
+#if JL_SPLIT
+#define JL_LDRU(o, r, u)                                    \
+  do {                                                      \
+    r = *(const MT *)(smem + (o));                          \
+    u = *(const MT *)(smem + (o) + 32u * sizeof(MT));       \
+  } while (0)
+#define JL_STRU(o, r, u)                                    \
+  do {                                                      \
+    *(MT *)(smem + (o)) = (MT)(r);                          \
+    *(MT *)(smem + (o) + 32u * sizeof(MT)) = (MT)(u);       \
+  } while (0)
+#else
 #define JL_LDRU(o, r, u)                                           \
   do {                                                             \
     if (W64) {                                                     \
@@ -2323,6 +2347,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     if (W64) *(ulonglong2 *)(smem + (o)) = make_ulonglong2((unsigned long long)(r), (unsigned long long)(u));      \
     else *(uint2 *)(smem + (o)) = make_uint2((unsigned)(r), (unsigned)(u));                                        \
   } while (0)
+#endif
 #define JL_MAP(d) (*(unsigned *)(smem + mA + 128u * (unsigned)(d)))
   auto popc = [](MT x) -> int { return W64 ? __popcll((unsigned long long)x) : __popc((unsigned)x); };
   auto highest = [](MT x) -> unsigned {  // index of the highest set bit (x != 0)
@@ -2461,12 +2486,27 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
       if (!Rn) ne ^= 1u << d;
       // map word of depth d = the adjacency index of f(pi_d); stored before the
       // back-edge slots are read, so a back-edge to d reads it
+#if JL_PRED
+      // back-edges to d take the popped node's word directly; the map slots are read (and
+      // the second adjacency word loaded) only when needed
+      const unsigned Av = ca + (v << sw);
+      JL_MAP(d) = Av;
+      const unsigned s0 = en.x & 0x7ffu, s1 = en.x >> 16, sd = 128u * d;
+      unsigned a0 = Av, a1 = Av;
+      if (s0 != sd) a0 = *(const unsigned *)(smem + mA + s0);
+      if (s1 != sd) a1 = *(const unsigned *)(smem + mA + s1);
+      const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
+      const MT used = U | bit;
+      MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0);
+      if (s1 != 128u * (unsigned)SD) X &= adj(i1);
+#else
       JL_MAP(d) = ca + (v << sw);
       const unsigned a0 = *(const unsigned *)(smem + mA + (en.x & 0x7ffu));
       const unsigned a1 = *(const unsigned *)(smem + mA + (en.x >> 16));
       const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
       const MT used = U | bit;
       MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0) & adj(i1);
+#endif
       if (en.x & 0xf000u) {  // > 2 back-edges at this depth (fused rings): rare
         const unsigned nex = (en.x >> 12) & 15u;
         const unsigned b0 = (unsigned)__ldg(&jp.qp_ent[cqb_of(pe) + d + 1u]).w;
@@ -2601,10 +2641,10 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
         }
         __syncwarp();
         if (recv) {
-          const unsigned dl = (unsigned)(src - lane);  // donor offsets = mine + dl * (ES | 4)
+          const unsigned dl = (unsigned)(src - lane);  // donor offsets = mine + dl * (LS | 4)
           {
             MT r, u;
-            JL_LDRU(oRU + 32u * ES * ds + ES * dl, r, u);
+            JL_LDRU(oRU + 32u * ES * ds + LS * dl, r, u);
             JL_STRU(oRU + 32u * ES * ds, r, u);
           }
           for (int j = 0; j < ds; j++) JL_MAP(j) = *(const unsigned *)(smem + mA + 128u * j + 4u * dl);

@@ -1,11 +1,12 @@
 """Streamed batches (10M molecules in batches of 250k per
 GPU) and query-size routing, above the C ABI.
 
-Data batches go through two contexts used alternately, each on its own CUDA
-stream: while the GPU runs filter + join of batch i in one context, the host
-validates/packs batch i+1 (``sigmo_load_batch``) into the other and its H2D
-copy overlaps the kernels of batch i.  Per-query totals are accumulated on
-the device (int64 adds on the context's stream) and read back once.
+Data batches go through three contexts used in turn, each on its own CUDA
+stream and driven from its own host thread: while the GPU runs filter + join
+of batch i in one context, batch i+1 is loaded (``sigmo_load_batch``: H2D
+copy, device validation and packing) into the next one, so the copies
+overlap the kernels of batch i.  Per-query totals are accumulated on the
+device (int64 adds on the context's stream) and read back once.
 
 Query routing: the per-lane join (``k_join_lane``) handles queries of at most
 ``LANE_MAX_QUERY_NODES`` nodes; a query set with larger ones (the 20-30-atom
@@ -71,12 +72,15 @@ def split_queries(Q, max_nodes: int = LANE_MAX_QUERY_NODES) -> List[np.ndarray]:
 
 
 class StreamRunner:
-    """Run the hot path over a sequence of data batches with double-buffered
-    contexts; ``run`` returns the per-query totals (uint64 [NQ], original
-    query order) summed over all batches."""
+    """Run the hot path over a sequence of data batches with ``buffers``
+    rotating contexts (each on its own stream; 3 by default, so a batch's copy
+    never waits for the join of the batch two earlier, which still owns the
+    previous buffer); ``run`` returns the per-query totals (uint64 [NQ],
+    original query order) summed over all batches."""
 
     def __init__(self, queries, device: int = 0, levels: int = 4, mode: int = SIGMO_FIND_ALL,
-                 split: bool = True, levels_large: Optional[int] = None):
+                 split: bool = True, levels_large: Optional[int] = None, induced: bool = False,
+                 neighbor_support: bool = False, buffers: int = 3):
         import torch
         self.torch = torch
         self.device = device
@@ -93,12 +97,24 @@ class StreamRunner:
             self.groups = [(g, _subset(queries, g)) for g in groups]
         dev = torch.device("cuda", device)
         self.dev = dev
-        self.streams = [torch.cuda.Stream(dev) for _ in range(2)]
+        self.nbuf = max(2, int(buffers))
+        self.streams = [torch.cuda.Stream(dev) for _ in range(self.nbuf)]
         # contexts[buffer][group]
-        self.ctx = [[Context(device, self.streams[b]) for _ in self.groups] for b in range(2)]
+        self.ctx = [[Context(device, self.streams[b]) for _ in self.groups] for b in range(self.nbuf)]
+        self.neighbor_support = neighbor_support
+        from concurrent.futures import ThreadPoolExecutor
+        self.pool = ThreadPoolExecutor(self.nbuf)
+        import threading
+        self.copy_lock = threading.Lock()
+        if induced:  # DESIGN.md R21 (set before the first load_batch)
+            for row in self.ctx:
+                for c in row:
+                    c.set_induced(True)
         # accumulators per buffer (each only touched on its own stream)
-        self.acc = [[torch.zeros(len(g), dtype=torch.int64, device=dev) for g, _ in self.groups] for _ in range(2)]
-        self.tmp = [[torch.zeros(len(g), dtype=torch.int64, device=dev) for g, _ in self.groups] for _ in range(2)]
+        self.acc = [[torch.zeros(len(g), dtype=torch.int64, device=dev) for g, _ in self.groups]
+                    for _ in range(self.nbuf)]
+        self.tmp = [[torch.zeros(len(g), dtype=torch.int64, device=dev) for g, _ in self.groups]
+                    for _ in range(self.nbuf)]
         self.batches_done = 0
         cur = torch.cuda.current_stream(dev)
         for st in self.streams:  # the buffers above were zeroed on the current stream
@@ -117,21 +133,29 @@ class StreamRunner:
 
     def submit(self, data):
         """Enqueue one data batch (host GraphBatch or as_c_batch) on the next buffer."""
+        b = self.batches_done % self.nbuf
+        self._submit_on(b, data)
+        self.batches_done += 1
+
+    def _submit_on(self, b: int, data):
         torch = self.torch
-        b = self.batches_done & 1
+        torch.cuda.set_device(self.dev)  # worker threads start on the default device
         s = self.streams[b]
         for gi, (_, qb) in enumerate(self.groups):
             c = self.ctx[b][gi]
-            c.load_batch(qb, data)  # waits only for this buffer's previous H2D
-            c.filter(self.group_levels(gi))
+            # load + filter of one batch at a time: their host-to-device copies go
+            # through one copy engine in submission order, so the next batch's
+            # large copies must not be queued ahead of this batch's small ones
+            with self.copy_lock:
+                c.load_batch(qb, data)  # waits only for this buffer's previous H2D
+                c.filter(self.group_levels(gi), neighbor_support=self.neighbor_support)
             c.join(self.mode, total=False)
             c.query_totals(device_tensor=self.tmp[b][gi])
             with torch.cuda.stream(s):
                 self.acc[b][gi].add_(self.tmp[b][gi])
-        self.batches_done += 1
 
     def totals(self) -> np.ndarray:
-        """Synchronise both buffers and gather the totals in query order."""
+        """Synchronise all buffers and gather the totals in query order."""
         torch = self.torch
         for s in self.streams:
             s.synchronize()
@@ -145,16 +169,30 @@ class StreamRunner:
                             raise
         out = np.zeros(self.nq, np.uint64)
         for gi, (idx, _) in enumerate(self.groups):
-            out[idx] = (self.acc[0][gi] + self.acc[1][gi]).cpu().numpy().astype(np.uint64)
+            out[idx] = sum(self.acc[b][gi] for b in range(self.nbuf)).cpu().numpy().astype(np.uint64)
         return out
 
     def run(self, batches: Iterable) -> np.ndarray:
+        """All batches, the two buffers driven from two host threads: a buffer's
+        sigmo_load_batch (copy, device validation, layout read-back) and filter
+        proceed while the other buffer's join runs, so the copies overlap the
+        kernels (the library releases the GIL in every call; the two contexts
+        share nothing)."""
         self.reset()
+        futs = [None] * self.nbuf
         for d in batches:
-            self.submit(d)
+            b = self.batches_done % self.nbuf
+            if futs[b] is not None:
+                futs[b].result()  # this buffer's previous batch is enqueued
+            futs[b] = self.pool.submit(self._submit_on, b, d)
+            self.batches_done += 1
+        for f in futs:
+            if f is not None:
+                f.result()
         return self.totals()
 
     def close(self):
+        self.pool.shutdown()
         for row in self.ctx:
             for c in row:
                 c.close()
