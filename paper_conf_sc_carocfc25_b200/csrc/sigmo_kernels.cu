@@ -1930,9 +1930,11 @@ int join_blocks_per_sm(int NW, int mode, const JoinParams &p, size_t smem) {
 // ===========================================================================
 __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
   const int lane = threadIdx.x & 31;
-  const int g = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (g >= pp.ND) return;
   const unsigned lt = (1u << lane) - 1u;
+  // grid-stride over graphs, one warp per graph (one block per 8 graphs was
+  // bound by block scheduling)
+  const int nwarps = (int)((gridDim.x * blockDim.x) >> 5);
+  for (int g = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5); g < pp.ND; g += nwarps) {
   // lane join: records of <= 32-node molecules first (off.a), then the others
   // at P_narrow + off.b; the general path only uses .a
   long long o = pp.off[g].a;
@@ -1963,6 +1965,7 @@ __global__ void __launch_bounds__(256) k_pairs(PairsParams pp) {
     }
     o += __popc(bits);
     oo += __popc(obits);
+  }
   }
 }
 
@@ -2121,8 +2124,8 @@ cudaError_t launch_gmcr_update(int ND, int NQW, const uint32_t *gm_old, const I6
 
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st) {
   if (p.ND <= 0) return cudaSuccess;
-  const long long threads = 32ll * p.ND;
-  k_pairs<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(p);
+  const long long blocks = std::min<long long>((32ll * p.ND + 255) / 256, 148ll * 16);
+  k_pairs<<<(unsigned)blocks, 256, 0, st>>>(p);
   return cudaGetLastError();
 }
 
@@ -2266,6 +2269,14 @@ __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
   return __ffs(m) - 1;
 }
 
+// 64-bit add to a little-endian {lo, hi} pair of shared words by 32-bit atomics
+// (a 64-bit shared atomic add is a compare-and-swap loop on sm_100)
+__device__ __forceinline__ void sh_add64(unsigned *w, unsigned long long x) {
+  const unsigned lo = (unsigned)x, old = atomicAdd(w, lo);
+  const unsigned hi = (unsigned)(x >> 32) + (old + lo < old ? 1u : 0u);
+  if (hi) atomicAdd(w + 1, hi);
+}
+
 __device__ __forceinline__ uint2 lds_u2(unsigned a) {
   uint2 v;
   asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(a));
@@ -2277,12 +2288,6 @@ __device__ __forceinline__ uint2 lds_u2(unsigned a) {
 // PS: the plan entries are copied to shared memory (VQ <= kJoinLanePlanSmemMax)
 #ifndef SIGMO_JL_MAXNREG
 #define SIGMO_JL_MAXNREG 56
-#endif
-#ifndef JL_PRED
-#define JL_PRED 0
-#endif
-#ifndef JL_SPLIT
-#define JL_SPLIT 0
 #endif
 template <int MODE, bool W64, bool PS>
 __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_JL_MAXNREG) k_join_lane(const __grid_constant__ JoinParams jp) {
@@ -2307,29 +2312,12 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   const unsigned oRec = wbase;                              // pair records of chunk buffer b: oRec + 16 kJoinChunk b
   const unsigned oNx = wbase + 32u * kJoinChunk + 16u * lane;  // record of the lane's next pair
   const unsigned oNp = wbase + 32u * kJoinChunk + 512u + 4u * lane;  // its index
-#if JL_SPLIT
-  // stack depth d: R_d of the 32 lanes, then U_d of the 32 lanes (one wavefront per 32-bit access)
-  constexpr unsigned LS = sizeof(MT);  // lane stride of a stack array
-#else
-  constexpr unsigned LS = ES;  // {R, U} interleaved per lane
-#endif
+  constexpr unsigned LS = ES;  // stack entries {R, U} interleaved per lane
   const unsigned oRU = wbase + 32u * kJoinChunk + 640u + LS * lane;  // stack entry of depth d: oRU + 32 ES d
   const unsigned mA = oRU - LS * lane + 32u * ES * SD + 4u * lane;  // map word of depth d: mA + 128 d (slot SD: absent)
   // stack entry {R, U} at byte offset o of the kernel's shared memory (macros,
   // not lambdas: a captured `smem` loses its address space and every access
   // would re-derive the shared window)
-#if JL_SPLIT
-#define JL_LDRU(o, r, u)                                    \
-  do {                                                      \
-    r = *(const MT *)(smem + (o));                          \
-    u = *(const MT *)(smem + (o) + 32u * sizeof(MT));       \
-  } while (0)
-#define JL_STRU(o, r, u)                                    \
-  do {                                                      \
-    *(MT *)(smem + (o)) = (MT)(r);                          \
-    *(MT *)(smem + (o) + 32u * sizeof(MT)) = (MT)(u);       \
-  } while (0)
-#else
 #define JL_LDRU(o, r, u)                                           \
   do {                                                             \
     if (W64) {                                                     \
@@ -2347,7 +2335,6 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     if (W64) *(ulonglong2 *)(smem + (o)) = make_ulonglong2((unsigned long long)(r), (unsigned long long)(u));      \
     else *(uint2 *)(smem + (o)) = make_uint2((unsigned)(r), (unsigned)(u));                                        \
   } while (0)
-#endif
 #define JL_MAP(d) (*(unsigned *)(smem + mA + 128u * (unsigned)(d)))
   auto popc = [](MT x) -> int { return W64 ? __popcll((unsigned long long)x) : __popc((unsigned)x); };
   auto highest = [](MT x) -> unsigned {  // index of the highest set bit (x != 0)
@@ -2486,27 +2473,12 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
       if (!Rn) ne ^= 1u << d;
       // map word of depth d = the adjacency index of f(pi_d); stored before the
       // back-edge slots are read, so a back-edge to d reads it
-#if JL_PRED
-      // back-edges to d take the popped node's word directly; the map slots are read (and
-      // the second adjacency word loaded) only when needed
-      const unsigned Av = ca + (v << sw);
-      JL_MAP(d) = Av;
-      const unsigned s0 = en.x & 0x7ffu, s1 = en.x >> 16, sd = 128u * d;
-      unsigned a0 = Av, a1 = Av;
-      if (s0 != sd) a0 = *(const unsigned *)(smem + mA + s0);
-      if (s1 != sd) a1 = *(const unsigned *)(smem + mA + s1);
-      const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
-      const MT used = U | bit;
-      MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0);
-      if (s1 != 128u * (unsigned)SD) X &= adj(i1);
-#else
       JL_MAP(d) = ca + (v << sw);
       const unsigned a0 = *(const unsigned *)(smem + mA + (en.x & 0x7ffu));
       const unsigned a1 = *(const unsigned *)(smem + mA + (en.x >> 16));
       const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
       const MT used = U | bit;
       MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0) & adj(i1);
-#endif
       if (en.x & 0xf000u) {  // > 2 back-edges at this depth (fused rings): rare
         const unsigned nex = (en.x >> 12) & 15u;
         const unsigned b0 = (unsigned)__ldg(&jp.qp_ent[cqb_of(pe) + d + 1u]).w;
@@ -2545,14 +2517,14 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
       if (MODE & 1) {
         if (!shared) {
           presult[cp] = cnt ? 1ull : 0ull;
-          if (cnt) atomicAdd((unsigned long long *)(smem + o_tot) + cq, 1ull);
+          if (cnt) sh_add64((unsigned *)(smem + o_tot) + 2 * cq, 1ull);
         } else if (cnt) {
-          if (atomicOr(&presult[cp], 1ull) == 0ull) atomicAdd((unsigned long long *)(smem + o_tot) + cq, 1ull);
+          if (atomicOr(&presult[cp], 1ull) == 0ull) sh_add64((unsigned *)(smem + o_tot) + 2 * cq, 1ull);
         }
       } else {
         if (!shared) presult[cp] = cnt;
         else if (cnt) atomicAdd(&presult[cp], cnt);
-        if (cnt) atomicAdd((unsigned long long *)(smem + o_tot) + cq, cnt);
+        if (cnt) sh_add64((unsigned *)(smem + o_tot) + 2 * cq, cnt);
       }
       pend = false;
     }
