@@ -2242,15 +2242,13 @@ cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const
 //   * Per-query totals are reduced in shared memory (one global atomic per
 //     query per CTA).
 // ===========================================================================
-constexpr int kJoinChunk = 16;    // GMCR pair records per warp buffer (copied to shared memory by lanes 0..15)
 constexpr int kJoinClaim = 128;   // GMCR pairs per warp claim (atomic on the launch's pair counter)
 
 // stack entry {R, U}: 2 x 32-bit masks (<= 32-node molecules) or 2 x 64-bit
 __host__ __device__ inline size_t join_lane_warp_bytes(int MQ, bool w64) {
   const int SD = MQ > 1 ? MQ - 1 : 1;  // pushed depths 0..n-2
-  // pair records [2][kJoinChunk] (current and next chunk) | next pair per lane: record [32] int4, index [32] |
   // {R, U} [SD][32] (8 or 16 B) | map words [SD + 1][32] (u32: adjacency index of f(pi_d); slot SD: all ones)
-  return 2 * 16 * (size_t)kJoinChunk + 16 * 32 + 4 * 32 + 32 * (size_t)(w64 ? 16 : 8) * SD + 128 * (size_t)(SD + 1);
+  return 32 * (size_t)(w64 ? 16 : 8) * SD + 128 * (size_t)(SD + 1);
 }
 // CTA: per-query totals [NQ] u64, then one region per warp
 // CTA: per-query totals [NQ] u64, then (optionally) the plan entries [VQ] uint2
@@ -2275,6 +2273,31 @@ __device__ __forceinline__ void sh_add64(unsigned *w, unsigned long long x) {
   const unsigned lo = (unsigned)x, old = atomicAdd(w, lo);
   const unsigned hi = (unsigned)(x >> 32) + (old + lo < old ? 1u : 0u);
   if (hi) atomicAdd(w + 1, hi);
+}
+
+// shared-space accesses at 32-bit shared addresses (volatile: kept in program
+// order among themselves; stores are compiler memory barriers)
+__device__ __forceinline__ unsigned lds32(unsigned a) {
+  unsigned v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ void sts32(unsigned a, unsigned v) { asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory"); }
+__device__ __forceinline__ void lds_pair(unsigned a, unsigned &x, unsigned &y) {
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(a));
+}
+__device__ __forceinline__ void lds_pair(unsigned a, unsigned long long &x, unsigned long long &y) {
+  asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(x), "=l"(y) : "r"(a));
+}
+__device__ __forceinline__ void sts_pair(unsigned a, unsigned x, unsigned y) {
+  asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(a), "r"(x), "r"(y) : "memory");
+}
+__device__ __forceinline__ void sts_pair(unsigned a, unsigned long long x, unsigned long long y) {
+  asm volatile("st.shared.v2.u64 [%0], {%1, %2};" ::"r"(a), "l"(x), "l"(y) : "memory");
+}
+__device__ __forceinline__ void sts_mask(unsigned a, unsigned x) { asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(x) : "memory"); }
+__device__ __forceinline__ void sts_mask(unsigned a, unsigned long long x) {
+  asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(x) : "memory");
 }
 
 __device__ __forceinline__ uint2 lds_u2(unsigned a) {
@@ -2309,33 +2332,17 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   const unsigned sbase = (unsigned)__cvta_generic_to_shared(smem);
 #define JL_PLAN(p) (PS ? lds_u2(p) : __ldg(&jp.qp_ent2[(p)]))
   const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ, jp.VQ, jp.plan_smem_max) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
-  const unsigned oRec = wbase;                              // pair records of chunk buffer b: oRec + 16 kJoinChunk b
-  const unsigned oNx = wbase + 32u * kJoinChunk + 16u * lane;  // record of the lane's next pair
-  const unsigned oNp = wbase + 32u * kJoinChunk + 512u + 4u * lane;  // its index
   constexpr unsigned LS = ES;  // stack entries {R, U} interleaved per lane
-  const unsigned oRU = wbase + 32u * kJoinChunk + 640u + LS * lane;  // stack entry of depth d: oRU + 32 ES d
+  const unsigned oRU = wbase + LS * lane;  // stack entry of depth d: oRU + 32 ES d
   const unsigned mA = oRU - LS * lane + 32u * ES * SD + 4u * lane;  // map word of depth d: mA + 128 d (slot SD: absent)
-  // stack entry {R, U} at byte offset o of the kernel's shared memory (macros,
-  // not lambdas: a captured `smem` loses its address space and every access
-  // would re-derive the shared window)
-#define JL_LDRU(o, r, u)                                           \
-  do {                                                             \
-    if (W64) {                                                     \
-      const ulonglong2 x_ = *(const ulonglong2 *)(smem + (o));     \
-      r = (MT)x_.x;                                                \
-      u = (MT)x_.y;                                                \
-    } else {                                                       \
-      const uint2 x_ = *(const uint2 *)(smem + (o));               \
-      r = (MT)x_.x;                                                \
-      u = (MT)x_.y;                                                \
-    }                                                              \
-  } while (0)
-#define JL_STRU(o, r, u)                                                                                           \
-  do {                                                                                                             \
-    if (W64) *(ulonglong2 *)(smem + (o)) = make_ulonglong2((unsigned long long)(r), (unsigned long long)(u));      \
-    else *(uint2 *)(smem + (o)) = make_uint2((unsigned)(r), (unsigned)(u));                                        \
-  } while (0)
-#define JL_MAP(d) (*(unsigned *)(smem + mA + 128u * (unsigned)(d)))
+  // stack entry {R, U} and map word of depth d at 32-bit shared addresses
+  // (explicit ld/st.shared: generic smem + offset accesses re-derive the
+  // shared window every step)
+  const unsigned sRU = sbase + oRU, sMA = sbase + mA;
+#define JL_LDRU(a, r, u) lds_pair((a), r, u)
+#define JL_STRU(a, r, u) sts_pair((a), (MT)(r), (MT)(u))
+#define JL_MAPR(d) lds32(sMA + 128u * (unsigned)(d))
+#define JL_MAPW(d, x) sts32(sMA + 128u * (unsigned)(d), (x))
   auto popc = [](MT x) -> int { return W64 ? __popcll((unsigned long long)x) : __popc((unsigned)x); };
   auto highest = [](MT x) -> unsigned {  // index of the highest set bit (x != 0)
     unsigned r;
@@ -2351,7 +2358,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   auto lowest = [](MT x) -> unsigned {  // index of the lowest set bit (x != 0)
     return W64 ? (unsigned)(__ffsll((long long)x) - 1) : (unsigned)(__ffs((unsigned)x) - 1);
   };
-  JL_MAP(SD) = jp.adj_ones;  // absent back-edges read the all-ones entry (class field 0)
+  JL_MAPW(SD, jp.adj_ones);  // absent back-edges read the all-ones entry (class field 0)
   __syncthreads();
 
   const unsigned lt = (1u << lane) - 1u;
@@ -2361,7 +2368,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   const long long pbase0 = W64 ? ptot.a : 0;
   const int4 *const recs = jp.prec + pbase0;
   unsigned long long *const presult = jp.pair_result + pbase0;
-  unsigned *const cursor = (unsigned *)jp.chunk_counter;
+  unsigned *const counter = (unsigned *)jp.chunk_counter;
   const uint32_t *const adjw = jp.adjw;
   // mask of adjacency word index i (entries of 1 or 2 words)
   auto adj = [&](unsigned i) -> MT {
@@ -2380,35 +2387,20 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   // plan position of depth 0 of the pair whose depth-1 plan address is a
   auto cqb_of = [&](unsigned a) -> unsigned { return PS ? (a - sbase - o_plan) / 8u - 1u : a - 1u; };
 
-  // ---- GMCR chunks of kJoinChunk pairs: the current one (cbase, chead taken) and the next, claimed a
-  // chunk ahead; their records are copied into the warp's two record buffers by cp.async (no registers,
-  // no stall: a buffer is waited for one chunk after its copy was issued) ----
-  const unsigned srec = sbase + oRec + 16u * lane;
-  auto fetch_chunk = [&](unsigned base, unsigned buf) {
-    if (lane < kJoinChunk && base + lane < P)
-      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(srec + 16u * kJoinChunk * buf), "l"(recs + base + lane)
-                   : "memory");
-    asm volatile("cp.async.commit_group;\n" ::: "memory");
-  };
-  // the warp claims blocks of kJoinClaim pairs (one same-address atomic per block: at one atomic per chunk the
-  // counter serialised the launch), a block ahead; lane 0 holds the next block's start until it is needed
-  unsigned cbase, pbase, pnext, bend, cbuf = 0u, bnext0 = 0u;
+  // ---- the warp's pairs: blocks of kJoinClaim consecutive GMCR pairs claimed by one same-address
+  // atomic per block (one atomic per chunk of 32 serialised the launch on the counter), a block ahead;
+  // lane 0 holds the pre-claimed block's start until it is needed.  Warp-uniform: cursor = the next
+  // pair to hand out, bend = the end of its block ----
+  unsigned cursor, bend, bnext0 = 0u;
   {
     unsigned x = 0u;
-    if (lane == 0) x = atomicAdd(cursor, 2u * kJoinClaim);
+    if (lane == 0) x = atomicAdd(counter, 2u * kJoinClaim);
     x = __shfl_sync(FULL_MASK, x, 0);
-    cbase = x;
-    pbase = x + kJoinChunk;
-    pnext = x + 2u * kJoinChunk;
+    cursor = x;
     bend = x + kJoinClaim;
     bnext0 = x + kJoinClaim;
-    fetch_chunk(cbase, 0u);
-    fetch_chunk(pbase, 1u);
-    asm volatile("cp.async.wait_group 1;\n" ::: "memory");  // the current chunk
-    __syncwarp();
   }
-  unsigned ccount = cbase < P ? min(P - cbase, (unsigned)kJoinChunk) : 0u, chead = 0u;
-  bool drained = ccount == 0u;
+  bool drained = cursor >= P;
   int keff = jp.batchK;  // free lanes that end a stepping phase (1 once the list is drained)
   if (drained) keff = 1;
 
@@ -2422,7 +2414,10 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   int cq = 0;
   unsigned long long cnt = 0ull;
   unsigned steps = 0u;
-  bool nv = false;  // next pair assigned (record and index in the lane's slots, root window in flight)
+  bool nv = false;  // next pair assigned (its record in registers)
+  bool nr = false;  // and the load of its root window issued (the refill pass after the record's)
+  int4 nrec = make_int4(0, 0, 0, 0);
+  unsigned nidx = 0u;
   MT nR0 = 0;
 
   // enumerate mode: the embeddings of a leaf step -- the
@@ -2435,7 +2430,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     unsigned long long r0 = 0ull, r1 = 0ull;
     for (int j = 0; j <= d; j++) {
       const unsigned qn = __ldg(&jp.qp_qn[cqb + (unsigned)j]);
-      const unsigned long long b = (JL_MAP(j) - ca) >> sw;
+      const unsigned long long b = (JL_MAPR(j) - ca) >> sw;
       if (qn < 8u) r0 |= b << (8u * qn);
       else r1 |= b << (8u * (qn - 8u));
     }
@@ -2460,7 +2455,8 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     // ---- one DFS step ----
     if (ne) {
       const unsigned d = bfind32(ne);  // deepest open depth
-      const unsigned od = oRU + 32u * ES * d;
+      const unsigned bd = 1u << d;
+      const unsigned od = sRU + 32u * ES * d;
       // plan entry of depth e = d + 1 (x: back-edge map slots, leaf, #extra;
       // y: bond classes, distinct row)
       const uint2 en = JL_PLAN(pe + PSTEP * d);
@@ -2469,13 +2465,13 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
       const unsigned v = highest(R);
       const MT bit = (MT)1 << v;
       const MT Rn = R ^ bit;
-      *(MT *)(smem + od) = Rn;
-      if (!Rn) ne ^= 1u << d;
+      sts_mask(od, Rn);
+      ne ^= Rn ? 0u : bd;
       // map word of depth d = the adjacency index of f(pi_d); stored before the
       // back-edge slots are read, so a back-edge to d reads it
-      JL_MAP(d) = ca + (v << sw);
-      const unsigned a0 = *(const unsigned *)(smem + mA + (en.x & 0x7ffu));
-      const unsigned a1 = *(const unsigned *)(smem + mA + (en.x >> 16));
+      JL_MAPW(d, ca + (v << sw));
+      const unsigned a0 = lds32(sMA + (en.x & 0x7ffu));
+      const unsigned a1 = lds32(sMA + (en.x >> 16));
       const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
       const MT used = U | bit;
       MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0) & adj(i1);
@@ -2485,7 +2481,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
 #pragma unroll 1
         for (unsigned k = 0; k < nex; k++) {
           const unsigned be = __ldg(&jp.qp_be[b0 + k]);
-          X &= adj((be & 255u) * ngs + JL_MAP(be >> 8));
+          X &= adj((be & 255u) * ngs + JL_MAPR(be >> 8));
         }
       }
       if (MODE & 2) {  // induced mode (R21): drop neighbours (any bond) of mapped non-adjacent depths
@@ -2493,9 +2489,9 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
         // two depths per iteration (the second reads the all-zeros entry when absent)
 #pragma unroll 1
         for (unsigned nm = __ldg(&jp.qp_non[cqb_of(pe) + d + 1u]); nm;) {
-          const unsigned ia = cn + JL_MAP(__ffs(nm) - 1);
+          const unsigned ia = cn + JL_MAPR(__ffs(nm) - 1);
           nm &= nm - 1u;
-          const unsigned ib = nm ? cn + JL_MAP(__ffs(nm) - 1) : jp.adj_ones + 2u;
+          const unsigned ib = nm ? cn + JL_MAPR(__ffs(nm) - 1) : jp.adj_ones + 2u;
           nm &= nm - 1u;
           X &= ~(adj(ia) | adj(ib));
         }
@@ -2506,7 +2502,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
         if ((MODE & 1) && X) ne = 0u;  // Find First: the pair (part) is decided
       } else if (X) {
         JL_STRU(od + 32u * ES, X, used);
-        ne += 2u << d;  // bit d + 1 is clear: d is the deepest open depth
+        ne += bd + bd;  // bit d + 1 is clear: d is the deepest open depth
       }
       steps++;
     }
@@ -2530,8 +2526,8 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     }
     // ---- free lanes activate their prefetched next pair ----
     if (ne == 0u && nv) {
-      const int4 nrec = *(const int4 *)(smem + oNx);
-      cp = *(const unsigned *)(smem + oNp);
+      if (!nr) nR0 = cand((unsigned)nrec.z + ((JL_PLAN(paddr((unsigned)nrec.w >> 16)).y >> 12) << sw));
+      cp = nidx;
       cmb = (unsigned)nrec.z;
       ca = (unsigned)nrec.x;  // adjacency word offset of the molecule
       cq = nrec.y;
@@ -2545,49 +2541,43 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
         cnt = (unsigned long long)popc(R0);
         if ((MODE & 4) && R0) emit(R0, -1, (MT)0);
       } else {
-        JL_STRU(oRU, R0, (MT)0);
+        JL_STRU(sRU, R0, (MT)0);
         ne = R0 ? 1u : 0u;
       }
       nv = false;
     }
-    // ---- lanes without a next pair take one from the chunk and prefetch its root window ----
-    unsigned wm = __ballot_sync(FULL_MASK, !nv && !drained);
-    while (wm) {
-      const unsigned avail = ccount - chead;
-      const unsigned n = (unsigned)__popc(wm);
-      const unsigned take = min(n, avail);
-      const unsigned rank = (unsigned)__popc(wm & lt);
-      const bool mine = ((wm >> lane) & 1u) && rank < take;
-      if (mine) {
-        const int4 nrec = *(const int4 *)(smem + oRec + 16u * kJoinChunk * cbuf + 16u * (chead + rank));
-        *(int4 *)(smem + oNx) = nrec;
-        *(unsigned *)(smem + oNp) = cbase + chead + rank;
-        nv = true;
-        // root candidates of the next pair: the loads complete while the current pair runs
-        nR0 = cand((unsigned)nrec.z + ((JL_PLAN(paddr((unsigned)nrec.w >> 16)).y >> 12) << sw));
+    // ---- root window of the next pair, its record loaded a pass ago ----
+    if (nv && !nr) {
+      nR0 = cand((unsigned)nrec.z + ((JL_PLAN(paddr((unsigned)nrec.w >> 16)).y >> 12) << sw));
+      nr = true;
+    }
+    // ---- lanes without a next pair take the next ones of the warp's blocks: record and root window
+    // are loaded now and used when the current pair ends ----
+    if (!drained) {
+      const unsigned f = __ballot_sync(FULL_MASK, !nv);
+      const unsigned n = (unsigned)__popc(f), rank = (unsigned)__popc(f & lt);
+      const unsigned left = bend - cursor;  // >= 1
+      unsigned bn = 0u;
+      if (n >= left) {  // the pass reaches the pre-claimed block: claim the one after it
+        bn = __shfl_sync(FULL_MASK, bnext0, 0);
+        if (lane == 0) bnext0 = atomicAdd(counter, (unsigned)kJoinClaim);
       }
-      chead += take;
-      wm = __ballot_sync(FULL_MASK, !nv) & wm;
-      if (chead == ccount) {  // chunk exhausted: switch to the prefetched one, claim the one after
-        cbase = pbase;
-        ccount = cbase < P ? min(P - cbase, (unsigned)kJoinChunk) : 0u;
-        chead = 0u;
-        if (ccount == 0u) {
-          drained = true;
-          keff = 1;
-          break;
-        }
-        asm volatile("cp.async.wait_all;\n" ::: "memory");  // the next chunk (issued a chunk ago)
-        __syncwarp();
-        cbuf ^= 1u;
-        if (pnext == bend) {  // the block is scheduled: continue with the claimed one, claim the one after
-          pnext = __shfl_sync(FULL_MASK, bnext0, 0);
-          bend = pnext + kJoinClaim;
-          if (lane == 0) bnext0 = atomicAdd(cursor, (unsigned)kJoinClaim);
-        }
-        pbase = pnext;
-        pnext += kJoinChunk;
-        fetch_chunk(pbase, cbuf ^ 1u);  // into the buffer just emptied
+      const unsigned idx = rank < left ? cursor + rank : bn + (rank - left);
+      if (((f >> lane) & 1u) && idx < P) {
+        nrec = __ldg(recs + idx);
+        nidx = idx;
+        nv = true;
+        nr = false;
+      }
+      if (n >= left) {
+        cursor = bn + (n - left);
+        bend = bn + kJoinClaim;
+      } else {
+        cursor += n;
+      }
+      if (cursor >= P) {
+        drained = true;
+        keff = 1;
       }
     }
     // ---- drained: idle lanes take the shallowest open depth of a busy lane ----
@@ -2616,10 +2606,10 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
           const unsigned dl = (unsigned)(src - lane);  // donor offsets = mine + dl * (LS | 4)
           {
             MT r, u;
-            JL_LDRU(oRU + 32u * ES * ds + LS * dl, r, u);
-            JL_STRU(oRU + 32u * ES * ds, r, u);
+            JL_LDRU(sRU + 32u * ES * ds + LS * dl, r, u);
+            JL_STRU(sRU + 32u * ES * ds, r, u);
           }
-          for (int j = 0; j < ds; j++) JL_MAP(j) = *(const unsigned *)(smem + mA + 128u * j + 4u * dl);
+          for (int j = 0; j < ds; j++) JL_MAPW(j, lds32(sMA + 128u * j + 4u * dl));
           cmb = s_cmb;
           cp = s_cp;
           cq = s_cq;
@@ -2637,7 +2627,6 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     }
     if (drained && __ballot_sync(FULL_MASK, ne != 0u || nv || pend) == 0u) break;
   }
-  asm volatile("cp.async.wait_all;\n" ::: "memory");  // no copy in flight into the CTA's shared memory at exit
   if (jp.stats) {
     unsigned long long s2 = steps;
 #pragma unroll
@@ -2652,7 +2641,8 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
 #undef JL_LDRU
 #undef JL_STRU
 #undef JL_PLAN
-#undef JL_MAP
+#undef JL_MAPR
+#undef JL_MAPW
 }
 
 // dynamic shared memory size and (optionally) the preferred shared-memory carveout of a k_join_lane instantiation
