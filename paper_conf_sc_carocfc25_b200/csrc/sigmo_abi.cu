@@ -2050,9 +2050,9 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
       jp.qp_ent2 = (const uint2 *)(c->lane_ns ? c->ent_ns.p : c->ent2.p);
       jp.cmol = (const uint32_t *)c->bitmap.p;
       // refill batch (lanes that must be free before a warp refills): swept on
-      // configs[2] (r1 final kernel), FA 6/8/12/16 -> 8.70/8.61/8.81/9.42 ms,
-      // FF 7.43/7.27/7.18/7.29 ms
-      jp.batchK = mode == SIGMO_FIND_FIRST ? 12 : 8;
+      // configs[2] (r2 kernel with registers-only pair hand-out), FA 4/6/8/10/12
+      // -> 5.91/5.58/5.42/5.35/5.34 ms join
+      jp.batchK = 12;
       jp.emaps = eo.emaps;
       jp.estride = eo.estride;
       jp.esets = eo.esets;
@@ -2099,6 +2099,10 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
         CUDA_TRY(c, cudaEventRecord(c->join_ev, c->aux));
         CUDA_TRY(c, cudaStreamWaitEvent(c->stream, c->join_ev, 0));
       }
+      // S7: per-query totals from the pair results
+      CUDA_TRY(c, launch_lane_totals(c->ND, c->NQ, c->NQW, (const uint32_t *)c->gm.p, (const I64x2 *)c->off.p,
+                                     jp.pair_result, jp.totals, c->sm_count, c->stream));
+      launches++;
       timing_join(c, 1);
     } else {
       const size_t smem = join_smem_bytes(c->NW, jp);

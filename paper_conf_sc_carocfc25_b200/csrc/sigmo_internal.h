@@ -331,6 +331,8 @@ int filter_lane_blocks_per_sm(const FilterLaneParams &p);
 cudaError_t launch_mrec(const int32_t *goff, const uint32_t *adj_off, const uint32_t *cand_units, int ND, uint4 *mrec,
                         cudaStream_t st);
 cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, cudaStream_t st);
+cudaError_t launch_lane_totals(int ND, int NQ, int NQW, const uint32_t *gm, const I64x2 *off,
+                               const unsigned long long *presult, unsigned long long *totals, int sm_count, cudaStream_t st);
 size_t join_lane_smem_bytes(const JoinParams &p, bool w64);
 int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem);
 constexpr int kJoinLaneThreads = 128;

@@ -2122,6 +2122,56 @@ cudaError_t launch_gmcr_update(int ND, int NQW, const uint32_t *gm_old, const I6
   return cudaGetLastError();
 }
 
+// S7 count reduction for the lane path: totals[q] += sum over the GMCR pairs (g, q)
+// of pair_result (Find All counts or Find First flags).  One warp per molecule
+// (grid-stride), lane = query within a 32-query word of the GMCR bits; per-warp
+// accumulators in shared memory owned by one lane each (no atomics), summed
+// over the CTA's warps and added to the global totals once per CTA.
+constexpr int kTotThreads = 256;
+__global__ void __launch_bounds__(kTotThreads) k_lane_totals(int ND, int NQ, int NQW, const uint32_t *gm, const I64x2 *off,
+                                                            const unsigned long long *presult, unsigned long long *totals) {
+  extern __shared__ unsigned long long s_acc[];  // [warps][NQW * 32]
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const unsigned lt = (1u << lane) - 1u;
+  const int QS = NQW * 32;
+  unsigned long long *acc = s_acc + (size_t)wid * QS;
+  for (int i = lane; i < QS; i += 32) acc[i] = 0ull;
+  const long long pn = off[ND].a;
+  const int nwarps = (int)((gridDim.x * blockDim.x) >> 5);
+  for (int g = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5); g < ND; g += nwarps) {
+    const I64x2 o0 = off[g], o1 = off[g + 1];
+    long long o = o1.b > o0.b ? pn + o0.b : o0.a;  // the records' order (k_pairs)
+    for (int qb = 0; qb < NQW; qb++) {
+      const uint32_t bits = __ldg(&gm[(size_t)g * NQW + qb]);
+      if ((bits >> lane) & 1u) acc[qb * 32 + lane] += __ldg(&presult[o + __popc(bits & lt)]);
+      o += __popc(bits);
+    }
+  }
+  __syncthreads();
+  for (int q = threadIdx.x; q < NQ; q += blockDim.x) {
+    unsigned long long t = 0ull;
+    for (int w = 0; w < nw; w++) t += s_acc[(size_t)w * QS + q];
+    if (t) atomicAdd(&totals[q], t);
+  }
+}
+
+cudaError_t launch_lane_totals(int ND, int NQ, int NQW, const uint32_t *gm, const I64x2 *off,
+                               const unsigned long long *presult, unsigned long long *totals, int sm_count, cudaStream_t st) {
+  if (ND <= 0 || NQ <= 0) return cudaSuccess;
+  // warps per CTA so that the accumulators fit 96 KB
+  int warps = kTotThreads / 32;
+  while (warps > 1 && (size_t)warps * NQW * 32 * 8 > 96 * 1024) warps--;
+  const size_t smem = (size_t)warps * NQW * 32 * 8;
+  if (smem > 200 * 1024) return cudaErrorInvalidValue;
+  if (smem > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(k_lane_totals, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+  }
+  const long long blocks = std::min<long long>((ND + warps - 1) / warps, (long long)sm_count * 8);
+  k_lane_totals<<<(unsigned)blocks, 32 * warps, smem, st>>>(ND, NQ, NQW, gm, off, presult, totals);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_pairs(const PairsParams &p, cudaStream_t st) {
   if (p.ND <= 0) return cudaSuccess;
   const long long blocks = std::min<long long>((32ll * p.ND + 255) / 256, 148ll * 16);
@@ -2250,11 +2300,11 @@ __host__ __device__ inline size_t join_lane_warp_bytes(int MQ, bool w64) {
   // {R, U} [SD][32] (8 or 16 B) | map words [SD + 1][32] (u32: adjacency index of f(pi_d); slot SD: all ones)
   return 32 * (size_t)(w64 ? 16 : 8) * SD + 128 * (size_t)(SD + 1);
 }
-// CTA: per-query totals [NQ] u64, then one region per warp
-// CTA: per-query totals [NQ] u64, then (optionally) the plan entries [VQ] uint2
+// CTA: (optionally) the plan entries [VQ] uint2, then one region per warp
 __host__ __device__ inline size_t join_lane_plan_bytes(int VQ, int pmax) { return VQ <= pmax ? align16(8 * (size_t)VQ) : 0; }
 __host__ __device__ inline size_t join_lane_cta_bytes(int NQ, int VQ, int pmax) {
-  return align16(8 * (size_t)(NQ > 0 ? NQ : 1)) + join_lane_plan_bytes(VQ, pmax);
+  (void)NQ;
+  return join_lane_plan_bytes(VQ, pmax);
 }
 __host__ __device__ inline size_t join_lane_smem(int NQ, int VQ, int MQ, bool w64, int pmax, int threads) {
   return join_lane_cta_bytes(NQ, VQ, pmax) + join_lane_warp_bytes(MQ, w64) * (size_t)(threads / 32);
@@ -2265,14 +2315,6 @@ size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_sm
 __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
   for (int i = 0; i < n; i++) m &= m - 1u;
   return __ffs(m) - 1;
-}
-
-// 64-bit add to a little-endian {lo, hi} pair of shared words by 32-bit atomics
-// (a 64-bit shared atomic add is a compare-and-swap loop on sm_100)
-__device__ __forceinline__ void sh_add64(unsigned *w, unsigned long long x) {
-  const unsigned lo = (unsigned)x, old = atomicAdd(w, lo);
-  const unsigned hi = (unsigned)(x >> 32) + (old + lo < old ? 1u : 0u);
-  if (hi) atomicAdd(w + 1, hi);
 }
 
 // shared-space accesses at 32-bit shared addresses (volatile: kept in program
@@ -2321,10 +2363,8 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int MQ = jp.maxq, SD = MQ > 1 ? MQ - 1 : 1;
   // ---- CTA tables ----
-  const unsigned o_tot = 0u;
-  for (int i = threadIdx.x; i < jp.NQ; i += blockDim.x) ((unsigned long long *)(smem + o_tot))[i] = 0ull;
   // plan entries (8 B, JoinParams::qp_ent2): a shared-memory copy when they fit, else through the read-only cache
-  const unsigned o_plan = (unsigned)align16(8 * (size_t)(jp.NQ > 0 ? jp.NQ : 1));
+  const unsigned o_plan = 0u;
   if (PS)
     for (int i = threadIdx.x; i < jp.VQ; i += blockDim.x) ((uint2 *)(smem + o_plan))[i] = __ldg(&jp.qp_ent2[i]);
   // plan entry at shared-space address / global index p (an explicit ld.shared:
@@ -2411,7 +2451,6 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   unsigned cmb = 0u;  // cmol index of the current pair's first candidate window
   unsigned ca = 0u, ngs = 0u, pe = 0u;  // ca: adjacency index of the molecule's node 0; pe: plan address of depth 1
   unsigned cp = 0u;
-  int cq = 0;
   unsigned long long cnt = 0ull;
   unsigned steps = 0u;
   bool nv = false;  // next pair assigned (its record in registers)
@@ -2508,19 +2547,15 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     }
     if (__popc(__ballot_sync(FULL_MASK, ne == 0u)) < keff) continue;
 
-    // ---- finished pairs (parts): result, per-query total in shared memory ----
+    // ---- finished pairs (parts): result (the per-query totals are reduced from the results by
+    // k_lane_totals) ----
     if (pend && ne == 0u) {
       if (MODE & 1) {
-        if (!shared) {
-          presult[cp] = cnt ? 1ull : 0ull;
-          if (cnt) sh_add64((unsigned *)(smem + o_tot) + 2 * cq, 1ull);
-        } else if (cnt) {
-          if (atomicOr(&presult[cp], 1ull) == 0ull) sh_add64((unsigned *)(smem + o_tot) + 2 * cq, 1ull);
-        }
+        if (!shared) presult[cp] = cnt ? 1ull : 0ull;
+        else if (cnt) atomicOr(&presult[cp], 1ull);
       } else {
         if (!shared) presult[cp] = cnt;
         else if (cnt) atomicAdd(&presult[cp], cnt);
-        if (cnt) sh_add64((unsigned *)(smem + o_tot) + 2 * cq, cnt);
       }
       pend = false;
     }
@@ -2530,7 +2565,6 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
       cp = nidx;
       cmb = (unsigned)nrec.z;
       ca = (unsigned)nrec.x;  // adjacency word offset of the molecule
-      cq = nrec.y;
       ngs = (((unsigned)nrec.w >> 8) & 0xffu) << sw;  // molecule size: class stride of the adjacency
       pe = paddr(((unsigned)nrec.w >> 16) + 1u);
       shared = false;
@@ -2592,7 +2626,6 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
         const int ds_own = __ffs(ne) - 1;  // shallowest open depth
         const int ds = __shfl_sync(FULL_MASK, ds_own, src);
         const unsigned s_cp = __shfl_sync(FULL_MASK, cp, src);
-        const int s_cq = __shfl_sync(FULL_MASK, cq, src);
         const unsigned s_ngs = __shfl_sync(FULL_MASK, ngs, src);
         const unsigned s_pe = __shfl_sync(FULL_MASK, pe, src);
         const unsigned s_ca = __shfl_sync(FULL_MASK, ca, src);
@@ -2612,7 +2645,6 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
           for (int j = 0; j < ds; j++) JL_MAPW(j, lds32(sMA + 128u * j + 4u * dl));
           cmb = s_cmb;
           cp = s_cp;
-          cq = s_cq;
           ngs = s_ngs;
           pe = s_pe;
           ca = s_ca;
@@ -2632,11 +2664,6 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s2 += __shfl_xor_sync(FULL_MASK, s2, o);
     if (lane == 0) atomicAdd(jp.stats, s2);
-  }
-  __syncthreads();
-  for (int q = threadIdx.x; q < jp.NQ; q += blockDim.x) {
-    const unsigned long long t = ((const unsigned long long *)(smem + o_tot))[q];
-    if (t) atomicAdd(&jp.totals[q], t);
   }
 #undef JL_LDRU
 #undef JL_STRU
