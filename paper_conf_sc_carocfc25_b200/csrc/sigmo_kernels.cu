@@ -2535,14 +2535,15 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
           X &= ~(adj(ia) | adj(ib));
         }
       }
-      if (en.x & 0x800u) {  // depth e is the last: count (or decide) its candidates
-        cnt += (unsigned long long)popc(X);
-        if ((MODE & 4) && X) emit(X, (int)d, used);  // enumerate mode: write the embeddings
-        if ((MODE & 1) && X) ne = 0u;  // Find First: the pair (part) is decided
-      } else if (X) {
-        JL_STRU(od + 32u * ES, X, used);
-        ne += bd + bd;  // bit d + 1 is clear: d is the deepest open depth
-      }
+      // depth e is the last: count (or decide) its candidates; else push them
+      // (no branches: the two outcomes are selects and a predicated store)
+      const bool leaf = (en.x & 0x800u) != 0u;
+      if ((MODE & 4) && leaf && X) emit(X, (int)d, used);  // enumerate mode: write the embeddings
+      cnt += (unsigned long long)popc(leaf ? X : (MT)0);
+      if ((MODE & 1) && leaf && X) ne = 0u;  // Find First: the pair (part) is decided
+      const bool push = !leaf && X;
+      if (push) JL_STRU(od + 32u * ES, X, used);
+      ne += push ? bd + bd : 0u;  // bit d + 1 is clear: d is the deepest open depth
       steps++;
     }
     if (__popc(__ballot_sync(FULL_MASK, ne == 0u)) < keff) continue;
