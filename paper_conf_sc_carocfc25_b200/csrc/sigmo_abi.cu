@@ -2088,6 +2088,8 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
         if (c->lane_ns) jp.cmol = (const uint32_t *)(w64 ? c->ns_win64.p : c->ns_win32.p);
         int bps = join_lane_blocks_per_sm((int)mode, w64, jp, smem);
         if (const char *e = getenv("SIGMO_JOIN_BPS")) bps = std::max(1, std::min(bps, atoi(e)));
+        if (const char *e = getenv(w64 ? "SIGMO_JOIN_BPS_FORCE_WIDE" : "SIGMO_JOIN_BPS_FORCE"))  // experiment knob
+          bps = std::max(1, std::min(32, atoi(e)));
         const int grid = bps * c->sm_count;
         if (getenv("SIGMO_DEBUG_JOIN"))
           fprintf(stderr, "sigmo join: lane %s mode %d threads %d smem %zu blocks/SM %d grid %d\n", w64 ? "wide" : "narrow",

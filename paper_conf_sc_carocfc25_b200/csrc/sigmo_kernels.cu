@@ -2300,11 +2300,12 @@ __host__ __device__ inline size_t join_lane_warp_bytes(int MQ, bool w64) {
   // {R, U} [SD][32] (8 or 16 B) | map words [SD + 1][32] (u32: adjacency index of f(pi_d); slot SD: all ones)
   return 32 * (size_t)(w64 ? 16 : 8) * SD + 128 * (size_t)(SD + 1);
 }
-// CTA: (optionally) the plan entries [VQ] uint2, then one region per warp
+// CTA: the window and adjacency base pointers (16 B), (optionally) the plan entries [VQ] uint2, then one
+// region per warp
 __host__ __device__ inline size_t join_lane_plan_bytes(int VQ, int pmax) { return VQ <= pmax ? align16(8 * (size_t)VQ) : 0; }
 __host__ __device__ inline size_t join_lane_cta_bytes(int NQ, int VQ, int pmax) {
   (void)NQ;
-  return join_lane_plan_bytes(VQ, pmax);
+  return 16 + join_lane_plan_bytes(VQ, pmax);
 }
 __host__ __device__ inline size_t join_lane_smem(int NQ, int VQ, int MQ, bool w64, int pmax, int threads) {
   return join_lane_cta_bytes(NQ, VQ, pmax) + join_lane_warp_bytes(MQ, w64) * (size_t)(threads / 32);
@@ -2364,7 +2365,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   const int MQ = jp.maxq, SD = MQ > 1 ? MQ - 1 : 1;
   // ---- CTA tables ----
   // plan entries (8 B, JoinParams::qp_ent2): a shared-memory copy when they fit, else through the read-only cache
-  const unsigned o_plan = 0u;
+  const unsigned o_plan = 16u;
   if (PS)
     for (int i = threadIdx.x; i < jp.VQ; i += blockDim.x) ((uint2 *)(smem + o_plan))[i] = __ldg(&jp.qp_ent2[i]);
   // plan entry at shared-space address / global index p (an explicit ld.shared:
@@ -2399,7 +2400,17 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     return W64 ? (unsigned)(__ffsll((long long)x) - 1) : (unsigned)(__ffs((unsigned)x) - 1);
   };
   JL_MAPW(SD, jp.adj_ones);  // absent back-edges read the all-ones entry (class field 0)
+  // the two base pointers of the step's global loads pass through shared memory: read back from there
+  // they stay in registers (a kernel-parameter value is re-loaded from the constant bank every step)
+  if (threadIdx.x == 0) *(ulonglong2 *)smem = make_ulonglong2((unsigned long long)jp.cmol, (unsigned long long)jp.adjw);
   __syncthreads();
+  const uint32_t *cmol, *adjw;
+  {
+    unsigned long long pc, pa;
+    asm volatile("ld.shared.v2.u64 {%0, %1}, [%2];" : "=l"(pc), "=l"(pa) : "r"(sbase));
+    cmol = (const uint32_t *)pc;
+    adjw = (const uint32_t *)pa;
+  }
 
   const unsigned lt = (1u << lane) - 1u;
   // this launch's pairs: records / results [pair_base, pair_base + pair_count)
@@ -2409,13 +2420,11 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   const int4 *const recs = jp.prec + pbase0;
   unsigned long long *const presult = jp.pair_result + pbase0;
   unsigned *const counter = (unsigned *)jp.chunk_counter;
-  const uint32_t *const adjw = jp.adjw;
   // mask of adjacency word index i (entries of 1 or 2 words)
   auto adj = [&](unsigned i) -> MT {
     if (W64) return (MT)__ldg((const unsigned long long *)(adjw + i));
     return (MT)__ldg(adjw + i);
   };
-  const uint32_t *const cmol = jp.cmol;
   // candidate window at cmol word index i
   auto cand = [&](unsigned i) -> MT {
     if (W64) return (MT)__ldg((const unsigned long long *)(cmol + i));
@@ -2537,11 +2546,12 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
       }
       // depth e is the last: count (or decide) its candidates; else push them
       // (no branches: the two outcomes are selects and a predicated store)
-      const bool leaf = (en.x & 0x800u) != 0u;
+      const unsigned leaf = en.x & 0x800u;
       if ((MODE & 4) && leaf && X) emit(X, (int)d, used);  // enumerate mode: write the embeddings
-      cnt += (unsigned long long)popc(leaf ? X : (MT)0);
-      if ((MODE & 1) && leaf && X) ne = 0u;  // Find First: the pair (part) is decided
-      const bool push = !leaf && X;
+      const MT Xl = leaf ? X : (MT)0;
+      cnt += (unsigned long long)popc(Xl);
+      if ((MODE & 1) && Xl) ne = 0u;  // Find First: the pair (part) is decided
+      const bool push = X != Xl;
       if (push) JL_STRU(od + 32u * ES, X, used);
       ne += push ? bd + bd : 0u;  // bit d + 1 is clear: d is the deepest open depth
       steps++;
