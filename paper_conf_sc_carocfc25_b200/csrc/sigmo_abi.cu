@@ -2061,7 +2061,10 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
       jp.plan_smem_max = kJoinLanePlanSmemMax;
       if (const char *e = getenv("SIGMO_JOIN_PLAN_SMEM")) jp.plan_smem_max = atoi(e);  // test knob: 0 = plan through L1
-      jp.carveout = -1;
+      // preferred shared-memory carveout: the driver default for Find All; 75 % for Find First (configs[2]
+      // sweep, r2: FA default/75/50 -> 5.04/5.06/5.12 ms, FF 3.75/3.61/3.83 ms; less shares the L1 that
+      // caches the adjacency and windows)
+      jp.carveout = mode == SIGMO_FIND_FIRST ? 75 : -1;
       if (const char *e = getenv("SIGMO_JOIN_CARVEOUT")) jp.carveout = atoi(e);  // test knob (percent)
       // two launches: pairs of <= 32-node molecules with 32-bit masks, and
       // the others with 64-bit masks (each finds its range in off[ND]); the

@@ -340,7 +340,10 @@ constexpr int kJoinLanePlanSmemMax = 2048;  // k_join_lane: plan positions copie
 // k_join_lane CTA size (the launch-bounds maximum; JoinParams::lane_threads is the launched size): 6 warps for
 // 32-bit masks (7 CTAs x 6 warps at <= 48 registers and ~30 KB of shared memory; the plan copy and the per-query
 // totals are per CTA), 4 for 64-bit masks
-__host__ __device__ constexpr int jl_threads(bool w64) { return w64 ? 128 : 192; }
+#ifndef SIGMO_JL_THREADS_NARROW
+#define SIGMO_JL_THREADS_NARROW 192
+#endif
+__host__ __device__ constexpr int jl_threads(bool w64) { return w64 ? 128 : SIGMO_JL_THREADS_NARROW; }
 constexpr int kJoinLaneMaxQ = 11;  // k_join_lane handles queries <= 11 nodes in <= 64-node graphs (map: 6 bits x 10 depths)
 size_t join_smem_bytes(int NW, const JoinParams &p);
 size_t join_gstack_bytes(int NW, const JoinParams &p, int grid);
