@@ -154,6 +154,7 @@ struct sigmo_ctx {
   // program last ran (ent_R), re-uploaded when R changes
   std::vector<int4> ent_host;
   std::vector<uint2> ent_up;  // compact entries for k_join_lane (8 B): see JoinParams::qp_ent2
+  bool lane_extras = true;     // some entry has > 2 back-edges (JoinParams::extras)
   std::vector<int32_t> ent_row;
   std::vector<int64_t> qgoff_host;  // query graph offsets (host copy, for the per-query row-word lists)
   int ent_R = -1;
@@ -1803,6 +1804,8 @@ sigmo_status sigmo_filter(sigmo_ctx *c, int levels, uint32_t flags) {
         c->ent_up[i].x = (s0 << 7) | (leaf << 11) | (nex << 12) | ((s1 << 7) << 16);
         c->ent_up[i].y = ((unsigned)e.y & 7u) | (((unsigned)e.z & 7u) << 3) | ((unsigned)qd[(size_t)c->ent_row[i]] << 12);
       }
+      c->lane_extras = false;  // some plan position has > 2 back-edges (fused rings): the join keeps its extra loop
+      for (const uint2 &u : c->ent_up) c->lane_extras = c->lane_extras || (u.x & 0xf000u);
       SIGMO_TRY(dreserve(c, c->ent2, sizeof(uint2) * (c->ent_up.size() + 1), "plan entries"));
       if (!c->ent_up.empty())
         CUDA_TRY(c, cudaMemcpyAsync(c->ent2.p, c->ent_up.data(), sizeof(uint2) * c->ent_up.size(),
@@ -2060,6 +2063,7 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
       jp.qp_qn = c->qp_qn;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
       jp.plan_smem_max = kJoinLanePlanSmemMax;
+      jp.extras = c->lane_extras ? 1 : 0;
       if (const char *e = getenv("SIGMO_JOIN_PLAN_SMEM")) jp.plan_smem_max = atoi(e);  // test knob: 0 = plan through L1
       // preferred shared-memory carveout: the driver default for Find All; 75 % for Find First (configs[2]
       // sweep, r2: FA default/75/50 -> 5.04/5.06/5.12 ms, FF 3.75/3.61/3.83 ms; less shares the L1 that

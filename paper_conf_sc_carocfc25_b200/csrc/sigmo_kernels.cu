@@ -2523,7 +2523,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
       const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
       const MT used = U | bit;
       MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0) & adj(i1);
-      if (en.x & 0xf000u) {  // > 2 back-edges at this depth (fused rings): rare
+      if (!(MODE & 8) && (en.x & 0xf000u)) {  // > 2 back-edges at this depth (fused rings): rare
         const unsigned nex = (en.x >> 12) & 15u;
         const unsigned b0 = (unsigned)__ldg(&jp.qp_ent[cqb_of(pe) + d + 1u]).w;
 #pragma unroll 1
@@ -2707,28 +2707,29 @@ static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_
   return cudaGetLastError();
 }
 
+// the k_join_lane instantiation of a launch: bit 0 Find First, bit 1 induced (p.induced), bit 2 enumerate
+// (p.emaps, Find All semantics), bit 3 no plan position with > 2 back-edges (p.extras == 0; Find All / First only)
+static int lane_mode(int mode, const JoinParams &p) {
+  if (p.emaps) return p.induced ? 6 : 4;
+  const int m = (mode & 1) | (p.induced ? 2 : 0);
+  return (m < 2 && !p.extras) ? (m | 8) : m;
+}
+
+#define SIGMO_JL_DISPATCH(F, ...)                                              \
+  switch (lane_mode(mode, p)) {                                                \
+    case 0: return w64 ? F<0, true>(__VA_ARGS__) : F<0, false>(__VA_ARGS__);   \
+    case 1: return w64 ? F<1, true>(__VA_ARGS__) : F<1, false>(__VA_ARGS__);   \
+    case 2: return w64 ? F<2, true>(__VA_ARGS__) : F<2, false>(__VA_ARGS__);   \
+    case 3: return w64 ? F<3, true>(__VA_ARGS__) : F<3, false>(__VA_ARGS__);   \
+    case 4: return w64 ? F<4, true>(__VA_ARGS__) : F<4, false>(__VA_ARGS__);   \
+    case 6: return w64 ? F<6, true>(__VA_ARGS__) : F<6, false>(__VA_ARGS__);   \
+    case 8: return w64 ? F<8, true>(__VA_ARGS__) : F<8, false>(__VA_ARGS__);   \
+    default: return w64 ? F<9, true>(__VA_ARGS__) : F<9, false>(__VA_ARGS__);  \
+  }
+
 cudaError_t launch_join_lane(int mode, bool w64, const JoinParams &p, int grid, cudaStream_t st) {
   if (grid <= 0) return cudaSuccess;
-  // mode bit 0: Find First; bit 1: induced (p.induced); p.emaps: enumerate (Find All semantics)
-  const int m = (mode & 1) | (p.induced ? 2 : 0);
-  if (p.emaps) {
-    if (w64) return p.induced ? launch_join_lane_t<6, true>(p, grid, st) : launch_join_lane_t<4, true>(p, grid, st);
-    return p.induced ? launch_join_lane_t<6, false>(p, grid, st) : launch_join_lane_t<4, false>(p, grid, st);
-  }
-  if (w64) {
-    switch (m) {
-      case 0: return launch_join_lane_t<0, true>(p, grid, st);
-      case 1: return launch_join_lane_t<1, true>(p, grid, st);
-      case 2: return launch_join_lane_t<2, true>(p, grid, st);
-      default: return launch_join_lane_t<3, true>(p, grid, st);
-    }
-  }
-  switch (m) {
-    case 0: return launch_join_lane_t<0, false>(p, grid, st);
-    case 1: return launch_join_lane_t<1, false>(p, grid, st);
-    case 2: return launch_join_lane_t<2, false>(p, grid, st);
-    default: return launch_join_lane_t<3, false>(p, grid, st);
-  }
+  SIGMO_JL_DISPATCH(launch_join_lane_t, p, grid, st)
 }
 
 template <int MODE, bool W64>
@@ -2750,27 +2751,10 @@ static int join_lane_occ_t(size_t smem, bool ps, int carveout, int threads) {
 }
 
 int join_lane_blocks_per_sm(int mode, bool w64, const JoinParams &p, size_t smem) {
-  // the instantiation launch_join_lane picks: bit 0 Find First, bit 1 induced, enumerate
-  const int m = (mode & 1) | (p.induced ? 2 : 0);
+  // the instantiation launch_join_lane picks
   const bool ps = join_lane_plan_bytes(p.VQ, p.plan_smem_max) > 0;
-  if (p.emaps) {
-    if (w64) return p.induced ? join_lane_occ_t<6, true>(smem, ps, p.carveout, p.lane_threads) : join_lane_occ_t<4, true>(smem, ps, p.carveout, p.lane_threads);
-    return p.induced ? join_lane_occ_t<6, false>(smem, ps, p.carveout, p.lane_threads) : join_lane_occ_t<4, false>(smem, ps, p.carveout, p.lane_threads);
-  }
-  if (w64) {
-    switch (m) {
-      case 0: return join_lane_occ_t<0, true>(smem, ps, p.carveout, p.lane_threads);
-      case 1: return join_lane_occ_t<1, true>(smem, ps, p.carveout, p.lane_threads);
-      case 2: return join_lane_occ_t<2, true>(smem, ps, p.carveout, p.lane_threads);
-      default: return join_lane_occ_t<3, true>(smem, ps, p.carveout, p.lane_threads);
-    }
-  }
-  switch (m) {
-    case 0: return join_lane_occ_t<0, false>(smem, ps, p.carveout, p.lane_threads);
-    case 1: return join_lane_occ_t<1, false>(smem, ps, p.carveout, p.lane_threads);
-    case 2: return join_lane_occ_t<2, false>(smem, ps, p.carveout, p.lane_threads);
-    default: return join_lane_occ_t<3, false>(smem, ps, p.carveout, p.lane_threads);
-  }
+  SIGMO_JL_DISPATCH(join_lane_occ_t, smem, ps, p.carveout, p.lane_threads)
 }
+#undef SIGMO_JL_DISPATCH
 
 }  // namespace sigmo

@@ -378,3 +378,22 @@ def test_neighbour_support_lane_path_c2(sigmo):
         F = fr.neighbour_support(Q, Dg, fr.candidates_bool(Q, Dg, 4))
         want = set(np.nonzero(fr.gmcr(Q, Dg, F)[:, 0])[0].tolist())
         assert set(qi[di == g].tolist()) == want, g
+
+
+def test_lane_join_extra_back_edges(ctx, sigmo):
+    """Queries with a plan depth of > 2 back-edges (K4, K5, a fused bicycle)
+    run the lane join's instantiation with the extra back-edge loop; the same
+    data with queries of <= 2 back-edges per depth runs the lean one
+    (JoinParams::extras).  Both against the oracle, Find All and Find First."""
+    rng = np.random.default_rng(5)
+    ds = [synth.random_labelled_graph(rng, int(rng.integers(4, 30)), float(rng.uniform(0.15, 0.6)),
+                                      labels=(6, 6, 7)) for _ in range(300)]
+    D = GraphBatch.from_graphs(ds)
+    k4 = ([6] * 4, [(i, j, 1) for i in range(4) for j in range(i + 1, 4)])
+    k5 = ([6] * 5, [(i, j, 1) for i in range(5) for j in range(i + 1, 5)])
+    bicycle = ([6] * 6, [(0, 1, 1), (1, 2, 1), (2, 3, 1), (3, 0, 1), (1, 4, 1), (4, 5, 1), (5, 3, 1), (0, 2, 1)])
+    for qs in ([k4, k5, bicycle, path(4)], [path(4), ring(5), ring(4), ([6, 7], [(0, 1, 1)])]):
+        Q = GraphBatch.from_graphs(qs)
+        for mode, om in ((sigmo.SIGMO_FIND_ALL, oracle.FIND_ALL), (sigmo.SIGMO_FIND_FIRST, oracle.FIND_FIRST)):
+            _, dense = run(ctx, Q, D, 2, mode)
+            assert np.array_equal(dense, oracle.count_dense(Q, D, om)), (len(qs), mode)
