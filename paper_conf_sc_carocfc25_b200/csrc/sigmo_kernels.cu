@@ -2449,21 +2449,21 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     bend = x + kJoinClaim;
     bnext0 = x + kJoinClaim;
   }
-  bool drained = cursor >= P;
+  unsigned drained = cursor >= P ? 1u : 0u;
   int keff = jp.batchK;  // free lanes that end a stepping phase (1 once the list is drained)
   if (drained) keff = 1;
 
   // ---- lane state ----
   unsigned ne = 0u;  // open depths of the current pair (0: no work)
-  bool pend = false;  // holds a pair (part) whose result is not yet written
-  bool shared = false;
+  unsigned pend = 0u;  // holds a pair (part) whose result is not yet written
+  unsigned shared = 0u;
   unsigned cmb = 0u;  // cmol index of the current pair's first candidate window
   unsigned ca = 0u, ngs = 0u, pe = 0u;  // ca: adjacency index of the molecule's node 0; pe: plan address of depth 1
   unsigned cp = 0u;
   unsigned long long cnt = 0ull;
   unsigned steps = 0u;
-  bool nv = false;  // next pair assigned (its record in registers)
-  bool nr = false;  // and the load of its root window issued (the refill pass after the record's)
+  unsigned nv = 0u;  // next pair assigned (its record in registers)
+  unsigned nr = 0u;  // and the load of its root window issued (the refill pass after the record's)
   int4 nrec = make_int4(0, 0, 0, 0);
   unsigned nidx = 0u;
   MT nR0 = 0;
