@@ -2500,61 +2500,64 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   };
 
   while (true) {
-    // ---- one DFS step ----
-    if (ne) {
-      const unsigned d = bfind32(ne);  // deepest open depth
-      const unsigned bd = 1u << d;
-      const unsigned od = sRU + 32u * ES * d;
-      // plan entry of depth e = d + 1 (x: back-edge map slots, leaf, #extra;
-      // y: bond classes, distinct row)
-      const uint2 en = JL_PLAN(pe + PSTEP * d);
-      MT R, U;
-      JL_LDRU(od, R, U);
-      const unsigned v = highest(R);
-      const MT bit = (MT)1 << v;
-      const MT Rn = R ^ bit;
-      sts_mask(od, Rn);
-      ne ^= Rn ? 0u : bd;
-      // map word of depth d = the adjacency index of f(pi_d); stored before the
-      // back-edge slots are read, so a back-edge to d reads it
-      JL_MAPW(d, ca + (v << sw));
-      const unsigned a0 = lds32(sMA + (en.x & 0x7ffu));
-      const unsigned a1 = lds32(sMA + (en.x >> 16));
-      const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
-      const MT used = U | bit;
-      MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0) & adj(i1);
-      if (!(MODE & 8) && (en.x & 0xf000u)) {  // > 2 back-edges at this depth (fused rings): rare
-        const unsigned nex = (en.x >> 12) & 15u;
-        const unsigned b0 = (unsigned)__ldg(&jp.qp_ent[cqb_of(pe) + d + 1u]).w;
-#pragma unroll 1
-        for (unsigned k = 0; k < nex; k++) {
-          const unsigned be = __ldg(&jp.qp_be[b0 + k]);
-          X &= adj((be & 255u) * ngs + JL_MAPR(be >> 8));
+    // ---- DFS steps: two per check of the free lanes (the check is a ballot and a popcount) ----
+#pragma unroll
+    for (int u = 0; u < 2; u++) {
+      if (ne) {
+        const unsigned d = bfind32(ne);  // deepest open depth
+        const unsigned bd = 1u << d;
+        const unsigned od = sRU + 32u * ES * d;
+        // plan entry of depth e = d + 1 (x: back-edge map slots, leaf, #extra;
+        // y: bond classes, distinct row)
+        const uint2 en = JL_PLAN(pe + PSTEP * d);
+        MT R, U;
+        JL_LDRU(od, R, U);
+        const unsigned v = highest(R);
+        const MT bit = (MT)1 << v;
+        const MT Rn = R ^ bit;
+        sts_mask(od, Rn);
+        ne ^= Rn ? 0u : bd;
+        // map word of depth d = the adjacency index of f(pi_d); stored before the
+        // back-edge slots are read, so a back-edge to d reads it
+        JL_MAPW(d, ca + (v << sw));
+        const unsigned a0 = lds32(sMA + (en.x & 0x7ffu));
+        const unsigned a1 = lds32(sMA + (en.x >> 16));
+        const unsigned i0 = (en.y & 7u) * ngs + a0, i1 = ((en.y >> 3) & 7u) * ngs + a1;
+        const MT used = U | bit;
+        MT X = cand(cmb + ((en.y >> 12) << sw)) & ~used & adj(i0) & adj(i1);
+        if (!(MODE & 8) && (en.x & 0xf000u)) {  // > 2 back-edges at this depth (fused rings): rare
+          const unsigned nex = (en.x >> 12) & 15u;
+          const unsigned b0 = (unsigned)__ldg(&jp.qp_ent[cqb_of(pe) + d + 1u]).w;
+  #pragma unroll 1
+          for (unsigned k = 0; k < nex; k++) {
+            const unsigned be = __ldg(&jp.qp_be[b0 + k]);
+            X &= adj((be & 255u) * ngs + JL_MAPR(be >> 8));
+          }
         }
-      }
-      if (MODE & 2) {  // induced mode (R21): drop neighbours (any bond) of mapped non-adjacent depths
-        const unsigned cn = (unsigned)jp.NB * ngs;
-        // two depths per iteration (the second reads the all-zeros entry when absent)
-#pragma unroll 1
-        for (unsigned nm = __ldg(&jp.qp_non[cqb_of(pe) + d + 1u]); nm;) {
-          const unsigned ia = cn + JL_MAPR(__ffs(nm) - 1);
-          nm &= nm - 1u;
-          const unsigned ib = nm ? cn + JL_MAPR(__ffs(nm) - 1) : jp.adj_ones + 2u;
-          nm &= nm - 1u;
-          X &= ~(adj(ia) | adj(ib));
+        if (MODE & 2) {  // induced mode (R21): drop neighbours (any bond) of mapped non-adjacent depths
+          const unsigned cn = (unsigned)jp.NB * ngs;
+          // two depths per iteration (the second reads the all-zeros entry when absent)
+  #pragma unroll 1
+          for (unsigned nm = __ldg(&jp.qp_non[cqb_of(pe) + d + 1u]); nm;) {
+            const unsigned ia = cn + JL_MAPR(__ffs(nm) - 1);
+            nm &= nm - 1u;
+            const unsigned ib = nm ? cn + JL_MAPR(__ffs(nm) - 1) : jp.adj_ones + 2u;
+            nm &= nm - 1u;
+            X &= ~(adj(ia) | adj(ib));
+          }
         }
+        // depth e is the last: count (or decide) its candidates; else push them
+        // (no branches: the two outcomes are selects and a predicated store)
+        const unsigned leaf = en.x & 0x800u;
+        if ((MODE & 4) && leaf && X) emit(X, (int)d, used);  // enumerate mode: write the embeddings
+        const MT Xl = leaf ? X : (MT)0;
+        cnt += (unsigned long long)popc(Xl);
+        if ((MODE & 1) && Xl) ne = 0u;  // Find First: the pair (part) is decided
+        const bool push = X != Xl;
+        if (push) JL_STRU(od + 32u * ES, X, used);
+        ne += push ? bd + bd : 0u;  // bit d + 1 is clear: d is the deepest open depth
+        steps++;
       }
-      // depth e is the last: count (or decide) its candidates; else push them
-      // (no branches: the two outcomes are selects and a predicated store)
-      const unsigned leaf = en.x & 0x800u;
-      if ((MODE & 4) && leaf && X) emit(X, (int)d, used);  // enumerate mode: write the embeddings
-      const MT Xl = leaf ? X : (MT)0;
-      cnt += (unsigned long long)popc(Xl);
-      if ((MODE & 1) && Xl) ne = 0u;  // Find First: the pair (part) is decided
-      const bool push = X != Xl;
-      if (push) JL_STRU(od + 32u * ES, X, used);
-      ne += push ? bd + bd : 0u;  // bit d + 1 is clear: d is the deepest open depth
-      steps++;
     }
     if (__popc(__ballot_sync(FULL_MASK, ne == 0u)) < keff) continue;
 
