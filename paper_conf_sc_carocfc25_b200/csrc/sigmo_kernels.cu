@@ -2352,6 +2352,9 @@ __device__ __forceinline__ uint2 lds_u2(unsigned a) {
 // W64: the launch's pairs are on > 32-node molecules (64-bit masks); else all
 // masks, stack entries and loads are 32-bit
 // PS: the plan entries are copied to shared memory (VQ <= kJoinLanePlanSmemMax)
+#ifndef SIGMO_JL_UNROLL
+#define SIGMO_JL_UNROLL 4  // DFS steps per check of the free lanes (configs[2] join: 1/2/3/4 -> 4.86/4.69/4.65/4.64 ms)
+#endif
 #ifndef SIGMO_JL_MAXNREG
 #define SIGMO_JL_MAXNREG 56
 #endif
@@ -2500,9 +2503,9 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   };
 
   while (true) {
-    // ---- DFS steps: two per check of the free lanes (the check is a ballot and a popcount) ----
+    // ---- DFS steps: SIGMO_JL_UNROLL per check of the free lanes (the check is a ballot and a popcount) ----
 #pragma unroll
-    for (int u = 0; u < 2; u++) {
+    for (int u = 0; u < SIGMO_JL_UNROLL; u++) {
       if (ne) {
         const unsigned d = bfind32(ne);  // deepest open depth
         const unsigned bd = 1u << d;
