@@ -2390,8 +2390,15 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   auto popc = [](MT x) -> int { return W64 ? __popcll((unsigned long long)x) : __popc((unsigned)x); };
   auto highest = [](MT x) -> unsigned {  // index of the highest set bit (x != 0)
     unsigned r;
-    if (W64) asm("bfind.u64 %0, %1;" : "=r"(r) : "l"((unsigned long long)x));
-    else asm("bfind.u32 %0, %1;" : "=r"(r) : "r"((unsigned)x));
+    if (W64) {  // two 32-bit bfinds and a select (bfind.u64 compiles to a branch)
+      const unsigned hi = (unsigned)((unsigned long long)x >> 32), lo = (unsigned)x;
+      unsigned fh, fl;
+      asm("bfind.u32 %0, %1;" : "=r"(fh) : "r"(hi));
+      asm("bfind.u32 %0, %1;" : "=r"(fl) : "r"(lo));
+      r = hi ? fh + 32u : fl;
+    } else {
+      asm("bfind.u32 %0, %1;" : "=r"(r) : "r"((unsigned)x));
+    }
     return r;
   };
   auto bfind32 = [](unsigned x) -> unsigned {
