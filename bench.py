@@ -371,7 +371,11 @@ def main():
     with sampler:
         ms_all, tim = timed_loop(sigmo.SIGMO_FIND_ALL, args.steps, True)
     clocks = sampler.summary()
+    # DFS steps of one Find All join (counted by the join's counting instantiation, outside the timed loop)
+    ctx.set_timing(False, count_steps=True)
     matches_local = int(ctx.join(sigmo.SIGMO_FIND_ALL))  # identical every step (deterministic)
+    dfs_steps = int(ctx.timings()["dfs_steps"])
+    ctx.set_timing(False)
     pairs_local = ctx.num_pairs()
     ms_ff, _ = timed_loop(sigmo.SIGMO_FIND_FIRST, args.steps, False)
     positive_local = int(ctx.join(sigmo.SIGMO_FIND_FIRST))
@@ -461,7 +465,7 @@ def main():
     sm_mhz = float(clocks.get("sm_mhz") or peaks.get("sm_max_mhz", 1965.0))
     ip = _load("profiles/r2/int_peak.json")
     lanes = float(ip.get("mixed_lanes_per_sm_per_clk", 128.0))
-    steps = tim.get("dfs_steps", 0)
+    steps = dfs_steps
     alu_peak = 148 * lanes * sm_mhz * 1e6 / 1e12
     join_ach = 12.0 * steps / (j_ms * 1e-3) / 1e12 if j_ms > 0 else 0.0
     jn, jw = nk.get("k_join_lane_narrow", {}), nk.get("k_join_lane_wide", {})

@@ -115,7 +115,8 @@ typedef struct {
   int64_t filter_launches, join_launches;  /* kernels launched by the last filter / join call */
   int64_t h2d_bytes;    /* bytes uploaded by the last sigmo_load_batch (one pinned H2D copy) */
   int64_t filter_calls, join_calls;        /* calls averaged */
-  int64_t dfs_steps;    /* DFS iterator steps (search-tree nodes) of the last join */
+  int64_t dfs_steps;    /* DFS iterator steps (search-tree nodes) of the last join (counted only
+                           with sigmo_set_timing bit 1; else 0 on the lane path) */
   int64_t dfs_iters, dfs_tail_iters, dfs_max_stack;  /* warp iterations, of which after the last pair claim; max stack */
   int64_t filter_jit;   /* 1 if the last lane-path filter ran the kernel specialised for the query program (NVRTC) */
   double jit_compile_ms; /* wall time of the last specialisation compile (0 if served from the process cache) */
@@ -260,7 +261,12 @@ SIGMO_API sigmo_status sigmo_set_induced(sigmo_ctx *ctx, int enable);
  * sigmo_get_signatures leaves '*' atoms out of every field.  Never fails for a
  * valid ctx. */
 SIGMO_API sigmo_status sigmo_set_wildcards(sigmo_ctx *ctx, int enable);
-/* Enable/disable per-stage CUDA-event timing (default off) and read it. */
+/* Per-stage CUDA-event timing and DFS step counting (default off), and their
+ * read-out.  enable bit 0: CUDA events around the filter, mapping and join
+ * stages; bit 1: the join counts its DFS steps (sigmo_timings.dfs_steps; the
+ * lane join then runs its counting instantiation instead of the lean one, so
+ * time it with bit 1 clear).  Other bits are ignored.  Never fails for a
+ * valid ctx. */
 SIGMO_API sigmo_status sigmo_set_timing(sigmo_ctx *ctx, int enable);
 SIGMO_API sigmo_status sigmo_get_timings(sigmo_ctx *ctx, sigmo_timings *out);
 

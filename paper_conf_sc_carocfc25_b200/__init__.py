@@ -302,8 +302,10 @@ class Context:
         (include/sigmo.h sigmo_set_wildcards)."""
         self._check(self._lib.sigmo_set_wildcards(self._handle, 1 if enable else 0), "sigmo_set_wildcards")
 
-    def set_timing(self, enable: bool = True):
-        self._check(self._lib.sigmo_set_timing(self._handle, 1 if enable else 0), "sigmo_set_timing")
+    def set_timing(self, enable=True, count_steps: bool = False):
+        """bit 0: per-stage CUDA-event timing; count_steps (bit 1): the join counts its DFS steps."""
+        flags = (1 if enable else 0) | (2 if count_steps else 0)
+        self._check(self._lib.sigmo_set_timing(self._handle, flags), "sigmo_set_timing")
 
     def timings(self) -> dict:
         t = _native.sigmo_timings()

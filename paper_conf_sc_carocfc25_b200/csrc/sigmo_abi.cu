@@ -154,7 +154,8 @@ struct sigmo_ctx {
   // program last ran (ent_R), re-uploaded when R changes
   std::vector<int4> ent_host;
   std::vector<uint2> ent_up;  // compact entries for k_join_lane (8 B): see JoinParams::qp_ent2
-  bool lane_extras = true;     // some entry has > 2 back-edges (JoinParams::extras)
+  bool lane_extras = true;     // some entry has > 2 back-edges (the lean lane join does not apply)
+  bool count_steps = false;    // sigmo_set_timing bit 1: the join counts its DFS steps (sigmo_timings.dfs_steps)
   std::vector<int32_t> ent_row;
   std::vector<int64_t> qgoff_host;  // query graph offsets (host copy, for the per-query row-word lists)
   int ent_R = -1;
@@ -1246,7 +1247,8 @@ sigmo_status sigmo_set_wildcards(sigmo_ctx *c, int enable) {
 
 sigmo_status sigmo_set_timing(sigmo_ctx *c, int enable) {
   if (!c) return SIGMO_ERR_INVALID_ARG;
-  c->timing.enabled = enable != 0;
+  c->timing.enabled = (enable & 1) != 0;
+  c->count_steps = (enable & 2) != 0;
   return SIGMO_OK;
 }
 
@@ -2063,7 +2065,7 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
       jp.qp_qn = c->qp_qn;
       if (const char *e = getenv("SIGMO_JOIN_BATCH")) jp.batchK = std::max(1, std::min(32, atoi(e)));
       jp.plan_smem_max = kJoinLanePlanSmemMax;
-      jp.extras = c->lane_extras ? 1 : 0;
+      jp.lean = (!c->lane_extras && !c->count_steps) ? 1 : 0;
       if (const char *e = getenv("SIGMO_JOIN_PLAN_SMEM")) jp.plan_smem_max = atoi(e);  // test knob: 0 = plan through L1
       // preferred shared-memory carveout: the driver default for Find All; 75 % for Find First (configs[2]
       // sweep, r2: FA default/75/50 -> 5.04/5.06/5.12 ms, FF 3.75/3.61/3.83 ms; less shares the L1 that

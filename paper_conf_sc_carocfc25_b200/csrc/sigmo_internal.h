@@ -202,7 +202,8 @@ struct JoinParams {
   int plan_smem_max;           // k_join_lane: plan entries copied to shared memory when VQ <= this
   int carveout;                // k_join_lane: preferred shared-memory carveout in percent (-1: driver default)
   int lane_threads;            // k_join_lane: threads per CTA of this launch (<= jl_threads(w64))
-  int extras;                  // k_join_lane: some plan position has > 2 back-edges (0: the lean instantiation)
+  int lean;                    // k_join_lane: no plan position has > 2 back-edges and DFS steps are not counted
+                               // (the lean instantiation: no extra back-edge loop, no step counter)
 };
 
 // k_pairs: GMCR pair list + per-pair candidate masks

@@ -2566,7 +2566,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
         const bool push = X != Xl;
         if (push) JL_STRU(od + 32u * ES, X, used);
         ne += push ? bd + bd : 0u;  // bit d + 1 is clear: d is the deepest open depth
-        steps++;
+        if (!(MODE & 8)) steps++;  // the lean instantiation does not count steps
       }
     }
     if (__popc(__ballot_sync(FULL_MASK, ne == 0u)) < keff) continue;
@@ -2683,7 +2683,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     }
     if (drained && __ballot_sync(FULL_MASK, ne != 0u || nv || pend) == 0u) break;
   }
-  if (jp.stats) {
+  if (!(MODE & 8) && jp.stats) {
     unsigned long long s2 = steps;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s2 += __shfl_xor_sync(FULL_MASK, s2, o);
@@ -2721,11 +2721,12 @@ static cudaError_t launch_join_lane_t(const JoinParams &p, int grid, cudaStream_
 }
 
 // the k_join_lane instantiation of a launch: bit 0 Find First, bit 1 induced (p.induced), bit 2 enumerate
-// (p.emaps, Find All semantics), bit 3 no plan position with > 2 back-edges (p.extras == 0; Find All / First only)
+// (p.emaps, Find All semantics), bit 3 lean (p.lean: no plan position with > 2 back-edges and no DFS step
+// counting; Find All / First only)
 static int lane_mode(int mode, const JoinParams &p) {
   if (p.emaps) return p.induced ? 6 : 4;
   const int m = (mode & 1) | (p.induced ? 2 : 0);
-  return (m < 2 && !p.extras) ? (m | 8) : m;
+  return (m < 2 && p.lean) ? (m | 8) : m;
 }
 
 #define SIGMO_JL_DISPATCH(F, ...)                                              \

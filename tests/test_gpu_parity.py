@@ -397,3 +397,23 @@ def test_lane_join_extra_back_edges(ctx, sigmo):
         for mode, om in ((sigmo.SIGMO_FIND_ALL, oracle.FIND_ALL), (sigmo.SIGMO_FIND_FIRST, oracle.FIND_FIRST)):
             _, dense = run(ctx, Q, D, 2, mode)
             assert np.array_equal(dense, oracle.count_dense(Q, D, om)), (len(qs), mode)
+
+
+def test_lane_join_step_counting(ctx, sigmo):
+    """sigmo_set_timing bit 1: the join counts its DFS steps (the counting
+    instantiation); without it the lean one runs and reports 0; both give the
+    oracle's counts."""
+    Q, D = synth.config_queries(2), synth.config_data(2, count=2000)
+    ref = oracle.count_dense(Q, D)
+    ctx.load_batch(Q, D)
+    ctx.filter(2)
+    ctx.set_timing(False, count_steps=True)
+    ctx.join(sigmo.SIGMO_FIND_ALL)
+    steps = ctx.timings()["dfs_steps"]
+    assert np.array_equal(ctx.dense_results(), ref)
+    ctx.set_timing(False)
+    ctx.join(sigmo.SIGMO_FIND_ALL)
+    assert ctx.timings()["dfs_steps"] == 0
+    assert np.array_equal(ctx.dense_results(), ref)
+    # every step pops one candidate: at least one step per surviving pair with a non-empty root window
+    assert steps >= int((ref > 0).sum())

@@ -17,7 +17,7 @@ ctx = sigmo.Context(0)
 ctx.load_batch(Q, D)
 for mode in (0, 1):
     ctx.filter(L)
-    ctx.set_timing(True)
+    ctx.set_timing(True, count_steps=True)
     tot = ctx.join(mode)
     t = ctx.timings()
     ctx.set_timing(False)
