@@ -61,6 +61,7 @@ struct ProgCache {
   std::vector<uint16_t> qdrow;  // host copy of prog.qdrow
   LaneJitSpec jit;              // the k_filter_lane program (host copy) for the NVRTC-specialised kernel
   bool valid = false;
+  int nw = 0;  // the data batch's window words it was packed for (pack_prog's table size)
 };
 
 struct HostGraphs {  // validated input view (int64 offsets as given)
@@ -159,6 +160,8 @@ struct sigmo_ctx {
   std::vector<int32_t> ent_row;
   std::vector<int64_t> qgoff_host;  // query graph offsets (host copy, for the per-query row-word lists)
   int ent_R = -1;
+  std::vector<unsigned char> qkey;  // the last successfully loaded query batch (sigmo_load_batch reuse check)
+  bool qkey_valid = false;
   int32_t *grp_narrow = nullptr, *grp_wide = nullptr;  // k_filter_lane groups (input arena)
   int NGN = 0, NGW = 0;
   DBuf nb4, mrec;                   // k_filter_lane: packed neighbours [VD], molecule records [ND]
@@ -908,7 +911,7 @@ sigmo_status pack_prog(sigmo_ctx *c, int R, ProgCache &pc) {
 
 sigmo_status ensure_prog(sigmo_ctx *c, int R, QueryProg *&out) {
   auto it = c->progs.find(R);
-  if (it != c->progs.end() && it->second.valid) {
+  if (it != c->progs.end() && it->second.valid && it->second.nw == c->NW) {
     out = &it->second.prog;
     return SIGMO_OK;
   }
@@ -952,6 +955,7 @@ sigmo_status ensure_prog(sigmo_ctx *c, int R, QueryProg *&out) {
   if (P.meta.err) return set_err(c, SIGMO_ERR_LIMIT, "query program error %d", P.meta.err);
   SIGMO_TRY(pack_prog(c, R, pc));
   pc.valid = true;
+  pc.nw = c->NW;
   out = &P;
   return SIGMO_OK;
 }
@@ -1283,6 +1287,26 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
   const auto t0 = std::chrono::steady_clock::now();
   sigmo_status s = validate(queries, 1, msg, hq);
   if (s != SIGMO_OK) return set_err(c, s, "query batch: %s", msg.c_str());
+  // the same query batch as the previous load (byte for byte, same wildcard mode): the query programs
+  // and the join's plan entries built for it are reused
+  bool same_q = false;
+  {
+    std::vector<unsigned char> key;
+    auto add = [&](const void *p, size_t n) {
+      const unsigned char *b = (const unsigned char *)p;
+      key.insert(key.end(), b, b + n);
+    };
+    const int64_t dims[4] = {hq.G, hq.V, hq.E, c->wildcard ? 1 : 0};
+    add(dims, sizeof(dims));
+    add(hq.goff, 8 * (size_t)(hq.G + 1));
+    add(hq.roff, 8 * (size_t)(hq.V + 1));
+    if (hq.E) add(hq.col, 4 * (size_t)hq.E);
+    if (hq.V) add(hq.nlab, (size_t)hq.V);
+    if (hq.E) add(hq.elab, (size_t)hq.E);
+    same_q = c->qkey_valid && key == c->qkey;
+    c->qkey.swap(key);
+    c->qkey_valid = false;  // valid again once this load succeeded
+  }
   // large data batches: O(#graphs) checks here, the per-entry checks and the
   // packing on the device (k_load_data) from the raw arrays
   const char *hl = getenv("SIGMO_HOST_LOAD");  // test knob: host validation + packing at any size
@@ -1598,10 +1622,15 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       for (int k = plan.beoff[i]; k < plan.beoff[i + 1]; k++) m &= ~(1ull << (plan.be[k] >> 8));
       non[i] = (uint32_t)m;
     }
+    // the join's plan entries stay valid when the query batch and its matching order did not change
+    // (a stream of data batches against the same queries: no re-upload and no host sync per batch)
+    const bool same_plan = same_q && c->ent_host.size() == (size_t)hq.V &&
+                           (hq.V == 0 || !memcmp(c->ent_host.data(), ent, sizeof(int4) * (size_t)hq.V)) &&
+                           c->ent_row == plan.row;
     c->ent_host.assign(ent, ent + hq.V);
     c->ent_row.assign(plan.row.begin(), plan.row.end());
     c->qgoff_host.assign(hq.goff, hq.goff + hq.G + 1);
-    c->ent_R = -1;
+    if (!same_plan) c->ent_R = -1;
   }
   if (!dev_load) pack_graphs(hb, pd, hd);
   memcpy(hb + o_tg0, tg0.data(), 4 * tg0.size());
@@ -1699,8 +1728,9 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
       c->MC = std::max(c->MC / 2, 1);
     }
   }
-  // query programs depend on the query batch only, but the batch changed
-  for (auto &kv : c->progs) kv.second.valid = false;
+  // query programs depend on the query batch (and the wildcard mode) only
+  if (!same_q)
+    for (auto &kv : c->progs) kv.second.valid = false;
 
   // ---- per-batch device buffers ----
   // (+64 B: the join reads up to two words past a molecule window)
@@ -1750,6 +1780,7 @@ sigmo_status sigmo_load_batch(sigmo_ctx *c, const sigmo_graph_batch *queries, co
             "drain %.1f ms\n", ms(t0, t1), ms(t1, t2), ms(t2, t3), ms(t3, t4), ms(t4, t5), ms(t5, t6));
   }
   c->state = 1;
+  c->qkey_valid = true;
   c->err.clear();
   return SIGMO_OK;
 }

@@ -106,6 +106,10 @@ class StreamRunner:
         self.pool = ThreadPoolExecutor(self.nbuf)
         import threading
         self.copy_lock = threading.Lock()
+        import contextlib
+        import os as _os
+        if _os.environ.get("SIGMO_STREAM_NOLOCK") == "1":  # experiment knob
+            self.copy_lock = contextlib.nullcontext()
         if induced:  # DESIGN.md R21 (set before the first load_batch)
             for row in self.ctx:
                 for c in row:

@@ -417,3 +417,23 @@ def test_lane_join_step_counting(ctx, sigmo):
     assert np.array_equal(ctx.dense_results(), ref)
     # every step pops one candidate: at least one step per surviving pair with a non-empty root window
     assert steps >= int((ref > 0).sum())
+
+
+def test_query_program_reuse_across_loads(ctx, sigmo):
+    """A load with the same query batch as the previous one reuses the query
+    programs and (when the matching order is unchanged) the join's plan
+    entries; data batches with other label frequencies (another order), another
+    query batch and the way back all match the oracle."""
+    Q1 = synth.config_queries(2)
+    Q2 = GraphBatch.from_graphs(synth.library(["benzene", "pyridine", "ester", "nitrile"]))
+    rng = np.random.default_rng(9)
+    D1 = synth.config_data(2, count=800)
+    D2 = synth.config_data(2, first=5000, count=800)
+    # label-skewed batch: many nitrogens (the planner's rarest-label root changes)
+    ds = [synth.random_labelled_graph(rng, int(rng.integers(3, 20)), 0.3, labels=(7, 7, 7, 6, 8)) for _ in range(300)]
+    D3 = GraphBatch.from_graphs(ds)
+    for Q, D in ((Q1, D1), (Q1, D2), (Q1, D3), (Q1, D1), (Q2, D1), (Q1, D2)):
+        for L in (2, 4):
+            for mode, om in ((sigmo.SIGMO_FIND_ALL, oracle.FIND_ALL), (sigmo.SIGMO_FIND_FIRST, oracle.FIND_FIRST)):
+                _, dense = run(ctx, Q, D, L, mode)
+                assert np.array_equal(dense, oracle.count_dense(Q, D, om)), (Q.num_graphs, L, mode)
