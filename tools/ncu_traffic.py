@@ -26,7 +26,8 @@ def val(r, k):
 res = {"source": rep.rsplit("/", 1)[-1], "levels": levels, "workload": "configs[2]", "kernels": {}}
 for r in rows[2:]:
     name = r[hdr.index("Kernel Name")]
-    m = re.search(r"k_join_lane<0, (\d)", name)  # <MODE, W64, PS>: Find All launches, narrow / wide masks
+    # <MODE, W64, PS>: Find All launches (MODE 0, or 8 = the lean instantiation), narrow / wide masks
+    m = re.search(r"k_join_lane<(?:0|8), (\d)", name)
     key = "sigmo_filter_lane_jit" if "filter_lane" in name else (
         ("k_join_lane_wide" if m.group(1) == "1" else "k_join_lane_narrow") if m else name)
     res["kernels"][key] = {
