@@ -2082,6 +2082,8 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
       jp.prec = (const int4 *)c->pair_rec.p;
       jp.adjw = (const uint32_t *)c->adjb.p;
       jp.adj_ones = c->adj_words;
+      jp.adj_limit = (unsigned long long)c->adj_words + 4;
+      jp.cmol_limit = c->bm_bytes / 4;
       jp.qp_ent = c->qp_ent;
       jp.qp_ent2 = (const uint2 *)(c->lane_ns ? c->ent_ns.p : c->ent2.p);
       jp.cmol = (const uint32_t *)c->bitmap.p;
@@ -2125,7 +2127,10 @@ sigmo_status join_impl(sigmo_ctx *c, sigmo_mode mode, uint64_t *total_matches_ou
         jp.smem_bytes = smem;
         jp.chunk_counter = (int *)((unsigned long long *)c->jcnt.p + (w64 ? 6 + (size_t)c->NQ : 0));
         // neighbour-support mode: the refined windows of each pair (plan-depth order)
-        if (c->lane_ns) jp.cmol = (const uint32_t *)(w64 ? c->ns_win64.p : c->ns_win32.p);
+        if (c->lane_ns) {
+          jp.cmol = (const uint32_t *)(w64 ? c->ns_win64.p : c->ns_win32.p);
+          jp.cmol_limit = (w64 ? c->ns_win64.cap : c->ns_win32.cap) / 4;
+        }
         int bps = join_lane_blocks_per_sm((int)mode, w64, jp, smem);
         if (const char *e = getenv("SIGMO_JOIN_BPS")) bps = std::max(1, std::min(bps, atoi(e)));
         if (const char *e = getenv(w64 ? "SIGMO_JOIN_BPS_FORCE_WIDE" : "SIGMO_JOIN_BPS_FORCE"))  // experiment knob

@@ -184,6 +184,8 @@ struct JoinParams {
   const uint32_t *adjw;        // bond-class adjacency masks (molecule-local bits), per molecule at word adj_off[g]:
                                // class-major [NB][n], u32 masks (n <= 32) or u64 (n > 32); all ones at word adj_ones
   unsigned adj_ones;
+  unsigned long long adj_limit;   // words of adjw / of the candidate-window array (SIGMO_BOUNDS_CHECK builds)
+  unsigned long long cmol_limit;
   const int4 *qp_ent;          // [VQ] per plan position {j0 | j1 << 4 (15 none) | #extra << 8 | node << 12, class0, class1, extra back-edge start}
   const uint2 *qp_ent2;        // [VQ] compact, k_join_lane: x = slot0 * 128 | leaf << 11 | #extra back-edges << 12 |
                                // slot1 * 128 << 16 (slot = back-edge depth, maxq - 1 = none: the map slot
@@ -346,6 +348,18 @@ constexpr int kJoinLanePlanSmemMax = 2048;  // k_join_lane: plan positions copie
 #define SIGMO_JL_THREADS_NARROW 192
 #endif
 __host__ __device__ constexpr int jl_threads(bool w64) { return w64 ? 128 : SIGMO_JL_THREADS_NARROW; }
+// SIGMO_BOUNDS_CHECK builds (tools/bounds_check.sh): index and address bounds of the lane join and the
+// totals reduction checked on the device (trap on violation); compiled out otherwise
+#ifdef SIGMO_BOUNDS_CHECK
+#define SIGMO_BOUND(cond) \
+  do {                    \
+    if (!(cond)) __trap(); \
+  } while (0)
+#else
+#define SIGMO_BOUND(cond) \
+  do {                    \
+  } while (0)
+#endif
 constexpr int kJoinLaneMaxQ = 11;  // k_join_lane handles queries <= 11 nodes in <= 64-node graphs (map: 6 bits x 10 depths)
 size_t join_smem_bytes(int NW, const JoinParams &p);
 size_t join_gstack_bytes(int NW, const JoinParams &p, int grid);

@@ -2143,6 +2143,7 @@ __global__ void __launch_bounds__(kTotThreads) k_lane_totals(int ND, int NQ, int
     long long o = o1.b > o0.b ? pn + o0.b : o0.a;  // the records' order (k_pairs)
     for (int qb = 0; qb < NQW; qb++) {
       const uint32_t bits = __ldg(&gm[(size_t)g * NQW + qb]);
+      SIGMO_BOUND(!((bits >> lane) & 1u) || o + __popc(bits & lt) < pn + off[ND].b);
       if ((bits >> lane) & 1u) acc[qb * 32 + lane] += __ldg(&presult[o + __popc(bits & lt)]);
       o += __popc(bits);
     }
@@ -2432,11 +2433,13 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   unsigned *const counter = (unsigned *)jp.chunk_counter;
   // mask of adjacency word index i (entries of 1 or 2 words)
   auto adj = [&](unsigned i) -> MT {
+    SIGMO_BOUND((unsigned long long)i + sw < jp.adj_limit);
     if (W64) return (MT)__ldg((const unsigned long long *)(adjw + i));
     return (MT)__ldg(adjw + i);
   };
   // candidate window at cmol word index i
   auto cand = [&](unsigned i) -> MT {
+    SIGMO_BOUND((unsigned long long)i + sw < jp.cmol_limit);
     if (W64) return (MT)__ldg((const unsigned long long *)(cmol + i));
     return (MT)__ldg(cmol + i);
   };
@@ -2517,6 +2520,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
         const unsigned d = bfind32(ne);  // deepest open depth
         const unsigned bd = 1u << d;
         const unsigned od = sRU + 32u * ES * d;
+        SIGMO_BOUND(d + 1u < (unsigned)MQ && od + ES <= sbase + (unsigned)jp.smem_bytes);
         // plan entry of depth e = d + 1 (x: back-edge map slots, leaf, #extra;
         // y: bond classes, distinct row)
         const uint2 en = JL_PLAN(pe + PSTEP * d);
@@ -2574,6 +2578,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
     // ---- finished pairs (parts): result (the per-query totals are reduced from the results by
     // k_lane_totals) ----
     if (pend && ne == 0u) {
+      SIGMO_BOUND(cp < P);
       if (MODE & 1) {
         if (!shared) presult[cp] = cnt ? 1ull : 0ull;
         else if (cnt) atomicOr(&presult[cp], 1ull);
@@ -2622,6 +2627,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
       }
       const unsigned idx = rank < left ? cursor + rank : bn + (rank - left);
       if (((f >> lane) & 1u) && idx < P) {
+        SIGMO_BOUND(idx < P);
         nrec = __ldg(recs + idx);
         nidx = idx;
         nv = true;
