@@ -2270,28 +2270,27 @@ cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const
 // per lane, for queries of <= kJoinLaneMaxQ nodes in <= 64-node data graphs.
 //   * Per lane, in shared memory: the DFS stack {R_d, U_d} (untried
 //     candidates of depth d, used set of f(pi_0..pi_{d-1})) and the map
-//     bytes f(pi_d); the candidate windows cm[u] are read from the filter's
-//     cmol[g][row] layout (a pair's rows are contiguous), the next pair's
-//     root window is loaded while the current pair runs.  A bitmask `ne`
-//     of open depths makes every step productive: a step pops the lowest
-//     candidate v of the deepest open depth d (backtracking is free) and
-//     builds the candidates of e = d + 1:
+//     words (adjacency index of f(pi_d)); the candidate windows cm[u] are
+//     read from the filter's cmol[g][row] layout.  A bitmask `ne` of open
+//     depths makes every step productive: a step pops the highest candidate
+//     v of the deepest open depth d (backtracking is free) and builds the
+//     candidates of e = d + 1:
 //        X = cm[pi_e] & ~(U_d | {v}) & AND_{(j,b) in back(e)} adjb[b][f(pi_j)]
-//     pushed as {X, U_d | {v}}; at the last depth they are counted with popc
-//     (Find All) or end the pair (Find First).  Absent back-edges read the
-//     all-ones adjacency class, so the step has no selects.
-//   * The warp claims the GMCR list in chunks of 32 pair records (one atomic
-//     per chunk, issued a chunk ahead; the records are held in registers,
-//     one per lane, and handed to lanes by shuffles).  Lanes whose pair
-//     finished refill together (>= batchK at a time): write the result,
-//     activate the prefetched next pair, take a new next pair and start its
-//     prefetch.  Lanes of a warp thus run pairs of very different sizes
-//     without waiting for each other (the paper runs one work-item per query
-//     of a data graph and sits at ~48% occupancy, divergence-bound,
-//     P:1854-1884); when the list is drained, idle lanes take the shallowest
-//     open depth of a busy lane (heavy pairs).
-//   * Per-query totals are reduced in shared memory (one global atomic per
-//     query per CTA).
+//     pushed as {X, U_d | {v}} (a predicated store); at the last depth they
+//     are counted with popc (Find All) or end the pair (Find First).  Absent
+//     back-edges read the all-ones adjacency entry, so the step has no
+//     selects; SIGMO_JL_UNROLL steps run between two checks of the free lanes.
+//   * The warp claims blocks of kJoinClaim consecutive GMCR pairs (one atomic
+//     per block, a block ahead).  Lanes whose pair finished refill together
+//     (>= batchK at a time): write the result, activate the next pair they
+//     hold (its record in registers, its root window loaded a pass earlier),
+//     and the lanes left without one take the next records of the warp's
+//     blocks.  Lanes of a warp thus run pairs of very different sizes without
+//     waiting for each other (the paper runs one work-item per query of a
+//     data graph and sits at ~48% occupancy, divergence-bound);
+//     when the list is drained, idle lanes take the shallowest open depth of
+//     a busy lane (heavy pairs).
+//   * Per-query totals: k_lane_totals, from the pair results.
 // ===========================================================================
 constexpr int kJoinClaim = 128;   // GMCR pairs per warp claim (atomic on the launch's pair counter)
 
