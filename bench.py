@@ -476,6 +476,11 @@ def main():
                  "peak_source": f"measured: 148 SM x {lanes:.1f} int lanes/clk (mixed LOP3+IMAD, profiles/r2/"
                                 f"int_peak.json) x {sm_mhz:.0f} MHz (this run's clock)",
                  "thread_instructions_per_step": (thr_instr / steps) if (steps and thr_instr) else None,
+                 "l1_global_sectors_per_step": (sum(k.get("l1_global_ld_sectors", 0) for k in (jn, jw)) / steps)
+                 if (steps and jn) else None,
+                 "l1_shared_wavefronts_per_step": (sum(k.get("l1_shared_wavefronts", 0) for k in (jn, jw)) / steps)
+                 if (steps and jn) else None,
+                 "l1_data_pipe_pct_narrow": jn.get("l1_data_pipe_pct"),
                  "issue_utilization": (jn.get("ipc", 0) / 4.0) if jn else None,
                  "pairs_per_launch": pairs_local, "matches_per_launch": matches_local}
     dominant = "join" if j_ms >= f_ms else "filter"

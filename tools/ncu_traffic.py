@@ -39,5 +39,9 @@ for r in rows[2:]:
         "ipc": val(r, "sm__inst_executed.avg.per_cycle_active"),
         "occupancy_pct": val(r, "sm__warps_active.avg.pct_of_peak_sustained_active"),
         "l2_hit_pct": val(r, "lts__t_sector_hit_rate.pct"),
+        "l1_global_ld_sectors": val(r, "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum"),
+        "l1_global_ld_hit_pct": val(r, "l1tex__t_sector_pipe_lsu_mem_global_op_ld_hit_rate.pct"),
+        "l1_shared_wavefronts": val(r, "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"),
+        "l1_data_pipe_pct": val(r, "l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed"),
     }
 print(json.dumps(res, indent=1))
