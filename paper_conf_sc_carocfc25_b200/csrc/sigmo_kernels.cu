@@ -2303,14 +2303,11 @@ __host__ __device__ inline size_t join_lane_warp_bytes(int MQ, bool w64) {
 // CTA: the window and adjacency base pointers (16 B), (optionally) the plan entries [VQ] uint2, then one
 // region per warp
 __host__ __device__ inline size_t join_lane_plan_bytes(int VQ, int pmax) { return VQ <= pmax ? align16(8 * (size_t)VQ) : 0; }
-__host__ __device__ inline size_t join_lane_cta_bytes(int NQ, int VQ, int pmax) {
-  (void)NQ;
-  return 16 + join_lane_plan_bytes(VQ, pmax);
+__host__ __device__ inline size_t join_lane_cta_bytes(int VQ, int pmax) { return 16 + join_lane_plan_bytes(VQ, pmax); }
+__host__ __device__ inline size_t join_lane_smem(int VQ, int MQ, bool w64, int pmax, int threads) {
+  return join_lane_cta_bytes(VQ, pmax) + join_lane_warp_bytes(MQ, w64) * (size_t)(threads / 32);
 }
-__host__ __device__ inline size_t join_lane_smem(int NQ, int VQ, int MQ, bool w64, int pmax, int threads) {
-  return join_lane_cta_bytes(NQ, VQ, pmax) + join_lane_warp_bytes(MQ, w64) * (size_t)(threads / 32);
-}
-size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_smem(p.NQ, p.VQ, p.maxq, w64, p.plan_smem_max, p.lane_threads); }
+size_t join_lane_smem_bytes(const JoinParams &p, bool w64) { return join_lane_smem(p.VQ, p.maxq, w64, p.plan_smem_max, p.lane_threads); }
 
 // n-th (0-based) set bit of m (m has > n set bits)
 __device__ __forceinline__ int nth_set_bit(unsigned m, int n) {
@@ -2375,7 +2372,7 @@ __global__ void __launch_bounds__(jl_threads(W64)) __maxnreg__(W64 ? 64 : SIGMO_
   // a generic smem + offset re-derives the shared window every step)
   const unsigned sbase = (unsigned)__cvta_generic_to_shared(smem);
 #define JL_PLAN(p) (PS ? lds_u2(p) : __ldg(&jp.qp_ent2[(p)]))
-  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.NQ, jp.VQ, jp.plan_smem_max) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
+  const unsigned wbase = (unsigned)(join_lane_cta_bytes(jp.VQ, jp.plan_smem_max) + (size_t)wid * join_lane_warp_bytes(MQ, W64));
   constexpr unsigned LS = ES;  // stack entries {R, U} interleaved per lane
   const unsigned oRU = wbase + LS * lane;  // stack entry of depth d: oRU + 32 ES d
   const unsigned mA = oRU - LS * lane + 32u * ES * SD + 4u * lane;  // map word of depth d: mA + 128 d (slot SD: absent)
