@@ -2292,7 +2292,10 @@ cudaError_t launch_adjb(const DevGraphs &d, const uint8_t *bclass, int NB, const
 //     a busy lane (heavy pairs).
 //   * Per-query totals: k_lane_totals, from the pair results.
 // ===========================================================================
-constexpr int kJoinClaim = 128;   // GMCR pairs per warp claim (atomic on the launch's pair counter)
+#ifndef SIGMO_JL_CLAIM
+#define SIGMO_JL_CLAIM 128  // configs[2] join: claims of 64/128/512 pairs -> 4.87/4.60/4.60 ms
+#endif
+constexpr int kJoinClaim = SIGMO_JL_CLAIM;  // GMCR pairs per warp claim (atomic on the launch's pair counter)
 
 // stack entry {R, U}: 2 x 32-bit masks (<= 32-node molecules) or 2 x 64-bit
 __host__ __device__ inline size_t join_lane_warp_bytes(int MQ, bool w64) {
